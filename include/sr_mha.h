@@ -1,0 +1,171 @@
+/*
+ * sr_mha.h -- C ABI of the B200-native softmax-recomposed multi-head attention hot path.
+ *
+ * Method: Choi, Li, Kim, Hwang, Ahn, "Accelerating Transformer Networks through Recomposing
+ * Softmax Layers", IISWC 2022.  The attention layer computes, per
+ * head, O = softmax(mask(Q K^T * scale)) V with the safe softmax of Eq. (1) (L55-L58).  This
+ * library computes it through the paper's softmax recomposition (Sec. 3.2-3.4):
+ *
+ *   kernel 1  GEMM1 + LS   x = Q K^T * scale, mask; per 128-row x T-column output tile the
+ *                          epilogue computes the Local Softmax (Eq. 2): m' = row max of the tile,
+ *                          X' = e^{x - m'} (written once), d' = row sum of X'     (L131-L145, L165)
+ *   kernel 2  IR           per row: m = max_k m'_k, d = sum_k e^{m'_k - m} d'_k,
+ *                          r'_k = e^{m'_k - m} / d                                 (L147-L149, L173)
+ *   kernel 3  GS + GEMM2   the prologue scales each X' tile row by its r' (Global Scaling, L151)
+ *                          as the tile is loaded, then O += Y V on the tensor cores (L165)
+ *
+ * The attention matrix therefore crosses HBM twice instead of four times (L171-L173).  The
+ * *_unfused entry points run the deliberately unfused baseline GEMM1 -> row softmax -> GEMM2
+ * (L102, L171) with the same tiles, skipping and layouts, as the in-repo traffic baseline.
+ *
+ * Conventions common to every entry point
+ * ---------------------------------------
+ *  - q, k, v, out: DEVICE pointers, [B][H][S][D] contiguous (the caller does the Split/Concat of
+ *    PAPER.md L49-L51), 16-byte aligned.  in_dtype for q/k/v; out_dtype for out.  out is fully
+ *    overwritten and must not overlap q, k or v.
+ *  - scale: multiplies Q K^T (PAPER.md L53 uses 1/sqrt(D_head)); finite and > 0.
+ *  - causal: key j is masked for query i when j > i (combines with every mask kind).
+ *  - Mask / layout descriptors and the arrays they point to are HOST memory, read during the
+ *    call.  The library derives a tile schedule from them and caches it on the device (small,
+ *    library-owned allocations made on the first call with a new mask; later calls with the same
+ *    mask content allocate nothing and are CUDA-graph capturable).
+ *  - All launches go to ex->stream; nothing synchronises it.  Calls are asynchronous: device-side
+ *    faults surface at the caller's next synchronisation (as with cuBLAS).
+ *  - A row whose every key is masked outputs 0 (reading R9).
+ *  - Supported: S % 128 == 0, S >= 128; D in {64, 128}; in_dtype F16 or BF16 (tensor-core path) or
+ *    F32 (SIMT fp32 path, every mask kind); out_dtype == in_dtype or F32; block == 64.
+ *    Anything else returns SR_ERR_UNSUPPORTED before touching the device.
+ *
+ * Errors: argument checks run before any CUDA call and return SR_ERR_INVALID /
+ * SR_ERR_UNSUPPORTED / SR_ERR_WORKSPACE; a failed CUDA call returns SR_ERR_CUDA.  Details of the
+ * last non-OK return on the calling thread: sr_last_error().
+ */
+#ifndef SR_MHA_H
+#define SR_MHA_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    SR_OK = 0,
+    SR_ERR_INVALID = 1,     /* bad pointer, shape, scale, overlapping out, malformed layout */
+    SR_ERR_UNSUPPORTED = 2, /* valid request outside the supported envelope (see above) */
+    SR_ERR_WORKSPACE = 3,   /* workspace NULL or smaller than sr_workspace_bytes() */
+    SR_ERR_CUDA = 4         /* a CUDA runtime/driver call failed; see sr_last_error() */
+} sr_status;
+
+typedef enum { SR_F32 = 0, SR_F16 = 1, SR_BF16 = 2 } sr_dtype;
+
+/* Dense mask: optional key-side padding.  kv_len: HOST array [B] or NULL;
+ * key j of batch b is masked iff j >= kv_len[b]  (0 <= kv_len[b] <= S). */
+typedef struct {
+    const int32_t* kv_len;
+} sr_dense_mask;
+
+/* Block-sparse layout (square blocks).  HOST arrays.
+ *   block         block edge, must be 64
+ *   layout_heads  1 (shared by all heads) or H (head h uses layout h, for every batch b)
+ *   row_ptr       [layout_heads][S/block + 1]: ABSOLUTE offsets into col_idx; row_ptr[h][0] is the
+ *                 start of head h, non-decreasing
+ *   col_idx       column-block ids, strictly ascending within a block-row, in [0, S/block)
+ * Element (i, j) is kept iff block (i/64, j/64) is listed (and causal allows it). */
+typedef struct {
+    int32_t block;
+    int32_t layout_heads;
+    const int32_t* row_ptr;
+    const int32_t* col_idx;
+} sr_block_layout;
+
+/* Longformer sliding window + symmetric global tokens:
+ * (i, j) kept iff |i - j| <= window/2  or  i < n_global  or  j < n_global. */
+typedef struct {
+    int32_t window;
+    int32_t n_global;
+} sr_window;
+
+/* Execution parameters. */
+typedef struct {
+    sr_dtype in_dtype;       /* dtype of q, k, v */
+    sr_dtype out_dtype;      /* in_dtype, or SR_F32 (fp32-accumulated context, validation mode) */
+    void* workspace;         /* DEVICE, caller-owned, >= sr_workspace_bytes(), 256-byte aligned */
+    size_t workspace_bytes;
+    void* stream;            /* cudaStream_t; NULL = legacy default stream */
+    int32_t tile_n;          /* T = LS sub-vector width = GEMM1 output-tile width:
+                                0 = default (128 dense 16-bit, 64 fp32 and sparse), or 64 / 128 */
+    int32_t flags;           /* reserved, must be 0 */
+} sr_exec;
+
+/* Entry points (north star).  Returns SR_OK after enqueueing the kernels on ex->stream. */
+sr_status sr_mha_dense(const void* q, const void* k, const void* v, void* out, int B, int H, int S,
+                       int D, float scale, const sr_dense_mask* mask_or_null, int causal,
+                       const sr_exec* ex);
+sr_status sr_mha_blocksparse(const void* q, const void* k, const void* v, void* out, int B, int H,
+                             int S, int D, float scale, const sr_block_layout* layout, int causal,
+                             const sr_exec* ex);
+sr_status sr_mha_sliding_window(const void* q, const void* k, const void* v, void* out, int B,
+                                int H, int S, int D, float scale, const sr_window* win, int causal,
+                                const sr_exec* ex);
+
+/* In-repo traffic baseline: GEMM1 (scale+mask, writes scores) -> row softmax (reads scores,
+ * writes P) -> GEMM2 (reads P).  Identical signatures and semantics; 16-bit dtypes only. */
+sr_status sr_mha_dense_unfused(const void* q, const void* k, const void* v, void* out, int B,
+                               int H, int S, int D, float scale, const sr_dense_mask* mask_or_null,
+                               int causal, const sr_exec* ex);
+sr_status sr_mha_blocksparse_unfused(const void* q, const void* k, const void* v, void* out, int B,
+                                     int H, int S, int D, float scale,
+                                     const sr_block_layout* layout, int causal, const sr_exec* ex);
+sr_status sr_mha_sliding_window_unfused(const void* q, const void* k, const void* v, void* out,
+                                        int B, int H, int S, int D, float scale,
+                                        const sr_window* win, int causal, const sr_exec* ex);
+
+/* Which entry point a workspace query is for. */
+typedef enum { SR_E_DENSE = 0, SR_E_BLOCKSPARSE = 1, SR_E_WINDOW = 2 } sr_entry;
+
+/* Workspace layout (all offsets in bytes from ex->workspace; 256-byte aligned):
+ *   A tile is 128 query rows x T keys.  Every (head, row-block, listed key tile) owns a "slot";
+ *   slot s of head g has global id  g * slots_per_head + s.
+ *   xprime   recomposed: X' tiles, unfused: the score tiles S and then P (2 regions), each tile
+ *            128*T elements of xprime_elt_bytes; 16-bit tiles are stored in the canonical
+ *            SWIZZLE_128B K-major layout [T/64][128 rows][64 cols] with the 16-byte chunk index
+ *            XOR (row & 7); fp32 tiles are plain row-major [128][T].
+ *   mprime, dprime, rprime   fp32 [slot id][128 rows]  (m' in natural-log units)
+ */
+typedef struct {
+    int32_t tile_n;           /* T actually used */
+    int32_t slots_per_head;
+    int64_t n_slots;          /* B*H*slots_per_head */
+    int32_t xprime_elt_bytes; /* 2 (16-bit paths) or 4 (fp32 path) */
+    size_t off_xprime, off_mprime, off_dprime, off_rprime, off_p;  /* off_p: unfused P region */
+    size_t total_bytes;
+} sr_ws_info;
+
+/* Workspace bytes needed by an entry point; `mask_or_layout` is the same pointer passed to it
+ * (sr_dense_mask*, sr_block_layout* or sr_window*; may be NULL for dense).  fused: 1 recomposed,
+ * 0 unfused.  Returns 0 on invalid/unsupported arguments (see sr_last_error()). */
+size_t sr_workspace_bytes(sr_entry entry, int fused, int B, int H, int S, int D, sr_dtype in_dtype,
+                          const void* mask_or_layout, int causal, int tile_n);
+/* Same, with the full layout of the workspace (for tests that read X', m', d', r' back). */
+sr_status sr_workspace_query(sr_entry entry, int fused, int B, int H, int S, int D,
+                             sr_dtype in_dtype, const void* mask_or_layout, int causal, int tile_n,
+                             sr_ws_info* info);
+
+/* Host-side tile schedule of a call, for tests and the byte model: number of stored score
+ * elements (tiles x 128 x T, counting only valid 64-row halves) and tile count. */
+sr_status sr_schedule_stats(sr_entry entry, int B, int H, int S, const void* mask_or_layout,
+                            int causal, int tile_n, int64_t* n_tiles, int64_t* stored_elems);
+
+const char* sr_status_string(sr_status s);
+const char* sr_last_error(void);
+/* Kernel launches issued by the calling thread since the library was loaded (for bench.py's
+ * gpu_launches count). */
+int64_t sr_launch_count(void);
+const char* sr_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SR_MHA_H */

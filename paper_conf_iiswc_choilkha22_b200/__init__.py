@@ -1,0 +1,240 @@
+"""Python binding of the B200-native softmax-recomposed attention library (libsr_mha.so).
+
+Argument marshalling only: every step of the hot path (GEMM1 + Local Softmax, IR, Global
+Scaling + GEMM2, and the unfused baseline) runs in the CUDA kernels behind the C ABI declared in
+``include/sr_mha.h``.  PyTorch supplies device memory and the current CUDA stream.  There is no
+CPU fallback: if the shared library is missing or a call fails, this module raises.
+
+Entry points (same names as the C ABI, PAPER.md L51-L53 semantics):
+    mha_dense(q, k, v, scale=None, kv_len=None, causal=False, ...)
+    mha_blocksparse(q, k, v, layout, scale=None, causal=False, ...)
+    mha_sliding_window(q, k, v, window, n_global, scale=None, causal=False, ...)
+with ``fused=False`` selecting the unfused GEMM -> softmax -> GEMM baseline.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import math
+import os
+import threading
+from typing import Optional
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libsr_mha.so")
+
+SR_OK, SR_ERR_INVALID, SR_ERR_UNSUPPORTED, SR_ERR_WORKSPACE, SR_ERR_CUDA = range(5)
+SR_F32, SR_F16, SR_BF16 = 0, 1, 2
+SR_E_DENSE, SR_E_BLOCKSPARSE, SR_E_WINDOW = 0, 1, 2
+
+# every symbol include/sr_mha.h declares
+EXPORTS = ["sr_mha_dense", "sr_mha_blocksparse", "sr_mha_sliding_window", "sr_mha_dense_unfused",
+           "sr_mha_blocksparse_unfused", "sr_mha_sliding_window_unfused", "sr_workspace_bytes",
+           "sr_workspace_query", "sr_schedule_stats", "sr_status_string", "sr_last_error",
+           "sr_launch_count", "sr_version"]
+
+
+class SrError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"{_STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+_STATUS = {0: "SR_OK", 1: "SR_ERR_INVALID", 2: "SR_ERR_UNSUPPORTED", 3: "SR_ERR_WORKSPACE", 4: "SR_ERR_CUDA"}
+
+
+class DenseMask(C.Structure):
+    _fields_ = [("kv_len", C.c_void_p)]
+
+
+class BlockLayoutC(C.Structure):
+    _fields_ = [("block", C.c_int32), ("layout_heads", C.c_int32), ("row_ptr", C.c_void_p),
+                ("col_idx", C.c_void_p)]
+
+
+class WindowC(C.Structure):
+    _fields_ = [("window", C.c_int32), ("n_global", C.c_int32)]
+
+
+class Exec(C.Structure):
+    _fields_ = [("in_dtype", C.c_int), ("out_dtype", C.c_int), ("workspace", C.c_void_p),
+                ("workspace_bytes", C.c_size_t), ("stream", C.c_void_p), ("tile_n", C.c_int32),
+                ("flags", C.c_int32)]
+
+
+class WsInfo(C.Structure):
+    _fields_ = [("tile_n", C.c_int32), ("slots_per_head", C.c_int32), ("n_slots", C.c_int64),
+                ("xprime_elt_bytes", C.c_int32), ("off_xprime", C.c_size_t), ("off_mprime", C.c_size_t),
+                ("off_dprime", C.c_size_t), ("off_rprime", C.c_size_t), ("off_p", C.c_size_t),
+                ("total_bytes", C.c_size_t)]
+
+
+_lib = None
+_lock = threading.Lock()
+
+
+def lib():
+    """Load libsr_mha.so (raises if it has not been built -- there is no fallback)."""
+    global _lib
+    with _lock:
+        if _lib is None:
+            if not os.path.exists(LIB_PATH):
+                raise RuntimeError(f"{LIB_PATH} is missing: build it with "
+                                   "`python -m paper_conf_iiswc_choilkha22_b200.build`")
+            L = C.CDLL(LIB_PATH)
+            vp, i, f = C.c_void_p, C.c_int, C.c_float
+            sig = [vp, vp, vp, vp, i, i, i, i, f, vp, i, C.POINTER(Exec)]
+            for n in EXPORTS[:6]:
+                getattr(L, n).argtypes = sig
+                getattr(L, n).restype = i
+            L.sr_workspace_bytes.argtypes = [i, i, i, i, i, i, i, vp, i, i]
+            L.sr_workspace_bytes.restype = C.c_size_t
+            L.sr_workspace_query.argtypes = [i, i, i, i, i, i, i, vp, i, i, C.POINTER(WsInfo)]
+            L.sr_workspace_query.restype = i
+            L.sr_schedule_stats.argtypes = [i, i, i, i, vp, i, i, C.POINTER(C.c_int64), C.POINTER(C.c_int64)]
+            L.sr_schedule_stats.restype = i
+            L.sr_status_string.argtypes = [i]
+            L.sr_status_string.restype = C.c_char_p
+            L.sr_last_error.restype = C.c_char_p
+            L.sr_launch_count.restype = C.c_int64
+            L.sr_version.restype = C.c_char_p
+            _lib = L
+    return _lib
+
+
+def last_error() -> str:
+    return lib().sr_last_error().decode()
+
+
+def launch_count() -> int:
+    return int(lib().sr_launch_count())
+
+
+def _check(st: int):
+    if st != SR_OK:
+        raise SrError(st, last_error())
+
+
+# ----------------------------------------------------------------------------- mask descriptors
+
+class _Mask:
+    """Holds a C mask descriptor and the host arrays it points to."""
+
+    def __init__(self, entry: int, obj, keep):
+        self.entry, self.obj, self.keep = entry, obj, keep
+
+    @property
+    def ptr(self):
+        return None if self.obj is None else C.cast(C.byref(self.obj), C.c_void_p)
+
+
+def dense_mask(kv_len=None) -> _Mask:
+    if kv_len is None:
+        return _Mask(SR_E_DENSE, None, None)
+    a = np.ascontiguousarray(np.asarray(kv_len), dtype=np.int32)
+    return _Mask(SR_E_DENSE, DenseMask(a.ctypes.data), a)
+
+
+def block_mask(layout) -> _Mask:
+    """layout: object with .block, .row_ptr [layout_heads, nb+1] (absolute offsets), .col_idx."""
+    rp = np.ascontiguousarray(layout.row_ptr, dtype=np.int32)
+    ci = np.ascontiguousarray(layout.col_idx, dtype=np.int32)
+    if ci.size == 0:
+        ci = np.zeros(1, dtype=np.int32)
+    return _Mask(SR_E_BLOCKSPARSE, BlockLayoutC(int(layout.block), int(rp.shape[0]), rp.ctypes.data,
+                                                ci.ctypes.data), (rp, ci))
+
+
+def window_mask(window: int, n_global: int) -> _Mask:
+    return _Mask(SR_E_WINDOW, WindowC(int(window), int(n_global)), None)
+
+
+# ----------------------------------------------------------------------------- queries
+
+def workspace_info(mask: _Mask, B, H, S, D, in_dtype: int, causal=False, tile_n=0, fused=True) -> dict:
+    info = WsInfo()
+    _check(lib().sr_workspace_query(mask.entry, int(fused), B, H, S, D, in_dtype, mask.ptr, int(causal),
+                                    int(tile_n), C.byref(info)))
+    return {k: getattr(info, k) for k, _ in WsInfo._fields_}
+
+
+def schedule_stats(mask: _Mask, B, H, S, causal=False, tile_n=0):
+    nt, ne = C.c_int64(), C.c_int64()
+    _check(lib().sr_schedule_stats(mask.entry, B, H, S, mask.ptr, int(causal), int(tile_n), C.byref(nt),
+                                   C.byref(ne)))
+    return int(nt.value), int(ne.value)
+
+
+# ----------------------------------------------------------------------------- torch entry points
+
+def _torch():
+    import torch
+    return torch
+
+
+def dtype_code(dt) -> int:
+    torch = _torch()
+    return {torch.float32: SR_F32, torch.float16: SR_F16, torch.bfloat16: SR_BF16}[dt]
+
+
+_ws_cache = {}
+
+
+def _workspace(device, nbytes):
+    torch = _torch()
+    key = (device.index if device.index is not None else torch.cuda.current_device())
+    buf = _ws_cache.get(key)
+    if buf is None or buf.numel() < nbytes:
+        buf = torch.empty(max(nbytes, 1 << 20), dtype=torch.uint8, device=device)
+        _ws_cache[key] = buf
+    return buf
+
+
+_FN = {(SR_E_DENSE, True): "sr_mha_dense", (SR_E_BLOCKSPARSE, True): "sr_mha_blocksparse",
+       (SR_E_WINDOW, True): "sr_mha_sliding_window", (SR_E_DENSE, False): "sr_mha_dense_unfused",
+       (SR_E_BLOCKSPARSE, False): "sr_mha_blocksparse_unfused",
+       (SR_E_WINDOW, False): "sr_mha_sliding_window_unfused"}
+
+
+def call(mask: _Mask, q, k, v, *, scale=None, causal=False, out_dtype=None, tile_n=0, fused=True,
+         out=None, workspace=None, stream=None):
+    """Run one attention layer through the C ABI.  q, k, v: CUDA tensors [B, H, S, D]."""
+    torch = _torch()
+    if not (q.is_cuda and k.is_cuda and v.is_cuda):
+        raise ValueError("q, k, v must be CUDA tensors")
+    if q.shape != k.shape or q.shape != v.shape or q.dim() != 4:
+        raise ValueError("q, k, v must share the shape [B, H, S, D]")
+    if not (q.is_contiguous() and k.is_contiguous() and v.is_contiguous()):
+        raise ValueError("q, k, v must be contiguous")
+    if q.dtype != k.dtype or q.dtype != v.dtype:
+        raise ValueError("q, k, v must share a dtype")
+    B, H, S, D = q.shape
+    scale = 1.0 / math.sqrt(D) if scale is None else float(scale)
+    in_dt = dtype_code(q.dtype)
+    out_dtype = q.dtype if out_dtype is None else out_dtype
+    if out is None:
+        out = torch.empty((B, H, S, D), dtype=out_dtype, device=q.device)
+    need = lib().sr_workspace_bytes(mask.entry, int(fused), B, H, S, D, in_dt, mask.ptr, int(causal), int(tile_n))
+    if need == 0:
+        raise SrError(lib().sr_workspace_query(mask.entry, int(fused), B, H, S, D, in_dt, mask.ptr, int(causal),
+                                               int(tile_n), C.byref(WsInfo())), last_error())
+    ws = workspace if workspace is not None else _workspace(q.device, need)
+    st = torch.cuda.current_stream(q.device).cuda_stream if stream is None else stream
+    ex = Exec(in_dt, dtype_code(out_dtype), ws.data_ptr(), ws.numel() * ws.element_size(), st, int(tile_n), 0)
+    fn = getattr(lib(), _FN[(mask.entry, bool(fused))])
+    _check(fn(q.data_ptr(), k.data_ptr(), v.data_ptr(), out.data_ptr(), B, H, S, D, C.c_float(scale), mask.ptr,
+              int(causal), C.byref(ex)))
+    return out
+
+
+def mha_dense(q, k, v, *, scale=None, kv_len=None, causal=False, **kw):
+    return call(dense_mask(kv_len), q, k, v, scale=scale, causal=causal, **kw)
+
+
+def mha_blocksparse(q, k, v, layout, *, scale=None, causal=False, **kw):
+    return call(block_mask(layout), q, k, v, scale=scale, causal=causal, **kw)
+
+
+def mha_sliding_window(q, k, v, window, n_global, *, scale=None, causal=False, **kw):
+    return call(window_mask(window, n_global), q, k, v, scale=scale, causal=causal, **kw)

@@ -1,0 +1,506 @@
+// abi.cu -- the C ABI of include/sr_mha.h: argument validation, tile schedules, workspace
+// layout, schedule cache, dispatch to the kernels.  Host code only.
+//
+// The tile schedule is the B200 form of the paper's TB work distribution (PAPER.md L112, L135,
+// Fig. 3-4): GEMM1 and GEMM2 iterate "items" (head, 128-row block) and, per item, the list of key
+// tiles that hold at least one kept element.  Fully masked tiles (causal upper triangle, padded
+// keys, absent sparse blocks, far-off band) are never computed, stored or read (reading R18).
+#include <algorithm>
+#include <atomic>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "../../include/sr_mha.h"
+#include "sr_internal.h"
+
+using namespace sr;
+
+namespace {
+
+thread_local char g_err[512] = "";
+std::atomic<int64_t> g_launches{0};
+
+sr_status fail(sr_status s, const char* fmt, ...)
+{
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(g_err, sizeof(g_err), fmt, ap);
+    va_end(ap);
+    return s;
+}
+
+int dtype_bytes(int dt) { return dt == SR_F32 ? 4 : 2; }
+
+// ------------------------------------------------------------------------------ schedules
+
+struct HostSched {
+    int T = 0, n_rb = 0, n_lh = 1, lh_mode = LH_ONE;
+    std::vector<int32_t> tp, tinfo, items, kv_len;
+    int slots_per_head = 0;
+    int64_t n_tiles = 0;       // over all B*H heads
+    int64_t stored_elems = 0;  // valid 64-row halves x 64 x T, over all heads
+};
+
+struct Request {
+    sr_entry entry;
+    int B, H, S, causal, T;
+    const int32_t* kv_len = nullptr;
+    const sr_block_layout* lay = nullptr;
+    int window = 0, n_global = 0;
+};
+
+// Does the half-tile rows [r0, r1] x keys [c0, c1] hold a kept element of the window mask?
+// (i, j) kept iff (|i-j| <= w2 or i < g or j < g) and (!causal or j <= i).
+bool window_half_valid(int r0, int r1, int c0, int c1, int w2, int g, bool causal)
+{
+    // band: j - i in [-w2, causal ? 0 : w2]  intersect  [c0 - r1, c1 - r0]
+    int hi = causal ? 0 : w2;
+    if (c0 - r1 <= hi && c1 - r0 >= -w2) return true;
+    // global rows i < g (with causal, needs some j <= i, best i = min(r1, g-1))
+    if (r0 < g) {
+        int imax = std::min(r1, g - 1);
+        if (!causal || c0 <= imax) return true;
+    }
+    // global columns j < g (with causal, needs some i >= j, best j = c0)
+    if (c0 < g) {
+        if (!causal || r1 >= c0) return true;
+    }
+    return false;
+}
+
+sr_status build_sched(const Request& r, HostSched& hs)
+{
+    const int S = r.S, T = r.T;
+    hs.T = T;
+    hs.n_rb = S / kRowBlock;
+    const int nkt = S / T;
+    std::vector<std::vector<std::pair<int, int>>> lists;  // per (lh, rb): (kt, half bits)
+    if (r.entry == SR_E_DENSE || r.entry == SR_E_WINDOW) {
+        hs.lh_mode = (r.entry == SR_E_DENSE && r.kv_len) ? LH_BATCH : LH_ONE;
+        hs.n_lh = hs.lh_mode == LH_BATCH ? r.B : 1;
+        for (int lh = 0; lh < hs.n_lh; ++lh) {
+            int kvl = (hs.lh_mode == LH_BATCH) ? r.kv_len[lh] : S;
+            for (int rb = 0; rb < hs.n_rb; ++rb) {
+                std::vector<std::pair<int, int>> L;
+                for (int kt = 0; kt < nkt; ++kt) {
+                    int c0 = kt * T, c1 = c0 + T - 1, bits = 0;
+                    for (int h = 0; h < 2; ++h) {
+                        int r0 = rb * kRowBlock + h * kHalf, r1 = r0 + kHalf - 1;
+                        bool ok;
+                        if (r.entry == SR_E_DENSE)
+                            ok = c0 < kvl && (!r.causal || c0 <= r1);
+                        else
+                            ok = window_half_valid(r0, r1, c0, c1, r.window / 2, r.n_global, r.causal);
+                        if (ok) bits |= 1 << h;
+                    }
+                    if (bits) L.push_back({kt, bits});
+                }
+                lists.push_back(std::move(L));
+            }
+        }
+    } else {  // block-sparse: pair the 64-row block-rows 2rb, 2rb+1 and take the union of columns
+        const sr_block_layout* lay = r.lay;
+        hs.lh_mode = lay->layout_heads == 1 ? LH_ONE : LH_HEAD;
+        hs.n_lh = lay->layout_heads;
+        const int nb = S / lay->block;
+        for (int lh = 0; lh < hs.n_lh; ++lh) {
+            const int32_t* rp = lay->row_ptr + (size_t)lh * (nb + 1);
+            for (int rb = 0; rb < hs.n_rb; ++rb) {
+                std::map<int, int> cols;
+                for (int h = 0; h < 2; ++h) {
+                    int br = 2 * rb + h;
+                    for (int32_t t = rp[br]; t < rp[br + 1]; ++t) {
+                        int c = lay->col_idx[t];
+                        if (r.causal && c > br) continue;  // block entirely above the diagonal
+                        cols[c] |= 1 << h;
+                    }
+                }
+                std::vector<std::pair<int, int>> L(cols.begin(), cols.end());
+                lists.push_back(std::move(L));
+            }
+        }
+    }
+    // flatten
+    hs.tp.assign((size_t)hs.n_lh * (hs.n_rb + 1), 0);
+    int32_t off = 0;
+    std::vector<int64_t> lh_elems(hs.n_lh, 0), lh_tiles(hs.n_lh, 0);
+    for (int lh = 0; lh < hs.n_lh; ++lh) {
+        hs.tp[(size_t)lh * (hs.n_rb + 1)] = off;
+        for (int rb = 0; rb < hs.n_rb; ++rb) {
+            for (auto& kb : lists[(size_t)lh * hs.n_rb + rb]) {
+                hs.tinfo.push_back(kb.first | (kb.second << 16));
+                lh_elems[lh] += (int64_t)__builtin_popcount(kb.second) * kHalf * T;
+                lh_tiles[lh] += 1;
+            }
+            off = (int32_t)hs.tinfo.size();
+            hs.tp[(size_t)lh * (hs.n_rb + 1) + rb + 1] = off;
+        }
+        hs.slots_per_head = std::max<int>(hs.slots_per_head, (int)lh_tiles[lh]);
+    }
+    // items, longest first (static LPT order; ties keep head-major order)
+    const int BH = r.B * r.H;
+    std::vector<std::pair<int, int32_t>> it;
+    it.reserve((size_t)BH * hs.n_rb);
+    for (int g = 0; g < BH; ++g) {
+        int lh = hs.lh_mode == LH_ONE ? 0 : (hs.lh_mode == LH_BATCH ? g / r.H : g % r.H);
+        hs.n_tiles += lh_tiles[lh];
+        hs.stored_elems += lh_elems[lh];
+        for (int rb = 0; rb < hs.n_rb; ++rb) {
+            const int32_t* tp = &hs.tp[(size_t)lh * (hs.n_rb + 1)];
+            it.push_back({tp[rb + 1] - tp[rb], g * hs.n_rb + rb});
+        }
+    }
+    std::stable_sort(it.begin(), it.end(), [](auto& a, auto& b) { return a.first > b.first; });
+    hs.items.resize(it.size());
+    for (size_t i = 0; i < it.size(); ++i) hs.items[i] = it[i].second;
+    if (r.kv_len) hs.kv_len.assign(r.kv_len, r.kv_len + r.B);
+    return SR_OK;
+}
+
+// ------------------------------------------------------------------------------ validation
+
+int default_T(sr_entry e, int in_dtype)
+{
+    if (in_dtype == SR_F32) return 64;
+    return e == SR_E_DENSE ? 128 : 64;
+}
+
+sr_status check_request(sr_entry e, int B, int H, int S, int D, int in_dtype,
+                        const void* mask_or_layout, int causal, int tile_n, Request& r)
+{
+    if (B <= 0 || H <= 0 || S <= 0 || D <= 0)
+        return fail(SR_ERR_INVALID, "B, H, S, D must be positive (got %d %d %d %d)", B, H, S, D);
+    if (in_dtype != SR_F32 && in_dtype != SR_F16 && in_dtype != SR_BF16)
+        return fail(SR_ERR_INVALID, "unknown in_dtype %d", in_dtype);
+    if (S % kRowBlock != 0) return fail(SR_ERR_UNSUPPORTED, "S=%d must be a multiple of 128", S);
+    if (S > 65536 * 64) return fail(SR_ERR_UNSUPPORTED, "S=%d too large", S);
+    if (D != 64 && D != 128) return fail(SR_ERR_UNSUPPORTED, "D=%d must be 64 or 128", D);
+    if ((int64_t)B * H * (S / kRowBlock) > INT32_MAX / 2)
+        return fail(SR_ERR_UNSUPPORTED, "too many (head, row-block) items");
+    if (tile_n != 0 && tile_n != 64 && tile_n != 128)
+        return fail(SR_ERR_UNSUPPORTED, "tile_n=%d must be 0, 64 or 128", tile_n);
+    int T = tile_n ? tile_n : default_T(e, in_dtype);
+    if (in_dtype == SR_F32 && T != 64) return fail(SR_ERR_UNSUPPORTED, "fp32 path uses T=64");
+    r = Request{e, B, H, S, causal ? 1 : 0, T};
+    if (e == SR_E_DENSE) {
+        const sr_dense_mask* m = (const sr_dense_mask*)mask_or_layout;
+        if (m && m->kv_len) {
+            for (int b = 0; b < B; ++b)
+                if (m->kv_len[b] < 0 || m->kv_len[b] > S)
+                    return fail(SR_ERR_INVALID, "kv_len[%d]=%d outside [0, S=%d]", b, m->kv_len[b], S);
+            r.kv_len = m->kv_len;
+        }
+    } else if (e == SR_E_BLOCKSPARSE) {
+        const sr_block_layout* l = (const sr_block_layout*)mask_or_layout;
+        if (!l || !l->row_ptr || !l->col_idx) return fail(SR_ERR_INVALID, "block layout missing");
+        if (l->block != 64) return fail(SR_ERR_UNSUPPORTED, "block=%d must be 64", l->block);
+        if (l->layout_heads != 1 && l->layout_heads != H)
+            return fail(SR_ERR_INVALID, "layout_heads=%d must be 1 or H=%d", l->layout_heads, H);
+        if (T != 64) return fail(SR_ERR_UNSUPPORTED, "block-sparse uses T = block = 64");
+        int nb = S / 64;
+        for (int h = 0; h < l->layout_heads; ++h) {
+            const int32_t* rp = l->row_ptr + (size_t)h * (nb + 1);
+            if (rp[0] < 0) return fail(SR_ERR_INVALID, "row_ptr[%d][0] < 0", h);
+            for (int rr = 0; rr < nb; ++rr) {
+                if (rp[rr + 1] < rp[rr]) return fail(SR_ERR_INVALID, "row_ptr decreasing (head %d row %d)", h, rr);
+                for (int32_t t = rp[rr]; t < rp[rr + 1]; ++t) {
+                    int c = l->col_idx[t];
+                    if (c < 0 || c >= nb) return fail(SR_ERR_INVALID, "col_idx %d out of range (head %d row %d)", c, h, rr);
+                    if (t > rp[rr] && c <= l->col_idx[t - 1])
+                        return fail(SR_ERR_INVALID, "col_idx not strictly ascending (head %d row %d)", h, rr);
+                }
+            }
+        }
+        r.lay = l;
+    } else if (e == SR_E_WINDOW) {
+        const sr_window* w = (const sr_window*)mask_or_layout;
+        if (!w) return fail(SR_ERR_INVALID, "window descriptor missing");
+        if (w->window < 0 || w->n_global < 0 || w->n_global > S)
+            return fail(SR_ERR_INVALID, "bad window=%d / n_global=%d", w->window, w->n_global);
+        r.window = w->window;
+        r.n_global = w->n_global;
+    } else {
+        return fail(SR_ERR_INVALID, "unknown entry %d", (int)e);
+    }
+    return SR_OK;
+}
+
+// ------------------------------------------------------------------------------ cache
+
+struct CachedSched {
+    HostSched hs;
+    void* dmem = nullptr;
+    DevSched dev{};
+};
+
+std::mutex g_mu;
+std::map<std::string, std::shared_ptr<CachedSched>> g_cache;
+
+std::string sched_key(const Request& r, int device)
+{
+    std::string k;
+    auto put = [&](int64_t x) { k.append((const char*)&x, sizeof(x)); };
+    put(device); put(r.entry); put(r.B); put(r.H); put(r.S); put(r.causal); put(r.T);
+    put(r.window); put(r.n_global);
+    if (r.kv_len) { put(1); for (int b = 0; b < r.B; ++b) put(r.kv_len[b]); } else put(0);
+    if (r.lay) {
+        int nb = r.S / 64;
+        put(r.lay->layout_heads);
+        for (int h = 0; h < r.lay->layout_heads; ++h) {
+            const int32_t* rp = r.lay->row_ptr + (size_t)h * (nb + 1);
+            for (int i = 0; i <= nb; ++i) put(rp[i] - rp[0]);
+            k.append((const char*)(r.lay->col_idx + rp[0]), sizeof(int32_t) * (rp[nb] - rp[0]));
+        }
+    }
+    return k;
+}
+
+// Host schedule only (no device), used by queries.
+sr_status host_sched(const Request& r, std::shared_ptr<CachedSched>& out, bool need_device)
+{
+    int dev = -1;
+    if (need_device) {
+        cudaError_t ce = cudaGetDevice(&dev);
+        if (ce != cudaSuccess) return fail(SR_ERR_CUDA, "cudaGetDevice: %s", cudaGetErrorString(ce));
+    }
+    std::string key = sched_key(r, need_device ? dev : -1);
+    std::lock_guard<std::mutex> lk(g_mu);
+    auto itc = g_cache.find(key);
+    if (itc != g_cache.end()) { out = itc->second; return SR_OK; }
+    auto cs = std::make_shared<CachedSched>();
+    sr_status s = build_sched(r, cs->hs);
+    if (s != SR_OK) return s;
+    if (need_device) {
+        HostSched& h = cs->hs;
+        size_t n_tp = h.tp.size(), n_ti = std::max<size_t>(h.tinfo.size(), 1), n_it = h.items.size(),
+               n_kv = h.kv_len.size();
+        size_t bytes = sizeof(int32_t) * (n_tp + n_ti + n_it + n_kv + 4);
+        cudaError_t ce = cudaMalloc(&cs->dmem, bytes);
+        if (ce != cudaSuccess) return fail(SR_ERR_CUDA, "cudaMalloc(schedule): %s", cudaGetErrorString(ce));
+        std::vector<int32_t> blob;
+        blob.reserve(bytes / 4);
+        blob.insert(blob.end(), h.tp.begin(), h.tp.end());
+        size_t o_ti = blob.size();
+        blob.insert(blob.end(), h.tinfo.begin(), h.tinfo.end());
+        if (h.tinfo.empty()) blob.push_back(0);
+        size_t o_it = blob.size();
+        blob.insert(blob.end(), h.items.begin(), h.items.end());
+        size_t o_kv = blob.size();
+        blob.insert(blob.end(), h.kv_len.begin(), h.kv_len.end());
+        ce = cudaMemcpy(cs->dmem, blob.data(), blob.size() * 4, cudaMemcpyHostToDevice);
+        if (ce != cudaSuccess) return fail(SR_ERR_CUDA, "cudaMemcpy(schedule): %s", cudaGetErrorString(ce));
+        int32_t* base = (int32_t*)cs->dmem;
+        cs->dev.tp = base;
+        cs->dev.tinfo = base + o_ti;
+        cs->dev.items = base + o_it;
+        cs->dev.kv_len = n_kv ? base + o_kv : nullptr;
+        cs->dev.n_rb = h.n_rb;
+        cs->dev.n_lh = h.n_lh;
+        cs->dev.lh_mode = h.lh_mode;
+        cs->dev.slots_per_head = h.slots_per_head;
+        cs->dev.n_items = (int)h.items.size();
+    }
+    g_cache[key] = cs;
+    out = cs;
+    return SR_OK;
+}
+
+size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
+
+void ws_layout(const HostSched& h, int B, int H, int in_dtype, int fused, sr_ws_info* info)
+{
+    memset(info, 0, sizeof(*info));
+    info->tile_n = h.T;
+    info->slots_per_head = h.slots_per_head;
+    info->n_slots = (int64_t)B * H * h.slots_per_head;
+    int elt = (in_dtype == SR_F32) ? 4 : 2;
+    info->xprime_elt_bytes = elt;
+    size_t tile_bytes = (size_t)kRowBlock * h.T * elt;
+    size_t stat_bytes = (size_t)info->n_slots * kRowBlock * sizeof(float);
+    size_t o = 0;
+    info->off_xprime = o;
+    o = align_up(o + (size_t)info->n_slots * tile_bytes, 1024);
+    if (fused) {
+        info->off_mprime = o; o = align_up(o + stat_bytes, 1024);
+        info->off_dprime = o; o = align_up(o + stat_bytes, 1024);
+        info->off_rprime = o; o = align_up(o + stat_bytes, 1024);
+    } else {
+        info->off_p = o; o = align_up(o + (size_t)info->n_slots * tile_bytes, 1024);
+    }
+    info->total_bytes = std::max<size_t>(o, 1024);
+}
+
+bool overlaps(const void* a, size_t na, const void* b, size_t nb)
+{
+    uintptr_t x = (uintptr_t)a, y = (uintptr_t)b;
+    return x < y + nb && y < x + na;
+}
+
+sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v, void* out, int B,
+              int H, int S, int D, float scale, const void* mask_or_layout, int causal,
+              const sr_exec* ex)
+{
+    if (!ex) return fail(SR_ERR_INVALID, "exec descriptor is NULL");
+    if (!q || !k || !v || !out) return fail(SR_ERR_INVALID, "q, k, v and out must be non-NULL");
+    if (!std::isfinite(scale) || !(scale > 0.f)) return fail(SR_ERR_INVALID, "scale must be finite and > 0");
+    if (ex->flags != 0) return fail(SR_ERR_INVALID, "flags must be 0");
+    Request r;
+    sr_status s = check_request(e, B, H, S, D, ex->in_dtype, mask_or_layout, causal, ex->tile_n, r);
+    if (s != SR_OK) return s;
+    if (ex->out_dtype != ex->in_dtype && ex->out_dtype != SR_F32)
+        return fail(SR_ERR_UNSUPPORTED, "out_dtype must equal in_dtype or be SR_F32");
+    if (!fused && ex->in_dtype == SR_F32)
+        return fail(SR_ERR_UNSUPPORTED, "the unfused baseline runs 16-bit dtypes only");
+    size_t in_bytes = (size_t)B * H * S * D * dtype_bytes(ex->in_dtype);
+    size_t out_bytes = (size_t)B * H * S * D * dtype_bytes(ex->out_dtype);
+    if (overlaps(out, out_bytes, q, in_bytes) || overlaps(out, out_bytes, k, in_bytes) ||
+        overlaps(out, out_bytes, v, in_bytes))
+        return fail(SR_ERR_INVALID, "out overlaps q, k or v");
+    if (((uintptr_t)q | (uintptr_t)k | (uintptr_t)v | (uintptr_t)out) & 15)
+        return fail(SR_ERR_INVALID, "q, k, v, out must be 16-byte aligned");
+    std::shared_ptr<CachedSched> cs;
+    s = host_sched(r, cs, true);
+    if (s != SR_OK) return s;
+    sr_ws_info wi;
+    ws_layout(cs->hs, B, H, ex->in_dtype, fused, &wi);
+    if (!ex->workspace || ex->workspace_bytes < wi.total_bytes)
+        return fail(SR_ERR_WORKSPACE, "workspace %zu bytes < required %zu", ex->workspace_bytes, wi.total_bytes);
+    if ((uintptr_t)ex->workspace & 255) return fail(SR_ERR_WORKSPACE, "workspace must be 256-byte aligned");
+
+    Params p{};
+    p.q = q; p.k = k; p.v = v; p.out = out;
+    p.B = B; p.H = H; p.S = S; p.D = D; p.T = r.T;
+    p.scale = scale;
+    p.scale_log2 = scale * 1.4426950408889634f;
+    p.causal = r.causal;
+    p.mask_kind = e == SR_E_WINDOW ? MK_WINDOW : (e == SR_E_BLOCKSPARSE ? MK_BLOCK : MK_DENSE);
+    p.win_half = r.window / 2;
+    p.n_global = r.n_global;
+    p.in_dtype = ex->in_dtype;
+    p.out_dtype = ex->out_dtype;
+    p.sc = cs->dev;
+    char* ws = (char*)ex->workspace;
+    p.xprime = ws + wi.off_xprime;
+    if (fused) {
+        p.mprime = (float*)(ws + wi.off_mprime);
+        p.dprime = (float*)(ws + wi.off_dprime);
+        p.rprime = (float*)(ws + wi.off_rprime);
+    } else {
+        p.pbuf = ws + wi.off_p;
+    }
+    cudaStream_t st = (cudaStream_t)ex->stream;
+    int64_t nl = 0;
+    cudaError_t ce;
+    if (fused) {
+        ce = ex->in_dtype == SR_F32 ? launch_simt_f32(p, st, &nl) : launch_tc_fused(p, st, &nl);
+    } else {
+        ce = launch_tc_unfused(p, st, &nl);
+    }
+    g_launches += nl;
+    if (ce != cudaSuccess) return fail(SR_ERR_CUDA, "kernel launch: %s", cudaGetErrorString(ce));
+    return SR_OK;
+}
+
+}  // namespace
+
+// ================================================================================== C ABI
+
+extern "C" {
+
+sr_status sr_mha_dense(const void* q, const void* k, const void* v, void* out, int B, int H, int S,
+                       int D, float scale, const sr_dense_mask* m, int causal, const sr_exec* ex)
+{
+    return run(SR_E_DENSE, 1, q, k, v, out, B, H, S, D, scale, m, causal, ex);
+}
+sr_status sr_mha_blocksparse(const void* q, const void* k, const void* v, void* out, int B, int H,
+                             int S, int D, float scale, const sr_block_layout* l, int causal,
+                             const sr_exec* ex)
+{
+    return run(SR_E_BLOCKSPARSE, 1, q, k, v, out, B, H, S, D, scale, l, causal, ex);
+}
+sr_status sr_mha_sliding_window(const void* q, const void* k, const void* v, void* out, int B,
+                                int H, int S, int D, float scale, const sr_window* w, int causal,
+                                const sr_exec* ex)
+{
+    return run(SR_E_WINDOW, 1, q, k, v, out, B, H, S, D, scale, w, causal, ex);
+}
+sr_status sr_mha_dense_unfused(const void* q, const void* k, const void* v, void* out, int B,
+                               int H, int S, int D, float scale, const sr_dense_mask* m, int causal,
+                               const sr_exec* ex)
+{
+    return run(SR_E_DENSE, 0, q, k, v, out, B, H, S, D, scale, m, causal, ex);
+}
+sr_status sr_mha_blocksparse_unfused(const void* q, const void* k, const void* v, void* out, int B,
+                                     int H, int S, int D, float scale, const sr_block_layout* l,
+                                     int causal, const sr_exec* ex)
+{
+    return run(SR_E_BLOCKSPARSE, 0, q, k, v, out, B, H, S, D, scale, l, causal, ex);
+}
+sr_status sr_mha_sliding_window_unfused(const void* q, const void* k, const void* v, void* out,
+                                        int B, int H, int S, int D, float scale, const sr_window* w,
+                                        int causal, const sr_exec* ex)
+{
+    return run(SR_E_WINDOW, 0, q, k, v, out, B, H, S, D, scale, w, causal, ex);
+}
+
+sr_status sr_workspace_query(sr_entry e, int fused, int B, int H, int S, int D, sr_dtype in_dtype,
+                             const void* mask_or_layout, int causal, int tile_n, sr_ws_info* info)
+{
+    if (!info) return fail(SR_ERR_INVALID, "info is NULL");
+    Request r;
+    sr_status s = check_request(e, B, H, S, D, in_dtype, mask_or_layout, causal, tile_n, r);
+    if (s != SR_OK) return s;
+    std::shared_ptr<CachedSched> cs;
+    s = host_sched(r, cs, false);
+    if (s != SR_OK) return s;
+    ws_layout(cs->hs, B, H, in_dtype, fused, info);
+    return SR_OK;
+}
+
+size_t sr_workspace_bytes(sr_entry e, int fused, int B, int H, int S, int D, sr_dtype in_dtype,
+                          const void* mask_or_layout, int causal, int tile_n)
+{
+    sr_ws_info info;
+    if (sr_workspace_query(e, fused, B, H, S, D, in_dtype, mask_or_layout, causal, tile_n, &info) != SR_OK)
+        return 0;
+    return info.total_bytes;
+}
+
+sr_status sr_schedule_stats(sr_entry e, int B, int H, int S, const void* mask_or_layout, int causal,
+                            int tile_n, int64_t* n_tiles, int64_t* stored_elems)
+{
+    Request r;
+    sr_status s = check_request(e, B, H, S, 64, SR_F16, mask_or_layout, causal, tile_n, r);
+    if (s != SR_OK) return s;
+    std::shared_ptr<CachedSched> cs;
+    s = host_sched(r, cs, false);
+    if (s != SR_OK) return s;
+    if (n_tiles) *n_tiles = cs->hs.n_tiles;
+    if (stored_elems) *stored_elems = cs->hs.stored_elems;
+    return SR_OK;
+}
+
+const char* sr_status_string(sr_status s)
+{
+    switch (s) {
+    case SR_OK: return "SR_OK";
+    case SR_ERR_INVALID: return "SR_ERR_INVALID";
+    case SR_ERR_UNSUPPORTED: return "SR_ERR_UNSUPPORTED";
+    case SR_ERR_WORKSPACE: return "SR_ERR_WORKSPACE";
+    case SR_ERR_CUDA: return "SR_ERR_CUDA";
+    }
+    return "SR_?";
+}
+
+const char* sr_last_error(void) { return g_err; }
+int64_t sr_launch_count(void) { return g_launches.load(); }
+const char* sr_version(void) { return "sr_mha 0.1 (sm_100a)"; }
+
+}  // extern "C"

@@ -1,0 +1,87 @@
+// sr_internal.h -- shared declarations of the sr_mha library (host + device).  Not installed.
+//
+// Terminology:
+//   row-block  128 consecutive query rows of one head (the M = 128 tcgen05 tile)
+//   key tile   T consecutive keys (T = LS sub-vector width = GEMM1 output-tile width)
+//   tile       (head, row-block, key tile); its two 64-row halves can be valid independently
+//              (block-sparse pairs of 64-row block-rows, causal diagonals with T = 64, band edges)
+//   slot       storage index of a tile inside the workspace: X' tile, and 128 m'/d'/r' floats
+//   item       (head, row-block): the unit of work of the GEMM kernels, scheduled longest-first
+#pragma once
+#include <cstddef>
+#include <cstdint>
+
+#include <cuda_runtime.h>
+
+namespace sr {
+
+constexpr int kRowBlock = 128;  // M of every tcgen05 tile
+constexpr int kHalf = 64;       // validity granularity of tile rows
+
+enum MaskKind : int { MK_DENSE = 0, MK_BLOCK = 1, MK_WINDOW = 2 };
+enum DType : int { DT_F32 = 0, DT_F16 = 1, DT_BF16 = 2 };
+// lh_mode: which layout list a head g = b*H + h uses
+enum LhMode : int { LH_ONE = 0, LH_BATCH = 1, LH_HEAD = 2 };
+
+// tile info word: key-tile index in units of T (bits 0-15) | half-valid bits (16: rows 0-63,
+// 17: rows 64-127)
+__host__ __device__ inline int tinfo_kt(int32_t w) { return w & 0xFFFF; }
+__host__ __device__ inline int tinfo_half(int32_t w) { return (w >> 16) & 3; }
+
+// Device-side view of a cached schedule.
+struct DevSched {
+    const int32_t* tp;      // [n_lh][n_rb+1] absolute offsets into tinfo
+    const int32_t* tinfo;   // [n_tiles_list]
+    const int32_t* items;   // [n_items] g * n_rb + rb, longest first
+    const int32_t* kv_len;  // [B] or nullptr
+    int n_rb, n_lh, lh_mode, slots_per_head, n_items;
+};
+
+// Everything a kernel needs to know about one call.
+struct Params {
+    const void* q;
+    const void* k;
+    const void* v;
+    void* out;
+    int B, H, S, D, T;
+    float scale;       // multiplies Q K^T
+    float scale_log2;  // scale * log2(e): the GEMM1 epilogue works in base 2
+    int causal;
+    int mask_kind;     // MaskKind (element masks: kv_len, causal, window; blocks come from tinfo)
+    int win_half;      // window / 2
+    int n_global;
+    int in_dtype, out_dtype;
+    DevSched sc;
+    void* xprime;      // X' tiles (recomposed) or score tiles S (unfused)
+    void* pbuf;        // unfused: P tiles
+    float* mprime;
+    float* dprime;
+    float* rprime;
+};
+
+__host__ __device__ inline int lh_of(const DevSched& s, int g, int H)
+{
+    return s.lh_mode == LH_ONE ? 0 : (s.lh_mode == LH_BATCH ? g / H : g % H);
+}
+
+// Element mask: kept iff every active criterion keeps (i, j).  Block-level
+// sparsity is not evaluated here: it is encoded in the tile list / half bits.
+__host__ __device__ inline bool elem_kept(const Params& p, int kvl, int i, int j)
+{
+    if (j >= kvl) return false;
+    if (p.causal && j > i) return false;
+    if (p.mask_kind == MK_WINDOW) {
+        int dd = i - j;
+        dd = dd < 0 ? -dd : dd;
+        if (!(dd <= p.win_half || i < p.n_global || j < p.n_global)) return false;
+    }
+    return true;
+}
+
+// ---- launchers (return cudaError_t of the launch)
+cudaError_t launch_simt_f32(const Params& p, cudaStream_t st, int64_t* nlaunch);
+cudaError_t launch_ir(const Params& p, cudaStream_t st, int64_t* nlaunch);
+cudaError_t launch_tc_fused(const Params& p, cudaStream_t st, int64_t* nlaunch);
+cudaError_t launch_tc_unfused(const Params& p, cudaStream_t st, int64_t* nlaunch);
+
+}  // namespace sr

@@ -1,0 +1,301 @@
+"""GPU parity: the CUDA path (through the C ABI) against the fp64 oracle, element by element.
+
+Tolerances (BASELINE.json north_star):
+  fp32 mode (SIMT):                       max |gpu - oracle| <= 1e-5
+  fp16 / bf16, fp32-accumulated context:  max |gpu - oracle| <= 1e-2   (out_dtype = float32)
+  fp16 / bf16 stored output:              <= 1e-2 + half an ulp of the output dtype at |o|
+Small cases span several tiles and ragged (masked) tails; full BASELINE configs are checked on
+sampled rows the oracle computes one by one, plus the V == 1 invariant on every row.
+"""
+import math
+
+import numpy as np
+import pytest
+
+import oracle
+import workloads as W
+from tests.gpu_util import oracle_mask, qkv
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+if not torch.cuda.is_available():  # pragma: no cover
+    pytest.skip("needs a CUDA device", allow_module_level=True)
+
+import paper_conf_iiswc_choilkha22_b200 as sr  # noqa: E402
+
+TORCH = {"f32": torch.float32, "f16": torch.float16, "bf16": torch.bfloat16}
+
+
+def _ulp_half(dtype, ref):
+    mant = {"f16": 10, "bf16": 7, "f32": 23}[dtype]
+    e = np.floor(np.log2(np.maximum(np.abs(ref), 2.0 ** -14)))
+    return 0.5 * 2.0 ** (e - mant)
+
+
+def run_case(kind, B, H, S, D, dtype, *, causal=False, kv_len=None, layout=None, window=0, n_global=0,
+             tile_n=0, fused=True, seed=0, out_f32=True):
+    t, q, k, v = qkv(B, H, S, D, dtype, seed)
+    scale = 1 / math.sqrt(D)
+    od = torch.float32 if out_f32 else TORCH[dtype]
+    kw = dict(scale=scale, causal=causal, tile_n=tile_n, fused=fused, out_dtype=od)
+    if kind == "dense":
+        o = sr.mha_dense(q, k, v, kv_len=kv_len, **kw)
+    elif kind == "block":
+        o = sr.mha_blocksparse(q, k, v, layout, **kw)
+    else:
+        o = sr.mha_sliding_window(q, k, v, window, n_global, **kw)
+    torch.cuda.synchronize()
+    ref = oracle.attention(t.q64, t.k64, t.v64, scale,
+                           oracle_mask(kind, kv_len, causal, layout, window, n_global))
+    return o.float().cpu().numpy().astype(np.float64), ref
+
+
+def assert_close(o, ref, dtype, out_f32=True, what=""):
+    err = np.abs(o - ref)
+    if dtype == "f32":
+        tol = 1e-5
+    elif out_f32:
+        tol = 1e-2
+    else:
+        tol = 1e-2 + _ulp_half(dtype, ref)
+    bad = err > tol
+    assert not bad.any(), f"{what}: {bad.sum()} elements over tolerance, max err {err.max():.3g}"
+    assert np.isfinite(o).all()
+    return float(err.max())
+
+
+# ------------------------------------------------------------------------------------ fp32 path
+
+def test_config1_fp32():
+    cfg = W.config(1)
+    t = W.config_tensors(cfg)
+    from tests.gpu_util import to_dev
+    q, k, v = (to_dev(x, "f32") for x in (t.q_s, t.k_s, t.v_s))
+    o = sr.mha_dense(q, k, v, scale=cfg.scale).cpu().numpy()
+    ref = oracle.attention(t.q64, t.k64, t.v64, cfg.scale)
+    assert np.abs(o - ref).max() <= 1e-5
+
+
+def test_p3_closed_form_fp32_with_intermediates():
+    """Pin P3 at the C1 shape through the GPU: O, and m', d', r' read back from the workspace."""
+    S, D, T = 128, 64, 64
+    q = torch.zeros(1, 1, S, D)
+    k = torch.zeros(1, 1, S, D)
+    for i in range(4):
+        q[0, 0, i, i] = math.log(3.0)
+        k[0, 0, i, i] = 1.0
+    q, k = q.cuda(), k.cuda()
+    v = k.clone()
+    mask = sr.dense_mask(None)
+    info = sr.workspace_info(mask, 1, 1, S, D, sr.SR_F32, tile_n=T)
+    ws = torch.zeros(info["total_bytes"], dtype=torch.uint8, device="cuda")
+    o = sr.call(mask, q, k, v, scale=1.0, tile_n=T, workspace=ws).cpu().numpy()[0, 0]
+    want = np.zeros((S, D))
+    for i in range(S):
+        for c in range(4):
+            want[i, c] = (3.0 if c == i else 1.0) / 130 if i < 4 else 1 / 128
+    np.testing.assert_allclose(o, want, atol=1e-7)
+    n = info["n_slots"] * 128
+    mp = ws[info["off_mprime"]:].view(torch.float32)[:n].cpu().numpy().reshape(-1, 128)
+    dp = ws[info["off_dprime"]:].view(torch.float32)[:n].cpu().numpy().reshape(-1, 128)
+    rp = ws[info["off_rprime"]:].view(torch.float32)[:n].cpu().numpy().reshape(-1, 128)
+    # slots of item (head 0, row-block 0): tiles kt = 0, 1
+    np.testing.assert_allclose(mp[:2, 0], [math.log(3.0), 0.0], atol=1e-6)
+    np.testing.assert_allclose(dp[:2, 0], [22.0, 64.0], rtol=1e-6)
+    np.testing.assert_allclose(rp[:2, 0], [3 / 130, 1 / 130], rtol=1e-6)
+
+
+@pytest.mark.parametrize("kind", ["dense", "causal", "kv", "block", "window"])
+def test_fp32_masks(kind):
+    B, H, S, D = 2, 2, 256, 64
+    kw = {}
+    mk = "dense"
+    if kind == "causal":
+        kw = dict(causal=True)
+    elif kind == "kv":
+        kw = dict(kv_len=[200, 3])
+    elif kind == "block":
+        mk, kw = "block", dict(layout=W.random_layout(H, S // 64, 64, 0.4, seed=4))
+    elif kind == "window":
+        mk, kw = "window", dict(window=100, n_global=5, causal=False)
+    o, ref = run_case(mk, B, H, S, D, "f32", **kw)
+    assert_close(o, ref, "f32", what=kind)
+
+
+# ------------------------------------------------------------------------------------ tensor cores
+
+DENSE_CASES = [
+    # (dtype, D, T, S, causal, kv_len)
+    ("f16", 64, 128, 128, False, None),
+    ("f16", 64, 128, 384, False, None),
+    ("bf16", 64, 128, 256, False, None),
+    ("f16", 128, 128, 256, False, None),
+    ("bf16", 128, 128, 384, True, None),
+    ("f16", 64, 64, 256, True, None),
+    ("bf16", 128, 64, 256, True, None),
+    ("f16", 64, 128, 512, False, [512, 511, 384, 300, 257, 128, 65, 1]),
+    ("f16", 64, 64, 384, True, [384, 100, 1]),
+]
+
+
+@pytest.mark.parametrize("case", DENSE_CASES, ids=lambda c: f"{c[0]}-D{c[1]}-T{c[2]}-S{c[3]}-c{int(c[4])}-kv{c[5] is not None}")
+@pytest.mark.parametrize("fused", [True, False], ids=["recomposed", "unfused"])
+def test_dense_tc(case, fused):
+    dtype, D, T, S, causal, kv = case
+    B = len(kv) if kv else 2
+    o, ref = run_case("dense", B, 3, S, D, dtype, causal=causal, kv_len=kv, tile_n=T, fused=fused)
+    assert_close(o, ref, dtype, what=str(case))
+
+
+@pytest.mark.parametrize("dtype", ["f16", "bf16"])
+def test_dense_tc_stored_dtype(dtype):
+    o, ref = run_case("dense", 2, 2, 256, 128, dtype, causal=True, out_f32=False)
+    assert_close(o, ref, dtype, out_f32=False)
+
+
+@pytest.mark.parametrize("fused", [True, False], ids=["recomposed", "unfused"])
+@pytest.mark.parametrize("density,causal,lh", [(0.3, False, 3), (0.6, True, 3), (0.25, False, 1)])
+def test_blocksparse_tc(fused, density, causal, lh):
+    S, H = 512, 3
+    lay = W.random_layout(lh, S // 64, 64, density, seed=int(density * 100) + lh)
+    o, ref = run_case("block", 2, H, S, 64, "f16", causal=causal, layout=lay, fused=fused)
+    assert_close(o, ref, "f16")
+
+
+def test_blocksparse_bigbird_small():
+    lay = W.bigbird_layout(2, 1024, 64)
+    o, ref = run_case("block", 1, 2, 1024, 64, "f16", layout=lay)
+    assert_close(o, ref, "f16")
+
+
+def test_blocksparse_empty_rows():
+    """A block-row with no blocks outputs 0 (reading R9)."""
+    S, nb = 256, 4
+    lay = W.csr_from_sets(64, [[{0, 1}, set(), {2}, {0, 3}]])
+    o, ref = run_case("block", 1, 1, S, 64, "f16", layout=lay)
+    assert np.all(o[0, 0, 64:128] == 0)
+    assert_close(o, ref, "f16")
+
+
+@pytest.mark.parametrize("fused", [True, False], ids=["recomposed", "unfused"])
+@pytest.mark.parametrize("window,n_global,causal,T", [(0, 0, False, 64), (2, 1, False, 64), (126, 8, False, 64),
+                                                      (128, 0, True, 64), (130, 64, False, 128),
+                                                      (254, 8, True, 128), (512, 8, False, 64)])
+def test_window_tc(fused, window, n_global, causal, T):
+    o, ref = run_case("window", 1, 2, 768, 64, "f16", window=window, n_global=n_global, causal=causal,
+                      tile_n=T, fused=fused)
+    assert_close(o, ref, "f16")
+
+
+def test_all_block_layouts_nb2():
+    """Pin P7 on the GPU: every block layout with non-empty rows at nb = 2 (9 layouts), S = 128."""
+    import itertools
+    opts = [c for r in (1, 2) for c in itertools.combinations(range(2), r)]
+    for rows in itertools.product(opts, repeat=2):
+        lay = W.csr_from_sets(64, [list(rows)])
+        o, ref = run_case("block", 1, 1, 128, 64, "f16", layout=lay)
+        assert_close(o, ref, "f16", what=str(rows))
+
+
+def test_kv_len_one_and_zero():
+    o, ref = run_case("dense", 3, 2, 256, 64, "f16", kv_len=[1, 0, 129])
+    assert np.all(o[1] == 0)
+    assert_close(o, ref, "f16")
+
+
+# ------------------------------------------------------------------------------------ intermediates
+
+def test_intermediates_match_recomposed_oracle():
+    """m', d', r' read back from the workspace vs the oracle's Eq. (2) decomposition (T = 128)."""
+    B, H, S, D, T = 1, 2, 384, 64, 128
+    t, q, k, v = qkv(B, H, S, D, "f16", seed=3)
+    mask = sr.dense_mask(None)
+    info = sr.workspace_info(mask, B, H, S, D, sr.SR_F16, causal=True, tile_n=T)
+    ws = torch.zeros(info["total_bytes"], dtype=torch.uint8, device="cuda")
+    sr.call(mask, q, k, v, scale=0.125, causal=True, tile_n=T, workspace=ws)
+    torch.cuda.synchronize()
+    _, mp_ref, dp_ref, rp_ref = oracle.recomposed(t.q64, t.k64, t.v64, 0.125, T, oracle.Mask(causal=True))
+    n = info["n_slots"] * 128
+    get = lambda key: ws[info[key]:].view(torch.float32)[:n].cpu().numpy().reshape(B * H, -1, 128)
+    mp, dp, rp = get("off_mprime"), get("off_dprime"), get("off_rprime")
+    # causal with T = M = 128: row-block rb owns tiles kt = 0..rb -> slots rb*(rb+1)/2 + kt
+    for g in range(B * H):
+        for rb in range(S // 128):
+            for kt in range(rb + 1):
+                s = rb * (rb + 1) // 2 + kt
+                rows = slice(rb * 128, rb * 128 + 128)
+                np.testing.assert_allclose(mp[g, s], mp_ref[g, kt, rows], atol=2e-5)
+                np.testing.assert_allclose(dp[g, s], dp_ref[g, kt, rows], rtol=2e-3)
+                np.testing.assert_allclose(rp[g, s], rp_ref[g, kt, rows], rtol=2e-3, atol=1e-7)
+
+
+def test_T64_equals_T128():
+    """Pin P5 on the GPU: sub-vector width 64 and 128 give the same context within tolerance."""
+    o64, ref = run_case("dense", 2, 2, 512, 64, "f16", causal=True, tile_n=64)
+    o128, _ = run_case("dense", 2, 2, 512, 64, "f16", causal=True, tile_n=128)
+    assert np.abs(o64 - o128).max() < 2e-3
+    assert_close(o64, ref, "f16")
+
+
+# ------------------------------------------------------------------------------------ full configs
+
+def _config_call(cfg, t, fused=True, out_f32=True):
+    from tests.gpu_util import to_dev
+    q, k, v = (to_dev(x, cfg.dtype) for x in (t.q_s, t.k_s, t.v_s))
+    od = torch.float32 if out_f32 else None
+    if cfg.kind == "dense":
+        o = sr.mha_dense(q, k, v, scale=cfg.scale, kv_len=cfg.kv_len, causal=cfg.causal, out_dtype=od, fused=fused)
+        m = oracle.Mask(kv_len=cfg.kv_len, causal=cfg.causal)
+    elif cfg.kind == "blocksparse":
+        lay = W.config_layout(cfg)
+        o = sr.mha_blocksparse(q, k, v, lay, scale=cfg.scale, out_dtype=od, fused=fused)
+        m = oracle.Mask(kind="block", layout=lay)
+    else:
+        o = sr.mha_sliding_window(q, k, v, cfg.window, cfg.n_global, scale=cfg.scale, out_dtype=od, fused=fused)
+        m = oracle.Mask(kind="window", window=cfg.window, n_global=cfg.n_global)
+    torch.cuda.synchronize()
+    return o, m
+
+
+def _sample_rows(cfg, n, seed):
+    rng = np.random.Generator(np.random.PCG64(seed))
+    BH, S = cfg.BH, cfg.S
+    edge = [0, 1, 63, 64, 127, 128, S - 1, S - 2, 255, 256]
+    rows = [g * S + i for g in (0, BH - 1) for i in edge]
+    rows += rng.integers(0, BH * S, size=n - len(rows)).tolist()
+    return np.array(sorted(set(rows)), dtype=np.int64)
+
+
+@pytest.mark.parametrize("idx", [2, 3, 4, 5])
+@pytest.mark.parametrize("fused", [True, False], ids=["recomposed", "unfused"])
+def test_full_config_sampled_rows(idx, fused):
+    cfg = W.config(idx)
+    t = W.config_tensors(cfg)
+    o, m = _config_call(cfg, t, fused=fused)
+    rows = _sample_rows(cfg, 192, seed=idx)
+    ref = oracle.attention_rows(t.q64, t.k64, t.v64, cfg.scale, rows, m)
+    got = o.reshape(-1, cfg.D)[torch.from_numpy(rows).cuda()].double().cpu().numpy()
+    assert_close(got, ref, cfg.dtype, what=f"config {idx}")
+
+
+@pytest.mark.parametrize("idx", [2, 3, 4, 5])
+def test_full_config_rows_sum_to_one(idx):
+    """Pin P4 at full size: with V == 1 every output element equals 1 (all rows keep >= 1 key)."""
+    cfg = W.config(idx)
+    t = W.config_tensors(cfg)
+    t.v_s = np.ones_like(t.v_s) if cfg.dtype != "bf16" else np.full_like(t.v_s, 0x3F80)
+    o, _ = _config_call(cfg, t, out_f32=True)
+    err = (o - 1).abs().max().item()
+    assert err < 2e-3, err
+
+
+def test_abi_errors_on_gpu():
+    q = torch.zeros(1, 1, 128, 64, dtype=torch.float16, device="cuda")
+    with pytest.raises(sr.SrError) as e:
+        sr.mha_dense(q, q, q, out=q)
+    assert e.value.status == sr.SR_ERR_INVALID
+    q2 = torch.zeros(1, 1, 100, 64, dtype=torch.float16, device="cuda")
+    with pytest.raises(sr.SrError) as e:
+        sr.mha_dense(q2, q2, q2)
+    assert e.value.status == sr.SR_ERR_UNSUPPORTED
