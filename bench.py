@@ -1,0 +1,434 @@
+#!/usr/bin/env python
+"""bench.py -- attention layers/s and HBM bytes/layer of the softmax-recomposed path vs the in-repo
+unfused path on B200 (BASELINE.json "metric").
+
+One step = one attention layer (all B*H heads of the workload config) through the C ABI: GEMM1 +
+Local Softmax -> IR -> GS + GEMM2.  Inputs are seeded synthetic tensors
+resident in HBM before the timed region; L2 is flushed (256 MiB write) before every timed step.
+Timing: CUDA events on the launching stream, barrier + synchronize around the timed region, max
+over ranks.  Multi-GPU (torchrun): every rank runs its own full layer on its own inputs (weak
+scaling, no collective on the data path); value = layers of all ranks / max-over-ranks time.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config 2] [--impl ours|reference]
+
+--impl reference times the fp64 CPU oracle (the only reference this paper-only task has) on a
+bounded sample of rows of the same workload, rank 0 only.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+import workloads as W  # noqa: E402
+
+METRIC = json.load(open(os.path.join(ROOT, "BASELINE.json")))["metric"]
+FLUSH_BYTES = 256 << 20
+
+
+def describe(cfg):
+    m = {"dense": (("padding kv_len=" + str(cfg.kv_len)) if cfg.kv_len else ("causal" if cfg.causal else "none")),
+         "blocksparse": "BigBird block 64: 3 window + 2 global + 3 random (622 blocks/head)",
+         "window": f"Longformer window {cfg.window} + {cfg.n_global} global"}[cfg.kind]
+    return (f"C{cfg.idx} {cfg.name}: B={cfg.B} H={cfg.H} S={cfg.S} D={cfg.D} {cfg.dtype}, mask: {m}")
+
+
+# ----------------------------------------------------------------------------- clocks
+
+class Clocks:
+    """nvidia-smi sampler running DURING the timed region (B200_PROFILING.md clocks line)."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index):
+        self.idx = gpu_index
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        self.p = None
+
+    def start(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                                       "-i", str(self.idx), "-lms", "200"], stdout=self.f, stderr=subprocess.DEVNULL)
+        except OSError:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return None
+        self.p.terminate()
+        self.p.wait()
+        self.f.flush()
+        rows = [l.split(",") for l in open(self.f.name).read().strip().splitlines() if l.strip()]
+        os.unlink(self.f.name)
+        if not rows:
+            return None
+        sm = [float(r[1]) for r in rows if r[1].strip().replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in rows if r[2].strip().replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({n for r in rows for n, v in zip(names, r[5:9]) if v.strip() == "Active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(rows)}
+
+
+# ----------------------------------------------------------------------------- byte model
+
+def alg_bytes(cfg, stored, T, out_bytes=None):
+    """Algorithmic HBM bytes per layer: Q, K, V, O once; the attention matrix
+    written and read once (recomposed) or four times (unfused); m', d', r'."""
+    e = 4 if cfg.dtype == "f32" else 2
+    eo = e if out_bytes is None else out_bytes
+    bhsd = cfg.BH * cfg.S * cfg.D
+    xe = 4 if cfg.dtype == "f32" else 2
+    rows_tiles = stored / T  # (row, tile) pairs
+    rec = {"gemm1_ls": 2 * bhsd * e + xe * stored + 8 * rows_tiles,
+           "ir": 12 * rows_tiles,
+           "gs_gemm2": xe * stored + 4 * rows_tiles + bhsd * e + bhsd * eo}
+    unf = {"gemm1": 2 * bhsd * e + 2 * stored, "softmax": 4 * stored, "gemm2": 2 * stored + bhsd * e + bhsd * eo}
+    return rec, unf
+
+
+def flops(cfg, stored):
+    return 4.0 * cfg.D * stored  # two GEMMs, 2 flops per MAC, over stored score elements
+
+
+# ----------------------------------------------------------------------------- GPU arm
+
+class Layer:
+    def __init__(self, cfg, device, seed_base, sr, torch):
+        self.cfg, self.sr, self.torch = cfg, sr, torch
+        t = W.make_qkv(cfg.B, cfg.H, cfg.S, cfg.D, cfg.dtype, seed_base=seed_base)
+        self.host = {}
+        self.dev = {}
+        for n in ("q", "k", "v"):
+            a = getattr(t, n + "_s")
+            if cfg.dtype == "bf16":
+                ht = torch.from_numpy(a.view(np.int16).copy()).view(torch.bfloat16)
+            else:
+                ht = torch.from_numpy(np.ascontiguousarray(a))
+            self.host[n] = ht.pin_memory()
+            self.dev[n] = self.host[n].to(device)
+        tdt = {"f32": torch.float32, "f16": torch.float16, "bf16": torch.bfloat16}[cfg.dtype]
+        self.out = torch.empty((cfg.B, cfg.H, cfg.S, cfg.D), dtype=tdt, device=device)
+        self.out_host = torch.empty_like(self.out, device="cpu").pin_memory()
+        if cfg.kind == "dense":
+            self.mask = sr.dense_mask(cfg.kv_len)
+        elif cfg.kind == "blocksparse":
+            self.mask = sr.block_mask(W.config_layout(cfg))
+        else:
+            self.mask = sr.window_mask(cfg.window, cfg.n_global)
+        self.kw = dict(scale=cfg.scale, causal=cfg.causal)
+        in_dt = sr.dtype_code(tdt)
+        self.ws = {}
+        for fused in (True, False):
+            if cfg.dtype == "f32" and not fused:
+                continue
+            info = sr.workspace_info(self.mask, cfg.B, cfg.H, cfg.S, cfg.D, in_dt, causal=cfg.causal, fused=fused)
+            self.ws[fused] = torch.empty(info["total_bytes"], dtype=torch.uint8, device=device)
+            self.T = info["tile_n"]
+        self.n_tiles, self.stored = sr.schedule_stats(self.mask, cfg.B, cfg.H, cfg.S, causal=cfg.causal)
+
+    def run(self, fused=True, stages=0, q=None, k=None, v=None):
+        d = self.dev
+        return self.sr.call(self.mask, q if q is not None else d["q"], k if k is not None else d["k"],
+                            v if v is not None else d["v"], out=self.out, fused=fused, stages=stages,
+                            workspace=self.ws[fused], **self.kw)
+
+
+def timed(torch, fn, steps, warmup, flush, per_step_pre=None):
+    """W warm-up + K timed steps; L2 flushed before each; returns per-step device ms list."""
+    ev = []
+    for s in range(warmup + steps):
+        if flush is not None:
+            flush.zero_()
+        if per_step_pre:
+            per_step_pre()
+        a = torch.cuda.Event(enable_timing=True)
+        b = torch.cuda.Event(enable_timing=True)
+        a.record()
+        fn()
+        b.record()
+        if s >= warmup:
+            ev.append((a, b))
+    torch.cuda.synchronize()
+    return [a.elapsed_time(b) for a, b in ev]
+
+
+def dist_max(torch, x, world):
+    if world == 1:
+        return x
+    t = torch.tensor([x], dtype=torch.float64, device="cuda")
+    torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+    return float(t.item())
+
+
+def barrier(torch, world):
+    if world > 1:
+        torch.distributed.barrier()
+    torch.cuda.synchronize()
+
+
+def load_ncu_traffic():
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(p):
+        try:
+            return json.load(open(p))
+        except ValueError:
+            return {}
+    return {}
+
+
+def gpu_arm(args, rank, world, local_rank):
+    import torch
+    import paper_conf_iiswc_choilkha22_b200 as sr
+    torch.cuda.set_device(local_rank)
+    device = torch.device("cuda", local_rank)
+    sr.lib()
+    peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))) if os.path.exists(
+        os.path.join(ROOT, "MEASURED_PEAKS.json")) else {}
+    hbm_peak = peaks.get("hbm_gbs", 6650.0)
+    peak_src = "MEASURED_PEAKS.json hbm_gbs (measured)" if "hbm_gbs" in peaks else "fallback 6650 GB/s (B200_PROFILING.md)"
+    cfg = W.config(args.config)
+    flush = None if args.no_flush else torch.empty(FLUSH_BYTES, dtype=torch.uint8, device=device)
+    L = Layer(cfg, device, seed_base=cfg.idx + 1000 * rank, sr=sr, torch=torch)
+    K, Wm = args.steps, args.warmup
+
+    # ---- headline: recomposed layer, inputs resident in HBM
+    L.run()
+    barrier(torch, world)
+    vis = os.environ.get("CUDA_VISIBLE_DEVICES")
+    phys = vis.split(",")[local_rank] if vis else str(local_rank)
+    clk = Clocks(phys)
+    clk.start()
+    t_end = time.perf_counter() + 0.8  # keep the GPU under this load while nvidia-smi samples
+    while time.perf_counter() < t_end:
+        timed(torch, lambda: L.run(), 5, 0, flush)
+    n0 = sr.launch_count()
+    ms_rec = timed(torch, lambda: L.run(), K, Wm, flush)
+    launches = (sr.launch_count() - n0) * K // (K + Wm)
+    clocks = clk.stop()
+    barrier(torch, world)
+    ms_step = dist_max(torch, statistics.mean(ms_rec), world)
+
+    # ---- unfused in-repo baseline (same tiles, same skipping)
+    ms_unf = None
+    if cfg.dtype != "f32":
+        L.run(fused=False)
+        barrier(torch, world)
+        ms_unf = dist_max(torch, statistics.mean(timed(torch, lambda: L.run(fused=False), K, Wm, flush)), world)
+
+    # ---- per-kernel durations inside the step (stage-selected launches, events on the stream)
+    rec_b, unf_b = alg_bytes(cfg, L.stored, L.T)
+    kern = {}
+    for name, bit in (("gemm1_ls", 1), ("ir", 2), ("gs_gemm2", 4)):
+        t = statistics.mean(timed(torch, lambda b=bit: L.run(stages=b), K, Wm, flush))
+        kern[name] = {"us": round(t * 1e3, 3), "alg_bytes": int(rec_b[name]),
+                      "GB/s": round(rec_b[name] / (t * 1e-3) / 1e9, 1)}
+    kern_unf = {}
+    if cfg.dtype != "f32":
+        for name, bit in (("gemm1", 1), ("softmax", 2), ("gemm2", 4)):
+            L.run(fused=False)
+            t = statistics.mean(timed(torch, lambda b=bit: L.run(fused=False, stages=b), K, Wm, flush))
+            kern_unf[name] = {"us": round(t * 1e3, 3), "alg_bytes": int(unf_b[name]),
+                              "GB/s": round(unf_b[name] / (t * 1e-3) / 1e9, 1)}
+
+    # ---- end to end through the public API: pinned host -> device, layer, device -> host
+    h2d = sum(L.host[n].numel() * L.host[n].element_size() for n in ("q", "k", "v"))
+    d2h = L.out.numel() * L.out.element_size()
+    qd, kd, vd = (torch.empty_like(L.dev[n]) for n in ("q", "k", "v"))
+
+    def e2e_step():
+        qd.copy_(L.host["q"], non_blocking=True)
+        kd.copy_(L.host["k"], non_blocking=True)
+        vd.copy_(L.host["v"], non_blocking=True)
+        L.run(q=qd, k=kd, v=vd)
+        L.out_host.copy_(L.out, non_blocking=True)
+
+    barrier(torch, world)
+    ms_e2e = dist_max(torch, statistics.mean(timed(torch, e2e_step, K, Wm, flush)), world)
+
+    # ---- other configs (same run, fewer steps): layers/s and bytes, recomposed vs unfused
+    others = {}
+    if args.all_configs and world == 1:
+        for c2 in W.CONFIGS:
+            if c2.idx == cfg.idx:
+                continue
+            L2 = Layer(c2, device, seed_base=c2.idx, sr=sr, torch=torch)
+            L2.run()
+            tr = statistics.mean(timed(torch, lambda: L2.run(), 10, 3, flush))
+            r2, u2 = alg_bytes(c2, L2.stored, L2.T)
+            ent = {"layers_per_s": round(1e3 / tr, 1), "ms": round(tr, 4),
+                   "alg_bytes_recomposed": int(sum(r2.values()))}
+            if c2.dtype != "f32":
+                L2.run(fused=False)
+                tu = statistics.mean(timed(torch, lambda: L2.run(fused=False), 10, 3, flush))
+                ent.update({"unfused_layers_per_s": round(1e3 / tu, 1), "alg_bytes_unfused": int(sum(u2.values())),
+                            "byte_reduction": round(1 - sum(r2.values()) / sum(u2.values()), 4),
+                            "speedup_vs_unfused": round(tu / tr, 3)})
+            ent["hbm_GBps_recomposed"] = round(sum(r2.values()) / (tr * 1e-3) / 1e9, 1)
+            others[f"C{c2.idx}"] = ent
+            del L2
+            torch.cuda.empty_cache()
+
+    if rank != 0:
+        return None
+    dom = max(kern, key=lambda n: kern[n]["us"])
+    ncu = load_ncu_traffic().get(f"C{cfg.idx}", {})
+    achieved = rec_b[dom] / (kern[dom]["us"] * 1e-6) / 1e9
+    value = world * 1e3 / ms_step
+    res = {
+        "metric": METRIC,
+        "value": round(value, 2),
+        "unit": "layers/s",
+        "n_gpus": world, "steps": K, "warmup": Wm,
+        "ms_per_step": round(ms_step, 5),
+        "higher_is_better": True,
+        "scaling": "weak",
+        "vs_baseline": None,
+        "dtype": cfg.dtype,
+        "data": "synthetic (seeded N(0,1) q/k/v rounded to dtype; no datasets or weights needed)",
+        "config": {"workload": describe(cfg), "B": cfg.B, "H": cfg.H, "S": cfg.S, "D": cfg.D, "T": L.T,
+                   "tiles": L.n_tiles, "stored_score_elems": L.stored,
+                   "l2": "flushed (256 MiB write) before every timed step" if flush is not None else "not flushed",
+                   "parallelism": f"dp{world} (weak: each rank runs its own full layer on its own inputs)"},
+        "hbm_bytes_per_layer": {"recomposed_alg": int(sum(rec_b.values())), "unfused_alg": int(sum(unf_b.values())),
+                                "reduction_alg": round(1 - sum(rec_b.values()) / sum(unf_b.values()), 4),
+                                "recomposed_ncu": ncu.get("recomposed_dram_bytes"),
+                                "unfused_ncu": ncu.get("unfused_dram_bytes")},
+        "unfused": None if ms_unf is None else {"value": round(world * 1e3 / ms_unf, 2), "ms_per_step": round(ms_unf, 5),
+                                                "speedup_recomposed_vs_unfused": round(ms_unf / ms_step, 3),
+                                                "kernels": kern_unf},
+        "kernels": kern,
+        "roofline": {"kernel": dom, "bound": "hbm", "achieved": round(achieved, 1), "peak": hbm_peak, "unit": "GB/s",
+                     "frac": round(achieved / hbm_peak, 4), "traffic": ncu.get(f"{dom}_dram_bytes"),
+                     "peak_source": peak_src,
+                     "tensor_frac": round(flops(cfg, L.stored) / (ms_step * 1e-3) / 1e12 / peaks.get("bf16_tflops", 1590.0), 4)},
+        "e2e": {"value": round(world * 1e3 / ms_e2e, 2), "unit": "layers/s", "h2d_bytes_per_step": int(h2d),
+                "d2h_bytes_per_step": int(d2h), "ms_per_step": round(ms_e2e, 5)},
+        "gpu_launches": int(launches),
+        "clocks": clocks,
+    }
+    if others:
+        res["all_configs"] = others
+    return res
+
+
+# ----------------------------------------------------------------------------- CPU (oracle) arm
+
+def oracle_sample(cfg, target_s, seed=0):
+    """Time the fp64 oracle on a bounded random sample of rows; returns (layers/s, rows, secs, threads)."""
+    import oracle
+    t = W.config_tensors(cfg)
+    m = oracle_mask_for(cfg)
+    rng = np.random.Generator(np.random.PCG64(seed))
+    total = cfg.BH * cfg.S
+    probe = rng.integers(0, total, size=min(64, total))
+    t0 = time.perf_counter()
+    _, nt = oracle.attention_rows(t.q64, t.k64, t.v64, cfg.scale, probe, m, return_threads=True)
+    dt = max(time.perf_counter() - t0, 1e-4)
+    n = int(min(total, max(64, len(probe) * target_s / dt)))
+    return t, m, n, nt
+
+
+def oracle_mask_for(cfg):
+    import oracle
+    if cfg.kind == "dense":
+        return oracle.Mask(kv_len=cfg.kv_len, causal=cfg.causal)
+    if cfg.kind == "blocksparse":
+        return oracle.Mask(kind="block", layout=W.config_layout(cfg))
+    return oracle.Mask(kind="window", window=cfg.window, n_global=cfg.n_global)
+
+
+def cpu_baseline(cfg, target_s=10.0):
+    import oracle
+    t, m, n, nt = oracle_sample(cfg, target_s)
+    rng = np.random.Generator(np.random.PCG64(1))
+    done, reps = 0, 0
+    t0 = time.perf_counter()
+    while True:  # repeat the bounded sample until ~target_s of CPU work has been timed
+        rows = rng.integers(0, cfg.BH * cfg.S, size=n)
+        oracle.attention_rows(t.q64, t.k64, t.v64, cfg.scale, rows, m)
+        done += n
+        reps += 1
+        dt = time.perf_counter() - t0
+        if dt >= 0.5 * target_s:
+            break
+    frac = done / (cfg.BH * cfg.S)
+    return {"value": round(frac / dt, 6), "unit": "layers/s", "cores": nt, "kind": "oracle",
+            "sample": f"{reps} x {n} uniformly drawn query rows of {cfg.BH * cfg.S} ({frac:.4f} layers in total), "
+                      f"{dt:.2f} s, fp64 textbook attention, pthreads over rows"}
+
+
+def reference_arm(args, rank, world):
+    cfg = W.config(args.config)
+    if rank != 0:
+        return None
+    import oracle
+    t, m, n, nt = oracle_sample(cfg, target_s=1.5)
+    rng = np.random.Generator(np.random.PCG64(2))
+    times = []
+    for s in range(args.warmup + args.steps):
+        rows = rng.integers(0, cfg.BH * cfg.S, size=n)
+        t0 = time.perf_counter()
+        oracle.attention_rows(t.q64, t.k64, t.v64, cfg.scale, rows, m)
+        if s >= args.warmup:
+            times.append(time.perf_counter() - t0)
+    frac = n / (cfg.BH * cfg.S)
+    sec = statistics.mean(times)
+    v = frac / sec
+    return {"metric": METRIC, "value": round(v, 6), "unit": "layers/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": round(sec * 1e3, 3), "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic", "impl": "reference",
+            "config": {"workload": describe(cfg), "B": cfg.B, "H": cfg.H, "S": cfg.S, "D": cfg.D},
+            "cpu_baseline": {"value": round(v, 6), "unit": "layers/s", "cores": nt, "kind": "oracle",
+                             "sample": f"{n} random query rows per step ({frac:.4%} of one layer)"},
+            "e2e": {"value": round(v, 6), "unit": "layers/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--config", type=int, default=2, help="BASELINE.json config index (1-5); default configs[1]")
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--no-flush", action="store_true")
+    ap.add_argument("--no-all-configs", dest="all_configs", action="store_false")
+    ap.add_argument("--cpu-seconds", type=float, default=10.0)
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        res = reference_arm(args, rank, world)
+        if res is not None:
+            print(json.dumps(res), flush=True)
+        return
+    import torch
+    if world > 1:
+        torch.cuda.set_device(local_rank)
+        torch.distributed.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+    res = gpu_arm(args, rank, world, local_rank)
+    if res is not None:
+        if world == 1:
+            res["cpu_baseline"] = cpu_baseline(W.config(args.config), args.cpu_seconds)
+        print(json.dumps(res), flush=True)
+    if world > 1:
+        torch.distributed.barrier()
+        torch.distributed.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -96,8 +96,16 @@ typedef struct {
     void* stream;            /* cudaStream_t; NULL = legacy default stream */
     int32_t tile_n;          /* T = LS sub-vector width = GEMM1 output-tile width:
                                 0 = default (128 dense 16-bit, 64 fp32 and sparse), or 64 / 128 */
-    int32_t flags;           /* reserved, must be 0 */
+    int32_t flags;           /* 0 = run the whole chain.  Otherwise an OR of SR_RUN_* stage bits:
+                                only those kernels are launched, consuming the intermediates an
+                                earlier call with the same arguments left in the workspace (used by
+                                bench.py to time each kernel with events on the stream). */
 } sr_exec;
+
+/* Stage bits for sr_exec.flags. */
+#define SR_RUN_GEMM1 1   /* GEMM1 + LS (recomposed) / GEMM1 writing scores (unfused) */
+#define SR_RUN_REDUCE 2  /* IR (recomposed) / row softmax (unfused) */
+#define SR_RUN_GEMM2 4   /* GS + GEMM2 (recomposed) / GEMM2 on P (unfused) */
 
 /* Entry points (north star).  Returns SR_OK after enqueueing the kernels on ex->stream. */
 sr_status sr_mha_dense(const void* q, const void* k, const void* v, void* out, int B, int H, int S,

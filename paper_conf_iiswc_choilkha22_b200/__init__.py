@@ -197,8 +197,11 @@ _FN = {(SR_E_DENSE, True): "sr_mha_dense", (SR_E_BLOCKSPARSE, True): "sr_mha_blo
        (SR_E_WINDOW, False): "sr_mha_sliding_window_unfused"}
 
 
+SR_RUN_GEMM1, SR_RUN_REDUCE, SR_RUN_GEMM2 = 1, 2, 4
+
+
 def call(mask: _Mask, q, k, v, *, scale=None, causal=False, out_dtype=None, tile_n=0, fused=True,
-         out=None, workspace=None, stream=None):
+         out=None, workspace=None, stream=None, stages=0):
     """Run one attention layer through the C ABI.  q, k, v: CUDA tensors [B, H, S, D]."""
     torch = _torch()
     if not (q.is_cuda and k.is_cuda and v.is_cuda):
@@ -221,7 +224,8 @@ def call(mask: _Mask, q, k, v, *, scale=None, causal=False, out_dtype=None, tile
                                                int(tile_n), C.byref(WsInfo())), last_error())
     ws = workspace if workspace is not None else _workspace(q.device, need)
     st = torch.cuda.current_stream(q.device).cuda_stream if stream is None else stream
-    ex = Exec(in_dt, dtype_code(out_dtype), ws.data_ptr(), ws.numel() * ws.element_size(), st, int(tile_n), 0)
+    ex = Exec(in_dt, dtype_code(out_dtype), ws.data_ptr(), ws.numel() * ws.element_size(), st, int(tile_n),
+              int(stages))
     fn = getattr(lib(), _FN[(mask.entry, bool(fused))])
     _check(fn(q.data_ptr(), k.data_ptr(), v.data_ptr(), out.data_ptr(), B, H, S, D, C.c_float(scale), mask.ptr,
               int(causal), C.byref(ex)))

@@ -350,7 +350,8 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
     if (!ex) return fail(SR_ERR_INVALID, "exec descriptor is NULL");
     if (!q || !k || !v || !out) return fail(SR_ERR_INVALID, "q, k, v and out must be non-NULL");
     if (!std::isfinite(scale) || !(scale > 0.f)) return fail(SR_ERR_INVALID, "scale must be finite and > 0");
-    if (ex->flags != 0) return fail(SR_ERR_INVALID, "flags must be 0");
+    if (ex->flags & ~(SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2))
+        return fail(SR_ERR_INVALID, "unknown flags 0x%x", ex->flags);
     Request r;
     sr_status s = check_request(e, B, H, S, D, ex->in_dtype, mask_or_layout, causal, ex->tile_n, r);
     if (s != SR_OK) return s;
@@ -386,6 +387,7 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
     p.in_dtype = ex->in_dtype;
     p.out_dtype = ex->out_dtype;
     p.sc = cs->dev;
+    p.stages = ex->flags ? ex->flags : (SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2);
     char* ws = (char*)ex->workspace;
     p.xprime = ws + wi.off_xprime;
     if (fused) {

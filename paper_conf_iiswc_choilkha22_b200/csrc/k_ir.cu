@@ -24,27 +24,47 @@ __global__ void __launch_bounds__(256) ir_kernel(Params p)
     const int t0 = tp[rb], t1 = tp[rb + 1], base = tp[0];
     const int64_t slot0 = (int64_t)g * sc.slots_per_head - base;
 
-    float m = -INFINITY;
-    for (int t = t0; t < t1; ++t) {
-        if (!((tinfo_half(__ldg(sc.tinfo + t)) >> half) & 1)) continue;
-        m = fmaxf(m, __ldg(p.mprime + (slot0 + t) * kRowBlock + lane));
-    }
-    float d = 0.f;
-    if (m != -INFINITY) {
-        for (int t = t0; t < t1; ++t) {
-            if (!((tinfo_half(__ldg(sc.tinfo + t)) >> half) & 1)) continue;
-            const float mk = __ldg(p.mprime + (slot0 + t) * kRowBlock + lane);
-            if (mk != -INFINITY) d += expf(mk - m) * __ldg(p.dprime + (slot0 + t) * kRowBlock + lane);
+    // m and d in one pass: batches of 8 independent (m'_k, d'_k) loads, merged with the running
+    // (m, d) -- d is rescaled by e^{m_old - m_new} whenever the running max grows.  Same reduction
+    // as PAPER.md L147 (m = max m'_k, d = sum e^{m'_k - m} d'_k), regrouped for memory-level
+    // parallelism.
+    const float* mp = p.mprime + slot0 * kRowBlock + lane;
+    const float* dp = p.dprime + slot0 * kRowBlock + lane;
+    float m = -INFINITY, d = 0.f;
+    for (int tb = t0; tb < t1; tb += 8) {
+        float mk[8], dk[8];
+#pragma unroll
+        for (int u = 0; u < 8; ++u) {
+            const int t = tb + u;
+            const bool ok = t < t1 && ((tinfo_half(__ldg(sc.tinfo + t)) >> half) & 1);
+            mk[u] = ok ? __ldg(mp + (int64_t)t * kRowBlock) : -INFINITY;
+            dk[u] = ok ? __ldg(dp + (int64_t)t * kRowBlock) : 0.f;
         }
+        float mb = mk[0];
+#pragma unroll
+        for (int u = 1; u < 8; ++u) mb = fmaxf(mb, mk[u]);
+        if (mb == -INFINITY) continue;
+        const float mn = fmaxf(m, mb);
+        float acc = (m == -INFINITY) ? 0.f : d * __expf(m - mn);
+#pragma unroll
+        for (int u = 0; u < 8; ++u)
+            if (mk[u] != -INFINITY) acc += dk[u] * __expf(mk[u] - mn);
+        m = mn;
+        d = acc;
     }
     const float inv_d = d > 0.f ? 1.f / d : 0.f;
-    for (int t = t0; t < t1; ++t) {
-        float r = 0.f;
-        if ((tinfo_half(__ldg(sc.tinfo + t)) >> half) & 1) {
-            const float mk = __ldg(p.mprime + (slot0 + t) * kRowBlock + lane);
-            if (mk != -INFINITY) r = expf(mk - m) * inv_d;
+    float* rp = p.rprime + slot0 * kRowBlock + lane;
+    for (int tb = t0; tb < t1; tb += 8) {
+        float mk[8];
+#pragma unroll
+        for (int u = 0; u < 8; ++u) {
+            const int t = tb + u;
+            const bool ok = t < t1 && ((tinfo_half(__ldg(sc.tinfo + t)) >> half) & 1);
+            mk[u] = ok ? __ldg(mp + (int64_t)t * kRowBlock) : -INFINITY;
         }
-        p.rprime[(slot0 + t) * kRowBlock + lane] = r;
+#pragma unroll
+        for (int u = 0; u < 8; ++u)
+            if (tb + u < t1) rp[(int64_t)(tb + u) * kRowBlock] = (mk[u] == -INFINITY) ? 0.f : __expf(mk[u] - m) * inv_d;
     }
 }
 

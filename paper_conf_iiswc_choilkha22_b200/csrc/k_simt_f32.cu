@@ -112,13 +112,18 @@ static cudaError_t launch_d(const Params& p, cudaStream_t st, int64_t* nl)
     if (e != cudaSuccess) return e;
     e = cudaFuncSetAttribute(simt_gs_gemm2_f32<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm2);
     if (e != cudaSuccess) return e;
-    simt_gemm1_ls_f32<D><<<n, 128, sm1, st>>>(p);
-    ++*nl;
-    if ((e = cudaGetLastError()) != cudaSuccess) return e;
-    if ((e = launch_ir(p, st, nl)) != cudaSuccess) return e;
-    simt_gs_gemm2_f32<D><<<n, 128, sm2, st>>>(p);
-    ++*nl;
-    return cudaGetLastError();
+    if (p.stages & 1) {
+        simt_gemm1_ls_f32<D><<<n, 128, sm1, st>>>(p);
+        ++*nl;
+        if ((e = cudaGetLastError()) != cudaSuccess) return e;
+    }
+    if ((p.stages & 2) && (e = launch_ir(p, st, nl)) != cudaSuccess) return e;
+    if (p.stages & 4) {
+        simt_gs_gemm2_f32<D><<<n, 128, sm2, st>>>(p);
+        ++*nl;
+        e = cudaGetLastError();
+    }
+    return e;
 }
 
 cudaError_t launch_simt_f32(const Params& p, cudaStream_t st, int64_t* nl)

@@ -71,7 +71,8 @@ struct G1 {
     static constexpr int OFF_X = OFF_K + NK * KB;
     static constexpr int OFF_BAR = OFF_X + 2 * XB;
     static constexpr int NBAR = 2 * NQ + 2 * NK + 2 * NACC;
-    static constexpr int SMEM = OFF_BAR + NBAR * 8 + 16 + 1024;  // + tmem ptr + alignment slack
+    static constexpr int SMEM_ = OFF_BAR + NBAR * 8 + 16 + 1024;  // + tmem ptr + alignment slack
+    static constexpr int SMEM = SMEM_ > 118 * 1024 ? SMEM_ : 118 * 1024;  // 1 CTA/SM (512 TMEM cols)
     static constexpr int THREADS = 384;
 };
 
@@ -105,7 +106,10 @@ __global__ void __launch_bounds__(384, 1)
     tc_fence_after();
     const uint32_t tmem_base = *tmem_ptr;
     const int n_items = p.sc.n_items;
-
+    // 168 regs/thread at launch; warpgroup 0 (producer, MMA, allocator) hands registers to the
+    // two epilogue warpgroups, which hold a whole 128 x T fp32 row block each
+    if (warp < 4) {
+    reg_dealloc<56>();
     if (warp == 0) {
         // ------------------------------------------------------------------ TMA producer
         if (lane == 0) {
@@ -167,7 +171,9 @@ __global__ void __launch_bounds__(384, 1)
                 if (++qi == C::NQ) { qi = 0; qph ^= 1; }
             }
         }
-    } else if (warp >= 4) {
+    }
+    } else {
+        reg_alloc<224>();
         // ------------------------------------------------------------------ epilogue warpgroups
         const int e = (warp - 4) / 4;                 // warpgroup 0 / 1: even / odd tiles
         const int r = (warp % 4) * 32 + lane;         // tile row == TMEM lane
@@ -195,62 +201,59 @@ __global__ void __launch_bounds__(384, 1)
                 const uint32_t taddr = tmem_base + lane_off + buf * T;
                 mbar_wait(&acc_full[buf], ph);
                 tc_fence_after();
-                float mx = -INFINITY;
-                if (LS && valid) {  // pass 1: row max of the masked tile
-#pragma unroll 1
-                    for (int c = 0; c < T / 32; ++c) {
-                        uint32_t v[32];
-                        tmem_ld32(taddr + c * 32, v);
-                        tmem_wait_ld();
+                // one TMEM read of the whole 128 x T fp32 row block; the accumulator buffer is
+                // released to the MMA warp before any math
+                uint32_t xr[T];
+                if (valid) {
 #pragma unroll
-                        for (int u = 0; u < 32; ++u) {
-                            float x = __uint_as_float(v[u]);
-                            if (!full && !elem_kept(p, kvl, i, c0 + c * 32 + u)) x = -INFINITY;
-                            mx = fmaxf(mx, x);
-                        }
-                    }
-                }
-                // staging buffer of this warpgroup must be free (previous bulk store read it)
-                if (issuer) bulk_wait_read0();
-                named_bar_sync(1 + e, 128);
-                float dsum = 0.f;
-                if (valid) {  // pass 2
-                    const float neg = (mx == -INFINITY) ? 0.f : -mx * sl2;
-#pragma unroll 1
-                    for (int c = 0; c < T / 32; ++c) {
-                        uint32_t v[32];
-                        tmem_ld32(taddr + c * 32, v);
-                        tmem_wait_ld();
-                        uint32_t pk[16];
-#pragma unroll
-                        for (int u = 0; u < 32; u += 2) {
-                            float x0 = __uint_as_float(v[u]), x1 = __uint_as_float(v[u + 1]);
-                            if (!full) {
-                                if (!elem_kept(p, kvl, i, c0 + c * 32 + u)) x0 = -INFINITY;
-                                if (!elem_kept(p, kvl, i, c0 + c * 32 + u + 1)) x1 = -INFINITY;
-                            }
-                            float y0, y1;
-                            if (LS) {  // X' = e^{x - m'} in base 2 with log2(e) folded into the scale
-                                y0 = ex2(fmaf(x0, sl2, neg));
-                                y1 = ex2(fmaf(x1, sl2, neg));
-                                dsum += y0 + y1;
-                            } else {  // unfused: the scaled, masked score
-                                y0 = x0 * p.scale;
-                                y1 = x1 * p.scale;
-                            }
-                            pk[u / 2] = pack_f16(y0, y1);
-                        }
-#pragma unroll
-                        for (int q4 = 0; q4 < 4; ++q4) {
-                            const uint32_t off = tile_chunk_off(r, c * 4 + q4);
-                            *reinterpret_cast<uint4*>(stage + off) =
-                                make_uint4(pk[q4 * 4], pk[q4 * 4 + 1], pk[q4 * 4 + 2], pk[q4 * 4 + 3]);
-                        }
-                    }
+                    for (int c = 0; c < T / 32; ++c) tmem_ld32(taddr + c * 32, *reinterpret_cast<uint32_t(*)[32]>(&xr[c * 32]));
+                    tmem_wait_ld();
                 }
                 tc_fence_before();
                 __syncwarp();
                 if (lane == 0) mbar_arrive(&acc_empty[buf]);
+                // the warpgroup's staging buffer must be free: its previous bulk store has read it
+                if (issuer) bulk_wait_read0();
+                named_bar_sync(1 + e, 128);
+                float mx = -INFINITY, dsum = 0.f;
+                if (valid) {
+                    if (!full) {  // edge tile: element mask (padding / causal diagonal / band edge)
+#pragma unroll
+                        for (int u = 0; u < T; ++u)
+                            if (!elem_kept(p, kvl, i, c0 + u)) xr[u] = 0xff800000u;  // -inf
+                    }
+                    float neg = 0.f;
+                    if (LS) {
+                        float m8[8];
+#pragma unroll
+                        for (int a = 0; a < 8; ++a) m8[a] = __uint_as_float(xr[a]);
+#pragma unroll
+                        for (int u = 8; u < T; ++u) m8[u & 7] = fmaxf(m8[u & 7], __uint_as_float(xr[u]));
+                        mx = fmaxf(fmaxf(fmaxf(m8[0], m8[1]), fmaxf(m8[2], m8[3])),
+                                   fmaxf(fmaxf(m8[4], m8[5]), fmaxf(m8[6], m8[7])));
+                        // X' = e^{x - m'} in base 2, log2(e) folded into the scale
+                        neg = (mx == -INFINITY) ? 0.f : -mx * sl2;
+                    }
+                    float s4[4] = {0.f, 0.f, 0.f, 0.f};
+#pragma unroll
+                    for (int q4 = 0; q4 < T / 8; ++q4) {  // 8 scores -> one 16-B chunk of the tile
+                        uint32_t w4[4];
+#pragma unroll
+                        for (int u = 0; u < 4; ++u) {
+                            const float x0 = __uint_as_float(xr[q4 * 8 + 2 * u]);
+                            const float x1 = __uint_as_float(xr[q4 * 8 + 2 * u + 1]);
+                            if (LS) {
+                                const float y0 = ex2(fmaf(x0, sl2, neg)), y1 = ex2(fmaf(x1, sl2, neg));
+                                s4[u] += y0 + y1;
+                                w4[u] = pack_f16(y0, y1);
+                            } else {  // unfused baseline: the scaled, masked score
+                                w4[u] = pack_f16(x0 * p.scale, x1 * p.scale);
+                            }
+                        }
+                        *reinterpret_cast<uint4*>(stage + tile_chunk_off(r, q4)) = make_uint4(w4[0], w4[1], w4[2], w4[3]);
+                    }
+                    dsum = (s4[0] + s4[1]) + (s4[2] + s4[3]);
+                }
                 fence_proxy_async_smem();
                 named_bar_sync(1 + e, 128);
                 const int64_t slot = I.slot0 + t;
@@ -288,7 +291,8 @@ template <int D, int T>
 struct G2 {
     static constexpr int XB = kRowBlock * T * 2;  // X' / P tile
     static constexpr int VB = T * D * 2;          // V tile
-    static constexpr int SB = XB + VB;
+    static constexpr int RB = 1024;               // r' of the tile (128 floats), padded to 1 KB
+    static constexpr int SB = XB + VB + RB;
     static constexpr int NS_ = (kSmemMax - 2048) / SB;
     static constexpr int NS = NS_ > 4 ? 4 : NS_;
     static_assert(NS >= 2, "smem budget");
@@ -299,7 +303,8 @@ struct G2 {
     static constexpr int OFF_S = 0;
     static constexpr int OFF_BAR = NS * SB;
     static constexpr int NBAR = 2 * NS + 2 * NA + 2 * NO;
-    static constexpr int SMEM = OFF_BAR + NBAR * 8 + 16 + 1024;
+    static constexpr int SMEM_ = OFF_BAR + NBAR * 8 + 16 + 1024;
+    static constexpr int SMEM = SMEM_ > 118 * 1024 ? SMEM_ : 118 * 1024;  // 1 CTA/SM (512 TMEM cols)
     static constexpr int THREADS = 384;
 };
 
@@ -349,7 +354,7 @@ __global__ void __launch_bounds__(384, 1)
                     const int kt = tinfo_kt(w), hv = tinfo_half(w);
                     const uint32_t xbytes = (hv == 3 ? 2 : 1) * (T / 64) * (kHalf * 128);
                     mbar_wait(&s_empty[s], sph ^ 1);
-                    mbar_arrive_expect_tx(&s_full[s], xbytes + C::VB);
+                    mbar_arrive_expect_tx(&s_full[s], xbytes + C::VB + (GS ? kRowBlock * 4 : 0));
                     uint8_t* st = smem + C::OFF_S + s * C::SB;
                     const uint8_t* xs = (const uint8_t*)src + (I.slot0 + t) * (int64_t)C::XB;
                     if (hv == 3) bulk_load(st, xs, C::XB, &s_full[s]);
@@ -360,6 +365,8 @@ __global__ void __launch_bounds__(384, 1)
                         }
                     for (int h = 0; h < D / 64; ++h)
                         tma_load_2d(st + C::XB + h * (T * 128), &tmV, h * 64, I.g * p.S + kt * T, &s_full[s]);
+                    if (GS)  // r' of the tile's 128 rows rides along with the tile (GS operand)
+                        bulk_load(st + C::XB + C::VB, p.rprime + (I.slot0 + t) * kRowBlock, kRowBlock * 4, &s_full[s]);
                     if (++s == C::NS) { s = 0; sph ^= 1; }
                 }
             }
@@ -412,9 +419,9 @@ __global__ void __launch_bounds__(384, 1)
             for (int t = I.t0; t < I.t1; ++t) {
                 const int hv = tinfo_half(__ldg(p.sc.tinfo + t));
                 const bool valid = (hv >> myhalf) & 1;
-                float rr = 1.f;
-                if (GS) rr = valid ? __ldg(p.rprime + (I.slot0 + t) * kRowBlock + r) : 0.f;
                 mbar_wait(&s_full[s], sph);
+                float rr = 1.f;
+                if (GS) rr = valid ? reinterpret_cast<const float*>(smem + C::OFF_S + s * C::SB + C::XB + C::VB)[r] : 0.f;
                 mbar_wait(&a_empty[a], aph ^ 1);
                 tc_fence_after();
                 const uint8_t* xs = smem + C::OFF_S + s * C::SB;
@@ -664,19 +671,21 @@ cudaError_t launch_softmax(const Params& p, cudaStream_t st, int64_t* nl)
 template <int D, int T>
 cudaError_t fused_dt(const Params& p, cudaStream_t st, int64_t* nl)
 {
-    cudaError_t e;
-    if ((e = launch_g1<D, T, true>(p, st, nl)) != cudaSuccess) return e;
-    if ((e = launch_ir(p, st, nl)) != cudaSuccess) return e;
-    return launch_g2<D, T, true>(p, st, nl);
+    cudaError_t e = cudaSuccess;
+    if ((p.stages & 1) && (e = launch_g1<D, T, true>(p, st, nl)) != cudaSuccess) return e;
+    if ((p.stages & 2) && (e = launch_ir(p, st, nl)) != cudaSuccess) return e;
+    if (p.stages & 4) e = launch_g2<D, T, true>(p, st, nl);
+    return e;
 }
 
 template <int D, int T>
 cudaError_t unfused_dt(const Params& p, cudaStream_t st, int64_t* nl)
 {
-    cudaError_t e;
-    if ((e = launch_g1<D, T, false>(p, st, nl)) != cudaSuccess) return e;
-    if ((e = launch_softmax<T>(p, st, nl)) != cudaSuccess) return e;
-    return launch_g2<D, T, false>(p, st, nl);
+    cudaError_t e = cudaSuccess;
+    if ((p.stages & 1) && (e = launch_g1<D, T, false>(p, st, nl)) != cudaSuccess) return e;
+    if ((p.stages & 2) && (e = launch_softmax<T>(p, st, nl)) != cudaSuccess) return e;
+    if (p.stages & 4) e = launch_g2<D, T, false>(p, st, nl);
+    return e;
 }
 
 }  // namespace

@@ -55,6 +55,19 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity)
     }
 }
 
+// ------------------------------------------------------------------ register rebalancing
+// (all 4 warps of a warpgroup must execute these; counts are multiples of 8 in [24, 256])
+template <int N>
+__device__ __forceinline__ void reg_dealloc()
+{
+    asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(N));
+}
+template <int N>
+__device__ __forceinline__ void reg_alloc()
+{
+    asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(N));
+}
+
 // ------------------------------------------------------------------ named barriers / fences
 __device__ __forceinline__ void named_bar_sync(int id, int nthreads)
 {

@@ -51,6 +51,7 @@ struct Params {
     int win_half;      // window / 2
     int n_global;
     int in_dtype, out_dtype;
+    int stages;        // SR_RUN_* bits to launch
     DevSched sc;
     void* xprime;      // X' tiles (recomposed) or score tiles S (unfused)
     void* pbuf;        // unfused: P tiles

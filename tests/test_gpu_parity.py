@@ -287,7 +287,11 @@ def test_full_config_rows_sum_to_one(idx):
     t.v_s = np.ones_like(t.v_s) if cfg.dtype != "bf16" else np.full_like(t.v_s, 0x3F80)
     o, _ = _config_call(cfg, t, out_f32=True)
     err = (o - 1).abs().max().item()
-    assert err < 2e-3, err
+    # Bound from the arithmetic: sum_j Y_j with Y = round_dtype(round_f16(X') * r'): each Y_j carries
+    # relative error <= 2^-11 (fp16 X') + half an ulp of the MMA operand dtype (2^-11 f16, 2^-9 bf16);
+    # a dominant element can carry it whole.  Plus fp32 accumulation noise.
+    bound = 2.0 ** -11 + (2.0 ** -9 if cfg.dtype == "bf16" else 2.0 ** -11) + 1e-4
+    assert err <= bound, (err, bound)
 
 
 def test_abi_errors_on_gpu():

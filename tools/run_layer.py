@@ -1,0 +1,20 @@
+"""Run one config's layer a few times (for ncu captures): python tools/run_layer.py CFG [unfused] [reps]"""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch  # noqa: E402
+
+import paper_conf_iiswc_choilkha22_b200 as sr  # noqa: E402
+import workloads as W  # noqa: E402
+from bench import Layer  # noqa: E402
+
+idx = int(sys.argv[1])
+fused = not (len(sys.argv) > 2 and sys.argv[2] == "unfused")
+reps = int(sys.argv[3]) if len(sys.argv) > 3 else 2
+cfg = W.config(idx)
+L = Layer(cfg, torch.device("cuda", 0), cfg.idx, sr, torch)
+for _ in range(reps):
+    L.run(fused=fused)
+torch.cuda.synchronize()
+print("ok", cfg.name, "fused" if fused else "unfused")
