@@ -151,7 +151,8 @@ def timed(torch, fn, steps, warmup, flush, per_step_pre=None):
     ev = []
     for s in range(warmup + steps):
         if flush is not None:
-            flush.zero_()
+            flush[0].zero_()  # write 256 MiB (evicts everything) ...
+            flush[1].sum()  # ... then read another 256 MiB so L2 starts the step clean, not dirty
         if per_step_pre:
             per_step_pre()
         a = torch.cuda.Event(enable_timing=True)
@@ -200,7 +201,8 @@ def gpu_arm(args, rank, world, local_rank):
     hbm_peak = peaks.get("hbm_gbs", 6650.0)
     peak_src = "MEASURED_PEAKS.json hbm_gbs (measured)" if "hbm_gbs" in peaks else "fallback 6650 GB/s (B200_PROFILING.md)"
     cfg = W.config(args.config)
-    flush = None if args.no_flush else torch.empty(FLUSH_BYTES, dtype=torch.uint8, device=device)
+    flush = None if args.no_flush else (torch.empty(FLUSH_BYTES, dtype=torch.uint8, device=device),
+                                        torch.ones(FLUSH_BYTES // 4, dtype=torch.float32, device=device))
     L = Layer(cfg, device, seed_base=cfg.idx + 1000 * rank, sr=sr, torch=torch)
     K, Wm = args.steps, args.warmup
 
@@ -300,7 +302,7 @@ def gpu_arm(args, rank, world, local_rank):
         "data": "synthetic (seeded N(0,1) q/k/v rounded to dtype; no datasets or weights needed)",
         "config": {"workload": describe(cfg), "B": cfg.B, "H": cfg.H, "S": cfg.S, "D": cfg.D, "T": L.T,
                    "tiles": L.n_tiles, "stored_score_elems": L.stored,
-                   "l2": "flushed (256 MiB write) before every timed step" if flush is not None else "not flushed",
+                   "l2": "flushed before every timed step (256 MiB write, then 256 MiB read of another buffer)" if flush is not None else "not flushed",
                    "parallelism": f"dp{world} (weak: each rank runs its own full layer on its own inputs)"},
         "hbm_bytes_per_layer": {"recomposed_alg": int(sum(rec_b.values())), "unfused_alg": int(sum(unf_b.values())),
                                 "reduction_alg": round(1 - sum(rec_b.values()) / sum(unf_b.values()), 4),

@@ -1,0 +1,331 @@
+// k_gemm2.cu -- GEMM2 = Y V with the Global Scaling (GS) sub-layer fused into its prologue
+// ("if element-wise scaling can be performed prior to the MatMul operation by
+// providing r' corresponding to X' allocated to the TB of the MatMul kernel following the GS kernel,
+// the GS kernel can easily be fused with its subsequent MatMul kernel").  GS=false builds the
+// unfused baseline's GEMM2 on the softmax output P.
+//
+// Per item (head, 128-row block) and each of its key tiles:
+//   Y_tile = X'_tile (fp16) * r'_row (fp32), rounded once to the MMA dtype   (GS, in registers)
+//   O     += Y_tile V_tile   (tcgen05.mma kind::f16, A from TMEM, B = V from smem, fp32 in TMEM)
+//
+// Warp roles (persistent CTA per SM, 384 threads):
+//   warp 0      producer: per tile one smem stage = X' tile (1-D bulk copy of its valid halves) +
+//               V tile (TMA, 128B swizzle) + r' of the 128 rows (bulk copy) + a stage header
+//               (half-valid bits, item boundaries); EMPTY items and the END of the schedule travel
+//               through the same ring as header-only stages
+//   warp 1      MMA issuer: T/16 MMAs of 128 x D x 16 per tile into one of two O accumulators;
+//               publishes the item's output row to the epilogue through an O header
+//   warp 2      TMEM allocator (512 columns: 2 x D for O, NA x T/2 for the A operand ring)
+//   warps 4-7   GS transform: smem X' row -> fp32 x r' -> dtype -> tcgen05.st into TMEM (A operand)
+//   warps 8-11  epilogue: tcgen05.ld of O rows -> out dtype -> global
+#include "tc_common.cuh"
+
+namespace sr {
+
+using namespace ptx;
+
+enum : int { SH_TILE = 1, SH_END = 2, SH_EMPTY = 4, SH_FIRST = 8, SH_LAST = 16 };
+struct G2Hdr {  // stage / O-buffer header
+    int32_t flags, hv, orow_lo, orow_hi;
+};
+
+template <int D, int T>
+struct G2 {
+    static constexpr int XB = kRowBlock * T * 2;  // X' / P tile
+    static constexpr int VB = T * D * 2;          // V tile
+    static constexpr int RB = 1024;               // r' (512 B) + stage header, padded to keep 1 KB alignment
+    static constexpr int SB = XB + VB + RB;
+    static constexpr int NS_ = (kSmemMax - 2048) / SB;
+    static constexpr int NS = NS_ > 6 ? 6 : NS_;
+    static_assert(NS >= 2, "smem budget");
+    static constexpr int NO = 2;                          // O accumulators (D cols each)
+    static constexpr int NA_ = (512 - NO * D) / (T / 2);  // A operand buffers (T/2 cols each)
+    static constexpr int NA = NA_ > 8 ? 8 : NA_;
+    static_assert(NA >= 2, "tmem budget");
+    static constexpr int OFF_S = 0;
+    static constexpr int OFF_BAR = NS * SB;
+    static constexpr int NBAR = 2 * NS + 2 * NA + 2 * NO;
+    static constexpr int OFF_OHDR = OFF_BAR + NBAR * 8;
+    static constexpr int OFF_TPTR = OFF_OHDR + NO * (int)sizeof(G2Hdr);
+    static constexpr int SMEM_ = OFF_TPTR + 16 + 1024;
+    static constexpr int SMEM = SMEM_ > 118 * 1024 ? SMEM_ : 118 * 1024;  // 1 CTA/SM (512 TMEM cols)
+    static constexpr int THREADS = 384;
+};
+
+template <int D, int T, bool GS>
+__global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUtensorMap tmV, const Params p)
+{
+    using C = G2<D, T>;
+    extern __shared__ uint8_t smem_raw[];
+    uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+    uint64_t* bars = (uint64_t*)(smem + C::OFF_BAR);
+    uint64_t* s_full = bars;
+    uint64_t* s_empty = s_full + C::NS;
+    uint64_t* a_full = s_empty + C::NS;
+    uint64_t* a_empty = a_full + C::NA;
+    uint64_t* o_full = a_empty + C::NA;
+    uint64_t* o_empty = o_full + C::NO;
+    G2Hdr* ohdr = (G2Hdr*)(smem + C::OFF_OHDR);
+    uint32_t* tmem_ptr = (uint32_t*)(smem + C::OFF_TPTR);
+    auto stage = [&](int s) { return smem + C::OFF_S + s * C::SB; };
+    auto shdr = [&](int s) { return (G2Hdr*)(stage(s) + C::XB + C::VB + 512); };
+
+    const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+    if (threadIdx.x == 0) {
+        for (int i = 0; i < C::NS; ++i) { mbar_init(&s_full[i], 1); mbar_init(&s_empty[i], 1); }
+        for (int i = 0; i < C::NA; ++i) { mbar_init(&a_full[i], 4); mbar_init(&a_empty[i], 1); }
+        // o_full: O-header arrive + MMA commit; o_empty: one arrive per epilogue warp
+        for (int i = 0; i < C::NO; ++i) { mbar_init(&o_full[i], 2); mbar_init(&o_empty[i], 4); }
+        fence_mbar_init();
+    }
+    if (warp == 0 && lane == 0) prefetch_tmap(&tmV);
+    if (warp == 2) tmem_alloc(tmem_ptr, 512);
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem_base = *tmem_ptr;
+    const uint32_t tmem_o = tmem_base;              // NO x D columns
+    const uint32_t tmem_a = tmem_base + C::NO * D;  // NA x T/2 columns
+    const int n_items = p.sc.n_items;
+    const uint8_t* src = (const uint8_t*)(GS ? p.xprime : p.pbuf);
+
+    if (warp == 0) {
+        if (lane == 0) {
+            // -------------------------------------------------------------- producer
+            int s = 0;
+            uint32_t sph = 0;
+            auto next_stage = [&]() {
+                mbar_wait(&s_empty[s], sph ^ 1);
+                return s;
+            };
+            auto advance = [&]() {
+                if (++s == C::NS) { s = 0; sph ^= 1; }
+            };
+            for (int it = blockIdx.x; it < n_items; it += gridDim.x) {
+                const ItemInfo I = decode_item(p, it);
+                if (I.t0 == I.t1) continue;  // empty items never touch the stage ring
+                int w_next = __ldg(p.sc.tinfo + I.t0);
+                for (int t = I.t0; t < I.t1; ++t) {
+                    const int w = w_next;
+                    if (t + 1 < I.t1) w_next = __ldg(p.sc.tinfo + t + 1);
+                    const int kt = tinfo_kt(w), hv = tinfo_half(w);
+                    const uint32_t xbytes = (hv == 3 ? 2 : 1) * (T / 64) * (kHalf * 128);
+                    next_stage();
+                    uint8_t* st = stage(s);
+                    *shdr(s) = G2Hdr{SH_TILE, hv, 0, 0};
+                    mbar_arrive_expect_tx(&s_full[s], xbytes + C::VB + (GS ? kRowBlock * 4 : 0));
+                    const uint8_t* xs = src + (I.slot0 + t) * (int64_t)C::XB;
+                    if (hv == 3) bulk_load(st, xs, C::XB, &s_full[s]);
+                    else
+                        for (int ch = 0; ch < T / 64; ++ch) {
+                            const int o = ch * (kRowBlock * 128) + (hv == 2 ? kHalf * 128 : 0);
+                            bulk_load(st + o, xs + o, kHalf * 128, &s_full[s]);
+                        }
+                    for (int h = 0; h < D / 64; ++h)
+                        tma_load_2d(st + C::XB + h * (T * 128), &tmV, h * 64, I.g * p.S + kt * T, &s_full[s]);
+                    if (GS)  // r' of the tile's 128 rows rides along with the tile
+                        bulk_load(st + C::XB + C::VB, p.rprime + (I.slot0 + t) * kRowBlock, kRowBlock * 4, &s_full[s]);
+                    advance();
+                }
+            }
+            next_stage();
+            shdr(s)->flags = SH_END;
+            mbar_arrive(&s_full[s]);
+        }
+    } else if (warp == 1) {
+        if (lane == 0) {
+            // -------------------------------------------------------------- MMA issuer
+            const uint32_t idesc = idesc_f16(p.in_dtype == DT_BF16 ? 1 : 0, kRowBlock, D, 0, 1);
+            int s = 0, a = 0, o = 0;
+            uint32_t sph = 0, aph = 0, oph = 0;
+            auto post = [&](int flags, int64_t orow) {  // O header to the epilogue, arrival 1 of 2
+                mbar_wait(&o_empty[o], oph ^ 1);
+                ohdr[o] = G2Hdr{flags, 0, (int32_t)(orow & 0xffffffff), (int32_t)(orow >> 32)};
+                mbar_arrive(&o_full[o]);
+            };
+            auto next_o = [&]() {
+                if (++o == C::NO) { o = 0; oph ^= 1; }
+            };
+            ItemInfo nxt;
+            if (blockIdx.x < n_items) nxt = decode_item(p, blockIdx.x);
+            for (int it = blockIdx.x; it < n_items; it += gridDim.x) {
+                const ItemInfo I = nxt;
+                if (it + (int)gridDim.x < n_items) nxt = decode_item(p, it + gridDim.x);  // prefetch
+                const int64_t orow = (int64_t)I.g * p.S + I.rb * kRowBlock;
+                if (I.t0 == I.t1) {  // no kept key in these rows: the epilogue writes zeros
+                    post(SH_EMPTY, orow);
+                    mbar_arrive(&o_full[o]);
+                    next_o();
+                    continue;
+                }
+                post(SH_TILE, orow);
+                const uint32_t d_tmem = tmem_o + o * D;
+                for (int t = I.t0; t < I.t1; ++t) {
+                    mbar_wait(&s_full[s], sph);
+                    mbar_wait(&a_full[a], aph);
+                    tc_fence_after();
+                    const uint32_t v_addr = smem_u32(stage(s) + C::XB);
+                    const uint32_t a_tm = tmem_a + a * (T / 2);
+#pragma unroll
+                    for (int kk = 0; kk < T / 16; ++kk) {
+                        // B = V tile, MN-major SW128: 16 keys per MMA = 2 KB; 64-wide d blocks at LBO = T*128 B
+                        const uint64_t bd = smem_desc_sw128(v_addr + kk * 2048, T * 128, 1024);
+                        mma_ts(d_tmem, a_tm + kk * 8, bd, idesc, (t == I.t0 && kk == 0) ? 0u : 1u);
+                    }
+                    mma_commit(&s_empty[s]);
+                    mma_commit(&a_empty[a]);
+                    if (++s == C::NS) { s = 0; sph ^= 1; }
+                    if (++a == C::NA) { a = 0; aph ^= 1; }
+                }
+                mma_commit(&o_full[o]);  // arrival 2 of 2 when the item's MMAs complete
+                next_o();
+            }
+            post(SH_END, 0);
+            mbar_arrive(&o_full[o]);
+        }
+    } else if (warp >= 4 && warp < 8) {
+        // ------------------------------------------------------------------ GS transform
+        const int r = (warp % 4) * 32 + lane;
+        const int myhalf = r / kHalf;
+        const uint32_t lane_off = (uint32_t)((warp % 4) * 32) << 16;
+        const bool bf = p.in_dtype == DT_BF16;
+        int s = 0, a = 0;
+        uint32_t sph = 0, aph = 0;
+        for (;;) {
+            mbar_wait(&s_full[s], sph);
+            const G2Hdr h = *shdr(s);
+            if (h.flags & SH_END) break;
+            if (h.flags & SH_EMPTY) {
+                if (++s == C::NS) { s = 0; sph ^= 1; }
+                continue;
+            }
+            const bool valid = (h.hv >> myhalf) & 1;
+            const uint32_t xs_s = smem_u32(stage(s));
+            float rr = valid ? 1.f : 0.f;
+            if (GS && valid) rr = lds_f32(xs_s + C::XB + C::VB + 4 * r);
+            mbar_wait(&a_empty[a], aph ^ 1);
+            tc_fence_after();
+            const uint32_t a_tm = tmem_a + lane_off + a * (T / 2);
+#pragma unroll
+            for (int c = 0; c < T / 32; ++c) {  // 32 keys -> 16 packed words per tcgen05.st
+                uint32_t pk[16];
+                if (rr != 0.f) {
+#pragma unroll
+                    for (int q4 = 0; q4 < 4; ++q4) {
+                        const uint4 x = lds128(xs_s + tile_chunk_off(r, c * 4 + q4));
+                        const uint32_t xw[4] = {x.x, x.y, x.z, x.w};
+#pragma unroll
+                        for (int u = 0; u < 4; ++u) {
+                            if (GS) {  // Y = X' * r'  (fp16 X' -> fp32 -> x r' -> dtype, one rounding)
+                                const float2 f = unpack_f16(xw[u]);
+                                pk[q4 * 4 + u] = bf ? pack_bf16(f.x * rr, f.y * rr) : pack_f16(f.x * rr, f.y * rr);
+                            } else {  // P already holds dtype values
+                                pk[q4 * 4 + u] = xw[u];
+                            }
+                        }
+                    }
+                } else {  // invalid half (not loaded) or r' = 0: zero rows of A
+#pragma unroll
+                    for (int u = 0; u < 16; ++u) pk[u] = 0u;
+                }
+                tmem_st16(a_tm + c * 16, pk);
+            }
+            tmem_wait_st();
+            tc_fence_before();
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&a_full[a]);
+            if (++s == C::NS) { s = 0; sph ^= 1; }
+            if (++a == C::NA) { a = 0; aph ^= 1; }
+        }
+    } else if (warp >= 8) {
+        // ------------------------------------------------------------------ output epilogue
+        const int r = (warp % 4) * 32 + lane;
+        const uint32_t lane_off = (uint32_t)((warp % 4) * 32) << 16;
+        int o = 0;
+        uint32_t oph = 0;
+        for (;;) {
+            mbar_wait(&o_full[o], oph);
+            tc_fence_after();
+            const G2Hdr h = ohdr[o];
+            if (h.flags & SH_END) break;
+            const int64_t orow = (((int64_t)h.orow_hi << 32) | (uint32_t)h.orow_lo) + r;
+            if (h.flags & SH_EMPTY) {  // no kept key anywhere in these rows: output 0 (reading R9)
+                if (p.out_dtype == DT_F32) {
+                    float4* O = reinterpret_cast<float4*>((float*)p.out + orow * D);
+                    for (int c = 0; c < D / 4; ++c) O[c] = make_float4(0.f, 0.f, 0.f, 0.f);
+                } else {
+                    uint4* O = reinterpret_cast<uint4*>((uint16_t*)p.out + orow * D);
+                    for (int c = 0; c < D / 8; ++c) O[c] = make_uint4(0, 0, 0, 0);
+                }
+            } else {
+                const uint32_t taddr = tmem_o + lane_off + o * D;
+#pragma unroll
+                for (int c = 0; c < D / 32; ++c) {
+                    uint32_t v[32];
+                    tmem_ld32(taddr + c * 32, v);
+                    tmem_wait_ld();
+                    if (p.out_dtype == DT_F32) {
+                        float4* O = reinterpret_cast<float4*>((float*)p.out + orow * D + c * 32);
+#pragma unroll
+                        for (int u = 0; u < 8; ++u)
+                            O[u] = make_float4(__uint_as_float(v[4 * u]), __uint_as_float(v[4 * u + 1]),
+                                               __uint_as_float(v[4 * u + 2]), __uint_as_float(v[4 * u + 3]));
+                    } else {
+                        uint32_t pk[16];
+#pragma unroll
+                        for (int u = 0; u < 16; ++u) {
+                            const float f0 = __uint_as_float(v[2 * u]), f1 = __uint_as_float(v[2 * u + 1]);
+                            pk[u] = p.out_dtype == DT_BF16 ? pack_bf16(f0, f1) : pack_f16(f0, f1);
+                        }
+                        uint4* O = reinterpret_cast<uint4*>((uint16_t*)p.out + orow * D + c * 32);
+#pragma unroll
+                        for (int u = 0; u < 4; ++u) O[u] = make_uint4(pk[4 * u], pk[4 * u + 1], pk[4 * u + 2], pk[4 * u + 3]);
+                    }
+                }
+                tc_fence_before();
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&o_empty[o]);
+            if (++o == C::NO) { o = 0; oph ^= 1; }
+        }
+    }
+    tc_fence_before();
+    __syncthreads();
+    if (warp == 2) {
+        tc_fence_after();
+        tmem_dealloc(tmem_base, 512);
+    }
+}
+
+// ----------------------------------------------------------------------------- launchers
+
+cudaError_t make_tmap_2d(CUtensorMap* m, const void* base, int64_t rows, int D, int box_rows, int dtype);
+int num_sms();
+
+template <int D, int T, bool GS>
+cudaError_t launch_g2_t(const Params& p, cudaStream_t st, int64_t* nl)
+{
+    using C = G2<D, T>;
+    CUtensorMap tv;
+    const int64_t rows = (int64_t)p.B * p.H * p.S;
+    cudaError_t e;
+    if ((e = make_tmap_2d(&tv, p.v, rows, D, T, p.in_dtype)) != cudaSuccess) return e;
+    auto kern = tc_gemm2<D, T, GS>;
+    if ((e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM)) != cudaSuccess) return e;
+    const int grid = std::min(p.sc.n_items, num_sms());
+    kern<<<grid, C::THREADS, C::SMEM, st>>>(tv, p);
+    ++*nl;
+    return cudaGetLastError();
+}
+
+cudaError_t launch_gemm2(const Params& p, bool gs, cudaStream_t st, int64_t* nl)
+{
+    if (p.D == 64) {
+        if (p.T == 64) return gs ? launch_g2_t<64, 64, true>(p, st, nl) : launch_g2_t<64, 64, false>(p, st, nl);
+        return gs ? launch_g2_t<64, 128, true>(p, st, nl) : launch_g2_t<64, 128, false>(p, st, nl);
+    }
+    if (p.T == 64) return gs ? launch_g2_t<128, 64, true>(p, st, nl) : launch_g2_t<128, 64, false>(p, st, nl);
+    return gs ? launch_g2_t<128, 128, true>(p, st, nl) : launch_g2_t<128, 128, false>(p, st, nl);
+}
+
+}  // namespace sr

@@ -1,0 +1,87 @@
+// tc_common.cuh -- device helpers shared by the tensor-core kernels (k_gemm1.cu, k_gemm2.cu,
+// k_softmax.cu): schedule decoding, the attention-tile smem/HBM layout, interval element masks.
+#pragma once
+#include <climits>
+#include <cstdint>
+
+#include "ptx.cuh"
+#include "sr_internal.h"
+
+namespace sr {
+
+constexpr int kSmemMax = 232448;  // 227 KB opt-in dynamic shared memory per CTA on sm_100
+
+struct ItemInfo {
+    int g, rb, t0, t1;
+    int64_t slot0;  // slot id of tile t is slot0 + t
+};
+
+__device__ __forceinline__ ItemInfo decode_item(const Params& p, int it)
+{
+    const DevSched& sc = p.sc;
+    const int item = __ldg(sc.items + it);
+    ItemInfo r;
+    r.g = item / sc.n_rb;
+    r.rb = item % sc.n_rb;
+    const int lh = lh_of(sc, r.g, p.H);
+    const int32_t* tp = sc.tp + (size_t)lh * (sc.n_rb + 1);
+    r.t0 = __ldg(tp + r.rb);
+    r.t1 = __ldg(tp + r.rb + 1);
+    r.slot0 = (int64_t)r.g * sc.slots_per_head - __ldg(tp);
+    return r;
+}
+
+// Attention-matrix tiles (X', S, P) are 128 rows x T keys of 16-bit values in the canonical
+// SWIZZLE_128B K-major layout [T/64][128 rows][64 cols]: row r of column-half h is 128 contiguous
+// bytes at h*16 KB + r*128 whose 16-B chunk c sits at position c ^ (r & 7).  Byte offset of
+// logical chunk c (0 .. T/8-1) of row r:
+__host__ __device__ __forceinline__ uint32_t tile_chunk_off(int r, int c)
+{
+    return (uint32_t)((c >> 3) * (kRowBlock * 128) + r * 128 + (((c & 7) ^ (r & 7)) << 4));
+}
+
+// ---------------------------------------------------------------- element masks as intervals
+// For query row i the kept keys (PAPER.md L53 mask layer) are
+//     j in [lo, hi]  and  (j in [blo, bhi]  or  j < gc)
+// lo/hi: key padding (kv_len) and causality; blo/bhi/gc: Longformer band and global columns
+// (a global row keeps everything).  Block sparsity is handled by the tile list, not here.
+struct RowMask {
+    int lo, hi, blo, bhi, gc;
+};
+
+__device__ __forceinline__ RowMask row_mask(const Params& p, int i, int kvl)
+{
+    RowMask m;
+    m.lo = 0;
+    m.hi = kvl - 1;
+    if (p.causal) m.hi = min(m.hi, i);
+    if (p.mask_kind == MK_WINDOW && i >= p.n_global) {
+        m.blo = i - p.win_half;
+        m.bhi = i + p.win_half;
+        m.gc = p.n_global;
+    } else {
+        m.blo = 0;
+        m.bhi = INT_MAX / 4;
+        m.gc = 0;
+    }
+    return m;
+}
+
+// bits u of a 32-bit word with a <= u <= b (a, b may lie outside [0, 31])
+__device__ __forceinline__ uint32_t ibits32(int a, int b)
+{
+    a = max(a, 0);
+    b = min(b, 31);
+    if (b < a) return 0u;
+    const uint32_t hi = (b == 31) ? 0xffffffffu : ((1u << (b + 1)) - 1u);
+    const uint32_t lo = ~((1u << a) - 1u);
+    return hi & lo;
+}
+
+// kept-key bits of keys c0 .. c0+31 for the row
+__device__ __forceinline__ uint32_t mask_bits32(const RowMask& m, int c0)
+{
+    return ibits32(m.lo - c0, m.hi - c0) & (ibits32(m.blo - c0, m.bhi - c0) | ibits32(-c0, m.gc - 1 - c0));
+}
+
+}  // namespace sr
