@@ -367,13 +367,15 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
     if (((uintptr_t)q | (uintptr_t)k | (uintptr_t)v | (uintptr_t)out) & 15)
         return fail(SR_ERR_INVALID, "q, k, v, out must be 16-byte aligned");
     std::shared_ptr<CachedSched> cs;
-    s = host_sched(r, cs, true);
+    s = host_sched(r, cs, false);  // host-only schedule: workspace checks precede any CUDA call
     if (s != SR_OK) return s;
     sr_ws_info wi;
     ws_layout(cs->hs, B, H, ex->in_dtype, fused, &wi);
     if (!ex->workspace || ex->workspace_bytes < wi.total_bytes)
         return fail(SR_ERR_WORKSPACE, "workspace %zu bytes < required %zu", ex->workspace_bytes, wi.total_bytes);
     if ((uintptr_t)ex->workspace & 255) return fail(SR_ERR_WORKSPACE, "workspace must be 256-byte aligned");
+    s = host_sched(r, cs, true);  // device copy of the schedule (cached per device)
+    if (s != SR_OK) return s;
 
     Params p{};
     p.q = q; p.k = k; p.v = v; p.out = out;

@@ -1,0 +1,211 @@
+"""CPU tests of the C ABI boundary (no GPU needed): the library loads and exports every symbol
+include/sr_mha.h declares, argument validation returns its documented status before any CUDA call,
+workspace sizes match the closed forms of PAPER.md L145/L149, and the tile schedule (which tiles are
+computed / stored) matches an independent numpy derivation from the mask definition."""
+import ctypes as C
+import os
+import re
+import subprocess
+
+import numpy as np
+import pytest
+
+import workloads as W
+from oracle import oracle_np
+
+import paper_conf_iiswc_choilkha22_b200 as sr
+from paper_conf_iiswc_choilkha22_b200 import build as B
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module", autouse=True)
+def built():
+    B.build()
+    sr.lib()
+
+
+def header_functions():
+    txt = open(os.path.join(ROOT, "include", "sr_mha.h")).read()
+    txt = re.sub(r"/\*.*?\*/", "", txt, flags=re.S)
+    return sorted(set(re.findall(r"\b(sr_[a-z_0-9]+)\s*\(", txt)))
+
+
+def test_exports_every_declared_symbol():
+    names = header_functions()
+    assert len(names) >= 13
+    out = subprocess.run(["nm", "-D", "--defined-only", sr.LIB_PATH], capture_output=True, text=True).stdout
+    exported = set(re.findall(r"\bT (sr_[a-z_0-9]+)\b", out))
+    missing = [n for n in names if n not in exported]
+    assert not missing, missing
+    assert set(sr.EXPORTS) == set(names)
+    assert sr.lib().sr_version().decode().startswith("sr_mha")
+
+
+def test_library_is_sm100a():
+    out = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "--list-elf", sr.LIB_PATH], capture_output=True,
+                         text=True).stdout
+    assert "sm_100a" in out
+
+
+# ------------------------------------------------------------------------------ validation
+
+def _call(entry_fn, q=0x10000, k=0x20000000, v=0x40000000, out=0x60000000, B_=1, H=1, S=128, D=64, scale=0.125,
+          mask=None, causal=0, in_dt=sr.SR_F16, out_dt=None, ws=0x80000000, ws_bytes=1 << 40, flags=0, tile_n=0):
+    ex = sr.Exec(in_dt, in_dt if out_dt is None else out_dt, ws, ws_bytes, None, tile_n, flags)
+    return getattr(sr.lib(), entry_fn)(q, k, v, out, B_, H, S, D, C.c_float(scale), mask, causal, C.byref(ex))
+
+
+@pytest.mark.parametrize("kw,status", [
+    (dict(S=100), sr.SR_ERR_UNSUPPORTED),
+    (dict(S=64), sr.SR_ERR_UNSUPPORTED),
+    (dict(D=96), sr.SR_ERR_UNSUPPORTED),
+    (dict(D=256), sr.SR_ERR_UNSUPPORTED),
+    (dict(B_=0), sr.SR_ERR_INVALID),
+    (dict(scale=0.0), sr.SR_ERR_INVALID),
+    (dict(scale=float("nan")), sr.SR_ERR_INVALID),
+    (dict(scale=-1.0), sr.SR_ERR_INVALID),
+    (dict(q=0), sr.SR_ERR_INVALID),
+    (dict(out=0), sr.SR_ERR_INVALID),
+    (dict(in_dt=7), sr.SR_ERR_INVALID),
+    (dict(out_dt=sr.SR_BF16), sr.SR_ERR_UNSUPPORTED),
+    (dict(out=0x10000 + 64), sr.SR_ERR_INVALID),          # out overlaps q
+    (dict(q=0x10008), sr.SR_ERR_INVALID),                 # misaligned
+    (dict(flags=8), sr.SR_ERR_INVALID),
+    (dict(tile_n=32), sr.SR_ERR_UNSUPPORTED),
+    (dict(in_dt=sr.SR_F32, tile_n=128), sr.SR_ERR_UNSUPPORTED),
+    (dict(ws=0), sr.SR_ERR_WORKSPACE),
+    (dict(ws_bytes=1024), sr.SR_ERR_WORKSPACE),
+    (dict(ws=0x80000010), sr.SR_ERR_WORKSPACE),           # workspace not 256-B aligned
+])
+def test_argument_errors_before_cuda(kw, status):
+    st = _call("sr_mha_dense", **kw)
+    assert st == status, (st, sr.last_error())
+    assert sr.last_error()
+
+
+def test_null_exec():
+    L = sr.lib()
+    assert L.sr_mha_dense(1, 1, 1, 1, 1, 1, 128, 64, C.c_float(1.0), None, 0, None) == sr.SR_ERR_INVALID
+
+
+def test_kv_len_range():
+    m = sr.dense_mask([129])
+    assert _call("sr_mha_dense", mask=m.ptr) == sr.SR_ERR_INVALID
+    m = sr.dense_mask([-1])
+    assert _call("sr_mha_dense", mask=m.ptr) == sr.SR_ERR_INVALID
+
+
+def test_block_layout_validation():
+    lay = W.csr_from_sets(64, [[{0}, {0, 1}]])
+    assert _call("sr_mha_blocksparse", mask=sr.block_mask(lay).ptr) != sr.SR_ERR_INVALID
+    bad = W.csr_from_sets(64, [[{0}, {0, 1}]])
+    bad.col_idx = bad.col_idx[::-1].copy()  # not ascending
+    assert _call("sr_mha_blocksparse", mask=sr.block_mask(bad).ptr) == sr.SR_ERR_INVALID
+    bad2 = W.csr_from_sets(64, [[{0}, {5}]])  # column out of range
+    assert _call("sr_mha_blocksparse", mask=sr.block_mask(bad2).ptr) == sr.SR_ERR_INVALID
+    two = W.csr_from_sets(64, [[{0}, {1}], [{1}, {0}]])  # layout_heads = 2 with H = 1
+    assert _call("sr_mha_blocksparse", mask=sr.block_mask(two).ptr) == sr.SR_ERR_INVALID
+    assert _call("sr_mha_blocksparse", mask=None) == sr.SR_ERR_INVALID
+    assert _call("sr_mha_blocksparse", mask=sr.block_mask(lay).ptr, tile_n=128) == sr.SR_ERR_UNSUPPORTED
+    lay32 = W.csr_from_sets(32, [[{0}, {1}, {2}, {3}]])
+    assert _call("sr_mha_blocksparse", mask=sr.block_mask(lay32).ptr) == sr.SR_ERR_UNSUPPORTED
+
+
+def test_window_validation():
+    assert _call("sr_mha_sliding_window", mask=None) == sr.SR_ERR_INVALID
+    assert _call("sr_mha_sliding_window", mask=sr.window_mask(-2, 0).ptr) == sr.SR_ERR_INVALID
+    assert _call("sr_mha_sliding_window", mask=sr.window_mask(8, 200).ptr) == sr.SR_ERR_INVALID
+
+
+def test_unfused_rejects_fp32():
+    assert _call("sr_mha_dense_unfused", in_dt=sr.SR_F32) == sr.SR_ERR_UNSUPPORTED
+
+
+def test_python_binding_rejects_cpu_tensors():
+    torch = pytest.importorskip("torch")
+    x = torch.zeros(1, 1, 128, 64, dtype=torch.float16)
+    with pytest.raises(ValueError):
+        sr.mha_dense(x, x, x)
+
+
+# ------------------------------------------------------------------------------ workspace sizes
+
+@pytest.mark.parametrize("T", [64, 128])
+def test_workspace_closed_form_dense(T):
+    """X' has L^2 H elements, m', d', r' have L N_sv H each (dense, no mask)."""
+    Bb, H, S, D = 2, 3, 512, 64
+    info = sr.workspace_info(sr.dense_mask(None), Bb, H, S, D, sr.SR_F16, tile_n=T)
+    L2H = Bb * H * S * S
+    assert info["tile_n"] == T
+    assert info["n_slots"] * 128 * T == L2H
+    assert info["n_slots"] * 128 == Bb * H * S * (S // T)  # L N_sv H
+    assert info["off_mprime"] >= L2H * 2
+    assert info["total_bytes"] >= L2H * 2 + 3 * 4 * Bb * H * S * (S // T)
+    unf = sr.workspace_info(sr.dense_mask(None), Bb, H, S, D, sr.SR_F16, tile_n=T, fused=False)
+    assert unf["off_p"] >= L2H * 2 and unf["total_bytes"] >= 2 * L2H * 2
+
+
+def test_workspace_bytes_matches_query():
+    m = sr.dense_mask([300, 17])
+    n = sr.lib().sr_workspace_bytes(sr.SR_E_DENSE, 1, 2, 4, 512, 128, sr.SR_BF16, m.ptr, 1, 0)
+    assert n == sr.workspace_info(m, 2, 4, 512, 128, sr.SR_BF16, causal=True)["total_bytes"]
+    assert sr.lib().sr_workspace_bytes(sr.SR_E_DENSE, 1, 2, 4, 100, 128, sr.SR_BF16, None, 0, 0) == 0
+
+
+# ------------------------------------------------------------------------------ tile schedules
+
+def numpy_schedule(S, T, allowed_fn, BH):
+    """Tiles (128 rows x T keys) holding >= 1 kept element, per 64-row half, from dense masks."""
+    tiles = elems = 0
+    for g in range(BH):
+        a = allowed_fn(g)
+        for rb in range(S // 128):
+            for kt in range(S // T):
+                blk = a[rb * 128:(rb + 1) * 128, kt * T:(kt + 1) * T]
+                halves = [blk[:64].any(), blk[64:].any()]
+                if any(halves):
+                    tiles += 1
+                    elems += sum(halves) * 64 * T
+    return tiles, elems
+
+
+@pytest.mark.parametrize("T", [64, 128])
+@pytest.mark.parametrize("causal", [False, True])
+def test_schedule_dense(T, causal):
+    S, H = 512, 2
+    kv = [512, 300, 65, 1]
+    got = sr.schedule_stats(sr.dense_mask(kv), len(kv), H, S, causal=causal, tile_n=T)
+    want = numpy_schedule(S, T, lambda g: oracle_np.allowed_matrix(S, b=g // H, kv_len=kv, causal=causal), len(kv) * H)
+    assert got == want
+
+
+@pytest.mark.parametrize("window,n_global,causal,T", [(0, 0, False, 64), (10, 3, False, 64), (300, 8, False, 64),
+                                                      (300, 8, True, 128), (130, 64, False, 128), (512, 8, True, 64)])
+def test_schedule_window(window, n_global, causal, T):
+    S = 768
+    got = sr.schedule_stats(sr.window_mask(window, n_global), 1, 1, S, causal=causal, tile_n=T)
+    a = oracle_np.allowed_matrix(S, kind="window", window=window, n_global=n_global, causal=causal)
+    assert got == numpy_schedule(S, T, lambda g: a, 1)
+
+
+@pytest.mark.parametrize("causal", [False, True])
+def test_schedule_blocksparse(causal):
+    S, H = 1024, 3
+    lay = W.random_layout(H, S // 64, 64, 0.3, seed=11)
+    got = sr.schedule_stats(sr.block_mask(lay), 2, H, S, causal=causal)
+    want = numpy_schedule(S, 64, lambda g: oracle_np.allowed_matrix(S, h=g % H, kind="block", layout=lay,
+                                                                     causal=causal), 2 * H)
+    assert got == want
+
+
+def test_schedule_configs_match_survey():
+    """Stored-element counts of the BASELINE configs."""
+    c3 = W.config(3)
+    assert sr.schedule_stats(sr.dense_mask(None), c3.B, c3.H, c3.S, causal=True) == (64 * 136, 142_606_336)
+    c4 = W.config(4)
+    assert sr.schedule_stats(sr.block_mask(W.config_layout(c4)), c4.B, c4.H, c4.S)[1] == 48 * 622 * 64 * 64
+    c5 = W.config(5)
+    assert sr.schedule_stats(sr.window_mask(c5.window, c5.n_global), c5.B, c5.H, c5.S)[1] == 24 * 674 * 64 * 64
+    c2 = W.config(2)
+    assert sr.schedule_stats(sr.dense_mask(c2.kv_len), c2.B, c2.H, c2.S)[0] == 12 * 20 * 4
