@@ -1,0 +1,98 @@
+"""Summarise ncu captures from gpurun_out/ into committed profiles/ files.
+
+  python tools/make_profiles.py ROUND   (e.g. r1)
+
+Reads gpurun_out/launches_c{2,3}.csv (ncu --metrics gpu__time_duration.sum,dram__bytes_*: every
+launch of a short bench.py run, cold-cache and serialised) and gpurun_out/full_c{2,3}_*.ncu-rep
+(ncu --set full of each kernel), writes profiles/ROUND_launches_cN.txt, profiles/ROUND_full_cN_K.txt
+and profiles/ncu_traffic.json (per-kernel DRAM bytes per launch, read by bench.py's roofline).
+"""
+import collections
+import csv
+import json
+import os
+import subprocess
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+OUT = os.path.join(ROOT, "gpurun_out")
+PROF = os.path.join(ROOT, "profiles")
+NAMES = {"tc_gemm1": "gemm1", "ir_kernel": "ir", "tc_gemm2": "gemm2", "row_softmax": "softmax"}
+
+
+def kname(full):
+    for k, v in NAMES.items():
+        if k in full:
+            fused = ", true>" in full or ", (bool)1>" in full or "1>(" in full
+            if k in ("tc_gemm1", "tc_gemm2"):
+                return (("gemm1_ls" if k == "tc_gemm1" else "gs_gemm2") if fused else v + "_plain")
+            return v
+    return None
+
+
+def launches(path):
+    rows = list(csv.reader(open(path)))
+    hdr = next(i for i, r in enumerate(rows) if "Kernel Name" in r)
+    h = rows[hdr]
+    agg = collections.defaultdict(lambda: collections.defaultdict(list))
+    order = []
+    for r in rows[hdr + 1:]:
+        if len(r) != len(h):
+            continue
+        d = dict(zip(h, r))
+        n = kname(d["Kernel Name"]) or ("other:" + d["Kernel Name"][:40])
+        if n not in order:
+            order.append(n)
+        agg[n][d["Metric Name"]].append(float(d["Metric Value"].replace(",", "")))
+    return order, agg
+
+
+def main(rnd):
+    os.makedirs(PROF, exist_ok=True)
+    traffic = {}
+    for c in (2, 3):
+        p = os.path.join(OUT, f"launches_c{c}.csv")
+        if not os.path.exists(p):
+            continue
+        order, agg = launches(p)
+        lines = [f"# ncu launch list, bench.py --config {c} (cold-cache, serialised launches; compare SHARES)",
+                 f"{'kernel':28s} {'launches':>8s} {'mean us':>10s} {'DRAM rd MB':>11s} {'DRAM wr MB':>11s}"]
+        ours = {}
+        for n in order:
+            m = agg[n]
+            t = sum(m["gpu__time_duration.sum"]) / len(m["gpu__time_duration.sum"])
+            rd = sum(m["dram__bytes_read.sum"]) / len(m["dram__bytes_read.sum"])
+            wr = sum(m["dram__bytes_write.sum"]) / len(m["dram__bytes_write.sum"])
+            unit = 1.0
+            lines.append(f"{n:28s} {len(m['gpu__time_duration.sum']):8d} {t / 1e3 * unit:10.2f} {rd / 1e6:11.2f} {wr / 1e6:11.2f}")
+            if not n.startswith("other"):
+                ours[n] = (t, rd + wr)
+        rec = [k for k in ("gemm1_ls", "ir", "gs_gemm2") if k in ours]
+        unf = [k for k in ("gemm1_plain", "softmax", "gemm2_plain") if k in ours]
+        tr = sum(ours[k][0] for k in rec)
+        lines.append("")
+        lines.append("recomposed layer shares: " + ", ".join(f"{k} {ours[k][0] / tr:.1%}" for k in rec))
+        tu = sum(ours[k][0] for k in unf) if unf else 0
+        if unf:
+            lines.append("unfused layer shares:    " + ", ".join(f"{k} {ours[k][0] / tu:.1%}" for k in unf))
+        e = {f"{k}_dram_bytes": int(ours[k][1]) for k in rec + unf}
+        e["recomposed_dram_bytes"] = int(sum(ours[k][1] for k in rec))
+        if unf:
+            e["unfused_dram_bytes"] = int(sum(ours[k][1] for k in unf))
+        lines.append(f"DRAM bytes per layer (cold, per-kernel sum): recomposed {e['recomposed_dram_bytes'] / 1e6:.1f} MB"
+                     + (f", unfused {e['unfused_dram_bytes'] / 1e6:.1f} MB" if unf else ""))
+        traffic[f"C{c}"] = e
+        open(os.path.join(PROF, f"{rnd}_launches_c{c}.txt"), "w").write("\n".join(lines) + "\n")
+        for k in ("tc_gemm1", "tc_gemm2", "ir_kernel"):
+            rep = os.path.join(OUT, f"full_c{c}_{k}.ncu-rep")
+            if os.path.exists(rep):
+                s = subprocess.run([sys.executable, os.path.join(ROOT, "tools", "ncu_summary.py"), rep, "25"],
+                                   capture_output=True, text=True).stdout
+                open(os.path.join(PROF, f"{rnd}_full_c{c}_{k}.txt"), "w").write(
+                    f"# ncu --set full --clock-control none, tools/run_layer.py {c} (second launch)\n" + s)
+    json.dump(traffic, open(os.path.join(PROF, "ncu_traffic.json"), "w"), indent=1)
+    print(json.dumps(traffic, indent=1))
+
+
+if __name__ == "__main__":
+    main(sys.argv[1] if len(sys.argv) > 1 else "r1")
