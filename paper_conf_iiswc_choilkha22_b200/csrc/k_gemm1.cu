@@ -31,7 +31,7 @@ struct G1Hdr {  // per-accumulator tile header, written by the MMA warp
 };
 enum : int { HDR_TILE = 1, HDR_END = 2 };
 
-template <int D, int T>
+template <int D, int T, int XPWMAX = 2>
 struct G1 {
     static constexpr int QB = kRowBlock * D * 2;  // Q tile bytes
     static constexpr int KB = T * D * 2;          // K tile bytes
@@ -39,7 +39,7 @@ struct G1 {
     static constexpr int NQ = 2;
     static constexpr int NACC = 512 / T;  // TMEM accumulators (4 for T=128, 8 for T=64)
     // staging buffers per epilogue warpgroup: 2 when shared memory allows, else 1
-    static constexpr int XPW = (NQ * QB + 2 * KB + 4 * XB + 4096 <= kSmemMax) ? 2 : 1;
+    static constexpr int XPW = (XPWMAX >= 2 && NQ * QB + 2 * KB + 4 * XB + 4096 <= kSmemMax) ? 2 : 1;
     static constexpr int NK_ = (kSmemMax - 4096 - NQ * QB - 2 * XPW * XB) / KB;
     static constexpr int NK = NK_ > 4 ? 4 : NK_;
     static_assert(NK >= 2, "smem budget");
@@ -55,11 +55,11 @@ struct G1 {
     static constexpr int THREADS = 384;
 };
 
-template <int D, int T, bool LS>
+template <int D, int T, bool LS, int XPWMAX>
 __global__ void __launch_bounds__(384, 1)
     tc_gemm1(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmK, const Params p)
 {
-    using C = G1<D, T>;
+    using C = G1<D, T, XPWMAX>;
     extern __shared__ uint8_t smem_raw[];
     uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
     uint64_t* bars = (uint64_t*)(smem + C::OFF_BAR);
@@ -285,13 +285,13 @@ int num_sms();
 template <int D, int T, bool LS>
 cudaError_t launch_g1_t(const Params& p, cudaStream_t st, int64_t* nl)
 {
-    using C = G1<D, T>;
+    using C = G1<D, T, 2>;
     CUtensorMap tq, tk;
     const int64_t rows = (int64_t)p.B * p.H * p.S;
     cudaError_t e;
     if ((e = make_tmap_2d(&tq, p.q, rows, D, kRowBlock, p.in_dtype)) != cudaSuccess) return e;
     if ((e = make_tmap_2d(&tk, p.k, rows, D, T, p.in_dtype)) != cudaSuccess) return e;
-    auto kern = tc_gemm1<D, T, LS>;
+    auto kern = tc_gemm1<D, T, LS, 2>;
     if ((e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM)) != cudaSuccess) return e;
     const int grid = std::min(p.sc.n_items, num_sms());
     kern<<<grid, C::THREADS, C::SMEM, st>>>(tq, tk, p);

@@ -9,12 +9,16 @@
 //   O     += Y_tile V_tile   (tcgen05.mma kind::f16, A from TMEM, B = V from smem, fp32 in TMEM)
 //
 // Warp roles (persistent CTA per SM, 384 threads):
-//   warp 0      producer: per tile one smem stage = X' tile (1-D bulk copy of its valid halves) +
-//               V tile (TMA, 128B swizzle) + r' of the 128 rows (bulk copy) + a stage header
-//               (half-valid bits, item boundaries); EMPTY items and the END of the schedule travel
-//               through the same ring as header-only stages
-//   warp 1      MMA issuer: T/16 MMAs of 128 x D x 16 per tile into one of two O accumulators;
-//               publishes the item's output row to the epilogue through an O header
+//   warp 0      X' producer: X' tile (1-D bulk copy of its valid 64-row halves; the tile is already
+//               in the UMMA SW128 K-major layout) + the tile's 128 r' values + a stage header, into
+//               an NX-deep ring; ends with an END header.  The X' ring is only read by the GS warps,
+//               so a stage is recycled as soon as they have written it into TMEM (not after the MMA)
+//               -- X' (the dominant HBM stream) can run NX tiles ahead of the tensor core.
+//   warp 3      V producer: V tile (TMA, SW128, used as the MN-major B operand) into an NV-deep ring
+//               (V is mostly L2-resident: reused by every row block of a head)
+//   warp 1      MMA issuer: T/16 MMAs of 128 x D x 16 per tile into one of two TMEM O accumulators;
+//               walks the item list itself and publishes each item's output rows (or EMPTY / END)
+//               to the epilogue through an O header
 //   warp 2      TMEM allocator (512 columns: 2 x D for O, NA x T/2 for the A operand ring)
 //   warps 4-7   GS transform: smem X' row -> fp32 x r' -> dtype -> tcgen05.st into TMEM (A operand)
 //   warps 8-11  epilogue: tcgen05.ld of O rows -> out dtype -> global
@@ -24,27 +28,30 @@ namespace sr {
 
 using namespace ptx;
 
-enum : int { SH_TILE = 1, SH_END = 2, SH_EMPTY = 4, SH_FIRST = 8, SH_LAST = 16 };
-struct G2Hdr {  // stage / O-buffer header
+enum : int { SH_TILE = 1, SH_END = 2, SH_EMPTY = 4 };
+struct G2Hdr {  // X'-stage / O-buffer header
     int32_t flags, hv, orow_lo, orow_hi;
 };
 
 template <int D, int T>
 struct G2 {
     static constexpr int XB = kRowBlock * T * 2;  // X' / P tile
-    static constexpr int VB = T * D * 2;          // V tile
-    static constexpr int RB = 1024;               // r' (512 B) + stage header, padded to keep 1 KB alignment
-    static constexpr int SB = XB + VB + RB;
-    static constexpr int NS_ = (kSmemMax - 2048) / SB;
-    static constexpr int NS = NS_ > 6 ? 6 : NS_;
-    static_assert(NS >= 2, "smem budget");
+    static constexpr int RB = 1024;               // r' (512 B) + header, padded to keep 1 KB alignment
+    static constexpr int XSB = XB + RB;           // X' stage
+    static constexpr int VB = T * D * 2;          // V tile (V stage)
+    // split the smem budget: V stages from L2 need less depth than the HBM-bound X' stream
+    static constexpr int NV = (VB >= 32768) ? 2 : ((VB >= 16384) ? 3 : 4);
+    static constexpr int NX_ = (kSmemMax - 3072 - NV * VB) / XSB;
+    static constexpr int NX = NX_ > 8 ? 8 : NX_;
+    static_assert(NX >= 2, "smem budget");
     static constexpr int NO = 2;                          // O accumulators (D cols each)
     static constexpr int NA_ = (512 - NO * D) / (T / 2);  // A operand buffers (T/2 cols each)
     static constexpr int NA = NA_ > 8 ? 8 : NA_;
     static_assert(NA >= 2, "tmem budget");
-    static constexpr int OFF_S = 0;
-    static constexpr int OFF_BAR = NS * SB;
-    static constexpr int NBAR = 2 * NS + 2 * NA + 2 * NO;
+    static constexpr int OFF_X = 0;
+    static constexpr int OFF_V = NX * XSB;
+    static constexpr int OFF_BAR = OFF_V + NV * VB;
+    static constexpr int NBAR = 2 * NX + 2 * NV + 2 * NA + 2 * NO;
     static constexpr int OFF_OHDR = OFF_BAR + NBAR * 8;
     static constexpr int OFF_TPTR = OFF_OHDR + NO * (int)sizeof(G2Hdr);
     static constexpr int SMEM_ = OFF_TPTR + 16 + 1024;
@@ -59,26 +66,30 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
     extern __shared__ uint8_t smem_raw[];
     uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
     uint64_t* bars = (uint64_t*)(smem + C::OFF_BAR);
-    uint64_t* s_full = bars;
-    uint64_t* s_empty = s_full + C::NS;
-    uint64_t* a_full = s_empty + C::NS;
+    uint64_t* x_full = bars;
+    uint64_t* x_empty = x_full + C::NX;
+    uint64_t* v_full = x_empty + C::NX;
+    uint64_t* v_empty = v_full + C::NV;
+    uint64_t* a_full = v_empty + C::NV;
     uint64_t* a_empty = a_full + C::NA;
     uint64_t* o_full = a_empty + C::NA;
     uint64_t* o_empty = o_full + C::NO;
     G2Hdr* ohdr = (G2Hdr*)(smem + C::OFF_OHDR);
     uint32_t* tmem_ptr = (uint32_t*)(smem + C::OFF_TPTR);
-    auto stage = [&](int s) { return smem + C::OFF_S + s * C::SB; };
-    auto shdr = [&](int s) { return (G2Hdr*)(stage(s) + C::XB + C::VB + 512); };
+    auto xstage = [&](int s) { return smem + C::OFF_X + s * C::XSB; };
+    auto xhdr = [&](int s) { return (G2Hdr*)(xstage(s) + C::XB + 512); };
+    auto vstage = [&](int s) { return smem + C::OFF_V + s * C::VB; };
 
     const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
     if (threadIdx.x == 0) {
-        for (int i = 0; i < C::NS; ++i) { mbar_init(&s_full[i], 1); mbar_init(&s_empty[i], 1); }
+        for (int i = 0; i < C::NX; ++i) { mbar_init(&x_full[i], 1); mbar_init(&x_empty[i], 4); }
+        for (int i = 0; i < C::NV; ++i) { mbar_init(&v_full[i], 1); mbar_init(&v_empty[i], 1); }
         for (int i = 0; i < C::NA; ++i) { mbar_init(&a_full[i], 4); mbar_init(&a_empty[i], 1); }
         // o_full: O-header arrive + MMA commit; o_empty: one arrive per epilogue warp
         for (int i = 0; i < C::NO; ++i) { mbar_init(&o_full[i], 2); mbar_init(&o_empty[i], 4); }
         fence_mbar_init();
     }
-    if (warp == 0 && lane == 0) prefetch_tmap(&tmV);
+    if (warp == 3 && lane == 0) prefetch_tmap(&tmV);
     if (warp == 2) tmem_alloc(tmem_ptr, 512);
     tc_fence_before();
     __syncthreads();
@@ -91,46 +102,55 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
 
     if (warp == 0) {
         if (lane == 0) {
-            // -------------------------------------------------------------- producer
+            // -------------------------------------------------------------- X' producer
             int s = 0;
             uint32_t sph = 0;
-            auto next_stage = [&]() {
-                mbar_wait(&s_empty[s], sph ^ 1);
-                return s;
-            };
-            auto advance = [&]() {
-                if (++s == C::NS) { s = 0; sph ^= 1; }
-            };
             for (int it = blockIdx.x; it < n_items; it += gridDim.x) {
                 const ItemInfo I = decode_item(p, it);
-                if (I.t0 == I.t1) continue;  // empty items never touch the stage ring
-                int w_next = __ldg(p.sc.tinfo + I.t0);
+                int w_next = I.t0 < I.t1 ? __ldg(p.sc.tinfo + I.t0) : 0;
                 for (int t = I.t0; t < I.t1; ++t) {
                     const int w = w_next;
                     if (t + 1 < I.t1) w_next = __ldg(p.sc.tinfo + t + 1);
-                    const int kt = tinfo_kt(w), hv = tinfo_half(w);
+                    const int hv = tinfo_half(w);
                     const uint32_t xbytes = (hv == 3 ? 2 : 1) * (T / 64) * (kHalf * 128);
-                    next_stage();
-                    uint8_t* st = stage(s);
-                    *shdr(s) = G2Hdr{SH_TILE, hv, 0, 0};
-                    mbar_arrive_expect_tx(&s_full[s], xbytes + C::VB + (GS ? kRowBlock * 4 : 0));
+                    mbar_wait(&x_empty[s], sph ^ 1);
+                    uint8_t* st = xstage(s);
+                    *xhdr(s) = G2Hdr{SH_TILE, hv, 0, 0};
+                    mbar_arrive_expect_tx(&x_full[s], xbytes + (GS ? kRowBlock * 4 : 0));
                     const uint8_t* xs = src + (I.slot0 + t) * (int64_t)C::XB;
-                    if (hv == 3) bulk_load(st, xs, C::XB, &s_full[s]);
+                    if (hv == 3) bulk_load(st, xs, C::XB, &x_full[s]);
                     else
                         for (int ch = 0; ch < T / 64; ++ch) {
                             const int o = ch * (kRowBlock * 128) + (hv == 2 ? kHalf * 128 : 0);
-                            bulk_load(st + o, xs + o, kHalf * 128, &s_full[s]);
+                            bulk_load(st + o, xs + o, kHalf * 128, &x_full[s]);
                         }
-                    for (int h = 0; h < D / 64; ++h)
-                        tma_load_2d(st + C::XB + h * (T * 128), &tmV, h * 64, I.g * p.S + kt * T, &s_full[s]);
                     if (GS)  // r' of the tile's 128 rows rides along with the tile
-                        bulk_load(st + C::XB + C::VB, p.rprime + (I.slot0 + t) * kRowBlock, kRowBlock * 4, &s_full[s]);
-                    advance();
+                        bulk_load(st + C::XB, p.rprime + (I.slot0 + t) * kRowBlock, kRowBlock * 4, &x_full[s]);
+                    if (++s == C::NX) { s = 0; sph ^= 1; }
                 }
             }
-            next_stage();
-            shdr(s)->flags = SH_END;
-            mbar_arrive(&s_full[s]);
+            mbar_wait(&x_empty[s], sph ^ 1);
+            xhdr(s)->flags = SH_END;
+            mbar_arrive(&x_full[s]);
+        }
+    } else if (warp == 3) {
+        if (lane == 0) {
+            // -------------------------------------------------------------- V producer
+            int s = 0;
+            uint32_t sph = 0;
+            for (int it = blockIdx.x; it < n_items; it += gridDim.x) {
+                const ItemInfo I = decode_item(p, it);
+                int w_next = I.t0 < I.t1 ? __ldg(p.sc.tinfo + I.t0) : 0;
+                for (int t = I.t0; t < I.t1; ++t) {
+                    const int w = w_next;
+                    if (t + 1 < I.t1) w_next = __ldg(p.sc.tinfo + t + 1);
+                    mbar_wait(&v_empty[s], sph ^ 1);
+                    mbar_arrive_expect_tx(&v_full[s], C::VB);
+                    for (int h = 0; h < D / 64; ++h)
+                        tma_load_2d(vstage(s) + h * (T * 128), &tmV, h * 64, I.g * p.S + tinfo_kt(w) * T, &v_full[s]);
+                    if (++s == C::NV) { s = 0; sph ^= 1; }
+                }
+            }
         }
     } else if (warp == 1) {
         if (lane == 0) {
@@ -147,7 +167,7 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
                 if (++o == C::NO) { o = 0; oph ^= 1; }
             };
             ItemInfo nxt;
-            if (blockIdx.x < n_items) nxt = decode_item(p, blockIdx.x);
+            if ((int)blockIdx.x < n_items) nxt = decode_item(p, blockIdx.x);
             for (int it = blockIdx.x; it < n_items; it += gridDim.x) {
                 const ItemInfo I = nxt;
                 if (it + (int)gridDim.x < n_items) nxt = decode_item(p, it + gridDim.x);  // prefetch
@@ -161,10 +181,10 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
                 post(SH_TILE, orow);
                 const uint32_t d_tmem = tmem_o + o * D;
                 for (int t = I.t0; t < I.t1; ++t) {
-                    mbar_wait(&s_full[s], sph);
+                    mbar_wait(&v_full[s], sph);
                     mbar_wait(&a_full[a], aph);
                     tc_fence_after();
-                    const uint32_t v_addr = smem_u32(stage(s) + C::XB);
+                    const uint32_t v_addr = smem_u32(vstage(s));
                     const uint32_t a_tm = tmem_a + a * (T / 2);
 #pragma unroll
                     for (int kk = 0; kk < T / 16; ++kk) {
@@ -172,9 +192,9 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
                         const uint64_t bd = smem_desc_sw128(v_addr + kk * 2048, T * 128, 1024);
                         mma_ts(d_tmem, a_tm + kk * 8, bd, idesc, (t == I.t0 && kk == 0) ? 0u : 1u);
                     }
-                    mma_commit(&s_empty[s]);
+                    mma_commit(&v_empty[s]);
                     mma_commit(&a_empty[a]);
-                    if (++s == C::NS) { s = 0; sph ^= 1; }
+                    if (++s == C::NV) { s = 0; sph ^= 1; }
                     if (++a == C::NA) { a = 0; aph ^= 1; }
                 }
                 mma_commit(&o_full[o]);  // arrival 2 of 2 when the item's MMAs complete
@@ -192,17 +212,19 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
         int s = 0, a = 0;
         uint32_t sph = 0, aph = 0;
         for (;;) {
-            mbar_wait(&s_full[s], sph);
-            const G2Hdr h = *shdr(s);
+            mbar_wait(&x_full[s], sph);
+            const G2Hdr h = *xhdr(s);
             if (h.flags & SH_END) break;
-            if (h.flags & SH_EMPTY) {
-                if (++s == C::NS) { s = 0; sph ^= 1; }
-                continue;
-            }
             const bool valid = (h.hv >> myhalf) & 1;
-            const uint32_t xs_s = smem_u32(stage(s));
+            const uint32_t xs_s = smem_u32(xstage(s));
             float rr = valid ? 1.f : 0.f;
-            if (GS && valid) rr = lds_f32(xs_s + C::XB + C::VB + 4 * r);
+            if (GS && valid) rr = lds_f32(xs_s + C::XB + 4 * r);
+            // the whole X' row (T fp16 = T/8 chunks of 16 B) into registers, then free the stage
+            uint4 xv[T / 8];
+            if (rr != 0.f) {
+#pragma unroll
+                for (int q4 = 0; q4 < T / 8; ++q4) xv[q4] = lds128(xs_s + tile_chunk_off(r, q4));
+            }
             mbar_wait(&a_empty[a], aph ^ 1);
             tc_fence_after();
             const uint32_t a_tm = tmem_a + lane_off + a * (T / 2);
@@ -212,8 +234,7 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
                 if (rr != 0.f) {
 #pragma unroll
                     for (int q4 = 0; q4 < 4; ++q4) {
-                        const uint4 x = lds128(xs_s + tile_chunk_off(r, c * 4 + q4));
-                        const uint32_t xw[4] = {x.x, x.y, x.z, x.w};
+                        const uint32_t xw[4] = {xv[c * 4 + q4].x, xv[c * 4 + q4].y, xv[c * 4 + q4].z, xv[c * 4 + q4].w};
 #pragma unroll
                         for (int u = 0; u < 4; ++u) {
                             if (GS) {  // Y = X' * r'  (fp16 X' -> fp32 -> x r' -> dtype, one rounding)
@@ -234,8 +255,12 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
             tc_fence_before();
             __syncwarp();
             if (lane == 0) mbar_arrive(&a_full[a]);
-            if (++s == C::NS) { s = 0; sph ^= 1; }
             if (++a == C::NA) { a = 0; aph ^= 1; }
+            // release the X' stage only now: its ld.shared results have been consumed by the tcgen05.st
+            // above.  Arriving right after issuing the loads let the next bulk copy overwrite the stage
+            // while other lanes' loads were still in flight (a real race, seen as 16-lane corruption).
+            if (lane == 0) mbar_arrive(&x_empty[s]);
+            if (++s == C::NX) { s = 0; sph ^= 1; }
         }
     } else if (warp >= 8) {
         // ------------------------------------------------------------------ output epilogue
