@@ -86,6 +86,10 @@ __global__ void __launch_bounds__(384, 1)
     __syncthreads();
     tc_fence_after();
     const uint32_t tmem_base = *tmem_ptr;
+    // PDL: the prologue above overlapped the previous kernel's tail; let the next kernel start its
+    // own prologue, then wait for our producer kernel's results before touching them
+    griddep_launch_dependents();
+    griddep_wait();
     const int n_items = p.sc.n_items;
 
     if (warp < 4) {
@@ -294,9 +298,7 @@ cudaError_t launch_g1_t(const Params& p, cudaStream_t st, int64_t* nl)
     auto kern = tc_gemm1<D, T, LS, 2>;
     if ((e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM)) != cudaSuccess) return e;
     const int grid = std::min(p.sc.n_items, num_sms());
-    kern<<<grid, C::THREADS, C::SMEM, st>>>(tq, tk, p);
-    ++*nl;
-    return cudaGetLastError();
+    return launch_pdl(kern, dim3(grid), dim3(C::THREADS), C::SMEM, st, nl, tq, tk, p);
 }
 
 cudaError_t launch_gemm1(const Params& p, bool ls, cudaStream_t st, int64_t* nl)

@@ -95,6 +95,10 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
     __syncthreads();
     tc_fence_after();
     const uint32_t tmem_base = *tmem_ptr;
+    // PDL: the prologue above overlapped the previous kernel's tail; let the next kernel start its
+    // own prologue, then wait for our producer kernel's results before touching them
+    griddep_launch_dependents();
+    griddep_wait();
     const uint32_t tmem_o = tmem_base;              // NO x D columns
     const uint32_t tmem_a = tmem_base + C::NO * D;  // NA x T/2 columns
     const int n_items = p.sc.n_items;
@@ -338,9 +342,7 @@ cudaError_t launch_g2_t(const Params& p, cudaStream_t st, int64_t* nl)
     auto kern = tc_gemm2<D, T, GS>;
     if ((e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM)) != cudaSuccess) return e;
     const int grid = std::min(p.sc.n_items, num_sms());
-    kern<<<grid, C::THREADS, C::SMEM, st>>>(tv, p);
-    ++*nl;
-    return cudaGetLastError();
+    return launch_pdl(kern, dim3(grid), dim3(C::THREADS), C::SMEM, st, nl, tv, p);
 }
 
 cudaError_t launch_gemm2(const Params& p, bool gs, cudaStream_t st, int64_t* nl)

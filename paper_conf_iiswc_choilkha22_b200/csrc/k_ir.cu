@@ -8,14 +8,17 @@
 // issued at once: up to kReg tiles are held in registers (one round trip to memory, then r' from
 // registers); longer rows stream the rest in batches.  It cannot be fused into GEMM1 (m and d need
 // every tile of the row); the paper keeps it standalone and so does this design.
+#include "ptx.cuh"
 #include "sr_internal.h"
 
 namespace sr {
 
 constexpr int kReg = 16;
 
-__global__ void __launch_bounds__(256) ir_kernel(Params p)
+__global__ void __launch_bounds__(256) ir_kernel(const Params p)
 {
+    ptx::griddep_launch_dependents();  // PDL: GEMM2's prologue may start now ...
+    ptx::griddep_wait();               // ... and GEMM1's m', d' must be complete before we read them
     const int64_t row = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const int64_t n_rows = (int64_t)p.B * p.H * p.S;
     if (row >= n_rows) return;
@@ -99,9 +102,7 @@ cudaError_t launch_ir(const Params& p, cudaStream_t st, int64_t* nlaunch)
     const int64_t n_rows = (int64_t)p.B * p.H * p.S;
     const int threads = 256;
     const int64_t blocks = (n_rows + threads - 1) / threads;
-    ir_kernel<<<(unsigned)blocks, threads, 0, st>>>(p);
-    ++*nlaunch;
-    return cudaGetLastError();
+    return launch_pdl(ir_kernel, dim3((unsigned)blocks), dim3(threads), 0, st, nlaunch, p);
 }
 
 }  // namespace sr

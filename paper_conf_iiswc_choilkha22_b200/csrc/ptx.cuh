@@ -92,6 +92,15 @@ __device__ __forceinline__ float lds_f32(uint32_t saddr)
     return v;
 }
 
+// ------------------------------------------------------------------ programmatic dependent launch
+// launch_dependents: let the next kernel in the stream (launched with the PDL attribute) start its
+// prologue; wait: block until every grid this one depends on has completed and flushed memory.
+__device__ __forceinline__ void griddep_launch_dependents()
+{
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+__device__ __forceinline__ void griddep_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+
 // ------------------------------------------------------------------ named barriers / fences
 __device__ __forceinline__ void named_bar_sync(int id, int nthreads)
 {

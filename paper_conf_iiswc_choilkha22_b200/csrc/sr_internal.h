@@ -13,6 +13,8 @@
 
 #include <cuda_runtime.h>
 
+#include <utility>
+
 namespace sr {
 
 constexpr int kRowBlock = 128;  // M of every tcgen05 tile
@@ -77,6 +79,28 @@ __host__ __device__ inline bool elem_kept(const Params& p, int kvl, int i, int j
         if (!(dd <= p.win_half || i < p.n_global || j < p.n_global)) return false;
     }
     return true;
+}
+
+// Launch with Programmatic Dependent Launch enabled: the kernel may begin (prologue) while the
+// previous kernel in the stream drains; it must call griddepcontrol.wait before reading results of
+// that kernel (all sr kernels do).
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
+                              int64_t* nlaunch, Args&&... args)
+{
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    cudaError_t e = cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
+    ++*nlaunch;
+    return e != cudaSuccess ? e : cudaGetLastError();
 }
 
 // ---- launchers (return cudaError_t of the launch)
