@@ -106,8 +106,9 @@ def flops(cfg, stored):
 # ----------------------------------------------------------------------------- GPU arm
 
 class Layer:
-    def __init__(self, cfg, device, seed_base, sr, torch):
+    def __init__(self, cfg, device, seed_base, sr, torch, tile_n=0):
         self.cfg, self.sr, self.torch = cfg, sr, torch
+        self.tile_n = tile_n
         t = W.make_qkv(cfg.B, cfg.H, cfg.S, cfg.D, cfg.dtype, seed_base=seed_base)
         self.host = {}
         self.dev = {}
@@ -134,16 +135,17 @@ class Layer:
         for fused in (True, False):
             if cfg.dtype == "f32" and not fused:
                 continue
-            info = sr.workspace_info(self.mask, cfg.B, cfg.H, cfg.S, cfg.D, in_dt, causal=cfg.causal, fused=fused)
+            info = sr.workspace_info(self.mask, cfg.B, cfg.H, cfg.S, cfg.D, in_dt, causal=cfg.causal, fused=fused,
+                                     tile_n=tile_n)
             self.ws[fused] = torch.empty(info["total_bytes"], dtype=torch.uint8, device=device)
             self.T = info["tile_n"]
-        self.n_tiles, self.stored = sr.schedule_stats(self.mask, cfg.B, cfg.H, cfg.S, causal=cfg.causal)
+        self.n_tiles, self.stored = sr.schedule_stats(self.mask, cfg.B, cfg.H, cfg.S, causal=cfg.causal, tile_n=tile_n)
 
     def run(self, fused=True, stages=0, q=None, k=None, v=None):
         d = self.dev
         return self.sr.call(self.mask, q if q is not None else d["q"], k if k is not None else d["k"],
                             v if v is not None else d["v"], out=self.out, fused=fused, stages=stages,
-                            workspace=self.ws[fused], **self.kw)
+                            workspace=self.ws[fused], tile_n=self.tile_n, **self.kw)
 
 
 def timed(torch, fn, steps, warmup, flush, per_step_pre=None):
@@ -203,7 +205,7 @@ def gpu_arm(args, rank, world, local_rank):
     cfg = W.config(args.config)
     flush = None if args.no_flush else (torch.empty(FLUSH_BYTES, dtype=torch.uint8, device=device),
                                         torch.ones(FLUSH_BYTES // 4, dtype=torch.float32, device=device))
-    L = Layer(cfg, device, seed_base=cfg.idx + 1000 * rank, sr=sr, torch=torch)
+    L = Layer(cfg, device, seed_base=cfg.idx + 1000 * rank, sr=sr, torch=torch, tile_n=args.tile_n)
     K, Wm = args.steps, args.warmup
 
     # ---- headline: recomposed layer, inputs resident in HBM
@@ -406,6 +408,7 @@ def main():
     ap.add_argument("--config", type=int, default=2, help="BASELINE.json config index (1-5); default configs[1]")
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--no-flush", action="store_true")
+    ap.add_argument("--tile-n", type=int, default=0, help="LS sub-vector width T (0 = library default)")
     ap.add_argument("--no-all-configs", dest="all_configs", action="store_false")
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
     args = ap.parse_args()

@@ -95,7 +95,8 @@ typedef struct {
     size_t workspace_bytes;
     void* stream;            /* cudaStream_t; NULL = legacy default stream */
     int32_t tile_n;          /* T = LS sub-vector width = GEMM1 output-tile width:
-                                0 = default (128 dense 16-bit, 64 fp32 and sparse), or 64 / 128 */
+                                0 = default (128 on the tensor cores; 64 for block-sparse
+                                layouts and the fp32 path), or 64 / 128 */
     int32_t flags;           /* 0 = run the whole chain.  Otherwise an OR of SR_RUN_* stage bits:
                                 only those kernels are launched, consuming the intermediates an
                                 earlier call with the same arguments left in the workspace (used by

@@ -169,7 +169,9 @@ sr_status build_sched(const Request& r, HostSched& hs)
 int default_T(sr_entry e, int in_dtype)
 {
     if (in_dtype == SR_F32) return 64;
-    return e == SR_E_DENSE ? 128 : 64;
+    // T = the GEMM1 output-tile width: 128 on the tensor cores; block-sparse
+    // layouts fix the sub-vector to the 64-key block (two of them share one 128-key MMA tile)
+    return e == SR_E_BLOCKSPARSE ? 64 : 128;
 }
 
 sr_status check_request(sr_entry e, int B, int H, int S, int D, int in_dtype,

@@ -4,42 +4,53 @@
 // fused as element-wise layers, L169).  LS=false builds the unfused baseline's GEMM1, which writes
 // the scaled, masked score tile S instead (L171).
 //
-// Per 128-row x T-key tile, fp32 accumulator in TMEM:
+// Per 128-row x T-key sub-tile (the LS sub-vector, T = 64 or 128), fp32 accumulator in TMEM:
 //   m'  = max_j x_j                    (x = Q K^T * scale, masked to -inf)
 //   X'  = e^{x - m'}  -> fp16 tile, written to HBM once (the only attention-matrix write)
 //   d'  = sum_j X'_j                   (fp32)
 // m', d' go to the workspace as fp32 [slot][128 rows].
 //
+// Macro tiles.  The tensor core always computes 128 x MW (MW = 128) score tiles: with T = 64 two
+// consecutive sub-tiles of the item's key list (any two key blocks, stacked in one K stage) share
+// one N = 128 MMA and one epilogue pass, each keeping its own mask, statistics, validity and slot
+// (consecutive list entries are adjacent slots, so the pair's X' is contiguous in HBM).
+//
 // Warp roles (persistent CTA per SM, 384 threads):
-//   warp 0      TMA producer: Q tile per item (double-buffered), K tiles (NK-stage ring)
-//   warp 1      MMA issuer: tcgen05.mma kind::f16, D/16 MMAs of 128 x T x 16 per tile into one
-//               of NACC TMEM accumulators; publishes a per-tile header (slot, rows, key tile,
-//               half-valid bits, kv_len) next to the accumulator -- acc_full completes when both
-//               the header arrive and the MMA commit have landed
+//   warp 0      TMA producer: Q tile per item, K blocks of each macro tile (NK-stage ring)
+//   warp 1      MMA issuer: D/16 tcgen05.mma kind::f16 of 128 x MW x 16 per macro tile into one of
+//               NACC TMEM accumulators; publishes a header (slot, rows, key tiles, half-valid bits,
+//               kv_len) next to the accumulator -- acc_full completes when both the header arrive and
+//               the MMA commit have landed
 //   warp 2      TMEM allocator (512 columns)
-//   warps 4-11  two epilogue warpgroups taking alternate tiles: one tcgen05.ld of the whole row,
-//               accumulator released immediately, mask (interval bits), max, ex2, sum, fp16 pack,
-//               st.shared into a swizzled staging tile, one cp.async.bulk store per tile
+//   warps 4-11  two epilogue warpgroups taking alternate macro tiles: one tcgen05.ld of the row's
+//               MW scores, accumulator released at once, interval-bitmask mask, max, FFMA2 + ex2,
+//               FADD2 sums, fp16 pack, st.shared into a swizzled staging tile; every warp bulk-stores
+//               its own 32 rows (no warpgroup barrier)
 #include "tc_common.cuh"
 
 namespace sr {
 
 using namespace ptx;
 
-struct G1Hdr {  // per-accumulator tile header, written by the MMA warp
-    int32_t slot_lo, slot_hi, i0, kvl, w, flags, pad0, pad1;
+constexpr int kMW = 128;  // macro tile width (MMA N of GEMM1, MMA K per step of GEMM2)
+
+struct G1Hdr {  // per-accumulator macro-tile header, written by the MMA warp
+    int32_t slot_lo, slot_hi, i0, kvl, w0, w1, flags, pad;
 };
 enum : int { HDR_TILE = 1, HDR_END = 2 };
 
-template <int D, int T, int XPWMAX = 2>
+template <int D, int T>
 struct G1 {
-    static constexpr int QB = kRowBlock * D * 2;  // Q tile bytes
-    static constexpr int KB = T * D * 2;          // K tile bytes
-    static constexpr int XB = kRowBlock * T * 2;  // X'/S tile bytes
-    static constexpr int NQ = 2;
-    static constexpr int NACC = 512 / T;  // TMEM accumulators (4 for T=128, 8 for T=64)
-    // staging buffers per epilogue warpgroup: 2 when shared memory allows, else 1
-    static constexpr int XPW = (XPWMAX >= 2 && NQ * QB + 2 * KB + 4 * XB + 4096 <= kSmemMax) ? 2 : 1;
+    static constexpr int NSUB = kMW / T;           // sub-tiles per macro tile
+    static constexpr int QB = kRowBlock * D * 2;   // Q tile bytes
+    static constexpr int KB = kMW * D * 2;         // K stage bytes (MW keys)
+    static constexpr int XB = kRowBlock * kMW * 2;  // staging tile bytes (macro tile)
+    static constexpr int XS = kRowBlock * T * 2;   // X' slot bytes (sub-tile)
+    static constexpr int NACC = 512 / kMW;         // TMEM accumulators
+    // staging buffers per epilogue warpgroup (2 if at all possible: the X' store stream is the
+    // bottleneck), then Q double-buffered if shared memory still allows
+    static constexpr int XPW = (QB + 2 * KB + 4 * XB + 4096 <= kSmemMax) ? 2 : 1;
+    static constexpr int NQ = (2 * QB + 2 * KB + 2 * XPW * XB + 4096 <= kSmemMax) ? 2 : 1;
     static constexpr int NK_ = (kSmemMax - 4096 - NQ * QB - 2 * XPW * XB) / KB;
     static constexpr int NK = NK_ > 4 ? 4 : NK_;
     static_assert(NK >= 2, "smem budget");
@@ -55,11 +66,12 @@ struct G1 {
     static constexpr int THREADS = 384;
 };
 
-template <int D, int T, bool LS, int XPWMAX>
+template <int D, int T, bool LS>
 __global__ void __launch_bounds__(384, 1)
     tc_gemm1(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmK, const Params p)
 {
-    using C = G1<D, T, XPWMAX>;
+    using C = G1<D, T>;
+    constexpr int NSUB = C::NSUB;
     extern __shared__ uint8_t smem_raw[];
     uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
     uint64_t* bars = (uint64_t*)(smem + C::OFF_BAR);
@@ -108,21 +120,29 @@ __global__ void __launch_bounds__(384, 1)
                 for (int h = 0; h < D / 64; ++h)
                     tma_load_2d(smem + C::OFF_Q + qi * C::QB + h * (kRowBlock * 128), &tmQ, h * 64, row0, &q_full[qi]);
                 if (++qi == C::NQ) { qi = 0; qph ^= 1; }
-                int w_next = __ldg(p.sc.tinfo + I.t0);
-                for (int t = I.t0; t < I.t1; ++t) {
-                    const int w = w_next;
-                    if (t + 1 < I.t1) w_next = __ldg(p.sc.tinfo + t + 1);
+                int wn[NSUB];  // schedule words of the next macro tile, prefetched one step ahead
+#pragma unroll
+                for (int s = 0; s < NSUB; ++s) wn[s] = I.t0 + s < I.t1 ? __ldg(p.sc.tinfo + I.t0 + s) : 0;
+                for (int t = I.t0; t < I.t1; t += NSUB) {
+                    const int nsub = min(NSUB, I.t1 - t);
+                    int w[NSUB];
+#pragma unroll
+                    for (int s = 0; s < NSUB; ++s) {
+                        w[s] = wn[s];
+                        wn[s] = t + NSUB + s < I.t1 ? __ldg(p.sc.tinfo + t + NSUB + s) : 0;
+                    }
                     mbar_wait(&k_empty[ks], kph ^ 1);
-                    mbar_arrive_expect_tx(&k_full[ks], C::KB);
-                    for (int h = 0; h < D / 64; ++h)
-                        tma_load_2d(smem + C::OFF_K + ks * C::KB + h * (T * 128), &tmK, h * 64,
-                                    I.g * p.S + tinfo_kt(w) * T, &k_full[ks]);
+                    mbar_arrive_expect_tx(&k_full[ks], nsub * T * D * 2);
+                    for (int s = 0; s < nsub; ++s)
+                        for (int h = 0; h < D / 64; ++h)
+                            tma_load_2d(smem + C::OFF_K + ks * C::KB + h * (kMW * 128) + s * (T * 128), &tmK, h * 64,
+                                        I.g * p.S + tinfo_kt(w[s]) * T, &k_full[ks]);
                     if (++ks == C::NK) { ks = 0; kph ^= 1; }
                 }
             }
         } else if (warp == 1 && lane == 0) {
             // -------------------------------------------------------------- MMA issuer
-            const uint32_t idesc = idesc_f16(p.in_dtype == DT_BF16 ? 1 : 0, kRowBlock, T, 0, 0);
+            const uint32_t idesc = idesc_f16(p.in_dtype == DT_BF16 ? 1 : 0, kRowBlock, kMW, 0, 0);
             int qi = 0, ks = 0, n = 0;
             uint32_t qph = 0, kph = 0;
             for (int it = blockIdx.x; it < n_items; it += gridDim.x) {
@@ -132,25 +152,26 @@ __global__ void __launch_bounds__(384, 1)
                 mbar_wait(&q_full[qi], qph);
                 tc_fence_after();
                 const uint32_t q_addr = smem_u32(smem + C::OFF_Q + qi * C::QB);
-                int w_next = __ldg(p.sc.tinfo + I.t0);
-                for (int t = I.t0; t < I.t1; ++t, ++n) {
-                    const int w = w_next;
-                    if (t + 1 < I.t1) w_next = __ldg(p.sc.tinfo + t + 1);
+                int wn0 = __ldg(p.sc.tinfo + I.t0), wn1 = (NSUB > 1 && I.t0 + 1 < I.t1) ? __ldg(p.sc.tinfo + I.t0 + 1) : -1;
+                for (int t = I.t0; t < I.t1; t += NSUB, ++n) {
+                    const int w0 = wn0, w1 = NSUB > 1 ? wn1 : -1;
+                    if (t + NSUB < I.t1) wn0 = __ldg(p.sc.tinfo + t + NSUB);  // prefetch the next macro tile
+                    wn1 = (NSUB > 1 && t + NSUB + 1 < I.t1) ? __ldg(p.sc.tinfo + t + NSUB + 1) : -1;
                     const int ab = n % C::NACC;
                     mbar_wait(&acc_empty[ab], ((n / C::NACC) & 1) ^ 1);
                     const int64_t slot = I.slot0 + t;
-                    hdr[ab] = G1Hdr{(int32_t)(slot & 0xffffffff), (int32_t)(slot >> 32), I.rb * kRowBlock, kvl, w,
-                                    HDR_TILE, I.g, 0};
+                    hdr[ab] = G1Hdr{(int32_t)(slot & 0xffffffff), (int32_t)(slot >> 32), I.rb * kRowBlock, kvl, w0, w1,
+                                    HDR_TILE, 0};
                     mbar_arrive(&acc_full[ab]);  // header published (arrival 1 of 2)
                     mbar_wait(&k_full[ks], kph);
                     tc_fence_after();
                     const uint32_t k_addr = smem_u32(smem + C::OFF_K + ks * C::KB);
-                    const uint32_t d_tmem = tmem_base + ab * T;
+                    const uint32_t d_tmem = tmem_base + ab * kMW;
 #pragma unroll
                     for (int kk = 0; kk < D / 16; ++kk) {
                         const uint32_t h = kk / 4, wk = kk % 4;
                         const uint64_t ad = smem_desc_sw128(q_addr + h * (kRowBlock * 128) + wk * 32, 16, 1024);
-                        const uint64_t bd = smem_desc_sw128(k_addr + h * (T * 128) + wk * 32, 16, 1024);
+                        const uint64_t bd = smem_desc_sw128(k_addr + h * (kMW * 128) + wk * 32, 16, 1024);
                         mma_ss(d_tmem, ad, bd, idesc, kk > 0 ? 1u : 0u);
                     }
                     mma_commit(&k_empty[ks]);
@@ -171,29 +192,35 @@ __global__ void __launch_bounds__(384, 1)
     } else {
         reg_alloc<224>();
         // ------------------------------------------------------------------ epilogue warpgroups
-        const int e = (warp - 4) / 4;          // warpgroup 0 / 1: even / odd tiles
+        const int e = (warp - 4) / 4;          // warpgroup 0 / 1: even / odd macro tiles
         const int r = (warp % 4) * 32 + lane;  // tile row == TMEM lane
         const int myhalf = r / kHalf;
         const uint32_t lane_off = (uint32_t)((warp % 4) * 32) << 16;
-        const bool issuer = (threadIdx.x % 128) == 0;
         const float sl2 = p.scale_log2;
-        int k = 0;  // tiles processed by this warpgroup
+        const int wrow0 = (warp % 4) * 32;  // this warp's 32 rows: a contiguous 4-KB run per column half
+        int k = 0;                          // macro tiles processed by this warpgroup
         for (int n = e;; n += 2, ++k) {
             const int buf = n % C::NACC;
             mbar_wait(&acc_full[buf], (uint32_t)(n / C::NACC) & 1);
             tc_fence_after();
             const G1Hdr H = hdr[buf];
             if (H.flags & HDR_END) break;
-            const int kt = tinfo_kt(H.w), hv = tinfo_half(H.w);
-            const bool valid = (hv >> myhalf) & 1;
-            const int c0 = kt * T, i = H.i0 + r;
-            const int64_t slot = ((int64_t)H.slot_hi << 32) | (uint32_t)H.slot_lo;
-            // one TMEM read of the row's T fp32 scores; the accumulator goes straight back to the MMA
-            uint32_t xr[T];
-            if (valid) {
+            const int wsub[2] = {H.w0, H.w1};
+            bool vs[NSUB];  // this row's 64-row half is valid in sub-tile s
+            bool any = false;
 #pragma unroll
-                for (int c = 0; c < T / 32; ++c)
-                    tmem_ld32(tmem_base + lane_off + buf * T + c * 32, *reinterpret_cast<uint32_t(*)[32]>(&xr[c * 32]));
+            for (int s = 0; s < NSUB; ++s) {
+                vs[s] = wsub[s] != -1 && ((tinfo_half(wsub[s]) >> myhalf) & 1);
+                any |= vs[s];
+            }
+            const int i = H.i0 + r;
+            const int64_t slot = ((int64_t)H.slot_hi << 32) | (uint32_t)H.slot_lo;
+            // one TMEM read of the row's MW fp32 scores; the accumulator goes straight back to the MMA
+            uint32_t xr[kMW];
+            if (any) {
+#pragma unroll
+                for (int c = 0; c < kMW / 32; ++c)
+                    tmem_ld32(tmem_base + lane_off + buf * kMW + c * 32, *reinterpret_cast<uint32_t(*)[32]>(&xr[c * 32]));
                 tmem_wait_ld();
             }
             tc_fence_before();
@@ -201,77 +228,105 @@ __global__ void __launch_bounds__(384, 1)
             if (lane == 0) mbar_arrive(&acc_empty[buf]);
             uint8_t* stage = smem + C::OFF_X + (e * C::XPW + (k % C::XPW)) * C::XB;
             const uint32_t stage_s = smem_u32(stage);
-            // staging buffer free: this warpgroup's store from it (XPW tiles ago) has read it
-            if (issuer) {
+            // Each warp stages and stores its own 32 rows (no warpgroup barrier): its slice of this
+            // staging buffer is free once the warp's own store from it (XPW macro tiles ago) has read
+            // it.  Every warp commits one bulk group per macro tile (possibly empty) so the count holds.
+            if (lane == 0) {
                 if (C::XPW == 2) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
                 else bulk_wait_read0();
             }
-            named_bar_sync(1 + e, 128);
-            float mx = -INFINITY, dsum = 0.f;
-            if (valid) {
-                // mask layer: kept keys of this row form <= 2 intervals
-                const RowMask rm = row_mask(p, i, H.kvl);
+            __syncwarp();
+            float mx[NSUB], dsum[NSUB];
+            const RowMask rm = row_mask(p, i, H.kvl);
 #pragma unroll
-                for (int c = 0; c < T / 32; ++c) {
-                    const uint32_t bits = mask_bits32(rm, c0 + c * 32);
-                    if (bits != 0xffffffffu) {
+            for (int s = 0; s < NSUB; ++s) {
+                mx[s] = -INFINITY;
+                dsum[s] = 0.f;
+                if (!vs[s]) continue;
+                uint32_t* x = xr + s * T;
+                const int c0 = tinfo_kt(wsub[s]) * T;
+                // mask layer: kept keys of this row form <= 2 intervals; interior
+                // sub-tiles (every key kept) skip the bit construction entirely
+                const bool full = c0 >= rm.lo && c0 + T - 1 <= rm.hi &&
+                                  ((c0 >= rm.blo && c0 + T - 1 <= rm.bhi) || c0 + T - 1 < rm.gc);
+                if (!full) {
+#pragma unroll
+                    for (int c = 0; c < T / 32; ++c) {
+                        const uint32_t bits = mask_bits32(rm, c0 + c * 32);
 #pragma unroll
                         for (int u = 0; u < 32; ++u)
-                            if (!((bits >> u) & 1u)) xr[c * 32 + u] = 0xff800000u;  // -inf
+                            if (!((bits >> u) & 1u)) x[c * 32 + u] = 0xff800000u;  // -inf
                     }
                 }
-                float neg = 0.f;
                 if (LS) {
                     float m8[8];
 #pragma unroll
-                    for (int a = 0; a < 8; ++a) m8[a] = __uint_as_float(xr[a]);
+                    for (int a = 0; a < 8; ++a) m8[a] = __uint_as_float(x[a]);
 #pragma unroll
-                    for (int u = 8; u < T; ++u) m8[u & 7] = fmaxf(m8[u & 7], __uint_as_float(xr[u]));
-                    mx = fmaxf(fmaxf(fmaxf(m8[0], m8[1]), fmaxf(m8[2], m8[3])),
-                               fmaxf(fmaxf(m8[4], m8[5]), fmaxf(m8[6], m8[7])));
-                    // X' = e^{x - m'}: base 2 with log2(e) folded into the scale, one FFMA + one MUFU
-                    neg = (mx == -INFINITY) ? 0.f : -mx * sl2;
+                    for (int u = 8; u < T; ++u) m8[u & 7] = fmaxf(m8[u & 7], __uint_as_float(x[u]));
+                    mx[s] = fmaxf(fmaxf(fmaxf(m8[0], m8[1]), fmaxf(m8[2], m8[3])),
+                                  fmaxf(fmaxf(m8[4], m8[5]), fmaxf(m8[6], m8[7])));
+                    // X' = e^{x - m'}: base 2 with log2(e) folded into the scale -- one FFMA2 per pair,
+                    // then one MUFU.EX2 per element (in place)
+                    const float neg = (mx[s] == -INFINITY) ? 0.f : -mx[s] * sl2;
+#pragma unroll
+                    for (int u = 0; u < T; u += 2) {
+                        float t0, t1;
+                        ffma2(t0, t1, __uint_as_float(x[u]), __uint_as_float(x[u + 1]), sl2, neg);
+                        x[u] = __float_as_uint(ex2(t0));
+                        x[u + 1] = __float_as_uint(ex2(t1));
+                    }
+                    // d' = sum X' (fp32, FADD2 into 4 independent pair accumulators)
+                    float sa[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+#pragma unroll
+                    for (int u = 0; u < T; u += 2)
+                        fadd2_acc(sa[(u >> 1) & 3], sa[4 + ((u >> 1) & 3)], __uint_as_float(x[u]), __uint_as_float(x[u + 1]));
+                    dsum[s] = ((sa[0] + sa[4]) + (sa[1] + sa[5])) + ((sa[2] + sa[6]) + (sa[3] + sa[7]));
+                } else {  // unfused baseline: the scaled, masked score
+#pragma unroll
+                    for (int u = 0; u < T; u += 2) {
+                        float t0, t1;
+                        fmul2(t0, t1, __uint_as_float(x[u]), __uint_as_float(x[u + 1]), p.scale);
+                        x[u] = __float_as_uint(t0);
+                        x[u + 1] = __float_as_uint(t1);
+                    }
                 }
-                float s4[4] = {0.f, 0.f, 0.f, 0.f};
 #pragma unroll
-                for (int q4 = 0; q4 < T / 8; ++q4) {  // 8 keys -> one 16-B chunk of the tile
+                for (int q4 = 0; q4 < T / 8; ++q4) {  // 8 keys -> one 16-B chunk of the fp16 tile
                     uint32_t w4[4];
 #pragma unroll
-                    for (int u = 0; u < 4; ++u) {
-                        const float x0 = __uint_as_float(xr[q4 * 8 + 2 * u]);
-                        const float x1 = __uint_as_float(xr[q4 * 8 + 2 * u + 1]);
-                        if (LS) {
-                            const float y0 = ex2(fmaf(x0, sl2, neg)), y1 = ex2(fmaf(x1, sl2, neg));
-                            s4[u] += y0 + y1;
-                            w4[u] = pack_f16(y0, y1);
-                        } else {  // unfused baseline: the scaled, masked score
-                            w4[u] = pack_f16(x0 * p.scale, x1 * p.scale);
-                        }
-                    }
-                    sts128(stage_s + tile_chunk_off(r, q4), w4[0], w4[1], w4[2], w4[3]);
+                    for (int u = 0; u < 4; ++u)
+                        w4[u] = pack_f16(__uint_as_float(x[q4 * 8 + 2 * u]), __uint_as_float(x[q4 * 8 + 2 * u + 1]));
+                    sts128(stage_s + tile_chunk_off(r, s * (T / 8) + q4), w4[0], w4[1], w4[2], w4[3]);
                 }
-                dsum = (s4[0] + s4[1]) + (s4[2] + s4[3]);
             }
+            // the warp's 32 rows of each valid sub-tile go to HBM: one 4-KB bulk copy per 64 columns
+            bool wv[NSUB];
+#pragma unroll
+            for (int s = 0; s < NSUB; ++s) wv[s] = __shfl_sync(0xffffffffu, vs[s] ? 1 : 0, 0) != 0;
             fence_proxy_async_smem();
-            named_bar_sync(1 + e, 128);
-            if (issuer) {  // the tile's valid 64-row halves go to HBM in one or two bulk copies
-                uint8_t* dst = (uint8_t*)p.xprime + slot * (int64_t)C::XB;
-                for (int ch = 0; ch < T / 64; ++ch) {
-                    const int o = ch * (kRowBlock * 128);
-                    if (hv == 3) bulk_store(dst + o, stage + o, kRowBlock * 128);
-                    else {
-                        const int o2 = o + (hv == 2 ? kHalf * 128 : 0);
-                        bulk_store(dst + o2, stage + o2, kHalf * 128);
-                    }
+            __syncwarp();
+            if (lane == 0) {
+#pragma unroll
+                for (int s = 0; s < NSUB; ++s) {
+                    if (!wv[s]) continue;
+                    uint8_t* dst = (uint8_t*)p.xprime + (slot + s) * (int64_t)C::XS;
+                    for (int ch = 0; ch < T / 64; ++ch)
+                        bulk_store(dst + ch * (kRowBlock * 128) + wrow0 * 128,
+                                   stage + (s * (T / 64) + ch) * (kRowBlock * 128) + wrow0 * 128, 32 * 128);
                 }
                 bulk_commit();
             }
-            if (LS && valid) {
-                p.mprime[slot * kRowBlock + r] = mx * p.scale;  // m' in natural-log units
-                p.dprime[slot * kRowBlock + r] = dsum;
+            if (LS) {
+#pragma unroll
+                for (int s = 0; s < NSUB; ++s)
+                    if (vs[s]) {
+                        p.mprime[(slot + s) * kRowBlock + r] = mx[s] * p.scale;  // m' in natural-log units
+                        p.dprime[(slot + s) * kRowBlock + r] = dsum[s];
+                    }
             }
         }
-        if (issuer) bulk_wait0();
+        if (lane == 0) bulk_wait0();
     }
     tc_fence_before();
     __syncthreads();
@@ -289,13 +344,13 @@ int num_sms();
 template <int D, int T, bool LS>
 cudaError_t launch_g1_t(const Params& p, cudaStream_t st, int64_t* nl)
 {
-    using C = G1<D, T, 2>;
+    using C = G1<D, T>;
     CUtensorMap tq, tk;
     const int64_t rows = (int64_t)p.B * p.H * p.S;
     cudaError_t e;
     if ((e = make_tmap_2d(&tq, p.q, rows, D, kRowBlock, p.in_dtype)) != cudaSuccess) return e;
     if ((e = make_tmap_2d(&tk, p.k, rows, D, T, p.in_dtype)) != cudaSuccess) return e;
-    auto kern = tc_gemm1<D, T, LS, 2>;
+    auto kern = tc_gemm1<D, T, LS>;
     if ((e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM)) != cudaSuccess) return e;
     const int grid = std::min(p.sc.n_items, num_sms());
     return launch_pdl(kern, dim3(grid), dim3(C::THREADS), C::SMEM, st, nl, tq, tk, p);

@@ -4,22 +4,22 @@
 // the GS kernel can easily be fused with its subsequent MatMul kernel").  GS=false builds the
 // unfused baseline's GEMM2 on the softmax output P.
 //
-// Per item (head, 128-row block) and each of its key tiles:
-//   Y_tile = X'_tile (fp16) * r'_row (fp32), rounded once to the MMA dtype   (GS, in registers)
-//   O     += Y_tile V_tile   (tcgen05.mma kind::f16, A from TMEM, B = V from smem, fp32 in TMEM)
+// Per item (head, 128-row block) and each of its key sub-tiles (width T):
+//   Y_sub = X'_sub (fp16) * r'_row,sub (fp32), rounded once to the MMA dtype   (GS, in registers)
+//   O    += Y_sub V_sub   (tcgen05.mma kind::f16, A from TMEM, B = V from smem, fp32 in TMEM)
+// Macro tiles: as in GEMM1, MW = 128 keys per step -- with T = 64 two consecutive sub-tiles of the
+// item (any two key blocks) are stacked along the MMA K dimension, each scaled by its own r'.
 //
 // Warp roles (persistent CTA per SM, 384 threads):
-//   warp 0      X' producer: X' tile (1-D bulk copy of its valid 64-row halves; the tile is already
-//               in the UMMA SW128 K-major layout) + the tile's 128 r' values + a stage header, into
-//               an NX-deep ring; ends with an END header.  The X' ring is only read by the GS warps,
-//               so a stage is recycled as soon as they have written it into TMEM (not after the MMA)
-//               -- X' (the dominant HBM stream) can run NX tiles ahead of the tensor core.
-//   warp 3      V producer: V tile (TMA, SW128, used as the MN-major B operand) into an NV-deep ring
-//               (V is mostly L2-resident: reused by every row block of a head)
-//   warp 1      MMA issuer: T/16 MMAs of 128 x D x 16 per tile into one of two TMEM O accumulators;
-//               walks the item list itself and publishes each item's output rows (or EMPTY / END)
-//               to the epilogue through an O header
-//   warp 2      TMEM allocator (512 columns: 2 x D for O, NA x T/2 for the A operand ring)
+//   warp 0      X' producer: the macro tile's X' sub-tiles (1-D bulk copies of their valid 64-row
+//               halves; the tiles are already in the UMMA SW128 K-major layout and adjacent in HBM) +
+//               their r' + a stage header, into an NX-deep ring, then an END header.  The ring is only
+//               read by the GS warps, so a stage is recycled once they have written it into TMEM.
+//   warp 3      V producer: the macro tile's V blocks (TMA, SW128, MN-major B operand), NV-deep ring
+//   warp 1      MMA issuer: per macro tile (nsub*T)/16 MMAs of 128 x D x 16 into one of two TMEM
+//               O accumulators; walks the item list itself and publishes each item's output rows
+//               (or EMPTY / END) to the epilogue through an O header
+//   warp 2      TMEM allocator (512 columns: 2 x D for O, NA x MW/2 for the A operand ring)
 //   warps 4-7   GS transform: smem X' row -> fp32 x r' -> dtype -> tcgen05.st into TMEM (A operand)
 //   warps 8-11  epilogue: tcgen05.ld of O rows -> out dtype -> global
 #include "tc_common.cuh"
@@ -28,24 +28,28 @@ namespace sr {
 
 using namespace ptx;
 
+constexpr int kMW2 = 128;  // macro tile width (keys per MMA step)
+
 enum : int { SH_TILE = 1, SH_END = 2, SH_EMPTY = 4 };
 struct G2Hdr {  // X'-stage / O-buffer header
-    int32_t flags, hv, orow_lo, orow_hi;
+    int32_t flags, hv0, hv1, nsub, orow_lo, orow_hi, pad0, pad1;
 };
 
 template <int D, int T>
 struct G2 {
-    static constexpr int XB = kRowBlock * T * 2;  // X' / P tile
-    static constexpr int RB = 1024;               // r' (512 B) + header, padded to keep 1 KB alignment
-    static constexpr int XSB = XB + RB;           // X' stage
-    static constexpr int VB = T * D * 2;          // V tile (V stage)
+    static constexpr int NSUB = kMW2 / T;
+    static constexpr int XS = kRowBlock * T * 2;     // X' slot (sub-tile)
+    static constexpr int XB = kRowBlock * kMW2 * 2;  // X' part of a stage (macro tile)
+    static constexpr int RB = 2048;                  // r' (NSUB x 512 B) + header, keeps 1 KB alignment
+    static constexpr int XSB = XB + RB;              // X' stage
+    static constexpr int VB = kMW2 * D * 2;          // V stage (macro tile)
     // split the smem budget: V stages from L2 need less depth than the HBM-bound X' stream
-    static constexpr int NV = (VB >= 32768) ? 2 : ((VB >= 16384) ? 3 : 4);
+    static constexpr int NV = (VB >= 32768) ? 2 : 3;
     static constexpr int NX_ = (kSmemMax - 3072 - NV * VB) / XSB;
     static constexpr int NX = NX_ > 8 ? 8 : NX_;
     static_assert(NX >= 2, "smem budget");
-    static constexpr int NO = 2;                          // O accumulators (D cols each)
-    static constexpr int NA_ = (512 - NO * D) / (T / 2);  // A operand buffers (T/2 cols each)
+    static constexpr int NO = 2;                             // O accumulators (D cols each)
+    static constexpr int NA_ = (512 - NO * D) / (kMW2 / 2);  // A operand buffers (MW/2 cols each)
     static constexpr int NA = NA_ > 8 ? 8 : NA_;
     static_assert(NA >= 2, "tmem budget");
     static constexpr int OFF_X = 0;
@@ -63,6 +67,7 @@ template <int D, int T, bool GS>
 __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUtensorMap tmV, const Params p)
 {
     using C = G2<D, T>;
+    constexpr int NSUB = C::NSUB;
     extern __shared__ uint8_t smem_raw[];
     uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
     uint64_t* bars = (uint64_t*)(smem + C::OFF_BAR);
@@ -77,7 +82,7 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
     G2Hdr* ohdr = (G2Hdr*)(smem + C::OFF_OHDR);
     uint32_t* tmem_ptr = (uint32_t*)(smem + C::OFF_TPTR);
     auto xstage = [&](int s) { return smem + C::OFF_X + s * C::XSB; };
-    auto xhdr = [&](int s) { return (G2Hdr*)(xstage(s) + C::XB + 512); };
+    auto xhdr = [&](int s) { return (G2Hdr*)(xstage(s) + C::XB + 1024); };
     auto vstage = [&](int s) { return smem + C::OFF_V + s * C::VB; };
 
     const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
@@ -100,7 +105,7 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
     griddep_launch_dependents();
     griddep_wait();
     const uint32_t tmem_o = tmem_base;              // NO x D columns
-    const uint32_t tmem_a = tmem_base + C::NO * D;  // NA x T/2 columns
+    const uint32_t tmem_a = tmem_base + C::NO * D;  // NA x MW/2 columns
     const int n_items = p.sc.n_items;
     const uint8_t* src = (const uint8_t*)(GS ? p.xprime : p.pbuf);
 
@@ -111,25 +116,34 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
             uint32_t sph = 0;
             for (int it = blockIdx.x; it < n_items; it += gridDim.x) {
                 const ItemInfo I = decode_item(p, it);
-                int w_next = I.t0 < I.t1 ? __ldg(p.sc.tinfo + I.t0) : 0;
-                for (int t = I.t0; t < I.t1; ++t) {
-                    const int w = w_next;
-                    if (t + 1 < I.t1) w_next = __ldg(p.sc.tinfo + t + 1);
-                    const int hv = tinfo_half(w);
-                    const uint32_t xbytes = (hv == 3 ? 2 : 1) * (T / 64) * (kHalf * 128);
+                int wn[2];  // schedule words of the next macro tile, prefetched one step ahead
+                for (int u = 0; u < NSUB; ++u) wn[u] = I.t0 + u < I.t1 ? __ldg(p.sc.tinfo + I.t0 + u) : 0;
+                for (int t = I.t0; t < I.t1; t += NSUB) {
+                    const int nsub = min(NSUB, I.t1 - t);
+                    int hv[2] = {tinfo_half(wn[0]), NSUB > 1 ? tinfo_half(wn[1]) : 0};
+                    for (int u = 0; u < NSUB; ++u) wn[u] = t + NSUB + u < I.t1 ? __ldg(p.sc.tinfo + t + NSUB + u) : 0;
+                    uint32_t bytes = GS ? nsub * kRowBlock * 4 : 0;
+                    for (int u = 0; u < nsub; ++u) bytes += (hv[u] == 3 ? 2 : 1) * (T / 64) * (kHalf * 128);
                     mbar_wait(&x_empty[s], sph ^ 1);
                     uint8_t* st = xstage(s);
-                    *xhdr(s) = G2Hdr{SH_TILE, hv, 0, 0};
-                    mbar_arrive_expect_tx(&x_full[s], xbytes + (GS ? kRowBlock * 4 : 0));
-                    const uint8_t* xs = src + (I.slot0 + t) * (int64_t)C::XB;
-                    if (hv == 3) bulk_load(st, xs, C::XB, &x_full[s]);
-                    else
-                        for (int ch = 0; ch < T / 64; ++ch) {
-                            const int o = ch * (kRowBlock * 128) + (hv == 2 ? kHalf * 128 : 0);
-                            bulk_load(st + o, xs + o, kHalf * 128, &x_full[s]);
-                        }
-                    if (GS)  // r' of the tile's 128 rows rides along with the tile
-                        bulk_load(st + C::XB, p.rprime + (I.slot0 + t) * kRowBlock, kRowBlock * 4, &x_full[s]);
+                    *xhdr(s) = G2Hdr{SH_TILE, hv[0], hv[1], nsub, 0, 0, 0, 0};
+                    mbar_arrive_expect_tx(&x_full[s], bytes);
+                    const uint8_t* xs = src + (I.slot0 + t) * (int64_t)C::XS;  // sub-tiles t, t+1 are adjacent
+                    if (hv[0] == 3 && (nsub == 1 || hv[1] == 3)) {
+                        bulk_load(st, xs, nsub * C::XS, &x_full[s]);
+                    } else {
+                        for (int u = 0; u < nsub; ++u)
+                            for (int ch = 0; ch < T / 64; ++ch) {
+                                const int o = u * C::XS + ch * (kRowBlock * 128);
+                                if (hv[u] == 3) bulk_load(st + o, xs + o, kRowBlock * 128, &x_full[s]);
+                                else {
+                                    const int o2 = o + (hv[u] == 2 ? kHalf * 128 : 0);
+                                    bulk_load(st + o2, xs + o2, kHalf * 128, &x_full[s]);
+                                }
+                            }
+                    }
+                    if (GS)  // r' of the sub-tiles' 128 rows ride along (adjacent in the workspace too)
+                        bulk_load(st + C::XB, p.rprime + (I.slot0 + t) * kRowBlock, nsub * kRowBlock * 4, &x_full[s]);
                     if (++s == C::NX) { s = 0; sph ^= 1; }
                 }
             }
@@ -144,14 +158,18 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
             uint32_t sph = 0;
             for (int it = blockIdx.x; it < n_items; it += gridDim.x) {
                 const ItemInfo I = decode_item(p, it);
-                int w_next = I.t0 < I.t1 ? __ldg(p.sc.tinfo + I.t0) : 0;
-                for (int t = I.t0; t < I.t1; ++t) {
-                    const int w = w_next;
-                    if (t + 1 < I.t1) w_next = __ldg(p.sc.tinfo + t + 1);
+                int wn[2];  // schedule words of the next macro tile, prefetched one step ahead
+                for (int u = 0; u < NSUB; ++u) wn[u] = I.t0 + u < I.t1 ? __ldg(p.sc.tinfo + I.t0 + u) : 0;
+                for (int t = I.t0; t < I.t1; t += NSUB) {
+                    const int nsub = min(NSUB, I.t1 - t);
+                    int kt[2] = {tinfo_kt(wn[0]), NSUB > 1 ? tinfo_kt(wn[1]) : 0};
+                    for (int u = 0; u < NSUB; ++u) wn[u] = t + NSUB + u < I.t1 ? __ldg(p.sc.tinfo + t + NSUB + u) : 0;
                     mbar_wait(&v_empty[s], sph ^ 1);
-                    mbar_arrive_expect_tx(&v_full[s], C::VB);
-                    for (int h = 0; h < D / 64; ++h)
-                        tma_load_2d(vstage(s) + h * (T * 128), &tmV, h * 64, I.g * p.S + tinfo_kt(w) * T, &v_full[s]);
+                    mbar_arrive_expect_tx(&v_full[s], nsub * T * D * 2);
+                    for (int u = 0; u < nsub; ++u)
+                        for (int h = 0; h < D / 64; ++h)
+                            tma_load_2d(vstage(s) + h * (kMW2 * 128) + u * (T * 128), &tmV, h * 64,
+                                        I.g * p.S + kt[u] * T, &v_full[s]);
                     if (++s == C::NV) { s = 0; sph ^= 1; }
                 }
             }
@@ -164,7 +182,7 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
             uint32_t sph = 0, aph = 0, oph = 0;
             auto post = [&](int flags, int64_t orow) {  // O header to the epilogue, arrival 1 of 2
                 mbar_wait(&o_empty[o], oph ^ 1);
-                ohdr[o] = G2Hdr{flags, 0, (int32_t)(orow & 0xffffffff), (int32_t)(orow >> 32)};
+                ohdr[o] = G2Hdr{flags, 0, 0, 0, (int32_t)(orow & 0xffffffff), (int32_t)(orow >> 32), 0, 0};
                 mbar_arrive(&o_full[o]);
             };
             auto next_o = [&]() {
@@ -184,16 +202,17 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
                 }
                 post(SH_TILE, orow);
                 const uint32_t d_tmem = tmem_o + o * D;
-                for (int t = I.t0; t < I.t1; ++t) {
+                for (int t = I.t0; t < I.t1; t += NSUB) {
+                    const int nk = min(NSUB, I.t1 - t) * (T / 16);  // K steps of 16 keys
                     mbar_wait(&v_full[s], sph);
                     mbar_wait(&a_full[a], aph);
                     tc_fence_after();
                     const uint32_t v_addr = smem_u32(vstage(s));
-                    const uint32_t a_tm = tmem_a + a * (T / 2);
-#pragma unroll
-                    for (int kk = 0; kk < T / 16; ++kk) {
-                        // B = V tile, MN-major SW128: 16 keys per MMA = 2 KB; 64-wide d blocks at LBO = T*128 B
-                        const uint64_t bd = smem_desc_sw128(v_addr + kk * 2048, T * 128, 1024);
+                    const uint32_t a_tm = tmem_a + a * (kMW2 / 2);
+#pragma unroll 8
+                    for (int kk = 0; kk < nk; ++kk) {
+                        // B = V, MN-major SW128: 16 keys per MMA = 2 KB; 64-wide d blocks at LBO = MW*128 B
+                        const uint64_t bd = smem_desc_sw128(v_addr + kk * 2048, kMW2 * 128, 1024);
                         mma_ts(d_tmem, a_tm + kk * 8, bd, idesc, (t == I.t0 && kk == 0) ? 0u : 1u);
                     }
                     mma_commit(&v_empty[s]);
@@ -219,39 +238,48 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
             mbar_wait(&x_full[s], sph);
             const G2Hdr h = *xhdr(s);
             if (h.flags & SH_END) break;
-            const bool valid = (h.hv >> myhalf) & 1;
             const uint32_t xs_s = smem_u32(xstage(s));
-            float rr = valid ? 1.f : 0.f;
-            if (GS && valid) rr = lds_f32(xs_s + C::XB + 4 * r);
-            // the whole X' row (T fp16 = T/8 chunks of 16 B) into registers, then free the stage
-            uint4 xv[T / 8];
-            if (rr != 0.f) {
+            const int hvs[2] = {h.hv0, h.hv1};
+            float rr[NSUB];
 #pragma unroll
-                for (int q4 = 0; q4 < T / 8; ++q4) xv[q4] = lds128(xs_s + tile_chunk_off(r, q4));
+            for (int u = 0; u < NSUB; ++u) {
+                const bool valid = u < h.nsub && ((hvs[u] >> myhalf) & 1);
+                rr[u] = valid ? 1.f : 0.f;
+                if (GS && valid) rr[u] = lds_f32(xs_s + C::XB + u * 512 + 4 * r);
             }
+            // the whole X' row (MW fp16 = 16 chunks of 16 B) into registers first: the loads overlap
+            // the wait for a free A buffer
+            uint4 xv[kMW2 / 8];
+#pragma unroll
+            for (int q = 0; q < kMW2 / 8; ++q)
+                if (rr[(q * 8) / T] != 0.f) xv[q] = lds128(xs_s + tile_chunk_off(r, q));
             mbar_wait(&a_empty[a], aph ^ 1);
             tc_fence_after();
-            const uint32_t a_tm = tmem_a + lane_off + a * (T / 2);
+            const uint32_t a_tm = tmem_a + lane_off + a * (kMW2 / 2);
 #pragma unroll
-            for (int c = 0; c < T / 32; ++c) {  // 32 keys -> 16 packed words per tcgen05.st
+            for (int c = 0; c < kMW2 / 32; ++c) {  // 32 keys -> 16 packed words per tcgen05.st
+                const int u = (c * 32) / T;         // sub-tile of these keys
                 uint32_t pk[16];
-                if (rr != 0.f) {
+                if (rr[u] != 0.f) {
 #pragma unroll
                     for (int q4 = 0; q4 < 4; ++q4) {
-                        const uint32_t xw[4] = {xv[c * 4 + q4].x, xv[c * 4 + q4].y, xv[c * 4 + q4].z, xv[c * 4 + q4].w};
+                        const uint4 x = xv[c * 4 + q4];
+                        const uint32_t xw[4] = {x.x, x.y, x.z, x.w};
 #pragma unroll
-                        for (int u = 0; u < 4; ++u) {
+                        for (int w = 0; w < 4; ++w) {
                             if (GS) {  // Y = X' * r'  (fp16 X' -> fp32 -> x r' -> dtype, one rounding)
-                                const float2 f = unpack_f16(xw[u]);
-                                pk[q4 * 4 + u] = bf ? pack_bf16(f.x * rr, f.y * rr) : pack_f16(f.x * rr, f.y * rr);
+                                const float2 f = unpack_f16(xw[w]);
+                                float y0, y1;
+                                fmul2(y0, y1, f.x, f.y, rr[u]);
+                                pk[q4 * 4 + w] = bf ? pack_bf16(y0, y1) : pack_f16(y0, y1);
                             } else {  // P already holds dtype values
-                                pk[q4 * 4 + u] = xw[u];
+                                pk[q4 * 4 + w] = xw[w];
                             }
                         }
                     }
-                } else {  // invalid half (not loaded) or r' = 0: zero rows of A
+                } else {  // absent sub-tile, invalid half (not loaded) or r' = 0: zero rows of A
 #pragma unroll
-                    for (int u = 0; u < 16; ++u) pk[u] = 0u;
+                    for (int w = 0; w < 16; ++w) pk[w] = 0u;
                 }
                 tmem_st16(a_tm + c * 16, pk);
             }

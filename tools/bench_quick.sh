@@ -2,7 +2,7 @@
 # quick per-config summary: tools/bench_quick.sh TAG [configs...]
 tag=$1; shift
 for c in "$@"; do
-  timeout 300 python bench.py --config $c --no-all-configs --cpu-seconds 0.2 --steps 30 > gpurun_out/q_${tag}_$c.json 2>gpurun_out/q_${tag}_$c.err
+  timeout 300 python bench.py ${BQ_ARGS} --config $c --no-all-configs --cpu-seconds 0.2 --steps 30 > gpurun_out/q_${tag}_$c.json 2>gpurun_out/q_${tag}_$c.err
   python - "$tag" "$c" <<'PY'
 import json, sys
 tag, c = sys.argv[1], sys.argv[2]
