@@ -12,27 +12,30 @@
 //
 // Macro tiles.  The tensor core always computes 128 x MW (MW = 128) score tiles: with T = 64 two
 // consecutive sub-tiles of the item's key list (any two key blocks, stacked in one K stage) share
-// one N = 128 MMA and one epilogue pass, each keeping its own mask, statistics, validity and slot
-// (consecutive list entries are adjacent slots, so the pair's X' is contiguous in HBM).
+// one N = 128 MMA, each keeping its own mask, statistics, validity and slot (consecutive list
+// entries are adjacent slots, so the pair's X' is contiguous in HBM).
 //
-// Warp roles (persistent CTA per SM, 384 threads):
+// Warp roles (persistent CTA per SM, 640 threads for T = 64, 384 for T = 128):
 //   warp 0      TMA producer: Q tile per item, K blocks of each macro tile (NK-stage ring)
 //   warp 1      MMA issuer: D/16 tcgen05.mma kind::f16 of 128 x MW x 16 per macro tile into one of
 //               NACC TMEM accumulators; publishes a header (slot, rows, key tiles, half-valid bits,
 //               kv_len) next to the accumulator -- acc_full completes when both the header arrive and
 //               the MMA commit have landed
 //   warp 2      TMEM allocator (512 columns)
-//   warps 4-11  two epilogue warpgroups taking alternate macro tiles: one tcgen05.ld of the row's
-//               MW scores, accumulator released at once, interval-bitmask mask, max, FFMA2 + ex2,
-//               FADD2 sums, fp16 pack, st.shared into a swizzled staging tile; every warp bulk-stores
-//               its own 32 rows (no warpgroup barrier)
+//   epilogue    T = 64 (SPLIT): warps 4-19, four warpgroups; a pair takes every other macro tile,
+//               one warpgroup per 64-key sub-tile.  T = 128 (FULL): warps 4-11, two warpgroups taking
+//               alternate macro tiles, full 128-key rows.  Each warp: one tcgen05.ld of its row's
+//               scores, accumulator released at once, interval-bitmask mask, max, FFMA2 + ex2, FADD2
+//               sums, fp16 pack, st.shared into a swizzled staging tile, a bulk store of its own rows.
+//               (Splitting a T = 128 row across warpgroups needs a max/sum exchange that costs more
+//               than it saves -- measured.)
 #include "tc_common.cuh"
 
 namespace sr {
 
 using namespace ptx;
 
-constexpr int kMW = 128;  // macro tile width (MMA N of GEMM1, MMA K per step of GEMM2)
+constexpr int kMW = 128;  // macro tile width (MMA N of GEMM1)
 
 struct G1Hdr {  // per-accumulator macro-tile header, written by the MMA warp
     int32_t slot_lo, slot_hi, i0, kvl, w0, w1, flags, pad;
@@ -41,37 +44,43 @@ enum : int { HDR_TILE = 1, HDR_END = 2 };
 
 template <int D, int T>
 struct G1 {
-    static constexpr int NSUB = kMW / T;           // sub-tiles per macro tile
-    static constexpr int QB = kRowBlock * D * 2;   // Q tile bytes
-    static constexpr int KB = kMW * D * 2;         // K stage bytes (MW keys)
-    static constexpr int XB = kRowBlock * kMW * 2;  // staging tile bytes (macro tile)
-    static constexpr int XS = kRowBlock * T * 2;   // X' slot bytes (sub-tile)
-    static constexpr int NACC = 512 / kMW;         // TMEM accumulators
+    static constexpr int NSUB = kMW / T;          // sub-tiles per macro tile
+    static constexpr int QB = kRowBlock * D * 2;  // Q tile bytes
+    static constexpr int KB = kMW * D * 2;        // K stage bytes (MW keys)
+    static constexpr bool SPLIT = (T == 64);      // epilogue organisation, see the file header
+    static constexpr int EPI_WG = SPLIT ? 4 : 2;  // epilogue warpgroups
+    static constexpr int HB = kRowBlock * 64 * 2;  // SPLIT staging tile: one warpgroup's 64 columns
+    static constexpr int XB2 = kRowBlock * kMW * 2;  // FULL staging tile: a whole macro tile
+    static constexpr int SB = SPLIT ? HB : XB2;    // staging buffer per warpgroup
+    static constexpr int XS = kRowBlock * T * 2;  // X' slot bytes (sub-tile)
+    static constexpr int NACC = 512 / kMW;        // TMEM accumulators
     // staging buffers per epilogue warpgroup (2 if at all possible: the X' store stream is the
     // bottleneck), then Q double-buffered if shared memory still allows
-    static constexpr int XPW = (QB + 2 * KB + 4 * XB + 4096 <= kSmemMax) ? 2 : 1;
-    static constexpr int NQ = (2 * QB + 2 * KB + 2 * XPW * XB + 4096 <= kSmemMax) ? 2 : 1;
-    static constexpr int NK_ = (kSmemMax - 4096 - NQ * QB - 2 * XPW * XB) / KB;
+    static constexpr int XPW = (QB + 2 * KB + EPI_WG * 2 * SB + 4096 <= kSmemMax) ? 2 : 1;
+    static constexpr int NQ = (2 * QB + 2 * KB + EPI_WG * XPW * SB + 4096 <= kSmemMax) ? 2 : 1;
+    static constexpr int NK_ = (kSmemMax - 4096 - NQ * QB - EPI_WG * XPW * SB) / KB;
     static constexpr int NK = NK_ > 4 ? 4 : NK_;
     static_assert(NK >= 2, "smem budget");
     static constexpr int OFF_Q = 0;
     static constexpr int OFF_K = OFF_Q + NQ * QB;
     static constexpr int OFF_X = OFF_K + NK * KB;
-    static constexpr int OFF_BAR = OFF_X + 2 * XPW * XB;
+    static constexpr int OFF_BAR = OFF_X + EPI_WG * XPW * SB;
     static constexpr int NBAR = 2 * NQ + 2 * NK + 2 * NACC;
     static constexpr int OFF_HDR = OFF_BAR + NBAR * 8;
     static constexpr int OFF_TPTR = OFF_HDR + NACC * (int)sizeof(G1Hdr);
     static constexpr int SMEM_ = OFF_TPTR + 16 + 1024;  // + alignment slack
     static constexpr int SMEM = SMEM_ > 118 * 1024 ? SMEM_ : 118 * 1024;  // 1 CTA/SM (512 TMEM cols)
-    static constexpr int THREADS = 384;
+    static_assert(SMEM <= kSmemMax, "smem budget");
+    static constexpr int THREADS = 128 + EPI_WG * 128;
 };
 
 template <int D, int T, bool LS>
-__global__ void __launch_bounds__(384, 1)
+__global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
     tc_gemm1(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmK, const Params p)
 {
     using C = G1<D, T>;
     constexpr int NSUB = C::NSUB;
+    constexpr bool SPLIT = C::SPLIT;
     extern __shared__ uint8_t smem_raw[];
     uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
     uint64_t* bars = (uint64_t*)(smem + C::OFF_BAR);
@@ -88,8 +97,9 @@ __global__ void __launch_bounds__(384, 1)
     if (threadIdx.x == 0) {
         for (int i = 0; i < C::NQ; ++i) { mbar_init(&q_full[i], 1); mbar_init(&q_empty[i], 1); }
         for (int i = 0; i < C::NK; ++i) { mbar_init(&k_full[i], 1); mbar_init(&k_empty[i], 1); }
-        // acc_full: header arrive (MMA thread) + tcgen05.commit; acc_empty: one arrive per epilogue warp
-        for (int i = 0; i < C::NACC; ++i) { mbar_init(&acc_full[i], 2); mbar_init(&acc_empty[i], 4); }
+        // acc_full: header arrive (MMA thread) + tcgen05.commit; acc_empty: one arrive per epilogue
+        // warp that reads the accumulator (the warpgroup pair in SPLIT, one warpgroup in FULL)
+        for (int i = 0; i < C::NACC; ++i) { mbar_init(&acc_full[i], 2); mbar_init(&acc_empty[i], SPLIT ? 8 : 4); }
         fence_mbar_init();
     }
     if (warp == 0 && lane == 0) { prefetch_tmap(&tmQ); prefetch_tmap(&tmK); }
@@ -105,8 +115,12 @@ __global__ void __launch_bounds__(384, 1)
     const int n_items = p.sc.n_items;
 
     if (warp < 4) {
-        // warpgroup 0 hands registers to the epilogue warpgroups (168/thread at launch)
-        reg_dealloc<56>();
+        // warpgroup 0 hands registers to the epilogue warpgroups.  setmaxnreg.inc can only draw what
+        // other warps of this CTA released, so the budgets balance exactly:
+        //   SPLIT (640 threads, 96 at launch): 4 warps x 32 x (96 - 64) = 16 warps x 32 x (104 - 96)
+        //   FULL  (384 threads, 168 at launch): 4 warps x 32 x (168 - 56) = 8 warps x 32 x (224 - 168)
+        if constexpr (SPLIT) reg_dealloc<64>();
+        else reg_dealloc<56>();
         if (warp == 0 && lane == 0) {
             // -------------------------------------------------------------- TMA producer
             int qi = 0, ks = 0;
@@ -181,7 +195,7 @@ __global__ void __launch_bounds__(384, 1)
                 mma_commit(&q_empty[qi]);
                 if (++qi == C::NQ) { qi = 0; qph ^= 1; }
             }
-            for (int e = 0; e < 2; ++e, ++n) {  // one END header for each epilogue warpgroup
+            for (int e = 0; e < 2; ++e, ++n) {  // one END header for each epilogue warpgroup pair
                 const int ab = n % C::NACC;
                 mbar_wait(&acc_empty[ab], ((n / C::NACC) & 1) ^ 1);
                 hdr[ab].flags = HDR_END;
@@ -189,8 +203,127 @@ __global__ void __launch_bounds__(384, 1)
                 mbar_arrive(&acc_full[ab]);
             }
         }
+    } else if constexpr (SPLIT) {
+        reg_alloc<104>();
+        // ------------------------------------------------------------------ epilogue warpgroups
+        const int ewg = (warp - 4) / 4;        // 0..3
+        const int pj = ewg / 2;                // warpgroup pair: macro tiles n = pj, pj + 2, ...
+        const int h = ewg % 2;                 // column half of the macro tile
+        const int q = warp % 4;                // TMEM lane quadrant
+        const int r = q * 32 + lane;           // tile row == TMEM lane
+        const int myhalf = r / kHalf;
+        const uint32_t lane_off = (uint32_t)(q * 32) << 16;
+        const float sl2 = p.scale_log2;
+        int k = 0;                            // macro tiles processed by this warpgroup
+        for (int n = pj;; n += 2, ++k) {
+            const int buf = n % C::NACC;
+            mbar_wait(&acc_full[buf], (uint32_t)(n / C::NACC) & 1);
+            tc_fence_after();
+            const G1Hdr H = hdr[buf];
+            if (H.flags & HDR_END) break;
+            // this warpgroup's 64 columns: sub-tile h (T = 64) or half h of the sub-tile (T = 128)
+            const int w = (NSUB == 2 && h == 1) ? H.w1 : H.w0;
+            const bool valid = w != -1 && ((tinfo_half(w) >> myhalf) & 1);
+            const int c0 = tinfo_kt(w) * T + (NSUB == 1 ? 64 * h : 0);
+            const int i = H.i0 + r;
+            const int64_t slot = (((int64_t)H.slot_hi << 32) | (uint32_t)H.slot_lo) + (NSUB == 2 ? h : 0);
+            // one TMEM read of the row's 64 fp32 scores; the accumulator goes straight back to the MMA
+            uint32_t x[64];
+            if (valid) {
+                tmem_ld32(tmem_base + lane_off + buf * kMW + 64 * h, *reinterpret_cast<uint32_t(*)[32]>(&x[0]));
+                tmem_ld32(tmem_base + lane_off + buf * kMW + 64 * h + 32, *reinterpret_cast<uint32_t(*)[32]>(&x[32]));
+                tmem_wait_ld();
+            }
+            tc_fence_before();
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&acc_empty[buf]);
+            uint8_t* stage = smem + C::OFF_X + (ewg * C::XPW + (k % C::XPW)) * C::HB;
+            const uint32_t stage_s = smem_u32(stage);
+            // Each warp stages and stores its own 32 rows: its slice of this staging buffer is free
+            // once the warp's own store from it (XPW tiles ago) has read it.  Every warp commits one
+            // bulk group per macro tile (possibly empty) so the count holds.
+            if (lane == 0) {
+                if (C::XPW == 2) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
+                else bulk_wait_read0();
+            }
+            __syncwarp();
+            float mx = -INFINITY, dsum = 0.f;
+            if (valid) {
+                // mask layer: kept keys of this row form <= 2 intervals; interior
+                // column ranges (every key kept) skip the bit construction entirely
+                const RowMask rm = row_mask(p, i, H.kvl);
+                const bool full = c0 >= rm.lo && c0 + 63 <= rm.hi &&
+                                  ((c0 >= rm.blo && c0 + 63 <= rm.bhi) || c0 + 63 < rm.gc);
+                if (!full) {
+#pragma unroll
+                    for (int c = 0; c < 2; ++c) {
+                        const uint32_t bits = mask_bits32(rm, c0 + c * 32);
+#pragma unroll
+                        for (int u = 0; u < 32; ++u)
+                            if (!((bits >> u) & 1u)) x[c * 32 + u] = 0xff800000u;  // -inf
+                    }
+                }
+                if (LS) {
+                    float m8[8];
+#pragma unroll
+                    for (int a = 0; a < 8; ++a) m8[a] = __uint_as_float(x[a]);
+#pragma unroll
+                    for (int u = 8; u < 64; ++u) m8[u & 7] = fmaxf(m8[u & 7], __uint_as_float(x[u]));
+                    mx = fmaxf(fmaxf(fmaxf(m8[0], m8[1]), fmaxf(m8[2], m8[3])),
+                               fmaxf(fmaxf(m8[4], m8[5]), fmaxf(m8[6], m8[7])));
+                    // X' = e^{x - m'}: base 2 with log2(e) folded into the scale -- one FFMA2 per pair,
+                    // then one MUFU.EX2 per element (in place)
+                    const float neg = (mx == -INFINITY) ? 0.f : -mx * sl2;
+#pragma unroll
+                    for (int u = 0; u < 64; u += 2) {
+                        float t0, t1;
+                        ffma2(t0, t1, __uint_as_float(x[u]), __uint_as_float(x[u + 1]), sl2, neg);
+                        x[u] = __float_as_uint(ex2(t0));
+                        x[u + 1] = __float_as_uint(ex2(t1));
+                    }
+                    // d' = sum X' (fp32, FADD2 into 4 independent pair accumulators)
+                    float sa[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+#pragma unroll
+                    for (int u = 0; u < 64; u += 2)
+                        fadd2_acc(sa[(u >> 1) & 3], sa[4 + ((u >> 1) & 3)], __uint_as_float(x[u]), __uint_as_float(x[u + 1]));
+                    dsum = ((sa[0] + sa[4]) + (sa[1] + sa[5])) + ((sa[2] + sa[6]) + (sa[3] + sa[7]));
+                } else {  // unfused baseline: the scaled, masked score
+#pragma unroll
+                    for (int u = 0; u < 64; u += 2) {
+                        float t0, t1;
+                        fmul2(t0, t1, __uint_as_float(x[u]), __uint_as_float(x[u + 1]), p.scale);
+                        x[u] = __float_as_uint(t0);
+                        x[u + 1] = __float_as_uint(t1);
+                    }
+                }
+#pragma unroll
+                for (int q4 = 0; q4 < 8; ++q4) {  // 8 keys -> one 16-B chunk of the fp16 tile
+                    uint32_t w4[4];
+#pragma unroll
+                    for (int u = 0; u < 4; ++u)
+                        w4[u] = pack_f16(__uint_as_float(x[q4 * 8 + 2 * u]), __uint_as_float(x[q4 * 8 + 2 * u + 1]));
+                    sts128(stage_s + tile_chunk_off(r, q4), w4[0], w4[1], w4[2], w4[3]);
+                }
+            }
+            // the warp's 32 rows x 64 columns (4 KB, contiguous in the tile layout) go to HBM
+            fence_proxy_async_smem();
+            __syncwarp();
+            if (lane == 0) {
+                if (valid) {  // warp-uniform: a warp's 32 rows lie in one 64-row half
+                    uint8_t* dst = (uint8_t*)p.xprime + slot * (int64_t)C::XS + (NSUB == 1 ? h * C::HB : 0) +
+                                   q * 32 * 128;
+                    bulk_store(dst, stage + q * 32 * 128, 32 * 128);
+                }
+                bulk_commit();
+            }
+            if (LS && valid && (NSUB == 2 || h == 0)) {
+                p.mprime[slot * kRowBlock + r] = mx * p.scale;  // m' in natural-log units
+                p.dprime[slot * kRowBlock + r] = dsum;
+            }
+        }
+        if (lane == 0) bulk_wait0();
     } else {
-        reg_alloc<224>();
+        reg_alloc<224>();  // frees/takes 14336 registers, see the dealloc above
         // ------------------------------------------------------------------ epilogue warpgroups
         const int e = (warp - 4) / 4;          // warpgroup 0 / 1: even / odd macro tiles
         const int r = (warp % 4) * 32 + lane;  // tile row == TMEM lane
@@ -226,7 +359,7 @@ __global__ void __launch_bounds__(384, 1)
             tc_fence_before();
             __syncwarp();
             if (lane == 0) mbar_arrive(&acc_empty[buf]);
-            uint8_t* stage = smem + C::OFF_X + (e * C::XPW + (k % C::XPW)) * C::XB;
+            uint8_t* stage = smem + C::OFF_X + (e * C::XPW + (k % C::XPW)) * C::XB2;
             const uint32_t stage_s = smem_u32(stage);
             // Each warp stages and stores its own 32 rows (no warpgroup barrier): its slice of this
             // staging buffer is free once the warp's own store from it (XPW macro tiles ago) has read
