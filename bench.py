@@ -141,11 +141,11 @@ class Layer:
             self.T = info["tile_n"]
         self.n_tiles, self.stored = sr.schedule_stats(self.mask, cfg.B, cfg.H, cfg.S, causal=cfg.causal, tile_n=tile_n)
 
-    def run(self, fused=True, stages=0, q=None, k=None, v=None):
+    def run(self, fused=True, stages=0, q=None, k=None, v=None, fuse_ir=False):
         d = self.dev
         return self.sr.call(self.mask, q if q is not None else d["q"], k if k is not None else d["k"],
                             v if v is not None else d["v"], out=self.out, fused=fused, stages=stages,
-                            workspace=self.ws[fused], tile_n=self.tile_n, **self.kw)
+                            workspace=self.ws[fused], tile_n=self.tile_n, fuse_ir=fuse_ir, **self.kw)
 
 
 def timed(torch, fn, steps, warmup, flush, per_step_pre=None):
@@ -232,6 +232,14 @@ def gpu_arm(args, rank, world, local_rank):
         barrier(torch, world)
         ms_unf = dist_max(torch, statistics.mean(timed(torch, lambda: L.run(fused=False), K, Wm, flush)), world)
 
+    # ---- SURVEY NEXT-2 variant: the IR sub-layer folded into GEMM2 (SR_FUSE_IR), same workload
+    ms_fir = None
+    if cfg.dtype != "f32":
+        L.run(fuse_ir=True)
+        barrier(torch, world)
+        ms_fir = dist_max(torch, statistics.mean(timed(torch, lambda: L.run(fuse_ir=True), K, Wm, flush)), world)
+        L.run()  # leave the paper-design intermediates (r') in the workspace for the stage timings
+
     # ---- per-kernel durations inside the step (stage-selected launches, events on the stream)
     rec_b, unf_b = alg_bytes(cfg, L.stored, L.T)
     kern = {}
@@ -281,6 +289,10 @@ def gpu_arm(args, rank, world, local_rank):
                             "byte_reduction": round(1 - sum(r2.values()) / sum(u2.values()), 4),
                             "speedup_vs_unfused": round(tu / tr, 3)})
             ent["hbm_GBps_recomposed"] = round(sum(r2.values()) / (tr * 1e-3) / 1e9, 1)
+            if c2.dtype != "f32":
+                L2.run(fuse_ir=True)
+                tf = statistics.mean(timed(torch, lambda: L2.run(fuse_ir=True), 10, 3, flush))
+                ent["fused_ir_layers_per_s"] = round(1e3 / tf, 1)
             others[f"C{c2.idx}"] = ent
             del L2
             torch.cuda.empty_cache()
@@ -313,6 +325,11 @@ def gpu_arm(args, rank, world, local_rank):
         "unfused": None if ms_unf is None else {"value": round(world * 1e3 / ms_unf, 2), "ms_per_step": round(ms_unf, 5),
                                                 "speedup_recomposed_vs_unfused": round(ms_unf / ms_step, 3),
                                                 "kernels": kern_unf},
+        "variants": None if ms_fir is None else {
+            "fused_ir": {"what": "IR folded into GS+GEMM2 (SURVEY NEXT-2, 2 kernels)",
+                         "value": round(world * 1e3 / ms_fir, 2), "ms_per_step": round(ms_fir, 5),
+                         "alg_bytes": int(sum(rec_b.values()) - 12 * L.stored / L.T - 4 * L.stored / L.T
+                                          + 8 * L.stored / L.T + 4 * L.stored / L.T)}},
         "kernels": kern,
         "roofline": {"kernel": dom, "bound": "hbm", "achieved": round(achieved, 1), "peak": hbm_peak, "unit": "GB/s",
                      "frac": round(achieved / hbm_peak, 4), "traffic": ncu.get(f"{dom}_dram_bytes"),

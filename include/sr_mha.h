@@ -107,6 +107,12 @@ typedef struct {
 #define SR_RUN_GEMM1 1   /* GEMM1 + LS (recomposed) / GEMM1 writing scores (unfused) */
 #define SR_RUN_REDUCE 2  /* IR (recomposed) / row softmax (unfused) */
 #define SR_RUN_GEMM2 4   /* GS + GEMM2 (recomposed) / GEMM2 on P (unfused) */
+/* Variant bit for sr_exec.flags (recomposed 16-bit path): fold the IR sub-layer into GEMM2 (one
+ * warp of each GEMM2 CTA reduces the item's m', d' before its GS warps need them; r' is formed on
+ * the fly and never written).  Same results up to rounding; one kernel and the r' round trip
+ * fewer.  SURVEY.md NEXT-2 -- a B200-specific departure from the paper's separate IR kernel
+ * (PAPER.md L173), off by default.  With SR_RUN_* stage bits, SR_RUN_REDUCE is then a no-op. */
+#define SR_FUSE_IR 16
 
 /* Entry points (north star).  Returns SR_OK after enqueueing the kernels on ex->stream. */
 sr_status sr_mha_dense(const void* q, const void* k, const void* v, void* out, int B, int H, int S,

@@ -198,11 +198,13 @@ _FN = {(SR_E_DENSE, True): "sr_mha_dense", (SR_E_BLOCKSPARSE, True): "sr_mha_blo
 
 
 SR_RUN_GEMM1, SR_RUN_REDUCE, SR_RUN_GEMM2 = 1, 2, 4
+SR_FUSE_IR = 16
 
 
 def call(mask: _Mask, q, k, v, *, scale=None, causal=False, out_dtype=None, tile_n=0, fused=True,
-         out=None, workspace=None, stream=None, stages=0):
-    """Run one attention layer through the C ABI.  q, k, v: CUDA tensors [B, H, S, D]."""
+         out=None, workspace=None, stream=None, stages=0, fuse_ir=False):
+    """Run one attention layer through the C ABI.  q, k, v: CUDA tensors [B, H, S, D].
+    fuse_ir=True selects the SR_FUSE_IR variant (IR folded into GEMM2)."""
     torch = _torch()
     if not (q.is_cuda and k.is_cuda and v.is_cuda):
         raise ValueError("q, k, v must be CUDA tensors")
@@ -225,7 +227,7 @@ def call(mask: _Mask, q, k, v, *, scale=None, causal=False, out_dtype=None, tile
     ws = workspace if workspace is not None else _workspace(q.device, need)
     st = torch.cuda.current_stream(q.device).cuda_stream if stream is None else stream
     ex = Exec(in_dt, dtype_code(out_dtype), ws.data_ptr(), ws.numel() * ws.element_size(), st, int(tile_n),
-              int(stages))
+              int(stages) | (SR_FUSE_IR if fuse_ir else 0))
     fn = getattr(lib(), _FN[(mask.entry, bool(fused))])
     _check(fn(q.data_ptr(), k.data_ptr(), v.data_ptr(), out.data_ptr(), B, H, S, D, C.c_float(scale), mask.ptr,
               int(causal), C.byref(ex)))

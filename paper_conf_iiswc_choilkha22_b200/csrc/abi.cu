@@ -352,8 +352,10 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
     if (!ex) return fail(SR_ERR_INVALID, "exec descriptor is NULL");
     if (!q || !k || !v || !out) return fail(SR_ERR_INVALID, "q, k, v and out must be non-NULL");
     if (!std::isfinite(scale) || !(scale > 0.f)) return fail(SR_ERR_INVALID, "scale must be finite and > 0");
-    if (ex->flags & ~(SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2))
+    if (ex->flags & ~(SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2 | SR_FUSE_IR))
         return fail(SR_ERR_INVALID, "unknown flags 0x%x", ex->flags);
+    if ((ex->flags & SR_FUSE_IR) && (!fused || ex->in_dtype == SR_F32))
+        return fail(SR_ERR_UNSUPPORTED, "SR_FUSE_IR applies to the recomposed 16-bit path only");
     Request r;
     sr_status s = check_request(e, B, H, S, D, ex->in_dtype, mask_or_layout, causal, ex->tile_n, r);
     if (s != SR_OK) return s;
@@ -391,7 +393,9 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
     p.in_dtype = ex->in_dtype;
     p.out_dtype = ex->out_dtype;
     p.sc = cs->dev;
-    p.stages = ex->flags ? ex->flags : (SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2);
+    const int stage_bits = ex->flags & (SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2);
+    p.stages = stage_bits ? stage_bits : (SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2);
+    p.fuse_ir = (ex->flags & SR_FUSE_IR) ? 1 : 0;
     char* ws = (char*)ex->workspace;
     p.xprime = ws + wi.off_xprime;
     if (fused) {

@@ -30,7 +30,7 @@ using namespace ptx;
 
 constexpr int kMW2 = 128;  // macro tile width (keys per MMA step)
 
-enum : int { SH_TILE = 1, SH_END = 2, SH_EMPTY = 4 };
+enum : int { SH_TILE = 1, SH_END = 2, SH_EMPTY = 4, SH_FIRST = 8, SH_LAST = 16 };
 struct G2Hdr {  // X'-stage / O-buffer header
     int32_t flags, hv0, hv1, nsub, orow_lo, orow_hi, pad0, pad1;
 };
@@ -55,15 +55,20 @@ struct G2 {
     static constexpr int OFF_X = 0;
     static constexpr int OFF_V = NX * XSB;
     static constexpr int OFF_BAR = OFF_V + NV * VB;
-    static constexpr int NBAR = 2 * NX + 2 * NV + 2 * NA + 2 * NO;
-    static constexpr int OFF_OHDR = OFF_BAR + NBAR * 8;
+    static constexpr int NSI = 4;  // fused-IR variant: per-item (m, 1/d) row statistics in flight
+    static constexpr int NBAR = 2 * NX + 2 * NV + 2 * NA + 2 * NO + 2 * NSI;
+    static constexpr int OFF_STATS = OFF_BAR + NBAR * 8;                      // [NSI][2][128] fp32
+    static constexpr int OFF_OHDR = OFF_STATS + NSI * 2 * kRowBlock * 4;
     static constexpr int OFF_TPTR = OFF_OHDR + NO * (int)sizeof(G2Hdr);
     static constexpr int SMEM_ = OFF_TPTR + 16 + 1024;
     static constexpr int SMEM = SMEM_ > 118 * 1024 ? SMEM_ : 118 * 1024;  // 1 CTA/SM (512 TMEM cols)
     static constexpr int THREADS = 384;
 };
 
-template <int D, int T, bool GS>
+// FI (fused IR): the IR sub-layer runs inside this kernel -- warp 2 reduces each
+// item's m', d' into per-row (m, 1/d) ahead of the GS warps, the X' stages carry m' instead of r',
+// and GS forms r' = e^{m' - m} / d on the fly.  No IR launch, no r' round trip through HBM.
+template <int D, int T, bool GS, bool FI>
 __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUtensorMap tmV, const Params p)
 {
     using C = G2<D, T>;
@@ -79,6 +84,9 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
     uint64_t* a_empty = a_full + C::NA;
     uint64_t* o_full = a_empty + C::NA;
     uint64_t* o_empty = o_full + C::NO;
+    uint64_t* st_full = o_empty + C::NO;  // fused IR: item statistics ready / consumed
+    uint64_t* st_empty = st_full + C::NSI;
+    float* stats = (float*)(smem + C::OFF_STATS);
     G2Hdr* ohdr = (G2Hdr*)(smem + C::OFF_OHDR);
     uint32_t* tmem_ptr = (uint32_t*)(smem + C::OFF_TPTR);
     auto xstage = [&](int s) { return smem + C::OFF_X + s * C::XSB; };
@@ -92,6 +100,7 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
         for (int i = 0; i < C::NA; ++i) { mbar_init(&a_full[i], 4); mbar_init(&a_empty[i], 1); }
         // o_full: O-header arrive + MMA commit; o_empty: one arrive per epilogue warp
         for (int i = 0; i < C::NO; ++i) { mbar_init(&o_full[i], 2); mbar_init(&o_empty[i], 4); }
+        for (int i = 0; i < C::NSI; ++i) { mbar_init(&st_full[i], 1); mbar_init(&st_empty[i], 4); }
         fence_mbar_init();
     }
     if (warp == 3 && lane == 0) prefetch_tmap(&tmV);
@@ -126,7 +135,8 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
                     for (int u = 0; u < nsub; ++u) bytes += (hv[u] == 3 ? 2 : 1) * (T / 64) * (kHalf * 128);
                     mbar_wait(&x_empty[s], sph ^ 1);
                     uint8_t* st = xstage(s);
-                    *xhdr(s) = G2Hdr{SH_TILE, hv[0], hv[1], nsub, 0, 0, 0, 0};
+                    *xhdr(s) = G2Hdr{SH_TILE | (t == I.t0 ? SH_FIRST : 0) | (t + NSUB >= I.t1 ? SH_LAST : 0), hv[0],
+                                     hv[1], nsub, 0, 0, 0, 0};
                     mbar_arrive_expect_tx(&x_full[s], bytes);
                     const uint8_t* xs = src + (I.slot0 + t) * (int64_t)C::XS;  // sub-tiles t, t+1 are adjacent
                     if (hv[0] == 3 && (nsub == 1 || hv[1] == 3)) {
@@ -142,14 +152,73 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
                                 }
                             }
                     }
-                    if (GS)  // r' of the sub-tiles' 128 rows ride along (adjacent in the workspace too)
-                        bulk_load(st + C::XB, p.rprime + (I.slot0 + t) * kRowBlock, nsub * kRowBlock * 4, &x_full[s]);
+                    if (GS)  // r' (or m' with the fused IR) of the sub-tiles' 128 rows rides along
+                        bulk_load(st + C::XB, (FI ? p.mprime : p.rprime) + (I.slot0 + t) * kRowBlock,
+                                  nsub * kRowBlock * 4, &x_full[s]);
                     if (++s == C::NX) { s = 0; sph ^= 1; }
                 }
             }
             mbar_wait(&x_empty[s], sph ^ 1);
             xhdr(s)->flags = SH_END;
             mbar_arrive(&x_full[s]);
+        }
+    } else if (warp == 2) {
+        if (FI) {
+            // -------------------------------------------------------------- fused IR (NEXT-2)
+            // Per non-empty item, per row: m = max_k m'_k, d = sum_k e^{m'_k - m} d'_k (PAPER.md
+            // L147), published as (m, 1/d) in a ring of NSI items.  Lane l reduces rows l + 32j.
+            int si = 0;
+            uint32_t sph = 0;
+            for (int it = blockIdx.x; it < n_items; it += gridDim.x) {
+                const ItemInfo I = decode_item(p, it);
+                if (I.t0 == I.t1) continue;
+                mbar_wait(&st_empty[si], sph ^ 1);
+                float* ms = stats + si * 2 * kRowBlock;
+                const float* mp = p.mprime + I.slot0 * kRowBlock + lane;
+                const float* dp = p.dprime + I.slot0 * kRowBlock + lane;
+                float m[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY}, d[4] = {0.f, 0.f, 0.f, 0.f};
+                for (int tb = I.t0; tb < I.t1; tb += 8) {
+                    // one memory round trip per batch: 8 tiles x 4 rows x (m', d') + the tile words
+                    float m8[4][8], d8[4][8];
+                    int w8[8];
+#pragma unroll
+                    for (int u = 0; u < 8; ++u) w8[u] = tb + u < I.t1 ? __ldg(p.sc.tinfo + tb + u) : 0;
+#pragma unroll
+                    for (int u = 0; u < 8; ++u)
+#pragma unroll
+                        for (int j = 0; j < 4; ++j) {
+                            const bool in = tb + u < I.t1;
+                            m8[j][u] = in ? __ldg(mp + (int64_t)(tb + u) * kRowBlock + 32 * j) : -INFINITY;
+                            d8[j][u] = in ? __ldg(dp + (int64_t)(tb + u) * kRowBlock + 32 * j) : 0.f;
+                        }
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) {
+                        const int half = (lane + 32 * j) / kHalf;
+                        float mb = -INFINITY;
+#pragma unroll
+                        for (int u = 0; u < 8; ++u) {
+                            if (!((tinfo_half(w8[u]) >> half) & 1) || tb + u >= I.t1) m8[j][u] = -INFINITY;
+                            mb = fmaxf(mb, m8[j][u]);
+                        }
+                        if (mb == -INFINITY) continue;
+                        const float mn = fmaxf(m[j], mb);
+                        float acc = (m[j] == -INFINITY) ? 0.f : d[j] * __expf(m[j] - mn);
+#pragma unroll
+                        for (int u = 0; u < 8; ++u)
+                            if (m8[j][u] != -INFINITY) acc += d8[j][u] * __expf(m8[j][u] - mn);
+                        m[j] = mn;
+                        d[j] = acc;
+                    }
+                }
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    ms[lane + 32 * j] = m[j];
+                    ms[kRowBlock + lane + 32 * j] = d[j] > 0.f ? 1.f / d[j] : 0.f;
+                }
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&st_full[si]);
+                if (++si == C::NSI) { si = 0; sph ^= 1; }
+            }
         }
     } else if (warp == 3) {
         if (lane == 0) {
@@ -232,12 +301,21 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
         const int myhalf = r / kHalf;
         const uint32_t lane_off = (uint32_t)((warp % 4) * 32) << 16;
         const bool bf = p.in_dtype == DT_BF16;
-        int s = 0, a = 0;
-        uint32_t sph = 0, aph = 0;
+        int s = 0, a = 0, si = 0;
+        uint32_t sph = 0, aph = 0, siph = 0;
+        float m_row = 0.f, invd_row = 0.f;  // fused IR: this row's (m, 1/d) for the current item
         for (;;) {
             mbar_wait(&x_full[s], sph);
             const G2Hdr h = *xhdr(s);
             if (h.flags & SH_END) break;
+            if (FI && (h.flags & SH_FIRST)) {  // a new item: its row statistics from the IR warp
+                mbar_wait(&st_full[si], siph);
+                m_row = stats[si * 2 * kRowBlock + r];
+                invd_row = stats[si * 2 * kRowBlock + kRowBlock + r];
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&st_empty[si]);
+                if (++si == C::NSI) { si = 0; siph ^= 1; }
+            }
             const uint32_t xs_s = smem_u32(xstage(s));
             const int hvs[2] = {h.hv0, h.hv1};
             float rr[NSUB];
@@ -245,7 +323,13 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
             for (int u = 0; u < NSUB; ++u) {
                 const bool valid = u < h.nsub && ((hvs[u] >> myhalf) & 1);
                 rr[u] = valid ? 1.f : 0.f;
-                if (GS && valid) rr[u] = lds_f32(xs_s + C::XB + u * 512 + 4 * r);
+                if (GS && valid) {
+                    const float v = lds_f32(xs_s + C::XB + u * 512 + 4 * r);
+                    if (FI)  // r'_k = e^{m'_k - m} / d  (0 for a fully masked sub-vector)
+                        rr[u] = (v == -INFINITY) ? 0.f : __expf(v - m_row) * invd_row;
+                    else
+                        rr[u] = v;
+                }
             }
             // the whole X' row (MW fp16 = 16 chunks of 16 B) into registers first: the loads overlap
             // the wait for a free A buffer
@@ -359,7 +443,7 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
 cudaError_t make_tmap_2d(CUtensorMap* m, const void* base, int64_t rows, int D, int box_rows, int dtype);
 int num_sms();
 
-template <int D, int T, bool GS>
+template <int D, int T, bool GS, bool FI>
 cudaError_t launch_g2_t(const Params& p, cudaStream_t st, int64_t* nl)
 {
     using C = G2<D, T>;
@@ -367,20 +451,25 @@ cudaError_t launch_g2_t(const Params& p, cudaStream_t st, int64_t* nl)
     const int64_t rows = (int64_t)p.B * p.H * p.S;
     cudaError_t e;
     if ((e = make_tmap_2d(&tv, p.v, rows, D, T, p.in_dtype)) != cudaSuccess) return e;
-    auto kern = tc_gemm2<D, T, GS>;
+    auto kern = tc_gemm2<D, T, GS, FI>;
     if ((e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM)) != cudaSuccess) return e;
     const int grid = std::min(p.sc.n_items, num_sms());
     return launch_pdl(kern, dim3(grid), dim3(C::THREADS), C::SMEM, st, nl, tv, p);
 }
 
-cudaError_t launch_gemm2(const Params& p, bool gs, cudaStream_t st, int64_t* nl)
+template <int D, int T>
+cudaError_t launch_g2_dt(const Params& p, int mode, cudaStream_t st, int64_t* nl)
 {
-    if (p.D == 64) {
-        if (p.T == 64) return gs ? launch_g2_t<64, 64, true>(p, st, nl) : launch_g2_t<64, 64, false>(p, st, nl);
-        return gs ? launch_g2_t<64, 128, true>(p, st, nl) : launch_g2_t<64, 128, false>(p, st, nl);
-    }
-    if (p.T == 64) return gs ? launch_g2_t<128, 64, true>(p, st, nl) : launch_g2_t<128, 64, false>(p, st, nl);
-    return gs ? launch_g2_t<128, 128, true>(p, st, nl) : launch_g2_t<128, 128, false>(p, st, nl);
+    if (mode == 0) return launch_g2_t<D, T, false, false>(p, st, nl);
+    if (mode == 1) return launch_g2_t<D, T, true, false>(p, st, nl);
+    return launch_g2_t<D, T, true, true>(p, st, nl);
+}
+
+// mode: 0 = unfused baseline (P . V), 1 = GS + GEMM2 (r' from the IR kernel), 2 = IR + GS + GEMM2
+cudaError_t launch_gemm2(const Params& p, int mode, cudaStream_t st, int64_t* nl)
+{
+    if (p.D == 64) return p.T == 64 ? launch_g2_dt<64, 64>(p, mode, st, nl) : launch_g2_dt<64, 128>(p, mode, st, nl);
+    return p.T == 64 ? launch_g2_dt<128, 64>(p, mode, st, nl) : launch_g2_dt<128, 128>(p, mode, st, nl);
 }
 
 }  // namespace sr

@@ -54,6 +54,7 @@ struct Params {
     int n_global;
     int in_dtype, out_dtype;
     int stages;        // SR_RUN_* bits to launch
+    int fuse_ir;       // SR_FUSE_IR: the IR sub-layer runs inside GEMM2
     DevSched sc;
     void* xprime;      // X' tiles (recomposed) or score tiles S (unfused)
     void* pbuf;        // unfused: P tiles

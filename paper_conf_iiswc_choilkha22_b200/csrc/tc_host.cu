@@ -11,7 +11,7 @@
 namespace sr {
 
 cudaError_t launch_gemm1(const Params& p, bool ls, cudaStream_t st, int64_t* nl);
-cudaError_t launch_gemm2(const Params& p, bool gs, cudaStream_t st, int64_t* nl);
+cudaError_t launch_gemm2(const Params& p, int mode, cudaStream_t st, int64_t* nl);
 cudaError_t launch_softmax(const Params& p, cudaStream_t st, int64_t* nl);
 
 namespace {
@@ -61,8 +61,9 @@ cudaError_t launch_tc_fused(const Params& p, cudaStream_t st, int64_t* nl)
 {
     cudaError_t e = cudaSuccess;
     if ((p.stages & 1) && (e = launch_gemm1(p, true, st, nl)) != cudaSuccess) return e;
-    if ((p.stages & 2) && (e = launch_ir(p, st, nl)) != cudaSuccess) return e;
-    if (p.stages & 4) e = launch_gemm2(p, true, st, nl);
+    // the IR sub-layer: its own kernel (the paper's design), or folded into GEMM2 (SR_FUSE_IR)
+    if (!p.fuse_ir && (p.stages & 2) && (e = launch_ir(p, st, nl)) != cudaSuccess) return e;
+    if (p.stages & 4) e = launch_gemm2(p, p.fuse_ir ? 2 : 1, st, nl);
     return e;
 }
 
@@ -72,7 +73,7 @@ cudaError_t launch_tc_unfused(const Params& p, cudaStream_t st, int64_t* nl)
     cudaError_t e = cudaSuccess;
     if ((p.stages & 1) && (e = launch_gemm1(p, false, st, nl)) != cudaSuccess) return e;
     if ((p.stages & 2) && (e = launch_softmax(p, st, nl)) != cudaSuccess) return e;
-    if (p.stages & 4) e = launch_gemm2(p, false, st, nl);
+    if (p.stages & 4) e = launch_gemm2(p, 0, st, nl);
     return e;
 }
 

@@ -34,11 +34,11 @@ def _ulp_half(dtype, ref):
 
 
 def run_case(kind, B, H, S, D, dtype, *, causal=False, kv_len=None, layout=None, window=0, n_global=0,
-             tile_n=0, fused=True, seed=0, out_f32=True):
+             tile_n=0, fused=True, seed=0, out_f32=True, fuse_ir=False):
     t, q, k, v = qkv(B, H, S, D, dtype, seed)
     scale = 1 / math.sqrt(D)
     od = torch.float32 if out_f32 else TORCH[dtype]
-    kw = dict(scale=scale, causal=causal, tile_n=tile_n, fused=fused, out_dtype=od)
+    kw = dict(scale=scale, causal=causal, tile_n=tile_n, fused=fused, out_dtype=od, fuse_ir=fuse_ir)
     if kind == "dense":
         o = sr.mha_dense(q, k, v, kv_len=kv_len, **kw)
     elif kind == "block":
@@ -319,3 +319,52 @@ def test_gemm2_bitwise_deterministic(idx, T):
     base = run()
     for _ in range(8):
         assert torch.equal(run(), base)
+
+
+# ------------------------------------------------------------------------------------ fused-IR variant
+
+FUSED_IR_CASES = [
+    ("dense", dict(B=8, H=2, S=512, D=64, dtype="f16", kv_len=[512, 511, 384, 300, 257, 128, 65, 1])),
+    ("dense", dict(B=2, H=2, S=384, D=128, dtype="bf16", causal=True)),
+    ("dense", dict(B=2, H=2, S=256, D=64, dtype="f16", causal=True, tile_n=64)),
+    ("dense", dict(B=3, H=2, S=256, D=64, dtype="f16", kv_len=[1, 0, 129])),
+    ("block", dict(B=2, H=3, S=512, D=64, dtype="f16", layout="rand")),
+    ("window", dict(B=1, H=2, S=768, D=64, dtype="f16", window=254, n_global=8, causal=True)),
+]
+
+
+@pytest.mark.parametrize("kind,kw", FUSED_IR_CASES, ids=lambda x: str(x)[:40] if isinstance(x, dict) else x)
+def test_fused_ir_variant(kind, kw):
+    """SR_FUSE_IR (IR folded into GEMM2) against the oracle, same tolerance."""
+    kw = dict(kw)
+    if kw.get("layout") == "rand":
+        kw["layout"] = W.random_layout(kw["H"], kw["S"] // 64, 64, 0.35, seed=8)
+    B, H, S, D, dtype = (kw.pop(x) for x in ("B", "H", "S", "D", "dtype"))
+    o, ref = run_case(kind, B, H, S, D, dtype, fuse_ir=True, **kw)
+    if kw.get("kv_len") and 0 in kw["kv_len"]:
+        assert np.all(o[list(kw["kv_len"]).index(0)] == 0)
+    assert_close(o, ref, dtype, what=f"fused-IR {kind}")
+
+
+@pytest.mark.parametrize("idx", [2, 3, 4, 5])
+def test_fused_ir_full_configs(idx):
+    cfg = W.config(idx)
+    t = W.config_tensors(cfg)
+    from tests.gpu_util import to_dev
+    q, k, v = (to_dev(x, cfg.dtype) for x in (t.q_s, t.k_s, t.v_s))
+    kw = dict(scale=cfg.scale, out_dtype=torch.float32, fuse_ir=True)
+    if cfg.kind == "dense":
+        o = sr.mha_dense(q, k, v, kv_len=cfg.kv_len, causal=cfg.causal, **kw)
+        m = oracle.Mask(kv_len=cfg.kv_len, causal=cfg.causal)
+    elif cfg.kind == "blocksparse":
+        lay = W.config_layout(cfg)
+        o = sr.mha_blocksparse(q, k, v, lay, **kw)
+        m = oracle.Mask(kind="block", layout=lay)
+    else:
+        o = sr.mha_sliding_window(q, k, v, cfg.window, cfg.n_global, **kw)
+        m = oracle.Mask(kind="window", window=cfg.window, n_global=cfg.n_global)
+    torch.cuda.synchronize()
+    rows = _sample_rows(cfg, 192, seed=idx + 50)
+    ref = oracle.attention_rows(t.q64, t.k64, t.v64, cfg.scale, rows, m)
+    got = o.reshape(-1, cfg.D)[torch.from_numpy(rows).cuda()].double().cpu().numpy()
+    assert_close(got, ref, cfg.dtype, what=f"fused-IR config {idx}")
