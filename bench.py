@@ -139,13 +139,18 @@ class Layer:
                                      tile_n=tile_n)
             self.ws[fused] = torch.empty(info["total_bytes"], dtype=torch.uint8, device=device)
             self.T = info["tile_n"]
+        if cfg.dtype != "f32":
+            info = sr.workspace_info(self.mask, cfg.B, cfg.H, cfg.S, cfg.D, in_dt, causal=cfg.causal, tile_n=tile_n,
+                                     sd=True)
+            self.ws["sd"] = torch.empty(info["total_bytes"], dtype=torch.uint8, device=device)
         self.n_tiles, self.stored = sr.schedule_stats(self.mask, cfg.B, cfg.H, cfg.S, causal=cfg.causal, tile_n=tile_n)
 
-    def run(self, fused=True, stages=0, q=None, k=None, v=None, fuse_ir=False):
+    def run(self, fused=True, stages=0, q=None, k=None, v=None, fuse_ir=False, sd=False):
         d = self.dev
         return self.sr.call(self.mask, q if q is not None else d["q"], k if k is not None else d["k"],
                             v if v is not None else d["v"], out=self.out, fused=fused, stages=stages,
-                            workspace=self.ws[fused], tile_n=self.tile_n, fuse_ir=fuse_ir, **self.kw)
+                            workspace=self.ws["sd" if sd else fused], tile_n=self.tile_n, fuse_ir=fuse_ir, sd=sd,
+                            **self.kw)
 
 
 def timed(torch, fn, steps, warmup, flush, per_step_pre=None):
@@ -233,11 +238,13 @@ def gpu_arm(args, rank, world, local_rank):
         ms_unf = dist_max(torch, statistics.mean(timed(torch, lambda: L.run(fused=False), K, Wm, flush)), world)
 
     # ---- SURVEY NEXT-2 variant: the IR sub-layer folded into GEMM2 (SR_FUSE_IR), same workload
-    ms_fir = None
+    ms_fir = ms_sd = None
     if cfg.dtype != "f32":
         L.run(fuse_ir=True)
         barrier(torch, world)
         ms_fir = dist_max(torch, statistics.mean(timed(torch, lambda: L.run(fuse_ir=True), K, Wm, flush)), world)
+        L.run(sd=True)
+        ms_sd = dist_max(torch, statistics.mean(timed(torch, lambda: L.run(sd=True), K, Wm, flush)), world)
         L.run()  # leave the paper-design intermediates (r') in the workspace for the stage timings
 
     # ---- per-kernel durations inside the step (stage-selected launches, events on the stream)
@@ -329,7 +336,10 @@ def gpu_arm(args, rank, world, local_rank):
             "fused_ir": {"what": "IR folded into GS+GEMM2 (SURVEY NEXT-2, 2 kernels)",
                          "value": round(world * 1e3 / ms_fir, 2), "ms_per_step": round(ms_fir, 5),
                          "alg_bytes": int(sum(rec_b.values()) - 12 * L.stored / L.T - 4 * L.stored / L.T
-                                          + 8 * L.stored / L.T + 4 * L.stored / L.T)}},
+                                          + 8 * L.stored / L.T + 4 * L.stored / L.T)},
+            "sd": {"what": "decomposition without fusion: GEMM1 -> LS -> IR -> GS -> GEMM2 (PAPER.md SD, NEXT-1)",
+                   "value": round(world * 1e3 / ms_sd, 2), "ms_per_step": round(ms_sd, 5),
+                   "alg_bytes": int(sum(unf_b.values()) + 4 * L.stored + 24 * L.stored / L.T)}},
         "kernels": kern,
         "roofline": {"kernel": dom, "bound": "hbm", "achieved": round(achieved, 1), "peak": hbm_peak, "unit": "GB/s",
                      "frac": round(achieved / hbm_peak, 4), "traffic": ncu.get(f"{dom}_dram_bytes"),

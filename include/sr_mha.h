@@ -113,6 +113,12 @@ typedef struct {
  * fewer.  SURVEY.md NEXT-2 -- a B200-specific departure from the paper's separate IR kernel
  * (PAPER.md L173), off by default.  With SR_RUN_* stage bits, SR_RUN_REDUCE is then a no-op. */
 #define SR_FUSE_IR 16
+/* Variant bit: SD, the softmax decomposition WITHOUT fusion ("SD" of Fig. 8):
+ * plain GEMM1 (writes S) -> standalone LS (S -> X', m', d') -> IR -> standalone GS (X', r' -> Y)
+ * -> plain GEMM2 (reads Y).  Six attention-matrix passes; the paper's intermediate ladder step
+ * between the unfused baseline and SDF.  Workspace: sr_workspace_bytes with
+ * fused = 2. */
+#define SR_DECOMPOSE 32
 
 /* Entry points (north star).  Returns SR_OK after enqueueing the kernels on ex->stream. */
 sr_status sr_mha_dense(const void* q, const void* k, const void* v, void* out, int B, int H, int S,
@@ -159,8 +165,9 @@ typedef struct {
 } sr_ws_info;
 
 /* Workspace bytes needed by an entry point; `mask_or_layout` is the same pointer passed to it
- * (sr_dense_mask*, sr_block_layout* or sr_window*; may be NULL for dense).  fused: 1 recomposed,
- * 0 unfused.  Returns 0 on invalid/unsupported arguments (see sr_last_error()). */
+ * (sr_dense_mask*, sr_block_layout* or sr_window*; may be NULL for dense).  fused: 1 recomposed
+ * (also SR_FUSE_IR), 0 unfused, 2 SD (SR_DECOMPOSE).  Returns 0 on invalid/unsupported arguments
+ * (see sr_last_error()). */
 size_t sr_workspace_bytes(sr_entry entry, int fused, int B, int H, int S, int D, sr_dtype in_dtype,
                           const void* mask_or_layout, int causal, int tile_n);
 /* Same, with the full layout of the workspace (for tests that read X', m', d', r' back). */

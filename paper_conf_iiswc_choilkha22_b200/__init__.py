@@ -152,9 +152,10 @@ def window_mask(window: int, n_global: int) -> _Mask:
 
 # ----------------------------------------------------------------------------- queries
 
-def workspace_info(mask: _Mask, B, H, S, D, in_dtype: int, causal=False, tile_n=0, fused=True) -> dict:
+def workspace_info(mask: _Mask, B, H, S, D, in_dtype: int, causal=False, tile_n=0, fused=True, sd=False) -> dict:
     info = WsInfo()
-    _check(lib().sr_workspace_query(mask.entry, int(fused), B, H, S, D, in_dtype, mask.ptr, int(causal),
+    _check(lib().sr_workspace_query(mask.entry, 2 if (sd and fused) else int(fused), B, H, S, D, in_dtype,
+                                    mask.ptr, int(causal),
                                     int(tile_n), C.byref(info)))
     return {k: getattr(info, k) for k, _ in WsInfo._fields_}
 
@@ -199,12 +200,14 @@ _FN = {(SR_E_DENSE, True): "sr_mha_dense", (SR_E_BLOCKSPARSE, True): "sr_mha_blo
 
 SR_RUN_GEMM1, SR_RUN_REDUCE, SR_RUN_GEMM2 = 1, 2, 4
 SR_FUSE_IR = 16
+SR_DECOMPOSE = 32
 
 
 def call(mask: _Mask, q, k, v, *, scale=None, causal=False, out_dtype=None, tile_n=0, fused=True,
-         out=None, workspace=None, stream=None, stages=0, fuse_ir=False):
+         out=None, workspace=None, stream=None, stages=0, fuse_ir=False, sd=False):
     """Run one attention layer through the C ABI.  q, k, v: CUDA tensors [B, H, S, D].
-    fuse_ir=True selects the SR_FUSE_IR variant (IR folded into GEMM2)."""
+    fuse_ir=True selects the SR_FUSE_IR variant (IR folded into GEMM2, SURVEY NEXT-2);
+    sd=True the SR_DECOMPOSE variant (decomposition without fusion, the paper's SD, NEXT-1)."""
     torch = _torch()
     if not (q.is_cuda and k.is_cuda and v.is_cuda):
         raise ValueError("q, k, v must be CUDA tensors")
@@ -220,14 +223,15 @@ def call(mask: _Mask, q, k, v, *, scale=None, causal=False, out_dtype=None, tile
     out_dtype = q.dtype if out_dtype is None else out_dtype
     if out is None:
         out = torch.empty((B, H, S, D), dtype=out_dtype, device=q.device)
-    need = lib().sr_workspace_bytes(mask.entry, int(fused), B, H, S, D, in_dt, mask.ptr, int(causal), int(tile_n))
+    wmode = 2 if (sd and fused) else int(fused)
+    need = lib().sr_workspace_bytes(mask.entry, wmode, B, H, S, D, in_dt, mask.ptr, int(causal), int(tile_n))
     if need == 0:
-        raise SrError(lib().sr_workspace_query(mask.entry, int(fused), B, H, S, D, in_dt, mask.ptr, int(causal),
+        raise SrError(lib().sr_workspace_query(mask.entry, wmode, B, H, S, D, in_dt, mask.ptr, int(causal),
                                                int(tile_n), C.byref(WsInfo())), last_error())
     ws = workspace if workspace is not None else _workspace(q.device, need)
     st = torch.cuda.current_stream(q.device).cuda_stream if stream is None else stream
     ex = Exec(in_dt, dtype_code(out_dtype), ws.data_ptr(), ws.numel() * ws.element_size(), st, int(tile_n),
-              int(stages) | (SR_FUSE_IR if fuse_ir else 0))
+              int(stages) | (SR_FUSE_IR if fuse_ir else 0) | (SR_DECOMPOSE if sd else 0))
     fn = getattr(lib(), _FN[(mask.entry, bool(fused))])
     _check(fn(q.data_ptr(), k.data_ptr(), v.data_ptr(), out.data_ptr(), B, H, S, D, C.c_float(scale), mask.ptr,
               int(causal), C.byref(ex)))

@@ -329,12 +329,14 @@ void ws_layout(const HostSched& h, int B, int H, int in_dtype, int fused, sr_ws_
     size_t o = 0;
     info->off_xprime = o;
     o = align_up(o + (size_t)info->n_slots * tile_bytes, 1024);
+    // fused: 1 recomposed (X' + statistics), 0 unfused (S + P), 2 SD (X' + S/Y + statistics)
+    if (fused == 0 || fused == 2) {
+        info->off_p = o; o = align_up(o + (size_t)info->n_slots * tile_bytes, 1024);
+    }
     if (fused) {
         info->off_mprime = o; o = align_up(o + stat_bytes, 1024);
         info->off_dprime = o; o = align_up(o + stat_bytes, 1024);
         info->off_rprime = o; o = align_up(o + stat_bytes, 1024);
-    } else {
-        info->off_p = o; o = align_up(o + (size_t)info->n_slots * tile_bytes, 1024);
     }
     info->total_bytes = std::max<size_t>(o, 1024);
 }
@@ -352,10 +354,13 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
     if (!ex) return fail(SR_ERR_INVALID, "exec descriptor is NULL");
     if (!q || !k || !v || !out) return fail(SR_ERR_INVALID, "q, k, v and out must be non-NULL");
     if (!std::isfinite(scale) || !(scale > 0.f)) return fail(SR_ERR_INVALID, "scale must be finite and > 0");
-    if (ex->flags & ~(SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2 | SR_FUSE_IR))
+    if (ex->flags & ~(SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2 | SR_FUSE_IR | SR_DECOMPOSE))
         return fail(SR_ERR_INVALID, "unknown flags 0x%x", ex->flags);
-    if ((ex->flags & SR_FUSE_IR) && (!fused || ex->in_dtype == SR_F32))
-        return fail(SR_ERR_UNSUPPORTED, "SR_FUSE_IR applies to the recomposed 16-bit path only");
+    if ((ex->flags & (SR_FUSE_IR | SR_DECOMPOSE)) && (!fused || ex->in_dtype == SR_F32))
+        return fail(SR_ERR_UNSUPPORTED, "SR_FUSE_IR / SR_DECOMPOSE apply to the recomposed 16-bit path only");
+    if ((ex->flags & SR_FUSE_IR) && (ex->flags & SR_DECOMPOSE))
+        return fail(SR_ERR_INVALID, "SR_FUSE_IR and SR_DECOMPOSE are exclusive");
+    if (fused && (ex->flags & SR_DECOMPOSE)) fused = 2;  // SD: workspace mode 2
     Request r;
     sr_status s = check_request(e, B, H, S, D, ex->in_dtype, mask_or_layout, causal, ex->tile_n, r);
     if (s != SR_OK) return s;
@@ -402,13 +407,14 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
         p.mprime = (float*)(ws + wi.off_mprime);
         p.dprime = (float*)(ws + wi.off_dprime);
         p.rprime = (float*)(ws + wi.off_rprime);
-    } else {
-        p.pbuf = ws + wi.off_p;
     }
+    if (fused != 1) p.pbuf = ws + wi.off_p;
     cudaStream_t st = (cudaStream_t)ex->stream;
     int64_t nl = 0;
     cudaError_t ce;
-    if (fused) {
+    if (fused == 2) {
+        ce = launch_tc_sd(p, st, &nl);
+    } else if (fused) {
         ce = ex->in_dtype == SR_F32 ? launch_simt_f32(p, st, &nl) : launch_tc_fused(p, st, &nl);
     } else {
         ce = launch_tc_unfused(p, st, &nl);

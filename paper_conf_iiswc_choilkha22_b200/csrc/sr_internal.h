@@ -109,5 +109,6 @@ cudaError_t launch_simt_f32(const Params& p, cudaStream_t st, int64_t* nlaunch);
 cudaError_t launch_ir(const Params& p, cudaStream_t st, int64_t* nlaunch);
 cudaError_t launch_tc_fused(const Params& p, cudaStream_t st, int64_t* nlaunch);
 cudaError_t launch_tc_unfused(const Params& p, cudaStream_t st, int64_t* nlaunch);
+cudaError_t launch_tc_sd(const Params& p, cudaStream_t st, int64_t* nlaunch);
 
 }  // namespace sr

@@ -368,3 +368,25 @@ def test_fused_ir_full_configs(idx):
     ref = oracle.attention_rows(t.q64, t.k64, t.v64, cfg.scale, rows, m)
     got = o.reshape(-1, cfg.D)[torch.from_numpy(rows).cuda()].double().cpu().numpy()
     assert_close(got, ref, cfg.dtype, what=f"fused-IR config {idx}")
+
+
+# ------------------------------------------------------------------------------------ SD variant
+
+@pytest.mark.parametrize("kind,kw", FUSED_IR_CASES, ids=lambda x: str(x)[:40] if isinstance(x, dict) else x)
+def test_sd_variant(kind, kw):
+    """SR_DECOMPOSE (the paper's SD: standalone LS / IR / GS between plain GEMMs, NEXT-1)."""
+    kw = dict(kw)
+    if kw.get("layout") == "rand":
+        kw["layout"] = W.random_layout(kw["H"], kw["S"] // 64, 64, 0.35, seed=8)
+    B, H, S, D, dtype = (kw.pop(x) for x in ("B", "H", "S", "D", "dtype"))
+    t, q, k, v = qkv(B, H, S, D, dtype, 0)
+    scale = 1 / math.sqrt(D)
+    mk = {"dense": sr.dense_mask(kw.get("kv_len")), "block": sr.block_mask(kw["layout"]) if "layout" in kw else None,
+          "window": sr.window_mask(kw.get("window", 0), kw.get("n_global", 0))}[kind]
+    o = sr.call(mk, q, k, v, scale=scale, causal=kw.get("causal", False), tile_n=kw.get("tile_n", 0),
+                out_dtype=torch.float32, sd=True)
+    torch.cuda.synchronize()
+    ref = oracle.attention(t.q64, t.k64, t.v64, scale,
+                           oracle_mask(kind, kw.get("kv_len"), kw.get("causal", False), kw.get("layout"),
+                                       kw.get("window", 0), kw.get("n_global", 0)))
+    assert_close(o.double().cpu().numpy(), ref, dtype, what=f"SD {kind}")
