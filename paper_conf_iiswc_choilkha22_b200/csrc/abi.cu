@@ -14,6 +14,7 @@
 #include <map>
 #include <memory>
 #include <mutex>
+#include <queue>
 #include <string>
 #include <vector>
 
@@ -41,8 +42,9 @@ int dtype_bytes(int dt) { return dt == SR_F32 ? 4 : 2; }
 // ------------------------------------------------------------------------------ schedules
 
 struct HostSched {
-    int T = 0, n_rb = 0, n_lh = 1, lh_mode = LH_ONE;
+    int T = 0, H = 1, n_rb = 0, n_lh = 1, lh_mode = LH_ONE;
     std::vector<int32_t> tp, tinfo, items, kv_len;
+    std::vector<int32_t> cta_ptr;  // device schedules only: items grouped per persistent CTA
     int slots_per_head = 0;
     int64_t n_tiles = 0;       // over all B*H heads
     int64_t stored_elems = 0;  // valid 64-row halves x 64 x T, over all heads
@@ -79,6 +81,7 @@ sr_status build_sched(const Request& r, HostSched& hs)
 {
     const int S = r.S, T = r.T;
     hs.T = T;
+    hs.H = r.H;
     hs.n_rb = S / kRowBlock;
     const int nkt = S / T;
     std::vector<std::vector<std::pair<int, int>>> lists;  // per (lh, rb): (kt, half bits)
@@ -264,10 +267,44 @@ std::string sched_key(const Request& r, int device)
     return k;
 }
 
+// Greedy longest-processing-time assignment of the (already longest-first) items to n_cta
+// persistent CTAs: each item goes to the CTA with the least work so far.  Cost of an item =
+// 2 x its tiles + 1 (the Q load / O store of a row-block is about half a tile's traffic).  Items
+// are regrouped per CTA in assignment order, so the first wave is the round-robin one (neighbouring
+// CTAs run items of the same head at the same time and share its K/V tiles in L2).
+void lpt_assign(HostSched& h, int n_cta)
+{
+    const size_t n = h.items.size();
+    n_cta = (int)std::max<size_t>(1, std::min<size_t>(n, (size_t)std::max(n_cta, 1)));
+    std::vector<int> owner(n);
+    std::vector<int32_t> count(n_cta, 0);
+    using E = std::pair<int64_t, int>;  // (load, cta)
+    std::priority_queue<E, std::vector<E>, std::greater<E>> pq;
+    for (int c = 0; c < n_cta; ++c) pq.push({0, c});
+    for (size_t i = 0; i < n; ++i) {
+        const int32_t w = h.items[i];
+        const int g = w / h.n_rb, rb = w % h.n_rb;
+        const int lh = h.lh_mode == LH_ONE ? 0 : (h.lh_mode == LH_BATCH ? g / h.H : g % h.H);
+        const int32_t* tp = &h.tp[(size_t)lh * (h.n_rb + 1)];
+        E e = pq.top();
+        pq.pop();
+        owner[i] = e.second;
+        ++count[e.second];
+        e.first += 2 * (int64_t)(tp[rb + 1] - tp[rb]) + 1;
+        pq.push(e);
+    }
+    h.cta_ptr.assign(n_cta + 1, 0);
+    for (int c = 0; c < n_cta; ++c) h.cta_ptr[c + 1] = h.cta_ptr[c] + count[c];
+    std::vector<int32_t> fill(h.cta_ptr.begin(), h.cta_ptr.end() - 1), out(n);
+    for (size_t i = 0; i < n; ++i) out[fill[owner[i]]++] = h.items[i];
+    h.items.swap(out);
+}
+
 // Host schedule only (no device), used by queries.
 sr_status host_sched(const Request& r, std::shared_ptr<CachedSched>& out, bool need_device)
 {
     int dev = -1;
+    cudaError_t ce0 = cudaSuccess;
     if (need_device) {
         cudaError_t ce = cudaGetDevice(&dev);
         if (ce != cudaSuccess) return fail(SR_ERR_CUDA, "cudaGetDevice: %s", cudaGetErrorString(ce));
@@ -281,9 +318,13 @@ sr_status host_sched(const Request& r, std::shared_ptr<CachedSched>& out, bool n
     if (s != SR_OK) return s;
     if (need_device) {
         HostSched& h = cs->hs;
+        int n_sm = 148;
+        if ((ce0 = cudaDeviceGetAttribute(&n_sm, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess)
+            return fail(SR_ERR_CUDA, "cudaDeviceGetAttribute: %s", cudaGetErrorString(ce0));
+        lpt_assign(h, n_sm);
         size_t n_tp = h.tp.size(), n_ti = std::max<size_t>(h.tinfo.size(), 1), n_it = h.items.size(),
                n_kv = h.kv_len.size();
-        size_t bytes = sizeof(int32_t) * (n_tp + n_ti + n_it + n_kv + 4);
+        size_t bytes = sizeof(int32_t) * (n_tp + n_ti + n_it + n_kv + h.cta_ptr.size() + 4);
         cudaError_t ce = cudaMalloc(&cs->dmem, bytes);
         if (ce != cudaSuccess) return fail(SR_ERR_CUDA, "cudaMalloc(schedule): %s", cudaGetErrorString(ce));
         std::vector<int32_t> blob;
@@ -296,6 +337,8 @@ sr_status host_sched(const Request& r, std::shared_ptr<CachedSched>& out, bool n
         blob.insert(blob.end(), h.items.begin(), h.items.end());
         size_t o_kv = blob.size();
         blob.insert(blob.end(), h.kv_len.begin(), h.kv_len.end());
+        size_t o_cp = blob.size();
+        blob.insert(blob.end(), h.cta_ptr.begin(), h.cta_ptr.end());
         ce = cudaMemcpy(cs->dmem, blob.data(), blob.size() * 4, cudaMemcpyHostToDevice);
         if (ce != cudaSuccess) return fail(SR_ERR_CUDA, "cudaMemcpy(schedule): %s", cudaGetErrorString(ce));
         int32_t* base = (int32_t*)cs->dmem;
@@ -308,6 +351,8 @@ sr_status host_sched(const Request& r, std::shared_ptr<CachedSched>& out, bool n
         cs->dev.lh_mode = h.lh_mode;
         cs->dev.slots_per_head = h.slots_per_head;
         cs->dev.n_items = (int)h.items.size();
+        cs->dev.cta_ptr = base + o_cp;
+        cs->dev.n_cta = (int)h.cta_ptr.size() - 1;
     }
     g_cache[key] = cs;
     out = cs;

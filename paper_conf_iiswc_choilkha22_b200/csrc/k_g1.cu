@@ -112,7 +112,8 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
     // own prologue, then wait for our producer kernel's results before touching them
     griddep_launch_dependents();
     griddep_wait();
-    const int n_items = p.sc.n_items;
+    // this CTA's items: a contiguous range of the longest-processing-time assignment (host)
+    const int it_begin = __ldg(p.sc.cta_ptr + blockIdx.x), it_end = __ldg(p.sc.cta_ptr + blockIdx.x + 1);
 
     if (warp < 4) {
         // warpgroup 0 hands registers to the epilogue warpgroups.  setmaxnreg.inc can only draw what
@@ -125,7 +126,7 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
             // -------------------------------------------------------------- TMA producer
             int qi = 0, ks = 0;
             uint32_t qph = 0, kph = 0;
-            for (int it = blockIdx.x; it < n_items; it += gridDim.x) {
+            for (int it = it_begin; it < it_end; ++it) {
                 const ItemInfo I = decode_item(p, it);
                 if (I.t0 == I.t1) continue;
                 const int row0 = I.g * p.S + I.rb * kRowBlock;
@@ -159,7 +160,7 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
             const uint32_t idesc = idesc_f16(p.in_dtype == DT_BF16 ? 1 : 0, kRowBlock, kMW, 0, 0);
             int qi = 0, ks = 0, n = 0;
             uint32_t qph = 0, kph = 0;
-            for (int it = blockIdx.x; it < n_items; it += gridDim.x) {
+            for (int it = it_begin; it < it_end; ++it) {
                 const ItemInfo I = decode_item(p, it);
                 if (I.t0 == I.t1) continue;
                 const int kvl = p.sc.kv_len ? __ldg(p.sc.kv_len + I.g / p.H) : p.S;
@@ -485,7 +486,7 @@ cudaError_t launch_g1_t(const Params& p, cudaStream_t st, int64_t* nl)
     if ((e = make_tmap_2d(&tk, p.k, rows, D, T, p.in_dtype)) != cudaSuccess) return e;
     auto kern = tc_gemm1<D, T, LS>;
     if ((e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM)) != cudaSuccess) return e;
-    const int grid = std::min(p.sc.n_items, num_sms());
+    const int grid = p.sc.n_cta;  // one persistent CTA per SM, items assigned by host LPT
     return launch_pdl(kern, dim3(grid), dim3(C::THREADS), C::SMEM, st, nl, tq, tk, p);
 }
 

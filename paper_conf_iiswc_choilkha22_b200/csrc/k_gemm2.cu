@@ -115,7 +115,8 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
     griddep_wait();
     const uint32_t tmem_o = tmem_base;              // NO x D columns
     const uint32_t tmem_a = tmem_base + C::NO * D;  // NA x MW/2 columns
-    const int n_items = p.sc.n_items;
+    // this CTA's items: a contiguous range of the longest-processing-time assignment (host)
+    const int it_begin = __ldg(p.sc.cta_ptr + blockIdx.x), it_end = __ldg(p.sc.cta_ptr + blockIdx.x + 1);
     const uint8_t* src = (const uint8_t*)(GS ? p.xprime : p.pbuf);
 
     if (warp == 0) {
@@ -123,7 +124,7 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
             // -------------------------------------------------------------- X' producer
             int s = 0;
             uint32_t sph = 0;
-            for (int it = blockIdx.x; it < n_items; it += gridDim.x) {
+            for (int it = it_begin; it < it_end; ++it) {
                 const ItemInfo I = decode_item(p, it);
                 int wn[2];  // schedule words of the next macro tile, prefetched one step ahead
                 for (int u = 0; u < NSUB; ++u) wn[u] = I.t0 + u < I.t1 ? __ldg(p.sc.tinfo + I.t0 + u) : 0;
@@ -169,7 +170,7 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
             // L147), published as (m, 1/d) in a ring of NSI items.  Lane l reduces rows l + 32j.
             int si = 0;
             uint32_t sph = 0;
-            for (int it = blockIdx.x; it < n_items; it += gridDim.x) {
+            for (int it = it_begin; it < it_end; ++it) {
                 const ItemInfo I = decode_item(p, it);
                 if (I.t0 == I.t1) continue;
                 mbar_wait(&st_empty[si], sph ^ 1);
@@ -225,7 +226,7 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
             // -------------------------------------------------------------- V producer
             int s = 0;
             uint32_t sph = 0;
-            for (int it = blockIdx.x; it < n_items; it += gridDim.x) {
+            for (int it = it_begin; it < it_end; ++it) {
                 const ItemInfo I = decode_item(p, it);
                 int wn[2];  // schedule words of the next macro tile, prefetched one step ahead
                 for (int u = 0; u < NSUB; ++u) wn[u] = I.t0 + u < I.t1 ? __ldg(p.sc.tinfo + I.t0 + u) : 0;
@@ -258,10 +259,10 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
                 if (++o == C::NO) { o = 0; oph ^= 1; }
             };
             ItemInfo nxt;
-            if ((int)blockIdx.x < n_items) nxt = decode_item(p, blockIdx.x);
-            for (int it = blockIdx.x; it < n_items; it += gridDim.x) {
+            if (it_begin < it_end) nxt = decode_item(p, it_begin);
+            for (int it = it_begin; it < it_end; ++it) {
                 const ItemInfo I = nxt;
-                if (it + (int)gridDim.x < n_items) nxt = decode_item(p, it + gridDim.x);  // prefetch
+                if (it + 1 < it_end) nxt = decode_item(p, it + 1);  // prefetch
                 const int64_t orow = (int64_t)I.g * p.S + I.rb * kRowBlock;
                 if (I.t0 == I.t1) {  // no kept key in these rows: the epilogue writes zeros
                     post(SH_EMPTY, orow);
@@ -453,7 +454,7 @@ cudaError_t launch_g2_t(const Params& p, cudaStream_t st, int64_t* nl)
     if ((e = make_tmap_2d(&tv, p.v, rows, D, T, p.in_dtype)) != cudaSuccess) return e;
     auto kern = tc_gemm2<D, T, GS, FI>;
     if ((e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM)) != cudaSuccess) return e;
-    const int grid = std::min(p.sc.n_items, num_sms());
+    const int grid = p.sc.n_cta;  // one persistent CTA per SM, items assigned by host LPT
     return launch_pdl(kern, dim3(grid), dim3(C::THREADS), C::SMEM, st, nl, tv, p);
 }
 

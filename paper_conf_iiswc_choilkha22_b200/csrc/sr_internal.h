@@ -34,9 +34,10 @@ __host__ __device__ inline int tinfo_half(int32_t w) { return (w >> 16) & 3; }
 struct DevSched {
     const int32_t* tp;      // [n_lh][n_rb+1] absolute offsets into tinfo
     const int32_t* tinfo;   // [n_tiles_list]
-    const int32_t* items;   // [n_items] g * n_rb + rb, longest first
+    const int32_t* items;   // [n_items] g * n_rb + rb; grouped by persistent CTA, longest first
+    const int32_t* cta_ptr; // [n_cta + 1]: CTA c runs items[cta_ptr[c] .. cta_ptr[c+1])
     const int32_t* kv_len;  // [B] or nullptr
-    int n_rb, n_lh, lh_mode, slots_per_head, n_items;
+    int n_rb, n_lh, lh_mode, slots_per_head, n_items, n_cta;
 };
 
 // Everything a kernel needs to know about one call.
