@@ -22,7 +22,8 @@ from typing import Optional
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libsr_mha.so")
+# SR_MHA_LIB: an experiment build of the same library (build.py --define ... --out PATH)
+LIB_PATH = os.environ.get("SR_MHA_LIB") or os.path.join(_HERE, "libsr_mha.so")
 
 SR_OK, SR_ERR_INVALID, SR_ERR_UNSUPPORTED, SR_ERR_WORKSPACE, SR_ERR_CUDA = range(5)
 SR_F32, SR_F16, SR_BF16 = 0, 1, 2

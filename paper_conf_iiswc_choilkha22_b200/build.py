@@ -1,6 +1,8 @@
 """Build libsr_mha.so in-tree: nvcc for sm_100a, one object per .cu, linked into one shared library.
 
 Usage: python -m paper_conf_iiswc_choilkha22_b200.build [--force] [--verbose]
+       [--define NAME=VALUE ...] [--out PATH]   (experiment builds: extra -D flags, another .so; load
+                                                  it with SR_MHA_LIB=PATH)
 """
 from __future__ import annotations
 
@@ -26,14 +28,15 @@ def _deps():
     return max(os.path.getmtime(f) for f in files)
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and os.path.exists(LIB) and os.path.getmtime(LIB) >= _deps():
-        return LIB
-    os.makedirs(BUILD, exist_ok=True)
-    extra = ["-Xptxas", "-v"] if verbose else []
+def build(force: bool = False, verbose: bool = False, defines=(), out: str = LIB) -> str:
+    if not force and not defines and os.path.exists(out) and os.path.getmtime(out) >= _deps():
+        return out
+    bdir = BUILD if not defines else os.path.join(BUILD, "x_" + "_".join(d.replace("=", "") for d in defines))
+    os.makedirs(bdir, exist_ok=True)
+    extra = (["-Xptxas", "-v"] if verbose else []) + [f"-D{d}" for d in defines]
 
     def compile_one(src):
-        obj = os.path.join(BUILD, src.replace(".cu", ".o"))
+        obj = os.path.join(bdir, src.replace(".cu", ".o"))
         cmd = [NVCC, *FLAGS, *extra, "-c", os.path.join(CSRC, src), "-o", obj]
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
@@ -44,14 +47,17 @@ def build(force: bool = False, verbose: bool = False) -> str:
 
     with ThreadPoolExecutor(max_workers=len(SOURCES)) as ex:
         objs = list(ex.map(compile_one, SOURCES))
-    tmp = LIB + f".tmp{os.getpid()}"
+    tmp = out + f".tmp{os.getpid()}"
     cmd = [NVCC, "-gencode", "arch=compute_100a,code=sm_100a", "-shared", "-o", tmp, *objs]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError(f"link failed:\n{r.stdout}\n{r.stderr}")
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, out)
+    return out
 
 
 if __name__ == "__main__":
-    print(build(force="--force" in sys.argv, verbose="--verbose" in sys.argv))
+    a = sys.argv[1:]
+    defs = [a[i + 1] for i, x in enumerate(a) if x == "--define"]
+    o = next((a[i + 1] for i, x in enumerate(a) if x == "--out"), LIB)
+    print(build(force="--force" in a, verbose="--verbose" in a, defines=defs, out=os.path.abspath(o)))

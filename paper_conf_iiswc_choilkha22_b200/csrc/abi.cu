@@ -46,6 +46,7 @@ struct HostSched {
     std::vector<int32_t> tp, tinfo, items, kv_len;
     std::vector<int32_t> cta_ptr;  // device schedules only: items grouped per persistent CTA
     int slots_per_head = 0;
+    int max_rb_tiles = 0;
     int64_t n_tiles = 0;       // over all B*H heads
     int64_t stored_elems = 0;  // valid 64-row halves x 64 x T, over all heads
 };
@@ -142,6 +143,7 @@ sr_status build_sched(const Request& r, HostSched& hs)
                 lh_elems[lh] += (int64_t)__builtin_popcount(kb.second) * kHalf * T;
                 lh_tiles[lh] += 1;
             }
+            hs.max_rb_tiles = std::max<int>(hs.max_rb_tiles, (int)hs.tinfo.size() - off);
             off = (int32_t)hs.tinfo.size();
             hs.tp[(size_t)lh * (hs.n_rb + 1) + rb + 1] = off;
         }
@@ -350,6 +352,8 @@ sr_status host_sched(const Request& r, std::shared_ptr<CachedSched>& out, bool n
         cs->dev.n_lh = h.n_lh;
         cs->dev.lh_mode = h.lh_mode;
         cs->dev.slots_per_head = h.slots_per_head;
+        cs->dev.max_rb_tiles = h.max_rb_tiles;
+        cs->dev.mean_rb_tiles = (int)((h.tinfo.size() + (size_t)h.n_lh * h.n_rb - 1) / ((size_t)h.n_lh * h.n_rb));
         cs->dev.n_items = (int)h.items.size();
         cs->dev.cta_ptr = base + o_cp;
         cs->dev.n_cta = (int)h.cta_ptr.size() - 1;

@@ -36,6 +36,12 @@ namespace sr {
 using namespace ptx;
 
 constexpr int kMW = 128;  // macro tile width (MMA N of GEMM1)
+// Of every 8 element pairs of the LS exponentials, this many are computed by ex2_poly2 on the FMA
+// pipe and the rest by MUFU.EX2 (16 / clock / SM): balances the two pipes in the epilogue.
+#ifndef SR_G1_POLY_PAIRS
+#define SR_G1_POLY_PAIRS 0
+#endif
+constexpr int kPolyPairs = SR_G1_POLY_PAIRS;
 
 struct G1Hdr {  // per-accumulator macro-tile header, written by the MMA warp
     int32_t slot_lo, slot_hi, i0, kvl, w0, w1, flags, pad;
@@ -57,7 +63,10 @@ struct G1 {
     // staging buffers per epilogue warpgroup (2 if at all possible: the X' store stream is the
     // bottleneck), then Q double-buffered if shared memory still allows
     static constexpr int XPW = (QB + 2 * KB + EPI_WG * 2 * SB + 4096 <= kSmemMax) ? 2 : 1;
-    static constexpr int NQ = (2 * QB + 2 * KB + EPI_WG * XPW * SB + 4096 <= kSmemMax) ? 2 : 1;
+#ifndef SR_G1_MAX_NQ
+#define SR_G1_MAX_NQ 2
+#endif
+    static constexpr int NQ = (SR_G1_MAX_NQ >= 2 && 2 * QB + 2 * KB + EPI_WG * XPW * SB + 4096 <= kSmemMax) ? 2 : 1;
     static constexpr int NK_ = (kSmemMax - 4096 - NQ * QB - EPI_WG * XPW * SB) / KB;
     static constexpr int NK = NK_ > 4 ? 4 : NK_;
     static_assert(NK >= 2, "smem budget");
@@ -279,8 +288,18 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
                     for (int u = 0; u < 64; u += 2) {
                         float t0, t1;
                         ffma2(t0, t1, __uint_as_float(x[u]), __uint_as_float(x[u + 1]), sl2, neg);
-                        x[u] = __float_as_uint(ex2(t0));
-                        x[u + 1] = __float_as_uint(ex2(t1));
+                        float y0, y1;
+#ifdef SR_DIAG_NOEXP
+                        if (true) { y0 = t0; y1 = t1; } else
+#endif
+                        if (((u >> 1) & 7) < kPolyPairs) {
+                            ex2_poly2(y0, y1, t0, t1);
+                        } else {
+                            y0 = ex2(t0);
+                            y1 = ex2(t1);
+                        }
+                        x[u] = __float_as_uint(y0);
+                        x[u + 1] = __float_as_uint(y1);
                     }
                     // d' = sum X' (fp32, FADD2 into 4 independent pair accumulators)
                     float sa[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
@@ -407,8 +426,18 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
                     for (int u = 0; u < T; u += 2) {
                         float t0, t1;
                         ffma2(t0, t1, __uint_as_float(x[u]), __uint_as_float(x[u + 1]), sl2, neg);
-                        x[u] = __float_as_uint(ex2(t0));
-                        x[u + 1] = __float_as_uint(ex2(t1));
+                        float y0, y1;
+#ifdef SR_DIAG_NOEXP
+                        if (true) { y0 = t0; y1 = t1; } else
+#endif
+                        if (((u >> 1) & 7) < kPolyPairs) {
+                            ex2_poly2(y0, y1, t0, t1);
+                        } else {
+                            y0 = ex2(t0);
+                            y1 = ex2(t1);
+                        }
+                        x[u] = __float_as_uint(y0);
+                        x[u + 1] = __float_as_uint(y1);
                     }
                     // d' = sum X' (fp32, FADD2 into 4 independent pair accumulators)
                     float sa[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
@@ -446,8 +475,12 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
                     if (!wv[s]) continue;
                     uint8_t* dst = (uint8_t*)p.xprime + (slot + s) * (int64_t)C::XS;
                     for (int ch = 0; ch < T / 64; ++ch)
+#ifndef SR_DIAG_NOSTORE
                         bulk_store(dst + ch * (kRowBlock * 128) + wrow0 * 128,
                                    stage + (s * (T / 64) + ch) * (kRowBlock * 128) + wrow0 * 128, 32 * 128);
+#else
+                        (void)dst;
+#endif
                 }
                 bulk_commit();
             }

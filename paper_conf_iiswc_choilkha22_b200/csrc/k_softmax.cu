@@ -1,77 +1,220 @@
 // k_softmax.cu -- the unfused baseline's softmax kernel (a row vector per thread
-// block held in on-chip memory; reads the attention matrix once and writes it once).  Part of the
+// block held in on-chip memory; the attention matrix is read once and written once).  Part of the
 // in-repo traffic baseline only; the recomposed path never runs it.
+//
+// One CTA per (row-block, slice of R rows): every score tile of the row-block holds the slice's R
+// rows of each 64-key chunk as R x 128 contiguous bytes (SWIZZLE_128B tile layout), so the CTA pulls
+// the slice's whole score rows into shared memory with one bulk copy per chunk (all in flight at
+// once), computes the safe softmax of Eq. (1) row by row in place (one warp per row: max, sum of
+// exponentials, normalised write), and bulk-stores P back.  R = 32 down to 2, chosen on the host so
+// the slice takes <= 48 KB (several CTAs per SM then overlap one CTA's loads with another's
+// arithmetic and stores): sized for the longest rows when that leaves R >= 8, else for the mean
+// row, and the few longer rows (global tokens) go through shared memory in groups, twice (online
+// max and sum, then the normalised write).  A memory-bound kernel meant to run at HBM bandwidth: a fair
+// baseline for the fused path's traffic savings.
 #include "tc_common.cuh"
 
 namespace sr {
 
 using namespace ptx;
 
-// One warp per query row (the paper's baseline keeps one row vector per TB in on-chip memory,
-// PAPER.md L102): read the row's score pieces once into shared memory, max, sum, write P once.
+constexpr int kSmBudget = 48 * 1024, kSmBudgetMax = 160 * 1024;
+
 template <int T>
-__global__ void __launch_bounds__(128) row_softmax(const Params p)
+__global__ void __launch_bounds__(256) row_softmax(const Params p, int R, int cap)  // min(R, 8) warps
 {
-    extern __shared__ uint32_t rowbuf[];  // per warp: S/2 words (fp16 pairs of this row)
-    const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
-    const int64_t row = (int64_t)blockIdx.x * 4 + warp;
-    if (row >= (int64_t)p.B * p.H * p.S) return;
-    uint32_t* buf = rowbuf + (size_t)warp * (p.S / 2);
-    const int g = (int)(row / p.S), i = (int)(row % p.S);
-    const int rb = i / kRowBlock, r = i % kRowBlock, myhalf = r / kHalf;
-    const DevSched& sc = p.sc;
-    const int lh = lh_of(sc, g, p.H);
-    const int32_t* tp = sc.tp + (size_t)lh * (sc.n_rb + 1);
-    const int t0 = tp[rb], t1 = tp[rb + 1];
-    const int64_t slot0 = (int64_t)g * sc.slots_per_head - tp[0];
+    extern __shared__ __align__(128) uint8_t rows[];  // [chunk][R rows][128 B]
+    __shared__ uint64_t bar;
+    __shared__ int n_chunks;
     constexpr int XB = kRowBlock * T * 2;
-    float mx = -INFINITY;
-    int nw = 0;
-    for (int t = t0; t < t1; ++t) {
-        if (!((tinfo_half(sc.tinfo[t]) >> myhalf) & 1)) continue;
-        const uint8_t* tile = (const uint8_t*)p.xprime + (slot0 + t) * (int64_t)XB;
-        for (int ch = 0; ch < T / 64; ++ch) {
-            const uint32_t w = *reinterpret_cast<const uint32_t*>(tile + ch * (kRowBlock * 128) + r * 128 + lane * 4);
-            buf[nw * 32 + lane] = w;
-            const float2 f = unpack_f16(w);
-            mx = fmaxf(mx, fmaxf(f.x, f.y));
-            ++nw;
+    const DevSched& sc = p.sc;
+    const int nsl = kRowBlock / R;
+    const int item = blockIdx.x / nsl;  // g * n_rb + rb
+    const int r0 = (blockIdx.x % nsl) * R;
+    const int g = item / sc.n_rb, rb = item % sc.n_rb;
+    const int myhalf = r0 / kHalf;  // R <= 64: the slice lies in one 64-row half
+    const int32_t* tp = sc.tp + (size_t)lh_of(sc, g, p.H) * (sc.n_rb + 1);
+    griddep_launch_dependents();
+    griddep_wait();
+    const int t0 = __ldg(tp + rb), t1 = __ldg(tp + rb + 1);
+    const int64_t slot0 = (int64_t)g * sc.slots_per_head - __ldg(tp);
+    const uint32_t slice = (uint32_t)R * 128;
+    // bulk copies of the slice's chunks k0 .. k1-1 (in row order) between HBM and shared memory
+    auto copy_chunks = [&](int k0, int k1, bool load) {
+        int k = 0;
+        for (int t = t0; t < t1 && k < k1; ++t) {
+            if (!((tinfo_half(__ldg(sc.tinfo + t)) >> myhalf) & 1)) continue;
+            const int64_t off = (slot0 + t) * (int64_t)XB + r0 * 128;
+            for (int ch = 0; ch < T / 64; ++ch, ++k) {
+                if (k < k0 || k >= k1) continue;
+                uint8_t* sm = rows + (k - k0) * slice;
+                if (load) bulk_load(sm, (const uint8_t*)p.xprime + off + ch * (kRowBlock * 128), slice, &bar);
+                else bulk_store((uint8_t*)p.pbuf + off + ch * (kRowBlock * 128), sm, slice);
+            }
+        }
+    };
+    if (threadIdx.x == 0) {
+        int n = 0;
+        for (int t = t0; t < t1; ++t) n += ((tinfo_half(__ldg(sc.tinfo + t)) >> myhalf) & 1) ? T / 64 : 0;
+        n_chunks = n;
+        mbar_init(&bar, 1);
+        fence_mbar_init();
+        if (n) {
+            mbar_arrive_expect_tx(&bar, min(n, cap) * slice);
+            copy_chunks(0, min(n, cap), true);
         }
     }
-    for (int o = 16; o > 0; o >>= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+    __syncthreads();
+    const int nck = n_chunks;
+    if (nck == 0) return;
+    const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
     const float l2e = 1.4426950408889634f;
-    const float neg = mx == -INFINITY ? 0.f : -mx * l2e;
-    float sum = 0.f;
-    for (int k = 0; k < nw; ++k) {
-        const float2 f = unpack_f16(buf[k * 32 + lane]);
-        sum += ex2(fmaf(f.x, l2e, neg)) + ex2(fmaf(f.y, l2e, neg));
-    }
-    for (int o = 16; o > 0; o >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, o);
-    const float inv = sum > 0.f ? 1.f / sum : 0.f;
     const bool bf = p.in_dtype == DT_BF16;
-    int k = 0;
-    for (int t = t0; t < t1; ++t) {
-        if (!((tinfo_half(sc.tinfo[t]) >> myhalf) & 1)) continue;
-        uint8_t* tile = (uint8_t*)p.pbuf + (slot0 + t) * (int64_t)XB;
-        for (int ch = 0; ch < T / 64; ++ch, ++k) {
-            const float2 f = unpack_f16(buf[k * 32 + lane]);
-            const float y0 = ex2(fmaf(f.x, l2e, neg)) * inv, y1 = ex2(fmaf(f.y, l2e, neg)) * inv;
-            *reinterpret_cast<uint32_t*>(tile + ch * (kRowBlock * 128) + r * 128 + lane * 4) =
-                bf ? pack_bf16(y0, y1) : pack_f16(y0, y1);
+    const int nwarps = blockDim.x / 32;
+    const int ngrp = (nck + cap - 1) / cap;  // > 1: rows longer than the slice capacity
+    if (ngrp == 1) {  // the whole row slice is on chip: max, then e = e^{x - m} (kept, fp16) and its
+                      // sum, then P = e / sum -- one exponential per element
+        mbar_wait(&bar, 0);
+        for (int rr = warp; rr < R; rr += nwarps) {
+            const uint32_t base = smem_u32(rows) + rr * 128 + lane * 4;  // lane: 2 keys of every chunk
+            float m = -INFINITY;
+            for (int k = 0; k < nck; ++k) {
+                const float2 f = unpack_f16(lds_u32(base + k * slice));
+                m = fmaxf(m, fmaxf(f.x, f.y));
+            }
+            for (int o = 16; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+            const float neg = m == -INFINITY ? 0.f : -m * l2e;
+            float s = 0.f;
+            for (int k = 0; k < nck; ++k) {
+                const float2 f = unpack_f16(lds_u32(base + k * slice));
+                const float e0 = ex2(fmaf(f.x, l2e, neg)), e1 = ex2(fmaf(f.y, l2e, neg));
+                s += e0 + e1;
+                sts_u32(base + k * slice, pack_f16(e0, e1));
+            }
+            for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+            const float inv = s > 0.f ? 1.f / s : 0.f;
+            for (int k = 0; k < nck; ++k) {
+                const float2 e = unpack_f16(lds_u32(base + k * slice));
+                sts_u32(base + k * slice, bf ? pack_bf16(e.x * inv, e.y * inv) : pack_f16(e.x * inv, e.y * inv));
+            }
+        }
+        fence_proxy_async_smem();
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            copy_chunks(0, nck, false);
+            bulk_commit();
+            bulk_wait_read0();
+        }
+        return;
+    }
+    uint32_t ph = 0;
+    // rows longer than the slice: pass 1 over groups of `cap` chunks, per-lane online max and sum
+    float mx[4], sm_[4];  // rows warp + 8j of this warp (R <= 32, nwarps = min(R, 8))
+#pragma unroll
+    for (int j = 0; j < 4; ++j) { mx[j] = -INFINITY; sm_[j] = 0.f; }
+    for (int gi = 0; gi < ngrp; ++gi) {
+        const int nk = min(cap, nck - gi * cap);
+        if (gi > 0) {
+            __syncthreads();  // everyone is done with the previous group
+            if (threadIdx.x == 0) {
+                mbar_arrive_expect_tx(&bar, nk * slice);
+                copy_chunks(gi * cap, gi * cap + nk, true);
+            }
+        }
+        mbar_wait(&bar, ph);
+        ph ^= 1;
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            const int rr = warp + j * nwarps;
+            if (rr >= R) break;
+            const uint32_t base = smem_u32(rows) + rr * 128 + lane * 4;  // lane: 2 keys of every chunk
+            float m = mx[j];
+            for (int k = 0; k < nk; ++k) {
+                const float2 f = unpack_f16(lds_u32(base + k * slice));
+                m = fmaxf(m, fmaxf(f.x, f.y));
+            }
+            const float neg = m == -INFINITY ? 0.f : -m * l2e;
+            float s = mx[j] == -INFINITY ? 0.f : sm_[j] * ex2(fmaf(mx[j], l2e, neg));
+            for (int k = 0; k < nk; ++k) {
+                const float2 f = unpack_f16(lds_u32(base + k * slice));
+                s += ex2(fmaf(f.x, l2e, neg)) + ex2(fmaf(f.y, l2e, neg));
+            }
+            mx[j] = m;
+            sm_[j] = s;
         }
     }
+    // warp reductions of the row statistics
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+        float m = mx[j];
+        for (int o = 16; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+        float s = mx[j] == -INFINITY ? 0.f : sm_[j] * ex2((mx[j] - m) * l2e);
+        for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+        mx[j] = m == -INFINITY ? 0.f : -m * l2e;  // now: the exponent offset
+        sm_[j] = s > 0.f ? 1.f / s : 0.f;          // now: 1 / row sum
+    }
+    // pass 2: P = e^{x - m} / d, in place, then out with bulk stores (re-loading groups if needed)
+    for (int gi = 0; gi < ngrp; ++gi) {
+        const int nk = min(cap, nck - gi * cap);
+        if (ngrp > 1) {
+            __syncthreads();
+            if (threadIdx.x == 0) {
+                if (gi > 0) bulk_wait_read0();  // the previous group's stores have left shared memory
+                mbar_arrive_expect_tx(&bar, nk * slice);
+                copy_chunks(gi * cap, gi * cap + nk, true);
+            }
+            __syncthreads();
+            mbar_wait(&bar, ph);
+            ph ^= 1;
+        }
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            const int rr = warp + j * nwarps;
+            if (rr >= R) break;
+            const uint32_t base = smem_u32(rows) + rr * 128 + lane * 4;
+            for (int k = 0; k < nk; ++k) {
+                const float2 f = unpack_f16(lds_u32(base + k * slice));
+                const float y0 = ex2(fmaf(f.x, l2e, mx[j])) * sm_[j], y1 = ex2(fmaf(f.y, l2e, mx[j])) * sm_[j];
+                sts_u32(base + k * slice, bf ? pack_bf16(y0, y1) : pack_f16(y0, y1));
+            }
+        }
+        fence_proxy_async_smem();
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            copy_chunks(gi * cap, gi * cap + nk, false);
+            bulk_commit();
+        }
+    }
+    if (threadIdx.x == 0) bulk_wait_read0();
+}
+
+// rows per CTA and slice capacity in chunks: the largest power of two R <= 32 whose slice fits 48 KB,
+// for the longest rows if that gives R >= 8, else for the mean row (2 rows in up to 160 KB at worst)
+static void softmax_shape(const DevSched& sc, int T, int* R_, int* cap_)
+{
+    const size_t nmax = (size_t)std::max(1, sc.max_rb_tiles * (T / 64));
+    const size_t nmean = (size_t)std::max(1, sc.mean_rb_tiles * (T / 64));
+    int R = 0;
+    for (int r = 32; r >= 8 && !R; r /= 2)
+        if (nmax * r * 128 <= (size_t)kSmBudget) R = r;
+    if (R) { *R_ = R; *cap_ = (int)nmax; return; }
+    for (int r = 32; r >= 2 && !R; r /= 2)
+        if (nmean * r * 128 <= (size_t)kSmBudget) R = r;
+    if (R) { *R_ = R; *cap_ = kSmBudget / (R * 128); return; }
+    *R_ = 2;
+    *cap_ = (int)std::min(nmax, (size_t)kSmBudgetMax / 256);
 }
 
 template <int T>
 cudaError_t launch_softmax_t(const Params& p, cudaStream_t st, int64_t* nl)
 {
-    const int64_t rows = (int64_t)p.B * p.H * p.S;
-    const size_t sm = 4 * (size_t)p.S * 2;
+    int R, cap;
+    softmax_shape(p.sc, T, &R, &cap);
+    const size_t sm = (size_t)cap * R * 128;
     cudaError_t e = cudaFuncSetAttribute(row_softmax<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
     if (e != cudaSuccess) return e;
-    row_softmax<T><<<(unsigned)((rows + 3) / 4), 128, sm, st>>>(p);
-    ++*nl;
-    return cudaGetLastError();
+    const int64_t blocks = (int64_t)p.B * p.H * p.sc.n_rb * (kRowBlock / R);
+    return launch_pdl(row_softmax<T>, dim3((unsigned)blocks), dim3(32 * std::min(R, 8)), sm, st, nl, p, R, cap);
 }
 
 cudaError_t launch_softmax(const Params& p, cudaStream_t st, int64_t* nl)

@@ -85,6 +85,16 @@ __device__ __forceinline__ uint4 lds128(uint32_t saddr)
     asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(saddr) : "memory");
     return v;
 }
+__device__ __forceinline__ uint32_t lds_u32(uint32_t saddr)
+{
+    uint32_t v;
+    asm volatile("ld.shared.b32 %0, [%1];" : "=r"(v) : "r"(saddr) : "memory");
+    return v;
+}
+__device__ __forceinline__ void sts_u32(uint32_t saddr, uint32_t v)
+{
+    asm volatile("st.shared.b32 [%0], %1;" ::"r"(saddr), "r"(v) : "memory");
+}
 __device__ __forceinline__ float lds_f32(uint32_t saddr)
 {
     float v;
@@ -271,6 +281,37 @@ __device__ __forceinline__ float ex2(float x)
     float y;
     asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
     return y;
+}
+// (2^t0, 2^t1) on the FMA/ALU pipes instead of MUFU, for t <= 0: t = j + f with j = rint(t) (the
+// 1.5 * 2^23 round-to-nearest trick: the low bits of t + 1.5 * 2^23 hold j), f in [-1/2, 1/2];
+// 2^f by a degree-3 minimax polynomial (relative error 7.5e-5, under half an fp16 ulp), 2^j added
+// to the exponent field.  t is clamped at -125 so the exponent cannot wrap: masked (-inf) inputs
+// give 2^-125 ~ 2e-38 (0 in fp16).  Used for a fraction of the elements when MUFU.EX2 (16 per
+// clock per SM) would otherwise bound the GEMM1 epilogue.
+__device__ __forceinline__ void ex2_poly2(float& y0, float& y1, float t0, float t1)
+{
+    t0 = fmaxf(t0, -125.f);
+    t1 = fmaxf(t1, -125.f);
+    float r0, r1, p0, p1;
+    asm("{\n\t.reg .b64 t, r, j, f, p, m, c;\n\t"
+        "mov.b64 t, {%4, %5};\n\t"
+        "mov.b64 m, {%6, %6};\n\t"
+        "add.rn.f32x2 r, t, m;\n\t"
+        "sub.rn.f32x2 j, r, m;\n\t"
+        "sub.rn.f32x2 f, t, j;\n\t"
+        "mov.b64 c, {%7, %7};\n\t"
+        "mov.b64 p, {%8, %8};\n\t"
+        "fma.rn.f32x2 p, f, c, p;\n\t"
+        "mov.b64 c, {%9, %9};\n\t"
+        "fma.rn.f32x2 p, p, f, c;\n\t"
+        "mov.b64 c, {%10, %10};\n\t"
+        "fma.rn.f32x2 p, p, f, c;\n\t"
+        "mov.b64 {%0, %1}, r;\n\tmov.b64 {%2, %3}, p;\n\t}"
+        : "=f"(r0), "=f"(r1), "=f"(p0), "=f"(p1)
+        : "f"(t0), "f"(t1), "f"(12582912.f), "f"(0.055171666814681324f), "f"(0.24261113509452378f),
+          "f"(0.6932609870112002f), "f"(0.9999280727914261f));
+    y0 = __uint_as_float(__float_as_uint(p0) + (__float_as_uint(r0) << 23));
+    y1 = __uint_as_float(__float_as_uint(p1) + (__float_as_uint(r1) << 23));
 }
 __device__ __forceinline__ uint32_t pack_f16(float lo, float hi)
 {

@@ -38,6 +38,8 @@ struct DevSched {
     const int32_t* cta_ptr; // [n_cta + 1]: CTA c runs items[cta_ptr[c] .. cta_ptr[c+1])
     const int32_t* kv_len;  // [B] or nullptr
     int n_rb, n_lh, lh_mode, slots_per_head, n_items, n_cta;
+    int max_rb_tiles;       // longest tile list of one (layout head, row-block)
+    int mean_rb_tiles;      // mean tile-list length, rounded up
 };
 
 // Everything a kernel needs to know about one call.

@@ -188,6 +188,14 @@ def test_window_tc(fused, window, n_global, causal, T):
     assert_close(o, ref, "f16")
 
 
+def test_unfused_softmax_streams_long_rows():
+    """The baseline's row softmax keeps row slices in shared memory sized for the mean row; the few
+    longer rows (global tokens here: 32 key tiles against a mean of ~5) take its streaming path."""
+    for fused in (False, True):
+        o, ref = run_case("window", 1, 2, 2048, 64, "f16", window=128, n_global=8, tile_n=64, fused=fused)
+        assert_close(o, ref, "f16", what=f"fused={fused}")
+
+
 def test_all_block_layouts_nb2():
     """Pin P7 on the GPU: every block layout with non-empty rows at nb = 2 (9 layouts), S = 128."""
     import itertools

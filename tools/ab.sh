@@ -1,0 +1,20 @@
+#!/bin/bash
+# A/B the experiment builds: tools/ab.sh "cfgs" lib1 lib2 ...   (lib "-" = the default build)
+cfgs=$1; shift
+for lib in "$@"; do
+  for c in $cfgs; do
+    if [ "$lib" = "-" ]; then L=""; else L="paper_conf_iiswc_choilkha22_b200/$lib"; fi
+    SR_MHA_LIB=$L timeout 300 python bench.py --config $c --no-all-configs --cpu-seconds 0.05 --steps 30 > gpurun_out/ab_${lib}_$c.json 2>gpurun_out/ab_${lib}_$c.err
+    python - "$lib" "$c" <<'PY'
+import json, sys
+lib, c = sys.argv[1], sys.argv[2]
+try:
+    d = json.load(open(f"gpurun_out/ab_{lib}_{c}.json"))
+except Exception:
+    print(lib, c, "FAILED", open(f"gpurun_out/ab_{lib}_{c}.err").read()[-400:]); sys.exit()
+k = {n: round(v["us"], 2) for n, v in d["kernels"].items()}
+fi = d.get("variants", {}).get("fused_ir", {}).get("ms_per_step")
+print(f"{lib:12s} C{c} ms={d['ms_per_step']:.4f} fir={fi} {k}")
+PY
+  done
+done

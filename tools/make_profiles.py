@@ -17,15 +17,21 @@ import sys
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 OUT = os.path.join(ROOT, "gpurun_out")
 PROF = os.path.join(ROOT, "profiles")
-NAMES = {"tc_gemm1": "gemm1", "ir_kernel": "ir", "tc_gemm2": "gemm2", "row_softmax": "softmax"}
-
-
 def kname(full):
-    for k, v in NAMES.items():
+    """Map an ncu kernel name to the bench.py stage name (template args decide the variant)."""
+    import re
+    m = re.search(r"(tc_gemm1|tc_gemm2)<([^>]*)>", full)
+    if m:
+        a = [x.strip() for x in m.group(2).split(",")]
+        flags = [x in ("true", "1", "(bool)1") for x in a[2:]]
+        if m.group(1) == "tc_gemm1":
+            return "gemm1_ls" if flags and flags[0] else "gemm1_plain"
+        if flags and flags[0]:
+            return "gs_gemm2_fused_ir" if len(flags) > 1 and flags[1] else "gs_gemm2"
+        return "gemm2_plain"
+    for k, v in (("ir_kernel", "ir"), ("row_softmax", "softmax"), ("sd_ls_kernel", "sd_ls"),
+                 ("sd_gs_kernel", "sd_gs")):
         if k in full:
-            fused = ", true>" in full or ", (bool)1>" in full or "1>(" in full
-            if k in ("tc_gemm1", "tc_gemm2"):
-                return (("gemm1_ls" if k == "tc_gemm1" else "gs_gemm2") if fused else v + "_plain")
             return v
     return None
 
@@ -50,7 +56,7 @@ def launches(path):
 def main(rnd):
     os.makedirs(PROF, exist_ok=True)
     traffic = {}
-    for c in (2, 3):
+    for c in (2, 3, 4, 5):
         p = os.path.join(OUT, f"launches_c{c}.csv")
         if not os.path.exists(p):
             continue
@@ -75,7 +81,15 @@ def main(rnd):
         tu = sum(ours[k][0] for k in unf) if unf else 0
         if unf:
             lines.append("unfused layer shares:    " + ", ".join(f"{k} {ours[k][0] / tu:.1%}" for k in unf))
-        e = {f"{k}_dram_bytes": int(ours[k][1]) for k in rec + unf}
+        fir = [k for k in ("gemm1_ls", "gs_gemm2_fused_ir") if k in ours]
+        if len(fir) == 2:
+            tf = sum(ours[k][0] for k in fir)
+            lines.append("fused-IR variant shares: " + ", ".join(f"{k} {ours[k][0] / tf:.1%}" for k in fir))
+        sd = [k for k in ("gemm1_plain", "sd_ls", "ir", "sd_gs", "gemm2_plain") if k in ours]
+        if len(sd) == 5:
+            ts = sum(ours[k][0] for k in sd)
+            lines.append("SD variant shares:       " + ", ".join(f"{k} {ours[k][0] / ts:.1%}" for k in sd))
+        e = {f"{k}_dram_bytes": int(ours[k][1]) for k in ours}
         e["recomposed_dram_bytes"] = int(sum(ours[k][1] for k in rec))
         if unf:
             e["unfused_dram_bytes"] = int(sum(ours[k][1] for k in unf))
@@ -83,7 +97,7 @@ def main(rnd):
                      + (f", unfused {e['unfused_dram_bytes'] / 1e6:.1f} MB" if unf else ""))
         traffic[f"C{c}"] = e
         open(os.path.join(PROF, f"{rnd}_launches_c{c}.txt"), "w").write("\n".join(lines) + "\n")
-        for k in ("tc_gemm1", "tc_gemm2", "ir_kernel"):
+        for k in ("tc_gemm1", "tc_gemm2", "ir_kernel", "tc_gemm2_fi"):
             rep = os.path.join(OUT, f"full_c{c}_{k}.ncu-rep")
             if os.path.exists(rep):
                 s = subprocess.run([sys.executable, os.path.join(ROOT, "tools", "ncu_summary.py"), rep, "25"],

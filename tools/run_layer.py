@@ -1,4 +1,5 @@
-"""Run one config's layer a few times (for ncu captures): python tools/run_layer.py CFG [unfused] [reps]"""
+"""Run one config's layer a few times (for ncu captures):
+    python tools/run_layer.py CFG [fused|unfused|fused_ir|sd] [reps]"""
 import os
 import sys
 
@@ -10,11 +11,12 @@ import workloads as W  # noqa: E402
 from bench import Layer  # noqa: E402
 
 idx = int(sys.argv[1])
-fused = not (len(sys.argv) > 2 and sys.argv[2] == "unfused")
+mode = sys.argv[2] if len(sys.argv) > 2 else "fused"
+fused = mode != "unfused"
 reps = int(sys.argv[3]) if len(sys.argv) > 3 else 2
 cfg = W.config(idx)
 L = Layer(cfg, torch.device("cuda", 0), cfg.idx, sr, torch)
 for _ in range(reps):
-    L.run(fused=fused)
+    L.run(fused=fused, fuse_ir=mode == "fused_ir", sd=mode == "sd")
 torch.cuda.synchronize()
-print("ok", cfg.name, "fused" if fused else "unfused")
+print("ok", cfg.name, mode)
