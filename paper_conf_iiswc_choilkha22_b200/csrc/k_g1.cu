@@ -1,4 +1,4 @@
-// k_gemm1.cu -- GEMM1 = Q K^T with scale + mask, and the Local Softmax (LS) sub-layer fused into
+// k_g1.cu -- GEMM1 = Q K^T with scale + mask, and the Local Softmax (LS) sub-layer fused into
 // its epilogue ("setting T of the LS kernel equal to the output tile width
 // of the MatMul kernel, the LS kernel can be fused to its preceding MatMul kernel"; scale and mask
 // fused as element-wise layers, L169).  LS=false builds the unfused baseline's GEMM1, which writes
@@ -102,7 +102,7 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
     G1Hdr* hdr = (G1Hdr*)(smem + C::OFF_HDR);
     uint32_t* tmem_ptr = (uint32_t*)(smem + C::OFF_TPTR);
 
-    const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+    const int warp = warp_uniform(), lane = threadIdx.x % 32;
     if (threadIdx.x == 0) {
         for (int i = 0; i < C::NQ; ++i) { mbar_init(&q_full[i], 1); mbar_init(&q_empty[i], 1); }
         for (int i = 0; i < C::NK; ++i) { mbar_init(&k_full[i], 1); mbar_init(&k_empty[i], 1); }
@@ -131,8 +131,9 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
         //   FULL  (384 threads, 168 at launch): 4 warps x 32 x (168 - 56) = 8 warps x 32 x (224 - 168)
         if constexpr (SPLIT) reg_dealloc<64>();
         else reg_dealloc<56>();
-        if (warp == 0 && lane == 0) {
-            // -------------------------------------------------------------- TMA producer
+        if (warp == 0) {
+            // -------------------------------------------------------------- TMA producer (whole
+            // warp walks the schedule; one elected lane issues)
             int qi = 0, ks = 0;
             uint32_t qph = 0, kph = 0;
             for (int it = it_begin; it < it_end; ++it) {
@@ -140,9 +141,12 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
                 if (I.t0 == I.t1) continue;
                 const int row0 = I.g * p.S + I.rb * kRowBlock;
                 mbar_wait(&q_empty[qi], qph ^ 1);
-                mbar_arrive_expect_tx(&q_full[qi], C::QB);
-                for (int h = 0; h < D / 64; ++h)
-                    tma_load_2d(smem + C::OFF_Q + qi * C::QB + h * (kRowBlock * 128), &tmQ, h * 64, row0, &q_full[qi]);
+                if (elect_one()) {
+                    mbar_arrive_expect_tx(&q_full[qi], C::QB);
+                    for (int h = 0; h < D / 64; ++h)
+                        tma_load_2d(smem + C::OFF_Q + qi * C::QB + h * (kRowBlock * 128), &tmQ, h * 64, row0, &q_full[qi]);
+                }
+                __syncwarp();
                 if (++qi == C::NQ) { qi = 0; qph ^= 1; }
                 int wn[NSUB];  // schedule words of the next macro tile, prefetched one step ahead
 #pragma unroll
@@ -156,16 +160,25 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
                         wn[s] = t + NSUB + s < I.t1 ? __ldg(p.sc.tinfo + t + NSUB + s) : 0;
                     }
                     mbar_wait(&k_empty[ks], kph ^ 1);
-                    mbar_arrive_expect_tx(&k_full[ks], nsub * T * D * 2);
-                    for (int s = 0; s < nsub; ++s)
-                        for (int h = 0; h < D / 64; ++h)
-                            tma_load_2d(smem + C::OFF_K + ks * C::KB + h * (kMW * 128) + s * (T * 128), &tmK, h * 64,
-                                        I.g * p.S + tinfo_kt(w[s]) * T, &k_full[ks]);
+                    if (elect_one()) {
+#ifdef SR_DIAG_NOKLOAD
+                        mbar_arrive(&k_full[ks]);
+                        if (false)
+#else
+                        mbar_arrive_expect_tx(&k_full[ks], nsub * T * D * 2);
+#endif
+                        for (int s = 0; s < nsub; ++s)
+                            for (int h = 0; h < D / 64; ++h)
+                                tma_load_2d(smem + C::OFF_K + ks * C::KB + h * (kMW * 128) + s * (T * 128), &tmK,
+                                            h * 64, I.g * p.S + tinfo_kt(w[s]) * T, &k_full[ks]);
+                    }
+                    __syncwarp();
                     if (++ks == C::NK) { ks = 0; kph ^= 1; }
                 }
             }
-        } else if (warp == 1 && lane == 0) {
-            // -------------------------------------------------------------- MMA issuer
+        } else if (warp == 1) {
+            // -------------------------------------------------------------- MMA issuer (whole warp
+            // walks the schedule; one elected lane issues)
             const uint32_t idesc = idesc_f16(p.in_dtype == DT_BF16 ? 1 : 0, kRowBlock, kMW, 0, 0);
             int qi = 0, ks = 0, n = 0;
             uint32_t qph = 0, kph = 0;
@@ -184,33 +197,43 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
                     const int ab = n % C::NACC;
                     mbar_wait(&acc_empty[ab], ((n / C::NACC) & 1) ^ 1);
                     const int64_t slot = I.slot0 + t;
-                    hdr[ab] = G1Hdr{(int32_t)(slot & 0xffffffff), (int32_t)(slot >> 32), I.rb * kRowBlock, kvl, w0, w1,
-                                    HDR_TILE, 0};
-                    mbar_arrive(&acc_full[ab]);  // header published (arrival 1 of 2)
+                    if (elect_one()) {
+                        hdr[ab] = G1Hdr{(int32_t)(slot & 0xffffffff), (int32_t)(slot >> 32), I.rb * kRowBlock, kvl, w0,
+                                        w1, HDR_TILE, 0};
+                        mbar_arrive(&acc_full[ab]);  // header published (arrival 1 of 2)
+                    }
+                    __syncwarp();
                     mbar_wait(&k_full[ks], kph);
                     tc_fence_after();
                     const uint32_t k_addr = smem_u32(smem + C::OFF_K + ks * C::KB);
                     const uint32_t d_tmem = tmem_base + ab * kMW;
+                    if (elect_one()) {
 #pragma unroll
-                    for (int kk = 0; kk < D / 16; ++kk) {
-                        const uint32_t h = kk / 4, wk = kk % 4;
-                        const uint64_t ad = smem_desc_sw128(q_addr + h * (kRowBlock * 128) + wk * 32, 16, 1024);
-                        const uint64_t bd = smem_desc_sw128(k_addr + h * (kMW * 128) + wk * 32, 16, 1024);
-                        mma_ss(d_tmem, ad, bd, idesc, kk > 0 ? 1u : 0u);
+                        for (int kk = 0; kk < D / 16; ++kk) {
+                            const uint32_t h = kk / 4, wk = kk % 4;
+                            const uint64_t ad = smem_desc_sw128(q_addr + h * (kRowBlock * 128) + wk * 32, 16, 1024);
+                            const uint64_t bd = smem_desc_sw128(k_addr + h * (kMW * 128) + wk * 32, 16, 1024);
+                            mma_ss(d_tmem, ad, bd, idesc, kk > 0 ? 1u : 0u);
+                        }
+                        mma_commit(&k_empty[ks]);
+                        mma_commit(&acc_full[ab]);  // arrival 2 of 2 when the MMAs complete
                     }
-                    mma_commit(&k_empty[ks]);
-                    mma_commit(&acc_full[ab]);  // arrival 2 of 2 when the MMAs complete
+                    __syncwarp();
                     if (++ks == C::NK) { ks = 0; kph ^= 1; }
                 }
-                mma_commit(&q_empty[qi]);
+                if (elect_one()) mma_commit(&q_empty[qi]);
+                __syncwarp();
                 if (++qi == C::NQ) { qi = 0; qph ^= 1; }
             }
             for (int e = 0; e < 2; ++e, ++n) {  // one END header for each epilogue warpgroup pair
                 const int ab = n % C::NACC;
                 mbar_wait(&acc_empty[ab], ((n / C::NACC) & 1) ^ 1);
-                hdr[ab].flags = HDR_END;
-                mbar_arrive(&acc_full[ab]);
-                mbar_arrive(&acc_full[ab]);
+                if (elect_one()) {
+                    hdr[ab].flags = HDR_END;
+                    mbar_arrive(&acc_full[ab]);
+                    mbar_arrive(&acc_full[ab]);
+                }
+                __syncwarp();
             }
         }
     } else if constexpr (SPLIT) {

@@ -93,7 +93,7 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
     auto xhdr = [&](int s) { return (G2Hdr*)(xstage(s) + C::XB + 1024); };
     auto vstage = [&](int s) { return smem + C::OFF_V + s * C::VB; };
 
-    const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+    const int warp = warp_uniform(), lane = threadIdx.x % 32;
     if (threadIdx.x == 0) {
         for (int i = 0; i < C::NX; ++i) { mbar_init(&x_full[i], 1); mbar_init(&x_empty[i], 4); }
         for (int i = 0; i < C::NV; ++i) { mbar_init(&v_full[i], 1); mbar_init(&v_empty[i], 1); }
@@ -120,8 +120,9 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
     const uint8_t* src = (const uint8_t*)(GS ? p.xprime : p.pbuf);
 
     if (warp == 0) {
-        if (lane == 0) {
-            // -------------------------------------------------------------- X' producer
+        {
+            // -------------------------------------------------------------- X' producer (whole
+            // warp walks the schedule; one elected lane issues)
             int s = 0;
             uint32_t sph = 0;
             for (int it = it_begin; it < it_end; ++it) {
@@ -136,6 +137,7 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
                     for (int u = 0; u < nsub; ++u) bytes += (hv[u] == 3 ? 2 : 1) * (T / 64) * (kHalf * 128);
                     mbar_wait(&x_empty[s], sph ^ 1);
                     uint8_t* st = xstage(s);
+                    if (elect_one()) {
                     *xhdr(s) = G2Hdr{SH_TILE | (t == I.t0 ? SH_FIRST : 0) | (t + NSUB >= I.t1 ? SH_LAST : 0), hv[0],
                                      hv[1], nsub, 0, 0, 0, 0};
                     mbar_arrive_expect_tx(&x_full[s], bytes);
@@ -156,12 +158,17 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
                     if (GS)  // r' (or m' with the fused IR) of the sub-tiles' 128 rows rides along
                         bulk_load(st + C::XB, (FI ? p.mprime : p.rprime) + (I.slot0 + t) * kRowBlock,
                                   nsub * kRowBlock * 4, &x_full[s]);
+                    }
+                    __syncwarp();
                     if (++s == C::NX) { s = 0; sph ^= 1; }
                 }
             }
             mbar_wait(&x_empty[s], sph ^ 1);
-            xhdr(s)->flags = SH_END;
-            mbar_arrive(&x_full[s]);
+            if (elect_one()) {
+                xhdr(s)->flags = SH_END;
+                mbar_arrive(&x_full[s]);
+            }
+            __syncwarp();
         }
     } else if (warp == 2) {
         if (FI) {
@@ -222,8 +229,9 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
             }
         }
     } else if (warp == 3) {
-        if (lane == 0) {
-            // -------------------------------------------------------------- V producer
+        {
+            // -------------------------------------------------------------- V producer (whole warp,
+            // one elected lane issues)
             int s = 0;
             uint32_t sph = 0;
             for (int it = it_begin; it < it_end; ++it) {
@@ -235,25 +243,33 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
                     int kt[2] = {tinfo_kt(wn[0]), NSUB > 1 ? tinfo_kt(wn[1]) : 0};
                     for (int u = 0; u < NSUB; ++u) wn[u] = t + NSUB + u < I.t1 ? __ldg(p.sc.tinfo + t + NSUB + u) : 0;
                     mbar_wait(&v_empty[s], sph ^ 1);
-                    mbar_arrive_expect_tx(&v_full[s], nsub * T * D * 2);
-                    for (int u = 0; u < nsub; ++u)
-                        for (int h = 0; h < D / 64; ++h)
-                            tma_load_2d(vstage(s) + h * (kMW2 * 128) + u * (T * 128), &tmV, h * 64,
-                                        I.g * p.S + kt[u] * T, &v_full[s]);
+                    if (elect_one()) {
+                        mbar_arrive_expect_tx(&v_full[s], nsub * T * D * 2);
+                        for (int u = 0; u < nsub; ++u)
+                            for (int h = 0; h < D / 64; ++h)
+                                tma_load_2d(vstage(s) + h * (kMW2 * 128) + u * (T * 128), &tmV, h * 64,
+                                            I.g * p.S + kt[u] * T, &v_full[s]);
+                    }
+                    __syncwarp();
                     if (++s == C::NV) { s = 0; sph ^= 1; }
                 }
             }
         }
     } else if (warp == 1) {
-        if (lane == 0) {
-            // -------------------------------------------------------------- MMA issuer
+        {
+            // -------------------------------------------------------------- MMA issuer (whole warp,
+            // one elected lane issues)
             const uint32_t idesc = idesc_f16(p.in_dtype == DT_BF16 ? 1 : 0, kRowBlock, D, 0, 1);
             int s = 0, a = 0, o = 0;
             uint32_t sph = 0, aph = 0, oph = 0;
-            auto post = [&](int flags, int64_t orow) {  // O header to the epilogue, arrival 1 of 2
+            auto post = [&](int flags, int64_t orow, bool second) {  // O header to the epilogue, arrival 1 of 2
                 mbar_wait(&o_empty[o], oph ^ 1);
-                ohdr[o] = G2Hdr{flags, 0, 0, 0, (int32_t)(orow & 0xffffffff), (int32_t)(orow >> 32), 0, 0};
-                mbar_arrive(&o_full[o]);
+                if (elect_one()) {
+                    ohdr[o] = G2Hdr{flags, 0, 0, 0, (int32_t)(orow & 0xffffffff), (int32_t)(orow >> 32), 0, 0};
+                    mbar_arrive(&o_full[o]);
+                    if (second) mbar_arrive(&o_full[o]);  // no MMA commit will follow
+                }
+                __syncwarp();
             };
             auto next_o = [&]() {
                 if (++o == C::NO) { o = 0; oph ^= 1; }
@@ -265,12 +281,11 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
                 if (it + 1 < it_end) nxt = decode_item(p, it + 1);  // prefetch
                 const int64_t orow = (int64_t)I.g * p.S + I.rb * kRowBlock;
                 if (I.t0 == I.t1) {  // no kept key in these rows: the epilogue writes zeros
-                    post(SH_EMPTY, orow);
-                    mbar_arrive(&o_full[o]);
+                    post(SH_EMPTY, orow, true);
                     next_o();
                     continue;
                 }
-                post(SH_TILE, orow);
+                post(SH_TILE, orow, false);
                 const uint32_t d_tmem = tmem_o + o * D;
                 for (int t = I.t0; t < I.t1; t += NSUB) {
                     const int nk = min(NSUB, I.t1 - t) * (T / 16);  // K steps of 16 keys
@@ -279,22 +294,25 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
                     tc_fence_after();
                     const uint32_t v_addr = smem_u32(vstage(s));
                     const uint32_t a_tm = tmem_a + a * (kMW2 / 2);
+                    if (elect_one()) {
 #pragma unroll 8
-                    for (int kk = 0; kk < nk; ++kk) {
-                        // B = V, MN-major SW128: 16 keys per MMA = 2 KB; 64-wide d blocks at LBO = MW*128 B
-                        const uint64_t bd = smem_desc_sw128(v_addr + kk * 2048, kMW2 * 128, 1024);
-                        mma_ts(d_tmem, a_tm + kk * 8, bd, idesc, (t == I.t0 && kk == 0) ? 0u : 1u);
+                        for (int kk = 0; kk < nk; ++kk) {
+                            // B = V, MN-major SW128: 16 keys per MMA = 2 KB; 64-wide d blocks at LBO = MW*128 B
+                            const uint64_t bd = smem_desc_sw128(v_addr + kk * 2048, kMW2 * 128, 1024);
+                            mma_ts(d_tmem, a_tm + kk * 8, bd, idesc, (t == I.t0 && kk == 0) ? 0u : 1u);
+                        }
+                        mma_commit(&v_empty[s]);
+                        mma_commit(&a_empty[a]);
                     }
-                    mma_commit(&v_empty[s]);
-                    mma_commit(&a_empty[a]);
+                    __syncwarp();
                     if (++s == C::NV) { s = 0; sph ^= 1; }
                     if (++a == C::NA) { a = 0; aph ^= 1; }
                 }
-                mma_commit(&o_full[o]);  // arrival 2 of 2 when the item's MMAs complete
+                if (elect_one()) mma_commit(&o_full[o]);  // arrival 2 of 2 when the item's MMAs complete
+                __syncwarp();
                 next_o();
             }
-            post(SH_END, 0);
-            mbar_arrive(&o_full[o]);
+            post(SH_END, 0, true);
         }
     } else if (warp >= 4 && warp < 8) {
         // ------------------------------------------------------------------ GS transform

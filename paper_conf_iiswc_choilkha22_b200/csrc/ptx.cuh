@@ -55,6 +55,18 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity)
     }
 }
 
+// ------------------------------------------------------------------ warp-uniform control
+// Role dispatch on a provably warp-uniform warp index, and single-thread work (TMA, MMA issue,
+// barrier arrivals) under elect.sync inside converged warp code: the compiler then keeps TMA / MMA
+// operands in uniform registers instead of wrapping every such instruction in a per-thread loop.
+__device__ __forceinline__ int warp_uniform() { return __shfl_sync(0xffffffffu, (int)(threadIdx.x / 32), 0); }
+__device__ __forceinline__ bool elect_one()
+{
+    uint32_t pred;
+    asm volatile("{\n\t.reg .pred P;\n\telect.sync _|P, 0xffffffff;\n\tselp.b32 %0, 1, 0, P;\n\t}" : "=r"(pred));
+    return pred != 0;
+}
+
 // ------------------------------------------------------------------ register rebalancing
 // (all 4 warps of a warpgroup must execute these; counts are multiples of 8 in [24, 256])
 template <int N>
