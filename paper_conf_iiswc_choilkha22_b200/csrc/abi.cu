@@ -10,6 +10,7 @@
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <map>
 #include <memory>
@@ -45,6 +46,12 @@ struct HostSched {
     int T = 0, H = 1, n_rb = 0, n_lh = 1, lh_mode = LH_ONE;
     std::vector<int32_t> tp, tinfo, items, kv_len;
     std::vector<int32_t> cta_ptr;  // device schedules only: items grouped per persistent CTA
+    // GEMM1 pair schedule: row-blocks 2j, 2j+1 of a head share every K tile of the union of their
+    // lists.  pp [n_lh][n_pair+1] offsets into pent; pent 4 ints per union entry
+    // {kt | half bits of 2j << 16 | half bits of 2j+1 << 18, tinfo index in 2j's list or -1, same
+    // for 2j+1, 0}; pitems g * n_pair + j grouped per CTA (pcta_ptr).
+    int n_pair = 0;
+    std::vector<int32_t> pp, pent, pitems, pcta_ptr;
     int slots_per_head = 0;
     int max_rb_tiles = 0;
     int64_t n_tiles = 0;       // over all B*H heads
@@ -166,6 +173,29 @@ sr_status build_sched(const Request& r, HostSched& hs)
     hs.items.resize(it.size());
     for (size_t i = 0; i < it.size(); ++i) hs.items[i] = it[i].second;
     if (r.kv_len) hs.kv_len.assign(r.kv_len, r.kv_len + r.B);
+    // pair lists: merge the (kt-ascending) lists of row-blocks 2j and 2j+1
+    hs.n_pair = (hs.n_rb + 1) / 2;
+    hs.pp.assign((size_t)hs.n_lh * (hs.n_pair + 1), 0);
+    for (int lh = 0; lh < hs.n_lh; ++lh) {
+        const int32_t* tp = &hs.tp[(size_t)lh * (hs.n_rb + 1)];
+        hs.pp[(size_t)lh * (hs.n_pair + 1)] = (int32_t)(hs.pent.size() / 4);
+        for (int j = 0; j < hs.n_pair; ++j) {
+            int ia = tp[2 * j], ea = tp[2 * j + 1];
+            int ib = 2 * j + 1 < hs.n_rb ? tp[2 * j + 1] : 0, eb = 2 * j + 1 < hs.n_rb ? tp[2 * j + 2] : 0;
+            while (ia < ea || ib < eb) {
+                const int ka = ia < ea ? tinfo_kt(hs.tinfo[ia]) : INT32_MAX;
+                const int kb = ib < eb ? tinfo_kt(hs.tinfo[ib]) : INT32_MAX;
+                const int kt = std::min(ka, kb);
+                int32_t w = kt, ta = -1, tb = -1;
+                if (ka == kt) { w |= tinfo_half(hs.tinfo[ia]) << 16; ta = ia++; }
+                if (kb == kt) { w |= tinfo_half(hs.tinfo[ib]) << 18; tb = ib++; }
+                hs.pent.insert(hs.pent.end(), {w, ta, tb, 0});
+            }
+            hs.pp[(size_t)lh * (hs.n_pair + 1) + j + 1] = (int32_t)(hs.pent.size() / 4);
+        }
+    }
+    for (int g = 0; g < BH; ++g)
+        for (int j = 0; j < hs.n_pair; ++j) hs.pitems.push_back(g * hs.n_pair + j);
     return SR_OK;
 }
 
@@ -274,32 +304,54 @@ std::string sched_key(const Request& r, int device)
 // 2 x its tiles + 1 (the Q load / O store of a row-block is about half a tile's traffic).  Items
 // are regrouped per CTA in assignment order, so the first wave is the round-robin one (neighbouring
 // CTAs run items of the same head at the same time and share its K/V tiles in L2).
-void lpt_assign(HostSched& h, int n_cta)
+void lpt_assign(std::vector<int32_t>& items, const std::vector<int64_t>& cost, int n_cta, std::vector<int32_t>& cta_ptr)
 {
-    const size_t n = h.items.size();
+    const size_t n = items.size();
     n_cta = (int)std::max<size_t>(1, std::min<size_t>(n, (size_t)std::max(n_cta, 1)));
+    // longest first (stable: ties keep head-major order), then each to the least loaded CTA
+    std::vector<size_t> order(n);
+    for (size_t i = 0; i < n; ++i) order[i] = i;
+    std::stable_sort(order.begin(), order.end(), [&](size_t a, size_t b) { return cost[a] > cost[b]; });
     std::vector<int> owner(n);
     std::vector<int32_t> count(n_cta, 0);
     using E = std::pair<int64_t, int>;  // (load, cta)
     std::priority_queue<E, std::vector<E>, std::greater<E>> pq;
     for (int c = 0; c < n_cta; ++c) pq.push({0, c});
-    for (size_t i = 0; i < n; ++i) {
-        const int32_t w = h.items[i];
-        const int g = w / h.n_rb, rb = w % h.n_rb;
-        const int lh = h.lh_mode == LH_ONE ? 0 : (h.lh_mode == LH_BATCH ? g / h.H : g % h.H);
-        const int32_t* tp = &h.tp[(size_t)lh * (h.n_rb + 1)];
+    for (size_t i : order) {
         E e = pq.top();
         pq.pop();
         owner[i] = e.second;
         ++count[e.second];
-        e.first += 2 * (int64_t)(tp[rb + 1] - tp[rb]) + 1;
+        e.first += cost[i];
         pq.push(e);
     }
-    h.cta_ptr.assign(n_cta + 1, 0);
-    for (int c = 0; c < n_cta; ++c) h.cta_ptr[c + 1] = h.cta_ptr[c] + count[c];
-    std::vector<int32_t> fill(h.cta_ptr.begin(), h.cta_ptr.end() - 1), out(n);
-    for (size_t i = 0; i < n; ++i) out[fill[owner[i]]++] = h.items[i];
-    h.items.swap(out);
+    cta_ptr.assign(n_cta + 1, 0);
+    for (int c = 0; c < n_cta; ++c) cta_ptr[c + 1] = cta_ptr[c] + count[c];
+    std::vector<int32_t> fill(cta_ptr.begin(), cta_ptr.end() - 1), out(n);
+    for (size_t i : order) out[fill[owner[i]]++] = items[i];
+    items.swap(out);
+}
+
+// Per-CTA item ranges for both schedules.  Cost of an item = 2 x its tiles + 1 (the Q load / O
+// store of a row-block is about half a tile's traffic); of a pair = its two row-blocks' tiles + 1.
+void lpt_assign(HostSched& h, int n_cta)
+{
+    auto lh_of_g = [&](int g) { return h.lh_mode == LH_ONE ? 0 : (h.lh_mode == LH_BATCH ? g / h.H : g % h.H); };
+    std::vector<int64_t> cost(h.items.size());
+    for (size_t i = 0; i < h.items.size(); ++i) {
+        const int g = h.items[i] / h.n_rb, rb = h.items[i] % h.n_rb;
+        const int32_t* tp = &h.tp[(size_t)lh_of_g(g) * (h.n_rb + 1)];
+        cost[i] = 2 * (int64_t)(tp[rb + 1] - tp[rb]) + 1;
+    }
+    lpt_assign(h.items, cost, n_cta, h.cta_ptr);
+    std::vector<int64_t> pcost(h.pitems.size());
+    for (size_t i = 0; i < h.pitems.size(); ++i) {
+        const int g = h.pitems[i] / h.n_pair, j = h.pitems[i] % h.n_pair;
+        const int32_t* tp = &h.tp[(size_t)lh_of_g(g) * (h.n_rb + 1)];
+        const int rb1 = std::min(2 * j + 2, h.n_rb);
+        pcost[i] = 2 * (int64_t)(tp[rb1] - tp[2 * j]) + 1;
+    }
+    lpt_assign(h.pitems, pcost, n_cta, h.pcta_ptr);
 }
 
 // Host schedule only (no device), used by queries.
@@ -326,11 +378,30 @@ sr_status host_sched(const Request& r, std::shared_ptr<CachedSched>& out, bool n
         lpt_assign(h, n_sm);
         size_t n_tp = h.tp.size(), n_ti = std::max<size_t>(h.tinfo.size(), 1), n_it = h.items.size(),
                n_kv = h.kv_len.size();
-        size_t bytes = sizeof(int32_t) * (n_tp + n_ti + n_it + n_kv + h.cta_ptr.size() + 4);
+        const size_t n_pit = h.pitems.size();
+        size_t bytes = sizeof(int32_t) * (4 * n_it + 4 * n_pit + h.pent.size() + 4 + n_tp + n_ti + n_it + n_kv +
+                                          h.cta_ptr.size() + h.pp.size() + h.pcta_ptr.size() + 4);
         cudaError_t ce = cudaMalloc(&cs->dmem, bytes);
         if (ce != cudaSuccess) return fail(SR_ERR_CUDA, "cudaMalloc(schedule): %s", cudaGetErrorString(ce));
         std::vector<int32_t> blob;
         blob.reserve(bytes / 4);
+        for (int32_t w : h.items) {  // item descriptors first (16-B aligned at the allocation base)
+            const int g = w / h.n_rb, rb = w % h.n_rb;
+            const int lh = h.lh_mode == LH_ONE ? 0 : (h.lh_mode == LH_BATCH ? g / h.H : g % h.H);
+            const int32_t* tp = &h.tp[(size_t)lh * (h.n_rb + 1)];
+            blob.insert(blob.end(), {w, tp[rb], tp[rb + 1], tp[0]});
+        }
+        size_t o_pd = blob.size();  // pair item descriptors {g * n_pair + j, e0, e1, tp[lh][0]}
+        for (int32_t w : h.pitems) {
+            const int g = w / h.n_pair, j = w % h.n_pair;
+            const int lh = h.lh_mode == LH_ONE ? 0 : (h.lh_mode == LH_BATCH ? g / h.H : g % h.H);
+            const int32_t* pp = &h.pp[(size_t)lh * (h.n_pair + 1)];
+            blob.insert(blob.end(), {w, pp[j], pp[j + 1], h.tp[(size_t)lh * (h.n_rb + 1)]});
+        }
+        size_t o_pe = blob.size();  // union entries (int4)
+        blob.insert(blob.end(), h.pent.begin(), h.pent.end());
+        if (h.pent.empty()) blob.insert(blob.end(), {0, -1, -1, 0});
+        size_t o_tp = blob.size();
         blob.insert(blob.end(), h.tp.begin(), h.tp.end());
         size_t o_ti = blob.size();
         blob.insert(blob.end(), h.tinfo.begin(), h.tinfo.end());
@@ -341,10 +412,13 @@ sr_status host_sched(const Request& r, std::shared_ptr<CachedSched>& out, bool n
         blob.insert(blob.end(), h.kv_len.begin(), h.kv_len.end());
         size_t o_cp = blob.size();
         blob.insert(blob.end(), h.cta_ptr.begin(), h.cta_ptr.end());
+        size_t o_pcp = blob.size();
+        blob.insert(blob.end(), h.pcta_ptr.begin(), h.pcta_ptr.end());
         ce = cudaMemcpy(cs->dmem, blob.data(), blob.size() * 4, cudaMemcpyHostToDevice);
         if (ce != cudaSuccess) return fail(SR_ERR_CUDA, "cudaMemcpy(schedule): %s", cudaGetErrorString(ce));
         int32_t* base = (int32_t*)cs->dmem;
-        cs->dev.tp = base;
+        cs->dev.item_desc = (const int4*)base;
+        cs->dev.tp = base + o_tp;
         cs->dev.tinfo = base + o_ti;
         cs->dev.items = base + o_it;
         cs->dev.kv_len = n_kv ? base + o_kv : nullptr;
@@ -357,6 +431,11 @@ sr_status host_sched(const Request& r, std::shared_ptr<CachedSched>& out, bool n
         cs->dev.n_items = (int)h.items.size();
         cs->dev.cta_ptr = base + o_cp;
         cs->dev.n_cta = (int)h.cta_ptr.size() - 1;
+        cs->dev.pair_desc = (const int4*)(base + o_pd);
+        cs->dev.pent = (const int4*)(base + o_pe);
+        cs->dev.pcta_ptr = base + o_pcp;
+        cs->dev.n_pair = h.n_pair;
+        cs->dev.n_pcta = (int)h.pcta_ptr.size() - 1;
     }
     g_cache[key] = cs;
     out = cs;
@@ -450,6 +529,13 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
     const int stage_bits = ex->flags & (SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2);
     p.stages = stage_bits ? stage_bits : (SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2);
     p.fuse_ir = (ex->flags & SR_FUSE_IR) ? 1 : 0;
+    {   // GEMM1 pair schedule: SR_G1_PAIR=0/1 overrides the default (experiments)
+        static const int env_pair = [] { const char* e = getenv("SR_G1_PAIR"); return e ? atoi(e) : -1; }();
+        // default: pairs when K tiles are as large as the X' tiles they produce (D = 128) and there
+        // are enough pairs to keep every SM busy (measured: C3 78 -> 75 us; D = 64 configs lose)
+        p.g1_pair = env_pair >= 0 ? env_pair : (D == 128 && cs->dev.n_pcta > 0 &&
+                                                 (int64_t)B * H * cs->dev.n_pair >= 2 * (int64_t)cs->dev.n_pcta);
+    }
     char* ws = (char*)ex->workspace;
     p.xprime = ws + wi.off_xprime;
     if (fused) {

@@ -48,10 +48,11 @@ struct G1Hdr {  // per-accumulator macro-tile header, written by the MMA warp
 };
 enum : int { HDR_TILE = 1, HDR_END = 2 };
 
-template <int D, int T>
+template <int D, int T, bool PAIR>
 struct G1 {
     static constexpr int NSUB = kMW / T;          // sub-tiles per macro tile
     static constexpr int QB = kRowBlock * D * 2;  // Q tile bytes
+    static constexpr int QS = (PAIR ? 2 : 1) * QB;  // Q stage: one row-block, or a pair
     static constexpr int KB = kMW * D * 2;        // K stage bytes (MW keys)
     static constexpr bool SPLIT = (T == 64);      // epilogue organisation, see the file header
     static constexpr int EPI_WG = SPLIT ? 4 : 2;  // epilogue warpgroups
@@ -62,16 +63,16 @@ struct G1 {
     static constexpr int NACC = 512 / kMW;        // TMEM accumulators
     // staging buffers per epilogue warpgroup (2 if at all possible: the X' store stream is the
     // bottleneck), then Q double-buffered if shared memory still allows
-    static constexpr int XPW = (QB + 2 * KB + EPI_WG * 2 * SB + 4096 <= kSmemMax) ? 2 : 1;
+    static constexpr int XPW = ((PAIR ? 2 * QS : QS) + 2 * KB + EPI_WG * 2 * SB + 4096 <= kSmemMax) ? 2 : 1;
 #ifndef SR_G1_MAX_NQ
 #define SR_G1_MAX_NQ 2
 #endif
-    static constexpr int NQ = (SR_G1_MAX_NQ >= 2 && 2 * QB + 2 * KB + EPI_WG * XPW * SB + 4096 <= kSmemMax) ? 2 : 1;
-    static constexpr int NK_ = (kSmemMax - 4096 - NQ * QB - EPI_WG * XPW * SB) / KB;
+    static constexpr int NQ = (SR_G1_MAX_NQ >= 2 && 2 * QS + 2 * KB + EPI_WG * XPW * SB + 4096 <= kSmemMax) ? 2 : 1;
+    static constexpr int NK_ = (kSmemMax - 4096 - NQ * QS - EPI_WG * XPW * SB) / KB;
     static constexpr int NK = NK_ > 4 ? 4 : NK_;
     static_assert(NK >= 2, "smem budget");
     static constexpr int OFF_Q = 0;
-    static constexpr int OFF_K = OFF_Q + NQ * QB;
+    static constexpr int OFF_K = OFF_Q + NQ * QS;
     static constexpr int OFF_X = OFF_K + NK * KB;
     static constexpr int OFF_BAR = OFF_X + EPI_WG * XPW * SB;
     static constexpr int NBAR = 2 * NQ + 2 * NK + 2 * NACC;
@@ -83,11 +84,11 @@ struct G1 {
     static constexpr int THREADS = 128 + EPI_WG * 128;
 };
 
-template <int D, int T, bool LS>
+template <int D, int T, bool LS, bool PAIR>
 __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
     tc_gemm1(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmK, const Params p)
 {
-    using C = G1<D, T>;
+    using C = G1<D, T, PAIR>;
     constexpr int NSUB = C::NSUB;
     constexpr bool SPLIT = C::SPLIT;
     extern __shared__ uint8_t smem_raw[];
@@ -121,8 +122,10 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
     // own prologue, then wait for our producer kernel's results before touching them
     griddep_launch_dependents();
     griddep_wait();
-    // this CTA's items: a contiguous range of the longest-processing-time assignment (host)
-    const int it_begin = __ldg(p.sc.cta_ptr + blockIdx.x), it_end = __ldg(p.sc.cta_ptr + blockIdx.x + 1);
+    // this CTA's items (row-blocks, or pairs of row-blocks): a contiguous range of the host's
+    // longest-processing-time assignment
+    const int32_t* cptr = PAIR ? p.sc.pcta_ptr : p.sc.cta_ptr;
+    const int it_begin = __ldg(cptr + blockIdx.x), it_end = __ldg(cptr + blockIdx.x + 1);
 
     if (warp < 4) {
         // warpgroup 0 hands registers to the epilogue warpgroups.  setmaxnreg.inc can only draw what
@@ -131,13 +134,147 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
         //   FULL  (384 threads, 168 at launch): 4 warps x 32 x (168 - 56) = 8 warps x 32 x (224 - 168)
         if constexpr (SPLIT) reg_dealloc<64>();
         else reg_dealloc<56>();
-        if (warp == 0) {
+        if (PAIR && warp == 0) {
+            // -------------------------------------------------------------- TMA producer, pairs:
+            // Q of row-blocks 2j and 2j+1 per item, then one K stage per union macro tile
+            int qi = 0, ks = 0;
+            uint32_t qph = 0, kph = 0;
+            int4 nd = it_begin < it_end ? __ldg(p.sc.pair_desc + it_begin) : make_int4(0, 0, 0, 0);
+            for (int it = it_begin; it < it_end; ++it) {
+                const int4 d = nd;
+                if (it + 1 < it_end) nd = __ldg(p.sc.pair_desc + it + 1);
+                const int g = d.x / p.sc.n_pair, j = d.x % p.sc.n_pair, e0 = d.y, e1 = d.z;
+                if (e0 == e1) continue;
+                const int nrb = 2 * j + 1 < p.sc.n_rb ? 2 : 1;
+                const int row0 = g * p.S + 2 * j * kRowBlock;
+                mbar_wait(&q_empty[qi], qph ^ 1);
+                if (elect_one()) {
+                    mbar_arrive_expect_tx(&q_full[qi], nrb * C::QB);
+                    for (int r = 0; r < nrb; ++r)
+                        for (int h = 0; h < D / 64; ++h)
+                            tma_load_2d(smem + C::OFF_Q + qi * C::QS + r * C::QB + h * (kRowBlock * 128), &tmQ, h * 64,
+                                        row0 + r * kRowBlock, &q_full[qi]);
+                }
+                __syncwarp();
+                if (++qi == C::NQ) { qi = 0; qph ^= 1; }
+                int wn[NSUB];
+#pragma unroll
+                for (int s2 = 0; s2 < NSUB; ++s2) wn[s2] = e0 + s2 < e1 ? __ldg(&p.sc.pent[e0 + s2].x) : 0;
+                for (int e = e0; e < e1; e += NSUB) {
+                    const int nsub = min(NSUB, e1 - e);
+                    int w[NSUB];
+#pragma unroll
+                    for (int s2 = 0; s2 < NSUB; ++s2) {
+                        w[s2] = wn[s2];
+                        wn[s2] = e + NSUB + s2 < e1 ? __ldg(&p.sc.pent[e + NSUB + s2].x) : 0;
+                    }
+                    mbar_wait(&k_empty[ks], kph ^ 1);
+                    if (elect_one()) {
+                        mbar_arrive_expect_tx(&k_full[ks], nsub * T * D * 2);
+                        for (int s2 = 0; s2 < nsub; ++s2)
+                            for (int h = 0; h < D / 64; ++h)
+                                tma_load_2d(smem + C::OFF_K + ks * C::KB + h * (kMW * 128) + s2 * (T * 128), &tmK,
+                                            h * 64, g * p.S + (w[s2] & 0xFFFF) * T, &k_full[ks]);
+                    }
+                    __syncwarp();
+                    if (++ks == C::NK) { ks = 0; kph ^= 1; }
+                }
+            }
+        } else if (PAIR && warp == 1) {
+            // -------------------------------------------------------------- MMA issuer, pairs: per
+            // union macro tile, the MMAs of each row-block that has a valid sub-tile in it, each into
+            // the next TMEM accumulator of the common ring (the epilogue is the same as unpaired)
+            const uint32_t idesc = idesc_f16(p.in_dtype == DT_BF16 ? 1 : 0, kRowBlock, kMW, 0, 0);
+            int qi = 0, ks = 0, n = 0;
+            uint32_t qph = 0, kph = 0;
+            int4 nd = it_begin < it_end ? __ldg(p.sc.pair_desc + it_begin) : make_int4(0, 0, 0, 0);
+            for (int it = it_begin; it < it_end; ++it) {
+                const int4 d = nd;
+                if (it + 1 < it_end) nd = __ldg(p.sc.pair_desc + it + 1);
+                const int g = d.x / p.sc.n_pair, j = d.x % p.sc.n_pair, e0 = d.y, e1 = d.z;
+                if (e0 == e1) continue;
+                const int nrb = 2 * j + 1 < p.sc.n_rb ? 2 : 1;
+                const int kvl = p.sc.kv_len ? __ldg(p.sc.kv_len + g / p.H) : p.S;
+                const int64_t slot0 = (int64_t)g * p.sc.slots_per_head - d.w;
+                mbar_wait(&q_full[qi], qph);
+                tc_fence_after();
+                const uint32_t q_addr = smem_u32(smem + C::OFF_Q + qi * C::QS);
+                int4 wn[NSUB];
+#pragma unroll
+                for (int s2 = 0; s2 < NSUB; ++s2) wn[s2] = e0 + s2 < e1 ? __ldg(p.sc.pent + e0 + s2) : make_int4(0, -1, -1, 0);
+                for (int e = e0; e < e1; e += NSUB) {
+                    int4 w[NSUB];
+#pragma unroll
+                    for (int s2 = 0; s2 < NSUB; ++s2) {
+                        w[s2] = wn[s2];
+                        wn[s2] = e + NSUB + s2 < e1 ? __ldg(p.sc.pent + e + NSUB + s2) : make_int4(0, -1, -1, 0);
+                    }
+                    mbar_wait(&k_full[ks], kph);
+                    tc_fence_after();
+                    const uint32_t k_addr = smem_u32(smem + C::OFF_K + ks * C::KB);
+                    for (int r = 0; r < nrb; ++r) {
+                        int ws[2] = {-1, -1};
+                        int64_t sl[2] = {0, 0};
+#pragma unroll
+                        for (int s2 = 0; s2 < NSUB; ++s2) {
+                            const int hb = (w[s2].x >> (16 + 2 * r)) & 3;
+                            if (e + s2 < e1 && hb) {
+                                ws[s2] = (w[s2].x & 0xFFFF) | (hb << 16);
+                                sl[s2] = slot0 + (r ? w[s2].z : w[s2].y);
+                            }
+                        }
+                        if (ws[0] == -1 && ws[1] == -1) continue;  // nothing of this row-block here
+                        const int buf = n % C::NACC;
+                        mbar_wait(&acc_empty[buf], ((n / C::NACC) & 1) ^ 1);
+                        // sub-tile s's slot = slot + (s ? dslot : 0)
+                        const int64_t slot = ws[0] != -1 ? sl[0] : sl[1];
+                        const int dslot = (ws[0] != -1 && ws[1] != -1) ? (int)(sl[1] - sl[0]) : 0;
+                        if (elect_one()) {
+                            hdr[buf] = G1Hdr{(int32_t)(slot & 0xffffffff), (int32_t)(slot >> 32),
+                                             (2 * j + r) * kRowBlock, kvl, ws[0], ws[1], HDR_TILE, dslot};
+                            mbar_arrive(&acc_full[buf]);  // header published (arrival 1 of 2)
+                        }
+                        __syncwarp();
+                        const uint32_t d_tmem = tmem_base + buf * kMW;
+                        const uint32_t qa = q_addr + r * C::QB;
+                        if (elect_one()) {
+#pragma unroll
+                            for (int kk = 0; kk < D / 16; ++kk) {
+                                const uint32_t h = kk / 4, wk = kk % 4;
+                                const uint64_t ad = smem_desc_sw128(qa + h * (kRowBlock * 128) + wk * 32, 16, 1024);
+                                const uint64_t bd = smem_desc_sw128(k_addr + h * (kMW * 128) + wk * 32, 16, 1024);
+                                mma_ss(d_tmem, ad, bd, idesc, kk > 0 ? 1u : 0u);
+                            }
+                            mma_commit(&acc_full[buf]);  // arrival 2 of 2 when the MMAs complete
+                        }
+                        __syncwarp();
+                        ++n;
+                    }
+                    if (elect_one()) mma_commit(&k_empty[ks]);
+                    __syncwarp();
+                    if (++ks == C::NK) { ks = 0; kph ^= 1; }
+                }
+                if (elect_one()) mma_commit(&q_empty[qi]);
+                __syncwarp();
+                if (++qi == C::NQ) { qi = 0; qph ^= 1; }
+            }
+            for (int e = 0; e < 2; ++e, ++n) {  // one END header for each epilogue warpgroup (pair)
+                const int buf = n % C::NACC;
+                mbar_wait(&acc_empty[buf], ((n / C::NACC) & 1) ^ 1);
+                if (elect_one()) {
+                    hdr[buf].flags = HDR_END;
+                    mbar_arrive(&acc_full[buf]);
+                    mbar_arrive(&acc_full[buf]);
+                }
+                __syncwarp();
+            }
+        } else if (warp == 0) {
             // -------------------------------------------------------------- TMA producer (whole
             // warp walks the schedule; one elected lane issues)
             int qi = 0, ks = 0;
             uint32_t qph = 0, kph = 0;
-            for (int it = it_begin; it < it_end; ++it) {
-                const ItemInfo I = decode_item(p, it);
+            for (ItemWalk iw(p, it_begin, it_end); iw.more();) {
+                const ItemInfo I = iw.next();
                 if (I.t0 == I.t1) continue;
                 const int row0 = I.g * p.S + I.rb * kRowBlock;
                 mbar_wait(&q_empty[qi], qph ^ 1);
@@ -182,8 +319,8 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
             const uint32_t idesc = idesc_f16(p.in_dtype == DT_BF16 ? 1 : 0, kRowBlock, kMW, 0, 0);
             int qi = 0, ks = 0, n = 0;
             uint32_t qph = 0, kph = 0;
-            for (int it = it_begin; it < it_end; ++it) {
-                const ItemInfo I = decode_item(p, it);
+            for (ItemWalk iw(p, it_begin, it_end); iw.more();) {
+                const ItemInfo I = iw.next();
                 if (I.t0 == I.t1) continue;
                 const int kvl = p.sc.kv_len ? __ldg(p.sc.kv_len + I.g / p.H) : p.S;
                 mbar_wait(&q_full[qi], qph);
@@ -199,7 +336,7 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
                     const int64_t slot = I.slot0 + t;
                     if (elect_one()) {
                         hdr[ab] = G1Hdr{(int32_t)(slot & 0xffffffff), (int32_t)(slot >> 32), I.rb * kRowBlock, kvl, w0,
-                                        w1, HDR_TILE, 0};
+                                        w1, HDR_TILE, 1};  // adjacent sub-tile slots
                         mbar_arrive(&acc_full[ab]);  // header published (arrival 1 of 2)
                     }
                     __syncwarp();
@@ -259,7 +396,7 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
             const bool valid = w != -1 && ((tinfo_half(w) >> myhalf) & 1);
             const int c0 = tinfo_kt(w) * T + (NSUB == 1 ? 64 * h : 0);
             const int i = H.i0 + r;
-            const int64_t slot = (((int64_t)H.slot_hi << 32) | (uint32_t)H.slot_lo) + (NSUB == 2 ? h : 0);
+            const int64_t slot = (((int64_t)H.slot_hi << 32) | (uint32_t)H.slot_lo) + (NSUB == 2 && h ? H.pad : 0);
             // one TMEM read of the row's 64 fp32 scores; the accumulator goes straight back to the MMA
             uint32_t x[64];
             if (valid) {
@@ -496,7 +633,7 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
 #pragma unroll
                 for (int s = 0; s < NSUB; ++s) {
                     if (!wv[s]) continue;
-                    uint8_t* dst = (uint8_t*)p.xprime + (slot + s) * (int64_t)C::XS;
+                    uint8_t* dst = (uint8_t*)p.xprime + (slot + (s ? H.pad : 0)) * (int64_t)C::XS;
                     for (int ch = 0; ch < T / 64; ++ch)
 #ifndef SR_DIAG_NOSTORE
                         bulk_store(dst + ch * (kRowBlock * 128) + wrow0 * 128,
@@ -511,8 +648,8 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
 #pragma unroll
                 for (int s = 0; s < NSUB; ++s)
                     if (vs[s]) {
-                        p.mprime[(slot + s) * kRowBlock + r] = mx[s] * p.scale;  // m' in natural-log units
-                        p.dprime[(slot + s) * kRowBlock + r] = dsum[s];
+                        p.mprime[(slot + (s ? H.pad : 0)) * kRowBlock + r] = mx[s] * p.scale;  // natural-log units
+                        p.dprime[(slot + (s ? H.pad : 0)) * kRowBlock + r] = dsum[s];
                     }
             }
         }
@@ -531,29 +668,35 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
 cudaError_t make_tmap_2d(CUtensorMap* m, const void* base, int64_t rows, int D, int box_rows, int dtype);
 int num_sms();
 
-template <int D, int T, bool LS>
+template <int D, int T, bool LS, bool PAIR>
 cudaError_t launch_g1_t(const Params& p, cudaStream_t st, int64_t* nl)
 {
-    using C = G1<D, T>;
+    using C = G1<D, T, PAIR>;
     CUtensorMap tq, tk;
     const int64_t rows = (int64_t)p.B * p.H * p.S;
     cudaError_t e;
     if ((e = make_tmap_2d(&tq, p.q, rows, D, kRowBlock, p.in_dtype)) != cudaSuccess) return e;
     if ((e = make_tmap_2d(&tk, p.k, rows, D, T, p.in_dtype)) != cudaSuccess) return e;
-    auto kern = tc_gemm1<D, T, LS>;
+    auto kern = tc_gemm1<D, T, LS, PAIR>;
     if ((e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM)) != cudaSuccess) return e;
-    const int grid = p.sc.n_cta;  // one persistent CTA per SM, items assigned by host LPT
+    const int grid = PAIR ? p.sc.n_pcta : p.sc.n_cta;  // one persistent CTA per SM, host LPT items
     return launch_pdl(kern, dim3(grid), dim3(C::THREADS), C::SMEM, st, nl, tq, tk, p);
+}
+
+template <int D, int T, bool LS>
+cudaError_t launch_g1_p(const Params& p, cudaStream_t st, int64_t* nl)
+{
+    return p.g1_pair ? launch_g1_t<D, T, LS, true>(p, st, nl) : launch_g1_t<D, T, LS, false>(p, st, nl);
 }
 
 cudaError_t launch_gemm1(const Params& p, bool ls, cudaStream_t st, int64_t* nl)
 {
     if (p.D == 64) {
-        if (p.T == 64) return ls ? launch_g1_t<64, 64, true>(p, st, nl) : launch_g1_t<64, 64, false>(p, st, nl);
-        return ls ? launch_g1_t<64, 128, true>(p, st, nl) : launch_g1_t<64, 128, false>(p, st, nl);
+        if (p.T == 64) return ls ? launch_g1_p<64, 64, true>(p, st, nl) : launch_g1_p<64, 64, false>(p, st, nl);
+        return ls ? launch_g1_p<64, 128, true>(p, st, nl) : launch_g1_p<64, 128, false>(p, st, nl);
     }
-    if (p.T == 64) return ls ? launch_g1_t<128, 64, true>(p, st, nl) : launch_g1_t<128, 64, false>(p, st, nl);
-    return ls ? launch_g1_t<128, 128, true>(p, st, nl) : launch_g1_t<128, 128, false>(p, st, nl);
+    if (p.T == 64) return ls ? launch_g1_p<128, 64, true>(p, st, nl) : launch_g1_p<128, 64, false>(p, st, nl);
+    return ls ? launch_g1_p<128, 128, true>(p, st, nl) : launch_g1_p<128, 128, false>(p, st, nl);
 }
 
 }  // namespace sr

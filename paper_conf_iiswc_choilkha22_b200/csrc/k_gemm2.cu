@@ -125,8 +125,8 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
             // warp walks the schedule; one elected lane issues)
             int s = 0;
             uint32_t sph = 0;
-            for (int it = it_begin; it < it_end; ++it) {
-                const ItemInfo I = decode_item(p, it);
+            for (ItemWalk iw(p, it_begin, it_end); iw.more();) {
+                const ItemInfo I = iw.next();
                 int wn[2];  // schedule words of the next macro tile, prefetched one step ahead
                 for (int u = 0; u < NSUB; ++u) wn[u] = I.t0 + u < I.t1 ? __ldg(p.sc.tinfo + I.t0 + u) : 0;
                 for (int t = I.t0; t < I.t1; t += NSUB) {
@@ -177,8 +177,8 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
             // L147), published as (m, 1/d) in a ring of NSI items.  Lane l reduces rows l + 32j.
             int si = 0;
             uint32_t sph = 0;
-            for (int it = it_begin; it < it_end; ++it) {
-                const ItemInfo I = decode_item(p, it);
+            for (ItemWalk iw(p, it_begin, it_end); iw.more();) {
+                const ItemInfo I = iw.next();
                 if (I.t0 == I.t1) continue;
                 mbar_wait(&st_empty[si], sph ^ 1);
                 float* ms = stats + si * 2 * kRowBlock;
@@ -234,8 +234,8 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
             // one elected lane issues)
             int s = 0;
             uint32_t sph = 0;
-            for (int it = it_begin; it < it_end; ++it) {
-                const ItemInfo I = decode_item(p, it);
+            for (ItemWalk iw(p, it_begin, it_end); iw.more();) {
+                const ItemInfo I = iw.next();
                 int wn[2];  // schedule words of the next macro tile, prefetched one step ahead
                 for (int u = 0; u < NSUB; ++u) wn[u] = I.t0 + u < I.t1 ? __ldg(p.sc.tinfo + I.t0 + u) : 0;
                 for (int t = I.t0; t < I.t1; t += NSUB) {

@@ -36,6 +36,13 @@ struct DevSched {
     const int32_t* tinfo;   // [n_tiles_list]
     const int32_t* items;   // [n_items] g * n_rb + rb; grouped by persistent CTA, longest first
     const int32_t* cta_ptr; // [n_cta + 1]: CTA c runs items[cta_ptr[c] .. cta_ptr[c+1])
+    const int4* item_desc;  // [n_items] {item, t0, t1, tp[lh][0]}: one 16-B load per item decode
+    // GEMM1 pair schedule (row-blocks 2j, 2j+1 share K tiles): pair items {g * n_pair + j, e0, e1,
+    // tp[lh][0]} grouped per CTA by pcta_ptr; pent[e] = {kt | ha << 16 | hb << 18, ta, tb, 0}
+    const int4* pair_desc;
+    const int4* pent;
+    const int32_t* pcta_ptr;
+    int n_pair, n_pcta;
     const int32_t* kv_len;  // [B] or nullptr
     int n_rb, n_lh, lh_mode, slots_per_head, n_items, n_cta;
     int max_rb_tiles;       // longest tile list of one (layout head, row-block)
@@ -58,6 +65,7 @@ struct Params {
     int in_dtype, out_dtype;
     int stages;        // SR_RUN_* bits to launch
     int fuse_ir;       // SR_FUSE_IR: the IR sub-layer runs inside GEMM2
+    int g1_pair;       // GEMM1 walks pairs of row-blocks sharing each K tile (pair schedule)
     DevSched sc;
     void* xprime;      // X' tiles (recomposed) or score tiles S (unfused)
     void* pbuf;        // unfused: P tiles

@@ -16,20 +16,41 @@ struct ItemInfo {
     int64_t slot0;  // slot id of tile t is slot0 + t
 };
 
-__device__ __forceinline__ ItemInfo decode_item(const Params& p, int it)
+__device__ __forceinline__ int4 item_desc(const Params& p, int it)
 {
-    const DevSched& sc = p.sc;
-    const int item = __ldg(sc.items + it);
+    return it < 0 ? make_int4(0, 0, 0, 0) : __ldg(p.sc.item_desc + it);  // precomputed on the host
+}
+__device__ __forceinline__ ItemInfo item_info(const Params& p, int4 d)
+{
     ItemInfo r;
-    r.g = item / sc.n_rb;
-    r.rb = item % sc.n_rb;
-    const int lh = lh_of(sc, r.g, p.H);
-    const int32_t* tp = sc.tp + (size_t)lh * (sc.n_rb + 1);
-    r.t0 = __ldg(tp + r.rb);
-    r.t1 = __ldg(tp + r.rb + 1);
-    r.slot0 = (int64_t)r.g * sc.slots_per_head - __ldg(tp);
+    r.g = d.x / p.sc.n_rb;
+    r.rb = d.x % p.sc.n_rb;
+    r.t0 = d.y;
+    r.t1 = d.z;
+    r.slot0 = (int64_t)r.g * p.sc.slots_per_head - d.w;
     return r;
 }
+__device__ __forceinline__ ItemInfo decode_item(const Params& p, int it) { return item_info(p, item_desc(p, it)); }
+
+// Walks [it_begin, it_end) with the next item's descriptor load in flight while the current item
+// runs:  for (ItemWalk w(p, b, e); w.more(); ) { const ItemInfo I = w.next(); ... }
+struct ItemWalk {
+    const Params& p;
+    int it, end;
+    int4 nd;
+    __device__ __forceinline__ ItemWalk(const Params& p_, int b, int e) : p(p_), it(b), end(e)
+    {
+        nd = item_desc(p, it < end ? it : -1);
+    }
+    __device__ __forceinline__ bool more() const { return it < end; }
+    __device__ __forceinline__ ItemInfo next()
+    {
+        const ItemInfo I = item_info(p, nd);
+        ++it;
+        nd = item_desc(p, it < end ? it : -1);
+        return I;
+    }
+};
 
 // Attention-matrix tiles (X', S, P) are 128 rows x T keys of 16-bit values in the canonical
 // SWIZZLE_128B K-major layout [T/64][128 rows][64 cols]: row r of column-half h is 128 contiguous
