@@ -10,7 +10,7 @@
 // Macro tiles: as in GEMM1, MW = 128 keys per step -- with T = 64 two consecutive sub-tiles of the
 // item (any two key blocks) are stacked along the MMA K dimension, each scaled by its own r'.
 //
-// Warp roles (persistent CTA per SM, 384 threads):
+// Warp roles (persistent CTA per SM, 512 threads):
 //   warp 0      X' producer: the macro tile's X' sub-tiles (1-D bulk copies of their valid 64-row
 //               halves; the tiles are already in the UMMA SW128 K-major layout and adjacent in HBM) +
 //               their r' + a stage header, into an NX-deep ring, then an END header.  The ring is only
@@ -20,8 +20,10 @@
 //               O accumulators; walks the item list itself and publishes each item's output rows
 //               (or EMPTY / END) to the epilogue through an O header
 //   warp 2      TMEM allocator (512 columns: 2 x D for O, NA x MW/2 for the A operand ring)
-//   warps 4-7   GS transform: smem X' row -> fp32 x r' -> dtype -> tcgen05.st into TMEM (A operand)
-//   warps 8-11  epilogue: tcgen05.ld of O rows -> out dtype -> global
+//   warps 4-11  GS transform: smem X' row -> fp32 x r' -> dtype -> tcgen05.st into TMEM (A operand);
+//               warp w covers TMEM lane quadrant (w-4) % 4 and key half (w-4) / 4 of each macro tile
+//               (two warps per SM sub-partition: with one, GS alone bounded the kernel -- measured)
+//   warps 12-15 epilogue: tcgen05.ld of O rows -> out dtype -> global
 #include "tc_common.cuh"
 
 namespace sr {
@@ -62,14 +64,15 @@ struct G2 {
     static constexpr int OFF_TPTR = OFF_OHDR + NO * (int)sizeof(G2Hdr);
     static constexpr int SMEM_ = OFF_TPTR + 16 + 1024;
     static constexpr int SMEM = SMEM_ > 118 * 1024 ? SMEM_ : 118 * 1024;  // 1 CTA/SM (512 TMEM cols)
-    static constexpr int THREADS = 384;
+    static constexpr int THREADS = 512;
+    static constexpr int NGS = 8;  // GS warps
 };
 
 // FI (fused IR): the IR sub-layer runs inside this kernel -- warp 2 reduces each
 // item's m', d' into per-row (m, 1/d) ahead of the GS warps, the X' stages carry m' instead of r',
 // and GS forms r' = e^{m' - m} / d on the fly.  No IR launch, no r' round trip through HBM.
 template <int D, int T, bool GS, bool FI>
-__global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUtensorMap tmV, const Params p)
+__global__ void __launch_bounds__(512, 1) tc_gemm2(const __grid_constant__ CUtensorMap tmV, const Params p)
 {
     using C = G2<D, T>;
     constexpr int NSUB = C::NSUB;
@@ -95,12 +98,12 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
 
     const int warp = warp_uniform(), lane = threadIdx.x % 32;
     if (threadIdx.x == 0) {
-        for (int i = 0; i < C::NX; ++i) { mbar_init(&x_full[i], 1); mbar_init(&x_empty[i], 4); }
+        for (int i = 0; i < C::NX; ++i) { mbar_init(&x_full[i], 1); mbar_init(&x_empty[i], C::NGS); }
         for (int i = 0; i < C::NV; ++i) { mbar_init(&v_full[i], 1); mbar_init(&v_empty[i], 1); }
-        for (int i = 0; i < C::NA; ++i) { mbar_init(&a_full[i], 4); mbar_init(&a_empty[i], 1); }
+        for (int i = 0; i < C::NA; ++i) { mbar_init(&a_full[i], C::NGS); mbar_init(&a_empty[i], 1); }
         // o_full: O-header arrive + MMA commit; o_empty: one arrive per epilogue warp
         for (int i = 0; i < C::NO; ++i) { mbar_init(&o_full[i], 2); mbar_init(&o_empty[i], 4); }
-        for (int i = 0; i < C::NSI; ++i) { mbar_init(&st_full[i], 1); mbar_init(&st_empty[i], 4); }
+        for (int i = 0; i < C::NSI; ++i) { mbar_init(&st_full[i], 1); mbar_init(&st_empty[i], C::NGS); }
         fence_mbar_init();
     }
     if (warp == 3 && lane == 0) prefetch_tmap(&tmV);
@@ -134,7 +137,9 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
                     int hv[2] = {tinfo_half(wn[0]), NSUB > 1 ? tinfo_half(wn[1]) : 0};
                     for (int u = 0; u < NSUB; ++u) wn[u] = t + NSUB + u < I.t1 ? __ldg(p.sc.tinfo + t + NSUB + u) : 0;
                     uint32_t bytes = GS ? nsub * kRowBlock * 4 : 0;
+#ifndef SR_DIAG2_NOX
                     for (int u = 0; u < nsub; ++u) bytes += (hv[u] == 3 ? 2 : 1) * (T / 64) * (kHalf * 128);
+#endif
                     mbar_wait(&x_empty[s], sph ^ 1);
                     uint8_t* st = xstage(s);
                     if (elect_one()) {
@@ -142,6 +147,9 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
                                      hv[1], nsub, 0, 0, 0, 0};
                     mbar_arrive_expect_tx(&x_full[s], bytes);
                     const uint8_t* xs = src + (I.slot0 + t) * (int64_t)C::XS;  // sub-tiles t, t+1 are adjacent
+#ifdef SR_DIAG2_NOX
+                    if (false)
+#endif
                     if (hv[0] == 3 && (nsub == 1 || hv[1] == 3)) {
                         bulk_load(st, xs, nsub * C::XS, &x_full[s]);
                     } else {
@@ -244,7 +252,12 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
                     for (int u = 0; u < NSUB; ++u) wn[u] = t + NSUB + u < I.t1 ? __ldg(p.sc.tinfo + t + NSUB + u) : 0;
                     mbar_wait(&v_empty[s], sph ^ 1);
                     if (elect_one()) {
+#ifdef SR_DIAG2_NOV
+                        mbar_arrive(&v_full[s]);
+                        if (false)
+#else
                         mbar_arrive_expect_tx(&v_full[s], nsub * T * D * 2);
+#endif
                         for (int u = 0; u < nsub; ++u)
                             for (int h = 0; h < D / 64; ++h)
                                 tma_load_2d(vstage(s) + h * (kMW2 * 128) + u * (T * 128), &tmV, h * 64,
@@ -314,11 +327,12 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
             }
             post(SH_END, 0, true);
         }
-    } else if (warp >= 4 && warp < 8) {
+    } else if (warp >= 4 && warp < 4 + C::NGS) {
         // ------------------------------------------------------------------ GS transform
-        const int r = (warp % 4) * 32 + lane;
+        const int gq = (warp - 4) % 4, ch = (warp - 4) / 4;  // lane quadrant, key half (64 keys)
+        const int r = gq * 32 + lane;
         const int myhalf = r / kHalf;
-        const uint32_t lane_off = (uint32_t)((warp % 4) * 32) << 16;
+        const uint32_t lane_off = (uint32_t)(gq * 32) << 16;
         const bool bf = p.in_dtype == DT_BF16;
         int s = 0, a = 0, si = 0;
         uint32_t sph = 0, aph = 0, siph = 0;
@@ -350,23 +364,27 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
                         rr[u] = v;
                 }
             }
-            // the whole X' row (MW fp16 = 16 chunks of 16 B) into registers first: the loads overlap
-            // the wait for a free A buffer
-            uint4 xv[kMW2 / 8];
+            // this warp's half of the X' row (64 fp16 = 8 chunks of 16 B) into registers first: the
+            // loads overlap the wait for a free A buffer
+            uint4 xv[kMW2 / 16];
+#ifdef SR_DIAG2_NOGS
+            if (false)
+#endif
 #pragma unroll
-            for (int q = 0; q < kMW2 / 8; ++q)
-                if (rr[(q * 8) / T] != 0.f) xv[q] = lds128(xs_s + tile_chunk_off(r, q));
+            for (int q = 0; q < kMW2 / 16; ++q)
+                if (rr[((ch * 8 + q) * 8) / T] != 0.f) xv[q] = lds128(xs_s + tile_chunk_off(r, ch * 8 + q));
             mbar_wait(&a_empty[a], aph ^ 1);
             tc_fence_after();
             const uint32_t a_tm = tmem_a + lane_off + a * (kMW2 / 2);
 #pragma unroll
-            for (int c = 0; c < kMW2 / 32; ++c) {  // 32 keys -> 16 packed words per tcgen05.st
-                const int u = (c * 32) / T;         // sub-tile of these keys
+            for (int c2 = 0; c2 < 2; ++c2) {  // 32 keys -> 16 packed words per tcgen05.st
+                const int c = ch * 2 + c2;
+                const int u = (c * 32) / T;   // sub-tile of these keys
                 uint32_t pk[16];
                 if (rr[u] != 0.f) {
 #pragma unroll
                     for (int q4 = 0; q4 < 4; ++q4) {
-                        const uint4 x = xv[c * 4 + q4];
+                        const uint4 x = xv[c2 * 4 + q4];
                         const uint32_t xw[4] = {x.x, x.y, x.z, x.w};
 #pragma unroll
                         for (int w = 0; w < 4; ++w) {
@@ -384,7 +402,11 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
 #pragma unroll
                     for (int w = 0; w < 16; ++w) pk[w] = 0u;
                 }
+#ifndef SR_DIAG2_NOGS
                 tmem_st16(a_tm + c * 16, pk);
+#else
+                (void)pk;
+#endif
             }
             tmem_wait_st();
             tc_fence_before();
@@ -397,7 +419,7 @@ __global__ void __launch_bounds__(384, 1) tc_gemm2(const __grid_constant__ CUten
             if (lane == 0) mbar_arrive(&x_empty[s]);
             if (++s == C::NX) { s = 0; sph ^= 1; }
         }
-    } else if (warp >= 8) {
+    } else if (warp >= 4 + C::NGS) {
         // ------------------------------------------------------------------ output epilogue
         const int r = (warp % 4) * 32 + lane;
         const uint32_t lane_off = (uint32_t)((warp % 4) * 32) << 16;

@@ -4,7 +4,7 @@ cfgs=$1; shift
 for lib in "$@"; do
   for c in $cfgs; do
     if [ "$lib" = "-" ]; then L=""; else L="paper_conf_iiswc_choilkha22_b200/$lib"; fi
-    SR_MHA_LIB=$L timeout 300 python bench.py --config $c --no-all-configs --cpu-seconds 0.05 --steps 30 > gpurun_out/ab_${lib}_$c.json 2>gpurun_out/ab_${lib}_$c.err
+    SR_MHA_LIB=$L timeout 150 python bench.py --config $c --no-all-configs --cpu-seconds 0.05 --steps 30 > gpurun_out/ab_${lib}_$c.json 2>gpurun_out/ab_${lib}_$c.err
     python - "$lib" "$c" <<'PY'
 import json, sys
 lib, c = sys.argv[1], sys.argv[2]
