@@ -99,6 +99,17 @@ def alg_bytes(cfg, stored, T, out_bytes=None):
     return rec, unf
 
 
+def alg_bytes_ir_in_gemm1(cfg, stored, T):
+    """SR_IR_IN_GEMM1: GEMM1 writes X' and m' (no d'), plus (m, 1/d) per query row; GEMM2 reads
+    X', m' and the row statistics -- no IR kernel, no r'."""
+    e = 4 if cfg.dtype == "f32" else 2
+    bhsd = cfg.BH * cfg.S * cfg.D
+    rows_tiles = stored / T
+    rows = cfg.BH * cfg.S
+    return {"gemm1_ls_ir": 2 * bhsd * e + 2 * stored + 4 * rows_tiles + 8 * rows,
+            "gs_gemm2": 2 * stored + 4 * rows_tiles + 8 * rows + 2 * bhsd * e}
+
+
 def flops(cfg, stored):
     return 4.0 * cfg.D * stored  # two GEMMs, 2 flops per MAC, over stored score elements
 
@@ -145,12 +156,12 @@ class Layer:
             self.ws["sd"] = torch.empty(info["total_bytes"], dtype=torch.uint8, device=device)
         self.n_tiles, self.stored = sr.schedule_stats(self.mask, cfg.B, cfg.H, cfg.S, causal=cfg.causal, tile_n=tile_n)
 
-    def run(self, fused=True, stages=0, q=None, k=None, v=None, fuse_ir=False, sd=False):
+    def run(self, fused=True, stages=0, q=None, k=None, v=None, fuse_ir=False, sd=False, ir_in_gemm1=False):
         d = self.dev
         return self.sr.call(self.mask, q if q is not None else d["q"], k if k is not None else d["k"],
                             v if v is not None else d["v"], out=self.out, fused=fused, stages=stages,
                             workspace=self.ws["sd" if sd else fused], tile_n=self.tile_n, fuse_ir=fuse_ir, sd=sd,
-                            **self.kw)
+                            ir_in_gemm1=ir_in_gemm1, **self.kw)
 
 
 def timed(torch, fn, steps, warmup, flush, per_step_pre=None):
@@ -238,11 +249,21 @@ def gpu_arm(args, rank, world, local_rank):
         ms_unf = dist_max(torch, statistics.mean(timed(torch, lambda: L.run(fused=False), K, Wm, flush)), world)
 
     # ---- SURVEY NEXT-2 variant: the IR sub-layer folded into GEMM2 (SR_FUSE_IR), same workload
-    ms_fir = ms_sd = None
+    ms_fir = ms_sd = ms_g1ir = None
+    kern_g1ir = {}
     if cfg.dtype != "f32":
         L.run(fuse_ir=True)
         barrier(torch, world)
         ms_fir = dist_max(torch, statistics.mean(timed(torch, lambda: L.run(fuse_ir=True), K, Wm, flush)), world)
+        # the IR merged inside GEMM1 (SR_IR_IN_GEMM1): 2 kernels, GEMM2 normalises with (m, 1/d)
+        L.run(ir_in_gemm1=True)
+        ms_g1ir = dist_max(torch, statistics.mean(timed(torch, lambda: L.run(ir_in_gemm1=True), K, Wm, flush)),
+                           world)
+        g1b = alg_bytes_ir_in_gemm1(cfg, L.stored, L.T)
+        for name, bit in (("gemm1_ls_ir", 1), ("gs_gemm2", 4)):
+            t = statistics.mean(timed(torch, lambda b=bit: L.run(stages=b, ir_in_gemm1=True), K, Wm, flush))
+            kern_g1ir[name] = {"us": round(t * 1e3, 3), "alg_bytes": int(g1b[name]),
+                               "GB/s": round(g1b[name] / (t * 1e-3) / 1e9, 1)}
         L.run(sd=True)
         ms_sd = dist_max(torch, statistics.mean(timed(torch, lambda: L.run(sd=True), K, Wm, flush)), world)
         L.run()  # leave the paper-design intermediates (r') in the workspace for the stage timings
@@ -300,6 +321,9 @@ def gpu_arm(args, rank, world, local_rank):
                 L2.run(fuse_ir=True)
                 tf = statistics.mean(timed(torch, lambda: L2.run(fuse_ir=True), 10, 3, flush))
                 ent["fused_ir_layers_per_s"] = round(1e3 / tf, 1)
+                L2.run(ir_in_gemm1=True)
+                tg = statistics.mean(timed(torch, lambda: L2.run(ir_in_gemm1=True), 10, 3, flush))
+                ent["ir_in_gemm1_layers_per_s"] = round(1e3 / tg, 1)
             others[f"C{c2.idx}"] = ent
             del L2
             torch.cuda.empty_cache()
@@ -337,6 +361,11 @@ def gpu_arm(args, rank, world, local_rank):
                          "value": round(world * 1e3 / ms_fir, 2), "ms_per_step": round(ms_fir, 5),
                          "alg_bytes": int(sum(rec_b.values()) - 12 * L.stored / L.T - 4 * L.stored / L.T
                                           + 8 * L.stored / L.T + 4 * L.stored / L.T)},
+            "ir_in_gemm1": {"what": "IR merged inside GEMM1 by a warp of each CTA (owns whole rows); GEMM2 applies "
+                                    "1/d * e^(m'-m) in its prologue (2 kernels)",
+                            "value": round(world * 1e3 / ms_g1ir, 2), "ms_per_step": round(ms_g1ir, 5),
+                            "alg_bytes": int(sum(alg_bytes_ir_in_gemm1(cfg, L.stored, L.T).values())),
+                            "kernels": kern_g1ir},
             "sd": {"what": "decomposition without fusion: GEMM1 -> LS -> IR -> GS -> GEMM2 (PAPER.md SD, NEXT-1)",
                    "value": round(world * 1e3 / ms_sd, 2), "ms_per_step": round(ms_sd, 5),
                    "alg_bytes": int(sum(unf_b.values()) + 4 * L.stored + 24 * L.stored / L.T)}},

@@ -119,6 +119,14 @@ typedef struct {
  * between the unfused baseline and SDF.  Workspace: sr_workspace_bytes with
  * fused = 2. */
 #define SR_DECOMPOSE 32
+/* Variant bit (recomposed 16-bit path): the IR sub-layer runs inside GEMM1.  Each GEMM1 CTA owns
+ * whole query rows (every key tile of its row-blocks), so one warp of it merges the per-tile
+ * (m', d') of each row as the epilogue produces them (m = max m', d = sum
+ * e^{m'-m} d') and writes the row's (m, 1/d); GEMM2 applies the normalisation 1/d * e^{m'-m} to
+ * each X' tile in its prologue (L151).  Two kernels, no IR launch, no r' or d' round trip.
+ * Exclusive with SR_FUSE_IR and SR_DECOMPOSE; with SR_RUN_* stage bits SR_RUN_REDUCE is a no-op.
+ * Workspace: the same sr_workspace_bytes(fused = 1) (its rowstat region). */
+#define SR_IR_IN_GEMM1 64
 
 /* Entry points (north star).  Returns SR_OK after enqueueing the kernels on ex->stream. */
 sr_status sr_mha_dense(const void* q, const void* k, const void* v, void* out, int B, int H, int S,
@@ -154,6 +162,7 @@ typedef enum { SR_E_DENSE = 0, SR_E_BLOCKSPARSE = 1, SR_E_WINDOW = 2 } sr_entry;
  *            SWIZZLE_128B K-major layout [T/64][128 rows][64 cols] with the 16-byte chunk index
  *            XOR (row & 7); fp32 tiles are plain row-major [128][T].
  *   mprime, dprime, rprime   fp32 [slot id][128 rows]  (m' in natural-log units)
+ *   rowstat  fp32 [2][B*H*S]: per query row m (natural-log units), then 1/d (SR_IR_IN_GEMM1)
  */
 typedef struct {
     int32_t tile_n;           /* T actually used */
@@ -161,6 +170,7 @@ typedef struct {
     int64_t n_slots;          /* B*H*slots_per_head */
     int32_t xprime_elt_bytes; /* 2 (16-bit paths) or 4 (fp32 path) */
     size_t off_xprime, off_mprime, off_dprime, off_rprime, off_p;  /* off_p: unfused P region */
+    size_t off_rowstat;       /* recomposed: per-row (m, 1/d) of the SR_IR_IN_GEMM1 variant */
     size_t total_bytes;
 } sr_ws_info;
 

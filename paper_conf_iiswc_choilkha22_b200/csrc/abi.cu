@@ -465,6 +465,7 @@ void ws_layout(const HostSched& h, int B, int H, int in_dtype, int fused, sr_ws_
         info->off_mprime = o; o = align_up(o + stat_bytes, 1024);
         info->off_dprime = o; o = align_up(o + stat_bytes, 1024);
         info->off_rprime = o; o = align_up(o + stat_bytes, 1024);
+        info->off_rowstat = o; o = align_up(o + (size_t)2 * B * H * h.n_rb * kRowBlock * sizeof(float), 1024);
     }
     info->total_bytes = std::max<size_t>(o, 1024);
 }
@@ -482,12 +483,15 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
     if (!ex) return fail(SR_ERR_INVALID, "exec descriptor is NULL");
     if (!q || !k || !v || !out) return fail(SR_ERR_INVALID, "q, k, v and out must be non-NULL");
     if (!std::isfinite(scale) || !(scale > 0.f)) return fail(SR_ERR_INVALID, "scale must be finite and > 0");
-    if (ex->flags & ~(SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2 | SR_FUSE_IR | SR_DECOMPOSE))
+    const int variant_bits = SR_FUSE_IR | SR_DECOMPOSE | SR_IR_IN_GEMM1;
+    if (ex->flags & ~(SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2 | variant_bits))
         return fail(SR_ERR_INVALID, "unknown flags 0x%x", ex->flags);
-    if ((ex->flags & (SR_FUSE_IR | SR_DECOMPOSE)) && (!fused || ex->in_dtype == SR_F32))
-        return fail(SR_ERR_UNSUPPORTED, "SR_FUSE_IR / SR_DECOMPOSE apply to the recomposed 16-bit path only");
-    if ((ex->flags & SR_FUSE_IR) && (ex->flags & SR_DECOMPOSE))
-        return fail(SR_ERR_INVALID, "SR_FUSE_IR and SR_DECOMPOSE are exclusive");
+    if ((ex->flags & variant_bits) && (!fused || ex->in_dtype == SR_F32))
+        return fail(SR_ERR_UNSUPPORTED, "SR_FUSE_IR / SR_DECOMPOSE / SR_IR_IN_GEMM1 apply to the recomposed 16-bit path only");
+    {
+        const int v = ex->flags & variant_bits;
+        if (v & (v - 1)) return fail(SR_ERR_INVALID, "SR_FUSE_IR, SR_DECOMPOSE and SR_IR_IN_GEMM1 are exclusive");
+    }
     if (fused && (ex->flags & SR_DECOMPOSE)) fused = 2;  // SD: workspace mode 2
     Request r;
     sr_status s = check_request(e, B, H, S, D, ex->in_dtype, mask_or_layout, causal, ex->tile_n, r);
@@ -528,7 +532,7 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
     p.sc = cs->dev;
     const int stage_bits = ex->flags & (SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2);
     p.stages = stage_bits ? stage_bits : (SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2);
-    p.fuse_ir = (ex->flags & SR_FUSE_IR) ? 1 : 0;
+    p.ir_mode = (ex->flags & SR_FUSE_IR) ? IR_IN_GEMM2 : ((ex->flags & SR_IR_IN_GEMM1) ? IR_IN_GEMM1 : IR_KERNEL);
     {   // GEMM1 pair schedule: SR_G1_PAIR=0/1 overrides the default (experiments)
         static const int env_pair = [] { const char* e = getenv("SR_G1_PAIR"); return e ? atoi(e) : -1; }();
         // default: pairs when K tiles are as large as the X' tiles they produce (D = 128) and there
@@ -542,6 +546,7 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
         p.mprime = (float*)(ws + wi.off_mprime);
         p.dprime = (float*)(ws + wi.off_dprime);
         p.rprime = (float*)(ws + wi.off_rprime);
+        p.rowstat = (float*)(ws + wi.off_rowstat);
     }
     if (fused != 1) p.pbuf = ws + wi.off_p;
     cudaStream_t st = (cudaStream_t)ex->stream;

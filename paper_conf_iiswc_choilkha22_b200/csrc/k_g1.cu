@@ -63,20 +63,24 @@ struct G1 {
     static constexpr int NACC = 512 / kMW;        // TMEM accumulators
     // staging buffers per epilogue warpgroup (2 if at all possible: the X' store stream is the
     // bottleneck), then Q double-buffered if shared memory still allows
-    static constexpr int XPW = ((PAIR ? 2 * QS : QS) + 2 * KB + EPI_WG * 2 * SB + 4096 <= kSmemMax) ? 2 : 1;
+    // statistics ring for the IR-in-GEMM1 variant: per accumulator, NSUB x (m', d') x 128 rows fp32
+    static constexpr int STB = NACC * 2 * 2 * kRowBlock * 4;
+    static constexpr int SLACK = 4096 + STB;
+    static constexpr int XPW = ((PAIR ? 2 * QS : QS) + 2 * KB + EPI_WG * 2 * SB + SLACK <= kSmemMax) ? 2 : 1;
 #ifndef SR_G1_MAX_NQ
 #define SR_G1_MAX_NQ 2
 #endif
-    static constexpr int NQ = (SR_G1_MAX_NQ >= 2 && 2 * QS + 2 * KB + EPI_WG * XPW * SB + 4096 <= kSmemMax) ? 2 : 1;
-    static constexpr int NK_ = (kSmemMax - 4096 - NQ * QS - EPI_WG * XPW * SB) / KB;
+    static constexpr int NQ = (SR_G1_MAX_NQ >= 2 && 2 * QS + 2 * KB + EPI_WG * XPW * SB + SLACK <= kSmemMax) ? 2 : 1;
+    static constexpr int NK_ = (kSmemMax - SLACK - NQ * QS - EPI_WG * XPW * SB) / KB;
     static constexpr int NK = NK_ > 4 ? 4 : NK_;
     static_assert(NK >= 2, "smem budget");
     static constexpr int OFF_Q = 0;
     static constexpr int OFF_K = OFF_Q + NQ * QS;
     static constexpr int OFF_X = OFF_K + NK * KB;
     static constexpr int OFF_BAR = OFF_X + EPI_WG * XPW * SB;
-    static constexpr int NBAR = 2 * NQ + 2 * NK + 2 * NACC;
-    static constexpr int OFF_HDR = OFF_BAR + NBAR * 8;
+    static constexpr int NBAR = 2 * NQ + 2 * NK + 4 * NACC;
+    static constexpr int OFF_STATS = OFF_BAR + NBAR * 8;
+    static constexpr int OFF_HDR = OFF_STATS + STB;
     static constexpr int OFF_TPTR = OFF_HDR + NACC * (int)sizeof(G1Hdr);
     static constexpr int SMEM_ = OFF_TPTR + 16 + 1024;  // + alignment slack
     static constexpr int SMEM = SMEM_ > 118 * 1024 ? SMEM_ : 118 * 1024;  // 1 CTA/SM (512 TMEM cols)
@@ -84,7 +88,10 @@ struct G1 {
     static constexpr int THREADS = 128 + EPI_WG * 128;
 };
 
-template <int D, int T, bool LS, bool PAIR>
+// IRT: the IR sub-layer runs in this kernel (SR_IR_IN_GEMM1): every CTA owns whole rows (all key
+// tiles of its row-blocks), so warp 3 merges the epilogue's per-tile (m', d') of each row as they
+// are produced and, at the end of the row-block, writes the row's (m, 1/d) -- see the IR warp below.
+template <int D, int T, bool LS, bool PAIR, bool IRT>
 __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
     tc_gemm1(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmK, const Params p)
 {
@@ -100,6 +107,9 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
     uint64_t* k_empty = k_full + C::NK;
     uint64_t* acc_full = k_empty + C::NK;
     uint64_t* acc_empty = acc_full + C::NACC;
+    uint64_t* st_full = acc_empty + C::NACC;  // IRT: per-accumulator (m', d') of its rows staged
+    uint64_t* st_empty = st_full + C::NACC;   // IRT: ... and merged by the IR warp
+    float* stats = (float*)(smem + C::OFF_STATS);  // [NACC][NSUB][m' | d'][128]
     G1Hdr* hdr = (G1Hdr*)(smem + C::OFF_HDR);
     uint32_t* tmem_ptr = (uint32_t*)(smem + C::OFF_TPTR);
 
@@ -110,6 +120,7 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
         // acc_full: header arrive (MMA thread) + tcgen05.commit; acc_empty: one arrive per epilogue
         // warp that reads the accumulator (the warpgroup pair in SPLIT, one warpgroup in FULL)
         for (int i = 0; i < C::NACC; ++i) { mbar_init(&acc_full[i], 2); mbar_init(&acc_empty[i], SPLIT ? 8 : 4); }
+        for (int i = 0; i < C::NACC; ++i) { mbar_init(&st_full[i], SPLIT ? 8 : 4); mbar_init(&st_empty[i], 1); }
         fence_mbar_init();
     }
     if (warp == 0 && lane == 0) { prefetch_tmap(&tmQ); prefetch_tmap(&tmK); }
@@ -372,6 +383,77 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
                 }
                 __syncwarp();
             }
+        } else if (IRT && warp == 3) {
+            // -------------------------------------------------------------- IR warp (SR_IR_IN_GEMM1)
+            // The IR sub-layer of every row this CTA owns: per accumulator (in
+            // the MMA warp's order) merge the staged (m'_k, d'_k) of each row into a running
+            //   m = max_k m'_k,   d = sum_k e^{m'_k - m} d'_k
+            // and at the end of a row-block write m (natural-log units) and 1/d; GEMM2 forms
+            // r'_k = e^{m'_k - m} / d in its prologue.  Lane l owns rows l + 32 j of a row-block.
+            const float sl2 = p.scale_log2;
+            int n = 0;
+            auto merge = [&](float (&m)[4], float (&d)[4]) {
+                const int buf = n % C::NACC;
+                mbar_wait(&st_full[buf], (uint32_t)(n / C::NACC) & 1);
+                const float* sb = stats + buf * (4 * kRowBlock);
+#pragma unroll
+                for (int s = 0; s < NSUB; ++s)
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) {
+                        const float mk = sb[(2 * s) * kRowBlock + lane + 32 * j];  // raw score units
+                        const float dk = sb[(2 * s + 1) * kRowBlock + lane + 32 * j];
+                        const float mn = fmaxf(m[j], mk);
+                        if (mn != -INFINITY) {  // ex2(-inf) = 0 covers an empty side
+                            d[j] = fmaf(d[j], ex2((m[j] - mn) * sl2), dk * ex2((mk - mn) * sl2));
+                            m[j] = mn;
+                        }
+                    }
+                __syncwarp();  // every lane's reads of the stage are done
+                if (lane == 0) mbar_arrive(&st_empty[buf]);
+                ++n;
+            };
+            auto flush = [&](int g, int rb, const float (&m)[4], const float (&d)[4]) {
+                const int64_t row = (int64_t)g * p.S + rb * kRowBlock + lane;
+                const int64_t nrow = (int64_t)p.B * p.H * p.S;
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    p.rowstat[row + 32 * j] = m[j] * p.scale;  // -inf stays -inf
+                    p.rowstat[nrow + row + 32 * j] = d[j] > 0.f ? 1.f / d[j] : 0.f;
+                }
+            };
+            if (PAIR) {
+                int4 nd = it_begin < it_end ? __ldg(p.sc.pair_desc + it_begin) : make_int4(0, 0, 0, 0);
+                for (int it = it_begin; it < it_end; ++it) {
+                    const int4 dd = nd;
+                    if (it + 1 < it_end) nd = __ldg(p.sc.pair_desc + it + 1);
+                    const int g = dd.x / p.sc.n_pair, j = dd.x % p.sc.n_pair, e0 = dd.y, e1 = dd.z;
+                    if (e0 == e1) continue;
+                    const int nrb = 2 * j + 1 < p.sc.n_rb ? 2 : 1;
+                    float m0[4], d0[4], m1[4], d1[4];
+#pragma unroll
+                    for (int u = 0; u < 4; ++u) { m0[u] = m1[u] = -INFINITY; d0[u] = d1[u] = 0.f; }
+                    for (int e = e0; e < e1; e += NSUB) {
+                        int hb = 0;  // union of the sub-tiles' half bits: bits 0-1 row-block 0, 2-3 row-block 1
+#pragma unroll
+                        for (int s2 = 0; s2 < NSUB; ++s2)
+                            if (e + s2 < e1) hb |= (__ldg(&p.sc.pent[e + s2].x) >> 16) & 15;
+                        if (hb & 3) merge(m0, d0);
+                        if (nrb == 2 && (hb & 12)) merge(m1, d1);
+                    }
+                    flush(g, 2 * j, m0, d0);
+                    if (nrb == 2) flush(g, 2 * j + 1, m1, d1);
+                }
+            } else {
+                for (ItemWalk iw(p, it_begin, it_end); iw.more();) {
+                    const ItemInfo I = iw.next();
+                    if (I.t0 == I.t1) continue;
+                    float m[4], d[4];
+#pragma unroll
+                    for (int u = 0; u < 4; ++u) { m[u] = -INFINITY; d[u] = 0.f; }
+                    for (int t = I.t0; t < I.t1; t += NSUB) merge(m, d);
+                    flush(I.g, I.rb, m, d);
+                }
+            }
         }
     } else if constexpr (SPLIT) {
         reg_alloc<104>();
@@ -496,9 +578,19 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
                 }
                 bulk_commit();
             }
+            if constexpr (IRT) {  // (m', d') of this row and sub-tile to the IR warp (-inf, 0 if invalid)
+                mbar_wait(&st_empty[buf], ((uint32_t)(n / C::NACC) & 1) ^ 1);
+                if (NSUB == 2 || h == 0) {
+                    float* sb = stats + buf * (4 * kRowBlock) + (NSUB == 2 ? 2 * h : 0) * kRowBlock;
+                    sb[r] = mx;
+                    sb[kRowBlock + r] = dsum;
+                }
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&st_full[buf]);
+            }
             if (LS && valid && (NSUB == 2 || h == 0)) {
                 p.mprime[slot * kRowBlock + r] = mx * p.scale;  // m' in natural-log units
-                p.dprime[slot * kRowBlock + r] = dsum;
+                if (!IRT) p.dprime[slot * kRowBlock + r] = dsum;
             }
         }
         if (lane == 0) bulk_wait0();
@@ -644,12 +736,23 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
                 }
                 bulk_commit();
             }
+            if constexpr (IRT) {  // (m', d') of this row per sub-tile to the IR warp (-inf, 0 if invalid)
+                mbar_wait(&st_empty[buf], ((uint32_t)(n / C::NACC) & 1) ^ 1);
+                float* sb = stats + buf * (4 * kRowBlock);
+#pragma unroll
+                for (int s = 0; s < NSUB; ++s) {
+                    sb[(2 * s) * kRowBlock + r] = mx[s];
+                    sb[(2 * s + 1) * kRowBlock + r] = dsum[s];
+                }
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&st_full[buf]);
+            }
             if (LS) {
 #pragma unroll
                 for (int s = 0; s < NSUB; ++s)
                     if (vs[s]) {
                         p.mprime[(slot + (s ? H.pad : 0)) * kRowBlock + r] = mx[s] * p.scale;  // natural-log units
-                        p.dprime[(slot + (s ? H.pad : 0)) * kRowBlock + r] = dsum[s];
+                        if (!IRT) p.dprime[(slot + (s ? H.pad : 0)) * kRowBlock + r] = dsum[s];
                     }
             }
         }
@@ -668,7 +771,7 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
 cudaError_t make_tmap_2d(CUtensorMap* m, const void* base, int64_t rows, int D, int box_rows, int dtype);
 int num_sms();
 
-template <int D, int T, bool LS, bool PAIR>
+template <int D, int T, bool LS, bool PAIR, bool IRT>
 cudaError_t launch_g1_t(const Params& p, cudaStream_t st, int64_t* nl)
 {
     using C = G1<D, T, PAIR>;
@@ -677,7 +780,7 @@ cudaError_t launch_g1_t(const Params& p, cudaStream_t st, int64_t* nl)
     cudaError_t e;
     if ((e = make_tmap_2d(&tq, p.q, rows, D, kRowBlock, p.in_dtype)) != cudaSuccess) return e;
     if ((e = make_tmap_2d(&tk, p.k, rows, D, T, p.in_dtype)) != cudaSuccess) return e;
-    auto kern = tc_gemm1<D, T, LS, PAIR>;
+    auto kern = tc_gemm1<D, T, LS, PAIR, IRT>;
     if ((e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM)) != cudaSuccess) return e;
     const int grid = PAIR ? p.sc.n_pcta : p.sc.n_cta;  // one persistent CTA per SM, host LPT items
     return launch_pdl(kern, dim3(grid), dim3(C::THREADS), C::SMEM, st, nl, tq, tk, p);
@@ -686,7 +789,9 @@ cudaError_t launch_g1_t(const Params& p, cudaStream_t st, int64_t* nl)
 template <int D, int T, bool LS>
 cudaError_t launch_g1_p(const Params& p, cudaStream_t st, int64_t* nl)
 {
-    return p.g1_pair ? launch_g1_t<D, T, LS, true>(p, st, nl) : launch_g1_t<D, T, LS, false>(p, st, nl);
+    if (LS && p.ir_mode == IR_IN_GEMM1)
+        return p.g1_pair ? launch_g1_t<D, T, LS, true, LS>(p, st, nl) : launch_g1_t<D, T, LS, false, LS>(p, st, nl);
+    return p.g1_pair ? launch_g1_t<D, T, LS, true, false>(p, st, nl) : launch_g1_t<D, T, LS, false, false>(p, st, nl);
 }
 
 cudaError_t launch_gemm1(const Params& p, bool ls, cudaStream_t st, int64_t* nl)

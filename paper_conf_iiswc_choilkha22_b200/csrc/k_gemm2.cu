@@ -71,7 +71,9 @@ struct G2 {
 // FI (fused IR): the IR sub-layer runs inside this kernel -- warp 2 reduces each
 // item's m', d' into per-row (m, 1/d) ahead of the GS warps, the X' stages carry m' instead of r',
 // and GS forms r' = e^{m' - m} / d on the fly.  No IR launch, no r' round trip through HBM.
-template <int D, int T, bool GS, bool FI>
+// RS (SR_IR_IN_GEMM1): as FI, but GEMM1 already merged the rows, so warp 2 only loads each item's
+// per-row (m, 1/d) -- GEMM2 applies the normalisation 1/d * e^{m' - m} in its prologue.
+template <int D, int T, bool GS, bool FI, bool RS>
 __global__ void __launch_bounds__(512, 1) tc_gemm2(const __grid_constant__ CUtensorMap tmV, const Params p)
 {
     using C = G2<D, T>;
@@ -179,7 +181,34 @@ __global__ void __launch_bounds__(512, 1) tc_gemm2(const __grid_constant__ CUten
             __syncwarp();
         }
     } else if (warp == 2) {
-        if (FI) {
+        if (RS) {
+            // -------------------------------------------------------------- row statistics of the
+            // IR merged in GEMM1: (m, 1/d) of the item's 128 rows into the ring (lane: rows l + 32 j)
+            int si = 0;
+            uint32_t sph = 0;
+            const int64_t nrow = (int64_t)p.B * p.H * p.S;
+            for (ItemWalk iw(p, it_begin, it_end); iw.more();) {
+                const ItemInfo I = iw.next();
+                if (I.t0 == I.t1) continue;
+                const int64_t row = (int64_t)I.g * p.S + I.rb * kRowBlock + lane;
+                float mv[4], iv[4];
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    mv[j] = __ldcg(p.rowstat + row + 32 * j);
+                    iv[j] = __ldcg(p.rowstat + nrow + row + 32 * j);
+                }
+                mbar_wait(&st_empty[si], sph ^ 1);
+                float* ms = stats + si * 2 * kRowBlock;
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    ms[lane + 32 * j] = mv[j];
+                    ms[kRowBlock + lane + 32 * j] = iv[j];
+                }
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&st_full[si]);
+                if (++si == C::NSI) { si = 0; sph ^= 1; }
+            }
+        } else if (FI) {
             // -------------------------------------------------------------- fused IR (NEXT-2)
             // Per non-empty item, per row: m = max_k m'_k, d = sum_k e^{m'_k - m} d'_k (PAPER.md
             // L147), published as (m, 1/d) in a ring of NSI items.  Lane l reduces rows l + 32j.
@@ -484,7 +513,7 @@ __global__ void __launch_bounds__(512, 1) tc_gemm2(const __grid_constant__ CUten
 cudaError_t make_tmap_2d(CUtensorMap* m, const void* base, int64_t rows, int D, int box_rows, int dtype);
 int num_sms();
 
-template <int D, int T, bool GS, bool FI>
+template <int D, int T, bool GS, bool FI, bool RS>
 cudaError_t launch_g2_t(const Params& p, cudaStream_t st, int64_t* nl)
 {
     using C = G2<D, T>;
@@ -492,7 +521,7 @@ cudaError_t launch_g2_t(const Params& p, cudaStream_t st, int64_t* nl)
     const int64_t rows = (int64_t)p.B * p.H * p.S;
     cudaError_t e;
     if ((e = make_tmap_2d(&tv, p.v, rows, D, T, p.in_dtype)) != cudaSuccess) return e;
-    auto kern = tc_gemm2<D, T, GS, FI>;
+    auto kern = tc_gemm2<D, T, GS, FI, RS>;
     if ((e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM)) != cudaSuccess) return e;
     const int grid = p.sc.n_cta;  // one persistent CTA per SM, items assigned by host LPT
     return launch_pdl(kern, dim3(grid), dim3(C::THREADS), C::SMEM, st, nl, tv, p);
@@ -501,12 +530,14 @@ cudaError_t launch_g2_t(const Params& p, cudaStream_t st, int64_t* nl)
 template <int D, int T>
 cudaError_t launch_g2_dt(const Params& p, int mode, cudaStream_t st, int64_t* nl)
 {
-    if (mode == 0) return launch_g2_t<D, T, false, false>(p, st, nl);
-    if (mode == 1) return launch_g2_t<D, T, true, false>(p, st, nl);
-    return launch_g2_t<D, T, true, true>(p, st, nl);
+    if (mode == 0) return launch_g2_t<D, T, false, false, false>(p, st, nl);
+    if (mode == 1) return launch_g2_t<D, T, true, false, false>(p, st, nl);
+    if (mode == 2) return launch_g2_t<D, T, true, true, false>(p, st, nl);
+    return launch_g2_t<D, T, true, true, true>(p, st, nl);
 }
 
-// mode: 0 = unfused baseline (P . V), 1 = GS + GEMM2 (r' from the IR kernel), 2 = IR + GS + GEMM2
+// mode: 0 = unfused baseline (P . V), 1 = GS + GEMM2 (r' from the IR kernel), 2 = IR + GS + GEMM2,
+// 3 = GS + GEMM2 on the (m, 1/d) rows GEMM1 merged
 cudaError_t launch_gemm2(const Params& p, int mode, cudaStream_t st, int64_t* nl)
 {
     if (p.D == 64) return p.T == 64 ? launch_g2_dt<64, 64>(p, mode, st, nl) : launch_g2_dt<64, 128>(p, mode, st, nl);

@@ -20,6 +20,9 @@ namespace sr {
 constexpr int kRowBlock = 128;  // M of every tcgen05 tile
 constexpr int kHalf = 64;       // validity granularity of tile rows
 
+// Where the IR sub-layer runs: its own kernel (the paper's design), folded into
+// GEMM2 (SR_FUSE_IR), or merged by a warp of GEMM1 as the row's tiles are produced (SR_IR_IN_GEMM1).
+enum IrMode : int { IR_KERNEL = 0, IR_IN_GEMM2 = 1, IR_IN_GEMM1 = 2 };
 enum MaskKind : int { MK_DENSE = 0, MK_BLOCK = 1, MK_WINDOW = 2 };
 enum DType : int { DT_F32 = 0, DT_F16 = 1, DT_BF16 = 2 };
 // lh_mode: which layout list a head g = b*H + h uses
@@ -64,7 +67,7 @@ struct Params {
     int n_global;
     int in_dtype, out_dtype;
     int stages;        // SR_RUN_* bits to launch
-    int fuse_ir;       // SR_FUSE_IR: the IR sub-layer runs inside GEMM2
+    int ir_mode;       // IrMode: where the IR sub-layer runs
     int g1_pair;       // GEMM1 walks pairs of row-blocks sharing each K tile (pair schedule)
     DevSched sc;
     void* xprime;      // X' tiles (recomposed) or score tiles S (unfused)
@@ -72,6 +75,7 @@ struct Params {
     float* mprime;
     float* dprime;
     float* rprime;
+    float* rowstat;    // IR_IN_GEMM1: per query row m (natural log) at [0, BHS), 1/d at [BHS, 2 BHS)
 };
 
 __host__ __device__ inline int lh_of(const DevSched& s, int g, int H)

@@ -34,11 +34,12 @@ def _ulp_half(dtype, ref):
 
 
 def run_case(kind, B, H, S, D, dtype, *, causal=False, kv_len=None, layout=None, window=0, n_global=0,
-             tile_n=0, fused=True, seed=0, out_f32=True, fuse_ir=False):
+             tile_n=0, fused=True, seed=0, out_f32=True, fuse_ir=False, ir_in_gemm1=False):
     t, q, k, v = qkv(B, H, S, D, dtype, seed)
     scale = 1 / math.sqrt(D)
     od = torch.float32 if out_f32 else TORCH[dtype]
-    kw = dict(scale=scale, causal=causal, tile_n=tile_n, fused=fused, out_dtype=od, fuse_ir=fuse_ir)
+    kw = dict(scale=scale, causal=causal, tile_n=tile_n, fused=fused, out_dtype=od, fuse_ir=fuse_ir,
+              ir_in_gemm1=ir_in_gemm1)
     if kind == "dense":
         o = sr.mha_dense(q, k, v, kv_len=kv_len, **kw)
     elif kind == "block":
@@ -238,6 +239,31 @@ def test_intermediates_match_recomposed_oracle():
                 np.testing.assert_allclose(rp[g, s], rp_ref[g, kt, rows], rtol=2e-3, atol=1e-7)
 
 
+@pytest.mark.parametrize("T", [64, 128])
+def test_row_statistics_ir_in_gemm1(T):
+    """SR_IR_IN_GEMM1: the per-row (m, 1/d) GEMM1's IR warp writes vs the oracle's Eq. (2) values:
+    m = max_k m'_k, and 1/d = max_k r'_k (r'_k = e^{m'_k - m}/d is 1/d on the tile holding the max)."""
+    B, H, S, D = 2, 2, 384, 64
+    t, q, k, v = qkv(B, H, S, D, "f16", seed=4)
+    kv = [384, 200]
+    mask = sr.dense_mask(kv)
+    info = sr.workspace_info(mask, B, H, S, D, sr.SR_F16, causal=True, tile_n=T)
+    ws = torch.zeros(info["total_bytes"], dtype=torch.uint8, device="cuda")
+    o = sr.call(mask, q, k, v, scale=0.125, causal=True, tile_n=T, workspace=ws, ir_in_gemm1=True,
+                out_dtype=torch.float32)
+    torch.cuda.synchronize()
+    om = oracle.Mask(causal=True, kv_len=kv)
+    o_ref, mp_ref, dp_ref, rp_ref = oracle.recomposed(t.q64, t.k64, t.v64, 0.125, T, om)
+    assert_close(o.double().cpu().numpy(), o_ref, "f16", what="ir_in_gemm1 output")
+    n = B * H * S
+    rs = ws[info["off_rowstat"]:].view(torch.float32)[:2 * n].cpu().numpy().reshape(2, B * H, S)
+    with np.errstate(invalid="ignore"):
+        m_ref = mp_ref.max(axis=1)  # [BH, S] over the row's sub-vectors
+        invd_ref = rp_ref.max(axis=1)
+    np.testing.assert_allclose(rs[0], m_ref, atol=2e-5)
+    np.testing.assert_allclose(rs[1], invd_ref, rtol=2e-3)
+
+
 def test_T64_equals_T128():
     """Pin P5 on the GPU: sub-vector width 64 and 128 give the same context within tolerance."""
     o64, ref = run_case("dense", 2, 2, 512, 64, "f16", causal=True, tile_n=64)
@@ -341,26 +367,32 @@ FUSED_IR_CASES = [
 ]
 
 
+VARIANTS = ["fuse_ir", "ir_in_gemm1"]
+
+
+@pytest.mark.parametrize("variant", VARIANTS)
 @pytest.mark.parametrize("kind,kw", FUSED_IR_CASES, ids=lambda x: str(x)[:40] if isinstance(x, dict) else x)
-def test_fused_ir_variant(kind, kw):
-    """SR_FUSE_IR (IR folded into GEMM2) against the oracle, same tolerance."""
+def test_fused_ir_variant(kind, kw, variant):
+    """The IR placements against the oracle, same tolerance: SR_FUSE_IR (IR folded into GEMM2,
+    SURVEY NEXT-2) and SR_IR_IN_GEMM1 (rows merged by a GEMM1 warp, GEMM2 normalises)."""
     kw = dict(kw)
     if kw.get("layout") == "rand":
         kw["layout"] = W.random_layout(kw["H"], kw["S"] // 64, 64, 0.35, seed=8)
     B, H, S, D, dtype = (kw.pop(x) for x in ("B", "H", "S", "D", "dtype"))
-    o, ref = run_case(kind, B, H, S, D, dtype, fuse_ir=True, **kw)
+    o, ref = run_case(kind, B, H, S, D, dtype, **{variant: True}, **kw)
     if kw.get("kv_len") and 0 in kw["kv_len"]:
         assert np.all(o[list(kw["kv_len"]).index(0)] == 0)
-    assert_close(o, ref, dtype, what=f"fused-IR {kind}")
+    assert_close(o, ref, dtype, what=f"{variant} {kind}")
 
 
+@pytest.mark.parametrize("variant", VARIANTS)
 @pytest.mark.parametrize("idx", [2, 3, 4, 5])
-def test_fused_ir_full_configs(idx):
+def test_fused_ir_full_configs(idx, variant):
     cfg = W.config(idx)
     t = W.config_tensors(cfg)
     from tests.gpu_util import to_dev
     q, k, v = (to_dev(x, cfg.dtype) for x in (t.q_s, t.k_s, t.v_s))
-    kw = dict(scale=cfg.scale, out_dtype=torch.float32, fuse_ir=True)
+    kw = dict(scale=cfg.scale, out_dtype=torch.float32, **{variant: True})
     if cfg.kind == "dense":
         o = sr.mha_dense(q, k, v, kv_len=cfg.kv_len, causal=cfg.causal, **kw)
         m = oracle.Mask(kv_len=cfg.kv_len, causal=cfg.causal)
@@ -375,7 +407,7 @@ def test_fused_ir_full_configs(idx):
     rows = _sample_rows(cfg, 192, seed=idx + 50)
     ref = oracle.attention_rows(t.q64, t.k64, t.v64, cfg.scale, rows, m)
     got = o.reshape(-1, cfg.D)[torch.from_numpy(rows).cuda()].double().cpu().numpy()
-    assert_close(got, ref, cfg.dtype, what=f"fused-IR config {idx}")
+    assert_close(got, ref, cfg.dtype, what=f"{variant} config {idx}")
 
 
 # ------------------------------------------------------------------------------------ SD variant
