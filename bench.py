@@ -2,8 +2,10 @@
 """bench.py -- attention layers/s and HBM bytes/layer of the softmax-recomposed path vs the in-repo
 unfused path on B200 (BASELINE.json "metric").
 
-One step = one attention layer (all B*H heads of the workload config) through the C ABI: GEMM1 +
-Local Softmax -> IR -> GS + GEMM2.  Inputs are seeded synthetic tensors
+One step = one attention layer (all B*H heads of the workload config) through the C ABI's default
+path: GEMM1 + Local Softmax (+ the IR merge inside GEMM1) -> GS + GEMM2.
+The paper's three-kernel layout (standalone IR kernel, SR_IR_KERNEL) and the other variants are
+timed in the same run and reported under "variants".  Inputs are seeded synthetic tensors
 resident in HBM before the timed region; L2 is flushed (256 MiB write) before every timed step.
 Timing: CUDA events on the launching stream, barrier + synchronize around the timed region, max
 over ranks.  Multi-GPU (torchrun): every rank runs its own full layer on its own inputs (weak
@@ -85,8 +87,9 @@ class Clocks:
 # ----------------------------------------------------------------------------- byte model
 
 def alg_bytes(cfg, stored, T, out_bytes=None):
-    """Algorithmic HBM bytes per layer: Q, K, V, O once; the attention matrix
-    written and read once (recomposed) or four times (unfused); m', d', r'."""
+    """Algorithmic HBM bytes per layer of the paper's three-kernel layout
+    (SR_IR_KERNEL): Q, K, V, O once; the attention matrix written and read once (recomposed) or
+    four times (unfused); m', d' written, read by IR, r' written and read."""
     e = 4 if cfg.dtype == "f32" else 2
     eo = e if out_bytes is None else out_bytes
     bhsd = cfg.BH * cfg.S * cfg.D
@@ -100,8 +103,8 @@ def alg_bytes(cfg, stored, T, out_bytes=None):
 
 
 def alg_bytes_ir_in_gemm1(cfg, stored, T):
-    """SR_IR_IN_GEMM1: GEMM1 writes X' and m' (no d'), plus (m, 1/d) per query row; GEMM2 reads
-    X', m' and the row statistics -- no IR kernel, no r'."""
+    """Default path (IR merged in GEMM1): GEMM1 writes X' and m' (no d'), plus (m, 1/d) per query
+    row; GEMM2 reads X', m' and the row statistics -- no IR kernel, no r'."""
     e = 4 if cfg.dtype == "f32" else 2
     bhsd = cfg.BH * cfg.S * cfg.D
     rows_tiles = stored / T
@@ -156,12 +159,12 @@ class Layer:
             self.ws["sd"] = torch.empty(info["total_bytes"], dtype=torch.uint8, device=device)
         self.n_tiles, self.stored = sr.schedule_stats(self.mask, cfg.B, cfg.H, cfg.S, causal=cfg.causal, tile_n=tile_n)
 
-    def run(self, fused=True, stages=0, q=None, k=None, v=None, fuse_ir=False, sd=False, ir_in_gemm1=False):
+    def run(self, fused=True, stages=0, q=None, k=None, v=None, fuse_ir=False, sd=False, ir_kernel=False):
         d = self.dev
         return self.sr.call(self.mask, q if q is not None else d["q"], k if k is not None else d["k"],
                             v if v is not None else d["v"], out=self.out, fused=fused, stages=stages,
                             workspace=self.ws["sd" if sd else fused], tile_n=self.tile_n, fuse_ir=fuse_ir, sd=sd,
-                            ir_in_gemm1=ir_in_gemm1, **self.kw)
+                            ir_kernel=ir_kernel, **self.kw)
 
 
 def timed(torch, fn, steps, warmup, flush, per_step_pre=None):
@@ -249,32 +252,32 @@ def gpu_arm(args, rank, world, local_rank):
         ms_unf = dist_max(torch, statistics.mean(timed(torch, lambda: L.run(fused=False), K, Wm, flush)), world)
 
     # ---- SURVEY NEXT-2 variant: the IR sub-layer folded into GEMM2 (SR_FUSE_IR), same workload
-    ms_fir = ms_sd = ms_g1ir = None
-    kern_g1ir = {}
+    ms_fir = ms_sd = ms_irk = None
+    kern_irk = {}
+    rec_b, unf_b = alg_bytes(cfg, L.stored, L.T)
     if cfg.dtype != "f32":
         L.run(fuse_ir=True)
         barrier(torch, world)
         ms_fir = dist_max(torch, statistics.mean(timed(torch, lambda: L.run(fuse_ir=True), K, Wm, flush)), world)
-        # the IR merged inside GEMM1 (SR_IR_IN_GEMM1): 2 kernels, GEMM2 normalises with (m, 1/d)
-        L.run(ir_in_gemm1=True)
-        ms_g1ir = dist_max(torch, statistics.mean(timed(torch, lambda: L.run(ir_in_gemm1=True), K, Wm, flush)),
-                           world)
-        g1b = alg_bytes_ir_in_gemm1(cfg, L.stored, L.T)
-        for name, bit in (("gemm1_ls_ir", 1), ("gs_gemm2", 4)):
-            t = statistics.mean(timed(torch, lambda b=bit: L.run(stages=b, ir_in_gemm1=True), K, Wm, flush))
-            kern_g1ir[name] = {"us": round(t * 1e3, 3), "alg_bytes": int(g1b[name]),
-                               "GB/s": round(g1b[name] / (t * 1e-3) / 1e9, 1)}
+        # the paper's three-kernel layout (SR_IR_KERNEL): GEMM1 + LS -> IR kernel -> GS + GEMM2
+        L.run(ir_kernel=True)
+        ms_irk = dist_max(torch, statistics.mean(timed(torch, lambda: L.run(ir_kernel=True), K, Wm, flush)), world)
+        for name, key, bit in (("gemm1_ls", "gemm1_ls", 1), ("ir", "ir", 2), ("gs_gemm2_rprime", "gs_gemm2", 4)):
+            t = statistics.mean(timed(torch, lambda b=bit: L.run(stages=b, ir_kernel=True), K, Wm, flush))
+            kern_irk[name] = {"us": round(t * 1e3, 3), "alg_bytes": int(rec_b[key]),
+                              "GB/s": round(rec_b[key] / (t * 1e-3) / 1e9, 1)}
         L.run(sd=True)
         ms_sd = dist_max(torch, statistics.mean(timed(torch, lambda: L.run(sd=True), K, Wm, flush)), world)
-        L.run()  # leave the paper-design intermediates (r') in the workspace for the stage timings
+        L.run()  # leave the default path's intermediates in the workspace for its stage timings
 
     # ---- per-kernel durations inside the step (stage-selected launches, events on the stream)
-    rec_b, unf_b = alg_bytes(cfg, L.stored, L.T)
+    hb = alg_bytes_ir_in_gemm1(cfg, L.stored, L.T) if cfg.dtype != "f32" else rec_b
     kern = {}
-    for name, bit in (("gemm1_ls", 1), ("ir", 2), ("gs_gemm2", 4)):
+    stages = (("gemm1_ls_ir", 1), ("gs_gemm2", 4)) if cfg.dtype != "f32" else (("gemm1_ls", 1), ("ir", 2), ("gs_gemm2", 4))
+    for name, bit in stages:
         t = statistics.mean(timed(torch, lambda b=bit: L.run(stages=b), K, Wm, flush))
-        kern[name] = {"us": round(t * 1e3, 3), "alg_bytes": int(rec_b[name]),
-                      "GB/s": round(rec_b[name] / (t * 1e-3) / 1e9, 1)}
+        kern[name] = {"us": round(t * 1e3, 3), "alg_bytes": int(hb[name]),
+                      "GB/s": round(hb[name] / (t * 1e-3) / 1e9, 1)}
     kern_unf = {}
     if cfg.dtype != "f32":
         for name, bit in (("gemm1", 1), ("softmax", 2), ("gemm2", 4)):
@@ -308,6 +311,8 @@ def gpu_arm(args, rank, world, local_rank):
             L2.run()
             tr = statistics.mean(timed(torch, lambda: L2.run(), 10, 3, flush))
             r2, u2 = alg_bytes(c2, L2.stored, L2.T)
+            if c2.dtype != "f32":
+                r2 = alg_bytes_ir_in_gemm1(c2, L2.stored, L2.T)
             ent = {"layers_per_s": round(1e3 / tr, 1), "ms": round(tr, 4),
                    "alg_bytes_recomposed": int(sum(r2.values()))}
             if c2.dtype != "f32":
@@ -321,9 +326,9 @@ def gpu_arm(args, rank, world, local_rank):
                 L2.run(fuse_ir=True)
                 tf = statistics.mean(timed(torch, lambda: L2.run(fuse_ir=True), 10, 3, flush))
                 ent["fused_ir_layers_per_s"] = round(1e3 / tf, 1)
-                L2.run(ir_in_gemm1=True)
-                tg = statistics.mean(timed(torch, lambda: L2.run(ir_in_gemm1=True), 10, 3, flush))
-                ent["ir_in_gemm1_layers_per_s"] = round(1e3 / tg, 1)
+                L2.run(ir_kernel=True)
+                tg = statistics.mean(timed(torch, lambda: L2.run(ir_kernel=True), 10, 3, flush))
+                ent["ir_kernel_layers_per_s"] = round(1e3 / tg, 1)
             others[f"C{c2.idx}"] = ent
             del L2
             torch.cuda.empty_cache()
@@ -332,7 +337,7 @@ def gpu_arm(args, rank, world, local_rank):
         return None
     dom = max(kern, key=lambda n: kern[n]["us"])
     ncu = load_ncu_traffic().get(f"C{cfg.idx}", {})
-    achieved = rec_b[dom] / (kern[dom]["us"] * 1e-6) / 1e9
+    achieved = hb[dom] / (kern[dom]["us"] * 1e-6) / 1e9
     value = world * 1e3 / ms_step
     res = {
         "metric": METRIC,
@@ -349,8 +354,9 @@ def gpu_arm(args, rank, world, local_rank):
                    "tiles": L.n_tiles, "stored_score_elems": L.stored,
                    "l2": "flushed before every timed step (256 MiB write, then 256 MiB read of another buffer)" if flush is not None else "not flushed",
                    "parallelism": f"dp{world} (weak: each rank runs its own full layer on its own inputs)"},
-        "hbm_bytes_per_layer": {"recomposed_alg": int(sum(rec_b.values())), "unfused_alg": int(sum(unf_b.values())),
-                                "reduction_alg": round(1 - sum(rec_b.values()) / sum(unf_b.values()), 4),
+        "hbm_bytes_per_layer": {"recomposed_alg": int(sum(hb.values())), "unfused_alg": int(sum(unf_b.values())),
+                                "reduction_alg": round(1 - sum(hb.values()) / sum(unf_b.values()), 4),
+                                "recomposed_alg_ir_kernel": int(sum(rec_b.values())),
                                 "recomposed_ncu": ncu.get("recomposed_dram_bytes"),
                                 "unfused_ncu": ncu.get("unfused_dram_bytes")},
         "unfused": None if ms_unf is None else {"value": round(world * 1e3 / ms_unf, 2), "ms_per_step": round(ms_unf, 5),
@@ -361,11 +367,10 @@ def gpu_arm(args, rank, world, local_rank):
                          "value": round(world * 1e3 / ms_fir, 2), "ms_per_step": round(ms_fir, 5),
                          "alg_bytes": int(sum(rec_b.values()) - 12 * L.stored / L.T - 4 * L.stored / L.T
                                           + 8 * L.stored / L.T + 4 * L.stored / L.T)},
-            "ir_in_gemm1": {"what": "IR merged inside GEMM1 by a warp of each CTA (owns whole rows); GEMM2 applies "
-                                    "1/d * e^(m'-m) in its prologue (2 kernels)",
-                            "value": round(world * 1e3 / ms_g1ir, 2), "ms_per_step": round(ms_g1ir, 5),
-                            "alg_bytes": int(sum(alg_bytes_ir_in_gemm1(cfg, L.stored, L.T).values())),
-                            "kernels": kern_g1ir},
+            "ir_kernel": {"what": "the paper's three-kernel layout: GEMM1+LS -> standalone IR kernel (writes r') -> "
+                                  "GS+GEMM2 (SR_IR_KERNEL, PAPER.md L165-L173)",
+                          "value": round(world * 1e3 / ms_irk, 2), "ms_per_step": round(ms_irk, 5),
+                          "alg_bytes": int(sum(rec_b.values())), "kernels": kern_irk},
             "sd": {"what": "decomposition without fusion: GEMM1 -> LS -> IR -> GS -> GEMM2 (PAPER.md SD, NEXT-1)",
                    "value": round(world * 1e3 / ms_sd, 2), "ms_per_step": round(ms_sd, 5),
                    "alg_bytes": int(sum(unf_b.values()) + 4 * L.stored + 24 * L.stored / L.T)}},

@@ -7,12 +7,16 @@
  * library computes it through the paper's softmax recomposition (Sec. 3.2-3.4):
  *
  *   kernel 1  GEMM1 + LS   x = Q K^T * scale, mask; per 128-row x T-column output tile the
- *                          epilogue computes the Local Softmax (Eq. 2): m' = row max of the tile,
- *                          X' = e^{x - m'} (written once), d' = row sum of X'     (L131-L145, L165)
- *   kernel 2  IR           per row: m = max_k m'_k, d = sum_k e^{m'_k - m} d'_k,
- *                          r'_k = e^{m'_k - m} / d                                 (L147-L149, L173)
- *   kernel 3  GS + GEMM2   the prologue scales each X' tile row by its r' (Global Scaling, L151)
- *                          as the tile is loaded, then O += Y V on the tensor cores (L165)
+ *             (+ IR)       epilogue computes the Local Softmax (Eq. 2): m' = row max of the tile,
+ *                          X' = e^{x - m'} (written once), d' = row sum of X'     (L131-L145, L165).
+ *                          The Inter-sub-vector Reduction runs in the same kernel: a GEMM1 CTA owns
+ *                          whole rows, so two of its warps merge each row's (m'_k, d'_k) as they are
+ *                          produced: m = max_k m'_k, d = sum_k e^{m'_k - m} d'_k  (L147-L149)
+ *   kernel 2  GS + GEMM2   the prologue scales each X' tile row by r'_k = e^{m'_k - m} / d (Global
+ *                          Scaling, L151) as the tile is loaded, then O += Y V on the tensor cores
+ *
+ * The paper's own layout -- IR as a third, standalone kernel writing r' (L173) -- is the
+ * SR_IR_KERNEL variant; SR_FUSE_IR and SR_DECOMPOSE are the other variants (see below).
  *
  * The attention matrix therefore crosses HBM twice instead of four times (L171-L173).  The
  * *_unfused entry points run the deliberately unfused baseline GEMM1 -> row softmax -> GEMM2
@@ -105,13 +109,13 @@ typedef struct {
 
 /* Stage bits for sr_exec.flags. */
 #define SR_RUN_GEMM1 1   /* GEMM1 + LS (recomposed) / GEMM1 writing scores (unfused) */
-#define SR_RUN_REDUCE 2  /* IR (recomposed) / row softmax (unfused) */
+#define SR_RUN_REDUCE 2  /* IR kernel (SR_IR_KERNEL variant) / row softmax (unfused); no-op otherwise */
 #define SR_RUN_GEMM2 4   /* GS + GEMM2 (recomposed) / GEMM2 on P (unfused) */
-/* Variant bit for sr_exec.flags (recomposed 16-bit path): fold the IR sub-layer into GEMM2 (one
- * warp of each GEMM2 CTA reduces the item's m', d' before its GS warps need them; r' is formed on
- * the fly and never written).  Same results up to rounding; one kernel and the r' round trip
- * fewer.  SURVEY.md NEXT-2 -- a B200-specific departure from the paper's separate IR kernel
- * (PAPER.md L173), off by default.  With SR_RUN_* stage bits, SR_RUN_REDUCE is then a no-op. */
+/* Variant bits for sr_exec.flags (recomposed 16-bit path; at most one).  Same results up to
+ * rounding.  Default (none): the IR sub-layer merged inside GEMM1 (header comment).
+ * SR_FUSE_IR: fold the IR sub-layer into GEMM2 instead (one warp of each GEMM2 CTA reduces the
+ * item's m', d' before its GS warps need them; r' is formed on the fly and never written).
+ * SURVEY.md NEXT-2. */
 #define SR_FUSE_IR 16
 /* Variant bit: SD, the softmax decomposition WITHOUT fusion ("SD" of Fig. 8):
  * plain GEMM1 (writes S) -> standalone LS (S -> X', m', d') -> IR -> standalone GS (X', r' -> Y)
@@ -119,14 +123,10 @@ typedef struct {
  * between the unfused baseline and SDF.  Workspace: sr_workspace_bytes with
  * fused = 2. */
 #define SR_DECOMPOSE 32
-/* Variant bit (recomposed 16-bit path): the IR sub-layer runs inside GEMM1.  Each GEMM1 CTA owns
- * whole query rows (every key tile of its row-blocks), so one warp of it merges the per-tile
- * (m', d') of each row as the epilogue produces them (m = max m', d = sum
- * e^{m'-m} d') and writes the row's (m, 1/d); GEMM2 applies the normalisation 1/d * e^{m'-m} to
- * each X' tile in its prologue (L151).  Two kernels, no IR launch, no r' or d' round trip.
- * Exclusive with SR_FUSE_IR and SR_DECOMPOSE; with SR_RUN_* stage bits SR_RUN_REDUCE is a no-op.
- * Workspace: the same sr_workspace_bytes(fused = 1) (its rowstat region). */
-#define SR_IR_IN_GEMM1 64
+/* Variant bit: the paper's three-kernel layout: GEMM1 + LS writes m', d';
+ * a standalone IR kernel reduces them per row and writes r'_k = e^{m'_k - m} / d; GS + GEMM2
+ * streams r' beside X'.  The only mode that writes d' and r' to the workspace. */
+#define SR_IR_KERNEL 64
 
 /* Entry points (north star).  Returns SR_OK after enqueueing the kernels on ex->stream. */
 sr_status sr_mha_dense(const void* q, const void* k, const void* v, void* out, int B, int H, int S,
@@ -162,7 +162,7 @@ typedef enum { SR_E_DENSE = 0, SR_E_BLOCKSPARSE = 1, SR_E_WINDOW = 2 } sr_entry;
  *            SWIZZLE_128B K-major layout [T/64][128 rows][64 cols] with the 16-byte chunk index
  *            XOR (row & 7); fp32 tiles are plain row-major [128][T].
  *   mprime, dprime, rprime   fp32 [slot id][128 rows]  (m' in natural-log units)
- *   rowstat  fp32 [2][B*H*S]: per query row m (natural-log units), then 1/d (SR_IR_IN_GEMM1)
+ *   rowstat  fp32 [2][B*H*S]: per query row m (natural-log units), then 1/d (default mode)
  */
 typedef struct {
     int32_t tile_n;           /* T actually used */
@@ -170,7 +170,7 @@ typedef struct {
     int64_t n_slots;          /* B*H*slots_per_head */
     int32_t xprime_elt_bytes; /* 2 (16-bit paths) or 4 (fp32 path) */
     size_t off_xprime, off_mprime, off_dprime, off_rprime, off_p;  /* off_p: unfused P region */
-    size_t off_rowstat;       /* recomposed: per-row (m, 1/d) of the SR_IR_IN_GEMM1 variant */
+    size_t off_rowstat;       /* recomposed: per-row (m, 1/d) of the default (IR in GEMM1) mode */
     size_t total_bytes;
 } sr_ws_info;
 

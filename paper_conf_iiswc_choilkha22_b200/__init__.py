@@ -202,15 +202,16 @@ _FN = {(SR_E_DENSE, True): "sr_mha_dense", (SR_E_BLOCKSPARSE, True): "sr_mha_blo
 SR_RUN_GEMM1, SR_RUN_REDUCE, SR_RUN_GEMM2 = 1, 2, 4
 SR_FUSE_IR = 16
 SR_DECOMPOSE = 32
-SR_IR_IN_GEMM1 = 64
+SR_IR_KERNEL = 64
 
 
 def call(mask: _Mask, q, k, v, *, scale=None, causal=False, out_dtype=None, tile_n=0, fused=True,
-         out=None, workspace=None, stream=None, stages=0, fuse_ir=False, sd=False, ir_in_gemm1=False):
+         out=None, workspace=None, stream=None, stages=0, fuse_ir=False, sd=False, ir_kernel=False):
     """Run one attention layer through the C ABI.  q, k, v: CUDA tensors [B, H, S, D].
-    fuse_ir=True selects the SR_FUSE_IR variant (IR folded into GEMM2, SURVEY NEXT-2);
-    ir_in_gemm1=True the SR_IR_IN_GEMM1 variant (IR merged inside GEMM1, GEMM2 normalises);
-    sd=True the SR_DECOMPOSE variant (decomposition without fusion, the paper's SD, NEXT-1)."""
+    Default (16-bit): GEMM1 + LS with the IR merged inside it -> GS + GEMM2 (2 kernels).
+    ir_kernel=True selects SR_IR_KERNEL (the paper's layout: a standalone IR kernel writing r');
+    fuse_ir=True SR_FUSE_IR (IR folded into GEMM2, SURVEY NEXT-2);
+    sd=True SR_DECOMPOSE (decomposition without fusion, the paper's SD, NEXT-1)."""
     torch = _torch()
     if not (q.is_cuda and k.is_cuda and v.is_cuda):
         raise ValueError("q, k, v must be CUDA tensors")
@@ -235,7 +236,7 @@ def call(mask: _Mask, q, k, v, *, scale=None, causal=False, out_dtype=None, tile
     st = torch.cuda.current_stream(q.device).cuda_stream if stream is None else stream
     ex = Exec(in_dt, dtype_code(out_dtype), ws.data_ptr(), ws.numel() * ws.element_size(), st, int(tile_n),
               int(stages) | (SR_FUSE_IR if fuse_ir else 0) | (SR_DECOMPOSE if sd else 0) |
-              (SR_IR_IN_GEMM1 if ir_in_gemm1 else 0))
+              (SR_IR_KERNEL if ir_kernel else 0))
     fn = getattr(lib(), _FN[(mask.entry, bool(fused))])
     _check(fn(q.data_ptr(), k.data_ptr(), v.data_ptr(), out.data_ptr(), B, H, S, D, C.c_float(scale), mask.ptr,
               int(causal), C.byref(ex)))

@@ -483,14 +483,14 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
     if (!ex) return fail(SR_ERR_INVALID, "exec descriptor is NULL");
     if (!q || !k || !v || !out) return fail(SR_ERR_INVALID, "q, k, v and out must be non-NULL");
     if (!std::isfinite(scale) || !(scale > 0.f)) return fail(SR_ERR_INVALID, "scale must be finite and > 0");
-    const int variant_bits = SR_FUSE_IR | SR_DECOMPOSE | SR_IR_IN_GEMM1;
+    const int variant_bits = SR_FUSE_IR | SR_DECOMPOSE | SR_IR_KERNEL;
     if (ex->flags & ~(SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2 | variant_bits))
         return fail(SR_ERR_INVALID, "unknown flags 0x%x", ex->flags);
     if ((ex->flags & variant_bits) && (!fused || ex->in_dtype == SR_F32))
-        return fail(SR_ERR_UNSUPPORTED, "SR_FUSE_IR / SR_DECOMPOSE / SR_IR_IN_GEMM1 apply to the recomposed 16-bit path only");
+        return fail(SR_ERR_UNSUPPORTED, "SR_FUSE_IR / SR_DECOMPOSE / SR_IR_KERNEL apply to the recomposed 16-bit path only");
     {
         const int v = ex->flags & variant_bits;
-        if (v & (v - 1)) return fail(SR_ERR_INVALID, "SR_FUSE_IR, SR_DECOMPOSE and SR_IR_IN_GEMM1 are exclusive");
+        if (v & (v - 1)) return fail(SR_ERR_INVALID, "SR_FUSE_IR, SR_DECOMPOSE and SR_IR_KERNEL are exclusive");
     }
     if (fused && (ex->flags & SR_DECOMPOSE)) fused = 2;  // SD: workspace mode 2
     Request r;
@@ -532,7 +532,7 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
     p.sc = cs->dev;
     const int stage_bits = ex->flags & (SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2);
     p.stages = stage_bits ? stage_bits : (SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2);
-    p.ir_mode = (ex->flags & SR_FUSE_IR) ? IR_IN_GEMM2 : ((ex->flags & SR_IR_IN_GEMM1) ? IR_IN_GEMM1 : IR_KERNEL);
+    p.ir_mode = (ex->flags & SR_FUSE_IR) ? IR_IN_GEMM2 : ((ex->flags & SR_IR_KERNEL) ? IR_KERNEL : IR_IN_GEMM1);
     {   // GEMM1 pair schedule: SR_G1_PAIR=0/1 overrides the default (experiments)
         static const int env_pair = [] { const char* e = getenv("SR_G1_PAIR"); return e ? atoi(e) : -1; }();
         // default: pairs when K tiles are as large as the X' tiles they produce (D = 128) and there

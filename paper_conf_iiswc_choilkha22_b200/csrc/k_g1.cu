@@ -35,7 +35,23 @@ namespace sr {
 
 using namespace ptx;
 
+#ifdef SR_DIAG_WAITS
+__device__ unsigned long long g_diag_g1[20 * (kDW + 1)];
+}  // namespace sr
+extern "C" int sr_diag_read_g1(unsigned long long* out)  // copies [20 warps][kDW + 1] and resets (diagnostic build)
+{
+    if (cudaMemcpyFromSymbol(out, sr::g_diag_g1, sizeof(sr::g_diag_g1)) != cudaSuccess) return 1;
+    static unsigned long long zero[20 * (sr::kDW + 1)];
+    return cudaMemcpyToSymbol(sr::g_diag_g1, zero, sizeof(zero)) != cudaSuccess;
+}
+namespace sr {
+#endif
+
 constexpr int kMW = 128;  // macro tile width (MMA N of GEMM1)
+#ifndef SR_G1_QPREFETCH
+#define SR_G1_QPREFETCH 0
+#endif
+constexpr bool kQPrefetch = SR_G1_QPREFETCH;  // L2 prefetch of the next item's Q (measured: C3 slower, off)
 // Of every 8 element pairs of the LS exponentials, this many are computed by ex2_poly2 on the FMA
 // pipe and the rest by MUFU.EX2 (16 / clock / SM): balances the two pipes in the epilogue.
 #ifndef SR_G1_POLY_PAIRS
@@ -88,7 +104,7 @@ struct G1 {
     static constexpr int THREADS = 128 + EPI_WG * 128;
 };
 
-// IRT: the IR sub-layer runs in this kernel (SR_IR_IN_GEMM1): every CTA owns whole rows (all key
+// IRT: the IR sub-layer runs in this kernel (the default mode): every CTA owns whole rows (all key
 // tiles of its row-blocks), so warp 3 merges the epilogue's per-tile (m', d') of each row as they
 // are produced and, at the end of the row-block, writes the row's (m, 1/d) -- see the IR warp below.
 template <int D, int T, bool LS, bool PAIR, bool IRT>
@@ -114,13 +130,14 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
     uint32_t* tmem_ptr = (uint32_t*)(smem + C::OFF_TPTR);
 
     const int warp = warp_uniform(), lane = threadIdx.x % 32;
+    DW_DECL
     if (threadIdx.x == 0) {
         for (int i = 0; i < C::NQ; ++i) { mbar_init(&q_full[i], 1); mbar_init(&q_empty[i], 1); }
         for (int i = 0; i < C::NK; ++i) { mbar_init(&k_full[i], 1); mbar_init(&k_empty[i], 1); }
         // acc_full: header arrive (MMA thread) + tcgen05.commit; acc_empty: one arrive per epilogue
         // warp that reads the accumulator (the warpgroup pair in SPLIT, one warpgroup in FULL)
         for (int i = 0; i < C::NACC; ++i) { mbar_init(&acc_full[i], 2); mbar_init(&acc_empty[i], SPLIT ? 8 : 4); }
-        for (int i = 0; i < C::NACC; ++i) { mbar_init(&st_full[i], SPLIT ? 8 : 4); mbar_init(&st_empty[i], 1); }
+        for (int i = 0; i < C::NACC; ++i) { mbar_init(&st_full[i], SPLIT ? 8 : 4); mbar_init(&st_empty[i], 2); }
         fence_mbar_init();
     }
     if (warp == 0 && lane == 0) { prefetch_tmap(&tmQ); prefetch_tmap(&tmK); }
@@ -158,13 +175,20 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
                 if (e0 == e1) continue;
                 const int nrb = 2 * j + 1 < p.sc.n_rb ? 2 : 1;
                 const int row0 = g * p.S + 2 * j * kRowBlock;
-                mbar_wait(&q_empty[qi], qph ^ 1);
+                DW_WAIT(&q_empty[qi], qph ^ 1, 0);
                 if (elect_one()) {
                     mbar_arrive_expect_tx(&q_full[qi], nrb * C::QB);
                     for (int r = 0; r < nrb; ++r)
                         for (int h = 0; h < D / 64; ++h)
                             tma_load_2d(smem + C::OFF_Q + qi * C::QS + r * C::QB + h * (kRowBlock * 128), &tmQ, h * 64,
                                         row0 + r * kRowBlock, &q_full[qi]);
+                    if (kQPrefetch && it + 1 < it_end) {  // the next item's Q into L2 (Q is single-buffered)
+                        const int g2 = nd.x / p.sc.n_pair, j2 = nd.x % p.sc.n_pair;
+                        const int nrb2 = 2 * j2 + 1 < p.sc.n_rb ? 2 : 1;
+                        for (int r = 0; r < nrb2; ++r)
+                            for (int h = 0; h < D / 64; ++h)
+                                tma_prefetch_2d(&tmQ, h * 64, g2 * p.S + (2 * j2 + r) * kRowBlock);
+                    }
                 }
                 __syncwarp();
                 if (++qi == C::NQ) { qi = 0; qph ^= 1; }
@@ -179,7 +203,7 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
                         w[s2] = wn[s2];
                         wn[s2] = e + NSUB + s2 < e1 ? __ldg(&p.sc.pent[e + NSUB + s2].x) : 0;
                     }
-                    mbar_wait(&k_empty[ks], kph ^ 1);
+                    DW_WAIT(&k_empty[ks], kph ^ 1, 1);
                     if (elect_one()) {
                         mbar_arrive_expect_tx(&k_full[ks], nsub * T * D * 2);
                         for (int s2 = 0; s2 < nsub; ++s2)
@@ -207,7 +231,7 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
                 const int nrb = 2 * j + 1 < p.sc.n_rb ? 2 : 1;
                 const int kvl = p.sc.kv_len ? __ldg(p.sc.kv_len + g / p.H) : p.S;
                 const int64_t slot0 = (int64_t)g * p.sc.slots_per_head - d.w;
-                mbar_wait(&q_full[qi], qph);
+                DW_WAIT(&q_full[qi], qph, 0);
                 tc_fence_after();
                 const uint32_t q_addr = smem_u32(smem + C::OFF_Q + qi * C::QS);
                 int4 wn[NSUB];
@@ -220,7 +244,7 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
                         w[s2] = wn[s2];
                         wn[s2] = e + NSUB + s2 < e1 ? __ldg(p.sc.pent + e + NSUB + s2) : make_int4(0, -1, -1, 0);
                     }
-                    mbar_wait(&k_full[ks], kph);
+                    DW_WAIT(&k_full[ks], kph, 1);
                     tc_fence_after();
                     const uint32_t k_addr = smem_u32(smem + C::OFF_K + ks * C::KB);
                     for (int r = 0; r < nrb; ++r) {
@@ -236,7 +260,7 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
                         }
                         if (ws[0] == -1 && ws[1] == -1) continue;  // nothing of this row-block here
                         const int buf = n % C::NACC;
-                        mbar_wait(&acc_empty[buf], ((n / C::NACC) & 1) ^ 1);
+                        DW_WAIT(&acc_empty[buf], ((n / C::NACC) & 1) ^ 1, 2);
                         // sub-tile s's slot = slot + (s ? dslot : 0)
                         const int64_t slot = ws[0] != -1 ? sl[0] : sl[1];
                         const int dslot = (ws[0] != -1 && ws[1] != -1) ? (int)(sl[1] - sl[0]) : 0;
@@ -271,7 +295,7 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
             }
             for (int e = 0; e < 2; ++e, ++n) {  // one END header for each epilogue warpgroup (pair)
                 const int buf = n % C::NACC;
-                mbar_wait(&acc_empty[buf], ((n / C::NACC) & 1) ^ 1);
+                DW_WAIT(&acc_empty[buf], ((n / C::NACC) & 1) ^ 1, 2);
                 if (elect_one()) {
                     hdr[buf].flags = HDR_END;
                     mbar_arrive(&acc_full[buf]);
@@ -288,7 +312,7 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
                 const ItemInfo I = iw.next();
                 if (I.t0 == I.t1) continue;
                 const int row0 = I.g * p.S + I.rb * kRowBlock;
-                mbar_wait(&q_empty[qi], qph ^ 1);
+                DW_WAIT(&q_empty[qi], qph ^ 1, 0);
                 if (elect_one()) {
                     mbar_arrive_expect_tx(&q_full[qi], C::QB);
                     for (int h = 0; h < D / 64; ++h)
@@ -307,7 +331,7 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
                         w[s] = wn[s];
                         wn[s] = t + NSUB + s < I.t1 ? __ldg(p.sc.tinfo + t + NSUB + s) : 0;
                     }
-                    mbar_wait(&k_empty[ks], kph ^ 1);
+                    DW_WAIT(&k_empty[ks], kph ^ 1, 1);
                     if (elect_one()) {
 #ifdef SR_DIAG_NOKLOAD
                         mbar_arrive(&k_full[ks]);
@@ -334,7 +358,7 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
                 const ItemInfo I = iw.next();
                 if (I.t0 == I.t1) continue;
                 const int kvl = p.sc.kv_len ? __ldg(p.sc.kv_len + I.g / p.H) : p.S;
-                mbar_wait(&q_full[qi], qph);
+                DW_WAIT(&q_full[qi], qph, 0);
                 tc_fence_after();
                 const uint32_t q_addr = smem_u32(smem + C::OFF_Q + qi * C::QB);
                 int wn0 = __ldg(p.sc.tinfo + I.t0), wn1 = (NSUB > 1 && I.t0 + 1 < I.t1) ? __ldg(p.sc.tinfo + I.t0 + 1) : -1;
@@ -343,7 +367,7 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
                     if (t + NSUB < I.t1) wn0 = __ldg(p.sc.tinfo + t + NSUB);  // prefetch the next macro tile
                     wn1 = (NSUB > 1 && t + NSUB + 1 < I.t1) ? __ldg(p.sc.tinfo + t + NSUB + 1) : -1;
                     const int ab = n % C::NACC;
-                    mbar_wait(&acc_empty[ab], ((n / C::NACC) & 1) ^ 1);
+                    DW_WAIT(&acc_empty[ab], ((n / C::NACC) & 1) ^ 1, 2);
                     const int64_t slot = I.slot0 + t;
                     if (elect_one()) {
                         hdr[ab] = G1Hdr{(int32_t)(slot & 0xffffffff), (int32_t)(slot >> 32), I.rb * kRowBlock, kvl, w0,
@@ -351,7 +375,7 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
                         mbar_arrive(&acc_full[ab]);  // header published (arrival 1 of 2)
                     }
                     __syncwarp();
-                    mbar_wait(&k_full[ks], kph);
+                    DW_WAIT(&k_full[ks], kph, 1);
                     tc_fence_after();
                     const uint32_t k_addr = smem_u32(smem + C::OFF_K + ks * C::KB);
                     const uint32_t d_tmem = tmem_base + ab * kMW;
@@ -375,7 +399,7 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
             }
             for (int e = 0; e < 2; ++e, ++n) {  // one END header for each epilogue warpgroup pair
                 const int ab = n % C::NACC;
-                mbar_wait(&acc_empty[ab], ((n / C::NACC) & 1) ^ 1);
+                DW_WAIT(&acc_empty[ab], ((n / C::NACC) & 1) ^ 1, 2);
                 if (elect_one()) {
                     hdr[ab].flags = HDR_END;
                     mbar_arrive(&acc_full[ab]);
@@ -383,40 +407,51 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
                 }
                 __syncwarp();
             }
-        } else if (IRT && warp == 3) {
-            // -------------------------------------------------------------- IR warp (SR_IR_IN_GEMM1)
+        } else if (IRT && (warp == 2 || warp == 3)) {
+            // -------------------------------------------------------------- IR warps (default mode)
             // The IR sub-layer of every row this CTA owns: per accumulator (in
             // the MMA warp's order) merge the staged (m'_k, d'_k) of each row into a running
             //   m = max_k m'_k,   d = sum_k e^{m'_k - m} d'_k
             // and at the end of a row-block write m (natural-log units) and 1/d; GEMM2 forms
-            // r'_k = e^{m'_k - m} / d in its prologue.  Lane l owns rows l + 32 j of a row-block.
+            // r'_k = e^{m'_k - m} / d in its prologue.  Warp 2 owns rows 0-63 of a row-block, warp 3
+            // rows 64-127 (lane l: rows l, l + 32 of its half).  Both arrive on st_empty.
             const float sl2 = p.scale_log2;
+            const int rbase = (warp - 2) * 64 + lane;
             int n = 0;
-            auto merge = [&](float (&m)[4], float (&d)[4]) {
+            auto merge = [&](float (&m)[2], float (&d)[2]) {
                 const int buf = n % C::NACC;
-                mbar_wait(&st_full[buf], (uint32_t)(n / C::NACC) & 1);
-                const float* sb = stats + buf * (4 * kRowBlock);
+                DW_WAIT(&st_full[buf], (uint32_t)(n / C::NACC) & 1, 0);
+                const float* sb = stats + buf * (4 * kRowBlock) + rbase;
+                float mk[2][NSUB], dk[2][NSUB];
 #pragma unroll
-                for (int s = 0; s < NSUB; ++s)
+                for (int j = 0; j < 2; ++j)
 #pragma unroll
-                    for (int j = 0; j < 4; ++j) {
-                        const float mk = sb[(2 * s) * kRowBlock + lane + 32 * j];  // raw score units
-                        const float dk = sb[(2 * s + 1) * kRowBlock + lane + 32 * j];
-                        const float mn = fmaxf(m[j], mk);
-                        if (mn != -INFINITY) {  // ex2(-inf) = 0 covers an empty side
-                            d[j] = fmaf(d[j], ex2((m[j] - mn) * sl2), dk * ex2((mk - mn) * sl2));
-                            m[j] = mn;
-                        }
+                    for (int s = 0; s < NSUB; ++s) {
+                        mk[j][s] = sb[(2 * s) * kRowBlock + 32 * j];  // raw score units, -inf if invalid
+                        dk[j][s] = sb[(2 * s + 1) * kRowBlock + 32 * j];
                     }
                 __syncwarp();  // every lane's reads of the stage are done
                 if (lane == 0) mbar_arrive(&st_empty[buf]);
+#pragma unroll
+                for (int j = 0; j < 2; ++j) {
+                    float mn = m[j];
+#pragma unroll
+                    for (int s = 0; s < NSUB; ++s) mn = fmaxf(mn, mk[j][s]);
+                    if (mn != -INFINITY) {  // ex2(-inf) = 0 covers empty sides
+                        float acc = d[j] * ex2((m[j] - mn) * sl2);
+#pragma unroll
+                        for (int s = 0; s < NSUB; ++s) acc = fmaf(dk[j][s], ex2((mk[j][s] - mn) * sl2), acc);
+                        d[j] = acc;
+                        m[j] = mn;
+                    }
+                }
                 ++n;
             };
-            auto flush = [&](int g, int rb, const float (&m)[4], const float (&d)[4]) {
-                const int64_t row = (int64_t)g * p.S + rb * kRowBlock + lane;
+            auto flush = [&](int g, int rb, const float (&m)[2], const float (&d)[2]) {
+                const int64_t row = (int64_t)g * p.S + rb * kRowBlock + rbase;
                 const int64_t nrow = (int64_t)p.B * p.H * p.S;
 #pragma unroll
-                for (int j = 0; j < 4; ++j) {
+                for (int j = 0; j < 2; ++j) {
                     p.rowstat[row + 32 * j] = m[j] * p.scale;  // -inf stays -inf
                     p.rowstat[nrow + row + 32 * j] = d[j] > 0.f ? 1.f / d[j] : 0.f;
                 }
@@ -429,9 +464,9 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
                     const int g = dd.x / p.sc.n_pair, j = dd.x % p.sc.n_pair, e0 = dd.y, e1 = dd.z;
                     if (e0 == e1) continue;
                     const int nrb = 2 * j + 1 < p.sc.n_rb ? 2 : 1;
-                    float m0[4], d0[4], m1[4], d1[4];
+                    float m0[2], d0[2], m1[2], d1[2];
 #pragma unroll
-                    for (int u = 0; u < 4; ++u) { m0[u] = m1[u] = -INFINITY; d0[u] = d1[u] = 0.f; }
+                    for (int u = 0; u < 2; ++u) { m0[u] = m1[u] = -INFINITY; d0[u] = d1[u] = 0.f; }
                     for (int e = e0; e < e1; e += NSUB) {
                         int hb = 0;  // union of the sub-tiles' half bits: bits 0-1 row-block 0, 2-3 row-block 1
 #pragma unroll
@@ -447,9 +482,9 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
                 for (ItemWalk iw(p, it_begin, it_end); iw.more();) {
                     const ItemInfo I = iw.next();
                     if (I.t0 == I.t1) continue;
-                    float m[4], d[4];
+                    float m[2], d[2];
 #pragma unroll
-                    for (int u = 0; u < 4; ++u) { m[u] = -INFINITY; d[u] = 0.f; }
+                    for (int u = 0; u < 2; ++u) { m[u] = -INFINITY; d[u] = 0.f; }
                     for (int t = I.t0; t < I.t1; t += NSUB) merge(m, d);
                     flush(I.g, I.rb, m, d);
                 }
@@ -469,7 +504,7 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
         int k = 0;                            // macro tiles processed by this warpgroup
         for (int n = pj;; n += 2, ++k) {
             const int buf = n % C::NACC;
-            mbar_wait(&acc_full[buf], (uint32_t)(n / C::NACC) & 1);
+            DW_WAIT(&acc_full[buf], (uint32_t)(n / C::NACC) & 1, 0);
             tc_fence_after();
             const G1Hdr H = hdr[buf];
             if (H.flags & HDR_END) break;
@@ -579,7 +614,7 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
                 bulk_commit();
             }
             if constexpr (IRT) {  // (m', d') of this row and sub-tile to the IR warp (-inf, 0 if invalid)
-                mbar_wait(&st_empty[buf], ((uint32_t)(n / C::NACC) & 1) ^ 1);
+                DW_WAIT(&st_empty[buf], ((uint32_t)(n / C::NACC) & 1) ^ 1, 2);
                 if (NSUB == 2 || h == 0) {
                     float* sb = stats + buf * (4 * kRowBlock) + (NSUB == 2 ? 2 * h : 0) * kRowBlock;
                     sb[r] = mx;
@@ -606,7 +641,7 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
         int k = 0;                          // macro tiles processed by this warpgroup
         for (int n = e;; n += 2, ++k) {
             const int buf = n % C::NACC;
-            mbar_wait(&acc_full[buf], (uint32_t)(n / C::NACC) & 1);
+            DW_WAIT(&acc_full[buf], (uint32_t)(n / C::NACC) & 1, 0);
             tc_fence_after();
             const G1Hdr H = hdr[buf];
             if (H.flags & HDR_END) break;
@@ -737,7 +772,7 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
                 bulk_commit();
             }
             if constexpr (IRT) {  // (m', d') of this row per sub-tile to the IR warp (-inf, 0 if invalid)
-                mbar_wait(&st_empty[buf], ((uint32_t)(n / C::NACC) & 1) ^ 1);
+                DW_WAIT(&st_empty[buf], ((uint32_t)(n / C::NACC) & 1) ^ 1, 2);
                 float* sb = stats + buf * (4 * kRowBlock);
 #pragma unroll
                 for (int s = 0; s < NSUB; ++s) {
@@ -758,6 +793,7 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
         }
         if (lane == 0) bulk_wait0();
     }
+    DW_FLUSH(g_diag_g1);
     tc_fence_before();
     __syncthreads();
     if (warp == 2) {

@@ -30,6 +30,18 @@ namespace sr {
 
 using namespace ptx;
 
+#ifdef SR_DIAG_WAITS
+__device__ unsigned long long g_diag_g2[20 * (kDW + 1)];
+}  // namespace sr
+extern "C" int sr_diag_read_g2(unsigned long long* out)  // copies [20 warps][kDW + 1] and resets (diagnostic build)
+{
+    if (cudaMemcpyFromSymbol(out, sr::g_diag_g2, sizeof(sr::g_diag_g2)) != cudaSuccess) return 1;
+    static unsigned long long zero[20 * (sr::kDW + 1)];
+    return cudaMemcpyToSymbol(sr::g_diag_g2, zero, sizeof(zero)) != cudaSuccess;
+}
+namespace sr {
+#endif
+
 constexpr int kMW2 = 128;  // macro tile width (keys per MMA step)
 
 enum : int { SH_TILE = 1, SH_END = 2, SH_EMPTY = 4, SH_FIRST = 8, SH_LAST = 16 };
@@ -46,9 +58,18 @@ struct G2 {
     static constexpr int XSB = XB + RB;              // X' stage
     static constexpr int VB = kMW2 * D * 2;          // V stage (macro tile)
     // split the smem budget: V stages from L2 need less depth than the HBM-bound X' stream
-    static constexpr int NV = (VB >= 32768) ? 2 : 3;
+#ifndef SR_G2_NV64
+#define SR_G2_NV64 3
+#endif
+#ifndef SR_G2_NV128
+#define SR_G2_NV128 2
+#endif
+#ifndef SR_G2_NX
+#define SR_G2_NX 8
+#endif
+    static constexpr int NV = D == 64 ? SR_G2_NV64 : SR_G2_NV128;
     static constexpr int NX_ = (kSmemMax - 3072 - NV * VB) / XSB;
-    static constexpr int NX = NX_ > 8 ? 8 : NX_;
+    static constexpr int NX = NX_ > SR_G2_NX ? SR_G2_NX : NX_;
     static_assert(NX >= 2, "smem budget");
     static constexpr int NO = 2;                             // O accumulators (D cols each)
     static constexpr int NA_ = (512 - NO * D) / (kMW2 / 2);  // A operand buffers (MW/2 cols each)
@@ -71,7 +92,7 @@ struct G2 {
 // FI (fused IR): the IR sub-layer runs inside this kernel -- warp 2 reduces each
 // item's m', d' into per-row (m, 1/d) ahead of the GS warps, the X' stages carry m' instead of r',
 // and GS forms r' = e^{m' - m} / d on the fly.  No IR launch, no r' round trip through HBM.
-// RS (SR_IR_IN_GEMM1): as FI, but GEMM1 already merged the rows, so warp 2 only loads each item's
+// RS (default mode, IR in GEMM1): as FI, but GEMM1 already merged the rows, so warp 2 only loads each item's
 // per-row (m, 1/d) -- GEMM2 applies the normalisation 1/d * e^{m' - m} in its prologue.
 template <int D, int T, bool GS, bool FI, bool RS>
 __global__ void __launch_bounds__(512, 1) tc_gemm2(const __grid_constant__ CUtensorMap tmV, const Params p)
@@ -99,6 +120,7 @@ __global__ void __launch_bounds__(512, 1) tc_gemm2(const __grid_constant__ CUten
     auto vstage = [&](int s) { return smem + C::OFF_V + s * C::VB; };
 
     const int warp = warp_uniform(), lane = threadIdx.x % 32;
+    DW_DECL
     if (threadIdx.x == 0) {
         for (int i = 0; i < C::NX; ++i) { mbar_init(&x_full[i], 1); mbar_init(&x_empty[i], C::NGS); }
         for (int i = 0; i < C::NV; ++i) { mbar_init(&v_full[i], 1); mbar_init(&v_empty[i], 1); }
@@ -142,7 +164,7 @@ __global__ void __launch_bounds__(512, 1) tc_gemm2(const __grid_constant__ CUten
 #ifndef SR_DIAG2_NOX
                     for (int u = 0; u < nsub; ++u) bytes += (hv[u] == 3 ? 2 : 1) * (T / 64) * (kHalf * 128);
 #endif
-                    mbar_wait(&x_empty[s], sph ^ 1);
+                    DW_WAIT(&x_empty[s], sph ^ 1, 0);
                     uint8_t* st = xstage(s);
                     if (elect_one()) {
                     *xhdr(s) = G2Hdr{SH_TILE | (t == I.t0 ? SH_FIRST : 0) | (t + NSUB >= I.t1 ? SH_LAST : 0), hv[0],
@@ -173,7 +195,7 @@ __global__ void __launch_bounds__(512, 1) tc_gemm2(const __grid_constant__ CUten
                     if (++s == C::NX) { s = 0; sph ^= 1; }
                 }
             }
-            mbar_wait(&x_empty[s], sph ^ 1);
+            DW_WAIT(&x_empty[s], sph ^ 1, 0);
             if (elect_one()) {
                 xhdr(s)->flags = SH_END;
                 mbar_arrive(&x_full[s]);
@@ -197,7 +219,7 @@ __global__ void __launch_bounds__(512, 1) tc_gemm2(const __grid_constant__ CUten
                     mv[j] = __ldcg(p.rowstat + row + 32 * j);
                     iv[j] = __ldcg(p.rowstat + nrow + row + 32 * j);
                 }
-                mbar_wait(&st_empty[si], sph ^ 1);
+                DW_WAIT(&st_empty[si], sph ^ 1, 0);
                 float* ms = stats + si * 2 * kRowBlock;
 #pragma unroll
                 for (int j = 0; j < 4; ++j) {
@@ -217,7 +239,7 @@ __global__ void __launch_bounds__(512, 1) tc_gemm2(const __grid_constant__ CUten
             for (ItemWalk iw(p, it_begin, it_end); iw.more();) {
                 const ItemInfo I = iw.next();
                 if (I.t0 == I.t1) continue;
-                mbar_wait(&st_empty[si], sph ^ 1);
+                DW_WAIT(&st_empty[si], sph ^ 1, 0);
                 float* ms = stats + si * 2 * kRowBlock;
                 const float* mp = p.mprime + I.slot0 * kRowBlock + lane;
                 const float* dp = p.dprime + I.slot0 * kRowBlock + lane;
@@ -279,7 +301,7 @@ __global__ void __launch_bounds__(512, 1) tc_gemm2(const __grid_constant__ CUten
                     const int nsub = min(NSUB, I.t1 - t);
                     int kt[2] = {tinfo_kt(wn[0]), NSUB > 1 ? tinfo_kt(wn[1]) : 0};
                     for (int u = 0; u < NSUB; ++u) wn[u] = t + NSUB + u < I.t1 ? __ldg(p.sc.tinfo + t + NSUB + u) : 0;
-                    mbar_wait(&v_empty[s], sph ^ 1);
+                    DW_WAIT(&v_empty[s], sph ^ 1, 0);
                     if (elect_one()) {
 #ifdef SR_DIAG2_NOV
                         mbar_arrive(&v_full[s]);
@@ -305,7 +327,7 @@ __global__ void __launch_bounds__(512, 1) tc_gemm2(const __grid_constant__ CUten
             int s = 0, a = 0, o = 0;
             uint32_t sph = 0, aph = 0, oph = 0;
             auto post = [&](int flags, int64_t orow, bool second) {  // O header to the epilogue, arrival 1 of 2
-                mbar_wait(&o_empty[o], oph ^ 1);
+                DW_WAIT(&o_empty[o], oph ^ 1, 2);
                 if (elect_one()) {
                     ohdr[o] = G2Hdr{flags, 0, 0, 0, (int32_t)(orow & 0xffffffff), (int32_t)(orow >> 32), 0, 0};
                     mbar_arrive(&o_full[o]);
@@ -331,8 +353,8 @@ __global__ void __launch_bounds__(512, 1) tc_gemm2(const __grid_constant__ CUten
                 const uint32_t d_tmem = tmem_o + o * D;
                 for (int t = I.t0; t < I.t1; t += NSUB) {
                     const int nk = min(NSUB, I.t1 - t) * (T / 16);  // K steps of 16 keys
-                    mbar_wait(&v_full[s], sph);
-                    mbar_wait(&a_full[a], aph);
+                    DW_WAIT(&v_full[s], sph, 0);
+                    DW_WAIT(&a_full[a], aph, 1);
                     tc_fence_after();
                     const uint32_t v_addr = smem_u32(vstage(s));
                     const uint32_t a_tm = tmem_a + a * (kMW2 / 2);
@@ -367,11 +389,11 @@ __global__ void __launch_bounds__(512, 1) tc_gemm2(const __grid_constant__ CUten
         uint32_t sph = 0, aph = 0, siph = 0;
         float m_row = 0.f, invd_row = 0.f;  // fused IR: this row's (m, 1/d) for the current item
         for (;;) {
-            mbar_wait(&x_full[s], sph);
+            DW_WAIT(&x_full[s], sph, 0);
             const G2Hdr h = *xhdr(s);
             if (h.flags & SH_END) break;
             if (FI && (h.flags & SH_FIRST)) {  // a new item: its row statistics from the IR warp
-                mbar_wait(&st_full[si], siph);
+                DW_WAIT(&st_full[si], siph, 2);
                 m_row = stats[si * 2 * kRowBlock + r];
                 invd_row = stats[si * 2 * kRowBlock + kRowBlock + r];
                 __syncwarp();
@@ -402,7 +424,7 @@ __global__ void __launch_bounds__(512, 1) tc_gemm2(const __grid_constant__ CUten
 #pragma unroll
             for (int q = 0; q < kMW2 / 16; ++q)
                 if (rr[((ch * 8 + q) * 8) / T] != 0.f) xv[q] = lds128(xs_s + tile_chunk_off(r, ch * 8 + q));
-            mbar_wait(&a_empty[a], aph ^ 1);
+            DW_WAIT(&a_empty[a], aph ^ 1, 1);
             tc_fence_after();
             const uint32_t a_tm = tmem_a + lane_off + a * (kMW2 / 2);
 #pragma unroll
@@ -455,7 +477,7 @@ __global__ void __launch_bounds__(512, 1) tc_gemm2(const __grid_constant__ CUten
         int o = 0;
         uint32_t oph = 0;
         for (;;) {
-            mbar_wait(&o_full[o], oph);
+            DW_WAIT(&o_full[o], oph, 0);
             tc_fence_after();
             const G2Hdr h = ohdr[o];
             if (h.flags & SH_END) break;
@@ -500,6 +522,7 @@ __global__ void __launch_bounds__(512, 1) tc_gemm2(const __grid_constant__ CUten
             if (++o == C::NO) { o = 0; oph ^= 1; }
         }
     }
+    DW_FLUSH(g_diag_g2);
     tc_fence_before();
     __syncthreads();
     if (warp == 2) {

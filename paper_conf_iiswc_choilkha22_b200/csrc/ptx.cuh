@@ -147,6 +147,13 @@ __device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* m, int
         "l"(reinterpret_cast<uint64_t>(m)), "r"(c0), "r"(c1), "r"(smem_u32(bar))
         : "memory");
 }
+// L2 prefetch of a 2-D TMA box (no shared memory, no barrier): warms the next item's tile
+__device__ __forceinline__ void tma_prefetch_2d(const CUtensorMap* m, int c0, int c1)
+{
+    asm volatile("cp.async.bulk.prefetch.tensor.2d.L2.global.tile [%0, {%1, %2}];" ::"l"(reinterpret_cast<uint64_t>(m)),
+                 "r"(c0), "r"(c1)
+                 : "memory");
+}
 // 1-D bulk copy global -> shared (bytes multiple of 16, both addresses 16-B aligned)
 __device__ __forceinline__ void bulk_load(void* dst, const void* src, uint32_t bytes, uint64_t* bar)
 {

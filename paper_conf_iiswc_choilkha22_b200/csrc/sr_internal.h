@@ -20,8 +20,8 @@ namespace sr {
 constexpr int kRowBlock = 128;  // M of every tcgen05 tile
 constexpr int kHalf = 64;       // validity granularity of tile rows
 
-// Where the IR sub-layer runs: its own kernel (the paper's design), folded into
-// GEMM2 (SR_FUSE_IR), or merged by a warp of GEMM1 as the row's tiles are produced (SR_IR_IN_GEMM1).
+// Where the IR sub-layer runs: its own kernel (SR_IR_KERNEL, the paper's layout), folded into
+// GEMM2 (SR_FUSE_IR), or merged by warps of GEMM1 as the row's tiles are produced (default).
 enum IrMode : int { IR_KERNEL = 0, IR_IN_GEMM2 = 1, IR_IN_GEMM1 = 2 };
 enum MaskKind : int { MK_DENSE = 0, MK_BLOCK = 1, MK_WINDOW = 2 };
 enum DType : int { DT_F32 = 0, DT_F16 = 1, DT_BF16 = 2 };

@@ -11,6 +11,33 @@ namespace sr {
 
 constexpr int kSmemMax = 232448;  // 227 KB opt-in dynamic shared memory per CTA on sm_100
 
+// Diagnostic build (-DSR_DIAG_WAITS, tools/diag_waits.py): every warp accumulates the clock cycles
+// it spends in each class of mbarrier wait (c = 0..3) plus its lifetime (slot 4); lane 0 adds them
+// to a per-kernel device array [warp][5] read back through sr_diag_read().  Off in product builds.
+#ifdef SR_DIAG_WAITS
+constexpr int kDW = 8;  // classes per warp (+1 lifetime slot)
+#define DW_DECL long long dw_[kDW] = {}; const long long dw_start_ = clock64(); long long dw_last_ = dw_start_;
+#define DW_WAIT(bar, ph, c) do { const long long t_ = clock64(); mbar_wait(bar, ph); dw_[c] += clock64() - t_; } while (0)
+#define DW_TIME(stmt, c) do { const long long t_ = clock64(); stmt; dw_[c] += clock64() - t_; } while (0)
+#define DW_PH0() do { dw_last_ = clock64(); } while (0)          /* start a phase sequence */
+#define DW_PH(c) do { const long long t_ = clock64(); dw_[c] += t_ - dw_last_; dw_last_ = t_; } while (0)
+#define DW_FLUSH(arr)                                                                                     \
+    do {                                                                                                  \
+        if ((threadIdx.x & 31) == 0) {                                                                    \
+            const int w_ = threadIdx.x / 32;                                                              \
+            for (int c_ = 0; c_ < kDW; ++c_) atomicAdd(&arr[w_ * (kDW + 1) + c_], (unsigned long long)dw_[c_]); \
+            atomicAdd(&arr[w_ * (kDW + 1) + kDW], (unsigned long long)(clock64() - dw_start_));            \
+        }                                                                                                 \
+    } while (0)
+#else
+#define DW_DECL
+#define DW_WAIT(bar, ph, c) mbar_wait(bar, ph)
+#define DW_TIME(stmt, c) stmt
+#define DW_PH0()
+#define DW_PH(c)
+#define DW_FLUSH(arr)
+#endif
+
 struct ItemInfo {
     int g, rb, t0, t1;
     int64_t slot0;  // slot id of tile t is slot0 + t

@@ -61,8 +61,8 @@ cudaError_t launch_tc_fused(const Params& p, cudaStream_t st, int64_t* nl)
 {
     cudaError_t e = cudaSuccess;
     if ((p.stages & 1) && (e = launch_gemm1(p, true, st, nl)) != cudaSuccess) return e;
-    // the IR sub-layer: its own kernel (the paper's design), folded into GEMM2 (SR_FUSE_IR), or
-    // merged inside GEMM1 (SR_IR_IN_GEMM1, GEMM2 then only reads each row's (m, 1/d))
+    // the IR sub-layer: its own kernel (SR_IR_KERNEL, the paper's layout), folded into GEMM2 (SR_FUSE_IR), or
+    // merged inside GEMM1 (the default, GEMM2 then only reads each row's (m, 1/d))
     if (p.ir_mode == IR_KERNEL && (p.stages & 2) && (e = launch_ir(p, st, nl)) != cudaSuccess) return e;
     if (p.stages & 4) e = launch_gemm2(p, p.ir_mode == IR_KERNEL ? 1 : (p.ir_mode == IR_IN_GEMM2 ? 2 : 3), st, nl);
     return e;

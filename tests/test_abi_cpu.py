@@ -73,8 +73,8 @@ def _call(entry_fn, q=0x10000, k=0x20000000, v=0x40000000, out=0x60000000, B_=1,
     (dict(q=0x10008), sr.SR_ERR_INVALID),                 # misaligned
     (dict(flags=8), sr.SR_ERR_INVALID),
     (dict(flags=128), sr.SR_ERR_INVALID),                 # unknown bit
-    (dict(flags=16 | 64), sr.SR_ERR_INVALID),             # SR_FUSE_IR with SR_IR_IN_GEMM1
-    (dict(flags=32 | 64), sr.SR_ERR_INVALID),             # SR_DECOMPOSE with SR_IR_IN_GEMM1
+    (dict(flags=16 | 64), sr.SR_ERR_INVALID),             # SR_FUSE_IR with SR_IR_KERNEL
+    (dict(flags=32 | 64), sr.SR_ERR_INVALID),             # SR_DECOMPOSE with SR_IR_KERNEL
     (dict(flags=64, in_dt=sr.SR_F32), sr.SR_ERR_UNSUPPORTED),  # variants are 16-bit only
     (dict(tile_n=32), sr.SR_ERR_UNSUPPORTED),
     (dict(in_dt=sr.SR_F32, tile_n=128), sr.SR_ERR_UNSUPPORTED),
@@ -146,7 +146,7 @@ def test_workspace_closed_form_dense(T):
     assert info["n_slots"] * 128 == Bb * H * S * (S // T)  # L N_sv H
     assert info["off_mprime"] >= L2H * 2
     assert info["total_bytes"] >= L2H * 2 + 3 * 4 * Bb * H * S * (S // T)
-    # per-row (m, 1/d) of the SR_IR_IN_GEMM1 variant: 8 bytes per query row, after r'
+    # per-row (m, 1/d) of the default mode (IR in GEMM1): 8 bytes per query row, after r'
     assert info["off_rowstat"] >= info["off_rprime"] + 4 * Bb * H * S * (S // T)
     assert info["total_bytes"] >= info["off_rowstat"] + 8 * Bb * H * S
     unf = sr.workspace_info(sr.dense_mask(None), Bb, H, S, D, sr.SR_F16, tile_n=T, fused=False)

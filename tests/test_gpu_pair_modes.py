@@ -25,11 +25,11 @@ cases = [
     ("window", 1, 2, 1024, 64, "f16", dict(window=128, n_global=8)),
     ("window", 1, 1, 768, 64, "f16", dict(window=126, n_global=8, tile_n=64, fused=False)),
     ("block", 1, 2, 768, 64, "f16", dict(layout=W.random_layout(2, 768 // 64, 64, 0.3, seed=5))),
-    # the IR merged inside GEMM1 follows each schedule's accumulator order
-    ("dense", 1, 2, 640, 128, "bf16", dict(causal=True, ir_in_gemm1=True)),
-    ("dense", 2, 1, 512, 64, "f16", dict(kv_len=[300, 1], ir_in_gemm1=True)),
-    ("dense", 1, 2, 384, 128, "f16", dict(tile_n=64, causal=True, ir_in_gemm1=True)),
-    ("block", 1, 2, 768, 64, "f16", dict(layout=W.random_layout(2, 768 // 64, 64, 0.3, seed=5), ir_in_gemm1=True)),
+    # the paper's standalone IR kernel (SR_IR_KERNEL) on each schedule
+    ("dense", 1, 2, 640, 128, "bf16", dict(causal=True, ir_kernel=True)),
+    ("dense", 2, 1, 512, 64, "f16", dict(kv_len=[300, 1], ir_kernel=True)),
+    ("dense", 1, 2, 384, 128, "f16", dict(tile_n=64, causal=True, ir_kernel=True)),
+    ("block", 1, 2, 768, 64, "f16", dict(layout=W.random_layout(2, 768 // 64, 64, 0.3, seed=5), ir_kernel=True)),
 ]
 for kind, B, H, S, D, dt, kw in cases:
     o, ref = run_case(kind, B, H, S, D, dt, **kw)

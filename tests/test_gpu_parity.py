@@ -34,12 +34,12 @@ def _ulp_half(dtype, ref):
 
 
 def run_case(kind, B, H, S, D, dtype, *, causal=False, kv_len=None, layout=None, window=0, n_global=0,
-             tile_n=0, fused=True, seed=0, out_f32=True, fuse_ir=False, ir_in_gemm1=False):
+             tile_n=0, fused=True, seed=0, out_f32=True, fuse_ir=False, ir_kernel=False):
     t, q, k, v = qkv(B, H, S, D, dtype, seed)
     scale = 1 / math.sqrt(D)
     od = torch.float32 if out_f32 else TORCH[dtype]
     kw = dict(scale=scale, causal=causal, tile_n=tile_n, fused=fused, out_dtype=od, fuse_ir=fuse_ir,
-              ir_in_gemm1=ir_in_gemm1)
+              ir_kernel=ir_kernel)
     if kind == "dense":
         o = sr.mha_dense(q, k, v, kv_len=kv_len, **kw)
     elif kind == "block":
@@ -216,13 +216,14 @@ def test_kv_len_one_and_zero():
 # ------------------------------------------------------------------------------------ intermediates
 
 def test_intermediates_match_recomposed_oracle():
-    """m', d', r' read back from the workspace vs the oracle's Eq. (2) decomposition (T = 128)."""
+    """m', d', r' read back from the workspace (SR_IR_KERNEL, the mode that writes d' and r') vs the
+    oracle's Eq. (2) decomposition (T = 128)."""
     B, H, S, D, T = 1, 2, 384, 64, 128
     t, q, k, v = qkv(B, H, S, D, "f16", seed=3)
     mask = sr.dense_mask(None)
     info = sr.workspace_info(mask, B, H, S, D, sr.SR_F16, causal=True, tile_n=T)
     ws = torch.zeros(info["total_bytes"], dtype=torch.uint8, device="cuda")
-    sr.call(mask, q, k, v, scale=0.125, causal=True, tile_n=T, workspace=ws)
+    sr.call(mask, q, k, v, scale=0.125, causal=True, tile_n=T, workspace=ws, ir_kernel=True)
     torch.cuda.synchronize()
     _, mp_ref, dp_ref, rp_ref = oracle.recomposed(t.q64, t.k64, t.v64, 0.125, T, oracle.Mask(causal=True))
     n = info["n_slots"] * 128
@@ -241,7 +242,7 @@ def test_intermediates_match_recomposed_oracle():
 
 @pytest.mark.parametrize("T", [64, 128])
 def test_row_statistics_ir_in_gemm1(T):
-    """SR_IR_IN_GEMM1: the per-row (m, 1/d) GEMM1's IR warp writes vs the oracle's Eq. (2) values:
+    """Default mode (IR in GEMM1): the per-row (m, 1/d) GEMM1's IR warps write vs the oracle's Eq. (2) values:
     m = max_k m'_k, and 1/d = max_k r'_k (r'_k = e^{m'_k - m}/d is 1/d on the tile holding the max)."""
     B, H, S, D = 2, 2, 384, 64
     t, q, k, v = qkv(B, H, S, D, "f16", seed=4)
@@ -249,8 +250,7 @@ def test_row_statistics_ir_in_gemm1(T):
     mask = sr.dense_mask(kv)
     info = sr.workspace_info(mask, B, H, S, D, sr.SR_F16, causal=True, tile_n=T)
     ws = torch.zeros(info["total_bytes"], dtype=torch.uint8, device="cuda")
-    o = sr.call(mask, q, k, v, scale=0.125, causal=True, tile_n=T, workspace=ws, ir_in_gemm1=True,
-                out_dtype=torch.float32)
+    o = sr.call(mask, q, k, v, scale=0.125, causal=True, tile_n=T, workspace=ws, out_dtype=torch.float32)
     torch.cuda.synchronize()
     om = oracle.Mask(causal=True, kv_len=kv)
     o_ref, mp_ref, dp_ref, rp_ref = oracle.recomposed(t.q64, t.k64, t.v64, 0.125, T, om)
@@ -367,14 +367,14 @@ FUSED_IR_CASES = [
 ]
 
 
-VARIANTS = ["fuse_ir", "ir_in_gemm1"]
+VARIANTS = ["fuse_ir", "ir_kernel"]
 
 
 @pytest.mark.parametrize("variant", VARIANTS)
 @pytest.mark.parametrize("kind,kw", FUSED_IR_CASES, ids=lambda x: str(x)[:40] if isinstance(x, dict) else x)
 def test_fused_ir_variant(kind, kw, variant):
-    """The IR placements against the oracle, same tolerance: SR_FUSE_IR (IR folded into GEMM2,
-    SURVEY NEXT-2) and SR_IR_IN_GEMM1 (rows merged by a GEMM1 warp, GEMM2 normalises)."""
+    """The other IR placements against the oracle, same tolerance: SR_FUSE_IR (IR folded into
+    GEMM2) and SR_IR_KERNEL (the paper's standalone IR kernel writing r')."""
     kw = dict(kw)
     if kw.get("layout") == "rand":
         kw["layout"] = W.random_layout(kw["H"], kw["S"] // 64, 64, 0.35, seed=8)

@@ -13,8 +13,11 @@ try:
 except Exception:
     print(lib, c, "FAILED", open(f"gpurun_out/ab_{lib}_{c}.err").read()[-400:]); sys.exit()
 k = {n: round(v["us"], 2) for n, v in d["kernels"].items()}
-fi = d.get("variants", {}).get("fused_ir", {}).get("ms_per_step")
-print(f"{lib:12s} C{c} ms={d['ms_per_step']:.4f} fir={fi} {k}")
+v = d.get("variants") or {}
+fi = v.get("fused_ir", {}).get("ms_per_step")
+g1 = v.get("ir_kernel", {})
+kg = {n: round(x["us"], 2) for n, x in (g1.get("kernels") or {}).items()}
+print(f"{lib:22s} C{c} ms={d['ms_per_step']:.4f} fir={fi} irk={g1.get('ms_per_step')} {k} irk_k={kg}")
 PY
   done
 done

@@ -14,7 +14,7 @@ k = {n: (v["us"], v["GB/s"]) for n, v in d["kernels"].items()}
 u = d["unfused"]["ms_per_step"] if d["unfused"] else None
 v = d.get("variants") or {}
 vs = {n: x["ms_per_step"] for n, x in v.items()}
-kg = {n: x["us"] for n, x in (v.get("ir_in_gemm1", {}).get("kernels") or {}).items()}
-print(f"{tag} C{c} ms={d['ms_per_step']:.4f} unf={u} frac={d['roofline']['frac']} {k} variants={vs} g1ir_kernels={kg}")
+kg = {n: x["us"] for n, x in (v.get("ir_kernel", {}).get("kernels") or {}).items()}
+print(f"{tag} C{c} ms={d['ms_per_step']:.4f} unf={u} frac={d['roofline']['frac']} {k} variants={vs} irk_kernels={kg}")
 PY
 done

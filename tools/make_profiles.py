@@ -24,10 +24,14 @@ def kname(full):
     if m:
         a = [x.strip() for x in m.group(2).split(",")]
         flags = [x in ("true", "1", "(bool)1") for x in a[2:]]
-        if m.group(1) == "tc_gemm1":
-            return "gemm1_ls" if flags and flags[0] else "gemm1_plain"
-        if flags and flags[0]:
-            return "gs_gemm2_fused_ir" if len(flags) > 1 and flags[1] else "gs_gemm2"
+        if m.group(1) == "tc_gemm1":  # <D, T, LS, PAIR, IRT>
+            if not (flags and flags[0]):
+                return "gemm1_plain"
+            return "gemm1_ls_ir" if len(flags) > 2 and flags[2] else "gemm1_ls"
+        if flags and flags[0]:  # <D, T, GS, FI, RS>
+            if len(flags) > 2 and flags[2]:
+                return "gs_gemm2"  # default path: (m, 1/d) from GEMM1
+            return "gs_gemm2_fused_ir" if len(flags) > 1 and flags[1] else "gs_gemm2_rprime"
         return "gemm2_plain"
     for k, v in (("ir_kernel", "ir"), ("row_softmax", "softmax"), ("sd_ls_kernel", "sd_ls"),
                  ("sd_gs_kernel", "sd_gs")):
@@ -73,7 +77,7 @@ def main(rnd):
             lines.append(f"{n:28s} {len(m['gpu__time_duration.sum']):8d} {t / 1e3 * unit:10.2f} {rd / 1e6:11.2f} {wr / 1e6:11.2f}")
             if not n.startswith("other"):
                 ours[n] = (t, rd + wr)
-        rec = [k for k in ("gemm1_ls", "ir", "gs_gemm2") if k in ours]
+        rec = [k for k in ("gemm1_ls_ir", "gs_gemm2") if k in ours]  # default path (IR in GEMM1)
         unf = [k for k in ("gemm1_plain", "softmax", "gemm2_plain") if k in ours]
         tr = sum(ours[k][0] for k in rec)
         lines.append("")
@@ -81,6 +85,10 @@ def main(rnd):
         tu = sum(ours[k][0] for k in unf) if unf else 0
         if unf:
             lines.append("unfused layer shares:    " + ", ".join(f"{k} {ours[k][0] / tu:.1%}" for k in unf))
+        irk = [k for k in ("gemm1_ls", "ir", "gs_gemm2_rprime") if k in ours]
+        if len(irk) == 3:
+            tk = sum(ours[k][0] for k in irk)
+            lines.append("IR-kernel (paper layout) shares: " + ", ".join(f"{k} {ours[k][0] / tk:.1%}" for k in irk))
         fir = [k for k in ("gemm1_ls", "gs_gemm2_fused_ir") if k in ours]
         if len(fir) == 2:
             tf = sum(ours[k][0] for k in fir)
@@ -91,6 +99,8 @@ def main(rnd):
             lines.append("SD variant shares:       " + ", ".join(f"{k} {ours[k][0] / ts:.1%}" for k in sd))
         e = {f"{k}_dram_bytes": int(ours[k][1]) for k in ours}
         e["recomposed_dram_bytes"] = int(sum(ours[k][1] for k in rec))
+        if len(irk) == 3:
+            e["ir_kernel_dram_bytes"] = int(sum(ours[k][1] for k in irk))
         if unf:
             e["unfused_dram_bytes"] = int(sum(ours[k][1] for k in unf))
         lines.append(f"DRAM bytes per layer (cold, per-kernel sum): recomposed {e['recomposed_dram_bytes'] / 1e6:.1f} MB"

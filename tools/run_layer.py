@@ -1,5 +1,5 @@
 """Run one config's layer a few times (for ncu captures):
-    python tools/run_layer.py CFG [fused|unfused|fused_ir|sd] [reps]"""
+    python tools/run_layer.py CFG [fused|unfused|fused_ir|ir_kernel|sd] [reps]"""
 import os
 import sys
 
@@ -17,6 +17,6 @@ reps = int(sys.argv[3]) if len(sys.argv) > 3 else 2
 cfg = W.config(idx)
 L = Layer(cfg, torch.device("cuda", 0), cfg.idx, sr, torch)
 for _ in range(reps):
-    L.run(fused=fused, fuse_ir=mode == "fused_ir", sd=mode == "sd")
+    L.run(fused=fused, fuse_ir=mode == "fused_ir", sd=mode == "sd", ir_kernel=mode == "ir_kernel")
 torch.cuda.synchronize()
 print("ok", cfg.name, mode)
