@@ -506,7 +506,7 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
             const int buf = n % C::NACC;
             DW_WAIT(&acc_full[buf], (uint32_t)(n / C::NACC) & 1, 0);
             tc_fence_after();
-            const G1Hdr H = hdr[buf];
+            const G1Hdr H = lds_hdr(hdr + buf);
             if (H.flags & HDR_END) break;
             // this warpgroup's 64 columns: sub-tile h (T = 64) or half h of the sub-tile (T = 128)
             const int w = (NSUB == 2 && h == 1) ? H.w1 : H.w0;
@@ -643,7 +643,7 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
             const int buf = n % C::NACC;
             DW_WAIT(&acc_full[buf], (uint32_t)(n / C::NACC) & 1, 0);
             tc_fence_after();
-            const G1Hdr H = hdr[buf];
+            const G1Hdr H = lds_hdr(hdr + buf);
             if (H.flags & HDR_END) break;
             const int wsub[2] = {H.w0, H.w1};
             bool vs[NSUB];  // this row's 64-row half is valid in sub-tile s

@@ -390,7 +390,7 @@ __global__ void __launch_bounds__(512, 1) tc_gemm2(const __grid_constant__ CUten
         float m_row = 0.f, invd_row = 0.f;  // fused IR: this row's (m, 1/d) for the current item
         for (;;) {
             DW_WAIT(&x_full[s], sph, 0);
-            const G2Hdr h = *xhdr(s);
+            const G2Hdr h = lds_hdr(xhdr(s));
             if (h.flags & SH_END) break;
             if (FI && (h.flags & SH_FIRST)) {  // a new item: its row statistics from the IR warp
                 DW_WAIT(&st_full[si], siph, 2);
@@ -422,8 +422,8 @@ __global__ void __launch_bounds__(512, 1) tc_gemm2(const __grid_constant__ CUten
             if (false)
 #endif
 #pragma unroll
-            for (int q = 0; q < kMW2 / 16; ++q)
-                if (rr[((ch * 8 + q) * 8) / T] != 0.f) xv[q] = lds128(xs_s + tile_chunk_off(r, ch * 8 + q));
+            for (int q = 0; q < kMW2 / 16; ++q)  // unconditional: issued beside the r' chain (unused if r' = 0)
+                xv[q] = lds128(xs_s + tile_chunk_off(r, ch * 8 + q));
             DW_WAIT(&a_empty[a], aph ^ 1, 1);
             tc_fence_after();
             const uint32_t a_tm = tmem_a + lane_off + a * (kMW2 / 2);
@@ -479,7 +479,7 @@ __global__ void __launch_bounds__(512, 1) tc_gemm2(const __grid_constant__ CUten
         for (;;) {
             DW_WAIT(&o_full[o], oph, 0);
             tc_fence_after();
-            const G2Hdr h = ohdr[o];
+            const G2Hdr h = lds_hdr(ohdr + o);
             if (h.flags & SH_END) break;
             const int64_t orow = (((int64_t)h.orow_hi << 32) | (uint32_t)h.orow_lo) + r;
             if (h.flags & SH_EMPTY) {  // no kept key anywhere in these rows: output 0 (reading R9)

@@ -38,6 +38,21 @@ constexpr int kDW = 8;  // classes per warp (+1 lifetime slot)
 #define DW_FLUSH(arr)
 #endif
 
+// 32-byte stage/accumulator headers are read with two ld.shared.v4 (a generic load of shared
+// memory costs a long-scoreboard round trip on the consumer's critical path)
+template <typename Hdr>
+__device__ __forceinline__ Hdr lds_hdr(const Hdr* h)
+{
+    static_assert(sizeof(Hdr) == 32, "32-byte header");
+    const uint32_t a = ptx::smem_u32(h);
+    const uint4 x = ptx::lds128(a), y = ptx::lds128(a + 16);
+    Hdr r;
+    int32_t* w = reinterpret_cast<int32_t*>(&r);
+    w[0] = (int32_t)x.x; w[1] = (int32_t)x.y; w[2] = (int32_t)x.z; w[3] = (int32_t)x.w;
+    w[4] = (int32_t)y.x; w[5] = (int32_t)y.y; w[6] = (int32_t)y.z; w[7] = (int32_t)y.w;
+    return r;
+}
+
 struct ItemInfo {
     int g, rb, t0, t1;
     int64_t slot0;  // slot id of tile t is slot0 + t
