@@ -52,6 +52,10 @@ constexpr int kMW = 128;  // macro tile width (MMA N of GEMM1)
 #define SR_G1_QPREFETCH 0
 #endif
 constexpr bool kQPrefetch = SR_G1_QPREFETCH;  // L2 prefetch of the next item's Q (measured: C3 slower, off)
+#ifndef SR_G1_HINTS
+#define SR_G1_HINTS 1
+#endif
+constexpr bool kG1Hints = SR_G1_HINTS;  // X' stores evict_first (streamed), K loads evict_last (re-read by every row-block)
 // Of every 8 element pairs of the LS exponentials, this many are computed by ex2_poly2 on the FMA
 // pipe and the rest by MUFU.EX2 (16 / clock / SM): balances the two pipes in the epilogue.
 #ifndef SR_G1_POLY_PAIRS
@@ -131,6 +135,15 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
 
     const int warp = warp_uniform(), lane = threadIdx.x % 32;
     DW_DECL
+    const uint64_t pol_k = kG1Hints ? policy_evict_last() : 0, pol_x = kG1Hints ? policy_evict_first() : 0;
+    auto kload = [&](void* d, const CUtensorMap* m, int c0, int c1, uint64_t* b) {
+        if (kG1Hints) tma_load_2d_hint(d, m, c0, c1, b, pol_k);
+        else tma_load_2d(d, m, c0, c1, b);
+    };
+    auto xstore = [&](void* d, const void* src, uint32_t nb) {
+        if (kG1Hints) bulk_store_hint(d, src, nb, pol_x);
+        else bulk_store(d, src, nb);
+    };
     if (threadIdx.x == 0) {
         for (int i = 0; i < C::NQ; ++i) { mbar_init(&q_full[i], 1); mbar_init(&q_empty[i], 1); }
         for (int i = 0; i < C::NK; ++i) { mbar_init(&k_full[i], 1); mbar_init(&k_empty[i], 1); }
@@ -208,7 +221,7 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
                         mbar_arrive_expect_tx(&k_full[ks], nsub * T * D * 2);
                         for (int s2 = 0; s2 < nsub; ++s2)
                             for (int h = 0; h < D / 64; ++h)
-                                tma_load_2d(smem + C::OFF_K + ks * C::KB + h * (kMW * 128) + s2 * (T * 128), &tmK,
+                                kload(smem + C::OFF_K + ks * C::KB + h * (kMW * 128) + s2 * (T * 128), &tmK,
                                             h * 64, g * p.S + (w[s2] & 0xFFFF) * T, &k_full[ks]);
                     }
                     __syncwarp();
@@ -341,7 +354,7 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
 #endif
                         for (int s = 0; s < nsub; ++s)
                             for (int h = 0; h < D / 64; ++h)
-                                tma_load_2d(smem + C::OFF_K + ks * C::KB + h * (kMW * 128) + s * (T * 128), &tmK,
+                                kload(smem + C::OFF_K + ks * C::KB + h * (kMW * 128) + s * (T * 128), &tmK,
                                             h * 64, I.g * p.S + tinfo_kt(w[s]) * T, &k_full[ks]);
                     }
                     __syncwarp();
@@ -609,7 +622,7 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
                 if (valid) {  // warp-uniform: a warp's 32 rows lie in one 64-row half
                     uint8_t* dst = (uint8_t*)p.xprime + slot * (int64_t)C::XS + (NSUB == 1 ? h * C::HB : 0) +
                                    q * 32 * 128;
-                    bulk_store(dst, stage + q * 32 * 128, 32 * 128);
+                    xstore(dst, stage + q * 32 * 128, 32 * 128);
                 }
                 bulk_commit();
             }
@@ -763,7 +776,7 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
                     uint8_t* dst = (uint8_t*)p.xprime + (slot + (s ? H.pad : 0)) * (int64_t)C::XS;
                     for (int ch = 0; ch < T / 64; ++ch)
 #ifndef SR_DIAG_NOSTORE
-                        bulk_store(dst + ch * (kRowBlock * 128) + wrow0 * 128,
+                        xstore(dst + ch * (kRowBlock * 128) + wrow0 * 128,
                                    stage + (s * (T / 64) + ch) * (kRowBlock * 128) + wrow0 * 128, 32 * 128);
 #else
                         (void)dst;

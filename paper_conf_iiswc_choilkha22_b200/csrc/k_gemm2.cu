@@ -43,6 +43,14 @@ namespace sr {
 #endif
 
 constexpr int kMW2 = 128;  // macro tile width (keys per MMA step)
+// L2 policy experiments: X' is streamed once (evict_first), V is re-read by every row-block of its
+// head (evict_last); V_PREFETCH: the V producer warms the macro tile NV ahead in L2
+#ifndef SR_G2_HINTS
+#define SR_G2_HINTS 1
+#endif
+#ifndef SR_G2_VPREFETCH
+#define SR_G2_VPREFETCH 0
+#endif
 
 enum : int { SH_TILE = 1, SH_END = 2, SH_EMPTY = 4, SH_FIRST = 8, SH_LAST = 16 };
 struct G2Hdr {  // X'-stage / O-buffer header
@@ -151,6 +159,7 @@ __global__ void __launch_bounds__(512, 1) tc_gemm2(const __grid_constant__ CUten
             // -------------------------------------------------------------- X' producer (whole
             // warp walks the schedule; one elected lane issues)
             int s = 0;
+            const uint64_t pol_x = SR_G2_HINTS ? policy_evict_first() : 0;
             uint32_t sph = 0;
             for (ItemWalk iw(p, it_begin, it_end); iw.more();) {
                 const ItemInfo I = iw.next();
@@ -174,16 +183,20 @@ __global__ void __launch_bounds__(512, 1) tc_gemm2(const __grid_constant__ CUten
 #ifdef SR_DIAG2_NOX
                     if (false)
 #endif
+                    auto xload = [&](uint8_t* d, const uint8_t* g, uint32_t n) {
+                        if (SR_G2_HINTS) bulk_load_hint(d, g, n, &x_full[s], pol_x);
+                        else bulk_load(d, g, n, &x_full[s]);
+                    };
                     if (hv[0] == 3 && (nsub == 1 || hv[1] == 3)) {
-                        bulk_load(st, xs, nsub * C::XS, &x_full[s]);
+                        xload(st, xs, nsub * C::XS);
                     } else {
                         for (int u = 0; u < nsub; ++u)
                             for (int ch = 0; ch < T / 64; ++ch) {
                                 const int o = u * C::XS + ch * (kRowBlock * 128);
-                                if (hv[u] == 3) bulk_load(st + o, xs + o, kRowBlock * 128, &x_full[s]);
+                                if (hv[u] == 3) xload(st + o, xs + o, kRowBlock * 128);
                                 else {
                                     const int o2 = o + (hv[u] == 2 ? kHalf * 128 : 0);
-                                    bulk_load(st + o2, xs + o2, kHalf * 128, &x_full[s]);
+                                    xload(st + o2, xs + o2, kHalf * 128);
                                 }
                             }
                     }
@@ -292,6 +305,7 @@ __global__ void __launch_bounds__(512, 1) tc_gemm2(const __grid_constant__ CUten
             // -------------------------------------------------------------- V producer (whole warp,
             // one elected lane issues)
             int s = 0;
+            const uint64_t pol_v = SR_G2_HINTS ? policy_evict_last() : 0;
             uint32_t sph = 0;
             for (ItemWalk iw(p, it_begin, it_end); iw.more();) {
                 const ItemInfo I = iw.next();
@@ -310,9 +324,22 @@ __global__ void __launch_bounds__(512, 1) tc_gemm2(const __grid_constant__ CUten
                         mbar_arrive_expect_tx(&v_full[s], nsub * T * D * 2);
 #endif
                         for (int u = 0; u < nsub; ++u)
-                            for (int h = 0; h < D / 64; ++h)
-                                tma_load_2d(vstage(s) + h * (kMW2 * 128) + u * (T * 128), &tmV, h * 64,
-                                            I.g * p.S + kt[u] * T, &v_full[s]);
+                            for (int h = 0; h < D / 64; ++h) {
+                                if (SR_G2_HINTS)
+                                    tma_load_2d_hint(vstage(s) + h * (kMW2 * 128) + u * (T * 128), &tmV, h * 64,
+                                                     I.g * p.S + kt[u] * T, &v_full[s], pol_v);
+                                else
+                                    tma_load_2d(vstage(s) + h * (kMW2 * 128) + u * (T * 128), &tmV, h * 64,
+                                                I.g * p.S + kt[u] * T, &v_full[s]);
+                            }
+                        if (SR_G2_VPREFETCH) {  // the macro tile NV steps ahead in this item, into L2
+                            const int tp = t + C::NV * NSUB;
+                            for (int u = 0; u < NSUB; ++u)
+                                if (tp + u < I.t1) {
+                                    const int ktp = tinfo_kt(__ldg(p.sc.tinfo + tp + u));
+                                    for (int h = 0; h < D / 64; ++h) tma_prefetch_2d(&tmV, h * 64, I.g * p.S + ktp * T);
+                                }
+                        }
                     }
                     __syncwarp();
                     if (++s == C::NV) { s = 0; sph ^= 1; }
