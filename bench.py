@@ -411,8 +411,8 @@ def oracle_mask_for(cfg):
     if cfg.kind == "dense":
         return oracle.Mask(kv_len=cfg.kv_len, causal=cfg.causal)
     if cfg.kind == "blocksparse":
-        return oracle.Mask(kind="block", layout=W.config_layout(cfg))
-    return oracle.Mask(kind="window", window=cfg.window, n_global=cfg.n_global)
+        return oracle.Mask(kind="block", layout=W.config_layout(cfg), causal=cfg.causal)
+    return oracle.Mask(kind="window", window=cfg.window, n_global=cfg.n_global, causal=cfg.causal)
 
 
 def cpu_baseline(cfg, target_s=10.0):
