@@ -180,13 +180,13 @@ __global__ void __launch_bounds__(512, 1) tc_gemm2(const __grid_constant__ CUten
                                      hv[1], nsub, 0, 0, 0, 0};
                     mbar_arrive_expect_tx(&x_full[s], bytes);
                     const uint8_t* xs = src + (I.slot0 + t) * (int64_t)C::XS;  // sub-tiles t, t+1 are adjacent
-#ifdef SR_DIAG2_NOX
-                    if (false)
-#endif
                     auto xload = [&](uint8_t* d, const uint8_t* g, uint32_t n) {
                         if (SR_G2_HINTS) bulk_load_hint(d, g, n, &x_full[s], pol_x);
                         else bulk_load(d, g, n, &x_full[s]);
                     };
+#ifdef SR_DIAG2_NOX
+                    if (false)
+#endif
                     if (hv[0] == 3 && (nsub == 1 || hv[1] == 3)) {
                         xload(st, xs, nsub * C::XS);
                     } else {
