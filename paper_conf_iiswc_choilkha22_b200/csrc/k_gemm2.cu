@@ -93,8 +93,12 @@ struct G2 {
     static constexpr int OFF_TPTR = OFF_OHDR + NO * (int)sizeof(G2Hdr);
     static constexpr int SMEM_ = OFF_TPTR + 16 + 1024;
     static constexpr int SMEM = SMEM_ > 118 * 1024 ? SMEM_ : 118 * 1024;  // 1 CTA/SM (512 TMEM cols)
-    static constexpr int THREADS = 512;
-    static constexpr int NGS = 8;  // GS warps
+#ifndef SR_G2_NGS
+#define SR_G2_NGS 8
+#endif
+    static constexpr int NGS = SR_G2_NGS;       // GS warps: 8 (64 keys each) or 16 (32 keys each)
+    static constexpr int KPW = kMW2 * 4 / NGS;  // keys of a macro tile per GS warp
+    static constexpr int THREADS = 128 + NGS * 32 + 128;
 };
 
 // FI (fused IR): the IR sub-layer runs inside this kernel -- warp 2 reduces each
@@ -103,7 +107,7 @@ struct G2 {
 // RS (default mode, IR in GEMM1): as FI, but GEMM1 already merged the rows, so warp 2 only loads each item's
 // per-row (m, 1/d) -- GEMM2 applies the normalisation 1/d * e^{m' - m} in its prologue.
 template <int D, int T, bool GS, bool FI, bool RS>
-__global__ void __launch_bounds__(512, 1) tc_gemm2(const __grid_constant__ CUtensorMap tmV, const Params p)
+__global__ void __launch_bounds__(G2<D, T>::THREADS, 1) tc_gemm2(const __grid_constant__ CUtensorMap tmV, const Params p)
 {
     using C = G2<D, T>;
     constexpr int NSUB = C::NSUB;
@@ -407,7 +411,8 @@ __global__ void __launch_bounds__(512, 1) tc_gemm2(const __grid_constant__ CUten
         }
     } else if (warp >= 4 && warp < 4 + C::NGS) {
         // ------------------------------------------------------------------ GS transform
-        const int gq = (warp - 4) % 4, ch = (warp - 4) / 4;  // lane quadrant, key half (64 keys)
+        const int gq = (warp - 4) % 4, ch = (warp - 4) / 4;  // lane quadrant, key slice (KPW keys)
+        constexpr int KPW = C::KPW;
         const int r = gq * 32 + lane;
         const int myhalf = r / kHalf;
         const uint32_t lane_off = (uint32_t)(gq * 32) << 16;
@@ -442,21 +447,21 @@ __global__ void __launch_bounds__(512, 1) tc_gemm2(const __grid_constant__ CUten
                         rr[u] = v;
                 }
             }
-            // this warp's half of the X' row (64 fp16 = 8 chunks of 16 B) into registers first: the
-            // loads overlap the wait for a free A buffer
-            uint4 xv[kMW2 / 16];
+            // this warp's slice of the X' row (KPW fp16 = KPW/8 chunks of 16 B) into registers first:
+            // the loads overlap the wait for a free A buffer
+            uint4 xv[KPW / 8];
 #ifdef SR_DIAG2_NOGS
             if (false)
 #endif
 #pragma unroll
-            for (int q = 0; q < kMW2 / 16; ++q)  // unconditional: issued beside the r' chain (unused if r' = 0)
-                xv[q] = lds128(xs_s + tile_chunk_off(r, ch * 8 + q));
+            for (int q = 0; q < KPW / 8; ++q)  // unconditional: issued beside the r' chain (unused if r' = 0)
+                xv[q] = lds128(xs_s + tile_chunk_off(r, ch * (KPW / 8) + q));
             DW_WAIT(&a_empty[a], aph ^ 1, 1);
             tc_fence_after();
             const uint32_t a_tm = tmem_a + lane_off + a * (kMW2 / 2);
 #pragma unroll
-            for (int c2 = 0; c2 < 2; ++c2) {  // 32 keys -> 16 packed words per tcgen05.st
-                const int c = ch * 2 + c2;
+            for (int c2 = 0; c2 < KPW / 32; ++c2) {  // 32 keys -> 16 packed words per tcgen05.st
+                const int c = ch * (KPW / 32) + c2;
                 const int u = (c * 32) / T;   // sub-tile of these keys
                 uint32_t pk[16];
                 if (rr[u] != 0.f) {
