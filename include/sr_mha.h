@@ -162,7 +162,8 @@ typedef enum { SR_E_DENSE = 0, SR_E_BLOCKSPARSE = 1, SR_E_WINDOW = 2 } sr_entry;
  *            SWIZZLE_128B K-major layout [T/64][128 rows][64 cols] with the 16-byte chunk index
  *            XOR (row & 7); fp32 tiles are plain row-major [128][T].
  *   mprime, dprime, rprime   fp32 [slot id][128 rows]  (m' in natural-log units)
- *   rowstat  fp32 [2][B*H*S]: per query row m (natural-log units), then 1/d (default mode)
+ *   rowstat  fp32 [2][2][B*H*S] (default mode): two partial row statistics per query row, each
+ *            m_w (natural-log units) then d_w; the row's m = max_w m_w, d = sum_w e^{m_w - m} d_w
  */
 typedef struct {
     int32_t tile_n;           /* T actually used */
@@ -170,7 +171,7 @@ typedef struct {
     int64_t n_slots;          /* B*H*slots_per_head */
     int32_t xprime_elt_bytes; /* 2 (16-bit paths) or 4 (fp32 path) */
     size_t off_xprime, off_mprime, off_dprime, off_rprime, off_p;  /* off_p: unfused P region */
-    size_t off_rowstat;       /* recomposed: per-row (m, 1/d) of the default (IR in GEMM1) mode */
+    size_t off_rowstat;       /* recomposed: per-row partial (m, d) of the default (IR in GEMM1) mode */
     size_t total_bytes;
 } sr_ws_info;
 

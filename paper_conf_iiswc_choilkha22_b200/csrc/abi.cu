@@ -465,7 +465,7 @@ void ws_layout(const HostSched& h, int B, int H, int in_dtype, int fused, sr_ws_
         info->off_mprime = o; o = align_up(o + stat_bytes, 1024);
         info->off_dprime = o; o = align_up(o + stat_bytes, 1024);
         info->off_rprime = o; o = align_up(o + stat_bytes, 1024);
-        info->off_rowstat = o; o = align_up(o + (size_t)2 * B * H * h.n_rb * kRowBlock * sizeof(float), 1024);
+        info->off_rowstat = o; o = align_up(o + (size_t)4 * B * H * h.n_rb * kRowBlock * sizeof(float), 1024);
     }
     info->total_bytes = std::max<size_t>(o, 1024);
 }

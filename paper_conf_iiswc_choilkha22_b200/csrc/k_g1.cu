@@ -150,7 +150,7 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
         // acc_full: header arrive (MMA thread) + tcgen05.commit; acc_empty: one arrive per epilogue
         // warp that reads the accumulator (the warpgroup pair in SPLIT, one warpgroup in FULL)
         for (int i = 0; i < C::NACC; ++i) { mbar_init(&acc_full[i], 2); mbar_init(&acc_empty[i], SPLIT ? 8 : 4); }
-        for (int i = 0; i < C::NACC; ++i) { mbar_init(&st_full[i], SPLIT ? 8 : 4); mbar_init(&st_empty[i], 2); }
+        for (int i = 0; i < C::NACC; ++i) { mbar_init(&st_full[i], SPLIT ? 8 : 4); mbar_init(&st_empty[i], 1); }
         fence_mbar_init();
     }
     if (warp == 0 && lane == 0) { prefetch_tmap(&tmQ); prefetch_tmap(&tmK); }
@@ -422,51 +422,55 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
             }
         } else if (IRT && (warp == 2 || warp == 3)) {
             // -------------------------------------------------------------- IR warps (default mode)
-            // The IR sub-layer of every row this CTA owns: per accumulator (in
-            // the MMA warp's order) merge the staged (m'_k, d'_k) of each row into a running
+            // The IR sub-layer of every row this CTA owns: merge the staged
+            // (m'_k, d'_k) of each row into a running
             //   m = max_k m'_k,   d = sum_k e^{m'_k - m} d'_k
-            // and at the end of a row-block write m (natural-log units) and 1/d; GEMM2 forms
-            // r'_k = e^{m'_k - m} / d in its prologue.  Warp 2 owns rows 0-63 of a row-block, warp 3
-            // rows 64-127 (lane l: rows l, l + 32 of its half).  Both arrive on st_empty.
+            // Warp 2 takes the even accumulators (epilogue warpgroup / pair 0), warp 3 the odd ones,
+            // so the two epilogue streams never wait on each other through the statistics ring; at a
+            // row-block's end each warp writes its partial (m_w in natural-log units, d_w) to its
+            // half of `rowstat`, and GEMM2 merges the two partials into the row's (m, 1/d) and forms
+            // r'_k = e^{m'_k - m} / d in its prologue.  Lane l owns rows l + 32 j of a row-block.
             const float sl2 = p.scale_log2;
-            const int rbase = (warp - 2) * 64 + lane;
+            const int par = warp - 2;
             int n = 0;
-            auto merge = [&](float (&m)[2], float (&d)[2]) {
-                const int buf = n % C::NACC;
-                DW_WAIT(&st_full[buf], (uint32_t)(n / C::NACC) & 1, 0);
-                const float* sb = stats + buf * (4 * kRowBlock) + rbase;
-                float mk[2][NSUB], dk[2][NSUB];
+            auto merge = [&](float (&m)[4], float (&d)[4]) {
+                if ((n & 1) == par) {
+                    const int buf = n % C::NACC;
+                    DW_WAIT(&st_full[buf], (uint32_t)(n / C::NACC) & 1, 0);
+                    const float* sb = stats + buf * (4 * kRowBlock) + lane;
+                    float mk[4][NSUB], dk[4][NSUB];
 #pragma unroll
-                for (int j = 0; j < 2; ++j)
+                    for (int j = 0; j < 4; ++j)
 #pragma unroll
-                    for (int s = 0; s < NSUB; ++s) {
-                        mk[j][s] = sb[(2 * s) * kRowBlock + 32 * j];  // raw score units, -inf if invalid
-                        dk[j][s] = sb[(2 * s + 1) * kRowBlock + 32 * j];
-                    }
-                __syncwarp();  // every lane's reads of the stage are done
-                if (lane == 0) mbar_arrive(&st_empty[buf]);
+                        for (int s = 0; s < NSUB; ++s) {
+                            mk[j][s] = sb[(2 * s) * kRowBlock + 32 * j];  // raw score units, -inf if invalid
+                            dk[j][s] = sb[(2 * s + 1) * kRowBlock + 32 * j];
+                        }
+                    __syncwarp();  // every lane's reads of the stage are done
+                    if (lane == 0) mbar_arrive(&st_empty[buf]);
 #pragma unroll
-                for (int j = 0; j < 2; ++j) {
-                    float mn = m[j];
+                    for (int j = 0; j < 4; ++j) {
+                        float mn = m[j];
 #pragma unroll
-                    for (int s = 0; s < NSUB; ++s) mn = fmaxf(mn, mk[j][s]);
-                    if (mn != -INFINITY) {  // ex2(-inf) = 0 covers empty sides
-                        float acc = d[j] * ex2((m[j] - mn) * sl2);
+                        for (int s = 0; s < NSUB; ++s) mn = fmaxf(mn, mk[j][s]);
+                        if (mn != -INFINITY) {  // ex2(-inf) = 0 covers empty sides
+                            float acc = d[j] * ex2((m[j] - mn) * sl2);
 #pragma unroll
-                        for (int s = 0; s < NSUB; ++s) acc = fmaf(dk[j][s], ex2((mk[j][s] - mn) * sl2), acc);
-                        d[j] = acc;
-                        m[j] = mn;
+                            for (int s = 0; s < NSUB; ++s) acc = fmaf(dk[j][s], ex2((mk[j][s] - mn) * sl2), acc);
+                            d[j] = acc;
+                            m[j] = mn;
+                        }
                     }
                 }
                 ++n;
             };
-            auto flush = [&](int g, int rb, const float (&m)[2], const float (&d)[2]) {
-                const int64_t row = (int64_t)g * p.S + rb * kRowBlock + rbase;
+            auto flush = [&](int g, int rb, const float (&m)[4], const float (&d)[4]) {
                 const int64_t nrow = (int64_t)p.B * p.H * p.S;
+                const int64_t row = (int64_t)g * p.S + rb * kRowBlock + lane + 2 * par * nrow;
 #pragma unroll
-                for (int j = 0; j < 2; ++j) {
+                for (int j = 0; j < 4; ++j) {
                     p.rowstat[row + 32 * j] = m[j] * p.scale;  // -inf stays -inf
-                    p.rowstat[nrow + row + 32 * j] = d[j] > 0.f ? 1.f / d[j] : 0.f;
+                    p.rowstat[nrow + row + 32 * j] = d[j];
                 }
             };
             if (PAIR) {
@@ -477,9 +481,9 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
                     const int g = dd.x / p.sc.n_pair, j = dd.x % p.sc.n_pair, e0 = dd.y, e1 = dd.z;
                     if (e0 == e1) continue;
                     const int nrb = 2 * j + 1 < p.sc.n_rb ? 2 : 1;
-                    float m0[2], d0[2], m1[2], d1[2];
+                    float m0[4], d0[4], m1[4], d1[4];
 #pragma unroll
-                    for (int u = 0; u < 2; ++u) { m0[u] = m1[u] = -INFINITY; d0[u] = d1[u] = 0.f; }
+                    for (int u = 0; u < 4; ++u) { m0[u] = m1[u] = -INFINITY; d0[u] = d1[u] = 0.f; }
                     for (int e = e0; e < e1; e += NSUB) {
                         int hb = 0;  // union of the sub-tiles' half bits: bits 0-1 row-block 0, 2-3 row-block 1
 #pragma unroll
@@ -495,9 +499,9 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
                 for (ItemWalk iw(p, it_begin, it_end); iw.more();) {
                     const ItemInfo I = iw.next();
                     if (I.t0 == I.t1) continue;
-                    float m[2], d[2];
+                    float m[4], d[4];
 #pragma unroll
-                    for (int u = 0; u < 2; ++u) { m[u] = -INFINITY; d[u] = 0.f; }
+                    for (int u = 0; u < 4; ++u) { m[u] = -INFINITY; d[u] = 0.f; }
                     for (int t = I.t0; t < I.t1; t += NSUB) merge(m, d);
                     flush(I.g, I.rb, m, d);
                 }

@@ -222,7 +222,8 @@ __global__ void __launch_bounds__(G2<D, T>::THREADS, 1) tc_gemm2(const __grid_co
     } else if (warp == 2) {
         if (RS) {
             // -------------------------------------------------------------- row statistics of the
-            // IR merged in GEMM1: (m, 1/d) of the item's 128 rows into the ring (lane: rows l + 32 j)
+            // IR merged in GEMM1: the two partials of each of the item's 128 rows merged into (m, 1/d)
+            // in the ring (lane: rows l + 32 j)
             int si = 0;
             uint32_t sph = 0;
             const int64_t nrow = (int64_t)p.B * p.H * p.S;
@@ -232,9 +233,14 @@ __global__ void __launch_bounds__(G2<D, T>::THREADS, 1) tc_gemm2(const __grid_co
                 const int64_t row = (int64_t)I.g * p.S + I.rb * kRowBlock + lane;
                 float mv[4], iv[4];
 #pragma unroll
-                for (int j = 0; j < 4; ++j) {
-                    mv[j] = __ldcg(p.rowstat + row + 32 * j);
-                    iv[j] = __ldcg(p.rowstat + nrow + row + 32 * j);
+                for (int j = 0; j < 4; ++j) {  // GEMM1's two IR warps' partials (m_w, d_w) of the row
+                    const float ma = __ldcg(p.rowstat + row + 32 * j), da = __ldcg(p.rowstat + nrow + row + 32 * j);
+                    const float mb = __ldcg(p.rowstat + 2 * nrow + row + 32 * j);
+                    const float db = __ldcg(p.rowstat + 3 * nrow + row + 32 * j);
+                    const float m = fmaxf(ma, mb);  // m = max_w m_w, d = sum_w e^{m_w - m} d_w
+                    const float d = m == -INFINITY ? 0.f : da * __expf(ma - m) + db * __expf(mb - m);
+                    mv[j] = m;
+                    iv[j] = d > 0.f ? 1.f / d : 0.f;
                 }
                 DW_WAIT(&st_empty[si], sph ^ 1, 0);
                 float* ms = stats + si * 2 * kRowBlock;

@@ -75,7 +75,7 @@ struct Params {
     float* mprime;
     float* dprime;
     float* rprime;
-    float* rowstat;    // IR_IN_GEMM1: per query row m (natural log) at [0, BHS), 1/d at [BHS, 2 BHS)
+    float* rowstat;    // IR_IN_GEMM1: [2 partials][m (natural log) | d][B*H*S] per query row
 };
 
 __host__ __device__ inline int lh_of(const DevSched& s, int g, int H)

@@ -146,9 +146,9 @@ def test_workspace_closed_form_dense(T):
     assert info["n_slots"] * 128 == Bb * H * S * (S // T)  # L N_sv H
     assert info["off_mprime"] >= L2H * 2
     assert info["total_bytes"] >= L2H * 2 + 3 * 4 * Bb * H * S * (S // T)
-    # per-row (m, 1/d) of the default mode (IR in GEMM1): 8 bytes per query row, after r'
+    # two partial (m, d) per query row of the default mode (IR in GEMM1): 16 bytes per row, after r'
     assert info["off_rowstat"] >= info["off_rprime"] + 4 * Bb * H * S * (S // T)
-    assert info["total_bytes"] >= info["off_rowstat"] + 8 * Bb * H * S
+    assert info["total_bytes"] >= info["off_rowstat"] + 16 * Bb * H * S
     unf = sr.workspace_info(sr.dense_mask(None), Bb, H, S, D, sr.SR_F16, tile_n=T, fused=False)
     assert unf["off_p"] >= L2H * 2 and unf["total_bytes"] >= 2 * L2H * 2
 

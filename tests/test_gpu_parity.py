@@ -242,7 +242,7 @@ def test_intermediates_match_recomposed_oracle():
 
 @pytest.mark.parametrize("T", [64, 128])
 def test_row_statistics_ir_in_gemm1(T):
-    """Default mode (IR in GEMM1): the per-row (m, 1/d) GEMM1's IR warps write vs the oracle's Eq. (2) values:
+    """Default mode (IR in GEMM1): the per-row partial (m, d) GEMM1's two IR warps write vs the oracle's Eq. (2) values:
     m = max_k m'_k, and 1/d = max_k r'_k (r'_k = e^{m'_k - m}/d is 1/d on the tile holding the max)."""
     B, H, S, D = 2, 2, 384, 64
     t, q, k, v = qkv(B, H, S, D, "f16", seed=4)
@@ -256,12 +256,17 @@ def test_row_statistics_ir_in_gemm1(T):
     o_ref, mp_ref, dp_ref, rp_ref = oracle.recomposed(t.q64, t.k64, t.v64, 0.125, T, om)
     assert_close(o.double().cpu().numpy(), o_ref, "f16", what="ir_in_gemm1 output")
     n = B * H * S
-    rs = ws[info["off_rowstat"]:].view(torch.float32)[:2 * n].cpu().numpy().reshape(2, B * H, S)
+    rs = ws[info["off_rowstat"]:].view(torch.float32)[:4 * n].cpu().numpy().reshape(4, B * H, S).astype(np.float64)
     with np.errstate(invalid="ignore"):
         m_ref = mp_ref.max(axis=1)  # [BH, S] over the row's sub-vectors
         invd_ref = rp_ref.max(axis=1)
-    np.testing.assert_allclose(rs[0], m_ref, atol=2e-5)
-    np.testing.assert_allclose(rs[1], invd_ref, rtol=2e-3)
+        # the two IR warps' partials (m_a, d_a), (m_b, d_b) of each row: their maximum is the row's m,
+        # and d_a e^{m_a - m} + d_b e^{m_b - m} its d
+        m = np.maximum(rs[0], rs[2])
+        d = rs[1] * np.exp(np.where(rs[0] == -np.inf, -np.inf, rs[0] - m)) + \
+            rs[3] * np.exp(np.where(rs[2] == -np.inf, -np.inf, rs[2] - m))
+    np.testing.assert_allclose(m, m_ref, atol=2e-5)
+    np.testing.assert_allclose(1.0 / d, invd_ref, rtol=2e-3)
 
 
 def test_T64_equals_T128():
