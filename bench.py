@@ -37,6 +37,7 @@ import workloads as W  # noqa: E402
 
 METRIC = json.load(open(os.path.join(ROOT, "BASELINE.json")))["metric"]
 FLUSH_BYTES = 256 << 20
+SPIN_CYCLES = 400_000  # ~0.2 ms at 1.97 GHz: device-side head start for the host enqueue (timed())
 
 
 def describe(cfg):
@@ -176,6 +177,10 @@ def timed(torch, fn, steps, warmup, flush, per_step_pre=None):
             flush[1].sum()  # ... then read another 256 MiB so L2 starts the step clean, not dirty
         if per_step_pre:
             per_step_pre()
+        # keep the GPU busy (outside the timed region) while the host enqueues the step, so host-side
+        # launch latency (ctypes marshalling, the clock-sampling thread) never shows up as idle device
+        # time between the two events
+        torch.cuda._sleep(SPIN_CYCLES)
         a = torch.cuda.Event(enable_timing=True)
         b = torch.cuda.Event(enable_timing=True)
         a.record()

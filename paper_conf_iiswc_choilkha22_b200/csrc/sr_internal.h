@@ -10,6 +10,7 @@
 #pragma once
 #include <cstddef>
 #include <cstdint>
+#include <cstdlib>
 
 #include <cuda_runtime.h>
 
@@ -113,7 +114,8 @@ inline cudaError_t launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, siz
     attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
     attr[0].val.programmaticStreamSerializationAllowed = 1;
     cfg.attrs = attr;
-    cfg.numAttrs = 1;
+    static const bool no_pdl = getenv("SR_NO_PDL") != nullptr;  // experiments: plain stream order
+    cfg.numAttrs = no_pdl ? 0 : 1;
     cudaError_t e = cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
     ++*nlaunch;
     return e != cudaSuccess ? e : cudaGetLastError();

@@ -1,0 +1,29 @@
+"""Time a config's layer in several modes back to back (L2 flushed before every step):
+    python tools/time_modes.py CFG [steps]   -> one line per mode, device ms per layer"""
+import os
+import statistics
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch  # noqa: E402
+
+import paper_conf_iiswc_choilkha22_b200 as sr  # noqa: E402
+import workloads as W  # noqa: E402
+from bench import FLUSH_BYTES, Layer, timed  # noqa: E402
+
+idx = int(sys.argv[1])
+K = int(sys.argv[2]) if len(sys.argv) > 2 else 30
+cfg = W.config(idx)
+dev = torch.device("cuda", 0)
+flush = (torch.empty(FLUSH_BYTES, dtype=torch.uint8, device=dev), torch.ones(FLUSH_BYTES // 4, device=dev))
+L = Layer(cfg, dev, cfg.idx, sr, torch)
+modes = {"default": {}, "fused_ir": {"fuse_ir": True}, "ir_kernel": {"ir_kernel": True},
+         "g1_only": {"stages": 1}, "g2_only": {"stages": 4}}
+out = []
+for rep in range(2):
+    for name, kw in modes.items():
+        L.run()
+        L.run(**kw)
+        ms = statistics.median(timed(torch, lambda: L.run(**kw), K, 3, flush))
+        out.append(f"{os.environ.get('TAG', '')} C{idx} rep{rep} {name:10s} {ms * 1e3:8.2f} us")
+print("\n".join(out))
