@@ -134,6 +134,12 @@ def make_qkv(B, H, S, D, dtype, seed_base: int = 0, heads: Optional[slice] = Non
     return Tensors(dtype=dtype, **out)
 
 
+def make_dout(B, H, S, D, dtype, seed_base: int = 0):
+    """Seeded N(0,1) upstream gradient dE/dO (training backward, NEXT-4), rounded to ``dtype``;
+    seed 4000 + seed_base.  Returns (storage array, fp64 upcast)."""
+    return round_to_dtype(normal((B, H, S, D), 4000 + seed_base), dtype)
+
+
 def config_tensors(cfg: Config) -> Tensors:
     return make_qkv(cfg.B, cfg.H, cfg.S, cfg.D, cfg.dtype, seed_base=cfg.idx)
 
