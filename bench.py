@@ -114,6 +114,21 @@ def alg_bytes_ir_in_gemm1(cfg, stored, T):
             "gs_gemm2": 2 * stored + 4 * rows_tiles + 8 * rows + 2 * bhsd * e}
 
 
+def alg_bytes_bwd(cfg, stored, T):
+    """Training backward (NEXT-4, include/sr_mha.h sr_mha_*_bwd), algorithmic HBM bytes per kernel:
+    X' is read twice (dS' kernel, dV kernel), dS' written once and read twice (dQ, dK); the dense
+    operands once each; per (row, tile) m' read and r' written then read; per row the statistics."""
+    e = 2
+    bhsd = cfg.BH * cfg.S * cfg.D
+    rt = stored / T
+    rows = cfg.BH * cfg.S
+    return {"prep": 2 * bhsd * e + 28 * rows,
+            "ds": 2 * bhsd * e + 2 * stored + 4 * rt + 12 * rows + 2 * stored + 4 * rt,
+            "dq": 2 * stored + 2 * bhsd * e,
+            "dk": 2 * stored + 2 * bhsd * e,
+            "dv": 2 * stored + 4 * rt + 2 * bhsd * e}
+
+
 def flops(cfg, stored):
     return 4.0 * cfg.D * stored  # two GEMMs, 2 flops per MAC, over stored score elements
 
@@ -159,6 +174,34 @@ class Layer:
                                      sd=True)
             self.ws["sd"] = torch.empty(info["total_bytes"], dtype=torch.uint8, device=device)
         self.n_tiles, self.stored = sr.schedule_stats(self.mask, cfg.B, cfg.H, cfg.S, causal=cfg.causal, tile_n=tile_n)
+
+    def setup_train(self, seed_base):
+        """Training (NEXT-4): dE/dO, gradient buffers and an SR_WS_TRAIN workspace."""
+        cfg, torch, sr = self.cfg, self.torch, self.sr
+        do_s, _ = W.make_dout(cfg.B, cfg.H, cfg.S, cfg.D, cfg.dtype, seed_base=seed_base)
+        if cfg.dtype == "bf16":
+            self.dout = torch.from_numpy(do_s.view(np.int16).copy()).view(torch.bfloat16).to(self.out.device)
+        else:
+            self.dout = torch.from_numpy(np.ascontiguousarray(do_s)).to(self.out.device)
+        info = sr.workspace_info(self.mask, cfg.B, cfg.H, cfg.S, cfg.D, sr.dtype_code(self.dout.dtype),
+                                 causal=cfg.causal, tile_n=self.tile_n, train=True)
+        self.ws_train = torch.empty(info["total_bytes"], dtype=torch.uint8, device=self.out.device)
+        self.grads = [torch.empty_like(self.out) for _ in range(3)]
+
+    def fwd_train(self):
+        d = self.dev
+        return self.sr.call(self.mask, d["q"], d["k"], d["v"], out=self.out, workspace=self.ws_train,
+                            tile_n=self.tile_n, **self.kw)
+
+    def bwd(self, stages=0):
+        d = self.dev
+        dq, dk, dv = self.grads
+        return self.sr.call_bwd(self.mask, d["q"], d["k"], d["v"], self.out, self.dout, workspace=self.ws_train,
+                                dq=dq, dk=dk, dv=dv, stages=stages, tile_n=self.tile_n, **self.kw)
+
+    def train_step(self):
+        self.fwd_train()
+        self.bwd()
 
     def run(self, fused=True, stages=0, q=None, k=None, v=None, fuse_ir=False, sd=False, ir_kernel=False):
         d = self.dev
@@ -291,6 +334,26 @@ def gpu_arm(args, rank, world, local_rank):
             kern_unf[name] = {"us": round(t * 1e3, 3), "alg_bytes": int(unf_b[name]),
                               "GB/s": round(unf_b[name] / (t * 1e-3) / 1e9, 1)}
 
+    # ---- training: forward + backward of the layer on one SR_WS_TRAIN workspace
+    train = None
+    if cfg.dtype != "f32":
+        L.setup_train(cfg.idx + 1000 * rank)
+        L.train_step()
+        ms_tr = dist_max(torch, statistics.mean(timed(torch, L.train_step, K, Wm, flush)), world)
+        ms_bw = dist_max(torch, statistics.mean(timed(torch, L.bwd, K, Wm, flush)), world)
+        bb = alg_bytes_bwd(cfg, L.stored, L.T)
+        kern_bw = {}
+        for name, bit, keys in (("prep_ds", 1, ("prep", "ds")), ("dq", 2, ("dq",)), ("dk_dv", 4, ("dk", "dv"))):
+            t = statistics.mean(timed(torch, lambda b=bit: L.bwd(stages=b), K, Wm, flush))
+            nb = sum(bb[k_] for k_ in keys)
+            kern_bw[name] = {"us": round(t * 1e3, 3), "alg_bytes": int(nb), "GB/s": round(nb / (t * 1e-3) / 1e9, 1)}
+        train = {"what": "training step = forward (default path) + backward (sr_mha_*_bwd: row statistics, "
+                         "dS' = scale*y*(dO V^T - delta) with y = X' r' recomposed per tile (Eq. 3), dQ = dS' K, "
+                         "dK = dS'^T Q, dV = y^T dO); L2 flushed before every step",
+                 "fwd_bwd_per_s": round(world * 1e3 / ms_tr, 2), "fwd_bwd_ms": round(ms_tr, 5),
+                 "bwd_ms": round(ms_bw, 5), "alg_bytes_bwd": int(sum(bb.values())),
+                 "bwd_hbm_GBps": round(sum(bb.values()) / (ms_bw * 1e-3) / 1e9, 1), "kernels": kern_bw}
+
     # ---- end to end through the public API: pinned host -> device, layer, device -> host
     h2d = sum(L.host[n].numel() * L.host[n].element_size() for n in ("q", "k", "v"))
     d2h = L.out.numel() * L.out.element_size()
@@ -334,6 +397,14 @@ def gpu_arm(args, rank, world, local_rank):
                 L2.run(ir_kernel=True)
                 tg = statistics.mean(timed(torch, lambda: L2.run(ir_kernel=True), 10, 3, flush))
                 ent["ir_kernel_layers_per_s"] = round(1e3 / tg, 1)
+            if c2.dtype != "f32":
+                L2.setup_train(c2.idx)
+                L2.train_step()
+                tt = statistics.mean(timed(torch, L2.train_step, 10, 3, flush))
+                tb = statistics.mean(timed(torch, L2.bwd, 10, 3, flush))
+                bb2 = alg_bytes_bwd(c2, L2.stored, L2.T)
+                ent.update({"train_fwd_bwd_ms": round(tt, 4), "bwd_ms": round(tb, 4),
+                            "bwd_hbm_GBps": round(sum(bb2.values()) / (tb * 1e-3) / 1e9, 1)})
             others[f"C{c2.idx}"] = ent
             del L2
             torch.cuda.empty_cache()
@@ -387,6 +458,7 @@ def gpu_arm(args, rank, world, local_rank):
         "e2e": {"value": round(world * 1e3 / ms_e2e, 2), "unit": "layers/s", "h2d_bytes_per_step": int(h2d),
                 "d2h_bytes_per_step": int(d2h), "ms_per_step": round(ms_e2e, 5)},
         "gpu_launches": int(launches),
+        "training": train,
         "clocks": clocks,
     }
     if others:

@@ -151,6 +151,44 @@ sr_status sr_mha_sliding_window_unfused(const void* q, const void* k, const void
                                         int B, int H, int S, int D, float scale,
                                         const sr_window* win, int causal, const sr_exec* ex);
 
+/* Training backward (Sec. 6).  Given the upstream gradient
+ * dout = dE/dO, computes dq = dE/dQ, dk = dE/dK, dv = dE/dV of the same layer, using only what the
+ * forward left in the workspace -- the unnormalised X' tiles, m' and the per-row statistics --
+ * never the softmax input x (the paper's argument: Eq. (3) expresses dE/dx through y alone):
+ *
+ *   P    = X' * r'_k,  r'_k = e^{m'_k - m} / d          (Global Scaling, recomputed per tile)
+ *   dP   = dO V^T                                         (tensor cores, dE/dy)
+ *   dS'  = scale * P (dP - delta),  delta_i = sum_d dO_id O_id      (Eq. 3 row form: dE/dx_k =
+ *          y_k (dE/dy_k - sum_i dE/dy_i y_i), and sum_j P_ij dP_ij = dO_i . O_i)
+ *   dq   = dS' K,   dk = dS'^T Q,   dv = P^T dO          (tensor cores)
+ *
+ * Contract: the call must follow a forward call of the SAME entry point with the same q, k, v,
+ * shape, mask / layout, causal, tile_n, in_dtype and out_dtype, in the default mode (flags 0: the
+ * IR merged in GEMM1 -- the only mode that leaves per-row statistics), on the same workspace,
+ * sized with sr_workspace_bytes(entry, SR_WS_TRAIN, ...).  `out` is that forward's output
+ * (out_dtype).  dout: DEVICE, [B][H][S][D], in_dtype.  dq, dk, dv: DEVICE, [B][H][S][D],
+ * out_dtype, fully overwritten, must not overlap q, k, v, out, dout or each other.  16-bit
+ * in_dtype only (SR_ERR_UNSUPPORTED for F32).  ex->flags: 0, or SR_RUN_GEMM1 (row statistics +
+ * dS' kernel), SR_RUN_REDUCE (dq kernel), SR_RUN_GEMM2 (dk and dv kernels) for per-kernel timing.
+ * Five launches, stream-ordered, asynchronous; errors as for the forward. */
+sr_status sr_mha_dense_bwd(const void* q, const void* k, const void* v, const void* out, const void* dout,
+                           void* dq, void* dk, void* dv, int B, int H, int S, int D, float scale,
+                           const sr_dense_mask* mask_or_null, int causal, const sr_exec* ex);
+sr_status sr_mha_blocksparse_bwd(const void* q, const void* k, const void* v, const void* out,
+                                 const void* dout, void* dq, void* dk, void* dv, int B, int H, int S,
+                                 int D, float scale, const sr_block_layout* layout, int causal,
+                                 const sr_exec* ex);
+sr_status sr_mha_sliding_window_bwd(const void* q, const void* k, const void* v, const void* out,
+                                    const void* dout, void* dq, void* dk, void* dv, int B, int H,
+                                    int S, int D, float scale, const sr_window* win, int causal,
+                                    const sr_exec* ex);
+
+/* Workspace modes for sr_workspace_bytes / sr_workspace_query (the `fused` argument). */
+#define SR_WS_UNFUSED 0
+#define SR_WS_RECOMPOSED 1
+#define SR_WS_SD 2
+#define SR_WS_TRAIN 3 /* recomposed forward + backward: adds the dS' tiles and bstat */
+
 /* Which entry point a workspace query is for. */
 typedef enum { SR_E_DENSE = 0, SR_E_BLOCKSPARSE = 1, SR_E_WINDOW = 2 } sr_entry;
 
@@ -164,6 +202,8 @@ typedef enum { SR_E_DENSE = 0, SR_E_BLOCKSPARSE = 1, SR_E_WINDOW = 2 } sr_entry;
  *   mprime, dprime, rprime   fp32 [slot id][128 rows]  (m' in natural-log units)
  *   rowstat  fp32 [2][2][B*H*S] (default mode): two partial row statistics per query row, each
  *            m_w (natural-log units) then d_w; the row's m = max_w m_w, d = sum_w e^{m_w - m} d_w
+ *   ds, bstat  SR_WS_TRAIN only (backward): dS' tiles; per-row m, 1/d, delta.  The backward also
+ *            writes r' (rprime) for every listed tile.
  */
 typedef struct {
     int32_t tile_n;           /* T actually used */
@@ -173,11 +213,13 @@ typedef struct {
     size_t off_xprime, off_mprime, off_dprime, off_rprime, off_p;  /* off_p: unfused P region */
     size_t off_rowstat;       /* recomposed: per-row partial (m, d) of the default (IR in GEMM1) mode */
     size_t total_bytes;
+    size_t off_ds;            /* SR_WS_TRAIN: dS' tiles, same slots / layout as X', in_dtype */
+    size_t off_bstat;         /* SR_WS_TRAIN: fp32 [3][B*H*S]: m, 1/d, delta per query row */
 } sr_ws_info;
 
 /* Workspace bytes needed by an entry point; `mask_or_layout` is the same pointer passed to it
  * (sr_dense_mask*, sr_block_layout* or sr_window*; may be NULL for dense).  fused: 1 recomposed
- * (also SR_FUSE_IR), 0 unfused, 2 SD (SR_DECOMPOSE).  Returns 0 on invalid/unsupported arguments
+ * (also SR_FUSE_IR), 0 unfused, 2 SD (SR_DECOMPOSE), 3 training forward + backward (SR_WS_TRAIN).  Returns 0 on invalid/unsupported arguments
  * (see sr_last_error()). */
 size_t sr_workspace_bytes(sr_entry entry, int fused, int B, int H, int S, int D, sr_dtype in_dtype,
                           const void* mask_or_layout, int causal, int tile_n);

@@ -9,7 +9,10 @@ Entry points (same names as the C ABI, PAPER.md L51-L53 semantics):
     mha_dense(q, k, v, scale=None, kv_len=None, causal=False, ...)
     mha_blocksparse(q, k, v, layout, scale=None, causal=False, ...)
     mha_sliding_window(q, k, v, window, n_global, scale=None, causal=False, ...)
-with ``fused=False`` selecting the unfused GEMM -> softmax -> GEMM baseline.
+with ``fused=False`` selecting the unfused GEMM -> softmax -> GEMM baseline, and the training
+backward (§6, Eq. 3) on the forward's workspace:
+    mha_dense_bwd / mha_blocksparse_bwd / mha_sliding_window_bwd (q, k, v, out, dout, ...)
+    AttentionTrain(mask): forward() keeps its workspace for backward()
 """
 from __future__ import annotations
 
@@ -33,7 +36,9 @@ SR_E_DENSE, SR_E_BLOCKSPARSE, SR_E_WINDOW = 0, 1, 2
 EXPORTS = ["sr_mha_dense", "sr_mha_blocksparse", "sr_mha_sliding_window", "sr_mha_dense_unfused",
            "sr_mha_blocksparse_unfused", "sr_mha_sliding_window_unfused", "sr_workspace_bytes",
            "sr_workspace_query", "sr_schedule_stats", "sr_status_string", "sr_last_error",
-           "sr_launch_count", "sr_version"]
+           "sr_launch_count", "sr_version", "sr_mha_dense_bwd", "sr_mha_blocksparse_bwd",
+           "sr_mha_sliding_window_bwd"]
+SR_WS_UNFUSED, SR_WS_RECOMPOSED, SR_WS_SD, SR_WS_TRAIN = 0, 1, 2, 3
 
 
 class SrError(RuntimeError):
@@ -68,7 +73,8 @@ class WsInfo(C.Structure):
     _fields_ = [("tile_n", C.c_int32), ("slots_per_head", C.c_int32), ("n_slots", C.c_int64),
                 ("xprime_elt_bytes", C.c_int32), ("off_xprime", C.c_size_t), ("off_mprime", C.c_size_t),
                 ("off_dprime", C.c_size_t), ("off_rprime", C.c_size_t), ("off_p", C.c_size_t),
-                ("off_rowstat", C.c_size_t), ("total_bytes", C.c_size_t)]
+                ("off_rowstat", C.c_size_t), ("total_bytes", C.c_size_t), ("off_ds", C.c_size_t),
+                ("off_bstat", C.c_size_t)]
 
 
 _lib = None
@@ -88,6 +94,10 @@ def lib():
             sig = [vp, vp, vp, vp, i, i, i, i, f, vp, i, C.POINTER(Exec)]
             for n in EXPORTS[:6]:
                 getattr(L, n).argtypes = sig
+                getattr(L, n).restype = i
+            bsig = [vp, vp, vp, vp, vp, vp, vp, vp, i, i, i, i, f, vp, i, C.POINTER(Exec)]
+            for n in ("sr_mha_dense_bwd", "sr_mha_blocksparse_bwd", "sr_mha_sliding_window_bwd"):
+                getattr(L, n).argtypes = bsig
                 getattr(L, n).restype = i
             L.sr_workspace_bytes.argtypes = [i, i, i, i, i, i, i, vp, i, i]
             L.sr_workspace_bytes.restype = C.c_size_t
@@ -153,9 +163,11 @@ def window_mask(window: int, n_global: int) -> _Mask:
 
 # ----------------------------------------------------------------------------- queries
 
-def workspace_info(mask: _Mask, B, H, S, D, in_dtype: int, causal=False, tile_n=0, fused=True, sd=False) -> dict:
+def workspace_info(mask: _Mask, B, H, S, D, in_dtype: int, causal=False, tile_n=0, fused=True, sd=False,
+                   train=False) -> dict:
     info = WsInfo()
-    _check(lib().sr_workspace_query(mask.entry, 2 if (sd and fused) else int(fused), B, H, S, D, in_dtype,
+    mode = SR_WS_TRAIN if train else (2 if (sd and fused) else int(fused))
+    _check(lib().sr_workspace_query(mask.entry, mode, B, H, S, D, in_dtype,
                                     mask.ptr, int(causal),
                                     int(tile_n), C.byref(info)))
     return {k: getattr(info, k) for k, _ in WsInfo._fields_}
@@ -253,3 +265,79 @@ def mha_blocksparse(q, k, v, layout, *, scale=None, causal=False, **kw):
 
 def mha_sliding_window(q, k, v, window, n_global, *, scale=None, causal=False, **kw):
     return call(window_mask(window, n_global), q, k, v, scale=scale, causal=causal, **kw)
+
+
+# ----------------------------------------------------------------------------- training backward
+
+_BWD = {SR_E_DENSE: "sr_mha_dense_bwd", SR_E_BLOCKSPARSE: "sr_mha_blocksparse_bwd",
+        SR_E_WINDOW: "sr_mha_sliding_window_bwd"}
+
+
+def train_workspace(mask: _Mask, q, causal=False, tile_n=0):
+    """A workspace sized for forward + backward (SR_WS_TRAIN) for q's shape and dtype."""
+    torch = _torch()
+    B, H, S, D = q.shape
+    info = workspace_info(mask, B, H, S, D, dtype_code(q.dtype), causal=causal, tile_n=tile_n, train=True)
+    return torch.empty(info["total_bytes"], dtype=torch.uint8, device=q.device)
+
+
+def call_bwd(mask: _Mask, q, k, v, out, dout, *, workspace, scale=None, causal=False, tile_n=0, dq=None,
+             dk=None, dv=None, stream=None, stages=0):
+    """Backward of the layer that a preceding ``call(..., workspace=workspace)`` (default mode)
+    computed.  out: that forward's output (its dtype is the gradients' dtype); dout: dE/dO in q's
+    dtype.  Returns (dq, dk, dv)."""
+    torch = _torch()
+    for t in (q, k, v, out, dout):
+        if not (t.is_cuda and t.is_contiguous()):
+            raise ValueError("q, k, v, out, dout must be contiguous CUDA tensors")
+    if dout.dtype != q.dtype or dout.shape != q.shape or out.shape != q.shape:
+        raise ValueError("dout must match q's dtype and shape, out q's shape")
+    B, H, S, D = q.shape
+    scale = 1.0 / math.sqrt(D) if scale is None else float(scale)
+    dq = torch.empty_like(out) if dq is None else dq
+    dk = torch.empty_like(out) if dk is None else dk
+    dv = torch.empty_like(out) if dv is None else dv
+    st = torch.cuda.current_stream(q.device).cuda_stream if stream is None else stream
+    ex = Exec(dtype_code(q.dtype), dtype_code(out.dtype), workspace.data_ptr(),
+              workspace.numel() * workspace.element_size(), st, int(tile_n), int(stages))
+    _check(getattr(lib(), _BWD[mask.entry])(q.data_ptr(), k.data_ptr(), v.data_ptr(), out.data_ptr(),
+                                            dout.data_ptr(), dq.data_ptr(), dk.data_ptr(), dv.data_ptr(), B, H, S, D,
+                                            C.c_float(scale), mask.ptr, int(causal), C.byref(ex)))
+    return dq, dk, dv
+
+
+class AttentionTrain:
+    """Forward + backward of one attention layer sharing one SR_WS_TRAIN workspace:
+        layer = AttentionTrain(dense_mask(kv_len), causal=True)
+        o = layer.forward(q, k, v);  dq, dk, dv = layer.backward(dout)"""
+
+    def __init__(self, mask: _Mask, causal=False, scale=None, tile_n=0):
+        self.mask, self.causal, self.scale, self.tile_n = mask, causal, scale, tile_n
+        self.ws = None
+
+    def forward(self, q, k, v, out_dtype=None, out=None):
+        need = workspace_info(self.mask, *q.shape, dtype_code(q.dtype), causal=self.causal, tile_n=self.tile_n,
+                              train=True)["total_bytes"]
+        if self.ws is None or self.ws.numel() < need or self.ws.device != q.device:
+            self.ws = train_workspace(self.mask, q, causal=self.causal, tile_n=self.tile_n)
+        self.saved = (q, k, v)
+        self.out = call(self.mask, q, k, v, scale=self.scale, causal=self.causal, out_dtype=out_dtype,
+                        tile_n=self.tile_n, out=out, workspace=self.ws)
+        return self.out
+
+    def backward(self, dout, **kw):
+        q, k, v = self.saved
+        return call_bwd(self.mask, q, k, v, self.out, dout, workspace=self.ws, scale=self.scale,
+                        causal=self.causal, tile_n=self.tile_n, **kw)
+
+
+def mha_dense_bwd(q, k, v, out, dout, *, workspace, kv_len=None, **kw):
+    return call_bwd(dense_mask(kv_len), q, k, v, out, dout, workspace=workspace, **kw)
+
+
+def mha_blocksparse_bwd(q, k, v, out, dout, layout, *, workspace, **kw):
+    return call_bwd(block_mask(layout), q, k, v, out, dout, workspace=workspace, **kw)
+
+
+def mha_sliding_window_bwd(q, k, v, out, dout, window, n_global, *, workspace, **kw):
+    return call_bwd(window_mask(window, n_global), q, k, v, out, dout, workspace=workspace, **kw)

@@ -6,6 +6,7 @@
 // tiles that hold at least one kept element.  Fully masked tiles (causal upper triangle, padded
 // keys, absent sparse blocks, far-off band) are never computed, stored or read (reading R18).
 #include <algorithm>
+#include <array>
 #include <atomic>
 #include <cmath>
 #include <cstdarg>
@@ -52,6 +53,10 @@ struct HostSched {
     // for 2j+1, 0}; pitems g * n_pair + j grouped per CTA (pcta_ptr).
     int n_pair = 0;
     std::vector<int32_t> pp, pent, pitems, pcta_ptr;
+    // column schedule (training backward, dK / dV): cpp [n_lh][n_cb+1] offsets into cent (4 ints
+    // per entry, see DevSched::cent); citems g * n_cb + c grouped per CTA (ccta_ptr)
+    int n_cb = 0;
+    std::vector<int32_t> cpp, cent, citems, ccta_ptr;
     int slots_per_head = 0;
     int max_rb_tiles = 0;
     int64_t n_tiles = 0;       // over all B*H heads
@@ -196,6 +201,30 @@ sr_status build_sched(const Request& r, HostSched& hs)
     }
     for (int g = 0; g < BH; ++g)
         for (int j = 0; j < hs.n_pair; ++j) hs.pitems.push_back(g * hs.n_pair + j);
+    // column lists (the transpose of the row lists, for dK = dS'^T Q and dV = P^T dO): per 128-key
+    // column block, the row-blocks that list one of its key tiles, ascending
+    hs.n_cb = S / kRowBlock;
+    const int per = kRowBlock / T;  // key tiles per column block
+    hs.cpp.assign((size_t)hs.n_lh * (hs.n_cb + 1), 0);
+    for (int lh = 0; lh < hs.n_lh; ++lh) {
+        const int32_t* tp = &hs.tp[(size_t)lh * (hs.n_rb + 1)];
+        std::vector<std::vector<std::array<int32_t, 4>>> cols(hs.n_cb);
+        for (int rb = 0; rb < hs.n_rb; ++rb)
+            for (int t = tp[rb]; t < tp[rb + 1]; ++t) {
+                const int kt = tinfo_kt(hs.tinfo[t]), c = kt / per, u = kt % per;
+                auto& L = cols[c];
+                if (L.empty() || (L.back()[0] & 0xFFFF) != rb) L.push_back({rb, -1, -1, 0});
+                L.back()[0] |= tinfo_half(hs.tinfo[t]) << (16 + 2 * u);
+                L.back()[1 + u] = t;
+            }
+        hs.cpp[(size_t)lh * (hs.n_cb + 1)] = (int32_t)(hs.cent.size() / 4);
+        for (int c = 0; c < hs.n_cb; ++c) {
+            for (auto& e : cols[c]) hs.cent.insert(hs.cent.end(), e.begin(), e.end());
+            hs.cpp[(size_t)lh * (hs.n_cb + 1) + c + 1] = (int32_t)(hs.cent.size() / 4);
+        }
+    }
+    for (int g = 0; g < BH; ++g)
+        for (int c = 0; c < hs.n_cb; ++c) hs.citems.push_back(g * hs.n_cb + c);
     return SR_OK;
 }
 
@@ -352,6 +381,13 @@ void lpt_assign(HostSched& h, int n_cta)
         pcost[i] = 2 * (int64_t)(tp[rb1] - tp[2 * j]) + 1;
     }
     lpt_assign(h.pitems, pcost, n_cta, h.pcta_ptr);
+    std::vector<int64_t> ccost(h.citems.size());
+    for (size_t i = 0; i < h.citems.size(); ++i) {
+        const int g = h.citems[i] / h.n_cb, c = h.citems[i] % h.n_cb;
+        const int32_t* cp = &h.cpp[(size_t)lh_of_g(g) * (h.n_cb + 1)];
+        ccost[i] = 2 * (int64_t)(cp[c + 1] - cp[c]) + 1;
+    }
+    lpt_assign(h.citems, ccost, n_cta, h.ccta_ptr);
 }
 
 // Host schedule only (no device), used by queries.
@@ -380,7 +416,8 @@ sr_status host_sched(const Request& r, std::shared_ptr<CachedSched>& out, bool n
                n_kv = h.kv_len.size();
         const size_t n_pit = h.pitems.size();
         size_t bytes = sizeof(int32_t) * (4 * n_it + 4 * n_pit + h.pent.size() + 4 + n_tp + n_ti + n_it + n_kv +
-                                          h.cta_ptr.size() + h.pp.size() + h.pcta_ptr.size() + 4);
+                                          h.cta_ptr.size() + h.pp.size() + h.pcta_ptr.size() + 4 +
+                                          4 * h.citems.size() + h.cent.size() + 4 + h.ccta_ptr.size());
         cudaError_t ce = cudaMalloc(&cs->dmem, bytes);
         if (ce != cudaSuccess) return fail(SR_ERR_CUDA, "cudaMalloc(schedule): %s", cudaGetErrorString(ce));
         std::vector<int32_t> blob;
@@ -398,6 +435,16 @@ sr_status host_sched(const Request& r, std::shared_ptr<CachedSched>& out, bool n
             const int32_t* pp = &h.pp[(size_t)lh * (h.n_pair + 1)];
             blob.insert(blob.end(), {w, pp[j], pp[j + 1], h.tp[(size_t)lh * (h.n_rb + 1)]});
         }
+        size_t o_cd = blob.size();  // column item descriptors {g * n_cb + c, e0, e1, tp[lh][0]}
+        for (int32_t w : h.citems) {
+            const int g = w / h.n_cb, c = w % h.n_cb;
+            const int lh = h.lh_mode == LH_ONE ? 0 : (h.lh_mode == LH_BATCH ? g / h.H : g % h.H);
+            const int32_t* cp = &h.cpp[(size_t)lh * (h.n_cb + 1)];
+            blob.insert(blob.end(), {w, cp[c], cp[c + 1], h.tp[(size_t)lh * (h.n_rb + 1)]});
+        }
+        size_t o_ce = blob.size();  // column entries (int4)
+        blob.insert(blob.end(), h.cent.begin(), h.cent.end());
+        if (h.cent.empty()) blob.insert(blob.end(), {0, -1, -1, 0});
         size_t o_pe = blob.size();  // union entries (int4)
         blob.insert(blob.end(), h.pent.begin(), h.pent.end());
         if (h.pent.empty()) blob.insert(blob.end(), {0, -1, -1, 0});
@@ -414,6 +461,8 @@ sr_status host_sched(const Request& r, std::shared_ptr<CachedSched>& out, bool n
         blob.insert(blob.end(), h.cta_ptr.begin(), h.cta_ptr.end());
         size_t o_pcp = blob.size();
         blob.insert(blob.end(), h.pcta_ptr.begin(), h.pcta_ptr.end());
+        size_t o_ccp = blob.size();
+        blob.insert(blob.end(), h.ccta_ptr.begin(), h.ccta_ptr.end());
         ce = cudaMemcpy(cs->dmem, blob.data(), blob.size() * 4, cudaMemcpyHostToDevice);
         if (ce != cudaSuccess) return fail(SR_ERR_CUDA, "cudaMemcpy(schedule): %s", cudaGetErrorString(ce));
         int32_t* base = (int32_t*)cs->dmem;
@@ -436,6 +485,11 @@ sr_status host_sched(const Request& r, std::shared_ptr<CachedSched>& out, bool n
         cs->dev.pcta_ptr = base + o_pcp;
         cs->dev.n_pair = h.n_pair;
         cs->dev.n_pcta = (int)h.pcta_ptr.size() - 1;
+        cs->dev.col_desc = (const int4*)(base + o_cd);
+        cs->dev.cent = (const int4*)(base + o_ce);
+        cs->dev.ccta_ptr = base + o_ccp;
+        cs->dev.n_cb = h.n_cb;
+        cs->dev.n_ccta = (int)h.ccta_ptr.size() - 1;
     }
     g_cache[key] = cs;
     out = cs;
@@ -457,7 +511,8 @@ void ws_layout(const HostSched& h, int B, int H, int in_dtype, int fused, sr_ws_
     size_t o = 0;
     info->off_xprime = o;
     o = align_up(o + (size_t)info->n_slots * tile_bytes, 1024);
-    // fused: 1 recomposed (X' + statistics), 0 unfused (S + P), 2 SD (X' + S/Y + statistics)
+    // fused: 1 recomposed (X' + statistics), 0 unfused (S + P), 2 SD (X' + S/Y + statistics),
+    // 3 training (the recomposed layout, then dS' tiles and the backward's row statistics)
     if (fused == 0 || fused == 2) {
         info->off_p = o; o = align_up(o + (size_t)info->n_slots * tile_bytes, 1024);
     }
@@ -466,6 +521,10 @@ void ws_layout(const HostSched& h, int B, int H, int in_dtype, int fused, sr_ws_
         info->off_dprime = o; o = align_up(o + stat_bytes, 1024);
         info->off_rprime = o; o = align_up(o + stat_bytes, 1024);
         info->off_rowstat = o; o = align_up(o + (size_t)4 * B * H * h.n_rb * kRowBlock * sizeof(float), 1024);
+    }
+    if (fused == 3) {
+        info->off_ds = o; o = align_up(o + (size_t)info->n_slots * tile_bytes, 1024);
+        info->off_bstat = o; o = align_up(o + (size_t)3 * B * H * h.n_rb * kRowBlock * sizeof(float), 1024);
     }
     info->total_bytes = std::max<size_t>(o, 1024);
 }
@@ -564,6 +623,82 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
     return SR_OK;
 }
 
+// Training backward (include/sr_mha.h): validation, then prep -> dS' -> dQ ->
+// dK -> dV on the forward's workspace.
+sr_status run_bwd(sr_entry e, const void* q, const void* k, const void* v, const void* out, const void* dout,
+                  void* dq, void* dk, void* dv, int B, int H, int S, int D, float scale, const void* mask_or_layout,
+                  int causal, const sr_exec* ex)
+{
+    if (!ex) return fail(SR_ERR_INVALID, "exec descriptor is NULL");
+    if (!q || !k || !v || !out || !dout || !dq || !dk || !dv)
+        return fail(SR_ERR_INVALID, "q, k, v, out, dout, dq, dk and dv must be non-NULL");
+    if (!std::isfinite(scale) || !(scale > 0.f)) return fail(SR_ERR_INVALID, "scale must be finite and > 0");
+    if (ex->flags & ~(SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2))
+        return fail(SR_ERR_INVALID, "backward flags must be SR_RUN_* stage bits (got 0x%x)", ex->flags);
+    Request r;
+    sr_status s = check_request(e, B, H, S, D, ex->in_dtype, mask_or_layout, causal, ex->tile_n, r);
+    if (s != SR_OK) return s;
+    if (ex->in_dtype == SR_F32) return fail(SR_ERR_UNSUPPORTED, "the backward runs 16-bit dtypes only");
+    if (ex->out_dtype != ex->in_dtype && ex->out_dtype != SR_F32)
+        return fail(SR_ERR_UNSUPPORTED, "out_dtype must equal in_dtype or be SR_F32");
+    const size_t in_bytes = (size_t)B * H * S * D * dtype_bytes(ex->in_dtype);
+    const size_t out_bytes = (size_t)B * H * S * D * dtype_bytes(ex->out_dtype);
+    const void* ins[5] = {q, k, v, dout, out};
+    const size_t ins_b[5] = {in_bytes, in_bytes, in_bytes, in_bytes, out_bytes};
+    void* gs[3] = {dq, dk, dv};
+    for (int a = 0; a < 3; ++a) {
+        for (int b = 0; b < 5; ++b)
+            if (overlaps(gs[a], out_bytes, ins[b], ins_b[b])) return fail(SR_ERR_INVALID, "a gradient overlaps an input");
+        for (int b = a + 1; b < 3; ++b)
+            if (overlaps(gs[a], out_bytes, gs[b], out_bytes)) return fail(SR_ERR_INVALID, "gradients overlap");
+    }
+    if (((uintptr_t)q | (uintptr_t)k | (uintptr_t)v | (uintptr_t)out | (uintptr_t)dout | (uintptr_t)dq |
+         (uintptr_t)dk | (uintptr_t)dv) & 15)
+        return fail(SR_ERR_INVALID, "all tensors must be 16-byte aligned");
+    std::shared_ptr<CachedSched> cs;
+    s = host_sched(r, cs, false);
+    if (s != SR_OK) return s;
+    sr_ws_info wi;
+    ws_layout(cs->hs, B, H, ex->in_dtype, 3, &wi);
+    if (!ex->workspace || ex->workspace_bytes < wi.total_bytes)
+        return fail(SR_ERR_WORKSPACE, "workspace %zu bytes < required %zu (SR_WS_TRAIN)", ex->workspace_bytes,
+                    wi.total_bytes);
+    if ((uintptr_t)ex->workspace & 255) return fail(SR_ERR_WORKSPACE, "workspace must be 256-byte aligned");
+    s = host_sched(r, cs, true);
+    if (s != SR_OK) return s;
+
+    Params p{};
+    p.q = q; p.k = k; p.v = v; p.out = const_cast<void*>(out);
+    p.B = B; p.H = H; p.S = S; p.D = D; p.T = r.T;
+    p.scale = scale;
+    p.scale_log2 = scale * 1.4426950408889634f;
+    p.causal = r.causal;
+    p.mask_kind = e == SR_E_WINDOW ? MK_WINDOW : (e == SR_E_BLOCKSPARSE ? MK_BLOCK : MK_DENSE);
+    p.win_half = r.window / 2;
+    p.n_global = r.n_global;
+    p.in_dtype = ex->in_dtype;
+    p.out_dtype = ex->out_dtype;
+    p.sc = cs->dev;
+    const int stage_bits = ex->flags & (SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2);
+    p.stages = stage_bits ? stage_bits : (SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2);
+    p.ir_mode = IR_IN_GEMM1;
+    char* ws = (char*)ex->workspace;
+    p.xprime = ws + wi.off_xprime;
+    p.mprime = (float*)(ws + wi.off_mprime);
+    p.dprime = (float*)(ws + wi.off_dprime);
+    p.rprime = (float*)(ws + wi.off_rprime);
+    p.rowstat = (float*)(ws + wi.off_rowstat);
+    p.dout = dout;
+    p.dq = dq; p.dk = dk; p.dv = dv;
+    p.dsbuf = ws + wi.off_ds;
+    p.bstat = (float*)(ws + wi.off_bstat);
+    int64_t nl = 0;
+    cudaError_t ce = launch_tc_bwd(p, (cudaStream_t)ex->stream, &nl);
+    g_launches += nl;
+    if (ce != cudaSuccess) return fail(SR_ERR_CUDA, "kernel launch: %s", cudaGetErrorString(ce));
+    return SR_OK;
+}
+
 }  // namespace
 
 // ================================================================================== C ABI
@@ -606,10 +741,31 @@ sr_status sr_mha_sliding_window_unfused(const void* q, const void* k, const void
     return run(SR_E_WINDOW, 0, q, k, v, out, B, H, S, D, scale, w, causal, ex);
 }
 
+sr_status sr_mha_dense_bwd(const void* q, const void* k, const void* v, const void* out, const void* dout,
+                           void* dq, void* dk, void* dv, int B, int H, int S, int D, float scale,
+                           const sr_dense_mask* m, int causal, const sr_exec* ex)
+{
+    return run_bwd(SR_E_DENSE, q, k, v, out, dout, dq, dk, dv, B, H, S, D, scale, m, causal, ex);
+}
+sr_status sr_mha_blocksparse_bwd(const void* q, const void* k, const void* v, const void* out, const void* dout,
+                                 void* dq, void* dk, void* dv, int B, int H, int S, int D, float scale,
+                                 const sr_block_layout* l, int causal, const sr_exec* ex)
+{
+    return run_bwd(SR_E_BLOCKSPARSE, q, k, v, out, dout, dq, dk, dv, B, H, S, D, scale, l, causal, ex);
+}
+sr_status sr_mha_sliding_window_bwd(const void* q, const void* k, const void* v, const void* out, const void* dout,
+                                    void* dq, void* dk, void* dv, int B, int H, int S, int D, float scale,
+                                    const sr_window* w, int causal, const sr_exec* ex)
+{
+    return run_bwd(SR_E_WINDOW, q, k, v, out, dout, dq, dk, dv, B, H, S, D, scale, w, causal, ex);
+}
+
 sr_status sr_workspace_query(sr_entry e, int fused, int B, int H, int S, int D, sr_dtype in_dtype,
                              const void* mask_or_layout, int causal, int tile_n, sr_ws_info* info)
 {
     if (!info) return fail(SR_ERR_INVALID, "info is NULL");
+    if (fused < 0 || fused > 3) return fail(SR_ERR_INVALID, "workspace mode %d must be 0..3", fused);
+    if (fused == 3 && in_dtype == SR_F32) return fail(SR_ERR_UNSUPPORTED, "the backward runs 16-bit dtypes only");
     Request r;
     sr_status s = check_request(e, B, H, S, D, in_dtype, mask_or_layout, causal, tile_n, r);
     if (s != SR_OK) return s;

@@ -51,6 +51,14 @@ struct DevSched {
     int n_rb, n_lh, lh_mode, slots_per_head, n_items, n_cta;
     int max_rb_tiles;       // longest tile list of one (layout head, row-block)
     int mean_rb_tiles;      // mean tile-list length, rounded up
+    // column schedule (training backward, dK / dV): column items = (head, 128-key column block c),
+    // col_desc[i] = {g * n_cb + c, e0, e1, tp[lh][0]} grouped per CTA by ccta_ptr; cent[e] =
+    // {rb | half bits of key tile a << 16 | of key tile b << 18, tinfo index of a or -1, of b or -1, 0}
+    // with a, b the key tiles 2c, 2c+1 (T = 64) or a = c alone (T = 128), row-blocks ascending
+    const int4* col_desc;
+    const int4* cent;
+    const int32_t* ccta_ptr;
+    int n_cb, n_ccta;
 };
 
 // Everything a kernel needs to know about one call.
@@ -77,6 +85,13 @@ struct Params {
     float* dprime;
     float* rprime;
     float* rowstat;    // IR_IN_GEMM1: [2 partials][m (natural log) | d][B*H*S] per query row
+    // training backward (NEXT-4)
+    const void* dout;  // dE/dO [B,H,S,D], in_dtype
+    void* dq;          // gradients [B,H,S,D], out_dtype
+    void* dk;
+    void* dv;
+    void* dsbuf;       // dS' = scale * dE/dx tiles (in_dtype), same slots and layout as X'
+    float* bstat;      // [3][B*H*S]: per query row m (natural log), 1/d, delta = sum_d dO * O
 };
 
 __host__ __device__ inline int lh_of(const DevSched& s, int g, int H)
@@ -127,5 +142,6 @@ cudaError_t launch_ir(const Params& p, cudaStream_t st, int64_t* nlaunch);
 cudaError_t launch_tc_fused(const Params& p, cudaStream_t st, int64_t* nlaunch);
 cudaError_t launch_tc_unfused(const Params& p, cudaStream_t st, int64_t* nlaunch);
 cudaError_t launch_tc_sd(const Params& p, cudaStream_t st, int64_t* nlaunch);
+cudaError_t launch_tc_bwd(const Params& p, cudaStream_t st, int64_t* nlaunch);
 
 }  // namespace sr

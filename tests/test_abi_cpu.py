@@ -217,3 +217,56 @@ def test_schedule_configs_match_survey():
     assert sr.schedule_stats(sr.window_mask(c5.window, c5.n_global), c5.B, c5.H, c5.S, tile_n=64)[1] == 24 * 674 * 64 * 64
     c2 = W.config(2)
     assert sr.schedule_stats(sr.dense_mask(c2.kv_len), c2.B, c2.H, c2.S)[0] == 12 * 20 * 4
+
+
+# ------------------------------------------------------------------------------ training backward
+
+def _call_bwd(entry_fn="sr_mha_dense_bwd", q=0x10000, k=0x20000000, v=0x40000000, out=0x60000000, dout=0x70000000,
+              dq=0x90000000, dk=0xA0000000, dv=0xB0000000, B_=1, H=1, S=128, D=64, scale=0.125, mask=None, causal=0,
+              in_dt=sr.SR_F16, out_dt=None, ws=0xC0000000, ws_bytes=1 << 40, flags=0, tile_n=0):
+    ex = sr.Exec(in_dt, in_dt if out_dt is None else out_dt, ws, ws_bytes, None, tile_n, flags)
+    return getattr(sr.lib(), entry_fn)(q, k, v, out, dout, dq, dk, dv, B_, H, S, D, C.c_float(scale), mask, causal,
+                                       C.byref(ex))
+
+
+@pytest.mark.parametrize("kw,status", [
+    (dict(dout=0), sr.SR_ERR_INVALID),
+    (dict(dk=0), sr.SR_ERR_INVALID),
+    (dict(dq=0x70000000 + 64), sr.SR_ERR_INVALID),   # dq overlaps dout
+    (dict(dv=0x90000000 + 128), sr.SR_ERR_INVALID),  # dv overlaps dq
+    (dict(dk=0x10000 + 16), sr.SR_ERR_INVALID),      # dk overlaps q
+    (dict(dv=0xB0000008), sr.SR_ERR_INVALID),        # misaligned
+    (dict(in_dt=sr.SR_F32), sr.SR_ERR_UNSUPPORTED),  # backward is 16-bit only
+    (dict(flags=16), sr.SR_ERR_INVALID),             # variants do not apply
+    (dict(scale=0.0), sr.SR_ERR_INVALID),
+    (dict(S=100), sr.SR_ERR_UNSUPPORTED),
+    (dict(ws=0), sr.SR_ERR_WORKSPACE),
+    (dict(ws=0xC0000010), sr.SR_ERR_WORKSPACE),
+])
+def test_backward_argument_errors_before_cuda(kw, status):
+    st = _call_bwd(**kw)
+    assert st == status, (st, sr.last_error())
+    assert sr.last_error()
+
+
+def test_backward_needs_training_workspace():
+    m = sr.dense_mask([300, 17])
+    rec = sr.workspace_info(m, 2, 4, 512, 64, sr.SR_F16, causal=True)
+    tr = sr.workspace_info(m, 2, 4, 512, 64, sr.SR_F16, causal=True, train=True)
+    # the training layout extends the recomposed one: same offsets, then dS' tiles and bstat
+    for key in ("off_xprime", "off_mprime", "off_dprime", "off_rprime", "off_rowstat"):
+        assert tr[key] == rec[key]
+    assert tr["off_ds"] >= rec["total_bytes"]
+    assert tr["off_bstat"] >= tr["off_ds"] + tr["n_slots"] * 128 * tr["tile_n"] * 2
+    assert tr["total_bytes"] >= tr["off_bstat"] + 3 * 4 * 2 * 4 * 512
+    st = _call_bwd(B_=2, H=4, S=512, mask=m.ptr, causal=1, ws_bytes=rec["total_bytes"])
+    assert st == sr.SR_ERR_WORKSPACE
+    assert sr.lib().sr_workspace_bytes(sr.SR_E_DENSE, 3, 1, 1, 128, 64, sr.SR_F32, None, 0, 0) == 0
+    assert sr.lib().sr_workspace_bytes(sr.SR_E_DENSE, 4, 1, 1, 128, 64, sr.SR_F16, None, 0, 0) == 0
+
+
+def test_backward_entry_points_validate_masks():
+    bad = sr.dense_mask([129])
+    assert _call_bwd(mask=bad.ptr) == sr.SR_ERR_INVALID
+    assert _call_bwd("sr_mha_blocksparse_bwd", mask=None) == sr.SR_ERR_INVALID
+    assert _call_bwd("sr_mha_sliding_window_bwd", mask=None) == sr.SR_ERR_INVALID
