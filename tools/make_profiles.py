@@ -33,8 +33,11 @@ def kname(full):
                 return "gs_gemm2"  # default path: (m, 1/d) from GEMM1
             return "gs_gemm2_fused_ir" if len(flags) > 1 and flags[1] else "gs_gemm2_rprime"
         return "gemm2_plain"
+    m = re.search(r"tc_bwd_kv<([^>]*)>", full)
+    if m:
+        return "bwd_dv" if m.group(1).split(",")[-1].strip() in ("true", "1", "(bool)1") else "bwd_dk"
     for k, v in (("ir_kernel", "ir"), ("row_softmax", "softmax"), ("sd_ls_kernel", "sd_ls"),
-                 ("sd_gs_kernel", "sd_gs")):
+                 ("sd_gs_kernel", "sd_gs"), ("tc_bwd_ds", "bwd_ds"), ("bwd_prep", "bwd_prep")):
         if k in full:
             return v
     return None
@@ -105,9 +108,30 @@ def main(rnd):
             e["unfused_dram_bytes"] = int(sum(ours[k][1] for k in unf))
         lines.append(f"DRAM bytes per layer (cold, per-kernel sum): recomposed {e['recomposed_dram_bytes'] / 1e6:.1f} MB"
                      + (f", unfused {e['unfused_dram_bytes'] / 1e6:.1f} MB" if unf else ""))
+        pt = os.path.join(OUT, f"launches_train_c{c}.csv")  # ncu of tools/run_layer.py C train
+        if os.path.exists(pt):
+            o2, a2 = launches(pt)
+            lines += ["", f"# training step (tools/run_layer.py {c} train): forward + backward, cold-cache launches",
+                      f"{'kernel':28s} {'launches':>8s} {'mean us':>10s} {'DRAM rd MB':>11s} {'DRAM wr MB':>11s}"]
+            bw = {}
+            for n in o2:
+                m = a2[n]
+                t = sum(m["gpu__time_duration.sum"]) / len(m["gpu__time_duration.sum"])
+                rd = sum(m["dram__bytes_read.sum"]) / len(m["dram__bytes_read.sum"])
+                wr = sum(m["dram__bytes_write.sum"]) / len(m["dram__bytes_write.sum"])
+                nm = "bwd_dq (gemm2_plain)" if n == "gemm2_plain" else n
+                lines.append(f"{nm:28s} {len(m['gpu__time_duration.sum']):8d} {t / 1e3:10.2f} {rd / 1e6:11.2f} {wr / 1e6:11.2f}")
+                if n in ("bwd_prep", "bwd_ds", "gemm2_plain", "bwd_dk", "bwd_dv"):
+                    bw["bwd_dq" if n == "gemm2_plain" else n] = (t, rd + wr)
+            if bw:
+                tb = sum(v[0] for v in bw.values())
+                lines.append("backward shares: " + ", ".join(f"{k} {v[0] / tb:.1%}" for k, v in bw.items()))
+                lines.append(f"backward DRAM bytes (cold, per-kernel sum): {sum(v[1] for v in bw.values()) / 1e6:.1f} MB")
+                e.update({f"{k}_dram_bytes": int(v[1]) for k, v in bw.items()})
+                e["backward_dram_bytes"] = int(sum(v[1] for v in bw.values()))
         traffic[f"C{c}"] = e
         open(os.path.join(PROF, f"{rnd}_launches_c{c}.txt"), "w").write("\n".join(lines) + "\n")
-        for k in ("tc_gemm1", "tc_gemm2", "ir_kernel", "tc_gemm2_fi"):
+        for k in ("tc_gemm1", "tc_gemm2", "ir_kernel", "tc_gemm2_fi", "tc_bwd_ds", "tc_bwd_dk", "tc_bwd_dv"):
             rep = os.path.join(OUT, f"full_c{c}_{k}.ncu-rep")
             if os.path.exists(rep):
                 s = subprocess.run([sys.executable, os.path.join(ROOT, "tools", "ncu_summary.py"), rep, "25"],

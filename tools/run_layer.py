@@ -1,5 +1,6 @@
 """Run one config's layer a few times (for ncu captures):
-    python tools/run_layer.py CFG [fused|unfused|fused_ir|ir_kernel|sd] [reps]"""
+    python tools/run_layer.py CFG [fused|unfused|fused_ir|ir_kernel|sd|train] [reps]
+(train: forward + training backward on an SR_WS_TRAIN workspace)"""
 import os
 import sys
 
@@ -16,7 +17,12 @@ fused = mode != "unfused"
 reps = int(sys.argv[3]) if len(sys.argv) > 3 else 2
 cfg = W.config(idx)
 L = Layer(cfg, torch.device("cuda", 0), cfg.idx, sr, torch)
+if mode == "train":
+    L.setup_train(cfg.idx)
 for _ in range(reps):
-    L.run(fused=fused, fuse_ir=mode == "fused_ir", sd=mode == "sd", ir_kernel=mode == "ir_kernel")
+    if mode == "train":
+        L.train_step()
+    else:
+        L.run(fused=fused, fuse_ir=mode == "fused_ir", sd=mode == "sd", ir_kernel=mode == "ir_kernel")
 torch.cuda.synchronize()
 print("ok", cfg.name, mode)
