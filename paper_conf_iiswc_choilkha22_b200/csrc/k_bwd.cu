@@ -167,6 +167,7 @@ __global__ void __launch_bounds__(384, 1)
         reg_dealloc<56>();  // 4 warps x 32 x (168 - 56) = 8 warps x 32 x (224 - 168)
         if (warp == 0) {
             // ------------------------------------------------------------------ dO + V producer
+            const uint64_t pol_v = policy_evict_last();  // V is re-read by every row-block of its head
             int qi = 0, ks = 0;
             uint32_t qph = 0, kph = 0;
             for (ItemWalk iw(p, it_begin, it_end); iw.more();) {
@@ -191,8 +192,8 @@ __global__ void __launch_bounds__(384, 1)
                         mbar_arrive_expect_tx(&k_full[ks], nsub * T * D * 2);
                         for (int s = 0; s < nsub; ++s)
                             for (int h = 0; h < D / 64; ++h)
-                                tma_load_2d(smem + C::OFF_K + ks * C::KB + h * (kMWB * 128) + s * (T * 128), &tmV,
-                                            h * 64, I.g * p.S + tinfo_kt(w[s]) * T, &k_full[ks]);
+                                tma_load_2d_hint(smem + C::OFF_K + ks * C::KB + h * (kMWB * 128) + s * (T * 128), &tmV,
+                                                 h * 64, I.g * p.S + tinfo_kt(w[s]) * T, &k_full[ks], pol_v);
                     }
                     __syncwarp();
                     if (++ks == C::NK) { ks = 0; kph ^= 1; }
@@ -200,6 +201,7 @@ __global__ void __launch_bounds__(384, 1)
             }
         } else if (warp == 3) {
             // ------------------------------------------------------------------ X' + m' producer
+            const uint64_t pol_x = policy_evict_first();  // X' is streamed
             int n = 0;  // macro tile counter, as the MMA warp and the epilogue count them
             for (ItemWalk iw(p, it_begin, it_end); iw.more();) {
                 const ItemInfo I = iw.next();
@@ -222,10 +224,10 @@ __global__ void __launch_bounds__(384, 1)
                         for (int u = 0; u < nsub; ++u) {
                             for (int ch = 0; ch < T / 64; ++ch) {
                                 const int o = u * XS + ch * (kRowBlock * 128);
-                                if (hv[u] == 3) bulk_load(st + o, src + o, kRowBlock * 128, &x_full[xs]);
+                                if (hv[u] == 3) bulk_load_hint(st + o, src + o, kRowBlock * 128, &x_full[xs], pol_x);
                                 else {
                                     const int o2 = o + (hv[u] == 2 ? kHalf * 128 : 0);
-                                    bulk_load(st + o2, src + o2, kHalf * 128, &x_full[xs]);
+                                    bulk_load_hint(st + o2, src + o2, kHalf * 128, &x_full[xs], pol_x);
                                 }
                             }
                             bulk_load(st + C::XB + u * 512, p.mprime + (I.slot0 + t + u) * kRowBlock, kRowBlock * 4,
@@ -461,6 +463,7 @@ __global__ void __launch_bounds__(384, 1) tc_bwd_kv(const __grid_constant__ CUte
 
     if (warp == 0) {
         // ---------------------------------------------------------------------- producer
+        const uint64_t pol_a = policy_evict_first();  // last read of dS' (dK) / X' (dV)
         int s = 0;
         uint32_t sph = 0;
         for (int it = it_begin; it < it_end; ++it) {
@@ -487,8 +490,8 @@ __global__ void __launch_bounds__(384, 1) tc_bwd_kv(const __grid_constant__ CUte
                         for (int hh = 0; hh < 2; ++hh) {
                             uint8_t* dst = st + ch * (kRowBlock * 128) + hh * (kHalf * 128);
                             if (ti[ch] >= 0 && ((hv[ch] >> hh) & 1))
-                                bulk_load(dst, asrc + (slot0 + ti[ch]) * XS + cc[ch] * (kRowBlock * 128) + hh * (kHalf * 128),
-                                          kHalf * 128, &full[s]);
+                                bulk_load_hint(dst, asrc + (slot0 + ti[ch]) * XS + cc[ch] * (kRowBlock * 128) + hh * (kHalf * 128),
+                                               kHalf * 128, &full[s], pol_a);
                             else
                                 bulk_load(dst, g_zero_half, kHalf * 128, &full[s]);
                         }
@@ -574,6 +577,9 @@ __global__ void __launch_bounds__(384, 1) tc_bwd_kv(const __grid_constant__ CUte
             if (h.flags & KV_END) break;
             const uint32_t st = smem_u32(stage(s));
             const int hv[2] = {h.hv0, h.hv1};
+#ifdef SR_DIAG_BWD_NOTRANSFORM
+            if (false)
+#endif
 #pragma unroll
             for (int ch = 0; ch < 2; ++ch) {
                 const bool valid = (hv[ch] >> myhalf) & 1;
