@@ -15,6 +15,8 @@
  *   kernel 2  GS + GEMM2   the prologue scales each X' tile row by r'_k = e^{m'_k - m} / d (Global
  *                          Scaling, L151) as the tile is loaded, then O += Y V on the tensor cores
  *
+ * By default (16-bit) both kernels' work runs in ONE launch: each CTA does kernel 1 for its rows,
+ * then kernel 2 for the same rows (SR_ONE_KERNEL below); SR_TWO_KERNELS launches them separately.
  * The paper's own layout -- IR as a third, standalone kernel writing r' (L173) -- is the
  * SR_IR_KERNEL variant; SR_FUSE_IR and SR_DECOMPOSE are the other variants (see below).
  *
@@ -99,8 +101,9 @@ typedef struct {
     size_t workspace_bytes;
     void* stream;            /* cudaStream_t; NULL = legacy default stream */
     int32_t tile_n;          /* T = LS sub-vector width = GEMM1 output-tile width:
-                                0 = default (128 on the tensor cores; 64 for block-sparse
-                                layouts and the fp32 path), or 64 / 128 */
+                                0 = default (64 for the recomposed 16-bit path, block-sparse
+                                layouts and the fp32 path; 128 for the unfused baseline and
+                                SR_DECOMPOSE), or 64 / 128 */
     int32_t flags;           /* 0 = run the whole chain.  Otherwise an OR of SR_RUN_* stage bits:
                                 only those kernels are launched, consuming the intermediates an
                                 earlier call with the same arguments left in the workspace (used by
@@ -127,6 +130,15 @@ typedef struct {
  * a standalone IR kernel reduces them per row and writes r'_k = e^{m'_k - m} / d; GS + GEMM2
  * streams r' beside X'.  The only mode that writes d' and r' to the workspace. */
 #define SR_IR_KERNEL 64
+/* The whole recomposed chain in ONE launch -- the DEFAULT of the 16-bit
+ * recomposed path (flags without a variant bit, tile_n 0 or 64): each persistent CTA runs GEMM1 +
+ * LS + IR over its row-blocks, then GS + GEMM2 over the same rows after a CTA barrier (a CTA owns
+ * whole rows, so no other CTA's results are needed).  X' still goes to the workspace and is read
+ * back.  T = 64; stage bits are ignored (one kernel).  SR_ONE_KERNEL requests it explicitly. */
+#define SR_ONE_KERNEL 128
+/* Variant bit: the two-kernel chain GEMM1 + LS + IR -> GS + GEMM2 (the default before the
+ * one-launch kernel; also what tile_n = 128 without a variant bit runs). */
+#define SR_TWO_KERNELS 256
 
 /* Entry points (north star).  Returns SR_OK after enqueueing the kernels on ex->stream. */
 sr_status sr_mha_dense(const void* q, const void* k, const void* v, void* out, int B, int H, int S,

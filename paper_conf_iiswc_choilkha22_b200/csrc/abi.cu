@@ -230,16 +230,19 @@ sr_status build_sched(const Request& r, HostSched& hs)
 
 // ------------------------------------------------------------------------------ validation
 
-int default_T(sr_entry e, int in_dtype)
+int default_T(sr_entry e, int in_dtype, int mode)
 {
     if (in_dtype == SR_F32) return 64;
+    // the recomposed 16-bit default (and training) is the one-launch kernel (k_fused.cu), whose
+    // SPLIT GEMM1 epilogue runs T = 64 sub-vectors in 128-key macro tiles
+    if (mode == 1 || mode == 3) return 64;
     // T = the GEMM1 output-tile width: 128 on the tensor cores; block-sparse
     // layouts fix the sub-vector to the 64-key block (two of them share one 128-key MMA tile)
     return e == SR_E_BLOCKSPARSE ? 64 : 128;
 }
 
 sr_status check_request(sr_entry e, int B, int H, int S, int D, int in_dtype,
-                        const void* mask_or_layout, int causal, int tile_n, Request& r)
+                        const void* mask_or_layout, int causal, int tile_n, Request& r, int mode)
 {
     if (B <= 0 || H <= 0 || S <= 0 || D <= 0)
         return fail(SR_ERR_INVALID, "B, H, S, D must be positive (got %d %d %d %d)", B, H, S, D);
@@ -252,7 +255,7 @@ sr_status check_request(sr_entry e, int B, int H, int S, int D, int in_dtype,
         return fail(SR_ERR_UNSUPPORTED, "too many (head, row-block) items");
     if (tile_n != 0 && tile_n != 64 && tile_n != 128)
         return fail(SR_ERR_UNSUPPORTED, "tile_n=%d must be 0, 64 or 128", tile_n);
-    int T = tile_n ? tile_n : default_T(e, in_dtype);
+    int T = tile_n ? tile_n : default_T(e, in_dtype, mode);
     if (in_dtype == SR_F32 && T != 64) return fail(SR_ERR_UNSUPPORTED, "fp32 path uses T=64");
     r = Request{e, B, H, S, causal ? 1 : 0, T};
     if (e == SR_E_DENSE) {
@@ -542,18 +545,24 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
     if (!ex) return fail(SR_ERR_INVALID, "exec descriptor is NULL");
     if (!q || !k || !v || !out) return fail(SR_ERR_INVALID, "q, k, v and out must be non-NULL");
     if (!std::isfinite(scale) || !(scale > 0.f)) return fail(SR_ERR_INVALID, "scale must be finite and > 0");
-    const int variant_bits = SR_FUSE_IR | SR_DECOMPOSE | SR_IR_KERNEL;
+    const int variant_bits = SR_FUSE_IR | SR_DECOMPOSE | SR_IR_KERNEL | SR_ONE_KERNEL | SR_TWO_KERNELS;
     if (ex->flags & ~(SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2 | variant_bits))
         return fail(SR_ERR_INVALID, "unknown flags 0x%x", ex->flags);
     if ((ex->flags & variant_bits) && (!fused || ex->in_dtype == SR_F32))
         return fail(SR_ERR_UNSUPPORTED, "SR_FUSE_IR / SR_DECOMPOSE / SR_IR_KERNEL apply to the recomposed 16-bit path only");
     {
         const int v = ex->flags & variant_bits;
-        if (v & (v - 1)) return fail(SR_ERR_INVALID, "SR_FUSE_IR, SR_DECOMPOSE and SR_IR_KERNEL are exclusive");
+        if (v & (v - 1)) return fail(SR_ERR_INVALID, "SR_FUSE_IR, SR_DECOMPOSE, SR_IR_KERNEL and SR_ONE_KERNEL are exclusive");
     }
+    // the one-launch kernel: asked for, or the 16-bit recomposed default at T = 64 (any tile_n = 128
+    // request without a variant bit runs the two-kernel chain at T = 128)
+    bool one = (ex->flags & SR_ONE_KERNEL) != 0;
+    if (one && ex->tile_n != 0 && ex->tile_n != 64) return fail(SR_ERR_UNSUPPORTED, "SR_ONE_KERNEL uses T = 64");
+    if (fused == 1 && ex->in_dtype != SR_F32 && !(ex->flags & variant_bits) && (ex->tile_n == 0 || ex->tile_n == 64))
+        one = true;
     if (fused && (ex->flags & SR_DECOMPOSE)) fused = 2;  // SD: workspace mode 2
     Request r;
-    sr_status s = check_request(e, B, H, S, D, ex->in_dtype, mask_or_layout, causal, ex->tile_n, r);
+    sr_status s = check_request(e, B, H, S, D, ex->in_dtype, mask_or_layout, causal, one ? 64 : ex->tile_n, r, fused);
     if (s != SR_OK) return s;
     if (ex->out_dtype != ex->in_dtype && ex->out_dtype != SR_F32)
         return fail(SR_ERR_UNSUPPORTED, "out_dtype must equal in_dtype or be SR_F32");
@@ -613,6 +622,10 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
     cudaError_t ce;
     if (fused == 2) {
         ce = launch_tc_sd(p, st, &nl);
+    } else if (fused && one) {
+        p.g1_pair = 0;
+
+        ce = launch_tc_one(p, st, &nl);
     } else if (fused) {
         ce = ex->in_dtype == SR_F32 ? launch_simt_f32(p, st, &nl) : launch_tc_fused(p, st, &nl);
     } else {
@@ -636,7 +649,7 @@ sr_status run_bwd(sr_entry e, const void* q, const void* k, const void* v, const
     if (ex->flags & ~(SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2))
         return fail(SR_ERR_INVALID, "backward flags must be SR_RUN_* stage bits (got 0x%x)", ex->flags);
     Request r;
-    sr_status s = check_request(e, B, H, S, D, ex->in_dtype, mask_or_layout, causal, ex->tile_n, r);
+    sr_status s = check_request(e, B, H, S, D, ex->in_dtype, mask_or_layout, causal, ex->tile_n, r, 3);
     if (s != SR_OK) return s;
     if (ex->in_dtype == SR_F32) return fail(SR_ERR_UNSUPPORTED, "the backward runs 16-bit dtypes only");
     if (ex->out_dtype != ex->in_dtype && ex->out_dtype != SR_F32)
@@ -767,7 +780,7 @@ sr_status sr_workspace_query(sr_entry e, int fused, int B, int H, int S, int D, 
     if (fused < 0 || fused > 3) return fail(SR_ERR_INVALID, "workspace mode %d must be 0..3", fused);
     if (fused == 3 && in_dtype == SR_F32) return fail(SR_ERR_UNSUPPORTED, "the backward runs 16-bit dtypes only");
     Request r;
-    sr_status s = check_request(e, B, H, S, D, in_dtype, mask_or_layout, causal, tile_n, r);
+    sr_status s = check_request(e, B, H, S, D, in_dtype, mask_or_layout, causal, tile_n, r, fused);
     if (s != SR_OK) return s;
     std::shared_ptr<CachedSched> cs;
     s = host_sched(r, cs, false);
@@ -789,7 +802,7 @@ sr_status sr_schedule_stats(sr_entry e, int B, int H, int S, const void* mask_or
                             int tile_n, int64_t* n_tiles, int64_t* stored_elems)
 {
     Request r;
-    sr_status s = check_request(e, B, H, S, 64, SR_F16, mask_or_layout, causal, tile_n, r);
+    sr_status s = check_request(e, B, H, S, 64, SR_F16, mask_or_layout, causal, tile_n, r, 1);
     if (s != SR_OK) return s;
     std::shared_ptr<CachedSched> cs;
     s = host_sched(r, cs, false);

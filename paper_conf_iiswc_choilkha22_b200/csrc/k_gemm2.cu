@@ -1,37 +1,11 @@
-// k_gemm2.cu -- GEMM2 = Y V with the Global Scaling (GS) sub-layer fused into its prologue
-// ("if element-wise scaling can be performed prior to the MatMul operation by
-// providing r' corresponding to X' allocated to the TB of the MatMul kernel following the GS kernel,
-// the GS kernel can easily be fused with its subsequent MatMul kernel").  GS=false builds the
-// unfused baseline's GEMM2 on the softmax output P.
-//
-// Per item (head, 128-row block) and each of its key sub-tiles (width T):
-//   Y_sub = X'_sub (fp16) * r'_row,sub (fp32), rounded once to the MMA dtype   (GS, in registers)
-//   O    += Y_sub V_sub   (tcgen05.mma kind::f16, A from TMEM, B = V from smem, fp32 in TMEM)
-// Macro tiles: as in GEMM1, MW = 128 keys per step -- with T = 64 two consecutive sub-tiles of the
-// item (any two key blocks) are stacked along the MMA K dimension, each scaled by its own r'.
-//
-// Warp roles (persistent CTA per SM, 512 threads):
-//   warp 0      X' producer: the macro tile's X' sub-tiles (1-D bulk copies of their valid 64-row
-//               halves; the tiles are already in the UMMA SW128 K-major layout and adjacent in HBM) +
-//               their r' + a stage header, into an NX-deep ring, then an END header.  The ring is only
-//               read by the GS warps, so a stage is recycled once they have written it into TMEM.
-//   warp 3      V producer: the macro tile's V blocks (TMA, SW128, MN-major B operand), NV-deep ring
-//   warp 1      MMA issuer: per macro tile (nsub*T)/16 MMAs of 128 x D x 16 into one of two TMEM
-//               O accumulators; walks the item list itself and publishes each item's output rows
-//               (or EMPTY / END) to the epilogue through an O header
-//   warp 2      TMEM allocator (512 columns: 2 x D for O, NA x MW/2 for the A operand ring)
-//   warps 4-11  GS transform: smem X' row -> fp32 x r' -> dtype -> tcgen05.st into TMEM (A operand);
-//               warp w covers TMEM lane quadrant (w-4) % 4 and key half (w-4) / 4 of each macro tile
-//               (two warps per SM sub-partition: with one, GS alone bounded the kernel -- measured)
-//   warps 12-15 epilogue: tcgen05.ld of O rows -> out dtype -> global
-#include "tc_common.cuh"
+// k_gemm2.cu -- GS + GEMM2 kernel and launchers; the device code is in g2_body.cuh.
+#include "g2_body.cuh"
 
 namespace sr {
 
 using namespace ptx;
 
 #ifdef SR_DIAG_WAITS
-__device__ unsigned long long g_diag_g2[20 * (kDW + 1)];
 }  // namespace sr
 extern "C" int sr_diag_read_g2(unsigned long long* out)  // copies [20 warps][kDW + 1] and resets (diagnostic build)
 {
@@ -42,106 +16,14 @@ extern "C" int sr_diag_read_g2(unsigned long long* out)  // copies [20 warps][kD
 namespace sr {
 #endif
 
-constexpr int kMW2 = 128;  // macro tile width (keys per MMA step)
-// L2 policy experiments: X' is streamed once (evict_first), V is re-read by every row-block of its
-// head (evict_last); V_PREFETCH: the V producer warms the macro tile NV ahead in L2
-#ifndef SR_G2_HINTS
-#define SR_G2_HINTS 1
-#endif
-#ifndef SR_G2_VPREFETCH
-#define SR_G2_VPREFETCH 0
-#endif
-
-enum : int { SH_TILE = 1, SH_END = 2, SH_EMPTY = 4, SH_FIRST = 8, SH_LAST = 16 };
-struct G2Hdr {  // X'-stage / O-buffer header
-    int32_t flags, hv0, hv1, nsub, orow_lo, orow_hi, pad0, pad1;
-};
-
-template <int D, int T>
-struct G2 {
-    static constexpr int NSUB = kMW2 / T;
-    static constexpr int XS = kRowBlock * T * 2;     // X' slot (sub-tile)
-    static constexpr int XB = kRowBlock * kMW2 * 2;  // X' part of a stage (macro tile)
-    static constexpr int RB = 2048;                  // r' (NSUB x 512 B) + header, keeps 1 KB alignment
-    static constexpr int XSB = XB + RB;              // X' stage
-    static constexpr int VB = kMW2 * D * 2;          // V stage (macro tile)
-    // split the smem budget: V stages from L2 need less depth than the HBM-bound X' stream
-#ifndef SR_G2_NV64
-#define SR_G2_NV64 3
-#endif
-#ifndef SR_G2_NV128
-#define SR_G2_NV128 2
-#endif
-#ifndef SR_G2_NX
-#define SR_G2_NX 8
-#endif
-    static constexpr int NV = D == 64 ? SR_G2_NV64 : SR_G2_NV128;
-    static constexpr int NX_ = (kSmemMax - 3072 - NV * VB) / XSB;
-    static constexpr int NX = NX_ > SR_G2_NX ? SR_G2_NX : NX_;
-    static_assert(NX >= 2, "smem budget");
-    static constexpr int NO = 2;                             // O accumulators (D cols each)
-    static constexpr int NA_ = (512 - NO * D) / (kMW2 / 2);  // A operand buffers (MW/2 cols each)
-    static constexpr int NA = NA_ > 8 ? 8 : NA_;
-    static_assert(NA >= 2, "tmem budget");
-    static constexpr int OFF_X = 0;
-    static constexpr int OFF_V = NX * XSB;
-    static constexpr int OFF_BAR = OFF_V + NV * VB;
-    static constexpr int NSI = 4;  // fused-IR variant: per-item (m, 1/d) row statistics in flight
-    static constexpr int NBAR = 2 * NX + 2 * NV + 2 * NA + 2 * NO + 2 * NSI;
-    static constexpr int OFF_STATS = OFF_BAR + NBAR * 8;                      // [NSI][2][128] fp32
-    static constexpr int OFF_OHDR = OFF_STATS + NSI * 2 * kRowBlock * 4;
-    static constexpr int OFF_TPTR = OFF_OHDR + NO * (int)sizeof(G2Hdr);
-    static constexpr int SMEM_ = OFF_TPTR + 16 + 1024;
-    static constexpr int SMEM = SMEM_ > 118 * 1024 ? SMEM_ : 118 * 1024;  // 1 CTA/SM (512 TMEM cols)
-#ifndef SR_G2_NGS
-#define SR_G2_NGS 8
-#endif
-    static constexpr int NGS = SR_G2_NGS;       // GS warps: 8 (64 keys each) or 16 (32 keys each)
-    static constexpr int KPW = kMW2 * 4 / NGS;  // keys of a macro tile per GS warp
-    static constexpr int THREADS = 128 + NGS * 32 + 128;
-};
-
-// FI (fused IR): the IR sub-layer runs inside this kernel -- warp 2 reduces each
-// item's m', d' into per-row (m, 1/d) ahead of the GS warps, the X' stages carry m' instead of r',
-// and GS forms r' = e^{m' - m} / d on the fly.  No IR launch, no r' round trip through HBM.
-// RS (default mode, IR in GEMM1): as FI, but GEMM1 already merged the rows, so warp 2 only loads each item's
-// per-row (m, 1/d) -- GEMM2 applies the normalisation 1/d * e^{m' - m} in its prologue.
 template <int D, int T, bool GS, bool FI, bool RS>
 __global__ void __launch_bounds__(G2<D, T>::THREADS, 1) tc_gemm2(const __grid_constant__ CUtensorMap tmV, const Params p)
 {
-    using C = G2<D, T>;
-    constexpr int NSUB = C::NSUB;
     extern __shared__ uint8_t smem_raw[];
     uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
-    uint64_t* bars = (uint64_t*)(smem + C::OFF_BAR);
-    uint64_t* x_full = bars;
-    uint64_t* x_empty = x_full + C::NX;
-    uint64_t* v_full = x_empty + C::NX;
-    uint64_t* v_empty = v_full + C::NV;
-    uint64_t* a_full = v_empty + C::NV;
-    uint64_t* a_empty = a_full + C::NA;
-    uint64_t* o_full = a_empty + C::NA;
-    uint64_t* o_empty = o_full + C::NO;
-    uint64_t* st_full = o_empty + C::NO;  // fused IR: item statistics ready / consumed
-    uint64_t* st_empty = st_full + C::NSI;
-    float* stats = (float*)(smem + C::OFF_STATS);
-    G2Hdr* ohdr = (G2Hdr*)(smem + C::OFF_OHDR);
-    uint32_t* tmem_ptr = (uint32_t*)(smem + C::OFF_TPTR);
-    auto xstage = [&](int s) { return smem + C::OFF_X + s * C::XSB; };
-    auto xhdr = [&](int s) { return (G2Hdr*)(xstage(s) + C::XB + 1024); };
-    auto vstage = [&](int s) { return smem + C::OFF_V + s * C::VB; };
-
+    uint32_t* tmem_ptr = (uint32_t*)(smem + G2<D, T>::OFF_TPTR);
     const int warp = warp_uniform(), lane = threadIdx.x % 32;
-    DW_DECL
-    if (threadIdx.x == 0) {
-        for (int i = 0; i < C::NX; ++i) { mbar_init(&x_full[i], 1); mbar_init(&x_empty[i], C::NGS); }
-        for (int i = 0; i < C::NV; ++i) { mbar_init(&v_full[i], 1); mbar_init(&v_empty[i], 1); }
-        for (int i = 0; i < C::NA; ++i) { mbar_init(&a_full[i], C::NGS); mbar_init(&a_empty[i], 1); }
-        // o_full: O-header arrive + MMA commit; o_empty: one arrive per epilogue warp
-        for (int i = 0; i < C::NO; ++i) { mbar_init(&o_full[i], 2); mbar_init(&o_empty[i], 4); }
-        for (int i = 0; i < C::NSI; ++i) { mbar_init(&st_full[i], 1); mbar_init(&st_empty[i], C::NGS); }
-        fence_mbar_init();
-    }
+    if (threadIdx.x == 0) g2_init<D, T, GS, FI, RS>(smem);
     if (warp == 3 && lane == 0) prefetch_tmap(&tmV);
     if (warp == 2) tmem_alloc(tmem_ptr, 512);
     tc_fence_before();
@@ -152,415 +34,8 @@ __global__ void __launch_bounds__(G2<D, T>::THREADS, 1) tc_gemm2(const __grid_co
     // own prologue, then wait for our producer kernel's results before touching them
     griddep_launch_dependents();
     griddep_wait();
-    const uint32_t tmem_o = tmem_base;              // NO x D columns
-    const uint32_t tmem_a = tmem_base + C::NO * D;  // NA x MW/2 columns
-    // this CTA's items: a contiguous range of the longest-processing-time assignment (host)
-    const int it_begin = __ldg(p.sc.cta_ptr + blockIdx.x), it_end = __ldg(p.sc.cta_ptr + blockIdx.x + 1);
-    const uint8_t* src = (const uint8_t*)(GS ? p.xprime : p.pbuf);
-
-    if (warp == 0) {
-        {
-            // -------------------------------------------------------------- X' producer (whole
-            // warp walks the schedule; one elected lane issues)
-            int s = 0;
-            const uint64_t pol_x = SR_G2_HINTS ? policy_evict_first() : 0;
-            uint32_t sph = 0;
-            for (ItemWalk iw(p, it_begin, it_end); iw.more();) {
-                const ItemInfo I = iw.next();
-                int wn[2];  // schedule words of the next macro tile, prefetched one step ahead
-                for (int u = 0; u < NSUB; ++u) wn[u] = I.t0 + u < I.t1 ? __ldg(p.sc.tinfo + I.t0 + u) : 0;
-                for (int t = I.t0; t < I.t1; t += NSUB) {
-                    const int nsub = min(NSUB, I.t1 - t);
-                    int hv[2] = {tinfo_half(wn[0]), NSUB > 1 ? tinfo_half(wn[1]) : 0};
-                    for (int u = 0; u < NSUB; ++u) wn[u] = t + NSUB + u < I.t1 ? __ldg(p.sc.tinfo + t + NSUB + u) : 0;
-                    uint32_t bytes = GS ? nsub * kRowBlock * 4 : 0;
-#ifndef SR_DIAG2_NOX
-                    for (int u = 0; u < nsub; ++u) bytes += (hv[u] == 3 ? 2 : 1) * (T / 64) * (kHalf * 128);
-#endif
-                    DW_WAIT(&x_empty[s], sph ^ 1, 0);
-                    uint8_t* st = xstage(s);
-                    if (elect_one()) {
-                    *xhdr(s) = G2Hdr{SH_TILE | (t == I.t0 ? SH_FIRST : 0) | (t + NSUB >= I.t1 ? SH_LAST : 0), hv[0],
-                                     hv[1], nsub, 0, 0, 0, 0};
-                    mbar_arrive_expect_tx(&x_full[s], bytes);
-                    const uint8_t* xs = src + (I.slot0 + t) * (int64_t)C::XS;  // sub-tiles t, t+1 are adjacent
-                    auto xload = [&](uint8_t* d, const uint8_t* g, uint32_t n) {
-                        if (SR_G2_HINTS) bulk_load_hint(d, g, n, &x_full[s], pol_x);
-                        else bulk_load(d, g, n, &x_full[s]);
-                    };
-#ifdef SR_DIAG2_NOX
-                    if (false)
-#endif
-                    if (hv[0] == 3 && (nsub == 1 || hv[1] == 3)) {
-                        xload(st, xs, nsub * C::XS);
-                    } else {
-                        for (int u = 0; u < nsub; ++u)
-                            for (int ch = 0; ch < T / 64; ++ch) {
-                                const int o = u * C::XS + ch * (kRowBlock * 128);
-                                if (hv[u] == 3) xload(st + o, xs + o, kRowBlock * 128);
-                                else {
-                                    const int o2 = o + (hv[u] == 2 ? kHalf * 128 : 0);
-                                    xload(st + o2, xs + o2, kHalf * 128);
-                                }
-                            }
-                    }
-                    if (GS)  // r' (or m' with the fused IR) of the sub-tiles' 128 rows rides along
-                        bulk_load(st + C::XB, (FI ? p.mprime : p.rprime) + (I.slot0 + t) * kRowBlock,
-                                  nsub * kRowBlock * 4, &x_full[s]);
-                    }
-                    __syncwarp();
-                    if (++s == C::NX) { s = 0; sph ^= 1; }
-                }
-            }
-            DW_WAIT(&x_empty[s], sph ^ 1, 0);
-            if (elect_one()) {
-                xhdr(s)->flags = SH_END;
-                mbar_arrive(&x_full[s]);
-            }
-            __syncwarp();
-        }
-    } else if (warp == 2) {
-        if (RS) {
-            // -------------------------------------------------------------- row statistics of the
-            // IR merged in GEMM1: the two partials of each of the item's 128 rows merged into (m, 1/d)
-            // in the ring (lane: rows l + 32 j)
-            int si = 0;
-            uint32_t sph = 0;
-            const int64_t nrow = (int64_t)p.B * p.H * p.S;
-            for (ItemWalk iw(p, it_begin, it_end); iw.more();) {
-                const ItemInfo I = iw.next();
-                if (I.t0 == I.t1) continue;
-                const int64_t row = (int64_t)I.g * p.S + I.rb * kRowBlock + lane;
-                float mv[4], iv[4];
-#pragma unroll
-                for (int j = 0; j < 4; ++j) {  // GEMM1's two IR warps' partials (m_w, d_w) of the row
-                    const float ma = __ldcg(p.rowstat + row + 32 * j), da = __ldcg(p.rowstat + nrow + row + 32 * j);
-                    const float mb = __ldcg(p.rowstat + 2 * nrow + row + 32 * j);
-                    const float db = __ldcg(p.rowstat + 3 * nrow + row + 32 * j);
-                    const float m = fmaxf(ma, mb);  // m = max_w m_w, d = sum_w e^{m_w - m} d_w
-                    const float d = m == -INFINITY ? 0.f : da * __expf(ma - m) + db * __expf(mb - m);
-                    mv[j] = m;
-                    iv[j] = d > 0.f ? 1.f / d : 0.f;
-                }
-                DW_WAIT(&st_empty[si], sph ^ 1, 0);
-                float* ms = stats + si * 2 * kRowBlock;
-#pragma unroll
-                for (int j = 0; j < 4; ++j) {
-                    ms[lane + 32 * j] = mv[j];
-                    ms[kRowBlock + lane + 32 * j] = iv[j];
-                }
-                __syncwarp();
-                if (lane == 0) mbar_arrive(&st_full[si]);
-                if (++si == C::NSI) { si = 0; sph ^= 1; }
-            }
-        } else if (FI) {
-            // -------------------------------------------------------------- fused IR (NEXT-2)
-            // Per non-empty item, per row: m = max_k m'_k, d = sum_k e^{m'_k - m} d'_k (PAPER.md
-            // L147), published as (m, 1/d) in a ring of NSI items.  Lane l reduces rows l + 32j.
-            int si = 0;
-            uint32_t sph = 0;
-            for (ItemWalk iw(p, it_begin, it_end); iw.more();) {
-                const ItemInfo I = iw.next();
-                if (I.t0 == I.t1) continue;
-                DW_WAIT(&st_empty[si], sph ^ 1, 0);
-                float* ms = stats + si * 2 * kRowBlock;
-                const float* mp = p.mprime + I.slot0 * kRowBlock + lane;
-                const float* dp = p.dprime + I.slot0 * kRowBlock + lane;
-                float m[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY}, d[4] = {0.f, 0.f, 0.f, 0.f};
-                for (int tb = I.t0; tb < I.t1; tb += 8) {
-                    // one memory round trip per batch: 8 tiles x 4 rows x (m', d') + the tile words
-                    float m8[4][8], d8[4][8];
-                    int w8[8];
-#pragma unroll
-                    for (int u = 0; u < 8; ++u) w8[u] = tb + u < I.t1 ? __ldg(p.sc.tinfo + tb + u) : 0;
-#pragma unroll
-                    for (int u = 0; u < 8; ++u)
-#pragma unroll
-                        for (int j = 0; j < 4; ++j) {
-                            const bool in = tb + u < I.t1;
-                            m8[j][u] = in ? __ldg(mp + (int64_t)(tb + u) * kRowBlock + 32 * j) : -INFINITY;
-                            d8[j][u] = in ? __ldg(dp + (int64_t)(tb + u) * kRowBlock + 32 * j) : 0.f;
-                        }
-#pragma unroll
-                    for (int j = 0; j < 4; ++j) {
-                        const int half = (lane + 32 * j) / kHalf;
-                        float mb = -INFINITY;
-#pragma unroll
-                        for (int u = 0; u < 8; ++u) {
-                            if (!((tinfo_half(w8[u]) >> half) & 1) || tb + u >= I.t1) m8[j][u] = -INFINITY;
-                            mb = fmaxf(mb, m8[j][u]);
-                        }
-                        if (mb == -INFINITY) continue;
-                        const float mn = fmaxf(m[j], mb);
-                        float acc = (m[j] == -INFINITY) ? 0.f : d[j] * __expf(m[j] - mn);
-#pragma unroll
-                        for (int u = 0; u < 8; ++u)
-                            if (m8[j][u] != -INFINITY) acc += d8[j][u] * __expf(m8[j][u] - mn);
-                        m[j] = mn;
-                        d[j] = acc;
-                    }
-                }
-#pragma unroll
-                for (int j = 0; j < 4; ++j) {
-                    ms[lane + 32 * j] = m[j];
-                    ms[kRowBlock + lane + 32 * j] = d[j] > 0.f ? 1.f / d[j] : 0.f;
-                }
-                __syncwarp();
-                if (lane == 0) mbar_arrive(&st_full[si]);
-                if (++si == C::NSI) { si = 0; sph ^= 1; }
-            }
-        }
-    } else if (warp == 3) {
-        {
-            // -------------------------------------------------------------- V producer (whole warp,
-            // one elected lane issues)
-            int s = 0;
-            const uint64_t pol_v = SR_G2_HINTS ? policy_evict_last() : 0;
-            uint32_t sph = 0;
-            for (ItemWalk iw(p, it_begin, it_end); iw.more();) {
-                const ItemInfo I = iw.next();
-                int wn[2];  // schedule words of the next macro tile, prefetched one step ahead
-                for (int u = 0; u < NSUB; ++u) wn[u] = I.t0 + u < I.t1 ? __ldg(p.sc.tinfo + I.t0 + u) : 0;
-                for (int t = I.t0; t < I.t1; t += NSUB) {
-                    const int nsub = min(NSUB, I.t1 - t);
-                    int kt[2] = {tinfo_kt(wn[0]), NSUB > 1 ? tinfo_kt(wn[1]) : 0};
-                    for (int u = 0; u < NSUB; ++u) wn[u] = t + NSUB + u < I.t1 ? __ldg(p.sc.tinfo + t + NSUB + u) : 0;
-                    DW_WAIT(&v_empty[s], sph ^ 1, 0);
-                    if (elect_one()) {
-#ifdef SR_DIAG2_NOV
-                        mbar_arrive(&v_full[s]);
-                        if (false)
-#else
-                        mbar_arrive_expect_tx(&v_full[s], nsub * T * D * 2);
-#endif
-                        for (int u = 0; u < nsub; ++u)
-                            for (int h = 0; h < D / 64; ++h) {
-                                if (SR_G2_HINTS)
-                                    tma_load_2d_hint(vstage(s) + h * (kMW2 * 128) + u * (T * 128), &tmV, h * 64,
-                                                     I.g * p.S + kt[u] * T, &v_full[s], pol_v);
-                                else
-                                    tma_load_2d(vstage(s) + h * (kMW2 * 128) + u * (T * 128), &tmV, h * 64,
-                                                I.g * p.S + kt[u] * T, &v_full[s]);
-                            }
-                        if (SR_G2_VPREFETCH) {  // the macro tile NV steps ahead in this item, into L2
-                            const int tp = t + C::NV * NSUB;
-                            for (int u = 0; u < NSUB; ++u)
-                                if (tp + u < I.t1) {
-                                    const int ktp = tinfo_kt(__ldg(p.sc.tinfo + tp + u));
-                                    for (int h = 0; h < D / 64; ++h) tma_prefetch_2d(&tmV, h * 64, I.g * p.S + ktp * T);
-                                }
-                        }
-                    }
-                    __syncwarp();
-                    if (++s == C::NV) { s = 0; sph ^= 1; }
-                }
-            }
-        }
-    } else if (warp == 1) {
-        {
-            // -------------------------------------------------------------- MMA issuer (whole warp,
-            // one elected lane issues)
-            const uint32_t idesc = idesc_f16(p.in_dtype == DT_BF16 ? 1 : 0, kRowBlock, D, 0, 1);
-            int s = 0, a = 0, o = 0;
-            uint32_t sph = 0, aph = 0, oph = 0;
-            auto post = [&](int flags, int64_t orow, bool second) {  // O header to the epilogue, arrival 1 of 2
-                DW_WAIT(&o_empty[o], oph ^ 1, 2);
-                if (elect_one()) {
-                    ohdr[o] = G2Hdr{flags, 0, 0, 0, (int32_t)(orow & 0xffffffff), (int32_t)(orow >> 32), 0, 0};
-                    mbar_arrive(&o_full[o]);
-                    if (second) mbar_arrive(&o_full[o]);  // no MMA commit will follow
-                }
-                __syncwarp();
-            };
-            auto next_o = [&]() {
-                if (++o == C::NO) { o = 0; oph ^= 1; }
-            };
-            ItemInfo nxt;
-            if (it_begin < it_end) nxt = decode_item(p, it_begin);
-            for (int it = it_begin; it < it_end; ++it) {
-                const ItemInfo I = nxt;
-                if (it + 1 < it_end) nxt = decode_item(p, it + 1);  // prefetch
-                const int64_t orow = (int64_t)I.g * p.S + I.rb * kRowBlock;
-                if (I.t0 == I.t1) {  // no kept key in these rows: the epilogue writes zeros
-                    post(SH_EMPTY, orow, true);
-                    next_o();
-                    continue;
-                }
-                post(SH_TILE, orow, false);
-                const uint32_t d_tmem = tmem_o + o * D;
-                for (int t = I.t0; t < I.t1; t += NSUB) {
-                    const int nk = min(NSUB, I.t1 - t) * (T / 16);  // K steps of 16 keys
-                    DW_WAIT(&v_full[s], sph, 0);
-                    DW_WAIT(&a_full[a], aph, 1);
-                    tc_fence_after();
-                    const uint32_t v_addr = smem_u32(vstage(s));
-                    const uint32_t a_tm = tmem_a + a * (kMW2 / 2);
-                    if (elect_one()) {
-#pragma unroll 8
-                        for (int kk = 0; kk < nk; ++kk) {
-                            // B = V, MN-major SW128: 16 keys per MMA = 2 KB; 64-wide d blocks at LBO = MW*128 B
-                            const uint64_t bd = smem_desc_sw128(v_addr + kk * 2048, kMW2 * 128, 1024);
-                            mma_ts(d_tmem, a_tm + kk * 8, bd, idesc, (t == I.t0 && kk == 0) ? 0u : 1u);
-                        }
-                        mma_commit(&v_empty[s]);
-                        mma_commit(&a_empty[a]);
-                    }
-                    __syncwarp();
-                    if (++s == C::NV) { s = 0; sph ^= 1; }
-                    if (++a == C::NA) { a = 0; aph ^= 1; }
-                }
-                if (elect_one()) mma_commit(&o_full[o]);  // arrival 2 of 2 when the item's MMAs complete
-                __syncwarp();
-                next_o();
-            }
-            post(SH_END, 0, true);
-        }
-    } else if (warp >= 4 && warp < 4 + C::NGS) {
-        // ------------------------------------------------------------------ GS transform
-        const int gq = (warp - 4) % 4, ch = (warp - 4) / 4;  // lane quadrant, key slice (KPW keys)
-        constexpr int KPW = C::KPW;
-        const int r = gq * 32 + lane;
-        const int myhalf = r / kHalf;
-        const uint32_t lane_off = (uint32_t)(gq * 32) << 16;
-        const bool bf = p.in_dtype == DT_BF16;
-        int s = 0, a = 0, si = 0;
-        uint32_t sph = 0, aph = 0, siph = 0;
-        float m_row = 0.f, invd_row = 0.f;  // fused IR: this row's (m, 1/d) for the current item
-        for (;;) {
-            DW_WAIT(&x_full[s], sph, 0);
-            const G2Hdr h = lds_hdr(xhdr(s));
-            if (h.flags & SH_END) break;
-            if (FI && (h.flags & SH_FIRST)) {  // a new item: its row statistics from the IR warp
-                DW_WAIT(&st_full[si], siph, 2);
-                m_row = stats[si * 2 * kRowBlock + r];
-                invd_row = stats[si * 2 * kRowBlock + kRowBlock + r];
-                __syncwarp();
-                if (lane == 0) mbar_arrive(&st_empty[si]);
-                if (++si == C::NSI) { si = 0; siph ^= 1; }
-            }
-            const uint32_t xs_s = smem_u32(xstage(s));
-            const int hvs[2] = {h.hv0, h.hv1};
-            float rr[NSUB];
-#pragma unroll
-            for (int u = 0; u < NSUB; ++u) {
-                const bool valid = u < h.nsub && ((hvs[u] >> myhalf) & 1);
-                rr[u] = valid ? 1.f : 0.f;
-                if (GS && valid) {
-                    const float v = lds_f32(xs_s + C::XB + u * 512 + 4 * r);
-                    if (FI)  // r'_k = e^{m'_k - m} / d  (0 for a fully masked sub-vector)
-                        rr[u] = (v == -INFINITY) ? 0.f : __expf(v - m_row) * invd_row;
-                    else
-                        rr[u] = v;
-                }
-            }
-            // this warp's slice of the X' row (KPW fp16 = KPW/8 chunks of 16 B) into registers first:
-            // the loads overlap the wait for a free A buffer
-            uint4 xv[KPW / 8];
-#ifdef SR_DIAG2_NOGS
-            if (false)
-#endif
-#pragma unroll
-            for (int q = 0; q < KPW / 8; ++q)  // unconditional: issued beside the r' chain (unused if r' = 0)
-                xv[q] = lds128(xs_s + tile_chunk_off(r, ch * (KPW / 8) + q));
-            DW_WAIT(&a_empty[a], aph ^ 1, 1);
-            tc_fence_after();
-            const uint32_t a_tm = tmem_a + lane_off + a * (kMW2 / 2);
-#pragma unroll
-            for (int c2 = 0; c2 < KPW / 32; ++c2) {  // 32 keys -> 16 packed words per tcgen05.st
-                const int c = ch * (KPW / 32) + c2;
-                const int u = (c * 32) / T;   // sub-tile of these keys
-                uint32_t pk[16];
-                if (rr[u] != 0.f) {
-#pragma unroll
-                    for (int q4 = 0; q4 < 4; ++q4) {
-                        const uint4 x = xv[c2 * 4 + q4];
-                        const uint32_t xw[4] = {x.x, x.y, x.z, x.w};
-#pragma unroll
-                        for (int w = 0; w < 4; ++w) {
-                            if (GS) {  // Y = X' * r'  (fp16 X' -> fp32 -> x r' -> dtype, one rounding)
-                                const float2 f = unpack_f16(xw[w]);
-                                float y0, y1;
-                                fmul2(y0, y1, f.x, f.y, rr[u]);
-                                pk[q4 * 4 + w] = bf ? pack_bf16(y0, y1) : pack_f16(y0, y1);
-                            } else {  // P already holds dtype values
-                                pk[q4 * 4 + w] = xw[w];
-                            }
-                        }
-                    }
-                } else {  // absent sub-tile, invalid half (not loaded) or r' = 0: zero rows of A
-#pragma unroll
-                    for (int w = 0; w < 16; ++w) pk[w] = 0u;
-                }
-#ifndef SR_DIAG2_NOGS
-                tmem_st16(a_tm + c * 16, pk);
-#else
-                (void)pk;
-#endif
-            }
-            tmem_wait_st();
-            tc_fence_before();
-            __syncwarp();
-            if (lane == 0) mbar_arrive(&a_full[a]);
-            if (++a == C::NA) { a = 0; aph ^= 1; }
-            // release the X' stage only now: its ld.shared results have been consumed by the tcgen05.st
-            // above.  Arriving right after issuing the loads let the next bulk copy overwrite the stage
-            // while other lanes' loads were still in flight (a real race, seen as 16-lane corruption).
-            if (lane == 0) mbar_arrive(&x_empty[s]);
-            if (++s == C::NX) { s = 0; sph ^= 1; }
-        }
-    } else if (warp >= 4 + C::NGS) {
-        // ------------------------------------------------------------------ output epilogue
-        const int r = (warp % 4) * 32 + lane;
-        const uint32_t lane_off = (uint32_t)((warp % 4) * 32) << 16;
-        int o = 0;
-        uint32_t oph = 0;
-        for (;;) {
-            DW_WAIT(&o_full[o], oph, 0);
-            tc_fence_after();
-            const G2Hdr h = lds_hdr(ohdr + o);
-            if (h.flags & SH_END) break;
-            const int64_t orow = (((int64_t)h.orow_hi << 32) | (uint32_t)h.orow_lo) + r;
-            if (h.flags & SH_EMPTY) {  // no kept key anywhere in these rows: output 0 (reading R9)
-                if (p.out_dtype == DT_F32) {
-                    float4* O = reinterpret_cast<float4*>((float*)p.out + orow * D);
-                    for (int c = 0; c < D / 4; ++c) O[c] = make_float4(0.f, 0.f, 0.f, 0.f);
-                } else {
-                    uint4* O = reinterpret_cast<uint4*>((uint16_t*)p.out + orow * D);
-                    for (int c = 0; c < D / 8; ++c) O[c] = make_uint4(0, 0, 0, 0);
-                }
-            } else {
-                const uint32_t taddr = tmem_o + lane_off + o * D;
-#pragma unroll
-                for (int c = 0; c < D / 32; ++c) {
-                    uint32_t v[32];
-                    tmem_ld32(taddr + c * 32, v);
-                    tmem_wait_ld();
-                    if (p.out_dtype == DT_F32) {
-                        float4* O = reinterpret_cast<float4*>((float*)p.out + orow * D + c * 32);
-#pragma unroll
-                        for (int u = 0; u < 8; ++u)
-                            O[u] = make_float4(__uint_as_float(v[4 * u]), __uint_as_float(v[4 * u + 1]),
-                                               __uint_as_float(v[4 * u + 2]), __uint_as_float(v[4 * u + 3]));
-                    } else {
-                        uint32_t pk[16];
-#pragma unroll
-                        for (int u = 0; u < 16; ++u) {
-                            const float f0 = __uint_as_float(v[2 * u]), f1 = __uint_as_float(v[2 * u + 1]);
-                            pk[u] = p.out_dtype == DT_BF16 ? pack_bf16(f0, f1) : pack_f16(f0, f1);
-                        }
-                        uint4* O = reinterpret_cast<uint4*>((uint16_t*)p.out + orow * D + c * 32);
-#pragma unroll
-                        for (int u = 0; u < 4; ++u) O[u] = make_uint4(pk[4 * u], pk[4 * u + 1], pk[4 * u + 2], pk[4 * u + 3]);
-                    }
-                }
-                tc_fence_before();
-            }
-            __syncwarp();
-            if (lane == 0) mbar_arrive(&o_empty[o]);
-            if (++o == C::NO) { o = 0; oph ^= 1; }
-        }
-    }
-    DW_FLUSH(g_diag_g2);
+    g2_roles<D, T, GS, FI, RS>(tmV, p, smem, tmem_base, __ldg(p.sc.cta_ptr + blockIdx.x),
+                               __ldg(p.sc.cta_ptr + blockIdx.x + 1));
     tc_fence_before();
     __syncthreads();
     if (warp == 2) {

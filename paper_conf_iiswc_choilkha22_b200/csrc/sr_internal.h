@@ -143,5 +143,6 @@ cudaError_t launch_tc_fused(const Params& p, cudaStream_t st, int64_t* nlaunch);
 cudaError_t launch_tc_unfused(const Params& p, cudaStream_t st, int64_t* nlaunch);
 cudaError_t launch_tc_sd(const Params& p, cudaStream_t st, int64_t* nlaunch);
 cudaError_t launch_tc_bwd(const Params& p, cudaStream_t st, int64_t* nlaunch);
+cudaError_t launch_tc_one(const Params& p, cudaStream_t st, int64_t* nlaunch);
 
 }  // namespace sr

@@ -72,7 +72,9 @@ def _call(entry_fn, q=0x10000, k=0x20000000, v=0x40000000, out=0x60000000, B_=1,
     (dict(out=0x10000 + 64), sr.SR_ERR_INVALID),          # out overlaps q
     (dict(q=0x10008), sr.SR_ERR_INVALID),                 # misaligned
     (dict(flags=8), sr.SR_ERR_INVALID),
-    (dict(flags=128), sr.SR_ERR_INVALID),                 # unknown bit
+    (dict(flags=512), sr.SR_ERR_INVALID),                 # unknown bit
+    (dict(flags=128 | 256), sr.SR_ERR_INVALID),           # SR_ONE_KERNEL with SR_TWO_KERNELS
+    (dict(flags=128, tile_n=128), sr.SR_ERR_UNSUPPORTED),  # the one-launch kernel runs T = 64
     (dict(flags=16 | 64), sr.SR_ERR_INVALID),             # SR_FUSE_IR with SR_IR_KERNEL
     (dict(flags=32 | 64), sr.SR_ERR_INVALID),             # SR_DECOMPOSE with SR_IR_KERNEL
     (dict(flags=64, in_dt=sr.SR_F32), sr.SR_ERR_UNSUPPORTED),  # variants are 16-bit only
@@ -209,14 +211,17 @@ def test_schedule_blocksparse(causal):
 def test_schedule_configs_match_survey():
     """Stored-element counts of the BASELINE configs."""
     c3 = W.config(3)
-    assert sr.schedule_stats(sr.dense_mask(None), c3.B, c3.H, c3.S, causal=True) == (64 * 136, 142_606_336)
+    # SURVEY's counts are at T = 128 (the two-kernel path); the one-launch default runs T = 64
+    assert sr.schedule_stats(sr.dense_mask(None), c3.B, c3.H, c3.S, causal=True, tile_n=128) == (64 * 136, 142_606_336)
     c4 = W.config(4)
     assert sr.schedule_stats(sr.block_mask(W.config_layout(c4)), c4.B, c4.H, c4.S)[1] == 48 * 622 * 64 * 64
     c5 = W.config(5)
     # 674 blocks of 64 x 64 per head at T = 64 (SURVEY App. A.1); the default T = 128 stores more
     assert sr.schedule_stats(sr.window_mask(c5.window, c5.n_global), c5.B, c5.H, c5.S, tile_n=64)[1] == 24 * 674 * 64 * 64
     c2 = W.config(2)
-    assert sr.schedule_stats(sr.dense_mask(c2.kv_len), c2.B, c2.H, c2.S)[0] == 12 * 20 * 4
+    assert sr.schedule_stats(sr.dense_mask(c2.kv_len), c2.B, c2.H, c2.S, tile_n=128)[0] == 12 * 20 * 4
+    # T = 64: live 64-key tiles per batch [8, 8, 6, 5, 5, 2, 2, 1] x 4 row-blocks x 12 heads
+    assert sr.schedule_stats(sr.dense_mask(c2.kv_len), c2.B, c2.H, c2.S)[0] == 12 * 37 * 4
 
 
 # ------------------------------------------------------------------------------ training backward

@@ -34,12 +34,12 @@ def _ulp_half(dtype, ref):
 
 
 def run_case(kind, B, H, S, D, dtype, *, causal=False, kv_len=None, layout=None, window=0, n_global=0,
-             tile_n=0, fused=True, seed=0, out_f32=True, fuse_ir=False, ir_kernel=False):
+             tile_n=0, fused=True, seed=0, out_f32=True, fuse_ir=False, ir_kernel=False, one_kernel=False):
     t, q, k, v = qkv(B, H, S, D, dtype, seed)
     scale = 1 / math.sqrt(D)
     od = torch.float32 if out_f32 else TORCH[dtype]
     kw = dict(scale=scale, causal=causal, tile_n=tile_n, fused=fused, out_dtype=od, fuse_ir=fuse_ir,
-              ir_kernel=ir_kernel)
+              ir_kernel=ir_kernel, one_kernel=one_kernel)
     if kind == "dense":
         o = sr.mha_dense(q, k, v, kv_len=kv_len, **kw)
     elif kind == "block":
@@ -372,14 +372,15 @@ FUSED_IR_CASES = [
 ]
 
 
-VARIANTS = ["fuse_ir", "ir_kernel"]
+VARIANTS = ["fuse_ir", "ir_kernel", "one_kernel"]
 
 
 @pytest.mark.parametrize("variant", VARIANTS)
 @pytest.mark.parametrize("kind,kw", FUSED_IR_CASES, ids=lambda x: str(x)[:40] if isinstance(x, dict) else x)
 def test_fused_ir_variant(kind, kw, variant):
     """The other IR placements against the oracle, same tolerance: SR_FUSE_IR (IR folded into
-    GEMM2) and SR_IR_KERNEL (the paper's standalone IR kernel writing r')."""
+    GEMM2), SR_IR_KERNEL (the paper's standalone IR kernel writing r') and
+    SR_ONE_KERNEL (GEMM1 and GEMM2 phases of each CTA in one launch)."""
     kw = dict(kw)
     if kw.get("layout") == "rand":
         kw["layout"] = W.random_layout(kw["H"], kw["S"] // 64, 64, 0.35, seed=8)

@@ -17,10 +17,14 @@ cfg = W.config(idx)
 dev = torch.device("cuda", 0)
 flush = (torch.empty(FLUSH_BYTES, dtype=torch.uint8, device=dev), torch.ones(FLUSH_BYTES // 4, device=dev))
 L = Layer(cfg, dev, cfg.idx, sr, torch)
-modes = {"default": {}, "fused_ir": {"fuse_ir": True}, "ir_kernel": {"ir_kernel": True},
-         "g1_only": {"stages": 1}, "g2_only": {"stages": 4}}
+modes = {"default": {}, "two_kernels": {"two_kernels": True}, "fused_ir": {"fuse_ir": True},
+         "ir_kernel": {"ir_kernel": True}, "g1_only": {"stages": 1, "two_kernels": True},
+         "g2_only": {"stages": 4, "two_kernels": True}}
+sel = os.environ.get("MODES")
+if sel:
+    modes = {k: v for k, v in modes.items() if k in sel.split(",")}
 out = []
-for rep in range(2):
+for rep in range(1):
     for name, kw in modes.items():
         L.run()
         L.run(**kw)
