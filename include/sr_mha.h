@@ -182,7 +182,8 @@ sr_status sr_mha_sliding_window_unfused(const void* q, const void* k, const void
  * out_dtype, fully overwritten, must not overlap q, k, v, out, dout or each other.  16-bit
  * in_dtype only (SR_ERR_UNSUPPORTED for F32).  ex->flags: 0, or SR_RUN_GEMM1 (row statistics +
  * dS' kernel), SR_RUN_REDUCE (dq kernel), SR_RUN_GEMM2 (dk and dv kernels) for per-kernel timing.
- * Five launches, stream-ordered, asynchronous; errors as for the forward. */
+ * Four launches (row statistics, dS', dq, dk + dv), stream-ordered, asynchronous; errors as for
+ * the forward. */
 sr_status sr_mha_dense_bwd(const void* q, const void* k, const void* v, const void* out, const void* dout,
                            void* dq, void* dk, void* dv, int B, int H, int S, int D, float scale,
                            const sr_dense_mask* mask_or_null, int causal, const sr_exec* ex);

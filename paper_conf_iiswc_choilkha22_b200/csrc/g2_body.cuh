@@ -46,6 +46,8 @@ constexpr int kMW2 = 128;  // macro tile width (keys per MMA step)
 #endif
 
 enum : int { SH_TILE = 1, SH_END = 2, SH_EMPTY = 4, SH_FIRST = 8, SH_LAST = 16 };
+// never written: zero rows for the invalid 64-row halves of a P tile read as an smem MMA operand
+static __device__ __align__(128) uint8_t g_zero_g2[kHalf * 128];
 struct G2Hdr {  // X'-stage / O-buffer header
     int32_t flags, hv0, hv1, nsub, orow_lo, orow_hi, pad0, pad1;
 };
@@ -116,7 +118,8 @@ __device__ __forceinline__ void g2_init(uint8_t* smem)
     uint64_t* st_full = o_empty + C::NO;
     uint64_t* st_empty = st_full + C::NSI;
     if (threadIdx.x == 0) {
-        for (int i = 0; i < C::NX; ++i) { mbar_init(&x_full[i], 1); mbar_init(&x_empty[i], C::NGS); }
+        // x_empty: the GS warps release a stage (GS), or the MMA commit (plain P . V: A read from smem)
+        for (int i = 0; i < C::NX; ++i) { mbar_init(&x_full[i], 1); mbar_init(&x_empty[i], GS ? C::NGS : 1); }
         for (int i = 0; i < C::NV; ++i) { mbar_init(&v_full[i], 1); mbar_init(&v_empty[i], 1); }
         for (int i = 0; i < C::NA; ++i) { mbar_init(&a_full[i], C::NGS); mbar_init(&a_empty[i], 1); }
         // o_full: O-header arrive + MMA commit; o_empty: one arrive per epilogue warp
@@ -175,7 +178,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                     for (int u = 0; u < NSUB; ++u) wn[u] = t + NSUB + u < I.t1 ? __ldg(p.sc.tinfo + t + NSUB + u) : 0;
                     uint32_t bytes = GS ? nsub * kRowBlock * 4 : 0;
 #ifndef SR_DIAG2_NOX
-                    for (int u = 0; u < nsub; ++u) bytes += (hv[u] == 3 ? 2 : 1) * (T / 64) * (kHalf * 128);
+                    for (int u = 0; u < nsub; ++u) bytes += (GS ? (hv[u] == 3 ? 2 : 1) : 2) * (T / 64) * (kHalf * 128);
 #endif
                     DW_WAIT(&x_empty[s], sph ^ 1, 0);
                     uint8_t* st = xstage(s);
@@ -201,6 +204,8 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                                 else {
                                     const int o2 = o + (hv[u] == 2 ? kHalf * 128 : 0);
                                     xload(st + o2, xs + o2, kHalf * 128);
+                                    if (!GS)  // the MMA reads every row of A: the invalid half is zeros
+                                        bulk_load(st + (o2 ^ (kHalf * 128)), g_zero_g2, kHalf * 128, &x_full[s]);
                                 }
                             }
                     }
@@ -361,8 +366,8 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
             // -------------------------------------------------------------- MMA issuer (whole warp,
             // one elected lane issues)
             const uint32_t idesc = idesc_f16(p.in_dtype == DT_BF16 ? 1 : 0, kRowBlock, D, 0, 1);
-            int s = 0, a = 0, o = 0;
-            uint32_t sph = 0, aph = 0, oph = 0;
+            int s = 0, a = 0, o = 0, xs = 0;
+            uint32_t sph = 0, aph = 0, oph = 0, xph = 0;
             auto post = [&](int flags, int64_t orow, bool second) {  // O header to the epilogue, arrival 1 of 2
                 DW_WAIT(&o_empty[o], oph ^ 1, 2);
                 if (elect_one()) {
@@ -391,23 +396,32 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                 for (int t = I.t0; t < I.t1; t += NSUB) {
                     const int nk = min(NSUB, I.t1 - t) * (T / 16);  // K steps of 16 keys
                     DW_WAIT(&v_full[s], sph, 0);
-                    DW_WAIT(&a_full[a], aph, 1);
+                    if (GS) DW_WAIT(&a_full[a], aph, 1);
+                    else DW_WAIT(&x_full[xs], xph, 1);
                     tc_fence_after();
                     const uint32_t v_addr = smem_u32(vstage(s));
                     const uint32_t a_tm = tmem_a + a * (kMW2 / 2);
+                    const uint32_t x_addr = smem_u32(xstage(xs));
                     if (elect_one()) {
 #pragma unroll 8
                         for (int kk = 0; kk < nk; ++kk) {
                             // B = V, MN-major SW128: 16 keys per MMA = 2 KB; 64-wide d blocks at LBO = MW*128 B
                             const uint64_t bd = smem_desc_sw128(v_addr + kk * 2048, kMW2 * 128, 1024);
-                            mma_ts(d_tmem, a_tm + kk * 8, bd, idesc, (t == I.t0 && kk == 0) ? 0u : 1u);
+                            if (GS) {
+                                mma_ts(d_tmem, a_tm + kk * 8, bd, idesc, (t == I.t0 && kk == 0) ? 0u : 1u);
+                            } else {  // A = the P tile in the stage: K-major SW128, 64-key blocks 16 KB apart
+                                const uint64_t ad = smem_desc_sw128(x_addr + (kk / 4) * (kRowBlock * 128) + (kk % 4) * 32, 16, 1024);
+                                mma_ss(d_tmem, ad, bd, idesc, (t == I.t0 && kk == 0) ? 0u : 1u);
+                            }
                         }
                         mma_commit(&v_empty[s]);
-                        mma_commit(&a_empty[a]);
+                        if (GS) mma_commit(&a_empty[a]);
+                        else mma_commit(&x_empty[xs]);
                     }
                     __syncwarp();
                     if (++s == C::NV) { s = 0; sph ^= 1; }
-                    if (++a == C::NA) { a = 0; aph ^= 1; }
+                    if (GS) { if (++a == C::NA) { a = 0; aph ^= 1; } }
+                    else if (++xs == C::NX) { xs = 0; xph ^= 1; }
                 }
                 if (elect_one()) mma_commit(&o_full[o]);  // arrival 2 of 2 when the item's MMAs complete
                 __syncwarp();
@@ -415,7 +429,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
             }
             post(SH_END, 0, true);
         }
-    } else if (warp >= 4 && warp < 4 + C::NGS) {
+    } else if (GS && warp >= 4 && warp < 4 + C::NGS) {
         // ------------------------------------------------------------------ GS transform
         const int gq = (warp - 4) % 4, ch = (warp - 4) / 4;  // lane quadrant, key slice (KPW keys)
         constexpr int KPW = C::KPW;

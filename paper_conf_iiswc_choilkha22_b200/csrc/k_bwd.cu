@@ -38,15 +38,20 @@ __device__ __forceinline__ uint32_t pack16(float a, float b, bool bf) { return b
 // ------------------------------------------------------------------------------ kernel 1
 // bstat[0][row] = m, bstat[1][row] = 1/d (merged from GEMM1's two IR partials exactly as GEMM2's
 // prologue merges them), bstat[2][row] = delta = sum_d dO[row, d] * O[row, d].  D/8 threads per
-// row, 16 B of dO each.
+// row for the dot product (16 B of dO each), then one thread per row for the statistics.
+constexpr int kPrepThreads = 512;
+
 template <int D>
-__global__ void __launch_bounds__(256) bwd_prep(const Params p)
+__global__ void __launch_bounds__(kPrepThreads) bwd_prep(const Params p)
 {
     griddep_launch_dependents();
     griddep_wait();
-    constexpr int TPR = D / 8;
+    constexpr int TPR = D / 8;                 // threads per row (16 B of dO each)
+    constexpr int RPB = kPrepThreads / TPR;    // rows per block
+    __shared__ float s_delta[RPB];
     const int64_t nrow = (int64_t)p.B * p.H * p.S;
-    const int64_t row = ((int64_t)blockIdx.x * 256 + threadIdx.x) / TPR;
+    const int64_t row0 = (int64_t)blockIdx.x * RPB;
+    const int64_t row = row0 + threadIdx.x / TPR;
     const int c = threadIdx.x % TPR;
     float acc = 0.f;
     if (row < nrow) {
@@ -79,14 +84,18 @@ __global__ void __launch_bounds__(256) bwd_prep(const Params p)
     }
 #pragma unroll
     for (int o = TPR / 2; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
-    if (row < nrow && c == 0) {
-        const float ma = __ldcg(p.rowstat + row), da = __ldcg(p.rowstat + nrow + row);
-        const float mb = __ldcg(p.rowstat + 2 * nrow + row), db = __ldcg(p.rowstat + 3 * nrow + row);
+    if (c == 0) s_delta[threadIdx.x / TPR] = acc;
+    __syncthreads();
+    // per-row statistics with one thread per row: coalesced loads of the IR partials and stores
+    if (threadIdx.x < RPB && row0 + threadIdx.x < nrow) {
+        const int64_t r = row0 + threadIdx.x;
+        const float ma = __ldcg(p.rowstat + r), da = __ldcg(p.rowstat + nrow + r);
+        const float mb = __ldcg(p.rowstat + 2 * nrow + r), db = __ldcg(p.rowstat + 3 * nrow + r);
         const float m = fmaxf(ma, mb);  // m = max_w m_w, d = sum_w e^{m_w - m} d_w
         const float d = m == -INFINITY ? 0.f : da * __expf(ma - m) + db * __expf(mb - m);
-        p.bstat[row] = m;
-        p.bstat[nrow + row] = d > 0.f ? 1.f / d : 0.f;
-        p.bstat[2 * nrow + row] = acc;
+        p.bstat[r] = m;
+        p.bstat[nrow + r] = d > 0.f ? 1.f / d : 0.f;
+        p.bstat[2 * nrow + r] = s_delta[threadIdx.x];
     }
 }
 
@@ -422,12 +431,17 @@ struct BK {
     static constexpr int THREADS = 384;
 };
 
-// PV = false: dK = dS'^T Q (A = dS' tiles, B = Q).  PV = true: dV = y^T dO (A = X' tiles scaled by
-// r' in shared memory -> y, B = dO).  Warps: 0 producer, 1 MMA, 2 TMEM allocator, 4-7 y transform
-// (PV), 8-11 epilogue.
-template <int D, bool PV>
-__global__ void __launch_bounds__(384, 1) tc_bwd_kv(const __grid_constant__ CUtensorMap tmB, const Params p)
+// One launch of 2 x n_ccta CTAs: the first n_ccta compute dV = y^T dO (PV: A = X' tiles scaled by
+// r' in shared memory -> y, B = dO), the rest dK = dS'^T Q (A = dS' tiles, B = Q) for the same
+// column items; dV CTAs (the heavier ones) start first, dK CTAs fill SMs as they free up.
+// Warps: 0 producer, 1 MMA, 2 TMEM allocator, 4-7 y transform (PV), 8-11 epilogue.
+template <int D>
+__global__ void __launch_bounds__(384, 1)
+    tc_bwd_kv(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmO, const Params p)
 {
+    const bool PV = blockIdx.x < (unsigned)p.sc.n_ccta;
+    const int cta = PV ? blockIdx.x : blockIdx.x - p.sc.n_ccta;
+    const CUtensorMap& tmB = PV ? tmO : tmQ;
     using C = BK<D>;
     extern __shared__ uint8_t smem_raw[];
     uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
@@ -456,7 +470,7 @@ __global__ void __launch_bounds__(384, 1) tc_bwd_kv(const __grid_constant__ CUte
     const uint32_t tmem_base = *tmem_ptr;
     griddep_launch_dependents();
     griddep_wait();
-    const int it_begin = __ldg(p.sc.ccta_ptr + blockIdx.x), it_end = __ldg(p.sc.ccta_ptr + blockIdx.x + 1);
+    const int it_begin = __ldg(p.sc.ccta_ptr + cta), it_end = __ldg(p.sc.ccta_ptr + cta + 1);
     const int T = p.T;
     const uint8_t* asrc = (const uint8_t*)(PV ? p.xprime : p.dsbuf);
     const int XS = kRowBlock * T * 2;
@@ -583,7 +597,8 @@ __global__ void __launch_bounds__(384, 1) tc_bwd_kv(const __grid_constant__ CUte
 #pragma unroll
             for (int ch = 0; ch < 2; ++ch) {
                 const bool valid = (hv[ch] >> myhalf) & 1;
-                const float rr = valid ? lds_f32(st + C::AB + C::BB + (T == 128 ? 0 : ch * 512) + 4 * r) : 0.f;
+                if (!valid) continue;  // this row of the chunk was zero-filled: y = 0 already
+                const float rr = lds_f32(st + C::AB + C::BB + (T == 128 ? 0 : ch * 512) + 4 * r);
 #pragma unroll
                 for (int q = 0; q < 8; ++q) {
                     const uint32_t off = tile_chunk_off(r, ch * 8 + q);
@@ -671,8 +686,9 @@ cudaError_t launch_bwd_d(const Params& p, cudaStream_t st, int64_t* nl)
     cudaError_t e;
     const int64_t rows = (int64_t)p.B * p.H * p.S;
     if (p.stages & 1) {
-        const int64_t nthr = rows * (D / 8);
-        if ((e = launch_pdl(bwd_prep<D>, dim3((unsigned)((nthr + 255) / 256)), dim3(256), 0, st, nl, p)) != cudaSuccess)
+        const int64_t rpb = kPrepThreads / (D / 8);
+        if ((e = launch_pdl(bwd_prep<D>, dim3((unsigned)((rows + rpb - 1) / rpb)), dim3(kPrepThreads), 0, st, nl, p)) !=
+            cudaSuccess)
             return e;
         CUtensorMap to, tv;
         if ((e = make_tmap_2d(&to, p.dout, rows, D, kRowBlock, p.in_dtype)) != cudaSuccess) return e;
@@ -694,13 +710,12 @@ cudaError_t launch_bwd_d(const Params& p, cudaStream_t st, int64_t* nl)
         CUtensorMap tq, to;
         if ((e = make_tmap_2d(&tq, p.q, rows, D, kRowBlock, p.in_dtype)) != cudaSuccess) return e;
         if ((e = make_tmap_2d(&to, p.dout, rows, D, kRowBlock, p.in_dtype)) != cudaSuccess) return e;
-        auto kk = tc_bwd_kv<D, false>;
-        auto kv = tc_bwd_kv<D, true>;
-        if ((e = cudaFuncSetAttribute(kk, cudaFuncAttributeMaxDynamicSharedMemorySize, BK<D>::SMEM)) != cudaSuccess) return e;
-        if ((e = cudaFuncSetAttribute(kv, cudaFuncAttributeMaxDynamicSharedMemorySize, BK<D>::SMEM)) != cudaSuccess) return e;
-        const dim3 grid(p.sc.n_ccta);
-        if ((e = launch_pdl(kk, grid, dim3(BK<D>::THREADS), BK<D>::SMEM, st, nl, tq, p)) != cudaSuccess) return e;
-        if ((e = launch_pdl(kv, grid, dim3(BK<D>::THREADS), BK<D>::SMEM, st, nl, to, p)) != cudaSuccess) return e;
+        auto kern = tc_bwd_kv<D>;
+        if ((e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, BK<D>::SMEM)) != cudaSuccess)
+            return e;
+        if ((e = launch_pdl(kern, dim3(2 * p.sc.n_ccta), dim3(BK<D>::THREADS), BK<D>::SMEM, st, nl, tq, to, p)) !=
+            cudaSuccess)
+            return e;
     }
     return cudaSuccess;
 }

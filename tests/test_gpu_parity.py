@@ -34,12 +34,13 @@ def _ulp_half(dtype, ref):
 
 
 def run_case(kind, B, H, S, D, dtype, *, causal=False, kv_len=None, layout=None, window=0, n_global=0,
-             tile_n=0, fused=True, seed=0, out_f32=True, fuse_ir=False, ir_kernel=False, one_kernel=False):
+             tile_n=0, fused=True, seed=0, out_f32=True, fuse_ir=False, ir_kernel=False, one_kernel=False,
+             two_kernels=False):
     t, q, k, v = qkv(B, H, S, D, dtype, seed)
     scale = 1 / math.sqrt(D)
     od = torch.float32 if out_f32 else TORCH[dtype]
     kw = dict(scale=scale, causal=causal, tile_n=tile_n, fused=fused, out_dtype=od, fuse_ir=fuse_ir,
-              ir_kernel=ir_kernel, one_kernel=one_kernel)
+              ir_kernel=ir_kernel, one_kernel=one_kernel, two_kernels=two_kernels)
     if kind == "dense":
         o = sr.mha_dense(q, k, v, kv_len=kv_len, **kw)
     elif kind == "block":
@@ -372,15 +373,16 @@ FUSED_IR_CASES = [
 ]
 
 
-VARIANTS = ["fuse_ir", "ir_kernel", "one_kernel"]
+VARIANTS = ["fuse_ir", "ir_kernel", "one_kernel", "two_kernels"]
 
 
 @pytest.mark.parametrize("variant", VARIANTS)
 @pytest.mark.parametrize("kind,kw", FUSED_IR_CASES, ids=lambda x: str(x)[:40] if isinstance(x, dict) else x)
 def test_fused_ir_variant(kind, kw, variant):
     """The other IR placements against the oracle, same tolerance: SR_FUSE_IR (IR folded into
-    GEMM2), SR_IR_KERNEL (the paper's standalone IR kernel writing r') and
-    SR_ONE_KERNEL (GEMM1 and GEMM2 phases of each CTA in one launch)."""
+    GEMM2), SR_IR_KERNEL (the paper's standalone IR kernel writing r'),
+    SR_ONE_KERNEL (GEMM1 and GEMM2 phases of each CTA in one launch, the 16-bit default) and
+    SR_TWO_KERNELS (the same chain as two launches)."""
     kw = dict(kw)
     if kw.get("layout") == "rand":
         kw["layout"] = W.random_layout(kw["H"], kw["S"] // 64, 64, 0.35, seed=8)
@@ -398,7 +400,9 @@ def test_fused_ir_full_configs(idx, variant):
     t = W.config_tensors(cfg)
     from tests.gpu_util import to_dev
     q, k, v = (to_dev(x, cfg.dtype) for x in (t.q_s, t.k_s, t.v_s))
-    kw = dict(scale=cfg.scale, out_dtype=torch.float32, **{variant: True})
+    # the two-launch variants at their tuned T = 128 (block-sparse: 64), the default at T = 64
+    tn = 0 if (variant == "one_kernel" or cfg.kind == "blocksparse") else 128
+    kw = dict(scale=cfg.scale, out_dtype=torch.float32, tile_n=tn, **{variant: True})
     if cfg.kind == "dense":
         o = sr.mha_dense(q, k, v, kv_len=cfg.kv_len, causal=cfg.causal, **kw)
         m = oracle.Mask(kv_len=cfg.kv_len, causal=cfg.causal)

@@ -16,7 +16,7 @@ import sys
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 OUT = os.path.join(ROOT, "gpurun_out")
-PROF = os.path.join(ROOT, "profiles")
+PROF = os.environ.get("PROF_OUT") or os.path.join(ROOT, "profiles")  # PROF_OUT: e.g. gpurun_out/prof on the box
 def kname(full):
     """Map an ncu kernel name to the bench.py stage name (template args decide the variant)."""
     import re
@@ -33,9 +33,10 @@ def kname(full):
                 return "gs_gemm2"  # default path: (m, 1/d) from GEMM1
             return "gs_gemm2_fused_ir" if len(flags) > 1 and flags[1] else "gs_gemm2_rprime"
         return "gemm2_plain"
-    m = re.search(r"tc_bwd_kv<([^>]*)>", full)
-    if m:
-        return "bwd_dv" if m.group(1).split(",")[-1].strip() in ("true", "1", "(bool)1") else "bwd_dk"
+    if "tc_fused" in full:
+        return "sr_layer_one_kernel"
+    if "tc_bwd_kv" in full:
+        return "bwd_dkdv"
     for k, v in (("ir_kernel", "ir"), ("row_softmax", "softmax"), ("sd_ls_kernel", "sd_ls"),
                  ("sd_gs_kernel", "sd_gs"), ("tc_bwd_ds", "bwd_ds"), ("bwd_prep", "bwd_prep")):
         if k in full:
@@ -80,11 +81,15 @@ def main(rnd):
             lines.append(f"{n:28s} {len(m['gpu__time_duration.sum']):8d} {t / 1e3 * unit:10.2f} {rd / 1e6:11.2f} {wr / 1e6:11.2f}")
             if not n.startswith("other"):
                 ours[n] = (t, rd + wr)
-        rec = [k for k in ("gemm1_ls_ir", "gs_gemm2") if k in ours]  # default path (IR in GEMM1)
+        rec = [k for k in ("sr_layer_one_kernel",) if k in ours]  # default path: one launch
+        two = [k for k in ("gemm1_ls_ir", "gs_gemm2") if k in ours]  # SR_TWO_KERNELS
         unf = [k for k in ("gemm1_plain", "softmax", "gemm2_plain") if k in ours]
         tr = sum(ours[k][0] for k in rec)
         lines.append("")
-        lines.append("recomposed layer shares: " + ", ".join(f"{k} {ours[k][0] / tr:.1%}" for k in rec))
+        lines.append("recomposed layer (default, one launch): " + ", ".join(f"{k} {ours[k][0] / 1e3:.2f} us" for k in rec))
+        if len(two) == 2:
+            t2 = sum(ours[k][0] for k in two)
+            lines.append("two-kernel variant shares: " + ", ".join(f"{k} {ours[k][0] / t2:.1%}" for k in two))
         tu = sum(ours[k][0] for k in unf) if unf else 0
         if unf:
             lines.append("unfused layer shares:    " + ", ".join(f"{k} {ours[k][0] / tu:.1%}" for k in unf))
@@ -121,7 +126,7 @@ def main(rnd):
                 wr = sum(m["dram__bytes_write.sum"]) / len(m["dram__bytes_write.sum"])
                 nm = "bwd_dq (gemm2_plain)" if n == "gemm2_plain" else n
                 lines.append(f"{nm:28s} {len(m['gpu__time_duration.sum']):8d} {t / 1e3:10.2f} {rd / 1e6:11.2f} {wr / 1e6:11.2f}")
-                if n in ("bwd_prep", "bwd_ds", "gemm2_plain", "bwd_dk", "bwd_dv"):
+                if n in ("bwd_prep", "bwd_ds", "gemm2_plain", "bwd_dkdv"):
                     bw["bwd_dq" if n == "gemm2_plain" else n] = (t, rd + wr)
             if bw:
                 tb = sum(v[0] for v in bw.values())
@@ -131,7 +136,7 @@ def main(rnd):
                 e["backward_dram_bytes"] = int(sum(v[1] for v in bw.values()))
         traffic[f"C{c}"] = e
         open(os.path.join(PROF, f"{rnd}_launches_c{c}.txt"), "w").write("\n".join(lines) + "\n")
-        for k in ("tc_gemm1", "tc_gemm2", "ir_kernel", "tc_gemm2_fi", "tc_bwd_ds", "tc_bwd_dk", "tc_bwd_dv"):
+        for k in ("tc_fused", "tc_gemm1", "tc_gemm2", "ir_kernel", "tc_gemm2_fi", "tc_bwd_ds", "tc_bwd_dkdv"):
             rep = os.path.join(OUT, f"full_c{c}_{k}.ncu-rep")
             if os.path.exists(rep):
                 s = subprocess.run([sys.executable, os.path.join(ROOT, "tools", "ncu_summary.py"), rep, "25"],

@@ -9,9 +9,7 @@ for c in ${CFGS:-2 3 4 5}; do
     --csv --log-file gpurun_out/launches_train_c$c.csv python tools/run_layer.py $c train 3 > /dev/null 2>&1
   timeout 300 $NCU --set full --clock-control none --import-source on -k regex:tc_bwd_ds -s 1 -c 1 \
     -o gpurun_out/full_c${c}_tc_bwd_ds -f python tools/run_layer.py $c train 3 > /dev/null 2>&1
-  timeout 300 $NCU --set full --clock-control none --import-source on -k regex:tc_bwd_kv -s 2 -c 1 \
-    -o gpurun_out/full_c${c}_tc_bwd_dk -f python tools/run_layer.py $c train 3 > /dev/null 2>&1
-  timeout 300 $NCU --set full --clock-control none --import-source on -k regex:tc_bwd_kv -s 3 -c 1 \
-    -o gpurun_out/full_c${c}_tc_bwd_dv -f python tools/run_layer.py $c train 3 > /dev/null 2>&1
+  timeout 300 $NCU --set full --clock-control none --import-source on -k regex:tc_bwd_kv -s 1 -c 1 \
+    -o gpurun_out/full_c${c}_tc_bwd_dkdv -f python tools/run_layer.py $c train 3 > /dev/null 2>&1
 done
 ls gpurun_out/
