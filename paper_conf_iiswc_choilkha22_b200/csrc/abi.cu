@@ -364,6 +364,15 @@ void lpt_assign(std::vector<int32_t>& items, const std::vector<int64_t>& cost, i
     items.swap(out);
 }
 
+// Fixed cost of an item (Q load, row statistics, O store, pipeline fill) in units of half a tile
+// (3: measured on the one-launch kernel, C2 25.8 -> 24.7 us; 1 and 6-10 are slower or equal);
+// SR_LPT_FIXED overrides for experiments.
+int64_t lpt_item_cost()
+{
+    static const int64_t v = [] { const char* e = getenv("SR_LPT_FIXED"); return e ? (int64_t)atoi(e) : (int64_t)3; }();
+    return v;
+}
+
 // Per-CTA item ranges for both schedules.  Cost of an item = 2 x its tiles + 1 (the Q load / O
 // store of a row-block is about half a tile's traffic); of a pair = its two row-blocks' tiles + 1.
 void lpt_assign(HostSched& h, int n_cta)
@@ -373,7 +382,7 @@ void lpt_assign(HostSched& h, int n_cta)
     for (size_t i = 0; i < h.items.size(); ++i) {
         const int g = h.items[i] / h.n_rb, rb = h.items[i] % h.n_rb;
         const int32_t* tp = &h.tp[(size_t)lh_of_g(g) * (h.n_rb + 1)];
-        cost[i] = 2 * (int64_t)(tp[rb + 1] - tp[rb]) + 1;
+        cost[i] = 2 * (int64_t)(tp[rb + 1] - tp[rb]) + lpt_item_cost();
     }
     lpt_assign(h.items, cost, n_cta, h.cta_ptr);
     std::vector<int64_t> pcost(h.pitems.size());

@@ -21,6 +21,21 @@ namespace sr {
 
 using namespace ptx;
 
+#ifdef SR_DIAG_PHASES
+// diagnostic build: per CTA, %globaltimer (ns) at kernel start, after the prologue, after phase 1,
+// after phase 2, plus the CTA's item count (read with sr_diag_read_phases)
+__device__ unsigned long long g_diag_phases[1024 * 5];
+__device__ __forceinline__ unsigned long long gtimer()
+{
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
+#define PH_MARK(i) do { if (threadIdx.x == 0) g_diag_phases[blockIdx.x * 5 + (i)] = gtimer(); } while (0)
+#else
+#define PH_MARK(i)
+#endif
+
 template <int D>
 __global__ void __launch_bounds__(640, 1)
     tc_fused(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmK,
@@ -33,6 +48,7 @@ __global__ void __launch_bounds__(640, 1)
     uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
     uint32_t* tmem_ptr = (uint32_t*)(smem + C1::OFF_TPTR);
     const int warp = warp_uniform(), lane = threadIdx.x % 32;
+    PH_MARK(0);
     if (threadIdx.x == 0) g1_init<D, 64, true, false, true>(smem);
     if (warp == 0 && lane == 0) { prefetch_tmap(&tmQ); prefetch_tmap(&tmK); prefetch_tmap(&tmV); }
     if (warp == 2) tmem_alloc(tmem_ptr, 512);
@@ -44,6 +60,7 @@ __global__ void __launch_bounds__(640, 1)
     griddep_wait();
 
     const int it_begin = __ldg(p.sc.cta_ptr + blockIdx.x), it_end = __ldg(p.sc.cta_ptr + blockIdx.x + 1);
+    PH_MARK(1);
     // ---- phase 1: GEMM1 + LS + IR over the CTA's row-blocks (all 20 warps)
     g1_roles<D, 64, true, false, true>(tmQ, tmK, p, smem, tmem_base, it_begin, it_end);
     // back to the launch split (phase 1 leaves warps 0-3 at 64 registers, the epilogue at 104)
@@ -55,6 +72,7 @@ __global__ void __launch_bounds__(640, 1)
     tc_fence_before();
     __syncthreads();
     tc_fence_after();
+    PH_MARK(2);
     if (threadIdx.x == 0) {
         uint64_t* b1 = (uint64_t*)(smem + C1::OFF_BAR);
         for (int i = 0; i < C1::NBAR; ++i) mbar_inval(&b1[i]);
@@ -65,6 +83,10 @@ __global__ void __launch_bounds__(640, 1)
     g2_roles<D, 64, true, true, true>(tmV, p, smem, tmem_base, it_begin, it_end);
     tc_fence_before();
     __syncthreads();
+    PH_MARK(3);
+#ifdef SR_DIAG_PHASES
+    if (threadIdx.x == 0) g_diag_phases[blockIdx.x * 5 + 4] = it_end - it_begin;
+#endif
     if (warp == 2) {
         tc_fence_after();
         tmem_dealloc(tmem_base, 512);
@@ -95,3 +117,10 @@ cudaError_t launch_tc_one(const Params& p, cudaStream_t st, int64_t* nl)
 }
 
 }  // namespace sr
+
+#ifdef SR_DIAG_PHASES
+extern "C" int sr_diag_read_phases(unsigned long long* out)  // [1024][5] (diagnostic build)
+{
+    return cudaMemcpyFromSymbol(out, sr::g_diag_phases, sizeof(sr::g_diag_phases)) != cudaSuccess;
+}
+#endif
