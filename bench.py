@@ -210,7 +210,7 @@ class Layer:
         self.bwd()
 
     def run(self, fused=True, stages=0, q=None, k=None, v=None, fuse_ir=False, sd=False, ir_kernel=False,
-            two_kernels=False):
+            two_kernels=False, gs_prologue=False):
         d = self.dev
         two = fuse_ir or ir_kernel or two_kernels
         if sd:
@@ -224,7 +224,7 @@ class Layer:
         return self.sr.call(self.mask, q if q is not None else d["q"], k if k is not None else d["k"],
                             v if v is not None else d["v"], out=self.out, fused=fused, stages=stages,
                             workspace=ws, tile_n=tn, fuse_ir=fuse_ir, sd=sd, ir_kernel=ir_kernel,
-                            two_kernels=two_kernels, **self.kw)
+                            two_kernels=two_kernels, gs_prologue=gs_prologue, **self.kw)
 
 
 def timed(torch, fn, steps, warmup, flush, per_step_pre=None):

@@ -139,6 +139,10 @@ typedef struct {
 /* Variant bit: the two-kernel chain GEMM1 + LS + IR -> GS + GEMM2 (the default before the
  * one-launch kernel; also what tile_n = 128 without a variant bit runs). */
 #define SR_TWO_KERNELS 256
+/* Modifier of the one-launch kernel (fp16): apply Global Scaling in GEMM2's prologue (Y = X' r'
+ * rounded to fp16, then Y V) instead of accumulator-side (O += r'_k (X'_k V_k) in fp32, the
+ * fp16 default).  bf16 always uses the prologue form. */
+#define SR_GS_PROLOGUE 512
 
 /* Entry points (north star).  Returns SR_OK after enqueueing the kernels on ex->stream. */
 sr_status sr_mha_dense(const void* q, const void* k, const void* v, void* out, int B, int H, int S,

@@ -217,18 +217,21 @@ SR_DECOMPOSE = 32
 SR_IR_KERNEL = 64
 SR_ONE_KERNEL = 128
 SR_TWO_KERNELS = 256
+SR_GS_PROLOGUE = 512
 
 
 def call(mask: _Mask, q, k, v, *, scale=None, causal=False, out_dtype=None, tile_n=0, fused=True,
          out=None, workspace=None, stream=None, stages=0, fuse_ir=False, sd=False, ir_kernel=False,
-         one_kernel=False, two_kernels=False):
+         one_kernel=False, two_kernels=False, gs_prologue=False):
     """Run one attention layer through the C ABI.  q, k, v: CUDA tensors [B, H, S, D].
     Default (16-bit): GEMM1 + LS with the IR merged inside it, then GS + GEMM2, both in one launch.
     ir_kernel=True selects SR_IR_KERNEL (the paper's layout: a standalone IR kernel writing r');
     fuse_ir=True SR_FUSE_IR (IR folded into GEMM2, SURVEY NEXT-2);
     sd=True SR_DECOMPOSE (decomposition without fusion, the paper's SD, NEXT-1);
     one_kernel=True SR_ONE_KERNEL (GEMM1+LS+IR then GS+GEMM2 per CTA in one launch, T = 64; the
-    16-bit default anyway); two_kernels=True SR_TWO_KERNELS (the same chain as two launches)."""
+    16-bit default anyway); two_kernels=True SR_TWO_KERNELS (the same chain as two launches);
+    gs_prologue=True SR_GS_PROLOGUE (one launch, fp16: Global Scaling in GEMM2's prologue instead of
+    accumulator-side)."""
     torch = _torch()
     if not (q.is_cuda and k.is_cuda and v.is_cuda):
         raise ValueError("q, k, v must be CUDA tensors")
@@ -256,7 +259,7 @@ def call(mask: _Mask, q, k, v, *, scale=None, causal=False, out_dtype=None, tile
     ex = Exec(in_dt, dtype_code(out_dtype), ws.data_ptr(), ws.numel() * ws.element_size(), st, int(tile_n),
               int(stages) | (SR_FUSE_IR if fuse_ir else 0) | (SR_DECOMPOSE if sd else 0) |
               (SR_IR_KERNEL if ir_kernel else 0) | (SR_ONE_KERNEL if one_kernel else 0) |
-              (SR_TWO_KERNELS if two_kernels else 0))
+              (SR_TWO_KERNELS if two_kernels else 0) | (SR_GS_PROLOGUE if gs_prologue else 0))
     fn = getattr(lib(), _FN[(mask.entry, bool(fused))])
     _check(fn(q.data_ptr(), k.data_ptr(), v.data_ptr(), out.data_ptr(), B, H, S, D, C.c_float(scale), mask.ptr,
               int(causal), C.byref(ex)))

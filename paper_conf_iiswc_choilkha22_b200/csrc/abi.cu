@@ -555,7 +555,7 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
     if (!q || !k || !v || !out) return fail(SR_ERR_INVALID, "q, k, v and out must be non-NULL");
     if (!std::isfinite(scale) || !(scale > 0.f)) return fail(SR_ERR_INVALID, "scale must be finite and > 0");
     const int variant_bits = SR_FUSE_IR | SR_DECOMPOSE | SR_IR_KERNEL | SR_ONE_KERNEL | SR_TWO_KERNELS;
-    if (ex->flags & ~(SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2 | variant_bits))
+    if (ex->flags & ~(SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2 | SR_GS_PROLOGUE | variant_bits))
         return fail(SR_ERR_INVALID, "unknown flags 0x%x", ex->flags);
     if ((ex->flags & variant_bits) && (!fused || ex->in_dtype == SR_F32))
         return fail(SR_ERR_UNSUPPORTED, "SR_FUSE_IR / SR_DECOMPOSE / SR_IR_KERNEL apply to the recomposed 16-bit path only");
@@ -633,6 +633,7 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
         ce = launch_tc_sd(p, st, &nl);
     } else if (fused && one) {
         p.g1_pair = 0;
+        p.gs_prologue = (ex->flags & SR_GS_PROLOGUE) != 0;
 
         ce = launch_tc_one(p, st, &nl);
     } else if (fused) {

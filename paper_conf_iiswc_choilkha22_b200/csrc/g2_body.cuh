@@ -91,6 +91,12 @@ struct G2 {
 #ifndef SR_G2_NGS
 #define SR_G2_NGS 8
 #endif
+// fp16 GS: Y = X' * r' as one mul.rn.f16x2 per pair (r' rounded to fp16 first: two roundings of
+// relative 2^-11 each instead of one; r' < 2^-24 flushes to 0, a product below fp16's subnormal
+// range anyway).  On by default (measured: C4 -2.2 us, C5 -1.5 us); the bf16 path goes through fp32.
+#ifndef SR_G2_HMUL
+#define SR_G2_HMUL 1
+#endif
     static constexpr int NGS = SR_G2_NGS;       // GS warps: 8 (64 keys each) or 16 (32 keys each)
     static constexpr int KPW = kMW2 * 4 / NGS;  // keys of a macro tile per GS warp
     static constexpr int THREADS = 128 + NGS * 32 + 128;
@@ -102,7 +108,7 @@ struct G2 {
 // RS (default mode, IR in GEMM1): as FI, but GEMM1 already merged the rows, so warp 2 only loads each item's
 // per-row (m, 1/d) -- GEMM2 applies the normalisation 1/d * e^{m' - m} in its prologue.
 // Barrier initialisation of GEMM2's shared-memory layout (thread 0; fence_mbar_init included).
-template <int D, int T, bool GS, bool FI, bool RS>
+template <int D, int T, bool GS, bool FI, bool RS, bool AS = false>
 __device__ __forceinline__ void g2_init(uint8_t* smem)
 {
     using C = G2<D, T>;
@@ -119,9 +125,12 @@ __device__ __forceinline__ void g2_init(uint8_t* smem)
     uint64_t* st_empty = st_full + C::NSI;
     if (threadIdx.x == 0) {
         // x_empty: the GS warps release a stage (GS), or the MMA commit (plain P . V: A read from smem)
-        for (int i = 0; i < C::NX; ++i) { mbar_init(&x_full[i], 1); mbar_init(&x_empty[i], GS ? C::NGS : 1); }
+        // (AS: the MMA commit and the NGS scaling warps, which read the stage's m')
+        for (int i = 0; i < C::NX; ++i) { mbar_init(&x_full[i], 1); mbar_init(&x_empty[i], AS ? 1 + C::NGS : (GS ? C::NGS : 1)); }
         for (int i = 0; i < C::NV; ++i) { mbar_init(&v_full[i], 1); mbar_init(&v_empty[i], 1); }
-        for (int i = 0; i < C::NA; ++i) { mbar_init(&a_full[i], C::NGS); mbar_init(&a_empty[i], 1); }
+        // a_full / a_empty: the TMEM A-operand ring (GS), or in AS mode the ring of per-sub-tile
+        // partial products X'_k V_k (full: MMA commit; empty: the NGS scaling warps)
+        for (int i = 0; i < C::NA; ++i) { mbar_init(&a_full[i], AS ? 1 : C::NGS); mbar_init(&a_empty[i], AS ? C::NGS : 1); }
         // o_full: O-header arrive + MMA commit; o_empty: one arrive per epilogue warp
         for (int i = 0; i < C::NO; ++i) { mbar_init(&o_full[i], 2); mbar_init(&o_empty[i], 4); }
         for (int i = 0; i < C::NSI; ++i) { mbar_init(&st_full[i], 1); mbar_init(&st_empty[i], C::NGS); }
@@ -130,7 +139,12 @@ __device__ __forceinline__ void g2_init(uint8_t* smem)
 }
 
 // Warp roles of GEMM2 after the prologue (warps 0 .. THREADS/32 - 1; extra warps of a larger CTA idle).
-template <int D, int T, bool GS, bool FI, bool RS>
+// AS (accumulator-side Global Scaling, SURVEY NEXT-2's second form; fp16, requires GS, FI, RS): the
+// MMA reads X' straight from its shared-memory stage (K-major SW128, invalid halves zero-filled)
+// and writes each sub-tile's partial product X'_k V_k to its own TMEM buffer; the scaling warps add
+// r'_k (X'_k V_k) to the rows' O in registers, r'_k = e^{m'_k - m} / d -- the same terms as
+// (X'_k r'_k) V_k (Eq. 2 is linear in each sub-vector), with no per-element GS pass over X'.
+template <int D, int T, bool GS, bool FI, bool RS, bool AS = false>
 __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p, uint8_t* smem, uint32_t tmem_base,
                                           int it_begin, int it_end)
 {
@@ -170,6 +184,18 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
             uint32_t sph = 0;
             for (ItemWalk iw(p, it_begin, it_end); iw.more();) {
                 const ItemInfo I = iw.next();
+                if (AS && I.t0 == I.t1) {  // no kept key in these rows: an EMPTY stage, written as zeros
+                    DW_WAIT(&x_empty[s], sph ^ 1, 0);
+                    if (elect_one()) {
+                        const int64_t orow = (int64_t)I.g * p.S + I.rb * kRowBlock;
+                        *xhdr(s) = G2Hdr{SH_EMPTY | SH_FIRST | SH_LAST, 0, 0, 0, (int32_t)(orow & 0xffffffff),
+                                         (int32_t)(orow >> 32), 0, 0};
+                        mbar_arrive(&x_full[s]);
+                    }
+                    __syncwarp();
+                    if (++s == C::NX) { s = 0; sph ^= 1; }
+                    continue;
+                }
                 int wn[2];  // schedule words of the next macro tile, prefetched one step ahead
                 for (int u = 0; u < NSUB; ++u) wn[u] = I.t0 + u < I.t1 ? __ldg(p.sc.tinfo + I.t0 + u) : 0;
                 for (int t = I.t0; t < I.t1; t += NSUB) {
@@ -178,13 +204,14 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                     for (int u = 0; u < NSUB; ++u) wn[u] = t + NSUB + u < I.t1 ? __ldg(p.sc.tinfo + t + NSUB + u) : 0;
                     uint32_t bytes = GS ? nsub * kRowBlock * 4 : 0;
 #ifndef SR_DIAG2_NOX
-                    for (int u = 0; u < nsub; ++u) bytes += (GS ? (hv[u] == 3 ? 2 : 1) : 2) * (T / 64) * (kHalf * 128);
+                    for (int u = 0; u < nsub; ++u) bytes += ((GS && !AS) ? (hv[u] == 3 ? 2 : 1) : 2) * (T / 64) * (kHalf * 128);
 #endif
                     DW_WAIT(&x_empty[s], sph ^ 1, 0);
                     uint8_t* st = xstage(s);
                     if (elect_one()) {
+                    const int64_t orow = (int64_t)I.g * p.S + I.rb * kRowBlock;
                     *xhdr(s) = G2Hdr{SH_TILE | (t == I.t0 ? SH_FIRST : 0) | (t + NSUB >= I.t1 ? SH_LAST : 0), hv[0],
-                                     hv[1], nsub, 0, 0, 0, 0};
+                                     hv[1], nsub, (int32_t)(orow & 0xffffffff), (int32_t)(orow >> 32), 0, 0};
                     mbar_arrive_expect_tx(&x_full[s], bytes);
                     const uint8_t* xs = src + (I.slot0 + t) * (int64_t)C::XS;  // sub-tiles t, t+1 are adjacent
                     auto xload = [&](uint8_t* d, const uint8_t* g, uint32_t n) {
@@ -204,7 +231,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                                 else {
                                     const int o2 = o + (hv[u] == 2 ? kHalf * 128 : 0);
                                     xload(st + o2, xs + o2, kHalf * 128);
-                                    if (!GS)  // the MMA reads every row of A: the invalid half is zeros
+                                    if (!GS || AS)  // the MMA reads every row of A: the invalid half is zeros
                                         bulk_load(st + (o2 ^ (kHalf * 128)), g_zero_g2, kHalf * 128, &x_full[s]);
                                 }
                             }
@@ -361,6 +388,133 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                 }
             }
         }
+    } else if (AS && warp == 1) {
+        // ------------------------------------------------------------------ MMA issuer (AS): per
+        // macro tile and sub-tile u, X'_u V_u into the next partial-product buffer (D columns)
+        const uint32_t idesc = idesc_f16(0, kRowBlock, D, 0, 1);
+        int s = 0, xs = 0, j = 0;
+        uint32_t sph = 0, xph = 0, jph = 0;
+        for (ItemWalk iw(p, it_begin, it_end); iw.more();) {
+            const ItemInfo I = iw.next();
+            if (I.t0 == I.t1) {  // the producer posted an EMPTY stage: add our release to it
+                DW_WAIT(&x_full[xs], xph, 1);
+                if (elect_one()) mbar_arrive(&x_empty[xs]);
+                __syncwarp();
+                if (++xs == C::NX) { xs = 0; xph ^= 1; }
+                continue;
+            }
+            for (int t = I.t0; t < I.t1; t += NSUB) {
+                const int nsub = min(NSUB, I.t1 - t);
+                DW_WAIT(&v_full[s], sph, 0);
+                DW_WAIT(&x_full[xs], xph, 1);
+                tc_fence_after();
+                const uint32_t v_addr = smem_u32(vstage(s)), x_addr = smem_u32(xstage(xs));
+                for (int u = 0; u < nsub; ++u) {
+                    DW_WAIT(&a_empty[j], jph ^ 1, 2);
+                    tc_fence_after();
+                    if (elect_one()) {
+#pragma unroll
+                        for (int k2 = 0; k2 < T / 16; ++k2) {
+                            const int kk = u * (T / 16) + k2;  // K step of 16 keys within the macro tile
+                            const uint64_t bd = smem_desc_sw128(v_addr + kk * 2048, kMW2 * 128, 1024);
+                            const uint64_t ad = smem_desc_sw128(x_addr + (kk / 4) * (kRowBlock * 128) + (kk % 4) * 32, 16, 1024);
+                            mma_ss(tmem_base + j * D, ad, bd, idesc, k2 > 0 ? 1u : 0u);
+                        }
+                        mma_commit(&a_full[j]);
+                    }
+                    __syncwarp();
+                    if (++j == C::NA) { j = 0; jph ^= 1; }
+                }
+                if (elect_one()) {
+                    mma_commit(&v_empty[s]);
+                    mma_commit(&x_empty[xs]);
+                }
+                __syncwarp();
+                if (++s == C::NV) { s = 0; sph ^= 1; }
+                if (++xs == C::NX) { xs = 0; xph ^= 1; }
+            }
+        }
+    } else if (AS && warp >= 4 && warp < 4 + C::NGS) {
+        // ------------------------------------------------------------------ accumulator-side GS:
+        // warp w owns TMEM lane quadrant (w-4) % 4 (32 rows) and column half (w-4) / 4 of O (D/2
+        // fp32 in registers); per sub-tile u: O += r'_u * (X'_u V_u), r'_u = e^{m'_u - m} / d
+        constexpr int DH = D / 2;
+        const int gq = (warp - 4) % 4, hh = (warp - 4) / 4;
+        const int r = gq * 32 + lane;
+        const int myhalf = r / kHalf;
+        const uint32_t lane_off = (uint32_t)(gq * 32) << 16;
+        int s = 0, si = 0, j = 0;
+        uint32_t sph = 0, siph = 0, jph = 0;
+        float m_row = 0.f, invd_row = 0.f;
+        float o[DH];
+#pragma unroll
+        for (int c = 0; c < DH; ++c) o[c] = 0.f;
+        for (;;) {
+            DW_WAIT(&x_full[s], sph, 0);
+            const G2Hdr h = lds_hdr(xhdr(s));
+            if (h.flags & SH_END) break;
+            const int64_t orow = (((int64_t)h.orow_hi << 32) | (uint32_t)h.orow_lo) + r;
+            if (h.flags & SH_FIRST) {
+#pragma unroll
+                for (int c = 0; c < DH; ++c) o[c] = 0.f;
+                if (!(h.flags & SH_EMPTY)) {  // the statistics warp skips empty items
+                    DW_WAIT(&st_full[si], siph, 2);
+                    m_row = stats[si * 2 * kRowBlock + r];
+                    invd_row = stats[si * 2 * kRowBlock + kRowBlock + r];
+                    __syncwarp();
+                    if (lane == 0) mbar_arrive(&st_empty[si]);
+                    if (++si == C::NSI) { si = 0; siph ^= 1; }
+                }
+            }
+            if (!(h.flags & SH_EMPTY)) {
+                const uint32_t xs_s = smem_u32(xstage(s));
+                const int hvs[2] = {h.hv0, h.hv1};
+                float rr[NSUB];
+#pragma unroll
+                for (int u = 0; u < NSUB; ++u) {
+                    const bool valid = u < h.nsub && ((hvs[u] >> myhalf) & 1);
+                    const float mp = valid ? lds_f32(xs_s + C::XB + u * 512 + 4 * r) : -INFINITY;
+                    rr[u] = (mp == -INFINITY) ? 0.f : __expf(mp - m_row) * invd_row;  // 0 for a masked sub-vector
+                }
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&x_empty[s]);  // m' read; the MMA commit releases the X' data
+#pragma unroll
+                for (int u = 0; u < NSUB; ++u) {
+                    if (u >= h.nsub) break;
+                    DW_WAIT(&a_full[j], jph, 1);
+                    tc_fence_after();
+#pragma unroll
+                    for (int c = 0; c < DH / 32; ++c) {
+                        uint32_t v[32];
+                        tmem_ld32(tmem_base + lane_off + j * D + hh * DH + c * 32, v);
+                        tmem_wait_ld();
+#pragma unroll
+                        for (int i = 0; i < 32; ++i) o[c * 32 + i] = fmaf(rr[u], __uint_as_float(v[i]), o[c * 32 + i]);
+                    }
+                    tc_fence_before();
+                    __syncwarp();
+                    if (lane == 0) mbar_arrive(&a_empty[j]);
+                    if (++j == C::NA) { j = 0; jph ^= 1; }
+                }
+            } else {
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&x_empty[s]);
+            }
+            if (h.flags & SH_LAST) {  // this warp's D/2 columns of its 32 output rows
+                if (p.out_dtype == DT_F32) {
+                    float4* O = reinterpret_cast<float4*>((float*)p.out + orow * D + hh * DH);
+#pragma unroll
+                    for (int c = 0; c < DH / 4; ++c) O[c] = make_float4(o[4 * c], o[4 * c + 1], o[4 * c + 2], o[4 * c + 3]);
+                } else {
+                    uint4* O = reinterpret_cast<uint4*>((uint16_t*)p.out + orow * D + hh * DH);
+#pragma unroll
+                    for (int c = 0; c < DH / 8; ++c)
+                        O[c] = make_uint4(pack_f16(o[8 * c], o[8 * c + 1]), pack_f16(o[8 * c + 2], o[8 * c + 3]),
+                                          pack_f16(o[8 * c + 4], o[8 * c + 5]), pack_f16(o[8 * c + 6], o[8 * c + 7]));
+                }
+            }
+            if (++s == C::NX) { s = 0; sph ^= 1; }
+        }
     } else if (warp == 1) {
         {
             // -------------------------------------------------------------- MMA issuer (whole warp,
@@ -429,7 +583,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
             }
             post(SH_END, 0, true);
         }
-    } else if (GS && warp >= 4 && warp < 4 + C::NGS) {
+    } else if (GS && !AS && warp >= 4 && warp < 4 + C::NGS) {
         // ------------------------------------------------------------------ GS transform
         const int gq = (warp - 4) % 4, ch = (warp - 4) / 4;  // lane quadrant, key slice (KPW keys)
         constexpr int KPW = C::KPW;
@@ -467,6 +621,9 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                         rr[u] = v;
                 }
             }
+            uint32_t rh[NSUB];  // r' as f16x2 (fp16 fast path)
+#pragma unroll
+            for (int u = 0; u < NSUB; ++u) rh[u] = pack_f16(rr[u], rr[u]);
             // this warp's slice of the X' row (KPW fp16 = KPW/8 chunks of 16 B) into registers first:
             // the loads overlap the wait for a free A buffer
             uint4 xv[KPW / 8];
@@ -491,7 +648,11 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                         const uint32_t xw[4] = {x.x, x.y, x.z, x.w};
 #pragma unroll
                         for (int w = 0; w < 4; ++w) {
-                            if (GS) {  // Y = X' * r'  (fp16 X' -> fp32 -> x r' -> dtype, one rounding)
+                            if (GS && SR_G2_HMUL && !bf) {  // fp16: one packed f16x2 multiply per pair
+                                uint32_t y;
+                                asm("mul.rn.f16x2 %0, %1, %2;" : "=r"(y) : "r"(xw[w]), "r"(rh[u]));
+                                pk[q4 * 4 + w] = y;
+                            } else if (GS) {  // Y = X' * r'  (fp16 X' -> fp32 -> x r' -> dtype, one rounding)
                                 const float2 f = unpack_f16(xw[w]);
                                 float y0, y1;
                                 fmul2(y0, y1, f.x, f.y, rr[u]);
@@ -522,7 +683,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
             if (lane == 0) mbar_arrive(&x_empty[s]);
             if (++s == C::NX) { s = 0; sph ^= 1; }
         }
-    } else if (warp >= 4 + C::NGS && warp < 8 + C::NGS) {
+    } else if (!AS && warp >= 4 + C::NGS && warp < 8 + C::NGS) {
         // ------------------------------------------------------------------ output epilogue
         const int r = (warp % 4) * 32 + lane;
         const uint32_t lane_off = (uint32_t)((warp % 4) * 32) << 16;

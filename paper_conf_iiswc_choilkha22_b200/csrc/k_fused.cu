@@ -60,6 +60,10 @@ __global__ void __launch_bounds__(640, 1)
     griddep_wait();
 
     const int it_begin = __ldg(p.sc.cta_ptr + blockIdx.x), it_end = __ldg(p.sc.cta_ptr + blockIdx.x + 1);
+    // phase 2 applies Global Scaling accumulator-side for fp16 (X' and V share the MMA type; see
+    // g2_body.cuh AS) unless p.gs_prologue; bf16 V needs the prologue form (Y rounded to bf16)
+    // (D = 64: the scaling warps hold D/2 fp32 of O each within the 96-register phase-2 budget)
+    const bool as = D == 64 && p.in_dtype == DT_F16 && !p.gs_prologue;
     PH_MARK(1);
     // ---- phase 1: GEMM1 + LS + IR over the CTA's row-blocks (all 20 warps)
     g1_roles<D, 64, true, false, true>(tmQ, tmK, p, smem, tmem_base, it_begin, it_end);
@@ -76,11 +80,17 @@ __global__ void __launch_bounds__(640, 1)
     if (threadIdx.x == 0) {
         uint64_t* b1 = (uint64_t*)(smem + C1::OFF_BAR);
         for (int i = 0; i < C1::NBAR; ++i) mbar_inval(&b1[i]);
-        g2_init<D, 64, true, true, true>(smem);
+        if (as) g2_init<D, 64, true, true, true, D == 64>(smem);
+        else g2_init<D, 64, true, true, true>(smem);
     }
     __syncthreads();
     // ---- phase 2: GS + GEMM2 over the same row-blocks (warps 0-15; 16-19 idle)
-    g2_roles<D, 64, true, true, true>(tmV, p, smem, tmem_base, it_begin, it_end);
+    if constexpr (D == 64) {
+        if (as) g2_roles<D, 64, true, true, true, true>(tmV, p, smem, tmem_base, it_begin, it_end);
+        else g2_roles<D, 64, true, true, true>(tmV, p, smem, tmem_base, it_begin, it_end);
+    } else {
+        g2_roles<D, 64, true, true, true>(tmV, p, smem, tmem_base, it_begin, it_end);
+    }
     tc_fence_before();
     __syncthreads();
     PH_MARK(3);
@@ -117,6 +127,18 @@ cudaError_t launch_tc_one(const Params& p, cudaStream_t st, int64_t* nl)
 }
 
 }  // namespace sr
+
+#ifdef SR_DIAG_WAITS
+// the fused kernel's phase-1 / phase-2 wait counters (this translation unit's copies)
+extern "C" int sr_diag_read_fused(int phase, unsigned long long* out)  // [20][kDW + 1], reset after read
+{
+    void* sym = nullptr;
+    if (cudaGetSymbolAddress(&sym, phase == 1 ? sr::g_diag_g1 : sr::g_diag_g2) != cudaSuccess) return 1;
+    const size_t n = sizeof(sr::g_diag_g1);
+    if (cudaMemcpy(out, sym, n, cudaMemcpyDeviceToHost) != cudaSuccess) return 1;
+    return cudaMemset(sym, 0, n) != cudaSuccess;
+}
+#endif
 
 #ifdef SR_DIAG_PHASES
 extern "C" int sr_diag_read_phases(unsigned long long* out)  // [1024][5] (diagnostic build)

@@ -78,6 +78,7 @@ struct Params {
     int stages;        // SR_RUN_* bits to launch
     int ir_mode;       // IrMode: where the IR sub-layer runs
     int g1_pair;       // GEMM1 walks pairs of row-blocks sharing each K tile (pair schedule)
+    int gs_prologue;   // one-launch kernel: Global Scaling in GEMM2's prologue even for fp16 (SR_GS_PROLOGUE)
     DevSched sc;
     void* xprime;      // X' tiles (recomposed) or score tiles S (unfused)
     void* pbuf;        // unfused: P tiles

@@ -35,12 +35,12 @@ def _ulp_half(dtype, ref):
 
 def run_case(kind, B, H, S, D, dtype, *, causal=False, kv_len=None, layout=None, window=0, n_global=0,
              tile_n=0, fused=True, seed=0, out_f32=True, fuse_ir=False, ir_kernel=False, one_kernel=False,
-             two_kernels=False):
+             two_kernels=False, gs_prologue=False):
     t, q, k, v = qkv(B, H, S, D, dtype, seed)
     scale = 1 / math.sqrt(D)
     od = torch.float32 if out_f32 else TORCH[dtype]
     kw = dict(scale=scale, causal=causal, tile_n=tile_n, fused=fused, out_dtype=od, fuse_ir=fuse_ir,
-              ir_kernel=ir_kernel, one_kernel=one_kernel, two_kernels=two_kernels)
+              ir_kernel=ir_kernel, one_kernel=one_kernel, two_kernels=two_kernels, gs_prologue=gs_prologue)
     if kind == "dense":
         o = sr.mha_dense(q, k, v, kv_len=kv_len, **kw)
     elif kind == "block":
@@ -373,7 +373,7 @@ FUSED_IR_CASES = [
 ]
 
 
-VARIANTS = ["fuse_ir", "ir_kernel", "one_kernel", "two_kernels"]
+VARIANTS = ["fuse_ir", "ir_kernel", "one_kernel", "two_kernels", "gs_prologue"]
 
 
 @pytest.mark.parametrize("variant", VARIANTS)
@@ -401,7 +401,7 @@ def test_fused_ir_full_configs(idx, variant):
     from tests.gpu_util import to_dev
     q, k, v = (to_dev(x, cfg.dtype) for x in (t.q_s, t.k_s, t.v_s))
     # the two-launch variants at their tuned T = 128 (block-sparse: 64), the default at T = 64
-    tn = 0 if (variant == "one_kernel" or cfg.kind == "blocksparse") else 128
+    tn = 0 if (variant in ("one_kernel", "gs_prologue") or cfg.kind == "blocksparse") else 128
     kw = dict(scale=cfg.scale, out_dtype=torch.float32, tile_n=tn, **{variant: True})
     if cfg.kind == "dense":
         o = sr.mha_dense(q, k, v, kv_len=cfg.kv_len, causal=cfg.causal, **kw)

@@ -28,14 +28,20 @@ variant = sys.argv[2] if len(sys.argv) > 2 else "default"
 reps = int(sys.argv[3]) if len(sys.argv) > 3 else 5
 cfg = W.config(idx)
 L = Layer(cfg, torch.device("cuda", 0), cfg.idx, sr, torch)
-kw = {"fuse_ir": variant == "fuse_ir", "ir_kernel": variant == "ir_kernel"}
+kw = {"fuse_ir": variant == "fuse_ir", "ir_kernel": variant == "ir_kernel", "two_kernels": variant == "two_kernels"}
 lib = sr.lib()
 KDW = 8
 buf = (C.c_ulonglong * (20 * (KDW + 1)))()
 L.run(**kw)
 torch.cuda.synchronize()
 ncta = 148
-for name, bit, fn in (("GEMM1", 1, lib.sr_diag_read_g1), ("GEMM2", 4, lib.sr_diag_read_g2)):
+if variant == "default":  # the one-launch kernel: phase 1 / phase 2 counters of k_fused.cu
+    f1 = lambda b: lib.sr_diag_read_fused(1, b)
+    f2 = lambda b: lib.sr_diag_read_fused(2, b)
+    stages = (("PHASE1 (GEMM1)", 0, f1), ("PHASE2 (GEMM2)", 0, f2))
+else:
+    stages = (("GEMM1", 1, lib.sr_diag_read_g1), ("GEMM2", 4, lib.sr_diag_read_g2))
+for name, bit, fn in stages:
     fn(buf)
     for _ in range(reps):
         L.run(stages=bit, **kw)

@@ -17,7 +17,7 @@ cfg = W.config(idx)
 dev = torch.device("cuda", 0)
 flush = (torch.empty(FLUSH_BYTES, dtype=torch.uint8, device=dev), torch.ones(FLUSH_BYTES // 4, device=dev))
 L = Layer(cfg, dev, cfg.idx, sr, torch)
-modes = {"default": {}, "two_kernels": {"two_kernels": True}, "fused_ir": {"fuse_ir": True},
+modes = {"default": {}, "gs_prologue": {"gs_prologue": True}, "two_kernels": {"two_kernels": True}, "fused_ir": {"fuse_ir": True},
          "ir_kernel": {"ir_kernel": True}, "g1_only": {"stages": 1, "two_kernels": True},
          "g2_only": {"stages": 4, "two_kernels": True}}
 sel = os.environ.get("MODES")
