@@ -138,6 +138,12 @@ DENSE_CASES = [
     ("bf16", 128, 64, 256, True, None),
     ("f16", 64, 128, 512, False, [512, 511, 384, 300, 257, 128, 65, 1]),
     ("f16", 64, 64, 384, True, [384, 100, 1]),
+    # T = 0: the library default (the one-launch kernel; fp16 D = 64 with accumulator-side GS)
+    ("f16", 64, 0, 128, False, None),
+    ("f16", 64, 0, 640, False, None),
+    ("f16", 128, 0, 256, False, None),
+    ("bf16", 64, 0, 512, False, [512, 511, 384, 300, 257, 128, 65, 1]),
+    ("f16", 64, 0, 512, True, [512, 17, 0, 129]),
 ]
 
 
