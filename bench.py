@@ -116,15 +116,16 @@ def alg_bytes_ir_in_gemm1(cfg, stored, T):
 
 def alg_bytes_bwd(cfg, stored, T):
     """Training backward (NEXT-4, include/sr_mha.h sr_mha_*_bwd), algorithmic HBM bytes per kernel:
-    X' is read twice (dS' kernel, dV kernel), dS' written once and read twice (dQ, dK); the dense
+    X' is read twice (dS' kernel, dV kernel), dS' written once and read once (dK; dQ is accumulated
+    in the dS' kernel); the dense
     operands once each; per (row, tile) m' read and r' written then read; per row the statistics."""
     e = 2
     bhsd = cfg.BH * cfg.S * cfg.D
     rt = stored / T
     rows = cfg.BH * cfg.S
     return {"prep": 2 * bhsd * e + 28 * rows,
-            "ds": 2 * bhsd * e + 2 * stored + 4 * rt + 12 * rows + 2 * stored + 4 * rt,
-            "dq": 2 * stored + 2 * bhsd * e,
+            # dS' kernel with dQ fused: + K read and dQ write, no separate dQ pass over dS'
+            "ds": 4 * bhsd * e + 2 * stored + 4 * rt + 12 * rows + 2 * stored + 4 * rt,
             "dk": 2 * stored + 2 * bhsd * e,
             "dv": 2 * stored + 4 * rt + 2 * bhsd * e}
 
@@ -410,7 +411,7 @@ def gpu_arm(args, rank, world, local_rank):
         ms_tr_eager = statistics.mean(timed(torch, L.train_step, K, Wm, flush))
         bb = alg_bytes_bwd(cfg, L.stored, L.T)
         kern_bw = {}
-        for name, bit, keys in (("prep_ds", 1, ("prep", "ds")), ("dq", 2, ("dq",)), ("dk_dv", 4, ("dk", "dv"))):
+        for name, bit, keys in (("prep_ds_dq", 1, ("prep", "ds")), ("dk_dv", 4, ("dk", "dv"))):
             t = statistics.mean(timed(torch, lambda b=bit: L.bwd(stages=b), K, Wm, flush))
             nb = sum(bb[k_] for k_ in keys)
             kern_bw[name] = {"us": round(t * 1e3, 3), "alg_bytes": int(nb), "GB/s": round(nb / (t * 1e-3) / 1e9, 1)}

@@ -176,7 +176,7 @@ sr_status sr_mha_sliding_window_unfused(const void* q, const void* k, const void
  *   dP   = dO V^T                                         (tensor cores, dE/dy)
  *   dS'  = scale * P (dP - delta),  delta_i = sum_d dO_id O_id      (Eq. 3 row form: dE/dx_k =
  *          y_k (dE/dy_k - sum_i dE/dy_i y_i), and sum_j P_ij dP_ij = dO_i . O_i)
- *   dq   = dS' K,   dk = dS'^T Q,   dv = P^T dO          (tensor cores)
+ *   dq   = dS' K (accumulated in the dS' kernel),  dk = dS'^T Q,  dv = P^T dO   (tensor cores)
  *
  * Contract: the call must follow a forward call of the SAME entry point with the same q, k, v,
  * shape, mask / layout, causal, tile_n, in_dtype and out_dtype, in the default mode (flags 0: the
@@ -185,9 +185,9 @@ sr_status sr_mha_sliding_window_unfused(const void* q, const void* k, const void
  * (out_dtype).  dout: DEVICE, [B][H][S][D], in_dtype.  dq, dk, dv: DEVICE, [B][H][S][D],
  * out_dtype, fully overwritten, must not overlap q, k, v, out, dout or each other.  16-bit
  * in_dtype only (SR_ERR_UNSUPPORTED for F32).  ex->flags: 0, or SR_RUN_GEMM1 (row statistics +
- * dS' kernel), SR_RUN_REDUCE (dq kernel), SR_RUN_GEMM2 (dk and dv kernels) for per-kernel timing.
- * Four launches (row statistics, dS', dq, dk + dv), stream-ordered, asynchronous; errors as for
- * the forward. */
+ * dS' + dq kernels), SR_RUN_GEMM2 (dk and dv kernel) for per-kernel timing (SR_RUN_REDUCE: the
+ * separate dq kernel of SR_BWD_DQ_SEPARATE=1 runs only).  Three launches (row statistics, dS' + dq,
+ * dk + dv), stream-ordered, asynchronous; errors as for the forward. */
 sr_status sr_mha_dense_bwd(const void* q, const void* k, const void* v, const void* out, const void* dout,
                            void* dq, void* dk, void* dv, int B, int H, int S, int D, float scale,
                            const sr_dense_mask* mask_or_null, int causal, const sr_exec* ex);

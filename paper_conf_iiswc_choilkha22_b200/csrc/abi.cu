@@ -715,6 +715,10 @@ sr_status run_bwd(sr_entry e, const void* q, const void* k, const void* v, const
     p.dq = dq; p.dk = dk; p.dv = dv;
     p.dsbuf = ws + wi.off_ds;
     p.bstat = (float*)(ws + wi.off_bstat);
+    {   // dQ inside the dS' kernel (default); SR_BWD_DQ_SEPARATE=1 keeps the separate GEMM2-based dQ kernel
+        static const bool sep = [] { const char* e = getenv("SR_BWD_DQ_SEPARATE"); return e && atoi(e) != 0; }();
+        p.bwd_dq_fused = sep ? 0 : 1;
+    }
     int64_t nl = 0;
     cudaError_t ce = launch_tc_bwd(p, (cudaStream_t)ex->stream, &nl);
     g_launches += nl;

@@ -96,6 +96,19 @@ __global__ void __launch_bounds__(kPrepThreads) bwd_prep(const Params p)
         p.bstat[r] = m;
         p.bstat[nrow + r] = d > 0.f ? 1.f / d : 0.f;
         p.bstat[2 * nrow + r] = s_delta[threadIdx.x];
+        if (p.bwd_dq_fused) {  // dQ of a row-block with no listed tile is 0 (the dS' kernel never visits it)
+            const int g = (int)(r / p.S), rb = (int)((r % p.S) / kRowBlock);
+            const int32_t* tp = p.sc.tp + (size_t)lh_of(p.sc, g, p.H) * (p.sc.n_rb + 1);
+            if (__ldg(tp + rb + 1) == __ldg(tp + rb)) {
+                if (p.out_dtype == DT_F32) {
+                    float4* O = reinterpret_cast<float4*>((float*)p.dq + r * D);
+                    for (int c = 0; c < D / 4; ++c) O[c] = make_float4(0.f, 0.f, 0.f, 0.f);
+                } else {
+                    uint4* O = reinterpret_cast<uint4*>((uint16_t*)p.dq + r * D);
+                    for (int c = 0; c < D / 8; ++c) O[c] = make_uint4(0, 0, 0, 0);
+                }
+            }
+        }
     }
 }
 
@@ -103,41 +116,50 @@ __global__ void __launch_bounds__(kPrepThreads) bwd_prep(const Params p)
 struct BHdr {  // per-accumulator macro-tile header (MMA warp -> epilogue)
     int32_t slot_lo, slot_hi, row_lo, row_hi, w0, w1, flags, pad;
 };
-enum : int { BH_TILE = 1, BH_END = 2 };
+enum : int { BH_TILE = 1, BH_END = 2, BH_LAST = 4 };
 
-template <int D>
+// DQ: dQ = dS' K is accumulated in TMEM inside this kernel (a CTA owns whole rows): after the
+// epilogue has written a macro tile's dS' in place, the MMA warp multiplies that shared-memory
+// tile (K-major A operand) by the tile's K rows (MN-major B, own ring loaded by warp 2); the
+// epilogue warpgroup that finished the item's last tile writes the item's dQ rows.  Saves the
+// separate dQ kernel's full re-read of dS'.
+template <int D, bool DQ = false>
 struct BD {
     static constexpr int QB = kRowBlock * D * 2;     // dO tile of a row-block
-    static constexpr int KB = kMWB * D * 2;          // V stage (128 keys)
+    static constexpr int KB = kMWB * D * 2;          // V stage (128 keys); also a K stage (DQ)
     static constexpr int XB = kRowBlock * kMWB * 2;  // X' (then dS') macro tile
     static constexpr int XSB = XB + 2048;            // + m' (2 x 512 B) + slack (1 KB aligned)
-    static constexpr int NQ = D == 64 ? 2 : 1;
-    static constexpr int NK = D == 64 ? 3 : 2;
+    static constexpr int NQ = (D == 64 && !DQ) ? 2 : 1;
+    static constexpr int NK = (D == 64 && !DQ) ? 3 : 2;
+    static constexpr int NKQ = DQ ? (D == 64 ? 2 : 1) : 0;  // K ring of the dQ MMA
     // X' stages: one ring per epilogue warpgroup (macro tile n -> warpgroup n % 2, its stage
     // (n / 2) % NXW).  A ring shared by both warpgroups would let one of them wait on a stage two
     // phases ahead of the other (an mbarrier parity wait cannot tell those phases apart).
-    static constexpr int NX_ = (kSmemMax - 4096 - NQ * QB - NK * KB) / XSB;
+    static constexpr int NX_ = (kSmemMax - 4096 - NQ * QB - (NK + NKQ) * KB) / XSB;
     static constexpr int NX = NX_ >= 4 ? 4 : 2;
     static_assert(NX_ >= 2, "smem budget");
     static constexpr int NXW = NX / 2;
-    static constexpr int NACC = 512 / kMWB;
+    static constexpr int NACC = DQ ? 2 : 512 / kMWB;  // dP accumulators (DQ: + 2 x D columns of dQ)
     static constexpr int OFF_Q = 0;
     static constexpr int OFF_K = OFF_Q + NQ * QB;
-    static constexpr int OFF_X = OFF_K + NK * KB;
+    static constexpr int OFF_KQ = OFF_K + NK * KB;
+    static constexpr int OFF_X = OFF_KQ + NKQ * KB;
     static constexpr int OFF_BAR = OFF_X + NX * XSB;
-    static constexpr int NBAR = 2 * NQ + 2 * NK + 2 * NX + 2 * NACC;
+    // + DQ: kq_full / kq_empty, ds_ready per X' stage, dq_full / dq_empty
+    static constexpr int NBAR = 2 * NQ + 2 * NK + 2 * NX + 2 * NACC + 2 * NKQ + NX + 4;
     static constexpr int OFF_HDR = OFF_BAR + NBAR * 8;
-    static constexpr int OFF_TPTR = OFF_HDR + NACC * (int)sizeof(BHdr);
+    static constexpr int OFF_TPTR = OFF_HDR + (NACC + 2) * (int)sizeof(BHdr);
     static constexpr int SMEM = OFF_TPTR + 16 + 1024;
     static_assert(SMEM <= kSmemMax, "smem budget");
     static constexpr int THREADS = 384;
 };
 
-template <int D, int T>
+template <int D, int T, bool DQ>
 __global__ void __launch_bounds__(384, 1)
-    tc_bwd_ds(const __grid_constant__ CUtensorMap tmO, const __grid_constant__ CUtensorMap tmV, const Params p)
+    tc_bwd_ds(const __grid_constant__ CUtensorMap tmO, const __grid_constant__ CUtensorMap tmV,
+              const __grid_constant__ CUtensorMap tmK, const Params p)
 {
-    using C = BD<D>;
+    using C = BD<D, DQ>;
     constexpr int NSUB = kMWB / T;
     constexpr int XS = kRowBlock * T * 2;  // slot bytes (sub-tile)
     extern __shared__ uint8_t smem_raw[];
@@ -151,18 +173,30 @@ __global__ void __launch_bounds__(384, 1)
     uint64_t* x_empty = x_full + C::NX;
     uint64_t* acc_full = x_empty + C::NX;
     uint64_t* acc_empty = acc_full + C::NACC;
+    uint64_t* kq_full = acc_empty + C::NACC;  // DQ
+    uint64_t* kq_empty = kq_full + C::NKQ;
+    uint64_t* ds_ready = kq_empty + C::NKQ;
+    uint64_t* dq_full = ds_ready + C::NX;
+    uint64_t* dq_empty = dq_full + 2;
     BHdr* hdr = (BHdr*)(smem + C::OFF_HDR);
+    BHdr* dqhdr = hdr + C::NACC;
     uint32_t* tmem_ptr = (uint32_t*)(smem + C::OFF_TPTR);
 
     const int warp = warp_uniform(), lane = threadIdx.x % 32;
     if (threadIdx.x == 0) {
         for (int i = 0; i < C::NQ; ++i) { mbar_init(&q_full[i], 1); mbar_init(&q_empty[i], 1); }
         for (int i = 0; i < C::NK; ++i) { mbar_init(&k_full[i], 1); mbar_init(&k_empty[i], 1); }
-        for (int i = 0; i < C::NX; ++i) { mbar_init(&x_full[i], 1); mbar_init(&x_empty[i], 4); }
+        // x_empty: the epilogue warps once their bulk store has read the dS' (+ the dQ MMA commit)
+        for (int i = 0; i < C::NX; ++i) { mbar_init(&x_full[i], 1); mbar_init(&x_empty[i], DQ ? 5 : 4); }
         for (int i = 0; i < C::NACC; ++i) { mbar_init(&acc_full[i], 2); mbar_init(&acc_empty[i], 4); }
+        for (int i = 0; i < C::NKQ; ++i) { mbar_init(&kq_full[i], 1); mbar_init(&kq_empty[i], 1); }
+        if (DQ) {
+            for (int i = 0; i < C::NX; ++i) mbar_init(&ds_ready[i], 4);
+            for (int i = 0; i < 2; ++i) { mbar_init(&dq_full[i], 2); mbar_init(&dq_empty[i], 4); }
+        }
         fence_mbar_init();
     }
-    if (warp == 0 && lane == 0) { prefetch_tmap(&tmO); prefetch_tmap(&tmV); }
+    if (warp == 0 && lane == 0) { prefetch_tmap(&tmO); prefetch_tmap(&tmV); if (DQ) prefetch_tmap(&tmK); }
     if (warp == 2) tmem_alloc(tmem_ptr, 512);
     tc_fence_before();
     __syncthreads();
@@ -208,6 +242,30 @@ __global__ void __launch_bounds__(384, 1)
                     if (++ks == C::NK) { ks = 0; kph ^= 1; }
                 }
             }
+        } else if (DQ && warp == 2) {
+            // ------------------------------------------------------------------ K producer (dQ)
+            const uint64_t pol_k = policy_evict_last();  // K is re-read by every row-block of its head
+            int ks = 0;
+            uint32_t kph = 0;
+            for (ItemWalk iw(p, it_begin, it_end); iw.more();) {
+                const ItemInfo I = iw.next();
+                for (int t = I.t0; t < I.t1; t += NSUB) {
+                    const int nsub = min(NSUB, I.t1 - t);
+                    int w[NSUB];
+#pragma unroll
+                    for (int s = 0; s < NSUB; ++s) w[s] = s < nsub ? __ldg(p.sc.tinfo + t + s) : 0;
+                    mbar_wait(&kq_empty[ks], kph ^ 1);
+                    if (elect_one()) {
+                        mbar_arrive_expect_tx(&kq_full[ks], nsub * T * D * 2);
+                        for (int s = 0; s < nsub; ++s)
+                            for (int h = 0; h < D / 64; ++h)
+                                tma_load_2d_hint(smem + C::OFF_KQ + ks * C::KB + h * (kMWB * 128) + s * (T * 128), &tmK,
+                                                 h * 64, I.g * p.S + tinfo_kt(w[s]) * T, &kq_full[ks], pol_k);
+                    }
+                    __syncwarp();
+                    if (++ks == C::NKQ) { ks = 0; kph ^= 1; }
+                }
+            }
         } else if (warp == 3) {
             // ------------------------------------------------------------------ X' + m' producer
             const uint64_t pol_x = policy_evict_first();  // X' is streamed
@@ -249,9 +307,43 @@ __global__ void __launch_bounds__(384, 1)
             }
         } else if (warp == 1) {
             // ------------------------------------------------------------------ MMA: dP = dO V^T
+            // (DQ: then, one macro tile behind, dQ += dS' K once the epilogue has written the dS')
             const uint32_t idesc = idesc_f16(p.in_dtype == DT_BF16 ? 1 : 0, kRowBlock, kMWB, 0, 0);
+            const uint32_t idesc_q = idesc_f16(p.in_dtype == DT_BF16 ? 1 : 0, kRowBlock, D, 0, 1);
             int qi = 0, ks = 0, n = 0;
             uint32_t qph = 0, kph = 0;
+            // the pending dQ step: macro tile pn (-1: none), its sub-tile count, item flags and rows
+            int pn = -1, pnsub = 0, pfirst = 0, plast = 0, pitem = 0, qs = 0, nitem = 0;
+            uint32_t qsph = 0;
+            int64_t prow0 = 0;
+            auto dq_step = [&]() {
+                if (!DQ || pn < 0) return;
+                const int sx = (pn % 2) * C::NXW + (pn / 2) % C::NXW;
+                const int b = pitem & 1;  // the pending tile's item: dQ accumulator buffer
+                mbar_wait(&ds_ready[sx], (uint32_t)((pn / 2) / C::NXW) & 1);
+                mbar_wait(&kq_full[qs], qsph);
+                if (pfirst) mbar_wait(&dq_empty[b], ((uint32_t)(pitem >> 1) & 1) ^ 1);
+                tc_fence_after();
+                const uint32_t x_addr = smem_u32(smem + C::OFF_X + sx * C::XSB);
+                const uint32_t k_addr = smem_u32(smem + C::OFF_KQ + qs * C::KB);
+                if (elect_one()) {
+                    for (int kk = 0; kk < pnsub * (T / 16); ++kk) {
+                        const uint64_t ad = smem_desc_sw128(x_addr + (kk / 4) * (kRowBlock * 128) + (kk % 4) * 32, 16, 1024);
+                        const uint64_t bd = smem_desc_sw128(k_addr + kk * 2048, kMWB * 128, 1024);
+                        mma_ss(tmem_base + C::NACC * kMWB + b * D, ad, bd, idesc_q, (pfirst && kk == 0) ? 0u : 1u);
+                    }
+                    mma_commit(&kq_empty[qs]);
+                    mma_commit(&x_empty[sx]);
+                    if (plast) {
+                        dqhdr[b] = BHdr{0, 0, (int32_t)(prow0 & 0xffffffff), (int32_t)(prow0 >> 32), 0, 0, BH_TILE, 0};
+                        mbar_arrive(&dq_full[b]);  // header (arrival 1 of 2)
+                        mma_commit(&dq_full[b]);   // the item's dQ is complete (arrival 2 of 2)
+                    }
+                }
+                __syncwarp();
+                if (++qs == C::NKQ) { qs = 0; qsph ^= 1; }
+                pn = -1;
+            };
             for (ItemWalk iw(p, it_begin, it_end); iw.more();) {
                 const ItemInfo I = iw.next();
                 if (I.t0 == I.t1) continue;
@@ -259,15 +351,17 @@ __global__ void __launch_bounds__(384, 1)
                 mbar_wait(&q_full[qi], qph);
                 tc_fence_after();
                 const uint32_t q_addr = smem_u32(smem + C::OFF_Q + qi * C::QB);
+                ++nitem;
                 for (int t = I.t0; t < I.t1; t += NSUB, ++n) {
                     const int w0 = __ldg(p.sc.tinfo + t);
                     const int w1 = (NSUB > 1 && t + 1 < I.t1) ? __ldg(p.sc.tinfo + t + 1) : -1;
                     const int ab = n % C::NACC;
                     mbar_wait(&acc_empty[ab], ((n / C::NACC) & 1) ^ 1);
                     const int64_t slot = I.slot0 + t;
+                    const bool last = t + NSUB >= I.t1;
                     if (elect_one()) {
                         hdr[ab] = BHdr{(int32_t)(slot & 0xffffffff), (int32_t)(slot >> 32), (int32_t)(row0 & 0xffffffff),
-                                       (int32_t)(row0 >> 32), w0, w1, BH_TILE, 0};
+                                       (int32_t)(row0 >> 32), w0, w1, BH_TILE | (last ? BH_LAST : 0), nitem - 1};
                         mbar_arrive(&acc_full[ab]);  // header published (arrival 1 of 2)
                     }
                     __syncwarp();
@@ -288,11 +382,21 @@ __global__ void __launch_bounds__(384, 1)
                     }
                     __syncwarp();
                     if (++ks == C::NK) { ks = 0; kph ^= 1; }
+                    dq_step();  // the previous macro tile's dQ (its dS' is being / has been written)
+                    if (DQ) {
+                        pn = n;
+                        pnsub = min(NSUB, I.t1 - t);
+                        pfirst = t == I.t0;
+                        plast = last;
+                        prow0 = row0;
+                        pitem = nitem - 1;
+                    }
                 }
                 if (elect_one()) mma_commit(&q_empty[qi]);
                 __syncwarp();
                 if (++qi == C::NQ) { qi = 0; qph ^= 1; }
             }
+            dq_step();  // the last macro tile's dQ
             for (int e = 0; e < 2; ++e, ++n) {  // one END header per epilogue warpgroup
                 const int ab = n % C::NACC;
                 mbar_wait(&acc_empty[ab], ((n / C::NACC) & 1) ^ 1);
@@ -354,7 +458,12 @@ __global__ void __launch_bounds__(384, 1)
             const uint32_t stage_s = smem_u32(stage);
 #pragma unroll
             for (int s = 0; s < NSUB; ++s) {
-                if (!vs[s]) continue;
+                if (!vs[s]) {
+                    if (DQ && wsub[s] != -1)  // rows of an invalid half: zeros, the dQ MMA reads every row
+#pragma unroll
+                        for (int q4 = 0; q4 < T / 8; ++q4) sts128(stage_s + tile_chunk_off(r, s * (T / 8) + q4), 0u, 0u, 0u, 0u);
+                    continue;
+                }
                 const float mp = lds_f32(stage_s + C::XB + s * 512 + 4 * r);
                 // r'_k = e^{m'_k - m} / d (Global Scaling); 0 for a masked sub-vector
                 const float rr = (mp == -INFINITY) ? 0.f : __expf(mp - m_row) * invd_row;
@@ -383,6 +492,7 @@ __global__ void __launch_bounds__(384, 1)
             for (int s = 0; s < NSUB; ++s) wv[s] = __shfl_sync(0xffffffffu, vs[s] ? 1 : 0, 0) != 0;
             fence_proxy_async_smem();
             __syncwarp();
+            if (DQ && lane == 0) mbar_arrive(&ds_ready[sx]);  // the dS' tile is ready for the dQ MMA
             if (lane == 0) {
 #pragma unroll
                 for (int s = 0; s < NSUB; ++s) {
@@ -397,6 +507,38 @@ __global__ void __launch_bounds__(384, 1)
             }
             __syncwarp();
             if (lane == 0) mbar_arrive(&x_empty[sx]);
+            if (DQ && (Hd.flags & BH_LAST)) {  // the item's dQ rows: TMEM -> out dtype -> global
+                const int b = Hd.pad & 1;
+                mbar_wait(&dq_full[b], (uint32_t)(Hd.pad >> 1) & 1);
+                tc_fence_after();
+                const BHdr qh = lds_hdr(dqhdr + b);
+                const int64_t qrow = (((int64_t)qh.row_hi << 32) | (uint32_t)qh.row_lo) + r;
+                const uint32_t taddr = tmem_base + lane_off + C::NACC * kMWB + b * D;
+#pragma unroll
+                for (int c = 0; c < D / 32; ++c) {
+                    uint32_t v[32];
+                    tmem_ld32(taddr + c * 32, v);
+                    tmem_wait_ld();
+                    if (p.out_dtype == DT_F32) {
+                        float4* O = reinterpret_cast<float4*>((float*)p.dq + qrow * D + c * 32);
+#pragma unroll
+                        for (int u = 0; u < 8; ++u)
+                            O[u] = make_float4(__uint_as_float(v[4 * u]), __uint_as_float(v[4 * u + 1]),
+                                               __uint_as_float(v[4 * u + 2]), __uint_as_float(v[4 * u + 3]));
+                    } else {
+                        uint32_t pk[16];
+#pragma unroll
+                        for (int u = 0; u < 16; ++u)
+                            pk[u] = pack16(__uint_as_float(v[2 * u]), __uint_as_float(v[2 * u + 1]), p.out_dtype == DT_BF16);
+                        uint4* O = reinterpret_cast<uint4*>((uint16_t*)p.dq + qrow * D + c * 32);
+#pragma unroll
+                        for (int u = 0; u < 4; ++u) O[u] = make_uint4(pk[4 * u], pk[4 * u + 1], pk[4 * u + 2], pk[4 * u + 3]);
+                    }
+                }
+                tc_fence_before();
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&dq_empty[b]);
+            }
         }
         if (lane == 0) bulk_wait0();
     }
@@ -690,16 +832,19 @@ cudaError_t launch_bwd_d(const Params& p, cudaStream_t st, int64_t* nl)
         if ((e = launch_pdl(bwd_prep<D>, dim3((unsigned)((rows + rpb - 1) / rpb)), dim3(kPrepThreads), 0, st, nl, p)) !=
             cudaSuccess)
             return e;
-        CUtensorMap to, tv;
+        CUtensorMap to, tv, tk;
         if ((e = make_tmap_2d(&to, p.dout, rows, D, kRowBlock, p.in_dtype)) != cudaSuccess) return e;
         if ((e = make_tmap_2d(&tv, p.v, rows, D, p.T, p.in_dtype)) != cudaSuccess) return e;
-        auto kern = p.T == 64 ? tc_bwd_ds<D, 64> : tc_bwd_ds<D, 128>;
-        if ((e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, BD<D>::SMEM)) != cudaSuccess)
+        if ((e = make_tmap_2d(&tk, p.k, rows, D, p.T, p.in_dtype)) != cudaSuccess) return e;
+        auto kern = p.bwd_dq_fused ? (p.T == 64 ? tc_bwd_ds<D, 64, true> : tc_bwd_ds<D, 128, true>)
+                                   : (p.T == 64 ? tc_bwd_ds<D, 64, false> : tc_bwd_ds<D, 128, false>);
+        const int smem = p.bwd_dq_fused ? BD<D, true>::SMEM : BD<D, false>::SMEM;
+        if ((e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess)
             return e;
-        if ((e = launch_pdl(kern, dim3(p.sc.n_cta), dim3(BD<D>::THREADS), BD<D>::SMEM, st, nl, to, tv, p)) != cudaSuccess)
+        if ((e = launch_pdl(kern, dim3(p.sc.n_cta), dim3(BD<D>::THREADS), smem, st, nl, to, tv, tk, p)) != cudaSuccess)
             return e;
     }
-    if (p.stages & 2) {  // dQ = dS' K: GEMM2 in its plain mode, A = dS' tiles, B = K
+    if ((p.stages & 2) && !p.bwd_dq_fused) {  // dQ = dS' K: GEMM2 in its plain mode, A = dS' tiles, B = K
         Params p2 = p;
         p2.pbuf = p.dsbuf;
         p2.v = p.k;

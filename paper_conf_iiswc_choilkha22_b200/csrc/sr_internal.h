@@ -93,6 +93,7 @@ struct Params {
     void* dv;
     void* dsbuf;       // dS' = scale * dE/dx tiles (in_dtype), same slots and layout as X'
     float* bstat;      // [3][B*H*S]: per query row m (natural log), 1/d, delta = sum_d dO * O
+    int bwd_dq_fused;  // dQ accumulated inside the dS' kernel (default; SR_BWD_DQ_SEPARATE=1: own kernel)
 };
 
 __host__ __device__ inline int lh_of(const DevSched& s, int g, int H)

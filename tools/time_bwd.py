@@ -21,6 +21,6 @@ L.setup_train(cfg.idx)
 L.train_step()
 res = {"fwd": statistics.median(timed(torch, L.fwd_train, K, 3, flush)),
        "bwd": statistics.median(timed(torch, L.bwd, K, 3, flush))}
-for name, st in (("prep_ds", 1), ("dq", 2), ("dk_dv", 4)):
+for name, st in (("prep_ds_dq", 1), ("dq_separate", 2), ("dk_dv", 4)):
     res[name] = statistics.median(timed(torch, lambda: L.bwd(stages=st), K, 3, flush))
 print(os.environ.get("TAG", ""), f"C{idx}", " ".join(f"{k}={v * 1e3:.1f}us" for k, v in res.items()))
