@@ -561,8 +561,14 @@ struct BK {
     static constexpr int AB = kRowBlock * kMWB * 2;  // A: [2 key chunks of 64][128 rows][64] = 32 KB
     static constexpr int BB = kRowBlock * D * 2;     // B: Q (dK) or dO (dV) rows of the row-block
     static constexpr int SB = AB + BB + 2048;        // + r' (2 x 512 B) + header, 1 KB aligned
-    static constexpr int NS_ = (kSmemMax - 4096) / SB;
+    // D = 64: two stages, so that a dV CTA and a dK CTA fit on one SM together (smem < 113 KB,
+    // TMEM 128 columns each) and overlap each other's latencies; D = 128: as deep as smem allows
+#ifndef SR_BWD_KV_NS64
+#define SR_BWD_KV_NS64 2
+#endif
+    static constexpr int NS_ = D == 64 ? SR_BWD_KV_NS64 : (kSmemMax - 4096) / SB;
     static constexpr int NS = NS_ > 4 ? 4 : NS_;
+    static constexpr uint32_t TMEM_COLS = 2 * D < 32 ? 32 : 2 * D;  // two D-column accumulators
     static_assert(NS >= 2, "smem budget");
     static constexpr int OFF_BAR = NS * SB;
     static constexpr int NBAR = 3 * NS + 4;
@@ -605,7 +611,7 @@ __global__ void __launch_bounds__(384, 1)
         fence_mbar_init();
     }
     if (warp == 0 && lane == 0) prefetch_tmap(&tmB);
-    if (warp == 2) tmem_alloc(tmem_ptr, 256);
+    if (warp == 2) tmem_alloc(tmem_ptr, C::TMEM_COLS);
     tc_fence_before();
     __syncthreads();
     tc_fence_after();
@@ -816,7 +822,7 @@ __global__ void __launch_bounds__(384, 1)
     __syncthreads();
     if (warp == 2) {
         tc_fence_after();
-        tmem_dealloc(tmem_base, 256);
+        tmem_dealloc(tmem_base, C::TMEM_COLS);
     }
 }
 
