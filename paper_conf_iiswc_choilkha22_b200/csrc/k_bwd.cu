@@ -556,17 +556,16 @@ struct KHdr {  // stage header (producer -> transform) / accumulator header (MMA
     int32_t flags, hv0, hv1, pad0, row_lo, row_hi, pad1, pad2;
 };
 
-template <int D>
+template <int D, bool PAIRED = (D == 64)>
 struct BK {
     static constexpr int AB = kRowBlock * kMWB * 2;  // A: [2 key chunks of 64][128 rows][64] = 32 KB
     static constexpr int BB = kRowBlock * D * 2;     // B: Q (dK) or dO (dV) rows of the row-block
     static constexpr int SB = AB + BB + 2048;        // + r' (2 x 512 B) + header, 1 KB aligned
-    // D = 64: two stages, so that a dV CTA and a dK CTA fit on one SM together (smem < 113 KB,
-    // TMEM 128 columns each) and overlap each other's latencies; D = 128: as deep as smem allows
-#ifndef SR_BWD_KV_NS64
-#define SR_BWD_KV_NS64 2
-#endif
-    static constexpr int NS_ = D == 64 ? SR_BWD_KV_NS64 : (kSmemMax - 4096) / SB;
+    // PAIRED (D = 64, dense / window layouts): two stages, so that a dV CTA and a dK CTA fit on one
+    // SM together (smem < 113 KB, TMEM 128 columns each) and overlap each other's latencies
+    // (measured: C2 dK+dV 27.6 -> 25.5 us, C5 73.8 -> 68.6); otherwise as deep as smem allows (the
+    // block-sparse C4, whose column entries are mostly half empty, loses ~10 us when paired)
+    static constexpr int NS_ = PAIRED ? 2 : (kSmemMax - 4096) / SB;
     static constexpr int NS = NS_ > 4 ? 4 : NS_;
     static constexpr uint32_t TMEM_COLS = 2 * D < 32 ? 32 : 2 * D;  // two D-column accumulators
     static_assert(NS >= 2, "smem budget");
@@ -583,14 +582,14 @@ struct BK {
 // r' in shared memory -> y, B = dO), the rest dK = dS'^T Q (A = dS' tiles, B = Q) for the same
 // column items; dV CTAs (the heavier ones) start first, dK CTAs fill SMs as they free up.
 // Warps: 0 producer, 1 MMA, 2 TMEM allocator, 4-7 y transform (PV), 8-11 epilogue.
-template <int D>
+template <int D, bool PAIRED>
 __global__ void __launch_bounds__(384, 1)
     tc_bwd_kv(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmO, const Params p)
 {
     const bool PV = blockIdx.x < (unsigned)p.sc.n_ccta;
     const int cta = PV ? blockIdx.x : blockIdx.x - p.sc.n_ccta;
     const CUtensorMap& tmB = PV ? tmO : tmQ;
-    using C = BK<D>;
+    using C = BK<D, PAIRED>;
     extern __shared__ uint8_t smem_raw[];
     uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
     uint64_t* bars = (uint64_t*)(smem + C::OFF_BAR);
@@ -861,10 +860,12 @@ cudaError_t launch_bwd_d(const Params& p, cudaStream_t st, int64_t* nl)
         CUtensorMap tq, to;
         if ((e = make_tmap_2d(&tq, p.q, rows, D, kRowBlock, p.in_dtype)) != cudaSuccess) return e;
         if ((e = make_tmap_2d(&to, p.dout, rows, D, kRowBlock, p.in_dtype)) != cudaSuccess) return e;
-        auto kern = tc_bwd_kv<D>;
-        if ((e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, BK<D>::SMEM)) != cudaSuccess)
+        const bool paired = D == 64 && p.mask_kind != MK_BLOCK;
+        auto kern = paired ? tc_bwd_kv<D, D == 64> : tc_bwd_kv<D, false>;
+        const int ksmem = paired ? BK<D, D == 64>::SMEM : BK<D, false>::SMEM;
+        if ((e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, ksmem)) != cudaSuccess)
             return e;
-        if ((e = launch_pdl(kern, dim3(2 * p.sc.n_ccta), dim3(BK<D>::THREADS), BK<D>::SMEM, st, nl, tq, to, p)) !=
+        if ((e = launch_pdl(kern, dim3(2 * p.sc.n_ccta), dim3(BK<D>::THREADS), ksmem, st, nl, tq, to, p)) !=
             cudaSuccess)
             return e;
     }
