@@ -53,6 +53,16 @@ __global__ void __launch_bounds__(kPrepThreads) bwd_prep(const Params p)
     const int64_t row0 = (int64_t)blockIdx.x * RPB;
     const int64_t row = row0 + threadIdx.x / TPR;
     const int c = threadIdx.x % TPR;
+    // the statistics threads issue their IR-partial loads first, so the two memory round trips of a
+    // block (dO / O, then rowstat) overlap instead of running back to back
+    const int64_t rs = row0 + threadIdx.x;
+    float ma = -INFINITY, da = 0.f, mb = -INFINITY, db = 0.f;
+    if (threadIdx.x < RPB && rs < nrow) {
+        ma = __ldcg(p.rowstat + rs);
+        da = __ldcg(p.rowstat + nrow + rs);
+        mb = __ldcg(p.rowstat + 2 * nrow + rs);
+        db = __ldcg(p.rowstat + 3 * nrow + rs);
+    }
     float acc = 0.f;
     if (row < nrow) {
         const bool bf = p.in_dtype == DT_BF16;
@@ -87,10 +97,8 @@ __global__ void __launch_bounds__(kPrepThreads) bwd_prep(const Params p)
     if (c == 0) s_delta[threadIdx.x / TPR] = acc;
     __syncthreads();
     // per-row statistics with one thread per row: coalesced loads of the IR partials and stores
-    if (threadIdx.x < RPB && row0 + threadIdx.x < nrow) {
-        const int64_t r = row0 + threadIdx.x;
-        const float ma = __ldcg(p.rowstat + r), da = __ldcg(p.rowstat + nrow + r);
-        const float mb = __ldcg(p.rowstat + 2 * nrow + r), db = __ldcg(p.rowstat + 3 * nrow + r);
+    if (threadIdx.x < RPB && rs < nrow) {
+        const int64_t r = rs;
         const float m = fmaxf(ma, mb);  // m = max_w m_w, d = sum_w e^{m_w - m} d_w
         const float d = m == -INFINITY ? 0.f : da * __expf(ma - m) + db * __expf(mb - m);
         p.bstat[r] = m;
