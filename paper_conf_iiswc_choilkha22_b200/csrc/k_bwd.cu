@@ -46,7 +46,8 @@ __global__ void __launch_bounds__(kPrepThreads) bwd_prep(const Params p)
 {
     griddep_launch_dependents();
     griddep_wait();
-    constexpr int TPR = D / 8;                 // threads per row (16 B of dO each)
+    constexpr int TPR = 8;                     // threads per row
+    constexpr int EPT = D / TPR;               // elements per thread (8 or 16: one or two 16-B loads)
     constexpr int RPB = kPrepThreads / TPR;    // rows per block
     __shared__ float s_delta[RPB];
     const int64_t nrow = (int64_t)p.B * p.H * p.S;
@@ -66,31 +67,46 @@ __global__ void __launch_bounds__(kPrepThreads) bwd_prep(const Params p)
     float acc = 0.f;
     if (row < nrow) {
         const bool bf = p.in_dtype == DT_BF16;
-        const uint4 g = __ldg(reinterpret_cast<const uint4*>((const uint16_t*)p.dout + row * D) + c);
-        float gd[8], od[8];
-        const uint32_t gw[4] = {g.x, g.y, g.z, g.w};
+        uint4 g[EPT / 8], o16[EPT / 8];
+        float4 o32[EPT / 4];
 #pragma unroll
-        for (int w = 0; w < 4; ++w) {
-            const float2 f = unpack16(gw[w], bf);
-            gd[2 * w] = f.x;
-            gd[2 * w + 1] = f.y;
-        }
+        for (int k = 0; k < EPT / 8; ++k)  // chunk c + k * TPR of the row: coalesced across the row's threads
+            g[k] = __ldg(reinterpret_cast<const uint4*>((const uint16_t*)p.dout + row * D) + c + k * TPR);
         if (p.out_dtype == DT_F32) {
-            const float4* o4 = reinterpret_cast<const float4*>((const float*)p.out + row * D) + 2 * c;
-            const float4 a = __ldg(o4), b = __ldg(o4 + 1);
-            od[0] = a.x; od[1] = a.y; od[2] = a.z; od[3] = a.w; od[4] = b.x; od[5] = b.y; od[6] = b.z; od[7] = b.w;
+#pragma unroll
+            for (int k = 0; k < EPT / 8; ++k) {
+                const float4* o4 = reinterpret_cast<const float4*>((const float*)p.out + row * D) + 2 * (c + k * TPR);
+                o32[2 * k] = __ldg(o4);
+                o32[2 * k + 1] = __ldg(o4 + 1);
+            }
         } else {
-            const uint4 o = __ldg(reinterpret_cast<const uint4*>((const uint16_t*)p.out + row * D) + c);
-            const uint32_t ow[4] = {o.x, o.y, o.z, o.w};
+#pragma unroll
+            for (int k = 0; k < EPT / 8; ++k)
+                o16[k] = __ldg(reinterpret_cast<const uint4*>((const uint16_t*)p.out + row * D) + c + k * TPR);
+        }
+#pragma unroll
+        for (int k = 0; k < EPT / 8; ++k) {
+            const uint32_t gw[4] = {g[k].x, g[k].y, g[k].z, g[k].w};
+            float od[8];
+            if (p.out_dtype == DT_F32) {
+                const float4 a = o32[2 * k], b = o32[2 * k + 1];
+                od[0] = a.x; od[1] = a.y; od[2] = a.z; od[3] = a.w; od[4] = b.x; od[5] = b.y; od[6] = b.z; od[7] = b.w;
+            } else {
+                const uint32_t ow[4] = {o16[k].x, o16[k].y, o16[k].z, o16[k].w};
+#pragma unroll
+                for (int w = 0; w < 4; ++w) {
+                    const float2 f = unpack16(ow[w], p.out_dtype == DT_BF16);
+                    od[2 * w] = f.x;
+                    od[2 * w + 1] = f.y;
+                }
+            }
 #pragma unroll
             for (int w = 0; w < 4; ++w) {
-                const float2 f = unpack16(ow[w], p.out_dtype == DT_BF16);
-                od[2 * w] = f.x;
-                od[2 * w + 1] = f.y;
+                const float2 f = unpack16(gw[w], bf);
+                acc = fmaf(f.x, od[2 * w], acc);
+                acc = fmaf(f.y, od[2 * w + 1], acc);
             }
         }
-#pragma unroll
-        for (int j = 0; j < 8; ++j) acc = fmaf(gd[j], od[j], acc);
     }
 #pragma unroll
     for (int o = TPR / 2; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
@@ -841,7 +857,7 @@ cudaError_t launch_bwd_d(const Params& p, cudaStream_t st, int64_t* nl)
     cudaError_t e;
     const int64_t rows = (int64_t)p.B * p.H * p.S;
     if (p.stages & 1) {
-        const int64_t rpb = kPrepThreads / (D / 8);
+        const int64_t rpb = kPrepThreads / 8;
         if ((e = launch_pdl(bwd_prep<D>, dim3((unsigned)((rows + rpb - 1) / rpb)), dim3(kPrepThreads), 0, st, nl, p)) !=
             cudaSuccess)
             return e;
