@@ -40,14 +40,17 @@ __device__ __forceinline__ uint32_t pack16(float a, float b, bool bf) { return b
 // prologue merges them), bstat[2][row] = delta = sum_d dO[row, d] * O[row, d].  D/8 threads per
 // row for the dot product (16 B of dO each), then one thread per row for the statistics.
 constexpr int kPrepThreads = 512;
+#ifndef SR_PREP_TPR
+#define SR_PREP_TPR 8  // threads per row of bwd_prep (measured on C3: 8 -> 16 us, 16 -> 23 us, 4 -> 21 us)
+#endif
 
 template <int D>
 __global__ void __launch_bounds__(kPrepThreads) bwd_prep(const Params p)
 {
     griddep_launch_dependents();
     griddep_wait();
-    constexpr int TPR = 8;                     // threads per row
-    constexpr int EPT = D / TPR;               // elements per thread (8 or 16: one or two 16-B loads)
+    constexpr int TPR = SR_PREP_TPR;           // threads per row
+    constexpr int EPT = D / TPR;               // elements per thread (16-B loads of 8)
     constexpr int RPB = kPrepThreads / TPR;    // rows per block
     __shared__ float s_delta[RPB];
     const int64_t nrow = (int64_t)p.B * p.H * p.S;
@@ -857,7 +860,7 @@ cudaError_t launch_bwd_d(const Params& p, cudaStream_t st, int64_t* nl)
     cudaError_t e;
     const int64_t rows = (int64_t)p.B * p.H * p.S;
     if (p.stages & 1) {
-        const int64_t rpb = kPrepThreads / 8;
+        const int64_t rpb = kPrepThreads / SR_PREP_TPR;
         if ((e = launch_pdl(bwd_prep<D>, dim3((unsigned)((rows + rpb - 1) / rpb)), dim3(kPrepThreads), 0, st, nl, p)) !=
             cudaSuccess)
             return e;
