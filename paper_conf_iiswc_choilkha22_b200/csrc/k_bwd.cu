@@ -445,6 +445,7 @@ __global__ void __launch_bounds__(384, 1)
         const int wrow0 = (warp % 4) * 32;
         const bool bf = p.in_dtype == DT_BF16;
         const int64_t nrow = (int64_t)p.B * p.H * p.S;
+        const uint64_t pol_ds = policy_evict_first();
         int64_t cur = -1;
         float m_row = 0.f, invd_row = 0.f, delta_row = 0.f;
         for (int n = e;; n += 2) {
@@ -526,8 +527,10 @@ __global__ void __launch_bounds__(384, 1)
                     if (!wv[s]) continue;  // a warp's 32 rows lie in one 64-row half
                     uint8_t* dst = (uint8_t*)p.dsbuf + (slot + s) * (int64_t)XS;
                     for (int ch = 0; ch < T / 64; ++ch)
-                        bulk_store(dst + ch * (kRowBlock * 128) + wrow0 * 128,
-                                   stage + (s * (T / 64) + ch) * (kRowBlock * 128) + wrow0 * 128, 32 * 128);
+                        // evict_first: dS' (as large as X') is re-read only by the next kernel; keep
+                        // the L2 for the V / K tiles every row-block of the head re-reads
+                        bulk_store_hint(dst + ch * (kRowBlock * 128) + wrow0 * 128,
+                                        stage + (s * (T / 64) + ch) * (kRowBlock * 128) + wrow0 * 128, 32 * 128, pol_ds);
                 }
                 bulk_commit();
                 bulk_wait_read0();  // the stage is recycled once the store has read it
