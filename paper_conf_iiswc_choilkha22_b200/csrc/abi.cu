@@ -390,7 +390,7 @@ void lpt_assign(HostSched& h, int n_cta)
         const int g = h.pitems[i] / h.n_pair, j = h.pitems[i] % h.n_pair;
         const int32_t* tp = &h.tp[(size_t)lh_of_g(g) * (h.n_rb + 1)];
         const int rb1 = std::min(2 * j + 2, h.n_rb);
-        pcost[i] = 2 * (int64_t)(tp[rb1] - tp[2 * j]) + 1;
+        pcost[i] = 2 * (int64_t)(tp[rb1] - tp[2 * j]) + 2 * lpt_item_cost();
     }
     lpt_assign(h.pitems, pcost, n_cta, h.pcta_ptr);
     std::vector<int64_t> ccost(h.citems.size());
@@ -429,7 +429,8 @@ sr_status host_sched(const Request& r, std::shared_ptr<CachedSched>& out, bool n
         const size_t n_pit = h.pitems.size();
         size_t bytes = sizeof(int32_t) * (4 * n_it + 4 * n_pit + h.pent.size() + 4 + n_tp + n_ti + n_it + n_kv +
                                           h.cta_ptr.size() + h.pp.size() + h.pcta_ptr.size() + 4 +
-                                          4 * h.citems.size() + h.cent.size() + 4 + h.ccta_ptr.size());
+                                          4 * h.citems.size() + h.cent.size() + 4 + h.ccta_ptr.size() +
+                                          8 * n_pit + h.pcta_ptr.size() + 4);
         cudaError_t ce = cudaMalloc(&cs->dmem, bytes);
         if (ce != cudaSuccess) return fail(SR_ERR_CUDA, "cudaMalloc(schedule): %s", cudaGetErrorString(ce));
         std::vector<int32_t> blob;
@@ -447,6 +448,21 @@ sr_status host_sched(const Request& r, std::shared_ptr<CachedSched>& out, bool n
             const int32_t* pp = &h.pp[(size_t)lh * (h.n_pair + 1)];
             blob.insert(blob.end(), {w, pp[j], pp[j + 1], h.tp[(size_t)lh * (h.n_rb + 1)]});
         }
+        size_t o_fp = blob.size();  // pair assignment as row-block item descriptors
+        std::vector<int32_t> fpcta(1, 0);
+        for (size_t c = 0; c + 1 < h.pcta_ptr.size(); ++c) {
+            for (int i = h.pcta_ptr[c]; i < h.pcta_ptr[c + 1]; ++i) {
+                const int w = h.pitems[i], g = w / h.n_pair, j = w % h.n_pair;
+                const int lh = h.lh_mode == LH_ONE ? 0 : (h.lh_mode == LH_BATCH ? g / h.H : g % h.H);
+                const int32_t* tp = &h.tp[(size_t)lh * (h.n_rb + 1)];
+                for (int rb = 2 * j; rb < std::min(2 * j + 2, h.n_rb); ++rb)
+                    blob.insert(blob.end(), {g * h.n_rb + rb, tp[rb], tp[rb + 1], tp[0]});
+            }
+            fpcta.push_back((int32_t)((blob.size() - o_fp) / 4));
+        }
+        size_t o_fpc = blob.size();
+        blob.insert(blob.end(), fpcta.begin(), fpcta.end());
+        while (blob.size() % 4) blob.push_back(0);  // the int4 arrays below stay 16-B aligned
         size_t o_cd = blob.size();  // column item descriptors {g * n_cb + c, e0, e1, tp[lh][0]}
         for (int32_t w : h.citems) {
             const int g = w / h.n_cb, c = w % h.n_cb;
@@ -497,6 +513,8 @@ sr_status host_sched(const Request& r, std::shared_ptr<CachedSched>& out, bool n
         cs->dev.pcta_ptr = base + o_pcp;
         cs->dev.n_pair = h.n_pair;
         cs->dev.n_pcta = (int)h.pcta_ptr.size() - 1;
+        cs->dev.fp_desc = (const int4*)(base + o_fp);
+        cs->dev.fpcta_ptr = base + o_fpc;
         cs->dev.col_desc = (const int4*)(base + o_cd);
         cs->dev.cent = (const int4*)(base + o_ce);
         cs->dev.ccta_ptr = base + o_ccp;
@@ -632,7 +650,13 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
     if (fused == 2) {
         ce = launch_tc_sd(p, st, &nl);
     } else if (fused && one) {
-        p.g1_pair = 0;
+        // pairs of row-blocks sharing each K tile in phase 1 (same choice as the two-kernel chain:
+        // D = 128 with enough pairs); phase 2 then walks the pair assignment as row-block items
+        if (p.g1_pair) {
+            p.sc.item_desc = cs->dev.fp_desc;
+            p.sc.cta_ptr = cs->dev.fpcta_ptr;
+            p.sc.n_cta = cs->dev.n_pcta;
+        }
         p.gs_prologue = (ex->flags & SR_GS_PROLOGUE) != 0;
 
         ce = launch_tc_one(p, st, &nl);

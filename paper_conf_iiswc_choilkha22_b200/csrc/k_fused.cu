@@ -36,12 +36,12 @@ __device__ __forceinline__ unsigned long long gtimer()
 #define PH_MARK(i)
 #endif
 
-template <int D>
+template <int D, bool PAIR>
 __global__ void __launch_bounds__(640, 1)
     tc_fused(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmK,
              const __grid_constant__ CUtensorMap tmV, const Params p)
 {
-    using C1 = G1<D, 64, false>;
+    using C1 = G1<D, 64, PAIR>;
     using C2 = G2<D, 64>;
     static_assert(C1::THREADS == 640 && C2::THREADS <= 640, "warp budget");
     extern __shared__ uint8_t smem_raw[];
@@ -49,7 +49,7 @@ __global__ void __launch_bounds__(640, 1)
     uint32_t* tmem_ptr = (uint32_t*)(smem + C1::OFF_TPTR);
     const int warp = warp_uniform(), lane = threadIdx.x % 32;
     PH_MARK(0);
-    if (threadIdx.x == 0) g1_init<D, 64, true, false, true>(smem);
+    if (threadIdx.x == 0) g1_init<D, 64, true, PAIR, true>(smem);
     if (warp == 0 && lane == 0) { prefetch_tmap(&tmQ); prefetch_tmap(&tmK); prefetch_tmap(&tmV); }
     if (warp == 2) tmem_alloc(tmem_ptr, 512);
     tc_fence_before();
@@ -59,6 +59,8 @@ __global__ void __launch_bounds__(640, 1)
     griddep_launch_dependents();
     griddep_wait();
 
+    // phase 2's row-blocks (with PAIR the host pointed cta_ptr / item_desc at the pair assignment
+    // unrolled into row-blocks, so both phases cover the same rows)
     const int it_begin = __ldg(p.sc.cta_ptr + blockIdx.x), it_end = __ldg(p.sc.cta_ptr + blockIdx.x + 1);
     // phase 2 applies Global Scaling accumulator-side for fp16 (X' and V share the MMA type; see
     // g2_body.cuh AS) unless p.gs_prologue; bf16 V needs the prologue form (Y rounded to bf16)
@@ -66,7 +68,11 @@ __global__ void __launch_bounds__(640, 1)
     const bool as = D == 64 && p.in_dtype == DT_F16 && !p.gs_prologue;
     PH_MARK(1);
     // ---- phase 1: GEMM1 + LS + IR over the CTA's row-blocks (all 20 warps)
-    g1_roles<D, 64, true, false, true>(tmQ, tmK, p, smem, tmem_base, it_begin, it_end);
+    if constexpr (PAIR)
+        g1_roles<D, 64, true, true, true>(tmQ, tmK, p, smem, tmem_base, __ldg(p.sc.pcta_ptr + blockIdx.x),
+                                          __ldg(p.sc.pcta_ptr + blockIdx.x + 1));
+    else
+        g1_roles<D, 64, true, false, true>(tmQ, tmK, p, smem, tmem_base, it_begin, it_end);
     // back to the launch split (phase 1 leaves warps 0-3 at 64 registers, the epilogue at 104)
     if (warp < 4) reg_alloc<96>();
     else reg_dealloc<96>();
@@ -114,8 +120,10 @@ cudaError_t launch_one_d(const Params& p, cudaStream_t st, int64_t* nl)
     if ((e = make_tmap_2d(&tq, p.q, rows, D, kRowBlock, p.in_dtype)) != cudaSuccess) return e;
     if ((e = make_tmap_2d(&tk, p.k, rows, D, 64, p.in_dtype)) != cudaSuccess) return e;
     if ((e = make_tmap_2d(&tv, p.v, rows, D, 64, p.in_dtype)) != cudaSuccess) return e;
-    constexpr int smem = G1<D, 64, false>::SMEM > G2<D, 64>::SMEM ? G1<D, 64, false>::SMEM : G2<D, 64>::SMEM;
-    auto kern = tc_fused<D>;
+    constexpr int s0 = G1<D, 64, false>::SMEM > G2<D, 64>::SMEM ? G1<D, 64, false>::SMEM : G2<D, 64>::SMEM;
+    constexpr int s1 = G1<D, 64, true>::SMEM > G2<D, 64>::SMEM ? G1<D, 64, true>::SMEM : G2<D, 64>::SMEM;
+    auto kern = p.g1_pair ? tc_fused<D, true> : tc_fused<D, false>;
+    const int smem = p.g1_pair ? s1 : s0;
     if ((e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
     return launch_pdl(kern, dim3(p.sc.n_cta), dim3(640), smem, st, nl, tq, tk, tv, p);
 }

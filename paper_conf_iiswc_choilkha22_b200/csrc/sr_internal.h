@@ -47,6 +47,10 @@ struct DevSched {
     const int4* pent;
     const int32_t* pcta_ptr;
     int n_pair, n_pcta;
+    // the same pair assignment as row-block items (one-launch kernel with pairs: phase 2 walks the
+    // row-blocks its phase 1 produced): fp_desc in item_desc format, grouped per CTA by fpcta_ptr
+    const int4* fp_desc;
+    const int32_t* fpcta_ptr;
     const int32_t* kv_len;  // [B] or nullptr
     int n_rb, n_lh, lh_mode, slots_per_head, n_items, n_cta;
     int max_rb_tiles;       // longest tile list of one (layout head, row-block)
