@@ -144,3 +144,27 @@ def test_backward_deterministic():
         outs.append(got)
     for a, b in zip(*outs):
         assert np.array_equal(a, b)
+
+
+def test_separate_dq_kernel():
+    """SR_BWD_DQ_SEPARATE=1 (read once per process, so it runs in its own interpreter): dQ from its
+    own kernel (the plain GEMM2 on dS' and K) instead of inside the dS' kernel."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    script = r"""
+from tests.test_gpu_backward import run_bwd, check
+import workloads as W
+for kind, kw in (("dense", dict(B=2, H=2, S=384, D=64, dtype="f16", causal=True, kv_len=[384, 0])),
+                 ("dense", dict(B=1, H=2, S=256, D=128, dtype="bf16")),
+                 ("block", dict(B=1, H=2, S=512, D=64, dtype="f16", layout=W.random_layout(2, 8, 64, 0.35, seed=5)))):
+    kw = dict(kw)
+    B, H, S, D, dt = (kw.pop(x) for x in ("B", "H", "S", "D", "dtype"))
+    got, ref = run_bwd(kind, B, H, S, D, dt, **kw)
+    check(got, ref, dt, what=kind)
+print("ok")
+"""
+    env = dict(os.environ, SR_BWD_DQ_SEPARATE="1", PYTHONPATH=root)
+    r = subprocess.run([sys.executable, "-c", script], cwd=root, env=env, capture_output=True, text=True, timeout=240)
+    assert r.returncode == 0 and "ok" in r.stdout, r.stdout[-2000:] + r.stderr[-4000:]
