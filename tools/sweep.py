@@ -2,8 +2,9 @@
 sequence length L and batch size -- plus GPT-Neo's local-attention layers (window 256, causal) as a
 second GPT-Neo workload (GPT-Neo alternates global and local attention).
 
-For every point: attention layers/s of the default recomposed path (GEMM1+LS+IR -> GS+GEMM2) and
-of the in-repo unfused baseline (GEMM1 -> row softmax -> GEMM2), the speedup, the algorithmic HBM
+For every point: attention layers/s of the default recomposed path (one launch: GEMM1+LS+IR then
+GS+GEMM2 per CTA) and of the in-repo unfused baseline (GEMM1 -> row softmax -> GEMM2), each as one
+L2-flushed call, the speedup, the algorithmic HBM
 bytes of both, and a parity spot check of 48 sampled rows against the fp64 oracle (fp32 context,
 tolerance 1e-2 as in tests/).  The paper reports whole-model speedups on A100 (context only); this
 measures the attention layer itself.
@@ -87,7 +88,7 @@ def main():
         L.run(fused=False)
         tu = statistics.mean(timed(torch, lambda: L.run(fused=False), args.steps, 3, flush))
         rb = sum(alg_bytes_ir_in_gemm1(cfg, L.stored, L.T).values())
-        ub = sum(alg_bytes(cfg, L.stored, L.T)[1].values())
+        ub = sum(alg_bytes(cfg, L.stored_u, L.Tu)[1].values())
         err = parity(L, cfg)
         e = {"axis": axis, "model": model, "name": cfg.name, "B": cfg.B, "H": cfg.H, "L": cfg.S, "D": cfg.D,
              "dtype": cfg.dtype, "layers_per_s": round(1e3 / tr, 1), "ms": round(tr, 4),
