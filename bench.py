@@ -228,6 +228,64 @@ class Layer:
                             two_kernels=two_kernels, gs_prologue=gs_prologue, **self.kw)
 
 
+def e2e_pipelined(torch, L, steps, warmup, nbuf=2):
+    """End-to-end throughput through the public API: K steps, each copying its q/k/v from pinned host
+    memory, running the layer and reading its output back to pinned host memory. Three streams
+    (copy-in, compute, copy-out) with double-buffered device inputs/outputs, so step i+1's H2D and
+    step i-1's D2H overlap step i's layer (PCIe is full duplex). Every step still moves all its bytes.
+    Returns device ms per step (events around the whole K-step region on the compute stream)."""
+    comp = torch.cuda.current_stream()
+    s_in, s_out = torch.cuda.Stream(), torch.cuda.Stream()
+    bufs = [{n: torch.empty_like(L.dev[n]) for n in ("q", "k", "v")} for _ in range(nbuf)]
+    outs = [torch.empty_like(L.out) for _ in range(nbuf)]
+    hosts = [torch.empty_like(L.out_host).pin_memory() for _ in range(nbuf)]
+    ws = L.ws[True]
+
+    def region(n):
+        comp_done = [None] * n
+        out_done = [None] * n
+        start = torch.cuda.Event(enable_timing=True)
+        end = torch.cuda.Event(enable_timing=True)
+        comp.record_event(start)
+        s_in.wait_event(start)
+        for i in range(n):
+            b = i % nbuf
+            with torch.cuda.stream(s_in):
+                if i >= nbuf:
+                    s_in.wait_event(comp_done[i - nbuf])  # layer i-nbuf finished reading this input set
+                for nm in ("q", "k", "v"):
+                    bufs[b][nm].copy_(L.host[nm], non_blocking=True)
+                ready = torch.cuda.Event()
+                s_in.record_event(ready)
+            comp.wait_event(ready)
+            if i >= nbuf:
+                comp.wait_event(out_done[i - nbuf])  # D2H of step i-nbuf finished reading this output
+            L.sr.call(L.mask, bufs[b]["q"], bufs[b]["k"], bufs[b]["v"], out=outs[b], workspace=ws,
+                      tile_n=L.tile_n, **L.kw)
+            comp_done[i] = torch.cuda.Event()
+            comp.record_event(comp_done[i])
+            s_out.wait_event(comp_done[i])
+            with torch.cuda.stream(s_out):
+                hosts[b].copy_(outs[b], non_blocking=True)
+                out_done[i] = torch.cuda.Event()
+                s_out.record_event(out_done[i])
+        comp.wait_event(out_done[n - 1])
+        comp.record_event(end)
+        return start, end
+
+    region(max(warmup, nbuf))
+    torch.cuda.synchronize()
+    torch.cuda._sleep(SPIN_CYCLES)
+    a, b = region(steps)
+    torch.cuda.synchronize()
+    # every step computed the same layer from the same host inputs: the pipelined result read back
+    # to the host must equal the device path's output bit for bit (the kernels are deterministic)
+    L.run()
+    torch.cuda.synchronize()
+    same = all(torch.equal(h, L.out.cpu()) for h in hosts)
+    return a.elapsed_time(b) / steps, same
+
+
 def timed(torch, fn, steps, warmup, flush, per_step_pre=None):
     """W warm-up + K timed steps; L2 flushed before each; returns per-step device ms list."""
     ev = []
@@ -489,7 +547,9 @@ def gpu_arm(args, rank, world, local_rank):
         L.out_host.copy_(L.out, non_blocking=True)
 
     barrier(torch, world)
-    ms_e2e = dist_max(torch, statistics.mean(timed(torch, e2e_step, K, Wm, flush)), world)
+    ms_e2e_serial = dist_max(torch, statistics.mean(timed(torch, e2e_step, K, Wm, flush)), world)
+    ms_e2e, e2e_same = e2e_pipelined(torch, L, K, Wm)
+    ms_e2e = dist_max(torch, ms_e2e, world)
 
     # ---- other configs (same run, fewer steps): layers/s and bytes, recomposed vs unfused
     others = {}
@@ -581,7 +641,13 @@ def gpu_arm(args, rank, world, local_rank):
                      "peak_source": peak_src,
                      "tensor_frac": round(flops(cfg, L.stored) / (ms_step * 1e-3) / 1e12 / peaks.get("bf16_tflops", 1590.0), 4)},
         "e2e": {"value": round(world * 1e3 / ms_e2e, 2), "unit": "layers/s", "h2d_bytes_per_step": int(h2d),
-                "d2h_bytes_per_step": int(d2h), "ms_per_step": round(ms_e2e, 5)},
+                "d2h_bytes_per_step": int(d2h), "ms_per_step": round(ms_e2e, 5),
+                "how": "K steps through the public API, each H2D of its q/k/v from pinned host memory, the "
+                       "layer, D2H of its output; copy-in / compute / copy-out streams, double-buffered",
+                "output_bitwise_equal_device_path": bool(e2e_same),
+                "pcie_GBps": round((h2d + d2h) / (ms_e2e * 1e-3) / 1e9, 1),
+                "single_step_serial": {"value": round(world * 1e3 / ms_e2e_serial, 2),
+                                       "ms_per_step": round(ms_e2e_serial, 5)}},
         "gpu_launches": int(launches),
         "training": train,
         "clocks": clocks,
@@ -629,7 +695,7 @@ def cpu_baseline(cfg, target_s=10.0):
         done += n
         reps += 1
         dt = time.perf_counter() - t0
-        if dt >= 0.5 * target_s:
+        if dt >= 0.9 * target_s:
             break
     frac = done / (cfg.BH * cfg.S)
     return {"value": round(frac / dt, 6), "unit": "layers/s", "cores": nt, "kind": "oracle",
@@ -673,7 +739,7 @@ def main():
     ap.add_argument("--no-flush", action="store_true")
     ap.add_argument("--tile-n", type=int, default=0, help="LS sub-vector width T (0 = library default)")
     ap.add_argument("--no-all-configs", dest="all_configs", action="store_false")
-    ap.add_argument("--cpu-seconds", type=float, default=10.0)
+    ap.add_argument("--cpu-seconds", type=float, default=12.0)
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     world = int(os.environ.get("WORLD_SIZE", "1"))
