@@ -275,3 +275,26 @@ def test_backward_entry_points_validate_masks():
     assert _call_bwd(mask=bad.ptr) == sr.SR_ERR_INVALID
     assert _call_bwd("sr_mha_blocksparse_bwd", mask=None) == sr.SR_ERR_INVALID
     assert _call_bwd("sr_mha_sliding_window_bwd", mask=None) == sr.SR_ERR_INVALID
+
+
+def test_missing_library_fails_loudly(tmp_path):
+    """No CPU fallback: with the shared library absent the binding raises on first use."""
+    code = ("import paper_conf_iiswc_choilkha22_b200 as sr\n"
+            "try:\n    sr.lib()\nexcept RuntimeError as e:\n    print('RAISED', e)\n")
+    env = dict(os.environ, SR_MHA_LIB=str(tmp_path / "absent" / "libsr_mha.so"))
+    r = subprocess.run(["python", "-c", code], cwd=ROOT, env=env, capture_output=True, text=True, timeout=300)
+    assert r.returncode == 0 and "RAISED" in r.stdout and "missing" in r.stdout, r.stdout + r.stderr
+
+
+def test_product_path_never_touches_the_oracle():
+    """The oracle is test infrastructure: nothing in the package (binding, sharding, CUDA sources)
+    imports or links it."""
+    pkg = os.path.join(ROOT, "paper_conf_iiswc_choilkha22_b200")
+    for dirpath, _, files in os.walk(pkg):
+        if "_build" in dirpath:
+            continue
+        for f in files:
+            if f.endswith((".py", ".cu", ".cuh", ".h", ".cpp")):
+                txt = open(os.path.join(dirpath, f)).read()
+                assert not re.search(r"^\s*(from|import)\s+oracle|#include\s+[<\"].*oracle", txt, flags=re.M), f
+                assert "liboracle" not in txt, f
