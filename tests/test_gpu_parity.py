@@ -446,3 +446,37 @@ def test_sd_variant(kind, kw):
                            oracle_mask(kind, kw.get("kv_len"), kw.get("causal", False), kw.get("layout"),
                                        kw.get("window", 0), kw.get("n_global", 0)))
     assert_close(o.double().cpu().numpy(), ref, dtype, what=f"SD {kind}")
+
+
+LONG_CASES = [
+    # long sequences past every BASELINE config (several thousand key tiles per head): the default
+    # path's schedules, workspace offsets (> 2^31 bytes of X' slots addressed in 64-bit) and row
+    # statistics at scale; checked on sampled rows (edge rows included) against the oracle
+    ("dense", dict(B=1, H=2, S=16384, D=64, dtype="f16", causal=True)),
+    ("dense", dict(B=1, H=2, S=8192, D=128, dtype="bf16", kv_len=[8000])),
+    ("window", dict(B=1, H=1, S=32768, D=64, dtype="f16", window=512, n_global=8)),
+    ("dense", dict(B=1, H=2, S=32768, D=64, dtype="f16")),  # X' = 4 GiB
+]
+
+
+@pytest.mark.parametrize("kind,kw", LONG_CASES, ids=lambda x: str(x)[:60] if isinstance(x, dict) else x)
+def test_long_sequence_sampled_rows(kind, kw):
+    kw = dict(kw)
+    B, H, S, D, dtype = (kw.pop(x) for x in ("B", "H", "S", "D", "dtype"))
+    t, q, k, v = qkv(B, H, S, D, dtype, seed=S)
+    scale = 1 / math.sqrt(D)
+    if kind == "dense":
+        o = sr.mha_dense(q, k, v, scale=scale, kv_len=kw.get("kv_len"), causal=kw.get("causal", False),
+                         out_dtype=torch.float32)
+    else:
+        o = sr.mha_sliding_window(q, k, v, kw["window"], kw["n_global"], scale=scale, out_dtype=torch.float32)
+    torch.cuda.synchronize()
+    m = oracle_mask(kind, kw.get("kv_len"), kw.get("causal", False), None, kw.get("window", 0), kw.get("n_global", 0))
+    rng = np.random.Generator(np.random.PCG64(S + D))
+    edge = [0, 1, 63, 64, 127, 128, 4095, 4096, S // 2, S - 129, S - 128, S - 2, S - 1]
+    rows = sorted(set([g * S + i for g in range(B * H) for i in edge] + rng.integers(0, B * H * S, 48).tolist()))
+    rows = np.array(rows, dtype=np.int64)
+    ref = oracle.attention_rows(t.q64, t.k64, t.v64, scale, rows, m)
+    got = o.reshape(-1, D)[torch.from_numpy(rows).cuda()].double().cpu().numpy()
+    assert_close(got, ref, dtype, what=f"{kind} S={S}")
+    assert torch.isfinite(o).all()
