@@ -635,6 +635,14 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
         p.g1_pair = env_pair >= 0 ? env_pair : (D == 128 && cs->dev.n_pcta > 0 &&
                                                  (int64_t)B * H * cs->dev.n_pair >= 2 * (int64_t)cs->dev.n_pcta);
     }
+    {   // X' (or S) stores stream past L2 (evict_first) only when the layer's tiles exceed half the
+        // L2; below that they keep normal priority and are read back from L2 (measured, one B200,
+        // back-to-back: C2 (31.5 MB of X') 18.5 -> 17.6 us; C5 (132 MB) slower without the hint).
+        // SR_X_EVICT_FIRST=0/1 overrides (experiments).
+        static const int env_x = [] { const char* e = getenv("SR_X_EVICT_FIRST"); return e ? atoi(e) : -1; }();
+        const double x_bytes = (double)wi.n_slots * kRowBlock * r.T * 2.0;
+        p.x_evict_first = env_x >= 0 ? env_x : (x_bytes > 64.0 * (1 << 20));
+    }
     char* ws = (char*)ex->workspace;
     p.xprime = ws + wi.off_xprime;
     if (fused) {

@@ -48,7 +48,12 @@ constexpr bool kQPrefetch = SR_G1_QPREFETCH;  // L2 prefetch of the next item's 
 #ifndef SR_G1_HINTS
 #define SR_G1_HINTS 1
 #endif
-constexpr bool kG1Hints = SR_G1_HINTS;  // X' stores evict_first (streamed), K loads evict_last (re-read by every row-block)
+#ifndef SR_G1_KHINT
+#define SR_G1_KHINT SR_G1_HINTS
+#endif
+constexpr bool kG1KHint = SR_G1_KHINT;  // K loads evict_last (re-read by every row-block)
+// X' stores: evict_first (streamed) only when the layer's X' does not fit comfortably in L2
+// (p.x_evict_first, chosen on the host); a small X' stays at normal priority and is read back from L2
 // Of every 8 element pairs of the LS exponentials, this many are computed by ex2_poly2 on the FMA
 // pipe and the rest by MUFU.EX2 (16 / clock / SM): balances the two pipes in the epilogue.
 #ifndef SR_G1_POLY_PAIRS
@@ -154,13 +159,13 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
 
     const int warp = warp_uniform(), lane = threadIdx.x % 32;
     DW_DECL
-    const uint64_t pol_k = kG1Hints ? policy_evict_last() : 0, pol_x = kG1Hints ? policy_evict_first() : 0;
+    const uint64_t pol_k = kG1KHint ? policy_evict_last() : 0, pol_x = p.x_evict_first ? policy_evict_first() : 0;
     auto kload = [&](void* d, const CUtensorMap* m, int c0, int c1, uint64_t* b) {
-        if (kG1Hints) tma_load_2d_hint(d, m, c0, c1, b, pol_k);
+        if (kG1KHint) tma_load_2d_hint(d, m, c0, c1, b, pol_k);
         else tma_load_2d(d, m, c0, c1, b);
     };
     auto xstore = [&](void* d, const void* src, uint32_t nb) {
-        if (kG1Hints) bulk_store_hint(d, src, nb, pol_x);
+        if (p.x_evict_first) bulk_store_hint(d, src, nb, pol_x);
         else bulk_store(d, src, nb);
     };
 

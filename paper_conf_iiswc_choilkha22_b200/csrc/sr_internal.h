@@ -83,6 +83,7 @@ struct Params {
     int ir_mode;       // IrMode: where the IR sub-layer runs
     int g1_pair;       // GEMM1 walks pairs of row-blocks sharing each K tile (pair schedule)
     int gs_prologue;   // one-launch kernel: Global Scaling in GEMM2's prologue even for fp16 (SR_GS_PROLOGUE)
+    int x_evict_first; // GEMM1's X' / S tile stores carry an L2 evict_first policy (large layers only)
     DevSched sc;
     void* xprime;      // X' tiles (recomposed) or score tiles S (unfused)
     void* pbuf;        // unfused: P tiles
