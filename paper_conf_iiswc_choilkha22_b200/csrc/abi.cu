@@ -746,6 +746,12 @@ sr_status run_bwd(sr_entry e, const void* q, const void* k, const void* v, const
     p.dout = dout;
     p.dq = dq; p.dk = dk; p.dv = dv;
     p.dsbuf = ws + wi.off_ds;
+    {   // X' reads and dS' stores stream past L2 only when X' + dS' exceed ~100 MiB of the 126 MB L2
+        // (measured: C2, 96 MiB, backward 50.1 -> 48.2-49.5 us at normal priority; C5 unchanged)
+        static const int env_x = [] { const char* e = getenv("SR_X_EVICT_FIRST"); return e ? atoi(e) : -1; }();
+        const double xds_bytes = 2.0 * (double)wi.n_slots * kRowBlock * r.T * 2.0;
+        p.x_evict_first = env_x >= 0 ? env_x : (xds_bytes > 100.0 * (1 << 20));
+    }
     p.bstat = (float*)(ws + wi.off_bstat);
     {   // dQ inside the dS' kernel (default); SR_BWD_DQ_SEPARATE=1 keeps the separate GEMM2-based dQ kernel
         static const bool sep = [] { const char* e = getenv("SR_BWD_DQ_SEPARATE"); return e && atoi(e) != 0; }();

@@ -295,7 +295,8 @@ __global__ void __launch_bounds__(384, 1)
             }
         } else if (warp == 3) {
             // ------------------------------------------------------------------ X' + m' producer
-            const uint64_t pol_x = policy_evict_first();  // X' is streamed
+            // X' is streamed (evict_first) unless X' and dS' together fit in half the L2 (p.x_evict_first)
+            const uint64_t pol_x = p.x_evict_first ? policy_evict_first() : policy_evict_normal();
             int n = 0;  // macro tile counter, as the MMA warp and the epilogue count them
             for (ItemWalk iw(p, it_begin, it_end); iw.more();) {
                 const ItemInfo I = iw.next();
@@ -445,7 +446,7 @@ __global__ void __launch_bounds__(384, 1)
         const int wrow0 = (warp % 4) * 32;
         const bool bf = p.in_dtype == DT_BF16;
         const int64_t nrow = (int64_t)p.B * p.H * p.S;
-        const uint64_t pol_ds = policy_evict_first();
+        const uint64_t pol_ds = p.x_evict_first ? policy_evict_first() : policy_evict_normal();
         int64_t cur = -1;
         float m_row = 0.f, invd_row = 0.f, delta_row = 0.f;
         for (int n = e;; n += 2) {
