@@ -63,7 +63,8 @@ def launches(path):
 
 def main(rnd):
     os.makedirs(PROF, exist_ok=True)
-    traffic = {}
+    tp = os.path.join(PROF, "ncu_traffic.json")
+    traffic = json.load(open(tp)) if os.path.exists(tp) else {}  # configs not re-profiled keep their entry
     for c in (2, 3, 4, 5):
         p = os.path.join(OUT, f"launches_c{c}.csv")
         if not os.path.exists(p):
