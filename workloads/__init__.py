@@ -68,7 +68,17 @@ CONFIGS = [
 ]
 
 
+# Second workload of SURVEY NEXT-3 (GPT-Neo's local-attention layers, window 256):
+# GPT-Neo's local layers let query i see keys i-255..i, i.e. causal with |i - j| <= 255 -- the
+# sliding-window entry with window/2 = 255 (window = 510), no global tokens, at the C3 shape.
+GPTNEO_LOCAL = Config(6, "gptneo_local", "window", B=4, H=16, S=2048, D=128, dtype="bf16", causal=True,
+                      window=510, n_global=0)
+EXTRA_CONFIGS = [GPTNEO_LOCAL]
+
+
 def config(idx: int) -> Config:
+    if idx == GPTNEO_LOCAL.idx:
+        return GPTNEO_LOCAL
     return CONFIGS[idx - 1]
 
 
