@@ -32,11 +32,16 @@
  *  - scale: multiplies Q K^T (PAPER.md L53 uses 1/sqrt(D_head)); finite and > 0.
  *  - causal: key j is masked for query i when j > i (combines with every mask kind).
  *  - Mask / layout descriptors and the arrays they point to are HOST memory, read during the
- *    call.  The library derives a tile schedule from them and caches it on the device (small,
- *    library-owned allocations made on the first call with a new mask; later calls with the same
- *    mask content allocate nothing and are CUDA-graph capturable).
- *  - All launches go to ex->stream; nothing synchronises it.  Calls are asynchronous: device-side
- *    faults surface at the caller's next synchronisation (as with cuBLAS).
+ *    call (they may be freed or changed once the call returns).  The library derives a tile
+ *    schedule from them on the host, keeps it in a bounded host-side cache keyed by the mask
+ *    content, and every call writes it into the caller's workspace (region off_sched) with a
+ *    stream-ordered copy kernel whose words travel in its launch parameters.
+ *  - Ownership: the caller owns q, k, v, out, the workspace, the mask arrays and the stream.  The
+ *    library never allocates device memory and never synchronises: every call -- including the
+ *    first call with a new mask -- only enqueues kernels on ex->stream, so any call can be captured
+ *    in a CUDA graph, and a replay is self-contained (it re-writes the schedule it captured).
+ *    Calls are asynchronous: device-side faults surface at the caller's next synchronisation (as
+ *    with cuBLAS).  Two calls in flight at once (other streams, other threads) need two workspaces.
  *  - A row whose every key is masked outputs 0 (reading R9).
  *  - Supported: S % 128 == 0, S >= 128; D in {64, 128}; in_dtype F16 or BF16 (tensor-core path) or
  *    F32 (SIMT fp32 path, every mask kind); out_dtype == in_dtype or F32; block == 64.
@@ -143,6 +148,11 @@ typedef struct {
  * rounded to fp16, then Y V) instead of accumulator-side (O += r'_k (X'_k V_k) in fp32, the
  * fp16 default).  bf16 always uses the prologue form. */
 #define SR_GS_PROLOGUE 512
+/* Modifier: skip the schedule upload.  The caller asserts that the workspace's schedule region
+ * still holds what an earlier call with identical arguments (shape, mask content, causal, tile_n,
+ * dtypes, variant and stage bits aside) wrote there, and that nothing has written it since (used by
+ * bench.py to time single kernels with SR_RUN_* stage bits).  Wrong use reads a stale schedule. */
+#define SR_SCHED_RESIDENT 1024
 
 /* Entry points (north star).  Returns SR_OK after enqueueing the kernels on ex->stream. */
 sr_status sr_mha_dense(const void* q, const void* k, const void* v, void* out, int B, int H, int S,
@@ -221,6 +231,8 @@ typedef enum { SR_E_DENSE = 0, SR_E_BLOCKSPARSE = 1, SR_E_WINDOW = 2 } sr_entry;
  *            m_w (natural-log units) then d_w; the row's m = max_w m_w, d = sum_w e^{m_w - m} d_w
  *   ds, bstat  SR_WS_TRAIN only (backward): dS' tiles; per-row m, 1/d, delta.  The backward also
  *            writes r' (rprime) for every listed tile.
+ *   sched    the call's tile schedule (int32 words: tile lists, item descriptors, per-CTA ranges),
+ *            written by each call before its kernels run; sched_bytes reserves room for any SM count
  */
 typedef struct {
     int32_t tile_n;           /* T actually used */
@@ -232,6 +244,8 @@ typedef struct {
     size_t total_bytes;
     size_t off_ds;            /* SR_WS_TRAIN: dS' tiles, same slots / layout as X', in_dtype */
     size_t off_bstat;         /* SR_WS_TRAIN: fp32 [3][B*H*S]: m, 1/d, delta per query row */
+    size_t off_sched;         /* tile schedule region (every mode) */
+    size_t sched_bytes;
 } sr_ws_info;
 
 /* Workspace bytes needed by an entry point; `mask_or_layout` is the same pointer passed to it

@@ -13,11 +13,13 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <list>
 #include <map>
 #include <memory>
 #include <mutex>
 #include <queue>
 #include <string>
+#include <unordered_map>
 #include <vector>
 
 #include "../../include/sr_mha.h"
@@ -302,21 +304,50 @@ sr_status check_request(sr_entry e, int B, int H, int S, int D, int in_dtype,
 }
 
 // ------------------------------------------------------------------------------ cache
+//
+// Host schedules are cached by mask content in a bounded LRU (host memory only: nothing on the
+// device is library-owned).  The device form of a schedule is a word blob that every call uploads
+// into its own workspace (k_sched.cu), so a cache eviction can never invalidate a pending launch or
+// a captured graph.
+
+// Word groups of the blob, each a contiguous, 16-B aligned range; a call uploads only the groups
+// its kernels read.
+enum BlobGroup { G_BASE = 0, G_ITEMS, G_PAIR, G_FP, G_COL, G_N };
+constexpr int kMaxCta = 1024;  // bound on persistent CTAs per launch (the workspace reserves it)
+
+struct BlobLayout {  // int32-word offsets inside the blob
+    size_t tp, tinfo, kv, desc, items, cta, pdesc, pent, pcta, fp, fpcta, cdesc, cent, ccta;
+    size_t g_off[G_N], g_len[G_N];
+    size_t words;
+};
+
+struct DevBlob {
+    int n_sm = 0;
+    std::vector<int32_t> w;
+    BlobLayout L{};
+    DevSched rel{};  // scalar fields of the device schedule (pointers filled per call)
+    // the groups a one-launch call reads, packed back to back for its kernel parameters (per group
+    // mask; built on first use)
+    std::mutex mu;
+    std::map<unsigned, std::shared_ptr<const std::vector<int32_t>>> packed;
+};
 
 struct CachedSched {
     HostSched hs;
-    void* dmem = nullptr;
-    DevSched dev{};
+    std::mutex mu;                              // guards blobs
+    std::vector<std::shared_ptr<DevBlob>> blobs;  // one per SM count seen (normally one)
 };
 
 std::mutex g_mu;
-std::map<std::string, std::shared_ptr<CachedSched>> g_cache;
+constexpr size_t kCacheCap = 128;
+std::list<std::string> g_lru;  // most recent first
+std::unordered_map<std::string, std::pair<std::shared_ptr<CachedSched>, std::list<std::string>::iterator>> g_cache;
 
-std::string sched_key(const Request& r, int device)
+std::string sched_key(const Request& r)
 {
     std::string k;
     auto put = [&](int64_t x) { k.append((const char*)&x, sizeof(x)); };
-    put(device); put(r.entry); put(r.B); put(r.H); put(r.S); put(r.causal); put(r.T);
+    put(r.entry); put(r.B); put(r.H); put(r.S); put(r.causal); put(r.T);
     put(r.window); put(r.n_global);
     if (r.kv_len) { put(1); for (int b = 0; b < r.B; ++b) put(r.kv_len[b]); } else put(0);
     if (r.lay) {
@@ -329,6 +360,194 @@ std::string sched_key(const Request& r, int device)
         }
     }
     return k;
+}
+
+// Word layout of the blob for given per-CTA-range lengths (n_cta + 1 entries each).  The workspace
+// region is sized with kMaxCta so it fits every device.
+BlobLayout blob_layout(const HostSched& h, size_t n_cta_ptr, size_t n_pcta_ptr, size_t n_ccta_ptr)
+{
+    BlobLayout L{};
+    size_t o = 0;
+    auto pad = [&] { o = (o + 3) / 4 * 4; };
+    auto grp = [&](int g, size_t start) { L.g_off[g] = start; pad(); L.g_len[g] = o - start; };
+    size_t s = o;  // G_BASE: tp, tinfo, kv_len
+    L.tp = o; o += h.tp.size();
+    L.tinfo = o; o += std::max<size_t>(h.tinfo.size(), 1);
+    L.kv = o; o += h.kv_len.size();
+    grp(G_BASE, s);
+    s = o;  // G_ITEMS: item descriptors (16-B aligned), items, cta_ptr
+    L.desc = o; o += 4 * h.items.size();
+    L.items = o; o += h.items.size();
+    L.cta = o; o += n_cta_ptr;
+    grp(G_ITEMS, s);
+    s = o;  // G_PAIR: pair descriptors, union entries, pcta_ptr
+    L.pdesc = o; o += 4 * h.pitems.size();
+    L.pent = o; o += std::max<size_t>(h.pent.size(), 4);
+    L.pcta = o; o += n_pcta_ptr;
+    grp(G_PAIR, s);
+    s = o;  // G_FP: the pair assignment unrolled into row-block descriptors, fpcta_ptr
+    L.fp = o; o += 4 * h.items.size();
+    L.fpcta = o; o += n_pcta_ptr;
+    grp(G_FP, s);
+    s = o;  // G_COL: column descriptors, column entries, ccta_ptr
+    L.cdesc = o; o += 4 * h.citems.size();
+    L.cent = o; o += std::max<size_t>(h.cent.size(), 4);
+    L.ccta = o; o += n_ccta_ptr;
+    grp(G_COL, s);
+    L.words = o;
+    return L;
+}
+
+size_t sched_region_bytes(const HostSched& h)
+{
+    return blob_layout(h, kMaxCta + 1, kMaxCta + 1, kMaxCta + 1).words * sizeof(int32_t);
+}
+
+void lpt_assign(HostSched& h, int n_cta);
+
+// The device blob of a schedule for n_sm persistent CTAs (built once, then shared read-only).
+std::shared_ptr<DevBlob> make_blob(const HostSched& h0, int n_sm)
+{
+    HostSched h = h0;  // the LPT pass reorders items: keep the cached host schedule device-neutral
+    lpt_assign(h, std::min(n_sm, kMaxCta));
+    auto db = std::make_shared<DevBlob>();
+    db->n_sm = n_sm;
+    BlobLayout L = blob_layout(h, h.cta_ptr.size(), h.pcta_ptr.size(), h.ccta_ptr.size());
+    db->L = L;
+    std::vector<int32_t>& w = db->w;
+    w.assign(L.words, 0);
+    auto put = [&](size_t off, const std::vector<int32_t>& v) { std::copy(v.begin(), v.end(), w.begin() + off); };
+    auto lh_of_g = [&](int g) { return h.lh_mode == LH_ONE ? 0 : (h.lh_mode == LH_BATCH ? g / h.H : g % h.H); };
+    put(L.tp, h.tp);
+    put(L.tinfo, h.tinfo);
+    put(L.kv, h.kv_len);
+    size_t o = L.desc;  // item descriptors {item, t0, t1, tp[lh][0]}
+    for (int32_t it : h.items) {
+        const int g = it / h.n_rb, rb = it % h.n_rb;
+        const int32_t* tp = &h.tp[(size_t)lh_of_g(g) * (h.n_rb + 1)];
+        const int32_t d[4] = {it, tp[rb], tp[rb + 1], tp[0]};
+        std::copy(d, d + 4, w.begin() + o);
+        o += 4;
+    }
+    put(L.items, h.items);
+    put(L.cta, h.cta_ptr);
+    o = L.pdesc;  // pair item descriptors {g * n_pair + j, e0, e1, tp[lh][0]}
+    for (int32_t it : h.pitems) {
+        const int g = it / h.n_pair, j = it % h.n_pair, lh = lh_of_g(g);
+        const int32_t* pp = &h.pp[(size_t)lh * (h.n_pair + 1)];
+        const int32_t d[4] = {it, pp[j], pp[j + 1], h.tp[(size_t)lh * (h.n_rb + 1)]};
+        std::copy(d, d + 4, w.begin() + o);
+        o += 4;
+    }
+    if (h.pent.empty()) { w[L.pent] = 0; w[L.pent + 1] = -1; w[L.pent + 2] = -1; }
+    put(L.pent, h.pent);
+    put(L.pcta, h.pcta_ptr);
+    o = L.fp;  // pair assignment as row-block item descriptors, per CTA
+    std::vector<int32_t> fpcta(1, 0);
+    for (size_t c = 0; c + 1 < h.pcta_ptr.size(); ++c) {
+        for (int i = h.pcta_ptr[c]; i < h.pcta_ptr[c + 1]; ++i) {
+            const int it = h.pitems[i], g = it / h.n_pair, j = it % h.n_pair;
+            const int32_t* tp = &h.tp[(size_t)lh_of_g(g) * (h.n_rb + 1)];
+            for (int rb = 2 * j; rb < std::min(2 * j + 2, h.n_rb); ++rb) {
+                const int32_t d[4] = {g * h.n_rb + rb, tp[rb], tp[rb + 1], tp[0]};
+                std::copy(d, d + 4, w.begin() + o);
+                o += 4;
+            }
+        }
+        fpcta.push_back((int32_t)((o - L.fp) / 4));
+    }
+    put(L.fpcta, fpcta);
+    o = L.cdesc;  // column item descriptors {g * n_cb + c, e0, e1, tp[lh][0]}
+    for (int32_t it : h.citems) {
+        const int g = it / h.n_cb, c = it % h.n_cb, lh = lh_of_g(g);
+        const int32_t* cp = &h.cpp[(size_t)lh * (h.n_cb + 1)];
+        const int32_t d[4] = {it, cp[c], cp[c + 1], h.tp[(size_t)lh * (h.n_rb + 1)]};
+        std::copy(d, d + 4, w.begin() + o);
+        o += 4;
+    }
+    if (h.cent.empty()) { w[L.cent] = 0; w[L.cent + 1] = -1; w[L.cent + 2] = -1; }
+    put(L.cent, h.cent);
+    put(L.ccta, h.ccta_ptr);
+    DevSched& d = db->rel;
+    d.n_rb = h.n_rb;
+    d.n_lh = h.n_lh;
+    d.lh_mode = h.lh_mode;
+    d.slots_per_head = h.slots_per_head;
+    d.max_rb_tiles = h.max_rb_tiles;
+    d.mean_rb_tiles = (int)((h.tinfo.size() + (size_t)h.n_lh * h.n_rb - 1) / ((size_t)h.n_lh * h.n_rb));
+    d.n_items = (int)h.items.size();
+    d.n_cta = (int)h.cta_ptr.size() - 1;
+    d.n_pair = h.n_pair;
+    d.n_pcta = (int)h.pcta_ptr.size() - 1;
+    d.n_cb = h.n_cb;
+    d.n_ccta = (int)h.ccta_ptr.size() - 1;
+    return db;
+}
+
+// The groups `groups` of a blob packed back to back (the one-launch kernel's parameter form), and
+// the device schedule whose pointer fields are byte offsets + 16 into that packing (0: not packed).
+std::shared_ptr<const std::vector<int32_t>> packed_blob(DevBlob& db, unsigned groups, DevSched& d, bool has_kv)
+{
+    size_t at[G_N], n = 0;
+    for (int g = 0; g < G_N; ++g) {
+        at[g] = SIZE_MAX;
+        if ((groups >> g) & 1) {
+            at[g] = n;
+            n += db.L.g_len[g];
+        }
+    }
+    auto rel = [&](size_t field, int g) -> uintptr_t {
+        return at[g] == SIZE_MAX ? 0 : (uintptr_t)((at[g] + field - db.L.g_off[g]) * sizeof(int32_t) + 16);
+    };
+    const BlobLayout& L = db.L;
+    d = db.rel;
+    d.tp = (const int32_t*)rel(L.tp, G_BASE);
+    d.tinfo = (const int32_t*)rel(L.tinfo, G_BASE);
+    d.kv_len = has_kv ? (const int32_t*)rel(L.kv, G_BASE) : nullptr;
+    d.item_desc = (const int4*)rel(L.desc, G_ITEMS);
+    d.items = (const int32_t*)rel(L.items, G_ITEMS);
+    d.cta_ptr = (const int32_t*)rel(L.cta, G_ITEMS);
+    d.pair_desc = (const int4*)rel(L.pdesc, G_PAIR);
+    d.pent = (const int4*)rel(L.pent, G_PAIR);
+    d.pcta_ptr = (const int32_t*)rel(L.pcta, G_PAIR);
+    d.fp_desc = (const int4*)rel(L.fp, G_FP);
+    d.fpcta_ptr = (const int32_t*)rel(L.fpcta, G_FP);
+    d.col_desc = (const int4*)rel(L.cdesc, G_COL);
+    d.cent = (const int4*)rel(L.cent, G_COL);
+    d.ccta_ptr = (const int32_t*)rel(L.ccta, G_COL);
+    std::lock_guard<std::mutex> lk(db.mu);
+    auto it = db.packed.find(groups);
+    if (it != db.packed.end()) return it->second;
+    auto pk = std::make_shared<std::vector<int32_t>>();
+    pk->reserve(n);
+    for (int g = 0; g < G_N; ++g)
+        if ((groups >> g) & 1)
+            pk->insert(pk->end(), db.w.begin() + db.L.g_off[g], db.w.begin() + db.L.g_off[g] + db.L.g_len[g]);
+    db.packed.emplace(groups, pk);
+    return pk;
+}
+
+// The device schedule with its pointers inside a workspace's schedule region.
+DevSched place(const DevBlob& db, void* region, bool has_kv)
+{
+    int32_t* b = (int32_t*)region;
+    const BlobLayout& L = db.L;
+    DevSched d = db.rel;
+    d.tp = b + L.tp;
+    d.tinfo = b + L.tinfo;
+    d.kv_len = has_kv ? b + L.kv : nullptr;
+    d.item_desc = (const int4*)(b + L.desc);
+    d.items = b + L.items;
+    d.cta_ptr = b + L.cta;
+    d.pair_desc = (const int4*)(b + L.pdesc);
+    d.pent = (const int4*)(b + L.pent);
+    d.pcta_ptr = b + L.pcta;
+    d.fp_desc = (const int4*)(b + L.fp);
+    d.fpcta_ptr = b + L.fpcta;
+    d.col_desc = (const int4*)(b + L.cdesc);
+    d.cent = (const int4*)(b + L.cent);
+    d.ccta_ptr = b + L.ccta;
+    return d;
 }
 
 // Greedy longest-processing-time assignment of the (already longest-first) items to n_cta
@@ -402,128 +621,106 @@ void lpt_assign(HostSched& h, int n_cta)
     lpt_assign(h.citems, ccost, n_cta, h.ccta_ptr);
 }
 
-// Host schedule only (no device), used by queries.
-sr_status host_sched(const Request& r, std::shared_ptr<CachedSched>& out, bool need_device)
+// The cached host schedule of a request (built on a miss; LRU-bounded, host memory only).
+sr_status host_sched(const Request& r, std::shared_ptr<CachedSched>& out)
 {
-    int dev = -1;
-    cudaError_t ce0 = cudaSuccess;
-    if (need_device) {
-        cudaError_t ce = cudaGetDevice(&dev);
-        if (ce != cudaSuccess) return fail(SR_ERR_CUDA, "cudaGetDevice: %s", cudaGetErrorString(ce));
+    std::string key = sched_key(r);
+    {
+        std::lock_guard<std::mutex> lk(g_mu);
+        auto itc = g_cache.find(key);
+        if (itc != g_cache.end()) {
+            g_lru.splice(g_lru.begin(), g_lru, itc->second.second);
+            out = itc->second.first;
+            return SR_OK;
+        }
     }
-    std::string key = sched_key(r, need_device ? dev : -1);
-    std::lock_guard<std::mutex> lk(g_mu);
-    auto itc = g_cache.find(key);
-    if (itc != g_cache.end()) { out = itc->second; return SR_OK; }
     auto cs = std::make_shared<CachedSched>();
     sr_status s = build_sched(r, cs->hs);
     if (s != SR_OK) return s;
-    if (need_device) {
-        HostSched& h = cs->hs;
-        int n_sm = 148;
-        if ((ce0 = cudaDeviceGetAttribute(&n_sm, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess)
-            return fail(SR_ERR_CUDA, "cudaDeviceGetAttribute: %s", cudaGetErrorString(ce0));
-        lpt_assign(h, n_sm);
-        size_t n_tp = h.tp.size(), n_ti = std::max<size_t>(h.tinfo.size(), 1), n_it = h.items.size(),
-               n_kv = h.kv_len.size();
-        const size_t n_pit = h.pitems.size();
-        size_t bytes = sizeof(int32_t) * (4 * n_it + 4 * n_pit + h.pent.size() + 4 + n_tp + n_ti + n_it + n_kv +
-                                          h.cta_ptr.size() + h.pp.size() + h.pcta_ptr.size() + 4 +
-                                          4 * h.citems.size() + h.cent.size() + 4 + h.ccta_ptr.size() +
-                                          8 * n_pit + h.pcta_ptr.size() + 4);
-        cudaError_t ce = cudaMalloc(&cs->dmem, bytes);
-        if (ce != cudaSuccess) return fail(SR_ERR_CUDA, "cudaMalloc(schedule): %s", cudaGetErrorString(ce));
-        std::vector<int32_t> blob;
-        blob.reserve(bytes / 4);
-        for (int32_t w : h.items) {  // item descriptors first (16-B aligned at the allocation base)
-            const int g = w / h.n_rb, rb = w % h.n_rb;
-            const int lh = h.lh_mode == LH_ONE ? 0 : (h.lh_mode == LH_BATCH ? g / h.H : g % h.H);
-            const int32_t* tp = &h.tp[(size_t)lh * (h.n_rb + 1)];
-            blob.insert(blob.end(), {w, tp[rb], tp[rb + 1], tp[0]});
-        }
-        size_t o_pd = blob.size();  // pair item descriptors {g * n_pair + j, e0, e1, tp[lh][0]}
-        for (int32_t w : h.pitems) {
-            const int g = w / h.n_pair, j = w % h.n_pair;
-            const int lh = h.lh_mode == LH_ONE ? 0 : (h.lh_mode == LH_BATCH ? g / h.H : g % h.H);
-            const int32_t* pp = &h.pp[(size_t)lh * (h.n_pair + 1)];
-            blob.insert(blob.end(), {w, pp[j], pp[j + 1], h.tp[(size_t)lh * (h.n_rb + 1)]});
-        }
-        size_t o_fp = blob.size();  // pair assignment as row-block item descriptors
-        std::vector<int32_t> fpcta(1, 0);
-        for (size_t c = 0; c + 1 < h.pcta_ptr.size(); ++c) {
-            for (int i = h.pcta_ptr[c]; i < h.pcta_ptr[c + 1]; ++i) {
-                const int w = h.pitems[i], g = w / h.n_pair, j = w % h.n_pair;
-                const int lh = h.lh_mode == LH_ONE ? 0 : (h.lh_mode == LH_BATCH ? g / h.H : g % h.H);
-                const int32_t* tp = &h.tp[(size_t)lh * (h.n_rb + 1)];
-                for (int rb = 2 * j; rb < std::min(2 * j + 2, h.n_rb); ++rb)
-                    blob.insert(blob.end(), {g * h.n_rb + rb, tp[rb], tp[rb + 1], tp[0]});
-            }
-            fpcta.push_back((int32_t)((blob.size() - o_fp) / 4));
-        }
-        size_t o_fpc = blob.size();
-        blob.insert(blob.end(), fpcta.begin(), fpcta.end());
-        while (blob.size() % 4) blob.push_back(0);  // the int4 arrays below stay 16-B aligned
-        size_t o_cd = blob.size();  // column item descriptors {g * n_cb + c, e0, e1, tp[lh][0]}
-        for (int32_t w : h.citems) {
-            const int g = w / h.n_cb, c = w % h.n_cb;
-            const int lh = h.lh_mode == LH_ONE ? 0 : (h.lh_mode == LH_BATCH ? g / h.H : g % h.H);
-            const int32_t* cp = &h.cpp[(size_t)lh * (h.n_cb + 1)];
-            blob.insert(blob.end(), {w, cp[c], cp[c + 1], h.tp[(size_t)lh * (h.n_rb + 1)]});
-        }
-        size_t o_ce = blob.size();  // column entries (int4)
-        blob.insert(blob.end(), h.cent.begin(), h.cent.end());
-        if (h.cent.empty()) blob.insert(blob.end(), {0, -1, -1, 0});
-        size_t o_pe = blob.size();  // union entries (int4)
-        blob.insert(blob.end(), h.pent.begin(), h.pent.end());
-        if (h.pent.empty()) blob.insert(blob.end(), {0, -1, -1, 0});
-        size_t o_tp = blob.size();
-        blob.insert(blob.end(), h.tp.begin(), h.tp.end());
-        size_t o_ti = blob.size();
-        blob.insert(blob.end(), h.tinfo.begin(), h.tinfo.end());
-        if (h.tinfo.empty()) blob.push_back(0);
-        size_t o_it = blob.size();
-        blob.insert(blob.end(), h.items.begin(), h.items.end());
-        size_t o_kv = blob.size();
-        blob.insert(blob.end(), h.kv_len.begin(), h.kv_len.end());
-        size_t o_cp = blob.size();
-        blob.insert(blob.end(), h.cta_ptr.begin(), h.cta_ptr.end());
-        size_t o_pcp = blob.size();
-        blob.insert(blob.end(), h.pcta_ptr.begin(), h.pcta_ptr.end());
-        size_t o_ccp = blob.size();
-        blob.insert(blob.end(), h.ccta_ptr.begin(), h.ccta_ptr.end());
-        ce = cudaMemcpy(cs->dmem, blob.data(), blob.size() * 4, cudaMemcpyHostToDevice);
-        if (ce != cudaSuccess) return fail(SR_ERR_CUDA, "cudaMemcpy(schedule): %s", cudaGetErrorString(ce));
-        int32_t* base = (int32_t*)cs->dmem;
-        cs->dev.item_desc = (const int4*)base;
-        cs->dev.tp = base + o_tp;
-        cs->dev.tinfo = base + o_ti;
-        cs->dev.items = base + o_it;
-        cs->dev.kv_len = n_kv ? base + o_kv : nullptr;
-        cs->dev.n_rb = h.n_rb;
-        cs->dev.n_lh = h.n_lh;
-        cs->dev.lh_mode = h.lh_mode;
-        cs->dev.slots_per_head = h.slots_per_head;
-        cs->dev.max_rb_tiles = h.max_rb_tiles;
-        cs->dev.mean_rb_tiles = (int)((h.tinfo.size() + (size_t)h.n_lh * h.n_rb - 1) / ((size_t)h.n_lh * h.n_rb));
-        cs->dev.n_items = (int)h.items.size();
-        cs->dev.cta_ptr = base + o_cp;
-        cs->dev.n_cta = (int)h.cta_ptr.size() - 1;
-        cs->dev.pair_desc = (const int4*)(base + o_pd);
-        cs->dev.pent = (const int4*)(base + o_pe);
-        cs->dev.pcta_ptr = base + o_pcp;
-        cs->dev.n_pair = h.n_pair;
-        cs->dev.n_pcta = (int)h.pcta_ptr.size() - 1;
-        cs->dev.fp_desc = (const int4*)(base + o_fp);
-        cs->dev.fpcta_ptr = base + o_fpc;
-        cs->dev.col_desc = (const int4*)(base + o_cd);
-        cs->dev.cent = (const int4*)(base + o_ce);
-        cs->dev.ccta_ptr = base + o_ccp;
-        cs->dev.n_cb = h.n_cb;
-        cs->dev.n_ccta = (int)h.ccta_ptr.size() - 1;
+    std::lock_guard<std::mutex> lk(g_mu);
+    auto itc = g_cache.find(key);  // another thread may have inserted it meanwhile
+    if (itc != g_cache.end()) {
+        out = itc->second.first;
+        return SR_OK;
     }
-    g_cache[key] = cs;
+    g_lru.push_front(key);
+    g_cache.emplace(key, std::make_pair(cs, g_lru.begin()));
+    while (g_cache.size() > kCacheCap) {  // evict the least recently used (callers hold shared_ptrs)
+        g_cache.erase(g_lru.back());
+        g_lru.pop_back();
+    }
     out = cs;
     return SR_OK;
+}
+
+// SM count of the current device (cached per device; no synchronisation).
+sr_status device_sms(int& n_sm)
+{
+    static std::mutex mu;
+    static std::map<int, int> sms;
+    int dev = -1;
+    cudaError_t ce = cudaGetDevice(&dev);
+    if (ce != cudaSuccess) return fail(SR_ERR_CUDA, "cudaGetDevice: %s", cudaGetErrorString(ce));
+    std::lock_guard<std::mutex> lk(mu);
+    auto it = sms.find(dev);
+    if (it == sms.end()) {
+        int n = 0;
+        if ((ce = cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess)
+            return fail(SR_ERR_CUDA, "cudaDeviceGetAttribute: %s", cudaGetErrorString(ce));
+        it = sms.emplace(dev, n).first;
+    }
+    n_sm = it->second;
+    return SR_OK;
+}
+
+// L2 size of the current device in bytes (cached; 0 if unknown).
+size_t device_l2_bytes()
+{
+    static std::mutex mu;
+    static std::map<int, size_t> l2;
+    int dev = -1;
+    if (cudaGetDevice(&dev) != cudaSuccess) return 0;
+    std::lock_guard<std::mutex> lk(mu);
+    auto it = l2.find(dev);
+    if (it == l2.end()) {
+        int n = 0;
+        if (cudaDeviceGetAttribute(&n, cudaDevAttrL2CacheSize, dev) != cudaSuccess) n = 0;
+        it = l2.emplace(dev, (size_t)n).first;
+    }
+    return it->second;
+}
+
+std::shared_ptr<DevBlob> device_blob(CachedSched& cs, int n_sm)
+{
+    std::lock_guard<std::mutex> lk(cs.mu);
+    for (auto& b : cs.blobs)
+        if (b->n_sm == n_sm) return b;
+    cs.blobs.push_back(make_blob(cs.hs, n_sm));
+    return cs.blobs.back();
+}
+
+double l2_or_default()
+{
+    const size_t l2 = device_l2_bytes();
+    return l2 ? (double)l2 : 126.0 * (1 << 20);
+}
+
+// Enqueue the upload of the given blob groups into the workspace's schedule region (k_sched.cu).
+cudaError_t upload(const DevBlob& db, void* region, unsigned groups, cudaStream_t st, int64_t* nl)
+{
+    size_t off[G_N], len[G_N];
+    int n = 0;
+    for (int g = 0; g < G_N; ++g)
+        if (((groups >> g) & 1) && db.L.g_len[g]) {
+            if (n && off[n - 1] + len[n - 1] == db.L.g_off[g]) {  // adjacent groups: one segment
+                len[n - 1] += db.L.g_len[g];
+                continue;
+            }
+            off[n] = db.L.g_off[g];
+            len[n] = db.L.g_len[g];
+            ++n;
+        }
+    return launch_sched_upload(region, db.w.data(), off, len, n, st, nl);
 }
 
 size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
@@ -539,6 +736,10 @@ void ws_layout(const HostSched& h, int B, int H, int in_dtype, int fused, sr_ws_
     size_t tile_bytes = (size_t)kRowBlock * h.T * elt;
     size_t stat_bytes = (size_t)info->n_slots * kRowBlock * sizeof(float);
     size_t o = 0;
+    // first: the call's tile schedule, uploaded into the workspace by every call (k_sched.cu); its
+    // size depends only on the mask, so every mode of one request (recomposed, training) shares it
+    info->sched_bytes = sched_region_bytes(h);
+    info->off_sched = o; o = align_up(o + info->sched_bytes, 1024);
     info->off_xprime = o;
     o = align_up(o + (size_t)info->n_slots * tile_bytes, 1024);
     // fused: 1 recomposed (X' + statistics), 0 unfused (S + P), 2 SD (X' + S/Y + statistics),
@@ -556,7 +757,7 @@ void ws_layout(const HostSched& h, int B, int H, int in_dtype, int fused, sr_ws_
         info->off_ds = o; o = align_up(o + (size_t)info->n_slots * tile_bytes, 1024);
         info->off_bstat = o; o = align_up(o + (size_t)3 * B * H * h.n_rb * kRowBlock * sizeof(float), 1024);
     }
-    info->total_bytes = std::max<size_t>(o, 1024);
+    info->total_bytes = o;
 }
 
 bool overlaps(const void* a, size_t na, const void* b, size_t nb)
@@ -573,7 +774,7 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
     if (!q || !k || !v || !out) return fail(SR_ERR_INVALID, "q, k, v and out must be non-NULL");
     if (!std::isfinite(scale) || !(scale > 0.f)) return fail(SR_ERR_INVALID, "scale must be finite and > 0");
     const int variant_bits = SR_FUSE_IR | SR_DECOMPOSE | SR_IR_KERNEL | SR_ONE_KERNEL | SR_TWO_KERNELS;
-    if (ex->flags & ~(SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2 | SR_GS_PROLOGUE | variant_bits))
+    if (ex->flags & ~(SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2 | SR_GS_PROLOGUE | SR_SCHED_RESIDENT | variant_bits))
         return fail(SR_ERR_INVALID, "unknown flags 0x%x", ex->flags);
     if ((ex->flags & variant_bits) && (!fused || ex->in_dtype == SR_F32))
         return fail(SR_ERR_UNSUPPORTED, "SR_FUSE_IR / SR_DECOMPOSE / SR_IR_KERNEL apply to the recomposed 16-bit path only");
@@ -603,15 +804,17 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
     if (((uintptr_t)q | (uintptr_t)k | (uintptr_t)v | (uintptr_t)out) & 15)
         return fail(SR_ERR_INVALID, "q, k, v, out must be 16-byte aligned");
     std::shared_ptr<CachedSched> cs;
-    s = host_sched(r, cs, false);  // host-only schedule: workspace checks precede any CUDA call
+    s = host_sched(r, cs);  // host-only schedule: workspace checks precede any CUDA call
     if (s != SR_OK) return s;
     sr_ws_info wi;
     ws_layout(cs->hs, B, H, ex->in_dtype, fused, &wi);
     if (!ex->workspace || ex->workspace_bytes < wi.total_bytes)
         return fail(SR_ERR_WORKSPACE, "workspace %zu bytes < required %zu", ex->workspace_bytes, wi.total_bytes);
     if ((uintptr_t)ex->workspace & 255) return fail(SR_ERR_WORKSPACE, "workspace must be 256-byte aligned");
-    s = host_sched(r, cs, true);  // device copy of the schedule (cached per device)
-    if (s != SR_OK) return s;
+    int n_sm = 0;
+    if ((s = device_sms(n_sm)) != SR_OK) return s;
+    std::shared_ptr<DevBlob> db = device_blob(*cs, n_sm);
+    void* region = (char*)ex->workspace + wi.off_sched;
 
     Params p{};
     p.q = q; p.k = k; p.v = v; p.out = out;
@@ -624,7 +827,7 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
     p.n_global = r.n_global;
     p.in_dtype = ex->in_dtype;
     p.out_dtype = ex->out_dtype;
-    p.sc = cs->dev;
+    p.sc = place(*db, region, r.kv_len != nullptr);
     const int stage_bits = ex->flags & (SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2);
     p.stages = stage_bits ? stage_bits : (SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2);
     p.ir_mode = (ex->flags & SR_FUSE_IR) ? IR_IN_GEMM2 : ((ex->flags & SR_IR_KERNEL) ? IR_KERNEL : IR_IN_GEMM1);
@@ -632,16 +835,16 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
         static const int env_pair = [] { const char* e = getenv("SR_G1_PAIR"); return e ? atoi(e) : -1; }();
         // default: pairs when K tiles are as large as the X' tiles they produce (D = 128) and there
         // are enough pairs to keep every SM busy (measured: C3 78 -> 75 us; D = 64 configs lose)
-        p.g1_pair = env_pair >= 0 ? env_pair : (D == 128 && cs->dev.n_pcta > 0 &&
-                                                 (int64_t)B * H * cs->dev.n_pair >= 2 * (int64_t)cs->dev.n_pcta);
+        p.g1_pair = env_pair >= 0 ? env_pair : (D == 128 && p.sc.n_pcta > 0 &&
+                                                 (int64_t)B * H * p.sc.n_pair >= 2 * (int64_t)p.sc.n_pcta);
     }
-    {   // X' (or S) stores stream past L2 (evict_first) only when the layer's tiles exceed half the
-        // L2; below that they keep normal priority and are read back from L2 (measured, one B200,
-        // back-to-back: C2 (31.5 MB of X') 18.5 -> 17.6 us; C5 (132 MB) slower without the hint).
-        // SR_X_EVICT_FIRST=0/1 overrides (experiments).
+    {   // X' (or S) stores stream past L2 (evict_first) only when the layer's stored tiles exceed
+        // half the device's L2; below that they keep normal priority and are read back from L2
+        // (measured, one B200, back-to-back: C2 (31.5 MB of X') 18.5 -> 17.6 us; C5 (132 MB) slower
+        // without the hint).  SR_X_EVICT_FIRST=0/1 overrides (experiments).
         static const int env_x = [] { const char* e = getenv("SR_X_EVICT_FIRST"); return e ? atoi(e) : -1; }();
-        const double x_bytes = (double)wi.n_slots * kRowBlock * r.T * 2.0;
-        p.x_evict_first = env_x >= 0 ? env_x : (x_bytes > 64.0 * (1 << 20));
+        const double x_bytes = (double)cs->hs.stored_elems * (ex->in_dtype == SR_F32 ? 4.0 : 2.0);
+        p.x_evict_first = env_x >= 0 ? env_x : (x_bytes > 0.5 * l2_or_default());
     }
     char* ws = (char*)ex->workspace;
     p.xprime = ws + wi.off_xprime;
@@ -655,19 +858,38 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
     cudaStream_t st = (cudaStream_t)ex->stream;
     int64_t nl = 0;
     cudaError_t ce;
+    // the schedule groups this call's kernels read, uploaded into the workspace ahead of them
+    const bool one_pair = fused == 1 && one && p.g1_pair;
+    const unsigned groups = one_pair ? (1u << G_BASE | 1u << G_PAIR | 1u << G_FP)
+                                     : (1u << G_BASE | 1u << G_ITEMS | (p.g1_pair ? 1u << G_PAIR : 0u));
+    // the one-launch kernel carries a small schedule in its own parameters; everything else reads
+    // it from the workspace, uploaded ahead of the kernels
+    size_t gw = 0;
+    for (int g = 0; g < G_N; ++g) gw += ((groups >> g) & 1) ? db->L.g_len[g] : 0;
+    std::shared_ptr<const std::vector<int32_t>> pk;
+#ifndef SR_NO_BLOB  // experiment builds: always upload into the workspace
+    if (fused == 1 && one && gw <= one_kernel_blob_words())
+#else
+    if (false)
+#endif
+        pk = packed_blob(*db, groups, p.sc, r.kv_len != nullptr);
+    else if (!(ex->flags & SR_SCHED_RESIDENT) && (ce = upload(*db, region, groups, st, &nl)) != cudaSuccess) {
+        g_launches += nl;
+        return fail(SR_ERR_CUDA, "schedule upload: %s", cudaGetErrorString(ce));
+    }
     if (fused == 2) {
         ce = launch_tc_sd(p, st, &nl);
     } else if (fused && one) {
         // pairs of row-blocks sharing each K tile in phase 1 (same choice as the two-kernel chain:
         // D = 128 with enough pairs); phase 2 then walks the pair assignment as row-block items
         if (p.g1_pair) {
-            p.sc.item_desc = cs->dev.fp_desc;
-            p.sc.cta_ptr = cs->dev.fpcta_ptr;
-            p.sc.n_cta = cs->dev.n_pcta;
+            p.sc.item_desc = p.sc.fp_desc;
+            p.sc.cta_ptr = p.sc.fpcta_ptr;
+            p.sc.n_cta = p.sc.n_pcta;
         }
         p.gs_prologue = (ex->flags & SR_GS_PROLOGUE) != 0;
 
-        ce = launch_tc_one(p, st, &nl);
+        ce = launch_tc_one(p, pk ? pk->data() : nullptr, pk ? pk->size() : 0, st, &nl);
     } else if (fused) {
         ce = ex->in_dtype == SR_F32 ? launch_simt_f32(p, st, &nl) : launch_tc_fused(p, st, &nl);
     } else {
@@ -688,8 +910,9 @@ sr_status run_bwd(sr_entry e, const void* q, const void* k, const void* v, const
     if (!q || !k || !v || !out || !dout || !dq || !dk || !dv)
         return fail(SR_ERR_INVALID, "q, k, v, out, dout, dq, dk and dv must be non-NULL");
     if (!std::isfinite(scale) || !(scale > 0.f)) return fail(SR_ERR_INVALID, "scale must be finite and > 0");
-    if (ex->flags & ~(SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2))
-        return fail(SR_ERR_INVALID, "backward flags must be SR_RUN_* stage bits (got 0x%x)", ex->flags);
+    if (ex->flags & ~(SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2 | SR_SCHED_RESIDENT))
+        return fail(SR_ERR_INVALID, "backward flags must be SR_RUN_* stage bits or SR_SCHED_RESIDENT (got 0x%x)",
+                    ex->flags);
     Request r;
     sr_status s = check_request(e, B, H, S, D, ex->in_dtype, mask_or_layout, causal, ex->tile_n, r, 3);
     if (s != SR_OK) return s;
@@ -711,7 +934,7 @@ sr_status run_bwd(sr_entry e, const void* q, const void* k, const void* v, const
          (uintptr_t)dk | (uintptr_t)dv) & 15)
         return fail(SR_ERR_INVALID, "all tensors must be 16-byte aligned");
     std::shared_ptr<CachedSched> cs;
-    s = host_sched(r, cs, false);
+    s = host_sched(r, cs);
     if (s != SR_OK) return s;
     sr_ws_info wi;
     ws_layout(cs->hs, B, H, ex->in_dtype, 3, &wi);
@@ -719,8 +942,10 @@ sr_status run_bwd(sr_entry e, const void* q, const void* k, const void* v, const
         return fail(SR_ERR_WORKSPACE, "workspace %zu bytes < required %zu (SR_WS_TRAIN)", ex->workspace_bytes,
                     wi.total_bytes);
     if ((uintptr_t)ex->workspace & 255) return fail(SR_ERR_WORKSPACE, "workspace must be 256-byte aligned");
-    s = host_sched(r, cs, true);
-    if (s != SR_OK) return s;
+    int n_sm = 0;
+    if ((s = device_sms(n_sm)) != SR_OK) return s;
+    std::shared_ptr<DevBlob> db = device_blob(*cs, n_sm);
+    void* region = (char*)ex->workspace + wi.off_sched;
 
     Params p{};
     p.q = q; p.k = k; p.v = v; p.out = const_cast<void*>(out);
@@ -733,7 +958,7 @@ sr_status run_bwd(sr_entry e, const void* q, const void* k, const void* v, const
     p.n_global = r.n_global;
     p.in_dtype = ex->in_dtype;
     p.out_dtype = ex->out_dtype;
-    p.sc = cs->dev;
+    p.sc = place(*db, region, r.kv_len != nullptr);
     const int stage_bits = ex->flags & (SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2);
     p.stages = stage_bits ? stage_bits : (SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2);
     p.ir_mode = IR_IN_GEMM1;
@@ -746,11 +971,12 @@ sr_status run_bwd(sr_entry e, const void* q, const void* k, const void* v, const
     p.dout = dout;
     p.dq = dq; p.dk = dk; p.dv = dv;
     p.dsbuf = ws + wi.off_ds;
-    {   // X' reads and dS' stores stream past L2 only when X' + dS' exceed ~100 MiB of the 126 MB L2
-        // (measured: C2, 96 MiB, backward 50.1 -> 48.2-49.5 us at normal priority; C5 unchanged)
+    {   // X' reads and dS' stores stream past L2 only when the layer's stored X' + dS' tiles exceed
+        // ~4/5 of the device's L2 (measured: C2, 63 MB, backward 50.1 -> 48.2-49.5 us at normal
+        // priority; C5 unchanged)
         static const int env_x = [] { const char* e = getenv("SR_X_EVICT_FIRST"); return e ? atoi(e) : -1; }();
-        const double xds_bytes = 2.0 * (double)wi.n_slots * kRowBlock * r.T * 2.0;
-        p.x_evict_first = env_x >= 0 ? env_x : (xds_bytes > 100.0 * (1 << 20));
+        const double xds_bytes = 2.0 * (double)cs->hs.stored_elems * 2.0;
+        p.x_evict_first = env_x >= 0 ? env_x : (xds_bytes > 0.8 * l2_or_default());
     }
     p.bstat = (float*)(ws + wi.off_bstat);
     {   // dQ inside the dS' kernel (default); SR_BWD_DQ_SEPARATE=1 keeps the separate GEMM2-based dQ kernel
@@ -758,7 +984,10 @@ sr_status run_bwd(sr_entry e, const void* q, const void* k, const void* v, const
         p.bwd_dq_fused = sep ? 0 : 1;
     }
     int64_t nl = 0;
-    cudaError_t ce = launch_tc_bwd(p, (cudaStream_t)ex->stream, &nl);
+    cudaError_t ce = cudaSuccess;
+    if (!(ex->flags & SR_SCHED_RESIDENT))
+        ce = upload(*db, region, 1u << G_BASE | 1u << G_ITEMS | 1u << G_COL, (cudaStream_t)ex->stream, &nl);
+    if (ce == cudaSuccess) ce = launch_tc_bwd(p, (cudaStream_t)ex->stream, &nl);
     g_launches += nl;
     if (ce != cudaSuccess) return fail(SR_ERR_CUDA, "kernel launch: %s", cudaGetErrorString(ce));
     return SR_OK;
@@ -835,7 +1064,7 @@ sr_status sr_workspace_query(sr_entry e, int fused, int B, int H, int S, int D, 
     sr_status s = check_request(e, B, H, S, D, in_dtype, mask_or_layout, causal, tile_n, r, fused);
     if (s != SR_OK) return s;
     std::shared_ptr<CachedSched> cs;
-    s = host_sched(r, cs, false);
+    s = host_sched(r, cs);
     if (s != SR_OK) return s;
     ws_layout(cs->hs, B, H, in_dtype, fused, info);
     return SR_OK;
@@ -857,7 +1086,7 @@ sr_status sr_schedule_stats(sr_entry e, int B, int H, int S, const void* mask_or
     sr_status s = check_request(e, B, H, S, 64, SR_F16, mask_or_layout, causal, tile_n, r, 1);
     if (s != SR_OK) return s;
     std::shared_ptr<CachedSched> cs;
-    s = host_sched(r, cs, false);
+    s = host_sched(r, cs);
     if (s != SR_OK) return s;
     if (n_tiles) *n_tiles = cs->hs.n_tiles;
     if (stored_elems) *stored_elems = cs->hs.stored_elems;

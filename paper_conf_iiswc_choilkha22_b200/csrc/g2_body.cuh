@@ -145,8 +145,8 @@ __device__ __forceinline__ void g2_init(uint8_t* smem)
 // r'_k (X'_k V_k) to the rows' O in registers, r'_k = e^{m'_k - m} / d -- the same terms as
 // (X'_k r'_k) V_k (Eq. 2 is linear in each sub-vector), with no per-element GS pass over X'.
 template <int D, int T, bool GS, bool FI, bool RS, bool AS = false>
-__device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p, uint8_t* smem, uint32_t tmem_base,
-                                          int it_begin, int it_end)
+__device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p, const DevSched& sc, uint8_t* smem,
+                                          uint32_t tmem_base, int it_begin, int it_end)
 {
     using C = G2<D, T>;
     constexpr int NSUB = C::NSUB;
@@ -182,7 +182,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
             int s = 0;
             const uint64_t pol_x = SR_G2_HINTS ? policy_evict_first() : 0;
             uint32_t sph = 0;
-            for (ItemWalk iw(p, it_begin, it_end); iw.more();) {
+            for (ItemWalk iw(sc, it_begin, it_end); iw.more();) {
                 const ItemInfo I = iw.next();
                 if (AS && I.t0 == I.t1) {  // no kept key in these rows: an EMPTY stage, written as zeros
                     DW_WAIT(&x_empty[s], sph ^ 1, 0);
@@ -197,11 +197,11 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                     continue;
                 }
                 int wn[2];  // schedule words of the next macro tile, prefetched one step ahead
-                for (int u = 0; u < NSUB; ++u) wn[u] = I.t0 + u < I.t1 ? __ldg(p.sc.tinfo + I.t0 + u) : 0;
+                for (int u = 0; u < NSUB; ++u) wn[u] = I.t0 + u < I.t1 ? sld(sc.tinfo + I.t0 + u) : 0;
                 for (int t = I.t0; t < I.t1; t += NSUB) {
                     const int nsub = min(NSUB, I.t1 - t);
                     int hv[2] = {tinfo_half(wn[0]), NSUB > 1 ? tinfo_half(wn[1]) : 0};
-                    for (int u = 0; u < NSUB; ++u) wn[u] = t + NSUB + u < I.t1 ? __ldg(p.sc.tinfo + t + NSUB + u) : 0;
+                    for (int u = 0; u < NSUB; ++u) wn[u] = t + NSUB + u < I.t1 ? sld(sc.tinfo + t + NSUB + u) : 0;
                     uint32_t bytes = GS ? nsub * kRowBlock * 4 : 0;
 #ifndef SR_DIAG2_NOX
                     for (int u = 0; u < nsub; ++u) bytes += ((GS && !AS) ? (hv[u] == 3 ? 2 : 1) : 2) * (T / 64) * (kHalf * 128);
@@ -259,7 +259,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
             int si = 0;
             uint32_t sph = 0;
             const int64_t nrow = (int64_t)p.B * p.H * p.S;
-            for (ItemWalk iw(p, it_begin, it_end); iw.more();) {
+            for (ItemWalk iw(sc, it_begin, it_end); iw.more();) {
                 const ItemInfo I = iw.next();
                 if (I.t0 == I.t1) continue;
                 const int64_t row = (int64_t)I.g * p.S + I.rb * kRowBlock + lane;
@@ -291,7 +291,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
             // L147), published as (m, 1/d) in a ring of NSI items.  Lane l reduces rows l + 32j.
             int si = 0;
             uint32_t sph = 0;
-            for (ItemWalk iw(p, it_begin, it_end); iw.more();) {
+            for (ItemWalk iw(sc, it_begin, it_end); iw.more();) {
                 const ItemInfo I = iw.next();
                 if (I.t0 == I.t1) continue;
                 DW_WAIT(&st_empty[si], sph ^ 1, 0);
@@ -304,7 +304,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                     float m8[4][8], d8[4][8];
                     int w8[8];
 #pragma unroll
-                    for (int u = 0; u < 8; ++u) w8[u] = tb + u < I.t1 ? __ldg(p.sc.tinfo + tb + u) : 0;
+                    for (int u = 0; u < 8; ++u) w8[u] = tb + u < I.t1 ? sld(sc.tinfo + tb + u) : 0;
 #pragma unroll
                     for (int u = 0; u < 8; ++u)
 #pragma unroll
@@ -349,14 +349,14 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
             int s = 0;
             const uint64_t pol_v = SR_G2_HINTS ? policy_evict_last() : 0;
             uint32_t sph = 0;
-            for (ItemWalk iw(p, it_begin, it_end); iw.more();) {
+            for (ItemWalk iw(sc, it_begin, it_end); iw.more();) {
                 const ItemInfo I = iw.next();
                 int wn[2];  // schedule words of the next macro tile, prefetched one step ahead
-                for (int u = 0; u < NSUB; ++u) wn[u] = I.t0 + u < I.t1 ? __ldg(p.sc.tinfo + I.t0 + u) : 0;
+                for (int u = 0; u < NSUB; ++u) wn[u] = I.t0 + u < I.t1 ? sld(sc.tinfo + I.t0 + u) : 0;
                 for (int t = I.t0; t < I.t1; t += NSUB) {
                     const int nsub = min(NSUB, I.t1 - t);
                     int kt[2] = {tinfo_kt(wn[0]), NSUB > 1 ? tinfo_kt(wn[1]) : 0};
-                    for (int u = 0; u < NSUB; ++u) wn[u] = t + NSUB + u < I.t1 ? __ldg(p.sc.tinfo + t + NSUB + u) : 0;
+                    for (int u = 0; u < NSUB; ++u) wn[u] = t + NSUB + u < I.t1 ? sld(sc.tinfo + t + NSUB + u) : 0;
                     DW_WAIT(&v_empty[s], sph ^ 1, 0);
                     if (elect_one()) {
 #ifdef SR_DIAG2_NOV
@@ -378,7 +378,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                             const int tp = t + C::NV * NSUB;
                             for (int u = 0; u < NSUB; ++u)
                                 if (tp + u < I.t1) {
-                                    const int ktp = tinfo_kt(__ldg(p.sc.tinfo + tp + u));
+                                    const int ktp = tinfo_kt(sld(sc.tinfo + tp + u));
                                     for (int h = 0; h < D / 64; ++h) tma_prefetch_2d(&tmV, h * 64, I.g * p.S + ktp * T);
                                 }
                         }
@@ -394,7 +394,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
         const uint32_t idesc = idesc_f16(0, kRowBlock, D, 0, 1);
         int s = 0, xs = 0, j = 0;
         uint32_t sph = 0, xph = 0, jph = 0;
-        for (ItemWalk iw(p, it_begin, it_end); iw.more();) {
+        for (ItemWalk iw(sc, it_begin, it_end); iw.more();) {
             const ItemInfo I = iw.next();
             if (I.t0 == I.t1) {  // the producer posted an EMPTY stage: add our release to it
                 DW_WAIT(&x_full[xs], xph, 1);
@@ -535,10 +535,10 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                 if (++o == C::NO) { o = 0; oph ^= 1; }
             };
             ItemInfo nxt;
-            if (it_begin < it_end) nxt = decode_item(p, it_begin);
+            if (it_begin < it_end) nxt = decode_item(sc, it_begin);
             for (int it = it_begin; it < it_end; ++it) {
                 const ItemInfo I = nxt;
-                if (it + 1 < it_end) nxt = decode_item(p, it + 1);  // prefetch
+                if (it + 1 < it_end) nxt = decode_item(sc, it + 1);  // prefetch
                 const int64_t orow = (int64_t)I.g * p.S + I.rb * kRowBlock;
                 if (I.t0 == I.t1) {  // no kept key in these rows: the epilogue writes zeros
                     post(SH_EMPTY, orow, true);

@@ -240,7 +240,7 @@ __global__ void __launch_bounds__(384, 1)
             const uint64_t pol_v = policy_evict_last();  // V is re-read by every row-block of its head
             int qi = 0, ks = 0;
             uint32_t qph = 0, kph = 0;
-            for (ItemWalk iw(p, it_begin, it_end); iw.more();) {
+            for (ItemWalk iw(p.sc, it_begin, it_end); iw.more();) {
                 const ItemInfo I = iw.next();
                 if (I.t0 == I.t1) continue;
                 mbar_wait(&q_empty[qi], qph ^ 1);
@@ -274,7 +274,7 @@ __global__ void __launch_bounds__(384, 1)
             const uint64_t pol_k = policy_evict_last();  // K is re-read by every row-block of its head
             int ks = 0;
             uint32_t kph = 0;
-            for (ItemWalk iw(p, it_begin, it_end); iw.more();) {
+            for (ItemWalk iw(p.sc, it_begin, it_end); iw.more();) {
                 const ItemInfo I = iw.next();
                 for (int t = I.t0; t < I.t1; t += NSUB) {
                     const int nsub = min(NSUB, I.t1 - t);
@@ -298,7 +298,7 @@ __global__ void __launch_bounds__(384, 1)
             // X' is streamed (evict_first) unless X' and dS' together fit in half the L2 (p.x_evict_first)
             const uint64_t pol_x = p.x_evict_first ? policy_evict_first() : policy_evict_normal();
             int n = 0;  // macro tile counter, as the MMA warp and the epilogue count them
-            for (ItemWalk iw(p, it_begin, it_end); iw.more();) {
+            for (ItemWalk iw(p.sc, it_begin, it_end); iw.more();) {
                 const ItemInfo I = iw.next();
                 for (int t = I.t0; t < I.t1; t += NSUB) {
                     const int nsub = min(NSUB, I.t1 - t);
@@ -372,7 +372,7 @@ __global__ void __launch_bounds__(384, 1)
                 if (++qs == C::NKQ) { qs = 0; qsph ^= 1; }
                 pn = -1;
             };
-            for (ItemWalk iw(p, it_begin, it_end); iw.more();) {
+            for (ItemWalk iw(p.sc, it_begin, it_end); iw.more();) {
                 const ItemInfo I = iw.next();
                 if (I.t0 == I.t1) continue;
                 const int64_t row0 = (int64_t)I.g * p.S + I.rb * kRowBlock;

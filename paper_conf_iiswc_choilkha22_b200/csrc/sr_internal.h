@@ -101,6 +101,14 @@ struct Params {
     int bwd_dq_fused;  // dQ accumulated inside the dS' kernel (default; SR_BWD_DQ_SEPARATE=1: own kernel)
 };
 
+// Generic load of schedule data: the schedule may live in the workspace (global memory) or, for the
+// one-launch kernel with a small schedule, in the kernel's own parameter space (k_fused.cu).
+template <class T>
+__device__ __forceinline__ T sld(const T* ptr)
+{
+    return *ptr;
+}
+
 __host__ __device__ inline int lh_of(const DevSched& s, int g, int H)
 {
     return s.lh_mode == LH_ONE ? 0 : (s.lh_mode == LH_BATCH ? g / H : g % H);
@@ -150,6 +158,14 @@ cudaError_t launch_tc_fused(const Params& p, cudaStream_t st, int64_t* nlaunch);
 cudaError_t launch_tc_unfused(const Params& p, cudaStream_t st, int64_t* nlaunch);
 cudaError_t launch_tc_sd(const Params& p, cudaStream_t st, int64_t* nlaunch);
 cudaError_t launch_tc_bwd(const Params& p, cudaStream_t st, int64_t* nlaunch);
-cudaError_t launch_tc_one(const Params& p, cudaStream_t st, int64_t* nlaunch);
+// one-launch kernel; blob != nullptr: the schedule words ride in the kernel parameters (p.sc pointer
+// fields hold byte offsets + 16 into blob), at most one_kernel_blob_words() words
+cudaError_t launch_tc_one(const Params& p, const int32_t* blob, size_t blob_words, cudaStream_t st, int64_t* nlaunch);
+size_t one_kernel_blob_words();
+// k_sched.cu: enqueue copies of n_seg word ranges [seg_off, seg_off + seg_len) of `words` (int32
+// offsets / lengths, multiples of 4) into the same offsets of `region` (device, 16-B aligned),
+// carried in kernel parameters
+cudaError_t launch_sched_upload(void* region, const int32_t* words, const size_t* seg_off, const size_t* seg_len,
+                                int n_seg, cudaStream_t st, int64_t* nlaunch);
 
 }  // namespace sr

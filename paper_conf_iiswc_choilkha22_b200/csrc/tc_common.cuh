@@ -58,38 +58,38 @@ struct ItemInfo {
     int64_t slot0;  // slot id of tile t is slot0 + t
 };
 
-__device__ __forceinline__ int4 item_desc(const Params& p, int it)
+__device__ __forceinline__ int4 item_desc(const DevSched& sc, int it)
 {
-    return it < 0 ? make_int4(0, 0, 0, 0) : __ldg(p.sc.item_desc + it);  // precomputed on the host
+    return it < 0 ? make_int4(0, 0, 0, 0) : sld(sc.item_desc + it);  // precomputed on the host
 }
-__device__ __forceinline__ ItemInfo item_info(const Params& p, int4 d)
+__device__ __forceinline__ ItemInfo item_info(const DevSched& sc, int4 d)
 {
     ItemInfo r;
-    r.g = d.x / p.sc.n_rb;
-    r.rb = d.x % p.sc.n_rb;
+    r.g = d.x / sc.n_rb;
+    r.rb = d.x % sc.n_rb;
     r.t0 = d.y;
     r.t1 = d.z;
-    r.slot0 = (int64_t)r.g * p.sc.slots_per_head - d.w;
+    r.slot0 = (int64_t)r.g * sc.slots_per_head - d.w;
     return r;
 }
-__device__ __forceinline__ ItemInfo decode_item(const Params& p, int it) { return item_info(p, item_desc(p, it)); }
+__device__ __forceinline__ ItemInfo decode_item(const DevSched& sc, int it) { return item_info(sc, item_desc(sc, it)); }
 
 // Walks [it_begin, it_end) with the next item's descriptor load in flight while the current item
-// runs:  for (ItemWalk w(p, b, e); w.more(); ) { const ItemInfo I = w.next(); ... }
+// runs:  for (ItemWalk w(sc, b, e); w.more(); ) { const ItemInfo I = w.next(); ... }
 struct ItemWalk {
-    const Params& p;
+    const DevSched& sc;
     int it, end;
     int4 nd;
-    __device__ __forceinline__ ItemWalk(const Params& p_, int b, int e) : p(p_), it(b), end(e)
+    __device__ __forceinline__ ItemWalk(const DevSched& sc_, int b, int e) : sc(sc_), it(b), end(e)
     {
-        nd = item_desc(p, it < end ? it : -1);
+        nd = item_desc(sc, it < end ? it : -1);
     }
     __device__ __forceinline__ bool more() const { return it < end; }
     __device__ __forceinline__ ItemInfo next()
     {
-        const ItemInfo I = item_info(p, nd);
+        const ItemInfo I = item_info(sc, nd);
         ++it;
-        nd = item_desc(p, it < end ? it : -1);
+        nd = item_desc(sc, it < end ? it : -1);
         return I;
     }
 };

@@ -7,9 +7,9 @@ the [B, H, S, D] layout -- and runs it as a layer of B' = n heads, H' = 1, with 
 re-packed (kv_len per head, one block layout per head).  Ranges are balanced by tile count
 (padding and layouts make per-head work uneven) while staying contiguous.
 
-bench.py measures weak scaling (every rank runs its own full layer); this module is what
-tools/multi_gpu_validate.py uses to split ONE layer and gather the output shards over NCCL for
-validation (tests/test_dist_gloo.py covers the same logic with gloo on CPU).
+bench.py --gpus N splits ONE layer this way (strong scaling: layer time = max over ranks) and also
+times each shard on one GPU (strong_scaling_shards); tools/multi_gpu_validate.py gathers the output
+shards over NCCL for validation (tests/test_dist_gloo.py covers the same logic with gloo on CPU).
 """
 from __future__ import annotations
 
@@ -67,18 +67,51 @@ def contiguous_ranges(costs, world: int):
     return [(cuts[r], cuts[r + 1]) for r in range(world)]
 
 
-def head_costs(B: int, H: int, S: int, T: int = 128, kv_len=None, layout=None):
-    """Relative work per flat head: kept key tiles per head (uniform for unpadded dense/window)."""
+def head_costs(B: int, H: int, S: int, T: int = 64, kv_len=None, layout=None, causal: bool = False):
+    """Relative work per flat head: its listed (row-block, key-tile) tiles at sub-vector width T (the
+    library default T = 64) plus a fixed cost of 1.5 tiles per row-block (Q load, row statistics,
+    O store), the same cost model as the library's LPT CTA schedule (abi.cu).  Heads of an unpadded
+    dense or windowed layer all cost the same."""
+    n_rb = S // 128
+    fixed = 1.5 * n_rb
     if kv_len is not None:
-        return [int(np.ceil(kv_len[g // H] / T)) for g in range(B * H)]
+        def tiles(kv):
+            n = 0
+            for rb in range(n_rb):
+                hi = kv if not causal else min(kv, (rb + 1) * 128)
+                n += -(-hi // T) if hi > 0 else 0
+            return n
+        per_b = [tiles(int(k)) for k in kv_len]
+        return [per_b[g // H] + fixed for g in range(B * H)]
     if layout is not None:
         rp = np.asarray(layout.row_ptr)
-        return [int(rp[lh, -1] - rp[lh, 0]) for lh in ((0 if rp.shape[0] == 1 else g % H) for g in range(B * H))]
-    return [1] * (B * H)
+        ci = np.asarray(layout.col_idx)
+
+        def tiles_lh(lh):  # block-rows 2p, 2p+1 share a 128-row tile over the union of their columns
+            n = 0
+            for p in range(n_rb):
+                cols = set()
+                for br in (2 * p, 2 * p + 1):
+                    c = ci[rp[lh, br]:rp[lh, br + 1]].tolist()
+                    cols.update(x for x in c if not causal or x <= br)
+                n += len(cols)
+            return n
+        per_lh = {}
+        out = []
+        for g in range(B * H):
+            lh = 0 if rp.shape[0] == 1 else g % H
+            if lh not in per_lh:
+                per_lh[lh] = tiles_lh(lh)
+            out.append(per_lh[lh] + fixed)
+        return out
+    return [1.0] * (B * H)
 
 
-def make_shard(rank: int, world: int, B: int, H: int, S: int, kv_len=None, layout=None, T: int = 128) -> Shard:
-    g0, g1 = contiguous_ranges(head_costs(B, H, S, T, kv_len, layout), world)[rank]
+def make_shard(rank: int, world: int, B: int, H: int, S: int, kv_len=None, layout=None, T: int = 64,
+               causal: bool = False, **_mask) -> Shard:
+    """Rank `rank`'s shard of the layer (window / n_global / kind in **_mask do not change per-head
+    costs: every head of a windowed layer has the same tiles)."""
+    g0, g1 = contiguous_ranges(head_costs(B, H, S, T, kv_len, layout, causal), world)[rank]
     sh = Shard(g0, g1)
     if kv_len is not None:
         sh.kv_len = np.asarray([kv_len[g // H] for g in range(g0, g1)], dtype=np.int32)
