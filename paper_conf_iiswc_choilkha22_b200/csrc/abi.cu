@@ -316,7 +316,7 @@ enum BlobGroup { G_BASE = 0, G_ITEMS, G_PAIR, G_FP, G_COL, G_N };
 constexpr int kMaxCta = 1024;  // bound on persistent CTAs per launch (the workspace reserves it)
 
 struct BlobLayout {  // int32-word offsets inside the blob
-    size_t tp, tinfo, kv, desc, items, cta, pdesc, pent, pcta, fp, fpcta, cdesc, cent, ccta;
+    size_t tp, tinfo, kv, desc, items, cta, iri, pdesc, pent, pcta, fp, fpcta, cdesc, cent, ccta;
     size_t g_off[G_N], g_len[G_N];
     size_t words;
 };
@@ -326,10 +326,6 @@ struct DevBlob {
     std::vector<int32_t> w;
     BlobLayout L{};
     DevSched rel{};  // scalar fields of the device schedule (pointers filled per call)
-    // the groups a one-launch call reads, packed back to back for its kernel parameters (per group
-    // mask; built on first use)
-    std::mutex mu;
-    std::map<unsigned, std::shared_ptr<const std::vector<int32_t>>> packed;
 };
 
 struct CachedSched {
@@ -379,6 +375,7 @@ BlobLayout blob_layout(const HostSched& h, size_t n_cta_ptr, size_t n_pcta_ptr, 
     L.desc = o; o += 4 * h.items.size();
     L.items = o; o += h.items.size();
     L.cta = o; o += n_cta_ptr;
+    L.iri = o; o += h.items.size();  // the standalone IR kernel's row-block order (longest first)
     grp(G_ITEMS, s);
     s = o;  // G_PAIR: pair descriptors, union entries, pcta_ptr
     L.pdesc = o; o += 4 * h.pitems.size();
@@ -431,6 +428,7 @@ std::shared_ptr<DevBlob> make_blob(const HostSched& h0, int n_sm)
     }
     put(L.items, h.items);
     put(L.cta, h.cta_ptr);
+    put(L.iri, h0.items);  // before the LPT pass: longest first
     o = L.pdesc;  // pair item descriptors {g * n_pair + j, e0, e1, tp[lh][0]}
     for (int32_t it : h.pitems) {
         const int g = it / h.n_pair, j = it % h.n_pair, lh = lh_of_g(g);
@@ -476,55 +474,23 @@ std::shared_ptr<DevBlob> make_blob(const HostSched& h0, int n_sm)
     d.max_rb_tiles = h.max_rb_tiles;
     d.mean_rb_tiles = (int)((h.tinfo.size() + (size_t)h.n_lh * h.n_rb - 1) / ((size_t)h.n_lh * h.n_rb));
     d.n_items = (int)h.items.size();
+    {   // the IR kernel's team classes over iri (longest first): 8 warps for > 4 * kIrWarpTiles tiles,
+        // then 4, 2, 1 (each warp merges <= kIrWarpTiles tiles in registers)
+        auto lh_of_g2 = [&](int g) { return h0.lh_mode == LH_ONE ? 0 : (h0.lh_mode == LH_BATCH ? g / h0.H : g % h0.H); };
+        for (int c = 0; c < 4; ++c) d.n_ir_class[c] = 0;
+        for (int32_t it : h0.items) {
+            const int g = it / h0.n_rb, rb = it % h0.n_rb;
+            const int32_t* tp = &h0.tp[(size_t)lh_of_g2(g) * (h0.n_rb + 1)];
+            const int n = tp[rb + 1] - tp[rb];
+            d.n_ir_class[n > 4 * kIrWarpTiles ? 0 : n > 2 * kIrWarpTiles ? 1 : n > kIrWarpTiles ? 2 : 3]++;
+        }
+    }
     d.n_cta = (int)h.cta_ptr.size() - 1;
     d.n_pair = h.n_pair;
     d.n_pcta = (int)h.pcta_ptr.size() - 1;
     d.n_cb = h.n_cb;
     d.n_ccta = (int)h.ccta_ptr.size() - 1;
     return db;
-}
-
-// The groups `groups` of a blob packed back to back (the one-launch kernel's parameter form), and
-// the device schedule whose pointer fields are byte offsets + 16 into that packing (0: not packed).
-std::shared_ptr<const std::vector<int32_t>> packed_blob(DevBlob& db, unsigned groups, DevSched& d, bool has_kv)
-{
-    size_t at[G_N], n = 0;
-    for (int g = 0; g < G_N; ++g) {
-        at[g] = SIZE_MAX;
-        if ((groups >> g) & 1) {
-            at[g] = n;
-            n += db.L.g_len[g];
-        }
-    }
-    auto rel = [&](size_t field, int g) -> uintptr_t {
-        return at[g] == SIZE_MAX ? 0 : (uintptr_t)((at[g] + field - db.L.g_off[g]) * sizeof(int32_t) + 16);
-    };
-    const BlobLayout& L = db.L;
-    d = db.rel;
-    d.tp = (const int32_t*)rel(L.tp, G_BASE);
-    d.tinfo = (const int32_t*)rel(L.tinfo, G_BASE);
-    d.kv_len = has_kv ? (const int32_t*)rel(L.kv, G_BASE) : nullptr;
-    d.item_desc = (const int4*)rel(L.desc, G_ITEMS);
-    d.items = (const int32_t*)rel(L.items, G_ITEMS);
-    d.cta_ptr = (const int32_t*)rel(L.cta, G_ITEMS);
-    d.pair_desc = (const int4*)rel(L.pdesc, G_PAIR);
-    d.pent = (const int4*)rel(L.pent, G_PAIR);
-    d.pcta_ptr = (const int32_t*)rel(L.pcta, G_PAIR);
-    d.fp_desc = (const int4*)rel(L.fp, G_FP);
-    d.fpcta_ptr = (const int32_t*)rel(L.fpcta, G_FP);
-    d.col_desc = (const int4*)rel(L.cdesc, G_COL);
-    d.cent = (const int4*)rel(L.cent, G_COL);
-    d.ccta_ptr = (const int32_t*)rel(L.ccta, G_COL);
-    std::lock_guard<std::mutex> lk(db.mu);
-    auto it = db.packed.find(groups);
-    if (it != db.packed.end()) return it->second;
-    auto pk = std::make_shared<std::vector<int32_t>>();
-    pk->reserve(n);
-    for (int g = 0; g < G_N; ++g)
-        if ((groups >> g) & 1)
-            pk->insert(pk->end(), db.w.begin() + db.L.g_off[g], db.w.begin() + db.L.g_off[g] + db.L.g_len[g]);
-    db.packed.emplace(groups, pk);
-    return pk;
 }
 
 // The device schedule with its pointers inside a workspace's schedule region.
@@ -539,6 +505,7 @@ DevSched place(const DevBlob& db, void* region, bool has_kv)
     d.item_desc = (const int4*)(b + L.desc);
     d.items = b + L.items;
     d.cta_ptr = b + L.cta;
+    d.ir_items = b + L.iri;
     d.pair_desc = (const int4*)(b + L.pdesc);
     d.pent = (const int4*)(b + L.pent);
     d.pcta_ptr = b + L.pcta;
@@ -862,18 +829,7 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
     const bool one_pair = fused == 1 && one && p.g1_pair;
     const unsigned groups = one_pair ? (1u << G_BASE | 1u << G_PAIR | 1u << G_FP)
                                      : (1u << G_BASE | 1u << G_ITEMS | (p.g1_pair ? 1u << G_PAIR : 0u));
-    // the one-launch kernel carries a small schedule in its own parameters; everything else reads
-    // it from the workspace, uploaded ahead of the kernels
-    size_t gw = 0;
-    for (int g = 0; g < G_N; ++g) gw += ((groups >> g) & 1) ? db->L.g_len[g] : 0;
-    std::shared_ptr<const std::vector<int32_t>> pk;
-#ifndef SR_NO_BLOB  // experiment builds: always upload into the workspace
-    if (fused == 1 && one && gw <= one_kernel_blob_words())
-#else
-    if (false)
-#endif
-        pk = packed_blob(*db, groups, p.sc, r.kv_len != nullptr);
-    else if (!(ex->flags & SR_SCHED_RESIDENT) && (ce = upload(*db, region, groups, st, &nl)) != cudaSuccess) {
+    if (!(ex->flags & SR_SCHED_RESIDENT) && (ce = upload(*db, region, groups, st, &nl)) != cudaSuccess) {
         g_launches += nl;
         return fail(SR_ERR_CUDA, "schedule upload: %s", cudaGetErrorString(ce));
     }
@@ -889,7 +845,7 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
         }
         p.gs_prologue = (ex->flags & SR_GS_PROLOGUE) != 0;
 
-        ce = launch_tc_one(p, pk ? pk->data() : nullptr, pk ? pk->size() : 0, st, &nl);
+        ce = launch_tc_one(p, st, &nl);
     } else if (fused) {
         ce = ex->in_dtype == SR_F32 ? launch_simt_f32(p, st, &nl) : launch_tc_fused(p, st, &nl);
     } else {

@@ -197,11 +197,11 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                     continue;
                 }
                 int wn[2];  // schedule words of the next macro tile, prefetched one step ahead
-                for (int u = 0; u < NSUB; ++u) wn[u] = I.t0 + u < I.t1 ? sld(sc.tinfo + I.t0 + u) : 0;
+                for (int u = 0; u < NSUB; ++u) wn[u] = I.t0 + u < I.t1 ? __ldg(sc.tinfo + I.t0 + u) : 0;
                 for (int t = I.t0; t < I.t1; t += NSUB) {
                     const int nsub = min(NSUB, I.t1 - t);
                     int hv[2] = {tinfo_half(wn[0]), NSUB > 1 ? tinfo_half(wn[1]) : 0};
-                    for (int u = 0; u < NSUB; ++u) wn[u] = t + NSUB + u < I.t1 ? sld(sc.tinfo + t + NSUB + u) : 0;
+                    for (int u = 0; u < NSUB; ++u) wn[u] = t + NSUB + u < I.t1 ? __ldg(sc.tinfo + t + NSUB + u) : 0;
                     uint32_t bytes = GS ? nsub * kRowBlock * 4 : 0;
 #ifndef SR_DIAG2_NOX
                     for (int u = 0; u < nsub; ++u) bytes += ((GS && !AS) ? (hv[u] == 3 ? 2 : 1) : 2) * (T / 64) * (kHalf * 128);
@@ -304,7 +304,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                     float m8[4][8], d8[4][8];
                     int w8[8];
 #pragma unroll
-                    for (int u = 0; u < 8; ++u) w8[u] = tb + u < I.t1 ? sld(sc.tinfo + tb + u) : 0;
+                    for (int u = 0; u < 8; ++u) w8[u] = tb + u < I.t1 ? __ldg(sc.tinfo + tb + u) : 0;
 #pragma unroll
                     for (int u = 0; u < 8; ++u)
 #pragma unroll
@@ -352,11 +352,11 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
             for (ItemWalk iw(sc, it_begin, it_end); iw.more();) {
                 const ItemInfo I = iw.next();
                 int wn[2];  // schedule words of the next macro tile, prefetched one step ahead
-                for (int u = 0; u < NSUB; ++u) wn[u] = I.t0 + u < I.t1 ? sld(sc.tinfo + I.t0 + u) : 0;
+                for (int u = 0; u < NSUB; ++u) wn[u] = I.t0 + u < I.t1 ? __ldg(sc.tinfo + I.t0 + u) : 0;
                 for (int t = I.t0; t < I.t1; t += NSUB) {
                     const int nsub = min(NSUB, I.t1 - t);
                     int kt[2] = {tinfo_kt(wn[0]), NSUB > 1 ? tinfo_kt(wn[1]) : 0};
-                    for (int u = 0; u < NSUB; ++u) wn[u] = t + NSUB + u < I.t1 ? sld(sc.tinfo + t + NSUB + u) : 0;
+                    for (int u = 0; u < NSUB; ++u) wn[u] = t + NSUB + u < I.t1 ? __ldg(sc.tinfo + t + NSUB + u) : 0;
                     DW_WAIT(&v_empty[s], sph ^ 1, 0);
                     if (elect_one()) {
 #ifdef SR_DIAG2_NOV
@@ -378,7 +378,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                             const int tp = t + C::NV * NSUB;
                             for (int u = 0; u < NSUB; ++u)
                                 if (tp + u < I.t1) {
-                                    const int ktp = tinfo_kt(sld(sc.tinfo + tp + u));
+                                    const int ktp = tinfo_kt(__ldg(sc.tinfo + tp + u));
                                     for (int h = 0; h < D / 64; ++h) tma_prefetch_2d(&tmV, h * 64, I.g * p.S + ktp * T);
                                 }
                         }

@@ -14,8 +14,6 @@
 // spill the setmaxnreg-rebalanced epilogues.  X' stores stay evict_first.
 // T = 64 (reading R3): the SPLIT GEMM1 epilogue (four warpgroups, 104 registers) leaves the
 // register budget of a 640-thread CTA that GEMM2's 16 warps can reuse in phase 2.
-#include <cstring>
-
 #include "g1_body.cuh"
 #include "g2_body.cuh"
 
@@ -38,50 +36,20 @@ __device__ __forceinline__ unsigned long long gtimer()
 #define PH_MARK(i)
 #endif
 
-// The tile schedule of a call rides in this kernel's parameters when it fits (kBlobWords int32
-// words): every CTA reads its items and tile lists straight from parameter space -- no upload
-// kernel, no workspace round trip, nothing for a CUDA graph to depend on.  Larger schedules are
-// uploaded into the workspace first (k_sched.cu) and read from there (BLOB = false).  Pointer fields
-// of p.sc then hold byte offsets + 16 into the blob (0 = absent) and are rebased here.
-constexpr int kBlobWords = 6912;  // 27 KB; the whole parameter block stays under 32764 B
-template <bool BLOB>
-struct SchedBlob {
-    int32_t w[BLOB ? kBlobWords : 4];
-};
-static_assert(3 * sizeof(CUtensorMap) + sizeof(Params) + sizeof(SchedBlob<true>) + 256 <= 32764,
-              "kernel parameter space");
-
-template <class T>
-__device__ __forceinline__ void rebase(const T*& ptr, uintptr_t base)
-{
-    if (ptr) ptr = (const T*)(base + (uintptr_t)ptr - 16);
-}
-
-template <int D, bool PAIR, bool BLOB>
+template <int D, bool PAIR>
 __global__ void __launch_bounds__(640, 1)
     tc_fused(const __grid_constant__ CUtensorMap tmQ, const __grid_constant__ CUtensorMap tmK,
-             const __grid_constant__ CUtensorMap tmV, const Params p, const __grid_constant__ SchedBlob<BLOB> sb)
+             const __grid_constant__ CUtensorMap tmV, const Params p)
 {
     using C1 = G1<D, 64, PAIR>;
     using C2 = G2<D, 64>;
     static_assert(C1::THREADS == 640 && C2::THREADS <= 640, "warp budget");
     extern __shared__ uint8_t smem_raw[];
-    __shared__ DevSched sc;  // the schedule's pointers as this kernel reads them
     uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
     uint32_t* tmem_ptr = (uint32_t*)(smem + C1::OFF_TPTR);
     const int warp = warp_uniform(), lane = threadIdx.x % 32;
+    const DevSched& sc = p.sc;  // the schedule the call uploaded into its workspace (k_sched.cu)
     PH_MARK(0);
-    if (threadIdx.x == 32) {
-        DevSched s = p.sc;
-        if constexpr (BLOB) {
-            const uintptr_t b = (uintptr_t)&sb.w[0];
-            rebase(s.tp, b); rebase(s.tinfo, b); rebase(s.items, b); rebase(s.cta_ptr, b);
-            rebase(s.item_desc, b); rebase(s.pair_desc, b); rebase(s.pent, b); rebase(s.pcta_ptr, b);
-            rebase(s.fp_desc, b); rebase(s.fpcta_ptr, b); rebase(s.kv_len, b); rebase(s.col_desc, b);
-            rebase(s.cent, b); rebase(s.ccta_ptr, b);
-        }
-        sc = s;
-    }
     if (threadIdx.x == 0) g1_init<D, 64, true, PAIR, true>(smem);
     if (warp == 0 && lane == 0) { prefetch_tmap(&tmQ); prefetch_tmap(&tmK); prefetch_tmap(&tmV); }
     if (warp == 2) tmem_alloc(tmem_ptr, 512);
@@ -94,7 +62,7 @@ __global__ void __launch_bounds__(640, 1)
 
     // phase 2's row-blocks (with PAIR the host pointed cta_ptr / item_desc at the pair assignment
     // unrolled into row-blocks, so both phases cover the same rows)
-    const int it_begin = sld(sc.cta_ptr + blockIdx.x), it_end = sld(sc.cta_ptr + blockIdx.x + 1);
+    const int it_begin = __ldg(sc.cta_ptr + blockIdx.x), it_end = __ldg(sc.cta_ptr + blockIdx.x + 1);
     // phase 2 applies Global Scaling accumulator-side for fp16 (X' and V share the MMA type; see
     // g2_body.cuh AS) unless p.gs_prologue; bf16 V needs the prologue form (Y rounded to bf16)
     // (D = 64: the scaling warps hold D/2 fp32 of O each within the 96-register phase-2 budget)
@@ -102,8 +70,8 @@ __global__ void __launch_bounds__(640, 1)
     PH_MARK(1);
     // ---- phase 1: GEMM1 + LS + IR over the CTA's row-blocks (all 20 warps)
     if constexpr (PAIR)
-        g1_roles<D, 64, true, true, true>(tmQ, tmK, p, sc, smem, tmem_base, sld(sc.pcta_ptr + blockIdx.x),
-                                          sld(sc.pcta_ptr + blockIdx.x + 1));
+        g1_roles<D, 64, true, true, true>(tmQ, tmK, p, sc, smem, tmem_base, __ldg(sc.pcta_ptr + blockIdx.x),
+                                          __ldg(sc.pcta_ptr + blockIdx.x + 1));
     else
         g1_roles<D, 64, true, false, true>(tmQ, tmK, p, sc, smem, tmem_base, it_begin, it_end);
     // back to the launch split (phase 1 leaves warps 0-3 at 64 registers, the epilogue at 104)
@@ -144,8 +112,8 @@ __global__ void __launch_bounds__(640, 1)
 
 cudaError_t make_tmap_2d(CUtensorMap* m, const void* base, int64_t rows, int D, int box_rows, int dtype);
 
-template <int D, bool BLOB>
-cudaError_t launch_one_b(const Params& p, const int32_t* blob, size_t blob_words, cudaStream_t st, int64_t* nl)
+template <int D>
+cudaError_t launch_one_d(const Params& p, cudaStream_t st, int64_t* nl)
 {
     CUtensorMap tq, tk, tv;
     const int64_t rows = (int64_t)p.B * p.H * p.S;
@@ -155,24 +123,16 @@ cudaError_t launch_one_b(const Params& p, const int32_t* blob, size_t blob_words
     if ((e = make_tmap_2d(&tv, p.v, rows, D, 64, p.in_dtype)) != cudaSuccess) return e;
     constexpr int s0 = G1<D, 64, false>::SMEM > G2<D, 64>::SMEM ? G1<D, 64, false>::SMEM : G2<D, 64>::SMEM;
     constexpr int s1 = G1<D, 64, true>::SMEM > G2<D, 64>::SMEM ? G1<D, 64, true>::SMEM : G2<D, 64>::SMEM;
-    static_assert(s0 + 1024 <= kSmemMax && s1 + 1024 <= kSmemMax, "dynamic + static shared memory");
-    auto kern = p.g1_pair ? tc_fused<D, true, BLOB> : tc_fused<D, false, BLOB>;
+    auto kern = p.g1_pair ? tc_fused<D, true> : tc_fused<D, false>;
     const int smem = p.g1_pair ? s1 : s0;
     if ((e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem)) != cudaSuccess) return e;
-    thread_local SchedBlob<BLOB> sb;  // staging of the launch parameters (copied at launch)
-    if (BLOB) memcpy(sb.w, blob, blob_words * sizeof(int32_t));
-    return launch_pdl(kern, dim3(p.sc.n_cta), dim3(640), smem, st, nl, tq, tk, tv, p, sb);
+    return launch_pdl(kern, dim3(p.sc.n_cta), dim3(640), smem, st, nl, tq, tk, tv, p);
 }
 
-size_t one_kernel_blob_words() { return kBlobWords; }
-
-cudaError_t launch_tc_one(const Params& p, const int32_t* blob, size_t blob_words, cudaStream_t st, int64_t* nl)
+cudaError_t launch_tc_one(const Params& p, cudaStream_t st, int64_t* nl)
 {
     if (p.T != 64) return cudaErrorInvalidValue;
-    if (blob && blob_words > (size_t)kBlobWords) return cudaErrorInvalidValue;
-    if (blob) return p.D == 64 ? launch_one_b<64, true>(p, blob, blob_words, st, nl)
-                               : launch_one_b<128, true>(p, blob, blob_words, st, nl);
-    return p.D == 64 ? launch_one_b<64, false>(p, nullptr, 0, st, nl) : launch_one_b<128, false>(p, nullptr, 0, st, nl);
+    return p.D == 64 ? launch_one_d<64>(p, st, nl) : launch_one_d<128>(p, st, nl);
 }
 
 }  // namespace sr

@@ -37,14 +37,18 @@ static_assert(sizeof(SchedChunk) + sizeof(void*) <= 32764, "kernel parameter spa
 __global__ void __launch_bounds__(256) sched_upload(int4* __restrict__ region, const __grid_constant__ SchedChunk c)
 {
     ptx::griddep_launch_dependents();
-    ptx::griddep_wait();
+    // one 16-B word per thread (the grid covers the chunk): every load in flight at once.  The
+    // payload is read through its generic address (coalesced; indexed constant-bank loads with a
+    // different address per lane would serialise).
+    const int4* data;
+    asm("mov.b64 %0, %1;" : "=l"(data) : "l"(&c.data[0]));  // opaque to the compiler: stays generic
+    int i = blockIdx.x * blockDim.x + threadIdx.x, s = 0;
+    while (s < c.n_seg && i >= c.len[s]) i -= c.len[s++];
     int src = 0;
-    for (int s = 0; s < c.n_seg; ++s) {
-        const int n = c.len[s];
-        int4* d = region + c.dst[s];
-        for (int i = threadIdx.x; i < n; i += blockDim.x) d[i] = c.data[src + i];
-        src += n;
-    }
+    for (int k = 0; k < s; ++k) src += c.len[k];
+    const int4 v = s < c.n_seg ? data[src + i] : make_int4(0, 0, 0, 0);
+    ptx::griddep_wait();  // the previous kernel may still read the region
+    if (s < c.n_seg) region[c.dst[s] + i] = v;
 }
 
 }  // namespace
@@ -58,7 +62,8 @@ cudaError_t launch_sched_upload(void* region, const int32_t* words, const size_t
     cudaError_t e = cudaSuccess;
     auto flush = [&]() -> cudaError_t {
         if (c.n_seg == 0) return cudaSuccess;
-        cudaError_t r = launch_pdl(sched_upload, dim3(1), dim3(256), 0, st, nl, (int4*)region, c);
+        cudaError_t r = launch_pdl(sched_upload, dim3((unsigned)((fill + 255) / 256)), dim3(256), 0, st, nl,
+                                   (int4*)region, c);
         c.n_seg = 0;
         fill = 0;
         return r;

@@ -20,6 +20,7 @@ namespace sr {
 
 constexpr int kRowBlock = 128;  // M of every tcgen05 tile
 constexpr int kHalf = 64;       // validity granularity of tile rows
+constexpr int kIrWarpTiles = 8;  // IR kernel: tiles one warp merges in registers
 
 // Where the IR sub-layer runs: its own kernel (SR_IR_KERNEL, the paper's layout), folded into
 // GEMM2 (SR_FUSE_IR), or merged by warps of GEMM1 as the row's tiles are produced (default).
@@ -63,6 +64,10 @@ struct DevSched {
     const int4* cent;
     const int32_t* ccta_ptr;
     int n_cb, n_ccta;
+    // standalone IR kernel (SR_IR_KERNEL): row-blocks longest first, in classes of team size 8, 4, 2, 1
+    // warps (> 32, 17-32, 9-16, <= 8 tiles); n_ir_class[c] row-blocks in class c
+    const int32_t* ir_items;
+    int n_ir_class[4];
 };
 
 // Everything a kernel needs to know about one call.
@@ -100,14 +105,6 @@ struct Params {
     float* bstat;      // [3][B*H*S]: per query row m (natural log), 1/d, delta = sum_d dO * O
     int bwd_dq_fused;  // dQ accumulated inside the dS' kernel (default; SR_BWD_DQ_SEPARATE=1: own kernel)
 };
-
-// Generic load of schedule data: the schedule may live in the workspace (global memory) or, for the
-// one-launch kernel with a small schedule, in the kernel's own parameter space (k_fused.cu).
-template <class T>
-__device__ __forceinline__ T sld(const T* ptr)
-{
-    return *ptr;
-}
 
 __host__ __device__ inline int lh_of(const DevSched& s, int g, int H)
 {
@@ -158,10 +155,7 @@ cudaError_t launch_tc_fused(const Params& p, cudaStream_t st, int64_t* nlaunch);
 cudaError_t launch_tc_unfused(const Params& p, cudaStream_t st, int64_t* nlaunch);
 cudaError_t launch_tc_sd(const Params& p, cudaStream_t st, int64_t* nlaunch);
 cudaError_t launch_tc_bwd(const Params& p, cudaStream_t st, int64_t* nlaunch);
-// one-launch kernel; blob != nullptr: the schedule words ride in the kernel parameters (p.sc pointer
-// fields hold byte offsets + 16 into blob), at most one_kernel_blob_words() words
-cudaError_t launch_tc_one(const Params& p, const int32_t* blob, size_t blob_words, cudaStream_t st, int64_t* nlaunch);
-size_t one_kernel_blob_words();
+cudaError_t launch_tc_one(const Params& p, cudaStream_t st, int64_t* nlaunch);
 // k_sched.cu: enqueue copies of n_seg word ranges [seg_off, seg_off + seg_len) of `words` (int32
 // offsets / lengths, multiples of 4) into the same offsets of `region` (device, 16-B aligned),
 // carried in kernel parameters

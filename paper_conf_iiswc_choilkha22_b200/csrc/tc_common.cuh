@@ -60,7 +60,7 @@ struct ItemInfo {
 
 __device__ __forceinline__ int4 item_desc(const DevSched& sc, int it)
 {
-    return it < 0 ? make_int4(0, 0, 0, 0) : sld(sc.item_desc + it);  // precomputed on the host
+    return it < 0 ? make_int4(0, 0, 0, 0) : __ldg(sc.item_desc + it);  // precomputed on the host
 }
 __device__ __forceinline__ ItemInfo item_info(const DevSched& sc, int4 d)
 {

@@ -57,20 +57,57 @@ def _worker(rank, world, port, case, q):
     dist.destroy_process_group()
 
 
+@pytest.mark.parametrize("world", [2, 4, 8])
 @pytest.mark.parametrize("case", list(CASES))
-def test_shard_and_gather_world2(case):
+def test_shard_and_gather(case, world):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
-    port = 29500 + (abs(hash(case)) % 1000)
-    procs = [ctx.Process(target=_worker, args=(r, 2, port, case, q)) for r in range(2)]
+    port = 29500 + (abs(hash(case)) % 500) + 500 * (world // 4)
+    procs = [ctx.Process(target=_worker, args=(r, world, port, case, q)) for r in range(world)]
     for p in procs:
         p.start()
-    ok, sizes = q.get(timeout=120)
+    ok, sizes = q.get(timeout=240)
     for p in procs:
-        p.join(timeout=60)
+        p.join(timeout=120)
         assert p.exitcode == 0
     assert ok, sizes
     assert sum(sizes) == CASES[case]["B"] * CASES[case]["H"]
+
+
+def test_head_costs_match_library_schedule():
+    """shard.py's per-head cost model counts exactly the tiles the library's schedule lists
+    (sr_schedule_stats on a one-head layer), for padding + causal and per-head block layouts."""
+    import paper_conf_iiswc_choilkha22_b200 as sr
+    S = 512
+    kv = [512, 300, 65, 1]
+    for causal in (False, True):
+        costs = SH.head_costs(len(kv), 1, S, 64, kv_len=kv, causal=causal)
+        for b, k in enumerate(kv):
+            n, _ = sr.schedule_stats(sr.dense_mask([k]), 1, 1, S, causal=causal, tile_n=64)
+            assert costs[b] - 1.5 * (S // 128) == n, (k, causal)
+    lay = W.random_layout(3, S // 64, 64, 0.4, seed=2)
+    costs = SH.head_costs(1, 3, S, 64, layout=lay)
+    for h in range(3):
+        one = W.csr_from_sets(64, [[set(lay.blocks(h, r)) for r in range(S // 64)]])
+        n, _ = sr.schedule_stats(sr.block_mask(one), 1, 1, S, tile_n=64)
+        assert costs[h] - 1.5 * (S // 128) == n
+
+
+def test_bench_shards_cover_the_layer():
+    """bench.py --gpus N splits each BASELINE config's heads into N contiguous shards that cover
+    every head exactly once, with per-shard masks re-packed."""
+    import bench
+    for idx in (2, 3, 4, 5):
+        cfg = W.config(idx)
+        for world in (2, 4, 8):
+            shards = [bench.make_shard(cfg, r, world) for r in range(world)]
+            assert shards[0].g0 == 0 and shards[-1].g1 == cfg.BH
+            assert all(a.g1 == b.g0 for a, b in zip(shards, shards[1:]))
+            for sh in shards:
+                if cfg.kv_len is not None:
+                    assert list(sh.kv_len) == [cfg.kv_len[g // cfg.H] for g in range(sh.g0, sh.g1)]
+                if cfg.kind == "blocksparse":
+                    assert sh.layout.layout_heads == sh.n
 
 
 def test_contiguous_ranges_balance():
