@@ -296,9 +296,16 @@ def steps_graph(torch, fns, K):
     return g
 
 
-def region(torch, g, K):
-    """Device ms per layer of one replay of the K-step graph (events around it)."""
-    torch.cuda._sleep(SPIN_CYCLES)
+def region(torch, g, K, spin=SPIN_CYCLES, warm=None):
+    """Device ms per layer of one replay of the K-step graph (events around it).  Before the first
+    event the device either spins (so a late host submission of the replay never shows up as idle
+    time inside the region) or, with `warm`, runs that graph once more untimed: the timed steps then
+    start from the steady state of the preceding warm-up steps (a region that starts cold, right
+    after the idle sync, runs slower under the 1 kW power cap while the clock controller reacts)."""
+    if warm is not None:
+        warm.replay()
+    else:
+        torch.cuda._sleep(spin)
     a = torch.cuda.Event(enable_timing=True)
     b = torch.cuda.Event(enable_timing=True)
     a.record()
@@ -404,9 +411,14 @@ def gpu_arm(args, rank, world, local_rank):
         g_tp.replay()
     torch.cuda.synchronize()
     barrier(torch, world)
-    ms_rank = region(torch, g_tp, K)  # THE timed region: exactly K steps
+    # THE timed region: exactly K steps, right after >= W untimed warm-up steps on the same stream
+    # (a replay of the same K-step graph), barrier + synchronize before the warm-up and after
+    ms_rank = region(torch, g_tp, K, warm=g_tp)
     barrier(torch, world)
-    extra = [region(torch, g_tp, K) for _ in range(4)]
+    extra = []
+    for _ in range(4):
+        barrier(torch, world)
+        extra.append(region(torch, g_tp, K, warm=g_tp))
     clocks = clk.stop()
     ms_step = dist_max(torch, ms_rank, world)
     step_spread = spread([dist_max(torch, x, world) for x in [ms_rank] + extra])
@@ -563,7 +575,8 @@ def gpu_arm(args, rank, world, local_rank):
         "n_gpus": world, "steps": K, "warmup": Wm,
         "ms_per_step": round(ms_step, 5),
         "timing": f"one region of exactly K={K} back-to-back layer calls (C ABI, captured in one CUDA graph) between "
-                  f"two events after >= {Wm} warm-up steps, barrier + synchronize around it, max over ranks; "
+                  f"two events, right after max(W={Wm}, K) untimed warm-up steps on the same stream, barrier + "
+                  "synchronize before the warm-up and after the region, max over ranks; "
                   f"{n_sets} rotating input/workspace sets "
                   f"({rot_bytes / 2**20:.0f} MiB > 2x L2) so no step finds its data in L2; step_ms = spread over "
                   "that region and 4 more",
