@@ -92,8 +92,9 @@ class Clocks:
         mx = [float(r[2]) for r in rows if r[2].strip().replace(".", "").isdigit()]
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         reasons = sorted({n for r in rows for n, v in zip(names, r[5:9]) if v.strip() == "Active"})
+        pw = [float(r[3]) for r in rows if r[3].strip().replace(".", "").isdigit()]
         return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": reasons, "samples": len(rows)}
+                "reasons": reasons, "samples": len(rows), "power_w_median": statistics.median(pw) if pw else None}
 
 
 # ----------------------------------------------------------------------------- byte model
@@ -553,6 +554,11 @@ def gpu_arm(args, rank, world, local_rank):
         torch.cuda.empty_cache()
         strong_model = shard_model(args, cfg, device, sr, torch, K, Wm, ms_step)
 
+    # ---- NEXT-3 (Fig. 9): sequence length and batch around GPT-Neo (C3), N = 1
+    sweep = None
+    if world == 1 and args.sweep and cfg.idx == 3:
+        sweep = sweep_points(cfg, device, sr, torch, hbm_peak)
+
     # ---- other configs (same run): layers/s and bytes, recomposed vs unfused, with spread
     others = {}
     if args.all_configs and world == 1:
@@ -620,6 +626,7 @@ def gpu_arm(args, rank, world, local_rank):
         "training": train,
         "weak": weak,
         "strong_scaling_shards": strong_model,
+        "sweep": sweep,
         "paper_context": PAPER_CONTEXT,
         "clocks": clocks,
     }
@@ -710,6 +717,28 @@ def shard_model(args, cfg, device, sr, torch, K, Wm, ms_full):
         out["k"][str(k)] = {"layer_ms": round(worst, 5), "layers_per_s": round(1e3 / worst, 2),
                             "efficiency_vs_1gpu": round(ms_full / (k * worst), 4),
                             "distinct_shards": len(seen)}
+    return out
+
+
+def sweep_points(cfg, device, sr, torch, hbm_peak):
+    """GPT-Neo attention at L = 512 .. 4096 (batch 4) and batch 1 .. 8 (L = 2048): layers/s of the
+    default path and of the unfused baseline, back to back with inputs larger than L2 (SURVEY NEXT-3;
+    parity of these shapes: tests/test_gpu_sweep.py)."""
+    import dataclasses
+    out = []
+    for axis, S, B in [("L", 512, 4), ("L", 1024, 4), ("L", 2048, 4), ("L", 4096, 4),
+                       ("batch", 2048, 1), ("batch", 2048, 2), ("batch", 2048, 8)]:
+        c = dataclasses.replace(cfg, S=S, B=B, name=f"gptneo_L{S}_B{B}")
+        Ls = Layer(c, device, seed_base=c.idx, sr=sr, torch=torch, variants=False)
+        sets, _ = rotation_sets(c, device, 0, sr, torch, Ls, 0, None, variants=False)
+        tr = statistics.median(back_to_back(torch, [x.run for x in sets], 10, 3, reps=3))
+        tu = statistics.median(back_to_back(torch, [(lambda x=x: x.run(fused=False)) for x in sets], 10, 3, reps=3))
+        rb = sum(alg_bytes_default(c, Ls.stored, Ls.T).values())
+        out.append({"axis": axis, "L": S, "B": B, "layers_per_s": round(1e3 / tr, 1), "ms": round(tr, 5),
+                    "unfused_ms": round(tu, 5), "speedup_vs_unfused": round(tu / tr, 3),
+                    "roofline_frac": round(rb / (tr * 1e-3) / 1e9 / hbm_peak, 4)})
+        del Ls, sets
+        torch.cuda.empty_cache()
     return out
 
 
@@ -828,6 +857,7 @@ def main():
     ap.add_argument("--tile-n", type=int, default=0, help="LS sub-vector width T (0 = library default)")
     ap.add_argument("--no-all-configs", dest="all_configs", action="store_false")
     ap.add_argument("--no-shard-model", dest="shard_model", action="store_false")
+    ap.add_argument("--no-sweep", dest="sweep", action="store_false")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)

@@ -22,6 +22,8 @@
 #include <unordered_map>
 #include <vector>
 
+#include <nvtx3/nvToolsExt.h>  // header-only NVTX v3: ranges show up in nsys / ncu --nvtx when a tool is attached
+
 #include "../../include/sr_mha.h"
 #include "sr_internal.h"
 
@@ -953,41 +955,54 @@ sr_status run_bwd(sr_entry e, const void* q, const void* k, const void* v, const
 
 // ================================================================================== C ABI
 
+// One NVTX range per layer call: the host-side span of the call, named after the entry
+// point; free when no profiler is attached.
+struct NvtxRange {
+    explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+};
+
 extern "C" {
 
 sr_status sr_mha_dense(const void* q, const void* k, const void* v, void* out, int B, int H, int S,
                        int D, float scale, const sr_dense_mask* m, int causal, const sr_exec* ex)
 {
+    NvtxRange nvtx("sr_mha_dense");
     return run(SR_E_DENSE, 1, q, k, v, out, B, H, S, D, scale, m, causal, ex);
 }
 sr_status sr_mha_blocksparse(const void* q, const void* k, const void* v, void* out, int B, int H,
                              int S, int D, float scale, const sr_block_layout* l, int causal,
                              const sr_exec* ex)
 {
+    NvtxRange nvtx("sr_mha_blocksparse");
     return run(SR_E_BLOCKSPARSE, 1, q, k, v, out, B, H, S, D, scale, l, causal, ex);
 }
 sr_status sr_mha_sliding_window(const void* q, const void* k, const void* v, void* out, int B,
                                 int H, int S, int D, float scale, const sr_window* w, int causal,
                                 const sr_exec* ex)
 {
+    NvtxRange nvtx("sr_mha_sliding_window");
     return run(SR_E_WINDOW, 1, q, k, v, out, B, H, S, D, scale, w, causal, ex);
 }
 sr_status sr_mha_dense_unfused(const void* q, const void* k, const void* v, void* out, int B,
                                int H, int S, int D, float scale, const sr_dense_mask* m, int causal,
                                const sr_exec* ex)
 {
+    NvtxRange nvtx("sr_mha_dense_unfused");
     return run(SR_E_DENSE, 0, q, k, v, out, B, H, S, D, scale, m, causal, ex);
 }
 sr_status sr_mha_blocksparse_unfused(const void* q, const void* k, const void* v, void* out, int B,
                                      int H, int S, int D, float scale, const sr_block_layout* l,
                                      int causal, const sr_exec* ex)
 {
+    NvtxRange nvtx("sr_mha_blocksparse_unfused");
     return run(SR_E_BLOCKSPARSE, 0, q, k, v, out, B, H, S, D, scale, l, causal, ex);
 }
 sr_status sr_mha_sliding_window_unfused(const void* q, const void* k, const void* v, void* out,
                                         int B, int H, int S, int D, float scale, const sr_window* w,
                                         int causal, const sr_exec* ex)
 {
+    NvtxRange nvtx("sr_mha_sliding_window_unfused");
     return run(SR_E_WINDOW, 0, q, k, v, out, B, H, S, D, scale, w, causal, ex);
 }
 
@@ -995,18 +1010,21 @@ sr_status sr_mha_dense_bwd(const void* q, const void* k, const void* v, const vo
                            void* dq, void* dk, void* dv, int B, int H, int S, int D, float scale,
                            const sr_dense_mask* m, int causal, const sr_exec* ex)
 {
+    NvtxRange nvtx("sr_mha_dense_bwd");
     return run_bwd(SR_E_DENSE, q, k, v, out, dout, dq, dk, dv, B, H, S, D, scale, m, causal, ex);
 }
 sr_status sr_mha_blocksparse_bwd(const void* q, const void* k, const void* v, const void* out, const void* dout,
                                  void* dq, void* dk, void* dv, int B, int H, int S, int D, float scale,
                                  const sr_block_layout* l, int causal, const sr_exec* ex)
 {
+    NvtxRange nvtx("sr_mha_blocksparse_bwd");
     return run_bwd(SR_E_BLOCKSPARSE, q, k, v, out, dout, dq, dk, dv, B, H, S, D, scale, l, causal, ex);
 }
 sr_status sr_mha_sliding_window_bwd(const void* q, const void* k, const void* v, const void* out, const void* dout,
                                     void* dq, void* dk, void* dv, int B, int H, int S, int D, float scale,
                                     const sr_window* w, int causal, const sr_exec* ex)
 {
+    NvtxRange nvtx("sr_mha_sliding_window_bwd");
     return run_bwd(SR_E_WINDOW, q, k, v, out, dout, dq, dk, dv, B, H, S, D, scale, w, causal, ex);
 }
 

@@ -24,14 +24,14 @@ using namespace ptx;
 #ifdef SR_DIAG_PHASES
 // diagnostic build: per CTA, %globaltimer (ns) at kernel start, after the prologue, after phase 1,
 // after phase 2, plus the CTA's item count (read with sr_diag_read_phases)
-__device__ unsigned long long g_diag_phases[1024 * 5];
+__device__ unsigned long long g_diag_phases[1024 * 8];
 __device__ __forceinline__ unsigned long long gtimer()
 {
     unsigned long long t;
     asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
     return t;
 }
-#define PH_MARK(i) do { if (threadIdx.x == 0) g_diag_phases[blockIdx.x * 5 + (i)] = gtimer(); } while (0)
+#define PH_MARK(i) do { if (threadIdx.x == 0) g_diag_phases[blockIdx.x * 8 + (i)] = gtimer(); } while (0)
 #else
 #define PH_MARK(i)
 #endif
@@ -102,7 +102,18 @@ __global__ void __launch_bounds__(640, 1)
     __syncthreads();
     PH_MARK(3);
 #ifdef SR_DIAG_PHASES
-    if (threadIdx.x == 0) g_diag_phases[blockIdx.x * 5 + 4] = it_end - it_begin;
+    if (threadIdx.x == 0) {
+        g_diag_phases[blockIdx.x * 8 + 4] = it_end - it_begin;
+        unsigned long long nt = 0;  // the CTA's listed tiles and its SM
+        for (int it = it_begin; it < it_end; ++it) {
+            const int4 d = __ldg(sc.item_desc + it);
+            nt += d.z - d.y;
+        }
+        unsigned smid;
+        asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+        g_diag_phases[blockIdx.x * 8 + 5] = nt;
+        g_diag_phases[blockIdx.x * 8 + 6] = smid;
+    }
 #endif
     if (warp == 2) {
         tc_fence_after();
@@ -150,7 +161,7 @@ extern "C" int sr_diag_read_fused(int phase, unsigned long long* out)  // [20][k
 #endif
 
 #ifdef SR_DIAG_PHASES
-extern "C" int sr_diag_read_phases(unsigned long long* out)  // [1024][5] (diagnostic build)
+extern "C" int sr_diag_read_phases(unsigned long long* out)  // [1024][8] (diagnostic build)
 {
     return cudaMemcpyFromSymbol(out, sr::g_diag_phases, sizeof(sr::g_diag_phases)) != cudaSuccess;
 }

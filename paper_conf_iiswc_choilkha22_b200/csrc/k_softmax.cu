@@ -2,6 +2,7 @@
 // block held in on-chip memory; the attention matrix is read once and written once).  Part of the
 // in-repo traffic baseline only; the recomposed path never runs it.
 //
+// row_softmax (rows longer than the register-resident kernel below takes, or SR_SOFTMAX_SMEM=1):
 // One CTA per (row-block, slice of R rows): every score tile of the row-block holds the slice's R
 // rows of each 64-key chunk as R x 128 contiguous bytes (SWIZZLE_128B tile layout), so the CTA pulls
 // the slice's whole score rows into shared memory with one bulk copy per chunk (all in flight at
@@ -188,6 +189,128 @@ __global__ void __launch_bounds__(256) row_softmax(const Params p, int R, int ca
     if (threadIdx.x == 0) bulk_wait_read0();
 }
 
+// ---------------------------------------------------------------- register-resident row softmax
+// The default baseline softmax for rows of up to 4 * kNiMax 64-key chunks (4096 keys): one CTA per
+// (row-block, 64-row half) -- the rows of a half share one list of stored tiles -- and one warp per
+// row at a time.  A warp-wide 16-B load covers 4 chunks x 128 B of its row (lane l: chunk l/8,
+// 16-B piece l%8 of the SWIZZLE_128B row), so a row of up to 4*NI chunks sits in 4*NI registers per
+// lane: the scores are read once and P written once straight from registers, every
+// load of a row in flight at once.  Arithmetic in packed fp16 (max, exponent argument, ex2.f16x2,
+// normalisation; the row sum accumulates in fp32): ~3 instructions per element.  Scores are the
+// fp16 values GEMM1 stored; masked ones are -inf; a row with no kept key writes zeros.
+constexpr int kNiMax = 16;
+
+__device__ __forceinline__ __half2 u2h(uint32_t w) { return *reinterpret_cast<__half2*>(&w); }
+__device__ __forceinline__ uint32_t h2u(__half2 h) { return *reinterpret_cast<uint32_t*>(&h); }
+__device__ __forceinline__ __half2 ex2_h2(__half2 t)  // one MUFU op for two fp16 results
+{
+    uint32_t y;
+    asm("ex2.approx.f16x2 %0, %1;" : "=r"(y) : "r"(h2u(t)));
+    return u2h(y);
+}
+
+template <int T, int NI, bool BF>
+__global__ void __launch_bounds__(256) row_softmax_reg(const Params p, int lo, int hi)  // halves with lo < chunks <= hi
+{
+    __shared__ int64_t slot_list[1024];  // stored tiles of this half, as slot ids
+    __shared__ int n_tiles;
+    constexpr int XB = kRowBlock * T * 2, CPT = T / 64;
+    const DevSched& sc = p.sc;
+    const int item = blockIdx.x >> 1, half = blockIdx.x & 1;  // item = g * n_rb + rb
+    const int g = item / sc.n_rb, rb = item % sc.n_rb;
+    const int32_t* tp = sc.tp + (size_t)lh_of(sc, g, p.H) * (sc.n_rb + 1);
+    const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+    griddep_launch_dependents();
+    griddep_wait();
+    const int t0 = __ldg(tp + rb), t1 = __ldg(tp + rb + 1);
+    const int64_t slot0 = (int64_t)g * sc.slots_per_head - __ldg(tp);
+    if (warp == 0) {  // compact the tiles whose `half` is valid (ballot + prefix, 32 at a time)
+        int n = 0;
+        for (int tb = t0; tb < t1; tb += 32) {
+            const int t = tb + lane;
+            const bool v = t < t1 && ((tinfo_half(__ldg(sc.tinfo + t)) >> half) & 1);
+            const unsigned m = __ballot_sync(0xffffffffu, v);
+            if (v) slot_list[n + __popc(m & ((1u << lane) - 1))] = slot0 + t;
+            n += __popc(m);
+        }
+        if (lane == 0) n_tiles = n;
+    }
+    __syncthreads();
+    const int nch = n_tiles * CPT;  // 64-key chunks of each row of this half
+    if (nch <= lo || nch > hi) return;  // another launch's length class (or nothing stored)
+    const int sub = lane >> 3;  // chunk within a group of 4
+    const int ni = (nch + 3) / 4;  // 16-B words per lane actually used by this half's rows (warp-uniform)
+    const __half2 l2e = __float2half2_rn(1.4426950408889634f);
+    // NR rows of the warp in flight at once (short rows: more of them, so a warp keeps ~8 loads out)
+    constexpr int NR = NI >= 8 ? 1 : 8 / NI;
+    for (int rr0 = warp * NR; rr0 < kHalf; rr0 += 8 * NR) {
+        uint4 x[NR][NI];
+        int64_t base[NR];
+#pragma unroll
+        for (int q = 0; q < NR; ++q) {
+            const int r = half * kHalf + rr0 + q;
+            base[q] = (int64_t)r * 128 + (int64_t)((((lane & 7) ^ (r & 7))) << 4);
+#pragma unroll
+            for (int i = 0; i < NI; ++i) {  // every load of the NR rows in flight at once
+                const int k = 4 * i + sub;
+                x[q][i] = make_uint4(0xFC00FC00u, 0xFC00FC00u, 0xFC00FC00u, 0xFC00FC00u);  // -inf (fp16)
+                if (k < nch)
+                    x[q][i] = __ldg(reinterpret_cast<const uint4*>((const uint8_t*)p.xprime + slot_list[k / CPT] * (int64_t)XB +
+                                                                   (k % CPT) * (kRowBlock * 128) + base[q]));
+            }
+        }
+#pragma unroll
+        for (int q = 0; q < NR; ++q) {
+            __half2 m2 = u2h(0xFC00FC00u);
+#pragma unroll
+            for (int i = 0; i < NI; ++i)
+                if (i < ni)  // warp-uniform: only the words this half's rows use
+                    m2 = __hmax2(__hmax2(m2, __hmax2(u2h(x[q][i].x), u2h(x[q][i].y))),
+                                 __hmax2(u2h(x[q][i].z), u2h(x[q][i].w)));
+            float m = fmaxf(__low2float(m2), __high2float(m2));
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+            // exponent argument (x - m) * log2(e) in fp16: x and m are fp16 values, so x - m is exact
+            // up to one rounding; 2^t on MUFU (fully masked row: every t is -inf -> 0)
+            const __half2 nm = __float2half2_rn(m == -INFINITY ? 0.f : -m);
+            float s0 = 0.f, s1 = 0.f;
+#pragma unroll
+            for (int i = 0; i < NI; ++i) {
+                if (i >= ni) continue;
+                __half2 e[4] = {u2h(x[q][i].x), u2h(x[q][i].y), u2h(x[q][i].z), u2h(x[q][i].w)};
+#pragma unroll
+                for (int u = 0; u < 4; ++u) e[u] = ex2_h2(__hmul2(__hadd2(e[u], nm), l2e));
+                const float2 f = __half22float2(__hadd2(__hadd2(e[0], e[1]), __hadd2(e[2], e[3])));
+                s0 += f.x;
+                s1 += f.y;
+                x[q][i] = make_uint4(h2u(e[0]), h2u(e[1]), h2u(e[2]), h2u(e[3]));
+            }
+            float sum = s0 + s1;
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, o);
+            const float inv = sum > 0.f ? 1.f / sum : 0.f;
+            const __half2 inv2 = __float2half2_rn(inv);
+#pragma unroll
+            for (int i = 0; i < NI; ++i) {
+                const int k = 4 * i + sub;
+                if (i >= ni || k >= nch) continue;
+                uint32_t w[4] = {x[q][i].x, x[q][i].y, x[q][i].z, x[q][i].w};
+#pragma unroll
+                for (int u = 0; u < 4; ++u) {
+                    if constexpr (BF) {
+                        const float2 f = __half22float2(u2h(w[u]));
+                        w[u] = pack_bf16(f.x * inv, f.y * inv);
+                    } else {
+                        w[u] = h2u(__hmul2(u2h(w[u]), inv2));
+                    }
+                }
+                stg128((uint8_t*)p.pbuf + slot_list[k / CPT] * (int64_t)XB + (k % CPT) * (kRowBlock * 128) + base[q],
+                       w[0], w[1], w[2], w[3]);
+            }
+        }
+    }
+}
+
 // rows per CTA and slice capacity in chunks: the largest power of two R <= 32 whose slice fits 48 KB,
 // for the longest rows if that gives R >= 8, else for the mean row (2 rows in up to 160 KB at worst)
 static void softmax_shape(const DevSched& sc, int T, int* R_, int* cap_)
@@ -217,8 +340,42 @@ cudaError_t launch_softmax_t(const Params& p, cudaStream_t st, int64_t* nl)
     return launch_pdl(row_softmax<T>, dim3((unsigned)blocks), dim3(32 * std::min(R, 8)), sm, st, nl, p, R, cap);
 }
 
+template <int T, bool BF>
+cudaError_t launch_softmax_reg(const Params& p, cudaStream_t st, int64_t* nl, int ni, int lo, int hi)
+{
+    const dim3 grid((unsigned)((int64_t)p.B * p.H * p.sc.n_rb * 2));
+    switch (ni) {
+    case 2: return launch_pdl(row_softmax_reg<T, 2, BF>, grid, dim3(256), 0, st, nl, p, lo, hi);
+    case 4: return launch_pdl(row_softmax_reg<T, 4, BF>, grid, dim3(256), 0, st, nl, p, lo, hi);
+    case 8: return launch_pdl(row_softmax_reg<T, 8, BF>, grid, dim3(256), 0, st, nl, p, lo, hi);
+    default: return launch_pdl(row_softmax_reg<T, 16, BF>, grid, dim3(256), 0, st, nl, p, lo, hi);
+    }
+}
+
+template <int T, bool BF>
+cudaError_t launch_softmax_classes(const Params& p, cudaStream_t st, int64_t* nl, int max_ch)
+{
+    // rows of <= 16 chunks with a short-row instantiation (several rows in flight per warp); longer
+    // ones (global rows of BigBird / Longformer) with a second launch sized for them
+    int ni = 2;
+    while (4 * ni < max_ch) ni *= 2;
+    if (ni <= 8) return launch_softmax_reg<T, BF>(p, st, nl, ni, 0, INT32_MAX);
+    cudaError_t e = launch_softmax_reg<T, BF>(p, st, nl, 4, 0, 16);
+    if (e != cudaSuccess) return e;
+    return launch_softmax_reg<T, BF>(p, st, nl, ni, 16, INT32_MAX);
+}
+
 cudaError_t launch_softmax(const Params& p, cudaStream_t st, int64_t* nl)
 {
+    // rows of up to 4 * kNiMax chunks (4096 keys): the register-resident kernel; longer rows stream
+    // through shared memory (row_softmax).  SR_SOFTMAX_SMEM=1 forces the latter (experiments).
+    const int max_ch = p.sc.max_rb_tiles * (p.T / 64);
+    static const bool force_smem = getenv("SR_SOFTMAX_SMEM") != nullptr;
+    if (!force_smem && max_ch <= 4 * kNiMax && p.sc.max_rb_tiles <= 1024) {
+        const bool bf = p.in_dtype == DT_BF16;
+        if (p.T == 64) return bf ? launch_softmax_classes<64, true>(p, st, nl, max_ch) : launch_softmax_classes<64, false>(p, st, nl, max_ch);
+        return bf ? launch_softmax_classes<128, true>(p, st, nl, max_ch) : launch_softmax_classes<128, false>(p, st, nl, max_ch);
+    }
     return p.T == 64 ? launch_softmax_t<64>(p, st, nl) : launch_softmax_t<128>(p, st, nl);
 }
 

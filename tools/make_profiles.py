@@ -35,6 +35,8 @@ def kname(full):
         return "gemm2_plain"
     if "tc_fused" in full:
         return "sr_layer_one_kernel"
+    if "sched_upload" in full:
+        return "sched_upload"
     if "tc_bwd_kv" in full:
         return "bwd_dkdv"
     for k, v in (("ir_kernel", "ir"), ("row_softmax", "softmax"), ("sd_ls_kernel", "sd_ls"),
@@ -65,7 +67,7 @@ def main(rnd):
     os.makedirs(PROF, exist_ok=True)
     tp = os.path.join(PROF, "ncu_traffic.json")
     traffic = json.load(open(tp)) if os.path.exists(tp) else {}  # configs not re-profiled keep their entry
-    for c in (2, 3, 4, 5):
+    for c in (2, 3, 4, 5, 6):
         p = os.path.join(OUT, f"launches_c{c}.csv")
         if not os.path.exists(p):
             continue
@@ -82,12 +84,16 @@ def main(rnd):
             lines.append(f"{n:28s} {len(m['gpu__time_duration.sum']):8d} {t / 1e3 * unit:10.2f} {rd / 1e6:11.2f} {wr / 1e6:11.2f}")
             if not n.startswith("other"):
                 ours[n] = (t, rd + wr)
-        rec = [k for k in ("sr_layer_one_kernel",) if k in ours]  # default path: one launch
+        rec = [k for k in ("sr_layer_one_kernel",) if k in ours]  # default path: one launch (+ schedule upload)
+        up = ours.get("sched_upload")
         two = [k for k in ("gemm1_ls_ir", "gs_gemm2") if k in ours]  # SR_TWO_KERNELS
         unf = [k for k in ("gemm1_plain", "softmax", "gemm2_plain") if k in ours]
         tr = sum(ours[k][0] for k in rec)
         lines.append("")
-        lines.append("recomposed layer (default, one launch): " + ", ".join(f"{k} {ours[k][0] / 1e3:.2f} us" for k in rec))
+        lines.append("recomposed layer (default, one launch): " + ", ".join(f"{k} {ours[k][0] / 1e3:.2f} us" for k in rec)
+                     + (f" (+ schedule upload {up[0] / 1e3:.2f} us per launch, "
+                        f"{ours['sr_layer_one_kernel'][0] / (ours['sr_layer_one_kernel'][0] + up[0]):.1%} kernel share)"
+                        if up and rec else ""))
         if len(two) == 2:
             t2 = sum(ours[k][0] for k in two)
             lines.append("two-kernel variant shares: " + ", ".join(f"{k} {ours[k][0] / t2:.1%}" for k in two))
@@ -137,7 +143,7 @@ def main(rnd):
                 e["backward_dram_bytes"] = int(sum(v[1] for v in bw.values()))
         traffic[f"C{c}"] = e
         open(os.path.join(PROF, f"{rnd}_launches_c{c}.txt"), "w").write("\n".join(lines) + "\n")
-        for k in ("tc_fused", "tc_gemm1", "tc_gemm2", "ir_kernel", "tc_gemm2_fi", "tc_bwd_ds", "tc_bwd_dkdv"):
+        for k in ("tc_fused", "tc_gemm1", "tc_gemm2", "ir_kernel", "softmax", "tc_gemm2_fi", "tc_bwd_ds", "tc_bwd_dkdv"):
             rep = os.path.join(OUT, f"full_c{c}_{k}.ncu-rep")
             if os.path.exists(rep):
                 s = subprocess.run([sys.executable, os.path.join(ROOT, "tools", "ncu_summary.py"), rep, "25"],

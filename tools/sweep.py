@@ -26,7 +26,7 @@ import torch  # noqa: E402
 import oracle  # noqa: E402  (test infrastructure: parity spot checks only)
 import paper_conf_iiswc_choilkha22_b200 as sr  # noqa: E402
 import workloads as W  # noqa: E402
-from bench import FLUSH_BYTES, Layer, alg_bytes, alg_bytes_ir_in_gemm1, oracle_mask_for, timed  # noqa: E402
+from bench import FLUSH_BYTES, Layer, alg_bytes, alg_bytes_default, oracle_mask_for, timed  # noqa: E402
 
 
 def points(quick):
@@ -73,7 +73,7 @@ def parity(L, cfg, n=48, seed=0):
 
 def main():
     ap = argparse.ArgumentParser()
-    ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "r1_sweep.json"))
+    ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "r2_sweep.json"))
     ap.add_argument("--quick", action="store_true")
     ap.add_argument("--steps", type=int, default=10)
     args = ap.parse_args()
@@ -87,7 +87,7 @@ def main():
         tr = statistics.mean(timed(torch, lambda: L.run(), args.steps, 3, flush))
         L.run(fused=False)
         tu = statistics.mean(timed(torch, lambda: L.run(fused=False), args.steps, 3, flush))
-        rb = sum(alg_bytes_ir_in_gemm1(cfg, L.stored, L.T).values())
+        rb = sum(alg_bytes_default(cfg, L.stored, L.T).values())
         ub = sum(alg_bytes(cfg, L.stored_u, L.Tu)[1].values())
         err = parity(L, cfg)
         e = {"axis": axis, "model": model, "name": cfg.name, "B": cfg.B, "H": cfg.H, "L": cfg.S, "D": cfg.D,
