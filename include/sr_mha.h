@@ -153,6 +153,14 @@ typedef struct {
  * dtypes, variant and stage bits aside) wrote there, and that nothing has written it since (used by
  * bench.py to time single kernels with SR_RUN_* stage bits).  Wrong use reads a stale schedule. */
 #define SR_SCHED_RESIDENT 1024
+/* Variant bit: key-range split of long rows (the paper's three-kernel layout with chunked items):
+ * GEMM1 + LS over chunks of <= L key tiles of a row-block (L = max(4, tiles / 296), about two chunks
+ * per SM of a B200, so a layer with few long rows -- e.g. one GPU's share of a head-sharded layer --
+ * still spreads over every SM), the standalone IR kernel over whole rows (writes r'), GS + GEMM2 over
+ * the chunks -- each chunk of a split row-block writes an fp32 partial context, already scaled by the
+ * global r' of its tiles -- and a combine kernel summing the partials in chunk order into out.
+ * Workspace: SR_WS_RECOMPOSED (it reserves the partial region, off_partial). */
+#define SR_SPLIT_KV 2048
 
 /* Entry points (north star).  Returns SR_OK after enqueueing the kernels on ex->stream. */
 sr_status sr_mha_dense(const void* q, const void* k, const void* v, void* out, int B, int H, int S,
@@ -246,6 +254,7 @@ typedef struct {
     size_t off_bstat;         /* SR_WS_TRAIN: fp32 [3][B*H*S]: m, 1/d, delta per query row */
     size_t off_sched;         /* tile schedule region (every mode) */
     size_t sched_bytes;
+    size_t off_partial;       /* SR_WS_RECOMPOSED: fp32 [slot][128][D] partial contexts of SR_SPLIT_KV */
 } sr_ws_info;
 
 /* Workspace bytes needed by an entry point; `mask_or_layout` is the same pointer passed to it

@@ -63,6 +63,11 @@ struct HostSched {
     std::vector<int32_t> cpp, cent, citems, ccta_ptr;
     int slots_per_head = 0;
     int max_rb_tiles = 0;
+    // key-range split plan (SR_SPLIT_KV): every item as chunks of <= split_L tiles, 4 ints each
+    // {item, t0, t1, partial slot or -1}; comb 4 ints per split row-block {item, slot0, chunks, 0}
+    int split_L = 0;
+    std::vector<int32_t> chunks, comb;
+    int64_t n_partial = 0;
     int64_t n_tiles = 0;       // over all B*H heads
     int64_t stored_elems = 0;  // valid 64-row halves x 64 x T, over all heads
 };
@@ -229,6 +234,26 @@ sr_status build_sched(const Request& r, HostSched& hs)
     }
     for (int g = 0; g < BH; ++g)
         for (int c = 0; c < hs.n_cb; ++c) hs.citems.push_back(g * hs.n_cb + c);
+    // key-range split: rows whose tile list exceeds L = max(4, tiles / (2 x 148)) -- a chunk count of
+    // about two per SM of a B200 -- are cut into near-equal chunks (device-independent, so the
+    // workspace size is known on the host)
+    hs.split_L = (int)std::max<int64_t>(4, (hs.n_tiles + 2 * kSplitRefSms - 1) / (2 * kSplitRefSms));
+    for (int g = 0; g < BH; ++g) {
+        const int lh = hs.lh_mode == LH_ONE ? 0 : (hs.lh_mode == LH_BATCH ? g / r.H : g % r.H);
+        const int32_t* tp = &hs.tp[(size_t)lh * (hs.n_rb + 1)];
+        for (int rb = 0; rb < hs.n_rb; ++rb) {
+            const int w = g * hs.n_rb + rb, t0 = tp[rb], n = tp[rb + 1] - tp[rb];
+            const int nc = n > hs.split_L ? (n + hs.split_L - 1) / hs.split_L : 1;
+            for (int c = 0; c < nc; ++c) {
+                const int a = t0 + (int)((int64_t)n * c / nc), b = t0 + (int)((int64_t)n * (c + 1) / nc);
+                hs.chunks.insert(hs.chunks.end(), {w, a, b, nc > 1 ? (int32_t)(hs.n_partial + c) : -1});
+            }
+            if (nc > 1) {
+                hs.comb.insert(hs.comb.end(), {w, (int32_t)hs.n_partial, nc, 0});
+                hs.n_partial += nc;
+            }
+        }
+    }
     return SR_OK;
 }
 
@@ -318,13 +343,15 @@ enum BlobGroup { G_BASE = 0, G_ITEMS, G_PAIR, G_FP, G_COL, G_N };
 constexpr int kMaxCta = 1024;  // bound on persistent CTAs per launch (the workspace reserves it)
 
 struct BlobLayout {  // int32-word offsets inside the blob
-    size_t tp, tinfo, kv, desc, items, cta, iri, pdesc, pent, pcta, fp, fpcta, cdesc, cent, ccta;
+    size_t tp, tinfo, kv, desc, items, cta, iri, psl, comb, pdesc, pent, pcta, fp, fpcta, cdesc, cent, ccta;
     size_t g_off[G_N], g_len[G_N];
     size_t words;
 };
 
 struct DevBlob {
     int n_sm = 0;
+    bool split = false;
+    double imbalance = 1.0;  // LPT: most loaded CTA / mean load over n_sm SMs (row-block items)
     std::vector<int32_t> w;
     BlobLayout L{};
     DevSched rel{};  // scalar fields of the device schedule (pointers filled per call)
@@ -362,7 +389,7 @@ std::string sched_key(const Request& r)
 
 // Word layout of the blob for given per-CTA-range lengths (n_cta + 1 entries each).  The workspace
 // region is sized with kMaxCta so it fits every device.
-BlobLayout blob_layout(const HostSched& h, size_t n_cta_ptr, size_t n_pcta_ptr, size_t n_ccta_ptr)
+BlobLayout blob_layout(const HostSched& h, size_t n_desc, size_t n_cta_ptr, size_t n_pcta_ptr, size_t n_ccta_ptr)
 {
     BlobLayout L{};
     size_t o = 0;
@@ -374,10 +401,13 @@ BlobLayout blob_layout(const HostSched& h, size_t n_cta_ptr, size_t n_pcta_ptr, 
     L.kv = o; o += h.kv_len.size();
     grp(G_BASE, s);
     s = o;  // G_ITEMS: item descriptors (16-B aligned), items, cta_ptr
-    L.desc = o; o += 4 * h.items.size();
+    L.desc = o; o += 4 * n_desc;    // row-blocks, or their chunks with SR_SPLIT_KV
     L.items = o; o += h.items.size();
     L.cta = o; o += n_cta_ptr;
     L.iri = o; o += h.items.size();  // the standalone IR kernel's row-block order (longest first)
+    L.psl = o; o += n_desc;          // SR_SPLIT_KV: partial slot of each descriptor
+    pad();                           // int4 records below
+    L.comb = o; o += std::max<size_t>(h.comb.size(), 4);
     grp(G_ITEMS, s);
     s = o;  // G_PAIR: pair descriptors, union entries, pcta_ptr
     L.pdesc = o; o += 4 * h.pitems.size();
@@ -399,38 +429,75 @@ BlobLayout blob_layout(const HostSched& h, size_t n_cta_ptr, size_t n_pcta_ptr, 
 
 size_t sched_region_bytes(const HostSched& h)
 {
-    return blob_layout(h, kMaxCta + 1, kMaxCta + 1, kMaxCta + 1).words * sizeof(int32_t);
+    return blob_layout(h, std::max(h.items.size(), h.chunks.size() / 4), kMaxCta + 1, kMaxCta + 1, kMaxCta + 1).words *
+           sizeof(int32_t);
 }
 
 void lpt_assign(HostSched& h, int n_cta);
 
 // The device blob of a schedule for n_sm persistent CTAs (built once, then shared read-only).
-std::shared_ptr<DevBlob> make_blob(const HostSched& h0, int n_sm)
+int64_t lpt_item_cost();
+void lpt_assign(std::vector<int32_t>& items, const std::vector<int64_t>& cost, int n_cta, std::vector<int32_t>& cta_ptr);
+
+std::shared_ptr<DevBlob> make_blob(const HostSched& h0, int n_sm, bool split)
 {
     HostSched h = h0;  // the LPT pass reorders items: keep the cached host schedule device-neutral
     lpt_assign(h, std::min(n_sm, kMaxCta));
     auto db = std::make_shared<DevBlob>();
     db->n_sm = n_sm;
-    BlobLayout L = blob_layout(h, h.cta_ptr.size(), h.pcta_ptr.size(), h.ccta_ptr.size());
+    db->split = split;
+    auto lh_of_g = [&](int g) { return h.lh_mode == LH_ONE ? 0 : (h.lh_mode == LH_BATCH ? g / h.H : g % h.H); };
+    // item descriptors {item, t0, t1, tp[lh][0]} grouped per CTA, and each one's partial slot: the
+    // LPT assignment of row-blocks, or (SR_SPLIT_KV) of the chunks of the split plan
+    std::vector<int32_t> desc, psl, cta_ptr;
+    if (!split) {
+        for (int32_t it : h.items) {
+            const int g = it / h.n_rb, rb = it % h.n_rb;
+            const int32_t* tp = &h.tp[(size_t)lh_of_g(g) * (h.n_rb + 1)];
+            desc.insert(desc.end(), {it, tp[rb], tp[rb + 1], tp[0]});
+            psl.push_back(-1);
+        }
+        cta_ptr = h.cta_ptr;
+        double tot = 0.0, mx = 0.0;  // how far the longest items stick out of a balanced share
+        for (size_t c = 0; c + 1 < cta_ptr.size(); ++c) {
+            double ld = 0.0;
+            for (int i = cta_ptr[c]; i < cta_ptr[c + 1]; ++i)
+                ld += 2.0 * (desc[4 * i + 2] - desc[4 * i + 1]) + (double)lpt_item_cost();
+            tot += ld;
+            mx = std::max(mx, ld);
+        }
+        db->imbalance = tot > 0.0 ? mx / (tot / std::max(n_sm, 1)) : 1.0;
+    } else {
+        const size_t nch = h.chunks.size() / 4;
+        std::vector<int32_t> order(nch);
+        std::vector<int64_t> cost(nch);
+        for (size_t i = 0; i < nch; ++i) {
+            order[i] = (int32_t)i;
+            cost[i] = 2 * (int64_t)(h.chunks[4 * i + 2] - h.chunks[4 * i + 1]) + lpt_item_cost();
+        }
+        lpt_assign(order, cost, std::min(n_sm, kMaxCta), cta_ptr);
+        for (int32_t i : order) {
+            const int32_t* c = &h.chunks[4 * (size_t)i];
+            const int g = c[0] / h.n_rb;
+            desc.insert(desc.end(), {c[0], c[1], c[2], h.tp[(size_t)lh_of_g(g) * (h.n_rb + 1)]});
+            psl.push_back(c[3]);
+        }
+    }
+    BlobLayout L = blob_layout(h, desc.size() / 4, cta_ptr.size(), h.pcta_ptr.size(), h.ccta_ptr.size());
     db->L = L;
     std::vector<int32_t>& w = db->w;
     w.assign(L.words, 0);
     auto put = [&](size_t off, const std::vector<int32_t>& v) { std::copy(v.begin(), v.end(), w.begin() + off); };
-    auto lh_of_g = [&](int g) { return h.lh_mode == LH_ONE ? 0 : (h.lh_mode == LH_BATCH ? g / h.H : g % h.H); };
     put(L.tp, h.tp);
     put(L.tinfo, h.tinfo);
     put(L.kv, h.kv_len);
-    size_t o = L.desc;  // item descriptors {item, t0, t1, tp[lh][0]}
-    for (int32_t it : h.items) {
-        const int g = it / h.n_rb, rb = it % h.n_rb;
-        const int32_t* tp = &h.tp[(size_t)lh_of_g(g) * (h.n_rb + 1)];
-        const int32_t d[4] = {it, tp[rb], tp[rb + 1], tp[0]};
-        std::copy(d, d + 4, w.begin() + o);
-        o += 4;
-    }
+    put(L.desc, desc);
     put(L.items, h.items);
-    put(L.cta, h.cta_ptr);
+    put(L.cta, cta_ptr);
     put(L.iri, h0.items);  // before the LPT pass: longest first
+    put(L.psl, psl);
+    put(L.comb, h.comb);
+    size_t o;
     o = L.pdesc;  // pair item descriptors {g * n_pair + j, e0, e1, tp[lh][0]}
     for (int32_t it : h.pitems) {
         const int g = it / h.n_pair, j = it % h.n_pair, lh = lh_of_g(g);
@@ -475,7 +542,8 @@ std::shared_ptr<DevBlob> make_blob(const HostSched& h0, int n_sm)
     d.slots_per_head = h.slots_per_head;
     d.max_rb_tiles = h.max_rb_tiles;
     d.mean_rb_tiles = (int)((h.tinfo.size() + (size_t)h.n_lh * h.n_rb - 1) / ((size_t)h.n_lh * h.n_rb));
-    d.n_items = (int)h.items.size();
+    d.n_items = (int)(desc.size() / 4);
+    d.n_comb = split ? (int)(h.comb.size() / 4) : 0;
     {   // the IR kernel's team classes over iri (longest first): 8 warps for > 4 * kIrWarpTiles tiles,
         // then 4, 2, 1 (each warp merges <= kIrWarpTiles tiles in registers)
         auto lh_of_g2 = [&](int g) { return h0.lh_mode == LH_ONE ? 0 : (h0.lh_mode == LH_BATCH ? g / h0.H : g % h0.H); };
@@ -487,7 +555,7 @@ std::shared_ptr<DevBlob> make_blob(const HostSched& h0, int n_sm)
             d.n_ir_class[n > 4 * kIrWarpTiles ? 0 : n > 2 * kIrWarpTiles ? 1 : n > kIrWarpTiles ? 2 : 3]++;
         }
     }
-    d.n_cta = (int)h.cta_ptr.size() - 1;
+    d.n_cta = (int)cta_ptr.size() - 1;
     d.n_pair = h.n_pair;
     d.n_pcta = (int)h.pcta_ptr.size() - 1;
     d.n_cb = h.n_cb;
@@ -508,6 +576,8 @@ DevSched place(const DevBlob& db, void* region, bool has_kv)
     d.items = b + L.items;
     d.cta_ptr = b + L.cta;
     d.ir_items = b + L.iri;
+    d.psl = b + L.psl;
+    d.comb = (const int4*)(b + L.comb);
     d.pair_desc = (const int4*)(b + L.pdesc);
     d.pent = (const int4*)(b + L.pent);
     d.pcta_ptr = b + L.pcta;
@@ -659,12 +729,12 @@ size_t device_l2_bytes()
     return it->second;
 }
 
-std::shared_ptr<DevBlob> device_blob(CachedSched& cs, int n_sm)
+std::shared_ptr<DevBlob> device_blob(CachedSched& cs, int n_sm, bool split = false)
 {
     std::lock_guard<std::mutex> lk(cs.mu);
     for (auto& b : cs.blobs)
-        if (b->n_sm == n_sm) return b;
-    cs.blobs.push_back(make_blob(cs.hs, n_sm));
+        if (b->n_sm == n_sm && b->split == split) return b;
+    cs.blobs.push_back(make_blob(cs.hs, n_sm, split));
     return cs.blobs.back();
 }
 
@@ -694,7 +764,7 @@ cudaError_t upload(const DevBlob& db, void* region, unsigned groups, cudaStream_
 
 size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 
-void ws_layout(const HostSched& h, int B, int H, int in_dtype, int fused, sr_ws_info* info)
+void ws_layout(const HostSched& h, int B, int H, int D, int in_dtype, int fused, sr_ws_info* info)
 {
     memset(info, 0, sizeof(*info));
     info->tile_n = h.T;
@@ -722,6 +792,9 @@ void ws_layout(const HostSched& h, int B, int H, int in_dtype, int fused, sr_ws_
         info->off_rprime = o; o = align_up(o + stat_bytes, 1024);
         info->off_rowstat = o; o = align_up(o + (size_t)4 * B * H * h.n_rb * kRowBlock * sizeof(float), 1024);
     }
+    if ((fused == 1 || fused == 3) && h.n_partial > 0) {  // SR_SPLIT_KV: fp32 partial outputs of split rows
+        info->off_partial = o; o = align_up(o + (size_t)h.n_partial * kRowBlock * D * sizeof(float), 1024);
+    }
     if (fused == 3) {
         info->off_ds = o; o = align_up(o + (size_t)info->n_slots * tile_bytes, 1024);
         info->off_bstat = o; o = align_up(o + (size_t)3 * B * H * h.n_rb * kRowBlock * sizeof(float), 1024);
@@ -742,7 +815,7 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
     if (!ex) return fail(SR_ERR_INVALID, "exec descriptor is NULL");
     if (!q || !k || !v || !out) return fail(SR_ERR_INVALID, "q, k, v and out must be non-NULL");
     if (!std::isfinite(scale) || !(scale > 0.f)) return fail(SR_ERR_INVALID, "scale must be finite and > 0");
-    const int variant_bits = SR_FUSE_IR | SR_DECOMPOSE | SR_IR_KERNEL | SR_ONE_KERNEL | SR_TWO_KERNELS;
+    const int variant_bits = SR_FUSE_IR | SR_DECOMPOSE | SR_IR_KERNEL | SR_ONE_KERNEL | SR_TWO_KERNELS | SR_SPLIT_KV;
     if (ex->flags & ~(SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2 | SR_GS_PROLOGUE | SR_SCHED_RESIDENT | variant_bits))
         return fail(SR_ERR_INVALID, "unknown flags 0x%x", ex->flags);
     if ((ex->flags & variant_bits) && (!fused || ex->in_dtype == SR_F32))
@@ -776,13 +849,27 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
     s = host_sched(r, cs);  // host-only schedule: workspace checks precede any CUDA call
     if (s != SR_OK) return s;
     sr_ws_info wi;
-    ws_layout(cs->hs, B, H, ex->in_dtype, fused, &wi);
+    ws_layout(cs->hs, B, H, D, ex->in_dtype, fused, &wi);
     if (!ex->workspace || ex->workspace_bytes < wi.total_bytes)
         return fail(SR_ERR_WORKSPACE, "workspace %zu bytes < required %zu", ex->workspace_bytes, wi.total_bytes);
     if ((uintptr_t)ex->workspace & 255) return fail(SR_ERR_WORKSPACE, "workspace must be 256-byte aligned");
     int n_sm = 0;
     if ((s = device_sms(n_sm)) != SR_OK) return s;
-    std::shared_ptr<DevBlob> db = device_blob(*cs, n_sm);
+    // key-range split: asked for, or chosen for the default 16-bit path when a few long rows would
+    // dominate the one-launch schedule (most loaded CTA >= 3x a balanced share, rows of >= 32 tiles:
+    // e.g. one GPU's share of a head-sharded BigBird / Longformer layer, whose global rows hold every
+    // key tile; measured C4 / C5 at 8-way sharding 50.3 -> 38.5 / 52.4 -> 30.7 us, while causal C3
+    // shards and all full configs stay faster in one launch).  SR_SPLIT_AUTO=0 disables the choice.
+    bool split = (ex->flags & SR_SPLIT_KV) != 0;
+    if (!split && fused == 1 && one && !(ex->flags & (variant_bits | SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2)) &&
+        cs->hs.n_partial > 0 && cs->hs.max_rb_tiles >= 32) {
+        static const bool auto_split = [] { const char* e = getenv("SR_SPLIT_AUTO"); return !e || atoi(e) != 0; }();
+        if (auto_split && device_blob(*cs, n_sm, false)->imbalance >= 3.0) {
+            split = true;
+            one = false;
+        }
+    }
+    std::shared_ptr<DevBlob> db = device_blob(*cs, n_sm, split);
     void* region = (char*)ex->workspace + wi.off_sched;
 
     Params p{};
@@ -799,13 +886,14 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
     p.sc = place(*db, region, r.kv_len != nullptr);
     const int stage_bits = ex->flags & (SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2);
     p.stages = stage_bits ? stage_bits : (SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2);
-    p.ir_mode = (ex->flags & SR_FUSE_IR) ? IR_IN_GEMM2 : ((ex->flags & SR_IR_KERNEL) ? IR_KERNEL : IR_IN_GEMM1);
+    p.ir_mode = (ex->flags & SR_FUSE_IR) ? IR_IN_GEMM2 : (((ex->flags & SR_IR_KERNEL) || split) ? IR_KERNEL : IR_IN_GEMM1);
     {   // GEMM1 pair schedule: SR_G1_PAIR=0/1 overrides the default (experiments)
         static const int env_pair = [] { const char* e = getenv("SR_G1_PAIR"); return e ? atoi(e) : -1; }();
         // default: pairs when K tiles are as large as the X' tiles they produce (D = 128) and there
         // are enough pairs to keep every SM busy (measured: C3 78 -> 75 us; D = 64 configs lose)
         p.g1_pair = env_pair >= 0 ? env_pair : (D == 128 && p.sc.n_pcta > 0 &&
                                                  (int64_t)B * H * p.sc.n_pair >= 2 * (int64_t)p.sc.n_pcta);
+        if (split) p.g1_pair = 0;  // chunks of row-blocks, not pairs
     }
     {   // X' (or S) stores stream past L2 (evict_first) only when the layer's stored tiles exceed
         // half the device's L2; below that they keep normal priority and are read back from L2
@@ -824,6 +912,7 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
         p.rowstat = (float*)(ws + wi.off_rowstat);
     }
     if (fused != 1) p.pbuf = ws + wi.off_p;
+    p.partial = split ? (float*)(ws + wi.off_partial) : nullptr;
     cudaStream_t st = (cudaStream_t)ex->stream;
     int64_t nl = 0;
     cudaError_t ce;
@@ -895,7 +984,7 @@ sr_status run_bwd(sr_entry e, const void* q, const void* k, const void* v, const
     s = host_sched(r, cs);
     if (s != SR_OK) return s;
     sr_ws_info wi;
-    ws_layout(cs->hs, B, H, ex->in_dtype, 3, &wi);
+    ws_layout(cs->hs, B, H, D, ex->in_dtype, 3, &wi);
     if (!ex->workspace || ex->workspace_bytes < wi.total_bytes)
         return fail(SR_ERR_WORKSPACE, "workspace %zu bytes < required %zu (SR_WS_TRAIN)", ex->workspace_bytes,
                     wi.total_bytes);
@@ -1040,7 +1129,7 @@ sr_status sr_workspace_query(sr_entry e, int fused, int B, int H, int S, int D, 
     std::shared_ptr<CachedSched> cs;
     s = host_sched(r, cs);
     if (s != SR_OK) return s;
-    ws_layout(cs->hs, B, H, in_dtype, fused, info);
+    ws_layout(cs->hs, B, H, D, in_dtype, fused, info);
     return SR_OK;
 }
 

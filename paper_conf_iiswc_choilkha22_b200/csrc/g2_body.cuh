@@ -45,7 +45,7 @@ constexpr int kMW2 = 128;  // macro tile width (keys per MMA step)
 #define SR_G2_VPREFETCH 0
 #endif
 
-enum : int { SH_TILE = 1, SH_END = 2, SH_EMPTY = 4, SH_FIRST = 8, SH_LAST = 16 };
+enum : int { SH_TILE = 1, SH_END = 2, SH_EMPTY = 4, SH_FIRST = 8, SH_LAST = 16, SH_PARTIAL = 32 };
 // never written: zero rows for the invalid 64-row halves of a P tile read as an smem MMA operand
 static __device__ __align__(128) uint8_t g_zero_g2[kHalf * 128];
 struct G2Hdr {  // X'-stage / O-buffer header
@@ -539,13 +539,15 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
             for (int it = it_begin; it < it_end; ++it) {
                 const ItemInfo I = nxt;
                 if (it + 1 < it_end) nxt = decode_item(sc, it + 1);  // prefetch
-                const int64_t orow = (int64_t)I.g * p.S + I.rb * kRowBlock;
+                // a chunk of a split row-block (SR_SPLIT_KV) writes fp32 partial rows to its slot
+                const int ps = (!AS && p.partial) ? __ldg(sc.psl + it) : -1;
+                const int64_t orow = ps >= 0 ? (int64_t)ps * kRowBlock : (int64_t)I.g * p.S + I.rb * kRowBlock;
                 if (I.t0 == I.t1) {  // no kept key in these rows: the epilogue writes zeros
                     post(SH_EMPTY, orow, true);
                     next_o();
                     continue;
                 }
-                post(SH_TILE, orow, false);
+                post(SH_TILE | (ps >= 0 ? SH_PARTIAL : 0), orow, false);
                 const uint32_t d_tmem = tmem_o + o * D;
                 for (int t = I.t0; t < I.t1; t += NSUB) {
                     const int nk = min(NSUB, I.t1 - t) * (T / 16);  // K steps of 16 keys
@@ -705,13 +707,14 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                 }
             } else {
                 const uint32_t taddr = tmem_o + lane_off + o * D;
+                const bool part = (h.flags & SH_PARTIAL) != 0;  // fp32 partial rows of a split row-block
 #pragma unroll
                 for (int c = 0; c < D / 32; ++c) {
                     uint32_t v[32];
                     tmem_ld32(taddr + c * 32, v);
                     tmem_wait_ld();
-                    if (p.out_dtype == DT_F32) {
-                        float4* O = reinterpret_cast<float4*>((float*)p.out + orow * D + c * 32);
+                    if (part || p.out_dtype == DT_F32) {
+                        float4* O = reinterpret_cast<float4*>((part ? p.partial : (float*)p.out) + orow * D + c * 32);
 #pragma unroll
                         for (int u = 0; u < 8; ++u)
                             O[u] = make_float4(__uint_as_float(v[4 * u]), __uint_as_float(v[4 * u + 1]),

@@ -169,4 +169,46 @@ cudaError_t launch_ir(const Params& p, cudaStream_t st, int64_t* nlaunch)
     return launch_pdl(ir_kernel, dim3((unsigned)blocks), dim3(kW * 32), 0, st, nlaunch, p);
 }
 
+// ---------------------------------------------------------------- SR_SPLIT_KV combine
+// O of a split row-block = the sum of its chunks' partial outputs.  Every chunk already applied the
+// row's global Global-Scaling factor r'_k = e^{m'_k - m} / d of its own tiles, so the
+// partial contexts add with no rescaling; they are summed in chunk order (deterministic).  One thread
+// per 4 output columns of a row.
+template <int D>
+__global__ void __launch_bounds__(256) combine_kernel(const Params p)
+{
+    ptx::griddep_launch_dependents();
+    ptx::griddep_wait();  // GEMM2's partial rows must be complete
+    constexpr int PER = kRowBlock * D / 4;  // float4 per row-block
+    const int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int j = (int)(idx / PER);
+    if (j >= p.sc.n_comb) return;
+    const int e = (int)(idx % PER), r = e / (D / 4), c4 = e % (D / 4);
+    const int4 cb = __ldg(p.sc.comb + j);  // {row-block item, first slot, chunks, 0}
+    const int g = cb.x / p.sc.n_rb, rb = cb.x % p.sc.n_rb;
+    float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+    for (int c = 0; c < cb.z; ++c) {
+        const float4 v = __ldcg(reinterpret_cast<const float4*>(p.partial + ((int64_t)(cb.y + c) * kRowBlock + r) * D) + c4);
+        acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w;
+    }
+    const int64_t orow = (int64_t)g * p.S + rb * kRowBlock + r;
+    if (p.out_dtype == DT_F32) {
+        reinterpret_cast<float4*>((float*)p.out + orow * D)[c4] = acc;
+    } else {
+        const bool bf = p.out_dtype == DT_BF16;
+        const uint2 w = make_uint2(bf ? ptx::pack_bf16(acc.x, acc.y) : ptx::pack_f16(acc.x, acc.y),
+                                   bf ? ptx::pack_bf16(acc.z, acc.w) : ptx::pack_f16(acc.z, acc.w));
+        reinterpret_cast<uint2*>((uint16_t*)p.out + orow * D)[c4] = w;
+    }
+}
+
+cudaError_t launch_combine(const Params& p, cudaStream_t st, int64_t* nlaunch)
+{
+    if (p.sc.n_comb == 0) return cudaSuccess;
+    const int64_t n = (int64_t)p.sc.n_comb * kRowBlock * p.D / 4;
+    const dim3 grid((unsigned)((n + 255) / 256));
+    return p.D == 64 ? launch_pdl(combine_kernel<64>, grid, dim3(256), 0, st, nlaunch, p)
+                     : launch_pdl(combine_kernel<128>, grid, dim3(256), 0, st, nlaunch, p);
+}
+
 }  // namespace sr

@@ -21,6 +21,7 @@ namespace sr {
 constexpr int kRowBlock = 128;  // M of every tcgen05 tile
 constexpr int kHalf = 64;       // validity granularity of tile rows
 constexpr int kIrWarpTiles = 8;  // IR kernel: tiles one warp merges in registers
+constexpr int kSplitRefSms = 148; // SR_SPLIT_KV chunk size reference: about two chunks per SM of a B200
 
 // Where the IR sub-layer runs: its own kernel (SR_IR_KERNEL, the paper's layout), folded into
 // GEMM2 (SR_FUSE_IR), or merged by warps of GEMM1 as the row's tiles are produced (default).
@@ -68,6 +69,11 @@ struct DevSched {
     // warps (> 32, 17-32, 9-16, <= 8 tiles); n_ir_class[c] row-blocks in class c
     const int32_t* ir_items;
     int n_ir_class[4];
+    // key-range split (SR_SPLIT_KV): psl[i] = partial-output slot of item descriptor i (a chunk of a
+    // split row-block) or -1; comb[j] = {row-block item, first slot, chunks, 0} of split row-block j
+    const int32_t* psl;
+    const int4* comb;
+    int n_comb;
 };
 
 // Everything a kernel needs to know about one call.
@@ -103,6 +109,7 @@ struct Params {
     void* dv;
     void* dsbuf;       // dS' = scale * dE/dx tiles (in_dtype), same slots and layout as X'
     float* bstat;      // [3][B*H*S]: per query row m (natural log), 1/d, delta = sum_d dO * O
+    float* partial;    // SR_SPLIT_KV: fp32 [slot][128][D] partial outputs of split row-blocks' chunks
     int bwd_dq_fused;  // dQ accumulated inside the dS' kernel (default; SR_BWD_DQ_SEPARATE=1: own kernel)
 };
 
@@ -151,6 +158,7 @@ inline cudaError_t launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, siz
 // ---- launchers (return cudaError_t of the launch)
 cudaError_t launch_simt_f32(const Params& p, cudaStream_t st, int64_t* nlaunch);
 cudaError_t launch_ir(const Params& p, cudaStream_t st, int64_t* nlaunch);
+cudaError_t launch_combine(const Params& p, cudaStream_t st, int64_t* nlaunch);
 cudaError_t launch_tc_fused(const Params& p, cudaStream_t st, int64_t* nlaunch);
 cudaError_t launch_tc_unfused(const Params& p, cudaStream_t st, int64_t* nlaunch);
 cudaError_t launch_tc_sd(const Params& p, cudaStream_t st, int64_t* nlaunch);

@@ -65,6 +65,8 @@ cudaError_t launch_tc_fused(const Params& p, cudaStream_t st, int64_t* nl)
     // merged inside GEMM1 (the default, GEMM2 then only reads each row's (m, 1/d))
     if (p.ir_mode == IR_KERNEL && (p.stages & 2) && (e = launch_ir(p, st, nl)) != cudaSuccess) return e;
     if (p.stages & 4) e = launch_gemm2(p, p.ir_mode == IR_KERNEL ? 1 : (p.ir_mode == IR_IN_GEMM2 ? 2 : 3), st, nl);
+    // SR_SPLIT_KV: the split row-blocks' partial outputs summed into O
+    if (e == cudaSuccess && (p.stages & 4) && p.partial) e = launch_combine(p, st, nl);
     return e;
 }
 

@@ -86,6 +86,7 @@ VARIANTS = {
     "ir_kernel": dict(ir_kernel=True, tile_n=128),
     "sd": dict(sd=True),
     "gs_prologue": dict(gs_prologue=True),
+    "split_kv": dict(split_kv=True),
 }
 
 

@@ -35,12 +35,13 @@ def _ulp_half(dtype, ref):
 
 def run_case(kind, B, H, S, D, dtype, *, causal=False, kv_len=None, layout=None, window=0, n_global=0,
              tile_n=0, fused=True, seed=0, out_f32=True, fuse_ir=False, ir_kernel=False, one_kernel=False,
-             two_kernels=False, gs_prologue=False):
+             two_kernels=False, gs_prologue=False, split_kv=False):
     t, q, k, v = qkv(B, H, S, D, dtype, seed)
     scale = 1 / math.sqrt(D)
     od = torch.float32 if out_f32 else TORCH[dtype]
     kw = dict(scale=scale, causal=causal, tile_n=tile_n, fused=fused, out_dtype=od, fuse_ir=fuse_ir,
-              ir_kernel=ir_kernel, one_kernel=one_kernel, two_kernels=two_kernels, gs_prologue=gs_prologue)
+              ir_kernel=ir_kernel, one_kernel=one_kernel, two_kernels=two_kernels, gs_prologue=gs_prologue,
+              split_kv=split_kv)
     if kind == "dense":
         o = sr.mha_dense(q, k, v, kv_len=kv_len, **kw)
     elif kind == "block":
@@ -432,3 +433,72 @@ def test_long_sequence_sampled_rows(kind, kw):
     got = o.reshape(-1, D)[torch.from_numpy(rows).cuda()].double().cpu().numpy()
     assert_close(got, ref, dtype, what=f"{kind} S={S}")
     assert torch.isfinite(o).all()
+
+
+# ------------------------------------------------------------------------------------ SR_SPLIT_KV
+
+SPLIT_CASES = [
+    # few heads, long rows: the split plan cuts rows into chunks of >= 4 key tiles
+    ("dense", dict(B=1, H=2, S=2048, D=128, dtype="bf16", causal=True)),
+    ("dense", dict(B=4, H=1, S=1024, D=64, dtype="f16", kv_len=[1024, 1000, 700, 1], causal=True)),
+    ("dense", dict(B=1, H=3, S=1024, D=64, dtype="f16")),
+    ("window", dict(B=1, H=2, S=4096, D=64, dtype="f16", window=512, n_global=8)),
+    ("block", dict(B=1, H=2, S=2048, D=64, dtype="f16", layout="bigbird")),
+]
+
+
+@pytest.mark.parametrize("stored", [False, True], ids=["fp32-context", "stored"])
+@pytest.mark.parametrize("kind,kw", SPLIT_CASES, ids=lambda x: str(x)[:50] if isinstance(x, dict) else x)
+def test_split_kv(kind, kw, stored):
+    """SR_SPLIT_KV (include/sr_mha.h): chunked GEMM1 + LS, IR over whole rows, chunked GS + GEMM2
+    writing partial contexts, combine -- every element against the oracle."""
+    kw = dict(kw)
+    if kw.get("layout") == "bigbird":
+        kw["layout"] = W.bigbird_layout(kw["H"], kw["S"], 64)
+    B, H, S, D, dtype = (kw.pop(x) for x in ("B", "H", "S", "D", "dtype"))
+    o, ref = run_case(kind, B, H, S, D, dtype, split_kv=True, out_f32=not stored, **kw)
+    assert_close(o, ref, dtype, out_f32=not stored, what=f"split {kind}")
+
+
+def test_split_kv_c3_shard():
+    """One GPU's share of C3 head-sharded over 8 GPUs (8 causal heads), the case SR_SPLIT_KV is for."""
+    from paper_conf_iiswc_choilkha22_b200 import shard as SH
+    cfg = W.config(3)
+    sh = SH.make_shard(0, 8, cfg.B, cfg.H, cfg.S, T=64, causal=True)
+    t = W.make_qkv(cfg.B, cfg.H, cfg.S, cfg.D, cfg.dtype, seed_base=cfg.idx)
+    from tests.gpu_util import to_dev
+    q, k, v = (SH.shard_view(to_dev(x, cfg.dtype), sh).contiguous() for x in (t.q_s, t.k_s, t.v_s))
+    o = sr.mha_dense(q, k, v, scale=cfg.scale, causal=True, out_dtype=torch.float32, split_kv=True)
+    torch.cuda.synchronize()
+    q64, k64, v64 = (SH.shard_view(torch.from_numpy(x), sh).numpy() for x in (t.q64, t.k64, t.v64))
+    ref = oracle.attention(q64, k64, v64, cfg.scale, oracle.Mask(causal=True))
+    assert_close(o.double().cpu().numpy(), ref, cfg.dtype, what="C3 shard split")
+
+
+@pytest.mark.parametrize("idx", [4, 5])
+def test_auto_split_on_global_row_shards(idx):
+    """The default call chooses SR_SPLIT_KV by itself when a few long rows dominate the one-launch
+    schedule -- one GPU's share of an 8-way head-sharded BigBird / Longformer layer (global rows hold
+    every key tile): every element against the oracle, and bitwise equal to the explicit split."""
+    from paper_conf_iiswc_choilkha22_b200 import shard as SH
+    from tests.gpu_util import to_dev
+    cfg = W.config(idx)
+    lay = W.config_layout(cfg)
+    sh = SH.make_shard(0, 8, cfg.B, cfg.H, cfg.S, layout=lay, T=64)
+    t = W.make_qkv(cfg.B, cfg.H, cfg.S, cfg.D, cfg.dtype, seed_base=cfg.idx)
+    q, k, v = (SH.shard_view(to_dev(x, cfg.dtype), sh).contiguous() for x in (t.q_s, t.k_s, t.v_s))
+    if cfg.kind == "blocksparse":
+        mask, om = sr.block_mask(sh.layout), oracle.Mask(kind="block", layout=sh.layout)
+    else:
+        mask = sr.window_mask(cfg.window, cfg.n_global)
+        om = oracle.Mask(kind="window", window=cfg.window, n_global=cfg.n_global)
+    n0 = sr.launch_count()
+    o = sr.call(mask, q, k, v, scale=cfg.scale, out_dtype=torch.float32)
+    torch.cuda.synchronize()
+    assert sr.launch_count() - n0 >= 4, "expected the split path (upload, GEMM1, IR, GEMM2, combine)"
+    o2 = sr.call(mask, q, k, v, scale=cfg.scale, out_dtype=torch.float32, split_kv=True)
+    torch.cuda.synchronize()
+    assert torch.equal(o, o2)
+    q64, k64, v64 = (SH.shard_view(torch.from_numpy(x), sh).numpy() for x in (t.q64, t.k64, t.v64))
+    ref = oracle.attention(q64, k64, v64, cfg.scale, om)
+    assert_close(o.double().cpu().numpy(), ref, cfg.dtype, what=f"C{idx} shard auto split")
