@@ -935,6 +935,18 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
             p.sc.n_cta = p.sc.n_pcta;
         }
         p.gs_prologue = (ex->flags & SR_GS_PROLOGUE) != 0;
+        {   // read part of X' back from L2: phase 2 walks the CTA's items last-first (the X' phase 1
+            // wrote most recently is the likeliest still in L2) and the last 2 items' X' is stored
+            // without the evict_first hint (measured, one B200, burst / sustained under the power cap:
+            // C3 140.5 -> 136.7 / 164.0 -> 158.7 us, C4 120.1 -> 115.3 / 141.2 -> 138.9, C5 63.6 -> 60.0 /
+            // 70.8 -> 68.5).  SR_X_KEEP / SR_P2_REVERSE override (experiments).
+            static const int env_keep = [] { const char* e = getenv("SR_X_KEEP"); return e ? atoi(e) : 2; }();
+            static const int env_rev = [] { const char* e = getenv("SR_P2_REVERSE"); return e ? atoi(e) : 1; }();
+            static const int env_rev1 = [] { const char* e = getenv("SR_P1_REVERSE"); return e ? atoi(e) : 0; }();
+            p.x_keep = env_keep;
+            p.p2_reverse = env_rev1 ? 0 : env_rev;
+            p.p1_reverse = env_rev1;
+        }
 
         ce = launch_tc_one(p, st, &nl);
     } else if (fused) {

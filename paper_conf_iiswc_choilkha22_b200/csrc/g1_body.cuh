@@ -64,7 +64,7 @@ constexpr int kPolyPairs = SR_G1_POLY_PAIRS;
 struct G1Hdr {  // per-accumulator macro-tile header, written by the MMA warp
     int32_t slot_lo, slot_hi, i0, kvl, w0, w1, flags, pad;
 };
-enum : int { HDR_TILE = 1, HDR_END = 2 };
+enum : int { HDR_TILE = 1, HDR_END = 2, HDR_KEEP = 4 };
 
 template <int D, int T, bool PAIR>
 struct G1 {
@@ -165,8 +165,11 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
         if (kG1KHint) tma_load_2d_hint(d, m, c0, c1, b, pol_k);
         else tma_load_2d(d, m, c0, c1, b);
     };
-    auto xstore = [&](void* d, const void* src, uint32_t nb) {
-        if (p.x_evict_first) bulk_store_hint(d, src, nb, pol_x);
+    // the CTA's items in processing order: last-first with p.p1_reverse (LPT order is longest first,
+    // so the largest items are then processed -- and their X' written -- last, see k_fused.cu)
+    auto p1at = [&](int j) { return p.p1_reverse ? it_begin + it_end - 1 - j : j; };
+    auto xstore = [&](void* d, const void* src, uint32_t nb, bool keep) {
+        if (p.x_evict_first && !keep) bulk_store_hint(d, src, nb, pol_x);
         else bulk_store(d, src, nb);
     };
 
@@ -183,10 +186,10 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
             // Q of row-blocks 2j and 2j+1 per item, then one K stage per union macro tile
             int qi = 0, ks = 0;
             uint32_t qph = 0, kph = 0;
-            int4 nd = it_begin < it_end ? __ldg(sc.pair_desc + it_begin) : make_int4(0, 0, 0, 0);
+            int4 nd = it_begin < it_end ? __ldg(sc.pair_desc + p1at(it_begin)) : make_int4(0, 0, 0, 0);
             for (int it = it_begin; it < it_end; ++it) {
                 const int4 d = nd;
-                if (it + 1 < it_end) nd = __ldg(sc.pair_desc + it + 1);
+                if (it + 1 < it_end) nd = __ldg(sc.pair_desc + p1at(it + 1));
                 const int g = d.x / sc.n_pair, j = d.x % sc.n_pair, e0 = d.y, e1 = d.z;
                 if (e0 == e1) continue;
                 const int nrb = 2 * j + 1 < sc.n_rb ? 2 : 1;
@@ -238,10 +241,10 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
             const uint32_t idesc = idesc_f16(p.in_dtype == DT_BF16 ? 1 : 0, kRowBlock, kMW, 0, 0);
             int qi = 0, ks = 0, n = 0;
             uint32_t qph = 0, kph = 0;
-            int4 nd = it_begin < it_end ? __ldg(sc.pair_desc + it_begin) : make_int4(0, 0, 0, 0);
+            int4 nd = it_begin < it_end ? __ldg(sc.pair_desc + p1at(it_begin)) : make_int4(0, 0, 0, 0);
             for (int it = it_begin; it < it_end; ++it) {
                 const int4 d = nd;
-                if (it + 1 < it_end) nd = __ldg(sc.pair_desc + it + 1);
+                if (it + 1 < it_end) nd = __ldg(sc.pair_desc + p1at(it + 1));
                 const int g = d.x / sc.n_pair, j = d.x % sc.n_pair, e0 = d.y, e1 = d.z;
                 if (e0 == e1) continue;
                 const int nrb = 2 * j + 1 < sc.n_rb ? 2 : 1;
@@ -282,7 +285,8 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
                         const int dslot = (ws[0] != -1 && ws[1] != -1) ? (int)(sl[1] - sl[0]) : 0;
                         if (elect_one()) {
                             hdr[buf] = G1Hdr{(int32_t)(slot & 0xffffffff), (int32_t)(slot >> 32),
-                                             (2 * j + r) * kRowBlock, kvl, ws[0], ws[1], HDR_TILE, dslot};
+                                             (2 * j + r) * kRowBlock, kvl, ws[0], ws[1],
+                                             HDR_TILE | (it >= it_end - p.x_keep ? HDR_KEEP : 0), dslot};
                             mbar_arrive(&acc_full[buf]);  // header published (arrival 1 of 2)
                         }
                         __syncwarp();
@@ -324,7 +328,7 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
             // warp walks the schedule; one elected lane issues)
             int qi = 0, ks = 0;
             uint32_t qph = 0, kph = 0;
-            for (ItemWalk iw(sc, it_begin, it_end); iw.more();) {
+            for (ItemWalk iw(sc, it_begin, it_end, p.p1_reverse); iw.more();) {
                 const ItemInfo I = iw.next();
                 if (I.t0 == I.t1) continue;
                 const int row0 = I.g * p.S + I.rb * kRowBlock;
@@ -370,7 +374,8 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
             const uint32_t idesc = idesc_f16(p.in_dtype == DT_BF16 ? 1 : 0, kRowBlock, kMW, 0, 0);
             int qi = 0, ks = 0, n = 0;
             uint32_t qph = 0, kph = 0;
-            for (ItemWalk iw(sc, it_begin, it_end); iw.more();) {
+            for (ItemWalk iw(sc, it_begin, it_end, p.p1_reverse); iw.more();) {
+                const bool keep = iw.it >= it_end - p.x_keep;  // before next(): the index of this item
                 const ItemInfo I = iw.next();
                 if (I.t0 == I.t1) continue;
                 const int kvl = sc.kv_len ? __ldg(sc.kv_len + I.g / p.H) : p.S;
@@ -387,7 +392,7 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
                     const int64_t slot = I.slot0 + t;
                     if (elect_one()) {
                         hdr[ab] = G1Hdr{(int32_t)(slot & 0xffffffff), (int32_t)(slot >> 32), I.rb * kRowBlock, kvl, w0,
-                                        w1, HDR_TILE, 1};  // adjacent sub-tile slots
+                                        w1, HDR_TILE | (keep ? HDR_KEEP : 0), 1};  // adjacent sub-tile slots
                         mbar_arrive(&acc_full[ab]);  // header published (arrival 1 of 2)
                     }
                     __syncwarp();
@@ -477,10 +482,10 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
                 }
             };
             if (PAIR) {
-                int4 nd = it_begin < it_end ? __ldg(sc.pair_desc + it_begin) : make_int4(0, 0, 0, 0);
+                int4 nd = it_begin < it_end ? __ldg(sc.pair_desc + p1at(it_begin)) : make_int4(0, 0, 0, 0);
                 for (int it = it_begin; it < it_end; ++it) {
                     const int4 dd = nd;
-                    if (it + 1 < it_end) nd = __ldg(sc.pair_desc + it + 1);
+                    if (it + 1 < it_end) nd = __ldg(sc.pair_desc + p1at(it + 1));
                     const int g = dd.x / sc.n_pair, j = dd.x % sc.n_pair, e0 = dd.y, e1 = dd.z;
                     if (e0 == e1) continue;
                     const int nrb = 2 * j + 1 < sc.n_rb ? 2 : 1;
@@ -499,7 +504,7 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
                     if (nrb == 2) flush(g, 2 * j + 1, m1, d1);
                 }
             } else {
-                for (ItemWalk iw(sc, it_begin, it_end); iw.more();) {
+                for (ItemWalk iw(sc, it_begin, it_end, p.p1_reverse); iw.more();) {
                     const ItemInfo I = iw.next();
                     if (I.t0 == I.t1) continue;
                     float m[4], d[4];
@@ -629,7 +634,7 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
                 if (valid) {  // warp-uniform: a warp's 32 rows lie in one 64-row half
                     uint8_t* dst = (uint8_t*)p.xprime + slot * (int64_t)C::XS + (NSUB == 1 ? h * C::HB : 0) +
                                    q * 32 * 128;
-                    xstore(dst, stage + q * 32 * 128, 32 * 128);
+                    xstore(dst, stage + q * 32 * 128, 32 * 128, (H.flags & HDR_KEEP) != 0);
                 }
                 bulk_commit();
             }
@@ -784,7 +789,8 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
                     for (int ch = 0; ch < T / 64; ++ch)
 #ifndef SR_DIAG_NOSTORE
                         xstore(dst + ch * (kRowBlock * 128) + wrow0 * 128,
-                                   stage + (s * (T / 64) + ch) * (kRowBlock * 128) + wrow0 * 128, 32 * 128);
+                                   stage + (s * (T / 64) + ch) * (kRowBlock * 128) + wrow0 * 128, 32 * 128,
+                                   (H.flags & HDR_KEEP) != 0);
 #else
                         (void)dst;
 #endif

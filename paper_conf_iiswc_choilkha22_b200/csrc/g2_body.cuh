@@ -182,7 +182,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
             int s = 0;
             const uint64_t pol_x = SR_G2_HINTS ? policy_evict_first() : 0;
             uint32_t sph = 0;
-            for (ItemWalk iw(sc, it_begin, it_end); iw.more();) {
+            for (ItemWalk iw(sc, it_begin, it_end, p.p2_reverse); iw.more();) {
                 const ItemInfo I = iw.next();
                 if (AS && I.t0 == I.t1) {  // no kept key in these rows: an EMPTY stage, written as zeros
                     DW_WAIT(&x_empty[s], sph ^ 1, 0);
@@ -259,7 +259,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
             int si = 0;
             uint32_t sph = 0;
             const int64_t nrow = (int64_t)p.B * p.H * p.S;
-            for (ItemWalk iw(sc, it_begin, it_end); iw.more();) {
+            for (ItemWalk iw(sc, it_begin, it_end, p.p2_reverse); iw.more();) {
                 const ItemInfo I = iw.next();
                 if (I.t0 == I.t1) continue;
                 const int64_t row = (int64_t)I.g * p.S + I.rb * kRowBlock + lane;
@@ -291,7 +291,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
             // L147), published as (m, 1/d) in a ring of NSI items.  Lane l reduces rows l + 32j.
             int si = 0;
             uint32_t sph = 0;
-            for (ItemWalk iw(sc, it_begin, it_end); iw.more();) {
+            for (ItemWalk iw(sc, it_begin, it_end, p.p2_reverse); iw.more();) {
                 const ItemInfo I = iw.next();
                 if (I.t0 == I.t1) continue;
                 DW_WAIT(&st_empty[si], sph ^ 1, 0);
@@ -349,7 +349,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
             int s = 0;
             const uint64_t pol_v = SR_G2_HINTS ? policy_evict_last() : 0;
             uint32_t sph = 0;
-            for (ItemWalk iw(sc, it_begin, it_end); iw.more();) {
+            for (ItemWalk iw(sc, it_begin, it_end, p.p2_reverse); iw.more();) {
                 const ItemInfo I = iw.next();
                 int wn[2];  // schedule words of the next macro tile, prefetched one step ahead
                 for (int u = 0; u < NSUB; ++u) wn[u] = I.t0 + u < I.t1 ? __ldg(sc.tinfo + I.t0 + u) : 0;
@@ -394,7 +394,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
         const uint32_t idesc = idesc_f16(0, kRowBlock, D, 0, 1);
         int s = 0, xs = 0, j = 0;
         uint32_t sph = 0, xph = 0, jph = 0;
-        for (ItemWalk iw(sc, it_begin, it_end); iw.more();) {
+        for (ItemWalk iw(sc, it_begin, it_end, p.p2_reverse); iw.more();) {
             const ItemInfo I = iw.next();
             if (I.t0 == I.t1) {  // the producer posted an EMPTY stage: add our release to it
                 DW_WAIT(&x_full[xs], xph, 1);
@@ -535,12 +535,13 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                 if (++o == C::NO) { o = 0; oph ^= 1; }
             };
             ItemInfo nxt;
-            if (it_begin < it_end) nxt = decode_item(sc, it_begin);
+            auto at = [&](int j) { return p.p2_reverse ? it_begin + it_end - 1 - j : j; };
+            if (it_begin < it_end) nxt = decode_item(sc, at(it_begin));
             for (int it = it_begin; it < it_end; ++it) {
                 const ItemInfo I = nxt;
-                if (it + 1 < it_end) nxt = decode_item(sc, it + 1);  // prefetch
+                if (it + 1 < it_end) nxt = decode_item(sc, at(it + 1));  // prefetch
                 // a chunk of a split row-block (SR_SPLIT_KV) writes fp32 partial rows to its slot
-                const int ps = (!AS && p.partial) ? __ldg(sc.psl + it) : -1;
+                const int ps = (!AS && p.partial) ? __ldg(sc.psl + at(it)) : -1;
                 const int64_t orow = ps >= 0 ? (int64_t)ps * kRowBlock : (int64_t)I.g * p.S + I.rb * kRowBlock;
                 if (I.t0 == I.t1) {  // no kept key in these rows: the epilogue writes zeros
                     post(SH_EMPTY, orow, true);

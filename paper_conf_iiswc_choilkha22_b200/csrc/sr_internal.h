@@ -95,6 +95,9 @@ struct Params {
     int g1_pair;       // GEMM1 walks pairs of row-blocks sharing each K tile (pair schedule)
     int gs_prologue;   // one-launch kernel: Global Scaling in GEMM2's prologue even for fp16 (SR_GS_PROLOGUE)
     int x_evict_first; // GEMM1's X' / S tile stores carry an L2 evict_first policy (large layers only)
+    int x_keep;        // one-launch kernel: the last x_keep items of each CTA store X' at normal L2 priority ...
+    int p2_reverse;    // ... and phase 2 walks the CTA's items last-first, reading that X' back from L2
+    int p1_reverse;    // one-launch kernel: phase 1 walks the CTA's items last-first (phase 2 then forward)
     DevSched sc;
     void* xprime;      // X' tiles (recomposed) or score tiles S (unfused)
     void* pbuf;        // unfused: P tiles

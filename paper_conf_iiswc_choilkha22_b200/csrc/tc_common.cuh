@@ -78,18 +78,21 @@ __device__ __forceinline__ ItemInfo decode_item(const DevSched& sc, int it) { re
 // runs:  for (ItemWalk w(sc, b, e); w.more(); ) { const ItemInfo I = w.next(); ... }
 struct ItemWalk {
     const DevSched& sc;
-    int it, end;
+    int it, begin, end;
+    bool rev;  // walk [begin, end) last-first
     int4 nd;
-    __device__ __forceinline__ ItemWalk(const DevSched& sc_, int b, int e) : sc(sc_), it(b), end(e)
+    __device__ __forceinline__ int at(int j) const { return rev ? begin + end - 1 - j : j; }
+    __device__ __forceinline__ ItemWalk(const DevSched& sc_, int b, int e, bool rev_ = false)
+        : sc(sc_), it(b), begin(b), end(e), rev(rev_)
     {
-        nd = item_desc(sc, it < end ? it : -1);
+        nd = item_desc(sc, it < end ? at(it) : -1);
     }
     __device__ __forceinline__ bool more() const { return it < end; }
     __device__ __forceinline__ ItemInfo next()
     {
         const ItemInfo I = item_info(sc, nd);
         ++it;
-        nd = item_desc(sc, it < end ? it : -1);
+        nd = item_desc(sc, it < end ? at(it) : -1);
         return I;
     }
 };
