@@ -894,6 +894,7 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
         p.g1_pair = env_pair >= 0 ? env_pair : (D == 128 && p.sc.n_pcta > 0 &&
                                                  (int64_t)B * H * p.sc.n_pair >= 2 * (int64_t)p.sc.n_pcta);
         if (split) p.g1_pair = 0;  // chunks of row-blocks, not pairs
+
     }
     {   // X' (or S) stores stream past L2 (evict_first) only when the layer's stored tiles exceed
         // half the device's L2; below that they keep normal priority and are read back from L2
