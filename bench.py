@@ -501,6 +501,9 @@ def gpu_arm(args, rank, world, local_rank):
         kern_two = {n: stage_us(bit, two_kernels=True) for n, bit in (("gemm1_ls_ir", 1), ("gs_gemm2", 4))}
         kern_irk = {n: stage_us(bit, ir_kernel=True) for n, bit in (("gemm1_ls", 1), ("ir", 2), ("gs_gemm2", 4))}
         irk_share = kern_irk["ir"] / sum(kern_irk.values())
+        # the IR kernel back to back (K launches in one graph, PDL-chained): its launch-to-launch time
+        # without the ~6 us single-launch event floor (diagnostic: its 8-23 MB of statistics stay L2-warm)
+        ir_b2b = statistics.median(back_to_back(torch, [lambda: L.run(ir_kernel=True, stages=2)], K, Wm)) * 1e3
         variants = {
             "how": "single-call CUDA-graph replays, L2 flushed before each; kernels: stage-selected launches",
             "two_kernels": {"what": f"GEMM1+LS+IR -> GS+GEMM2 as two launches (SR_TWO_KERNELS, T={L.T2})",
@@ -510,7 +513,11 @@ def gpu_arm(args, rank, world, local_rank):
             "ir_kernel": {"what": "the paper's three-kernel layout: GEMM1+LS -> standalone IR kernel (writes r') -> "
                                   f"GS+GEMM2 (SR_IR_KERNEL, PAPER.md L165-L173, T={L.T2})",
                           "ms_per_step": round(ms_irk, 5), "alg_bytes": int(sum(r2.values())),
-                          "kernels": kd(kern_irk, r2), "ir_share_of_layer": round(irk_share, 4)},
+                          "kernels": kd(kern_irk, r2), "ir_share_of_layer": round(irk_share, 4),
+                          "ir_back_to_back": {"us": round(ir_b2b, 3), "GB/s": round(r2["ir"] / (ir_b2b * 1e-6) / 1e9, 1),
+                                              "frac": round(r2["ir"] / (ir_b2b * 1e-6) / 1e9 / hbm_peak, 4),
+                                              "share_of_layer": round(ir_b2b * 1e-3 / ms_irk, 4),
+                                              "note": "L2-warm statistics; diagnostic, not a roofline claim"}},
             "sd": {"what": f"decomposition without fusion: GEMM1 -> LS -> IR -> GS -> GEMM2 (PAPER.md SD, NEXT-1, T={L.Tsd})",
                    "ms_per_step": round(ms_sd, 5)}}
         L.run()
