@@ -232,7 +232,7 @@ class Layer:
         self.bwd()
 
     def run(self, fused=True, stages=0, q=None, k=None, v=None, fuse_ir=False, sd=False, ir_kernel=False,
-            two_kernels=False, unfused_T=64, resident=False):
+            two_kernels=False, unfused_T=64, resident=False, concurrent=False):
         d = self.dev
         two = fuse_ir or ir_kernel or two_kernels
         if sd:
@@ -246,7 +246,7 @@ class Layer:
         return self.sr.call(self.mask, q if q is not None else d["q"], k if k is not None else d["k"],
                             v if v is not None else d["v"], out=self.out, fused=fused, stages=stages,
                             workspace=ws, tile_n=tn, fuse_ir=fuse_ir, sd=sd, ir_kernel=ir_kernel,
-                            two_kernels=two_kernels,
+                            two_kernels=two_kernels, concurrent=concurrent,
                             # single-kernel timing: the schedule is already in the workspace
                             sched_resident=resident or stages != 0, **self.kw)
 

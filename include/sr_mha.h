@@ -161,6 +161,12 @@ typedef struct {
  * global r' of its tiles -- and a combine kernel summing the partials in chunk order into out.
  * Workspace: SR_WS_RECOMPOSED (it reserves the partial region, off_partial). */
 #define SR_SPLIT_KV 2048
+/* Variant bit: GEMM1 + LS + IR and GS + GEMM2 run CONCURRENTLY in one persistent CTA per SM
+ * (k_conc.cu): disjoint warps, shared memory and TMEM; GEMM2 takes each item (head,
+ * 128-row block) over as soon as GEMM1 has stored its X' tiles, m' and row statistics, so the two
+ * GEMMs overlap and X' is read back while it is still in L2 (it is still written to the workspace,
+ * PAPER.md L171-L173).  16-bit inputs, D = 128, T = 64; same workspace as the default. */
+#define SR_CONCURRENT 4096
 
 /* Entry points (north star).  Returns SR_OK after enqueueing the kernels on ex->stream. */
 sr_status sr_mha_dense(const void* q, const void* k, const void* v, void* out, int B, int H, int S,

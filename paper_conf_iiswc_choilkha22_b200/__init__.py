@@ -253,11 +253,13 @@ SR_TWO_KERNELS = 256
 SR_GS_PROLOGUE = 512
 SR_SCHED_RESIDENT = 1024
 SR_SPLIT_KV = 2048
+SR_CONCURRENT = 4096
 
 
 def call(mask: _Mask, q, k, v, *, scale=None, causal=False, out_dtype=None, tile_n=0, fused=True,
          out=None, workspace=None, stream=None, stages=0, fuse_ir=False, sd=False, ir_kernel=False,
-         one_kernel=False, two_kernels=False, gs_prologue=False, sched_resident=False, split_kv=False):
+         one_kernel=False, two_kernels=False, gs_prologue=False, sched_resident=False, split_kv=False,
+         concurrent=False):
     """Run one attention layer through the C ABI.  q, k, v: CUDA tensors [B, H, S, D].
     Default (16-bit): GEMM1 + LS with the IR merged inside it, then GS + GEMM2, both in one launch.
     ir_kernel=True selects SR_IR_KERNEL (the paper's layout: a standalone IR kernel writing r');
@@ -268,7 +270,8 @@ def call(mask: _Mask, q, k, v, *, scale=None, causal=False, out_dtype=None, tile
     gs_prologue=True SR_GS_PROLOGUE (one launch, fp16: Global Scaling in GEMM2's prologue instead of
     accumulator-side); sched_resident=True SR_SCHED_RESIDENT (skip the schedule upload: the workspace
     still holds it from an identical earlier call -- bench.py's per-kernel timing); split_kv=True
-    SR_SPLIT_KV (long rows cut into key-range chunks: the paper's three-kernel layout + a combine)."""
+    SR_SPLIT_KV (long rows cut into key-range chunks: the paper's three-kernel layout + a combine);
+    concurrent=True SR_CONCURRENT (GEMM1 and GEMM2 concurrently in one CTA per SM, D = 128)."""
     torch = _torch()
     if not (q.is_cuda and k.is_cuda and v.is_cuda):
         raise ValueError("q, k, v must be CUDA tensors")
@@ -307,7 +310,8 @@ def call(mask: _Mask, q, k, v, *, scale=None, causal=False, out_dtype=None, tile
               int(stages) | (SR_FUSE_IR if fuse_ir else 0) | (SR_DECOMPOSE if sd else 0) |
               (SR_IR_KERNEL if ir_kernel else 0) | (SR_ONE_KERNEL if one_kernel else 0) |
               (SR_TWO_KERNELS if two_kernels else 0) | (SR_GS_PROLOGUE if gs_prologue else 0) |
-              (SR_SCHED_RESIDENT if sched_resident else 0) | (SR_SPLIT_KV if split_kv else 0))
+              (SR_SCHED_RESIDENT if sched_resident else 0) | (SR_SPLIT_KV if split_kv else 0) |
+              (SR_CONCURRENT if concurrent else 0))
     fn = getattr(lib(), _FN[(mask.entry, bool(fused))])
     with torch.cuda.device(q.device):  # the library launches on the current device
         _check(fn(q.data_ptr(), k.data_ptr(), v.data_ptr(), out.data_ptr(), B, H, S, D, C.c_float(scale),

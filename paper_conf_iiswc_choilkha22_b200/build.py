@@ -17,7 +17,7 @@ ROOT = os.path.dirname(HERE)
 LIB = os.path.join(HERE, "libsr_mha.so")
 BUILD = os.path.join(HERE, "_build")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
-SOURCES = ["abi.cu", "k_ir.cu", "k_simt_f32.cu", "k_g1.cu", "k_gemm2.cu", "k_softmax.cu", "k_sd.cu", "k_bwd.cu", "k_fused.cu", "tc_host.cu", "k_sched.cu"]
+SOURCES = ["abi.cu", "k_ir.cu", "k_simt_f32.cu", "k_g1.cu", "k_gemm2.cu", "k_softmax.cu", "k_sd.cu", "k_bwd.cu", "k_fused.cu", "k_conc.cu", "tc_host.cu", "k_sched.cu"]
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          "-Xcompiler", "-fPIC", "-Xcompiler", "-Wall", "--expt-relaxed-constexpr",
          "-I", os.path.join(ROOT, "include"), "-I", CSRC]

@@ -57,6 +57,7 @@ struct HostSched {
     // for 2j+1, 0}; pitems g * n_pair + j grouped per CTA (pcta_ptr).
     int n_pair = 0;
     std::vector<int32_t> pp, pent, pitems, pcta_ptr;
+    double pair_saving = 0.0;  // 1 - (pair union entries / listed tiles): the K-tile loads pairs save
     // column schedule (training backward, dK / dV): cpp [n_lh][n_cb+1] offsets into cent (4 ints
     // per entry, see DevSched::cent); citems g * n_cb + c grouped per CTA (ccta_ptr)
     int n_cb = 0;
@@ -210,6 +211,7 @@ sr_status build_sched(const Request& r, HostSched& hs)
     }
     for (int g = 0; g < BH; ++g)
         for (int j = 0; j < hs.n_pair; ++j) hs.pitems.push_back(g * hs.n_pair + j);
+    if (!hs.tinfo.empty()) hs.pair_saving = 1.0 - (double)(hs.pent.size() / 4) / (double)hs.tinfo.size();
     // column lists (the transpose of the row lists, for dK = dS'^T Q and dV = P^T dO): per 128-key
     // column block, the row-blocks that list one of its key tiles, ascending
     hs.n_cb = S / kRowBlock;
@@ -815,7 +817,8 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
     if (!ex) return fail(SR_ERR_INVALID, "exec descriptor is NULL");
     if (!q || !k || !v || !out) return fail(SR_ERR_INVALID, "q, k, v and out must be non-NULL");
     if (!std::isfinite(scale) || !(scale > 0.f)) return fail(SR_ERR_INVALID, "scale must be finite and > 0");
-    const int variant_bits = SR_FUSE_IR | SR_DECOMPOSE | SR_IR_KERNEL | SR_ONE_KERNEL | SR_TWO_KERNELS | SR_SPLIT_KV;
+    const int variant_bits =
+        SR_FUSE_IR | SR_DECOMPOSE | SR_IR_KERNEL | SR_ONE_KERNEL | SR_TWO_KERNELS | SR_SPLIT_KV | SR_CONCURRENT;
     if (ex->flags & ~(SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2 | SR_GS_PROLOGUE | SR_SCHED_RESIDENT | variant_bits))
         return fail(SR_ERR_INVALID, "unknown flags 0x%x", ex->flags);
     if ((ex->flags & variant_bits) && (!fused || ex->in_dtype == SR_F32))
@@ -828,6 +831,11 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
     // request without a variant bit runs the two-kernel chain at T = 128)
     bool one = (ex->flags & SR_ONE_KERNEL) != 0;
     if (one && ex->tile_n != 0 && ex->tile_n != 64) return fail(SR_ERR_UNSUPPORTED, "SR_ONE_KERNEL uses T = 64");
+    const bool conc_req = (ex->flags & SR_CONCURRENT) != 0;
+    if (conc_req && ((ex->tile_n != 0 && ex->tile_n != 64) ||
+                     (ex->flags & (SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2))))
+        return fail(SR_ERR_UNSUPPORTED, "SR_CONCURRENT runs T = 64, whole layers only");
+    if (conc_req) one = true;  // same workspace and schedule as the one-launch default
     if (fused == 1 && ex->in_dtype != SR_F32 && !(ex->flags & variant_bits) && (ex->tile_n == 0 || ex->tile_n == 64))
         one = true;
     if (fused && (ex->flags & SR_DECOMPOSE)) fused = 2;  // SD: workspace mode 2
@@ -869,6 +877,14 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
             one = false;
         }
     }
+    // concurrent GEMM1 / GEMM2 kernel (k_conc.cu): D = 128 one-launch layers (SR_CONC=1 selects it;
+    // experiment switch while it is being measured)
+    bool conc = conc_req;
+    {
+        static const int env_conc = [] { const char* e = getenv("SR_CONC"); return e ? atoi(e) : 0; }();
+        conc = conc || (env_conc == 1 && one && !split && fused == 1 &&
+                        !(ex->flags & (variant_bits | SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2)));
+    }
     std::shared_ptr<DevBlob> db = device_blob(*cs, n_sm, split);
     void* region = (char*)ex->workspace + wi.off_sched;
 
@@ -889,11 +905,16 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
     p.ir_mode = (ex->flags & SR_FUSE_IR) ? IR_IN_GEMM2 : (((ex->flags & SR_IR_KERNEL) || split) ? IR_KERNEL : IR_IN_GEMM1);
     {   // GEMM1 pair schedule: SR_G1_PAIR=0/1 overrides the default (experiments)
         static const int env_pair = [] { const char* e = getenv("SR_G1_PAIR"); return e ? atoi(e) : -1; }();
-        // default: pairs when K tiles are as large as the X' tiles they produce (D = 128) and there
-        // are enough pairs to keep every SM busy (measured: C3 78 -> 75 us; D = 64 configs lose)
+        // default: pairs when K tiles are as large as the X' tiles they produce (D = 128), there are
+        // enough pairs to keep every SM busy, and the two row-blocks of a pair share most of their K
+        // tiles (>= 45 % of the K loads saved: causal dense layers from S ~ 1536 on; measured one
+        // B200, back to back: causal S = 4096 572 -> 531 us, C3 136.0 -> 134.4; banded layouts lose --
+        // GPT-Neo local S = 2048 window 510 58.1 -> 66.2 us, window 254 47.0 -> 73.2 -- and stay unpaired;
+        // D = 64 configs lose)
         p.g1_pair = env_pair >= 0 ? env_pair : (D == 128 && p.sc.n_pcta > 0 &&
-                                                 (int64_t)B * H * p.sc.n_pair >= 2 * (int64_t)p.sc.n_pcta);
-        if (split) p.g1_pair = 0;  // chunks of row-blocks, not pairs
+                                                 (int64_t)B * H * p.sc.n_pair >= 2 * (int64_t)p.sc.n_pcta &&
+                                                 cs->hs.pair_saving >= 0.45);
+        if (split || conc) p.g1_pair = 0;  // chunks of row-blocks, not pairs / row-block items
 
     }
     {   // X' (or S) stores stream past L2 (evict_first) only when the layer's stored tiles exceed
@@ -903,6 +924,7 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
         static const int env_x = [] { const char* e = getenv("SR_X_EVICT_FIRST"); return e ? atoi(e) : -1; }();
         const double x_bytes = (double)cs->hs.stored_elems * (ex->in_dtype == SR_F32 ? 4.0 : 2.0);
         p.x_evict_first = env_x >= 0 ? env_x : (x_bytes > 0.5 * l2_or_default());
+        if (conc && env_x < 0) p.x_evict_first = 0;  // GEMM2 reads each item's X' back soon after it is written
     }
     char* ws = (char*)ex->workspace;
     p.xprime = ws + wi.off_xprime;
@@ -927,6 +949,8 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
     }
     if (fused == 2) {
         ce = launch_tc_sd(p, st, &nl);
+    } else if (conc) {
+        ce = launch_tc_conc(p, st, &nl);
     } else if (fused && one) {
         // pairs of row-blocks sharing each K tile in phase 1 (same choice as the two-kernel chain:
         // D = 128 with enough pairs); phase 2 then walks the pair assignment as row-block items

@@ -37,7 +37,7 @@ namespace sr {
 using namespace ptx;
 
 #ifdef SR_DIAG_WAITS
-static __device__ unsigned long long g_diag_g1[20 * (kDW + 1)];
+static __device__ unsigned long long g_diag_g1[32 * (kDW + 1)];
 #endif
 
 constexpr int kMW = 128;  // macro tile width (MMA N of GEMM1)
@@ -64,33 +64,39 @@ constexpr int kPolyPairs = SR_G1_POLY_PAIRS;
 struct G1Hdr {  // per-accumulator macro-tile header, written by the MMA warp
     int32_t slot_lo, slot_hi, i0, kvl, w0, w1, flags, pad;
 };
-enum : int { HDR_TILE = 1, HDR_END = 2, HDR_KEEP = 4 };
+// HDR_LASTT / HDR_MARK (concurrent kernel): the header ends item (flags >> 8) of the CTA's list --
+// its last tile, or a tile-less notice to the other epilogue warpgroup (both for an empty item)
+enum : int { HDR_TILE = 1, HDR_END = 2, HDR_KEEP = 4, HDR_LASTT = 8, HDR_MARK = 16 };
 
-template <int D, int T, bool PAIR>
+template <int D, int T, bool PAIR, int MW_ = kMW, int BUDGET = kSmemMax>
 struct G1 {
-    static constexpr int NSUB = kMW / T;          // sub-tiles per macro tile
+    // MW_ = 64 / BUDGET < kSmemMax: the concurrent kernel's GEMM1 half (k_conc.cu): 64-key macro
+    // tiles, two 64-column TMEM accumulators, FULL epilogue (one warpgroup per macro tile)
+    static constexpr int MW = MW_;                // macro tile width (MMA N)
+    static constexpr int NSUB = MW / T;           // sub-tiles per macro tile
     static constexpr int QB = kRowBlock * D * 2;  // Q tile bytes
     static constexpr int QS = (PAIR ? 2 : 1) * QB;  // Q stage: one row-block, or a pair
-    static constexpr int KB = kMW * D * 2;        // K stage bytes (MW keys)
-    static constexpr bool SPLIT = (T == 64);      // epilogue organisation, see the file header
+    static constexpr int KB = MW * D * 2;         // K stage bytes (MW keys)
+    static constexpr bool SPLIT = (T == 64 && MW == 128);  // epilogue organisation, see the file header
     static constexpr int EPI_WG = SPLIT ? 4 : 2;  // epilogue warpgroups
     static constexpr int HB = kRowBlock * 64 * 2;  // SPLIT staging tile: one warpgroup's 64 columns
-    static constexpr int XB2 = kRowBlock * kMW * 2;  // FULL staging tile: a whole macro tile
+    static constexpr int XB2 = kRowBlock * MW * 2;  // FULL staging tile: a whole macro tile
     static constexpr int SB = SPLIT ? HB : XB2;    // staging buffer per warpgroup
     static constexpr int XS = kRowBlock * T * 2;  // X' slot bytes (sub-tile)
-    static constexpr int NACC = 512 / kMW;        // TMEM accumulators
+    static constexpr int NACC = MW == 128 ? 4 : 2;  // TMEM accumulators (512 or 128 columns)
     // staging buffers per epilogue warpgroup (2 if at all possible: the X' store stream is the
     // bottleneck), then Q double-buffered if shared memory still allows
     // statistics ring for the IR-in-GEMM1 variant: per accumulator, NSUB x (m', d') x 128 rows fp32
     static constexpr int STB = NACC * 2 * 2 * kRowBlock * 4;
-    static constexpr int SLACK = 4096 + STB;
-    static constexpr int XPW = ((PAIR ? 2 * QS : QS) + 2 * KB + EPI_WG * 2 * SB + SLACK <= kSmemMax) ? 2 : 1;
+    static constexpr int SLACK = (BUDGET == kSmemMax ? 4096 : 1024) + STB;
+    static constexpr int XPW = ((PAIR ? 2 * QS : QS) + 2 * KB + EPI_WG * 2 * SB + SLACK <= BUDGET) ? 2 : 1;
 #ifndef SR_G1_MAX_NQ
 #define SR_G1_MAX_NQ 2
 #endif
-    static constexpr int NQ = (SR_G1_MAX_NQ >= 2 && 2 * QS + 2 * KB + EPI_WG * XPW * SB + SLACK <= kSmemMax) ? 2 : 1;
-    static constexpr int NK_ = (kSmemMax - SLACK - NQ * QS - EPI_WG * XPW * SB) / KB;
-    static constexpr int NK = NK_ > 4 ? 4 : NK_;
+    static constexpr int NQ = (SR_G1_MAX_NQ >= 2 && 2 * QS + 2 * KB + EPI_WG * XPW * SB + SLACK <= BUDGET) ? 2 : 1;
+    static constexpr int NK_ = (BUDGET - SLACK - NQ * QS - EPI_WG * XPW * SB) / KB;
+    static constexpr int NK_MAX = MW == 128 ? 4 : 6;
+    static constexpr int NK = NK_ > NK_MAX ? NK_MAX : NK_;
     static_assert(NK >= 2, "smem budget");
     static constexpr int OFF_Q = 0;
     static constexpr int OFF_K = OFF_Q + NQ * QS;
@@ -101,7 +107,7 @@ struct G1 {
     static constexpr int OFF_HDR = OFF_STATS + STB;
     static constexpr int OFF_TPTR = OFF_HDR + NACC * (int)sizeof(G1Hdr);
     static constexpr int SMEM_ = OFF_TPTR + 16 + 1024;  // + alignment slack
-    static constexpr int SMEM = SMEM_ > 118 * 1024 ? SMEM_ : 118 * 1024;  // 1 CTA/SM (512 TMEM cols)
+    static constexpr int SMEM = (BUDGET == kSmemMax && SMEM_ < 118 * 1024) ? 118 * 1024 : SMEM_;  // 1 CTA/SM
     static_assert(SMEM <= kSmemMax, "smem budget");
     static constexpr int THREADS = 128 + EPI_WG * 128;
 };
@@ -110,10 +116,10 @@ struct G1 {
 // tiles of its row-blocks), so warp 3 merges the epilogue's per-tile (m', d') of each row as they
 // are produced and, at the end of the row-block, writes the row's (m, 1/d) -- see the IR warp below.
 // Barrier initialisation of GEMM1's shared-memory layout (thread 0; fence_mbar_init included).
-template <int D, int T, bool LS, bool PAIR, bool IRT>
+template <int D, int T, bool LS, bool PAIR, bool IRT, int MW = kMW, int BUDGET = kSmemMax>
 __device__ __forceinline__ void g1_init(uint8_t* smem)
 {
-    using C = G1<D, T, PAIR>;
+    using C = G1<D, T, PAIR, MW, BUDGET>;
     constexpr bool SPLIT = C::SPLIT;
     uint64_t* bars = (uint64_t*)(smem + C::OFF_BAR);
     uint64_t* q_full = bars;
@@ -137,12 +143,21 @@ __device__ __forceinline__ void g1_init(uint8_t* smem)
 
 // Warp roles of GEMM1 (everything after the prologue): TMA producer, MMA issuer, IR warps,
 // epilogue warpgroups; uses every warp of the CTA (384 threads for T = 128, 640 for T = 64).
-template <int D, int T, bool LS, bool PAIR, bool IRT, bool REGS = true>
+// CONC (concurrent kernel, k_conc.cu): GEMM2 runs beside this GEMM1 in the same CTA and takes each
+// item over as soon as it is complete.  `ibar` = item_done[kConcNI] (10 arrivals per item: the eight
+// epilogue warps once their X' stores and m' of the item have landed, the two IR warps once its
+// row statistics are written) followed by item_free[kConcNI] (GEMM2 has taken the item; the MMA warp
+// waits on it before starting the item kConcNI places later).
+template <int D, int T, bool LS, bool PAIR, bool IRT, bool REGS = true, int MW = kMW, int BUDGET = kSmemMax,
+          bool CONC = false, int RM = 3>
 __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorMap& tmK, const Params& p,
                                           const DevSched& sc, uint8_t* smem, uint32_t tmem_base, int it_begin,
-                                          int it_end)
+                                          int it_end, uint64_t* ibar = nullptr)
 {
-    using C = G1<D, T, PAIR>;
+    using C = G1<D, T, PAIR, MW, BUDGET>;
+    static_assert(!CONC || (!PAIR && !C::SPLIT && IRT), "concurrent kernel: unpaired FULL epilogue, IR in GEMM1");
+    uint64_t* item_done = ibar;
+    uint64_t* item_free = CONC ? ibar + kConcNI : nullptr;
     constexpr int NSUB = C::NSUB;
     constexpr bool SPLIT = C::SPLIT;
     uint64_t* bars = (uint64_t*)(smem + C::OFF_BAR);
@@ -173,7 +188,9 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
         else bulk_store(d, src, nb);
     };
 
-    if (warp < 4) {
+    // RM: role groups compiled into this call (1: warps 0-3, 2: epilogue warpgroups), so a caller can
+    // run each group under its own setmaxnreg budget (k_conc.cu)
+    if ((RM & 1) && (!(RM & 2) || warp < 4)) {
         // warpgroup 0 hands registers to the epilogue warpgroups.  setmaxnreg.inc can only draw what
         // other warps of this CTA released, so the budgets balance exactly:
         //   SPLIT (640 threads, 96 at launch): 4 warps x 32 x (96 - 64) = 16 warps x 32 x (104 - 96)
@@ -227,7 +244,7 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
                         mbar_arrive_expect_tx(&k_full[ks], nsub * T * D * 2);
                         for (int s2 = 0; s2 < nsub; ++s2)
                             for (int h = 0; h < D / 64; ++h)
-                                kload(smem + C::OFF_K + ks * C::KB + h * (kMW * 128) + s2 * (T * 128), &tmK,
+                                kload(smem + C::OFF_K + ks * C::KB + h * (C::MW * 128) + s2 * (T * 128), &tmK,
                                             h * 64, g * p.S + (w[s2] & 0xFFFF) * T, &k_full[ks]);
                     }
                     __syncwarp();
@@ -238,7 +255,7 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
             // -------------------------------------------------------------- MMA issuer, pairs: per
             // union macro tile, the MMAs of each row-block that has a valid sub-tile in it, each into
             // the next TMEM accumulator of the common ring (the epilogue is the same as unpaired)
-            const uint32_t idesc = idesc_f16(p.in_dtype == DT_BF16 ? 1 : 0, kRowBlock, kMW, 0, 0);
+            const uint32_t idesc = idesc_f16(p.in_dtype == DT_BF16 ? 1 : 0, kRowBlock, C::MW, 0, 0);
             int qi = 0, ks = 0, n = 0;
             uint32_t qph = 0, kph = 0;
             int4 nd = it_begin < it_end ? __ldg(sc.pair_desc + p1at(it_begin)) : make_int4(0, 0, 0, 0);
@@ -290,14 +307,14 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
                             mbar_arrive(&acc_full[buf]);  // header published (arrival 1 of 2)
                         }
                         __syncwarp();
-                        const uint32_t d_tmem = tmem_base + buf * kMW;
+                        const uint32_t d_tmem = tmem_base + buf * C::MW;
                         const uint32_t qa = q_addr + r * C::QB;
                         if (elect_one()) {
 #pragma unroll
                             for (int kk = 0; kk < D / 16; ++kk) {
                                 const uint32_t h = kk / 4, wk = kk % 4;
                                 const uint64_t ad = smem_desc_sw128(qa + h * (kRowBlock * 128) + wk * 32, 16, 1024);
-                                const uint64_t bd = smem_desc_sw128(k_addr + h * (kMW * 128) + wk * 32, 16, 1024);
+                                const uint64_t bd = smem_desc_sw128(k_addr + h * (C::MW * 128) + wk * 32, 16, 1024);
                                 mma_ss(d_tmem, ad, bd, idesc, kk > 0 ? 1u : 0u);
                             }
                             mma_commit(&acc_full[buf]);  // arrival 2 of 2 when the MMAs complete
@@ -361,7 +378,7 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
 #endif
                         for (int s = 0; s < nsub; ++s)
                             for (int h = 0; h < D / 64; ++h)
-                                kload(smem + C::OFF_K + ks * C::KB + h * (kMW * 128) + s * (T * 128), &tmK,
+                                kload(smem + C::OFF_K + ks * C::KB + h * (C::MW * 128) + s * (T * 128), &tmK,
                                             h * 64, I.g * p.S + tinfo_kt(w[s]) * T, &k_full[ks]);
                     }
                     __syncwarp();
@@ -371,13 +388,33 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
         } else if (warp == 1) {
             // -------------------------------------------------------------- MMA issuer (whole warp
             // walks the schedule; one elected lane issues)
-            const uint32_t idesc = idesc_f16(p.in_dtype == DT_BF16 ? 1 : 0, kRowBlock, kMW, 0, 0);
+            const uint32_t idesc = idesc_f16(p.in_dtype == DT_BF16 ? 1 : 0, kRowBlock, C::MW, 0, 0);
             int qi = 0, ks = 0, n = 0;
             uint32_t qph = 0, kph = 0;
+            // CONC: item-end notices for the epilogue warpgroup(s) that did not get the item's last
+            // tile (tile-less headers: no MMA, both acc_full arrivals from here)
+            auto post_marks = [&](int cnt, int kord) {
+                for (int e = 0; e < cnt; ++e, ++n) {
+                    const int ab = n % C::NACC;
+                    DW_WAIT(&acc_empty[ab], ((n / C::NACC) & 1) ^ 1, 2);
+                    if (elect_one()) {
+                        hdr[ab].flags = HDR_MARK | (kord << 8);
+                        mbar_arrive(&acc_full[ab]);
+                        mbar_arrive(&acc_full[ab]);
+                    }
+                    __syncwarp();
+                }
+            };
             for (ItemWalk iw(sc, it_begin, it_end, p.p1_reverse); iw.more();) {
                 const bool keep = iw.it >= it_end - p.x_keep;  // before next(): the index of this item
+                const int kord = iw.it - it_begin;             // CONC: the item's place in the CTA's list
                 const ItemInfo I = iw.next();
-                if (I.t0 == I.t1) continue;
+                // CONC: at most kConcNI items ahead of GEMM2 (bounds the X' in flight, keeps it in L2)
+                if constexpr (CONC) DW_WAIT(&item_free[kord % kConcNI], ((kord / kConcNI) & 1) ^ 1, 3);
+                if (I.t0 == I.t1) {
+                    if constexpr (CONC) post_marks(2, kord);
+                    continue;
+                }
                 const int kvl = sc.kv_len ? __ldg(sc.kv_len + I.g / p.H) : p.S;
                 DW_WAIT(&q_full[qi], qph, 0);
                 tc_fence_after();
@@ -391,21 +428,22 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
                     DW_WAIT(&acc_empty[ab], ((n / C::NACC) & 1) ^ 1, 2);
                     const int64_t slot = I.slot0 + t;
                     if (elect_one()) {
+                        const int last = (CONC && t + NSUB >= I.t1) ? (HDR_LASTT | (kord << 8)) : 0;
                         hdr[ab] = G1Hdr{(int32_t)(slot & 0xffffffff), (int32_t)(slot >> 32), I.rb * kRowBlock, kvl, w0,
-                                        w1, HDR_TILE | (keep ? HDR_KEEP : 0), 1};  // adjacent sub-tile slots
+                                        w1, HDR_TILE | (keep ? HDR_KEEP : 0) | last, 1};  // adjacent sub-tile slots
                         mbar_arrive(&acc_full[ab]);  // header published (arrival 1 of 2)
                     }
                     __syncwarp();
                     DW_WAIT(&k_full[ks], kph, 1);
                     tc_fence_after();
                     const uint32_t k_addr = smem_u32(smem + C::OFF_K + ks * C::KB);
-                    const uint32_t d_tmem = tmem_base + ab * kMW;
+                    const uint32_t d_tmem = tmem_base + ab * C::MW;
                     if (elect_one()) {
 #pragma unroll
                         for (int kk = 0; kk < D / 16; ++kk) {
                             const uint32_t h = kk / 4, wk = kk % 4;
                             const uint64_t ad = smem_desc_sw128(q_addr + h * (kRowBlock * 128) + wk * 32, 16, 1024);
-                            const uint64_t bd = smem_desc_sw128(k_addr + h * (kMW * 128) + wk * 32, 16, 1024);
+                            const uint64_t bd = smem_desc_sw128(k_addr + h * (C::MW * 128) + wk * 32, 16, 1024);
                             mma_ss(d_tmem, ad, bd, idesc, kk > 0 ? 1u : 0u);
                         }
                         mma_commit(&k_empty[ks]);
@@ -417,6 +455,7 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
                 if (elect_one()) mma_commit(&q_empty[qi]);
                 __syncwarp();
                 if (++qi == C::NQ) { qi = 0; qph ^= 1; }
+                if constexpr (CONC) post_marks(1, kord);
             }
             for (int e = 0; e < 2; ++e, ++n) {  // one END header for each epilogue warpgroup pair
                 const int ab = n % C::NACC;
@@ -472,6 +511,16 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
                 }
                 ++n;
             };
+            // CONC: an item-end notice occupies a slot of the statistics ring without data
+            auto skip_mark = [&]() {
+                if ((n & 1) == par) {
+                    const int buf = n % C::NACC;
+                    DW_WAIT(&st_full[buf], (uint32_t)(n / C::NACC) & 1, 0);
+                    __syncwarp();
+                    if (lane == 0) mbar_arrive(&st_empty[buf]);
+                }
+                ++n;
+            };
             auto flush = [&](int g, int rb, const float (&m)[4], const float (&d)[4]) {
                 const int64_t nrow = (int64_t)p.B * p.H * p.S;
                 const int64_t row = (int64_t)g * p.S + rb * kRowBlock + lane + 2 * par * nrow;
@@ -505,16 +554,30 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
                 }
             } else {
                 for (ItemWalk iw(sc, it_begin, it_end, p.p1_reverse); iw.more();) {
+                    const int kord = iw.it - it_begin;
                     const ItemInfo I = iw.next();
-                    if (I.t0 == I.t1) continue;
+                    if (I.t0 == I.t1) {
+                        if constexpr (CONC) {  // the item's two tile-less notices; nothing to merge
+                            skip_mark();
+                            skip_mark();
+                            if (lane == 0) mbar_arrive(&item_done[kord % kConcNI]);
+                        }
+                        continue;
+                    }
                     float m[4], d[4];
 #pragma unroll
                     for (int u = 0; u < 4; ++u) { m[u] = -INFINITY; d[u] = 0.f; }
                     for (int t = I.t0; t < I.t1; t += NSUB) merge(m, d);
                     flush(I.g, I.rb, m, d);
+                    if constexpr (CONC) {  // the item-end notice; rowstat of the item is written
+                        skip_mark();
+                        __syncwarp();
+                        if (lane == 0) mbar_arrive(&item_done[kord % kConcNI]);
+                    }
                 }
             }
         }
+    } else if constexpr (!(RM & 2)) {
     } else if constexpr (SPLIT) {
         if constexpr (REGS) reg_alloc<104>();
         // ------------------------------------------------------------------ epilogue warpgroups
@@ -530,6 +593,7 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
         for (int n = pj;; n += 2, ++k) {
             const int buf = n % C::NACC;
             DW_WAIT(&acc_full[buf], (uint32_t)(n / C::NACC) & 1, 0);
+            DW_PH0();
             tc_fence_after();
             const G1Hdr H = lds_hdr(hdr + buf);
             if (H.flags & HDR_END) break;
@@ -542,13 +606,14 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
             // one TMEM read of the row's 64 fp32 scores; the accumulator goes straight back to the MMA
             uint32_t x[64];
             if (valid) {
-                tmem_ld32(tmem_base + lane_off + buf * kMW + 64 * h, *reinterpret_cast<uint32_t(*)[32]>(&x[0]));
-                tmem_ld32(tmem_base + lane_off + buf * kMW + 64 * h + 32, *reinterpret_cast<uint32_t(*)[32]>(&x[32]));
+                tmem_ld32(tmem_base + lane_off + buf * C::MW + 64 * h, *reinterpret_cast<uint32_t(*)[32]>(&x[0]));
+                tmem_ld32(tmem_base + lane_off + buf * C::MW + 64 * h + 32, *reinterpret_cast<uint32_t(*)[32]>(&x[32]));
                 tmem_wait_ld();
             }
             tc_fence_before();
             __syncwarp();
             if (lane == 0) mbar_arrive(&acc_empty[buf]);
+            DW_PH(3);
             uint8_t* stage = smem + C::OFF_X + (ewg * C::XPW + (k % C::XPW)) * C::HB;
             const uint32_t stage_s = smem_u32(stage);
             // Each warp stages and stores its own 32 rows: its slice of this staging buffer is free
@@ -559,6 +624,7 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
                 else bulk_wait_read0();
             }
             __syncwarp();
+            DW_PH(7);
             float mx = -INFINITY, dsum = 0.f;
             if (valid) {
                 // mask layer: kept keys of this row form <= 2 intervals; interior
@@ -609,6 +675,7 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
                     for (int u = 0; u < 64; u += 2)
                         fadd2_acc(sa[(u >> 1) & 3], sa[4 + ((u >> 1) & 3)], __uint_as_float(x[u]), __uint_as_float(x[u + 1]));
                     dsum = ((sa[0] + sa[4]) + (sa[1] + sa[5])) + ((sa[2] + sa[6]) + (sa[3] + sa[7]));
+                    DW_PH(4);
                 } else {  // unfused baseline: the scaled, masked score
 #pragma unroll
                     for (int u = 0; u < 64; u += 2) {
@@ -638,6 +705,7 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
                 }
                 bulk_commit();
             }
+            DW_PH(5);
             if constexpr (IRT) {  // (m', d') of this row and sub-tile to the IR warp (-inf, 0 if invalid)
                 DW_WAIT(&st_empty[buf], ((uint32_t)(n / C::NACC) & 1) ^ 1, 2);
                 if (NSUB == 2 || h == 0) {
@@ -652,10 +720,11 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
                 p.mprime[slot * kRowBlock + r] = mx * p.scale;  // m' in natural-log units
                 if (!IRT) p.dprime[slot * kRowBlock + r] = dsum;
             }
+            DW_PH(6);
         }
         if (lane == 0) bulk_wait0();
     } else {
-        reg_alloc<224>();  // frees/takes 14336 registers, see the dealloc above
+        if constexpr (REGS) reg_alloc<224>();  // frees/takes 14336 registers, see the dealloc above
         // ------------------------------------------------------------------ epilogue warpgroups
         const int e = (warp - 4) / 4;          // warpgroup 0 / 1: even / odd macro tiles
         const int r = (warp % 4) * 32 + lane;  // tile row == TMEM lane
@@ -664,12 +733,43 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
         const float sl2 = p.scale_log2;
         const int wrow0 = (warp % 4) * 32;  // this warp's 32 rows: a contiguous 4-KB run per column half
         int k = 0;                          // macro tiles processed by this warpgroup
+        // CONC: the item whose end this warp has seen but not yet announced.  It is announced one
+        // header later (after that header's store group is committed, "all but the newest group
+        // complete" covers every store of the item) so the X' stores overlap the next tile.
+        int pend = -1;
+        auto announce = [&](bool all) {
+            if (lane == 0) {
+                if (all) bulk_wait0();
+                else asm volatile("cp.async.bulk.wait_group 1;" ::: "memory");
+            }
+            fence_proxy_async_global();  // this lane's m' stores before GEMM2's bulk reads of them
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&item_done[pend % kConcNI]);
+            pend = -1;
+        };
         for (int n = e;; n += 2, ++k) {
             const int buf = n % C::NACC;
             DW_WAIT(&acc_full[buf], (uint32_t)(n / C::NACC) & 1, 0);
+            DW_PH0();
             tc_fence_after();
             const G1Hdr H = lds_hdr(hdr + buf);
             if (H.flags & HDR_END) break;
+            if constexpr (CONC) {
+                if (H.flags & HDR_MARK) {  // item-end notice: release the slot, commit an empty group,
+                    __syncwarp();          // pass an empty entry through the IR statistics ring
+                    if (lane == 0) {
+                        mbar_arrive(&acc_empty[buf]);
+                        bulk_commit();
+                    }
+                    DW_WAIT(&st_empty[buf], ((uint32_t)(n / C::NACC) & 1) ^ 1, 2);
+                    __syncwarp();
+                    if (lane == 0) mbar_arrive(&st_full[buf]);
+                    if (pend >= 0) announce(false);
+                    pend = H.flags >> 8;
+                    if (kConcNI == 1) announce(true);  // one item in hand-over: announce at once
+                    continue;
+                }
+            }
             const int wsub[2] = {H.w0, H.w1};
             bool vs[NSUB];  // this row's 64-row half is valid in sub-tile s
             bool any = false;
@@ -681,16 +781,17 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
             const int i = H.i0 + r;
             const int64_t slot = ((int64_t)H.slot_hi << 32) | (uint32_t)H.slot_lo;
             // one TMEM read of the row's MW fp32 scores; the accumulator goes straight back to the MMA
-            uint32_t xr[kMW];
+            uint32_t xr[C::MW];
             if (any) {
 #pragma unroll
-                for (int c = 0; c < kMW / 32; ++c)
-                    tmem_ld32(tmem_base + lane_off + buf * kMW + c * 32, *reinterpret_cast<uint32_t(*)[32]>(&xr[c * 32]));
+                for (int c = 0; c < C::MW / 32; ++c)
+                    tmem_ld32(tmem_base + lane_off + buf * C::MW + c * 32, *reinterpret_cast<uint32_t(*)[32]>(&xr[c * 32]));
                 tmem_wait_ld();
             }
             tc_fence_before();
             __syncwarp();
             if (lane == 0) mbar_arrive(&acc_empty[buf]);
+            DW_PH(3);
             uint8_t* stage = smem + C::OFF_X + (e * C::XPW + (k % C::XPW)) * C::XB2;
             const uint32_t stage_s = smem_u32(stage);
             // Each warp stages and stores its own 32 rows (no warpgroup barrier): its slice of this
@@ -701,6 +802,7 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
                 else bulk_wait_read0();
             }
             __syncwarp();
+            DW_PH(7);
             float mx[NSUB], dsum[NSUB];
             const RowMask rm = row_mask(p, i, H.kvl);
 #pragma unroll
@@ -775,6 +877,7 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
                     sts128(stage_s + tile_chunk_off(r, s * (T / 8) + q4), w4[0], w4[1], w4[2], w4[3]);
                 }
             }
+            DW_PH(4);
             // the warp's 32 rows of each valid sub-tile go to HBM: one 4-KB bulk copy per 64 columns
             bool wv[NSUB];
 #pragma unroll
@@ -797,6 +900,7 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
                 }
                 bulk_commit();
             }
+            DW_PH(5);
             if constexpr (IRT) {  // (m', d') of this row per sub-tile to the IR warp (-inf, 0 if invalid)
                 DW_WAIT(&st_empty[buf], ((uint32_t)(n / C::NACC) & 1) ^ 1, 2);
                 float* sb = stats + buf * (4 * kRowBlock);
@@ -816,8 +920,20 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
                         if (!IRT) p.dprime[(slot + (s ? H.pad : 0)) * kRowBlock + r] = dsum[s];
                     }
             }
+            DW_PH(6);
+            if constexpr (CONC) {
+                if (pend >= 0) announce(false);
+                if (H.flags & HDR_LASTT) {
+                    pend = H.flags >> 8;
+                    if (kConcNI == 1) announce(true);
+                }
+            }
+            DW_PH(1);
         }
         if (lane == 0) bulk_wait0();
+        if constexpr (CONC) {
+            if (pend >= 0) announce(true);
+        }
     }
     DW_FLUSH(g_diag_g1);
 }

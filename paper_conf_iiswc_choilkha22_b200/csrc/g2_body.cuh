@@ -32,7 +32,7 @@ namespace sr {
 using namespace ptx;
 
 #ifdef SR_DIAG_WAITS
-static __device__ unsigned long long g_diag_g2[20 * (kDW + 1)];
+static __device__ unsigned long long g_diag_g2[32 * (kDW + 1)];
 #endif
 
 constexpr int kMW2 = 128;  // macro tile width (keys per MMA step)
@@ -52,14 +52,18 @@ struct G2Hdr {  // X'-stage / O-buffer header
     int32_t flags, hv0, hv1, nsub, orow_lo, orow_hi, pad0, pad1;
 };
 
-template <int D, int T>
+// MW_ = 64 / BUDGET / TCOLS (concurrent kernel, k_conc.cu): 64-key macro tiles in BUDGET bytes of
+// shared memory and TCOLS TMEM columns (GEMM1 holds the rest of both)
+template <int D, int T, int MW_ = kMW2, int BUDGET = kSmemMax, int TCOLS = 512>
 struct G2 {
-    static constexpr int NSUB = kMW2 / T;
+    static constexpr int MW = MW_;
+    static constexpr int NSUB = MW / T;
     static constexpr int XS = kRowBlock * T * 2;     // X' slot (sub-tile)
-    static constexpr int XB = kRowBlock * kMW2 * 2;  // X' part of a stage (macro tile)
-    static constexpr int RB = 2048;                  // r' (NSUB x 512 B) + header, keeps 1 KB alignment
+    static constexpr int XB = kRowBlock * MW * 2;    // X' part of a stage (macro tile)
+    static constexpr int RB = NSUB == 1 ? 1024 : 2048;  // r' (NSUB x 512 B) + header, keeps 1 KB alignment
+    static constexpr int HDR_OFF = NSUB * 512;       // stage header after the r' / m' rows
     static constexpr int XSB = XB + RB;              // X' stage
-    static constexpr int VB = kMW2 * D * 2;          // V stage (macro tile)
+    static constexpr int VB = MW * D * 2;            // V stage (macro tile)
     // split the smem budget: V stages from L2 need less depth than the HBM-bound X' stream
 #ifndef SR_G2_NV64
 #define SR_G2_NV64 3
@@ -70,12 +74,12 @@ struct G2 {
 #ifndef SR_G2_NX
 #define SR_G2_NX 8
 #endif
-    static constexpr int NV = D == 64 ? SR_G2_NV64 : SR_G2_NV128;
-    static constexpr int NX_ = (kSmemMax - 3072 - NV * VB) / XSB;
+    static constexpr int NV = (MW == 64 && BUDGET < kSmemMax) ? 2 : (D == 64 ? SR_G2_NV64 : SR_G2_NV128);
+    static constexpr int NX_ = (BUDGET - 3072 - NV * VB) / XSB;
     static constexpr int NX = NX_ > SR_G2_NX ? SR_G2_NX : NX_;
     static_assert(NX >= 2, "smem budget");
     static constexpr int NO = 2;                             // O accumulators (D cols each)
-    static constexpr int NA_ = (512 - NO * D) / (kMW2 / 2);  // A operand buffers (MW/2 cols each)
+    static constexpr int NA_ = (TCOLS - NO * D) / (MW / 2);  // A operand buffers (MW/2 cols each)
     static constexpr int NA = NA_ > 8 ? 8 : NA_;
     static_assert(NA >= 2, "tmem budget");
     static constexpr int OFF_X = 0;
@@ -87,7 +91,7 @@ struct G2 {
     static constexpr int OFF_OHDR = OFF_STATS + NSI * 2 * kRowBlock * 4;
     static constexpr int OFF_TPTR = OFF_OHDR + NO * (int)sizeof(G2Hdr);
     static constexpr int SMEM_ = OFF_TPTR + 16 + 1024;
-    static constexpr int SMEM = SMEM_ > 118 * 1024 ? SMEM_ : 118 * 1024;  // 1 CTA/SM (512 TMEM cols)
+    static constexpr int SMEM = (BUDGET == kSmemMax && SMEM_ < 118 * 1024) ? 118 * 1024 : SMEM_;  // 1 CTA/SM
 #ifndef SR_G2_NGS
 #define SR_G2_NGS 8
 #endif
@@ -98,7 +102,8 @@ struct G2 {
 #define SR_G2_HMUL 1
 #endif
     static constexpr int NGS = SR_G2_NGS;       // GS warps: 8 (64 keys each) or 16 (32 keys each)
-    static constexpr int KPW = kMW2 * 4 / NGS;  // keys of a macro tile per GS warp
+    static constexpr int KPW = MW * 4 / NGS;    // keys of a macro tile per GS warp
+    static_assert(KPW % 32 == 0, "GS warp slices of whole tcgen05.st chunks");
     static constexpr int THREADS = 128 + NGS * 32 + 128;
 };
 
@@ -108,10 +113,11 @@ struct G2 {
 // RS (default mode, IR in GEMM1): as FI, but GEMM1 already merged the rows, so warp 2 only loads each item's
 // per-row (m, 1/d) -- GEMM2 applies the normalisation 1/d * e^{m' - m} in its prologue.
 // Barrier initialisation of GEMM2's shared-memory layout (thread 0; fence_mbar_init included).
-template <int D, int T, bool GS, bool FI, bool RS, bool AS = false>
+template <int D, int T, bool GS, bool FI, bool RS, bool AS = false, int MW = kMW2, int BUDGET = kSmemMax,
+          int TCOLS = 512>
 __device__ __forceinline__ void g2_init(uint8_t* smem)
 {
-    using C = G2<D, T>;
+    using C = G2<D, T, MW, BUDGET, TCOLS>;
     uint64_t* bars = (uint64_t*)(smem + C::OFF_BAR);
     uint64_t* x_full = bars;
     uint64_t* x_empty = x_full + C::NX;
@@ -144,11 +150,31 @@ __device__ __forceinline__ void g2_init(uint8_t* smem)
 // and writes each sub-tile's partial product X'_k V_k to its own TMEM buffer; the scaling warps add
 // r'_k (X'_k V_k) to the rows' O in registers, r'_k = e^{m'_k - m} / d -- the same terms as
 // (X'_k r'_k) V_k (Eq. 2 is linear in each sub-vector), with no per-element GS pass over X'.
-template <int D, int T, bool GS, bool FI, bool RS, bool AS = false>
+// CONC (concurrent kernel, k_conc.cu): these roles run on warps WB .. WB+15 beside GEMM1's and take
+// each item over from it: the X' producer and the statistics warp wait for item_done (ibar[0 ..
+// kConcNI)) of every item in list order and then arrive on item_free (ibar[kConcNI ..)).
+template <int D, int T, bool GS, bool FI, bool RS, bool AS = false, int MW = kMW2, int BUDGET = kSmemMax,
+          int TCOLS = 512, int WB = 0, bool CONC = false, int RM = 7>
 __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p, const DevSched& sc, uint8_t* smem,
-                                          uint32_t tmem_base, int it_begin, int it_end)
+                                          uint32_t tmem_base, int it_begin, int it_end, uint64_t* ibar = nullptr)
 {
-    using C = G2<D, T>;
+    using C = G2<D, T, MW, BUDGET, TCOLS>;
+    // RM: role groups compiled into this call (1: warps 0-3, 2: GS / scaling warps, 4: epilogue), so
+    // a caller can run each group under its own setmaxnreg budget (k_conc.cu)
+    constexpr bool R0 = RM & 1, R1 = RM & 2, R2 = RM & 4;
+    static_assert(WB % 4 == 0, "TMEM lane quadrants follow warp % 4");
+    static_assert(!CONC || (GS && RS && !AS), "concurrent kernel: GS prologue with GEMM1's row statistics");
+    uint64_t* item_done = ibar;
+    uint64_t* item_free = CONC ? ibar + kConcNI : nullptr;
+    // CONC: wait until GEMM1 has completed the item at list position kord, then hand the slot back
+    auto take_item = [&](int kord) {
+        if constexpr (CONC) {
+            mbar_wait(&item_done[kord % kConcNI], (uint32_t)(kord / kConcNI) & 1);
+            __syncwarp();
+            if (elect_one()) mbar_arrive(&item_free[kord % kConcNI]);
+            __syncwarp();
+        }
+    };
     constexpr int NSUB = C::NSUB;
     uint64_t* bars = (uint64_t*)(smem + C::OFF_BAR);
     uint64_t* x_full = bars;
@@ -165,17 +191,17 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
     G2Hdr* ohdr = (G2Hdr*)(smem + C::OFF_OHDR);
     uint32_t* tmem_ptr = (uint32_t*)(smem + C::OFF_TPTR);
     auto xstage = [&](int s) { return smem + C::OFF_X + s * C::XSB; };
-    auto xhdr = [&](int s) { return (G2Hdr*)(xstage(s) + C::XB + 1024); };
+    auto xhdr = [&](int s) { return (G2Hdr*)(xstage(s) + C::XB + C::HDR_OFF); };
     auto vstage = [&](int s) { return smem + C::OFF_V + s * C::VB; };
 
-    const int warp = warp_uniform(), lane = threadIdx.x % 32;
+    const int warp = warp_uniform() - WB, lane = threadIdx.x % 32;
     DW_DECL
     const uint32_t tmem_o = tmem_base;              // NO x D columns
     const uint32_t tmem_a = tmem_base + C::NO * D;  // NA x MW/2 columns
     // this CTA's items: a contiguous range of the longest-processing-time assignment (host)
     const uint8_t* src = (const uint8_t*)(GS ? p.xprime : p.pbuf);
 
-    if (warp == 0) {
+    if (R0 && warp == 0) {
         {
             // -------------------------------------------------------------- X' producer (whole
             // warp walks the schedule; one elected lane issues)
@@ -183,6 +209,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
             const uint64_t pol_x = SR_G2_HINTS ? policy_evict_first() : 0;
             uint32_t sph = 0;
             for (ItemWalk iw(sc, it_begin, it_end, p.p2_reverse); iw.more();) {
+                take_item(iw.it - it_begin);  // CONC: the item's X' and m' are complete
                 const ItemInfo I = iw.next();
                 if (AS && I.t0 == I.t1) {  // no kept key in these rows: an EMPTY stage, written as zeros
                     DW_WAIT(&x_empty[s], sph ^ 1, 0);
@@ -251,7 +278,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
             }
             __syncwarp();
         }
-    } else if (warp == 2) {
+    } else if (R0 && warp == 2) {
         if (RS) {
             // -------------------------------------------------------------- row statistics of the
             // IR merged in GEMM1: the two partials of each of the item's 128 rows merged into (m, 1/d)
@@ -260,6 +287,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
             uint32_t sph = 0;
             const int64_t nrow = (int64_t)p.B * p.H * p.S;
             for (ItemWalk iw(sc, it_begin, it_end, p.p2_reverse); iw.more();) {
+                take_item(iw.it - it_begin);  // CONC: the item's row statistics are written
                 const ItemInfo I = iw.next();
                 if (I.t0 == I.t1) continue;
                 const int64_t row = (int64_t)I.g * p.S + I.rb * kRowBlock + lane;
@@ -342,7 +370,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                 if (++si == C::NSI) { si = 0; sph ^= 1; }
             }
         }
-    } else if (warp == 3) {
+    } else if (R0 && warp == 3) {
         {
             // -------------------------------------------------------------- V producer (whole warp,
             // one elected lane issues)
@@ -368,10 +396,10 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                         for (int u = 0; u < nsub; ++u)
                             for (int h = 0; h < D / 64; ++h) {
                                 if (SR_G2_HINTS)
-                                    tma_load_2d_hint(vstage(s) + h * (kMW2 * 128) + u * (T * 128), &tmV, h * 64,
+                                    tma_load_2d_hint(vstage(s) + h * (C::MW * 128) + u * (T * 128), &tmV, h * 64,
                                                      I.g * p.S + kt[u] * T, &v_full[s], pol_v);
                                 else
-                                    tma_load_2d(vstage(s) + h * (kMW2 * 128) + u * (T * 128), &tmV, h * 64,
+                                    tma_load_2d(vstage(s) + h * (C::MW * 128) + u * (T * 128), &tmV, h * 64,
                                                 I.g * p.S + kt[u] * T, &v_full[s]);
                             }
                         if (SR_G2_VPREFETCH) {  // the macro tile NV steps ahead in this item, into L2
@@ -388,7 +416,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                 }
             }
         }
-    } else if (AS && warp == 1) {
+    } else if (AS && R0 && warp == 1) {
         // ------------------------------------------------------------------ MMA issuer (AS): per
         // macro tile and sub-tile u, X'_u V_u into the next partial-product buffer (D columns)
         const uint32_t idesc = idesc_f16(0, kRowBlock, D, 0, 1);
@@ -416,7 +444,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
 #pragma unroll
                         for (int k2 = 0; k2 < T / 16; ++k2) {
                             const int kk = u * (T / 16) + k2;  // K step of 16 keys within the macro tile
-                            const uint64_t bd = smem_desc_sw128(v_addr + kk * 2048, kMW2 * 128, 1024);
+                            const uint64_t bd = smem_desc_sw128(v_addr + kk * 2048, C::MW * 128, 1024);
                             const uint64_t ad = smem_desc_sw128(x_addr + (kk / 4) * (kRowBlock * 128) + (kk % 4) * 32, 16, 1024);
                             mma_ss(tmem_base + j * D, ad, bd, idesc, k2 > 0 ? 1u : 0u);
                         }
@@ -434,7 +462,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                 if (++xs == C::NX) { xs = 0; xph ^= 1; }
             }
         }
-    } else if (AS && warp >= 4 && warp < 4 + C::NGS) {
+    } else if (AS && R1 && warp >= 4 && warp < 4 + C::NGS) {
         // ------------------------------------------------------------------ accumulator-side GS:
         // warp w owns TMEM lane quadrant (w-4) % 4 (32 rows) and column half (w-4) / 4 of O (D/2
         // fp32 in registers); per sub-tile u: O += r'_u * (X'_u V_u), r'_u = e^{m'_u - m} / d
@@ -515,7 +543,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
             }
             if (++s == C::NX) { s = 0; sph ^= 1; }
         }
-    } else if (warp == 1) {
+    } else if (R0 && warp == 1) {
         {
             // -------------------------------------------------------------- MMA issuer (whole warp,
             // one elected lane issues)
@@ -557,13 +585,13 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                     else DW_WAIT(&x_full[xs], xph, 1);
                     tc_fence_after();
                     const uint32_t v_addr = smem_u32(vstage(s));
-                    const uint32_t a_tm = tmem_a + a * (kMW2 / 2);
+                    const uint32_t a_tm = tmem_a + a * (C::MW / 2);
                     const uint32_t x_addr = smem_u32(xstage(xs));
                     if (elect_one()) {
 #pragma unroll 8
                         for (int kk = 0; kk < nk; ++kk) {
                             // B = V, MN-major SW128: 16 keys per MMA = 2 KB; 64-wide d blocks at LBO = MW*128 B
-                            const uint64_t bd = smem_desc_sw128(v_addr + kk * 2048, kMW2 * 128, 1024);
+                            const uint64_t bd = smem_desc_sw128(v_addr + kk * 2048, C::MW * 128, 1024);
                             if (GS) {
                                 mma_ts(d_tmem, a_tm + kk * 8, bd, idesc, (t == I.t0 && kk == 0) ? 0u : 1u);
                             } else {  // A = the P tile in the stage: K-major SW128, 64-key blocks 16 KB apart
@@ -586,7 +614,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
             }
             post(SH_END, 0, true);
         }
-    } else if (GS && !AS && warp >= 4 && warp < 4 + C::NGS) {
+    } else if (GS && !AS && R1 && warp >= 4 && warp < 4 + C::NGS) {
         // ------------------------------------------------------------------ GS transform
         const int gq = (warp - 4) % 4, ch = (warp - 4) / 4;  // lane quadrant, key slice (KPW keys)
         constexpr int KPW = C::KPW;
@@ -638,7 +666,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                 xv[q] = lds128(xs_s + tile_chunk_off(r, ch * (KPW / 8) + q));
             DW_WAIT(&a_empty[a], aph ^ 1, 1);
             tc_fence_after();
-            const uint32_t a_tm = tmem_a + lane_off + a * (kMW2 / 2);
+            const uint32_t a_tm = tmem_a + lane_off + a * (C::MW / 2);
 #pragma unroll
             for (int c2 = 0; c2 < KPW / 32; ++c2) {  // 32 keys -> 16 packed words per tcgen05.st
                 const int c = ch * (KPW / 32) + c2;
@@ -686,7 +714,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
             if (lane == 0) mbar_arrive(&x_empty[s]);
             if (++s == C::NX) { s = 0; sph ^= 1; }
         }
-    } else if (!AS && warp >= 4 + C::NGS && warp < 8 + C::NGS) {
+    } else if (!AS && R2 && warp >= 4 + C::NGS && warp < 8 + C::NGS) {
         // ------------------------------------------------------------------ output epilogue
         const int r = (warp % 4) * 32 + lane;
         const uint32_t lane_off = (uint32_t)((warp % 4) * 32) << 16;

@@ -150,7 +150,7 @@ cudaError_t launch_tc_one(const Params& p, cudaStream_t st, int64_t* nl)
 
 #ifdef SR_DIAG_WAITS
 // the fused kernel's phase-1 / phase-2 wait counters (this translation unit's copies)
-extern "C" int sr_diag_read_fused(int phase, unsigned long long* out)  // [20][kDW + 1], reset after read
+extern "C" int sr_diag_read_fused(int phase, unsigned long long* out)  // [32][kDW + 1], reset after read
 {
     void* sym = nullptr;
     if (cudaGetSymbolAddress(&sym, phase == 1 ? sr::g_diag_g1 : sr::g_diag_g2) != cudaSuccess) return 1;

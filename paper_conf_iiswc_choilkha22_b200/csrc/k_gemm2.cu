@@ -7,10 +7,10 @@ using namespace ptx;
 
 #ifdef SR_DIAG_WAITS
 }  // namespace sr
-extern "C" int sr_diag_read_g2(unsigned long long* out)  // copies [20 warps][kDW + 1] and resets (diagnostic build)
+extern "C" int sr_diag_read_g2(unsigned long long* out)  // copies [32 warps][kDW + 1] and resets (diagnostic build)
 {
     if (cudaMemcpyFromSymbol(out, sr::g_diag_g2, sizeof(sr::g_diag_g2)) != cudaSuccess) return 1;
-    static unsigned long long zero[20 * (sr::kDW + 1)];
+    static unsigned long long zero[32 * (sr::kDW + 1)];
     return cudaMemcpyToSymbol(sr::g_diag_g2, zero, sizeof(zero)) != cudaSuccess;
 }
 namespace sr {

@@ -167,6 +167,7 @@ cudaError_t launch_tc_unfused(const Params& p, cudaStream_t st, int64_t* nlaunch
 cudaError_t launch_tc_sd(const Params& p, cudaStream_t st, int64_t* nlaunch);
 cudaError_t launch_tc_bwd(const Params& p, cudaStream_t st, int64_t* nlaunch);
 cudaError_t launch_tc_one(const Params& p, cudaStream_t st, int64_t* nlaunch);
+cudaError_t launch_tc_conc(const Params& p, cudaStream_t st, int64_t* nlaunch);
 // k_sched.cu: enqueue copies of n_seg word ranges [seg_off, seg_off + seg_len) of `words` (int32
 // offsets / lengths, multiples of 4) into the same offsets of `region` (device, 16-B aligned),
 // carried in kernel parameters

@@ -10,6 +10,10 @@
 namespace sr {
 
 constexpr int kSmemMax = 232448;  // 227 KB opt-in dynamic shared memory per CTA on sm_100
+#ifndef SR_CONC_NI
+#define SR_CONC_NI 2
+#endif
+constexpr int kConcNI = SR_CONC_NI;  // concurrent kernel (k_conc.cu): GEMM1 -> GEMM2 item hand-over ring depth
 
 // Diagnostic build (-DSR_DIAG_WAITS, tools/diag_waits.py): every warp accumulates the clock cycles
 // it spends in each class of mbarrier wait (c = 0..3) plus its lifetime (slot 4); lane 0 adds them

@@ -72,7 +72,10 @@ def _call(entry_fn, q=0x10000, k=0x20000000, v=0x40000000, out=0x60000000, B_=1,
     (dict(out=0x10000 + 64), sr.SR_ERR_INVALID),          # out overlaps q
     (dict(q=0x10008), sr.SR_ERR_INVALID),                 # misaligned
     (dict(flags=8), sr.SR_ERR_INVALID),
-    (dict(flags=4096), sr.SR_ERR_INVALID),                # unknown bit
+    (dict(flags=8192), sr.SR_ERR_INVALID),                # unknown bit
+    (dict(flags=4096, tile_n=128), sr.SR_ERR_UNSUPPORTED),  # SR_CONCURRENT runs T = 64 ...
+    (dict(flags=4096 | 1), sr.SR_ERR_UNSUPPORTED),        # ... whole layers (no stage bits)
+    (dict(flags=4096 | 128), sr.SR_ERR_INVALID),          # SR_CONCURRENT with SR_ONE_KERNEL
     (dict(flags=128 | 256), sr.SR_ERR_INVALID),           # SR_ONE_KERNEL with SR_TWO_KERNELS
     (dict(flags=128, tile_n=128), sr.SR_ERR_UNSUPPORTED),  # the one-launch kernel runs T = 64
     (dict(flags=16 | 64), sr.SR_ERR_INVALID),             # SR_FUSE_IR with SR_IR_KERNEL

@@ -87,6 +87,7 @@ VARIANTS = {
     "sd": dict(sd=True),
     "gs_prologue": dict(gs_prologue=True),
     "split_kv": dict(split_kv=True),
+    "concurrent": dict(concurrent=True),
 }
 
 

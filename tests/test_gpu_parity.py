@@ -35,13 +35,13 @@ def _ulp_half(dtype, ref):
 
 def run_case(kind, B, H, S, D, dtype, *, causal=False, kv_len=None, layout=None, window=0, n_global=0,
              tile_n=0, fused=True, seed=0, out_f32=True, fuse_ir=False, ir_kernel=False, one_kernel=False,
-             two_kernels=False, gs_prologue=False, split_kv=False):
+             two_kernels=False, gs_prologue=False, split_kv=False, concurrent=False):
     t, q, k, v = qkv(B, H, S, D, dtype, seed)
     scale = 1 / math.sqrt(D)
     od = torch.float32 if out_f32 else TORCH[dtype]
     kw = dict(scale=scale, causal=causal, tile_n=tile_n, fused=fused, out_dtype=od, fuse_ir=fuse_ir,
               ir_kernel=ir_kernel, one_kernel=one_kernel, two_kernels=two_kernels, gs_prologue=gs_prologue,
-              split_kv=split_kv)
+              split_kv=split_kv, concurrent=concurrent)
     if kind == "dense":
         o = sr.mha_dense(q, k, v, kv_len=kv_len, **kw)
     elif kind == "block":
@@ -359,7 +359,7 @@ FUSED_IR_CASES = [
 ]
 
 
-VARIANTS = ["fuse_ir", "ir_kernel", "one_kernel", "two_kernels", "gs_prologue"]
+VARIANTS = ["fuse_ir", "ir_kernel", "one_kernel", "two_kernels", "gs_prologue", "concurrent"]
 
 
 @pytest.mark.parametrize("variant", VARIANTS)
@@ -367,8 +367,9 @@ VARIANTS = ["fuse_ir", "ir_kernel", "one_kernel", "two_kernels", "gs_prologue"]
 def test_fused_ir_variant(kind, kw, variant):
     """The other IR placements against the oracle, same tolerance: SR_FUSE_IR (IR folded into
     GEMM2), SR_IR_KERNEL (the paper's standalone IR kernel writing r'),
-    SR_ONE_KERNEL (GEMM1 and GEMM2 phases of each CTA in one launch, the 16-bit default) and
-    SR_TWO_KERNELS (the same chain as two launches)."""
+    SR_ONE_KERNEL (GEMM1 and GEMM2 phases of each CTA in one launch, the 16-bit default),
+    SR_TWO_KERNELS (the same chain as two launches) and SR_CONCURRENT (GEMM1 and GEMM2 concurrently
+    in one CTA, item hand-over through mbarriers)."""
     kw = dict(kw)
     if kw.get("layout") == "rand":
         kw["layout"] = W.random_layout(kw["H"], kw["S"] // 64, 64, 0.35, seed=8)
@@ -377,6 +378,30 @@ def test_fused_ir_variant(kind, kw, variant):
     if kw.get("kv_len") and 0 in kw["kv_len"]:
         assert np.all(o[list(kw["kv_len"]).index(0)] == 0)
     assert_close(o, ref, dtype, what=f"{variant} {kind}")
+
+
+CONC_CASES = [
+    # empty row-blocks (no tile: both item-end notices, nothing to merge) between full ones
+    ("block", dict(B=1, H=2, S=512, D=128, dtype="bf16",
+                   layout=W.csr_from_sets(64, [[{0, 1}, set(), set(), set(), {2}, {0, 3}, set(), {7}]] * 2))),
+    ("block", dict(B=2, H=1, S=512, D=64, dtype="f16",
+                   layout=W.csr_from_sets(64, [[set(), set(), {2}, {0, 3}, set(), set(), {1, 5, 6}, set()]]))),
+    ("dense", dict(B=3, H=2, S=384, D=128, dtype="f16", kv_len=[0, 200, 384])),  # a head with no key
+    ("dense", dict(B=1, H=1, S=128, D=128, dtype="bf16")),                        # one row-block
+    ("dense", dict(B=8, H=8, S=1024, D=128, dtype="bf16", causal=True)),          # 512 items: rings wrap
+    ("window", dict(B=2, H=2, S=1024, D=128, dtype="bf16", window=510, n_global=8, causal=True)),
+]
+
+
+@pytest.mark.parametrize("kind,kw", CONC_CASES, ids=lambda x: str(x)[:40] if isinstance(x, dict) else x)
+def test_concurrent_edge_cases(kind, kw):
+    """SR_CONCURRENT (k_conc.cu) on the item hand-over's edge cases: empty items (two tile-less
+    notices each), single-row-block layers, many items per CTA (the item_done / item_free rings wrap),
+    and both D; every element against the oracle."""
+    kw = dict(kw)
+    B, H, S, D, dtype = (kw.pop(x) for x in ("B", "H", "S", "D", "dtype"))
+    o, ref = run_case(kind, B, H, S, D, dtype, concurrent=True, **kw)
+    assert_close(o, ref, dtype, what=f"concurrent {kind}")
 
 
 # ------------------------------------------------------------------------------------ SD variant

@@ -10,6 +10,7 @@ mean lifetime per CTA (us at the sampled clock) and the share spent in each wait
                    c7 staging wait, c4 mask/max/exp/sum, c5 pack/st.shared/bulk store, c6 statistics
   GEMM2  X' w0: c0 x_empty | MMA w1: c0 v_full c1 a_full c2 o_empty | stats w2: c0 st_empty
          V w3: c0 v_empty | GS w4-11: c0 x_full c1 a_empty c2 st_full | epilogue w12-15: c0 o_full
+  concurrent (k_conc.cu): GEMM1 as above on warps 0-11 (MMA w1: c3 item_free), GEMM2 on warps 12-27
 """
 import ctypes as C
 import os
@@ -31,11 +32,15 @@ L = Layer(cfg, torch.device("cuda", 0), cfg.idx, sr, torch)
 kw = {"fuse_ir": variant == "fuse_ir", "ir_kernel": variant == "ir_kernel", "two_kernels": variant == "two_kernels"}
 lib = sr.lib()
 KDW = 8
-buf = (C.c_ulonglong * (20 * (KDW + 1)))()
+NW = 32
+buf = (C.c_ulonglong * (NW * (KDW + 1)))()
 L.run(**kw)
 torch.cuda.synchronize()
 ncta = 148
-if variant == "default":  # the one-launch kernel: phase 1 / phase 2 counters of k_fused.cu
+if variant == "concurrent":  # the concurrent kernel (k_conc.cu): GEMM1 warps 0-11, GEMM2 warps 12-27
+    kw = {"concurrent": True}
+    stages = (("CONC GEMM1", 0, lambda b: lib.sr_diag_read_conc(1, b)), ("CONC GEMM2", 0, lambda b: lib.sr_diag_read_conc(2, b)))
+elif variant == "default":  # the one-launch kernel: phase 1 / phase 2 counters of k_fused.cu
     f1 = lambda b: lib.sr_diag_read_fused(1, b)
     f2 = lambda b: lib.sr_diag_read_fused(2, b)
     stages = (("PHASE1 (GEMM1)", 0, f1), ("PHASE2 (GEMM2)", 0, f2))
@@ -47,9 +52,9 @@ for name, bit, fn in stages:
         L.run(stages=bit, **kw)
     torch.cuda.synchronize()
     fn(buf)
-    a = np.array(buf[:], dtype=np.float64).reshape(20, KDW + 1) / reps / ncta
+    a = np.array(buf[:], dtype=np.float64).reshape(NW, KDW + 1) / reps / ncta
     print(f"{name} C{idx} {variant}: per CTA per launch (us at 1.965 GHz); wait shares of lifetime")
-    for w in range(20):
+    for w in range(NW):
         if a[w, KDW] == 0:
             continue
         life = a[w, KDW]

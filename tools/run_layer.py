@@ -1,5 +1,5 @@
 """Run one config's layer a few times (for ncu captures):
-    python tools/run_layer.py CFG [fused|unfused|two_kernels|fused_ir|ir_kernel|sd|train] [reps]
+    python tools/run_layer.py CFG [fused|unfused|two_kernels|fused_ir|ir_kernel|sd|conc|train] [reps]
 (train: forward + training backward on an SR_WS_TRAIN workspace)"""
 import os
 import sys
@@ -24,6 +24,6 @@ for _ in range(reps):
         L.train_step()
     else:
         L.run(fused=fused, fuse_ir=mode == "fused_ir", sd=mode == "sd", ir_kernel=mode == "ir_kernel",
-              two_kernels=mode == "two_kernels")
+              two_kernels=mode == "two_kernels", concurrent=mode == "conc")
 torch.cuda.synchronize()
 print("ok", cfg.name, mode)
