@@ -406,10 +406,10 @@ BlobLayout blob_layout(const HostSched& h, size_t n_desc, size_t n_cta_ptr, size
     L.desc = o; o += 4 * n_desc;    // row-blocks, or their chunks with SR_SPLIT_KV
     L.items = o; o += h.items.size();
     L.cta = o; o += n_cta_ptr;
-    L.iri = o; o += h.items.size();  // the standalone IR kernel's row-block order (longest first)
     L.psl = o; o += n_desc;          // SR_SPLIT_KV: partial slot of each descriptor
     pad();                           // int4 records below
     L.comb = o; o += std::max<size_t>(h.comb.size(), 4);
+    L.iri = o; o += 4 * h.items.size();  // the standalone IR kernel's row-blocks (longest first), as descriptors
     grp(G_ITEMS, s);
     s = o;  // G_PAIR: pair descriptors, union entries, pcta_ptr
     L.pdesc = o; o += 4 * h.pitems.size();
@@ -496,10 +496,18 @@ std::shared_ptr<DevBlob> make_blob(const HostSched& h0, int n_sm, bool split)
     put(L.desc, desc);
     put(L.items, h.items);
     put(L.cta, cta_ptr);
-    put(L.iri, h0.items);  // before the LPT pass: longest first
+    size_t o;
+    o = L.iri;  // the IR kernel's row-block descriptors {item, t0, t1, tp[lh][0]}, before the LPT pass (longest first)
+    for (int32_t it : h0.items) {
+        const int g = it / h0.n_rb, rb = it % h0.n_rb;
+        const int32_t* tp = &h0.tp[(size_t)(h0.lh_mode == LH_ONE ? 0 : (h0.lh_mode == LH_BATCH ? g / h0.H : g % h0.H)) *
+                                   (h0.n_rb + 1)];
+        const int32_t dd[4] = {it, tp[rb], tp[rb + 1], tp[0]};
+        std::copy(dd, dd + 4, w.begin() + o);
+        o += 4;
+    }
     put(L.psl, psl);
     put(L.comb, h.comb);
-    size_t o;
     o = L.pdesc;  // pair item descriptors {g * n_pair + j, e0, e1, tp[lh][0]}
     for (int32_t it : h.pitems) {
         const int g = it / h.n_pair, j = it % h.n_pair, lh = lh_of_g(g);
@@ -577,7 +585,7 @@ DevSched place(const DevBlob& db, void* region, bool has_kv)
     d.item_desc = (const int4*)(b + L.desc);
     d.items = b + L.items;
     d.cta_ptr = b + L.cta;
-    d.ir_items = b + L.iri;
+    d.ir_desc = (const int4*)(b + L.iri);
     d.psl = b + L.psl;
     d.comb = (const int4*)(b + L.comb);
     d.pair_desc = (const int4*)(b + L.pdesc);

@@ -17,7 +17,7 @@ namespace sr {
 // takes tiles t, t + TW, ..., loads all of them at once (m' and d' in registers: one memory round
 // trip), merges them into a partial (m, d) per row; the team's partials meet in shared memory; each
 // warp then writes r' for its own tiles from the m' it still holds.  Row-blocks come longest first
-// (sc.ir_items) in classes of equal TW; a CTA of 8 warps runs 8 / TW row-blocks of one class.  Rows
+// (sc.ir_desc) in classes of equal TW; a CTA of 8 warps runs 8 / TW row-blocks of one class.  Rows
 // longer than 64 tiles (S > 4096 global rows) fold the excess 4 tiles at a time and re-read m'.
 // About 10-15 thread-instructions per (row, tile) merge; 12 B per (row, tile).
 constexpr int kW = 8;
@@ -30,12 +30,15 @@ __device__ __forceinline__ void ir_load(const float* mp, const float* dp, const 
                                         float (&m4)[4], float (&d4)[4], bool with_d)
 {
     const float l2e = 1.4426950408889634f;
-    const bool v = in && ((__ldg(ti + u) >> hbit) & 1);
+    // the statistics are loaded whether or not the half is valid (the slot exists; an invalid half's
+    // values are never used), so these loads and the tile word's load share one memory round trip
     float4 mm = make_float4(0.f, 0.f, 0.f, 0.f), dd = mm;
-    if (v) {
+    if (in) {
         mm = ldg4(mp + (int64_t)u * kRowBlock);
         if (with_d) dd = ldg4(dp + (int64_t)u * kRowBlock);
     }
+    const bool v = in && ((__ldg(ti + u) >> hbit) & 1);
+    if (!v) dd = make_float4(0.f, 0.f, 0.f, 0.f);
     m4[0] = v ? mm.x * l2e : -INFINITY; m4[1] = v ? mm.y * l2e : -INFINITY;
     m4[2] = v ? mm.z * l2e : -INFINITY; m4[3] = v ? mm.w * l2e : -INFINITY;
     d4[0] = dd.x; d4[1] = dd.y; d4[2] = dd.z; d4[3] = dd.w;
@@ -78,10 +81,8 @@ __global__ void __launch_bounds__(kW * 32, 2) ir_kernel(const Params p)
     float* rp = nullptr;
     const int32_t* ti = nullptr;
     if (live) {
-        const int item = __ldg(sc.ir_items + idx);
-        const int g = item / sc.n_rb, rb = item % sc.n_rb;
-        const int32_t* tp = sc.tp + (size_t)lh_of(sc, g, p.H) * (sc.n_rb + 1);
-        const int t0 = __ldg(tp + rb), t1 = __ldg(tp + rb + 1), base = __ldg(tp);
+        const int4 dsc = __ldg(sc.ir_desc + idx);  // one 16-B load: row-block, its tile range, head base
+        const int g = dsc.x / sc.n_rb, t0 = dsc.y, t1 = dsc.z, base = dsc.w;
         const int64_t s0 = ((int64_t)g * sc.slots_per_head - base + t0 + tmw) * kRowBlock + 4 * lane;
         mp = p.mprime + s0; dp = p.dprime + s0; rp = p.rprime + s0; ti = sc.tinfo + t0 + tmw;
         n = t1 - t0;

@@ -67,7 +67,7 @@ struct DevSched {
     int n_cb, n_ccta;
     // standalone IR kernel (SR_IR_KERNEL): row-blocks longest first, in classes of team size 8, 4, 2, 1
     // warps (> 32, 17-32, 9-16, <= 8 tiles); n_ir_class[c] row-blocks in class c
-    const int32_t* ir_items;
+    const int4* ir_desc;  // {g * n_rb + rb, t0, t1, tp[lh][0]} per row-block, class order
     int n_ir_class[4];
     // key-range split (SR_SPLIT_KV): psl[i] = partial-output slot of item descriptor i (a chunk of a
     // split row-block) or -1; comb[j] = {row-block item, first slot, chunks, 0} of split row-block j
