@@ -62,6 +62,9 @@ struct HostSched {
     // per entry, see DevSched::cent); citems g * n_cb + c grouped per CTA (ccta_ptr)
     int n_cb = 0;
     std::vector<int32_t> cpp, cent, citems, ccta_ptr;
+    // unfused softmax: the 64-row halves whose rows hold more than kSmShortChunks 64-key chunks
+    // ((g * n_rb + rb) * 2 + half), run by their own launch with their rows spread over CTAs
+    std::vector<int32_t> sm_long;
     int slots_per_head = 0;
     int max_rb_tiles = 0;
     // key-range split plan (SR_SPLIT_KV): every item as chunks of <= split_L tiles, 4 ints each
@@ -188,6 +191,16 @@ sr_status build_sched(const Request& r, HostSched& hs)
     hs.items.resize(it.size());
     for (size_t i = 0; i < it.size(); ++i) hs.items[i] = it[i].second;
     if (r.kv_len) hs.kv_len.assign(r.kv_len, r.kv_len + r.B);
+    for (int g = 0; g < BH; ++g) {  // long softmax halves (global rows of BigBird / Longformer, dense rows)
+        const int lh = hs.lh_mode == LH_ONE ? 0 : (hs.lh_mode == LH_BATCH ? g / r.H : g % r.H);
+        const int32_t* tp = &hs.tp[(size_t)lh * (hs.n_rb + 1)];
+        for (int rb = 0; rb < hs.n_rb; ++rb)
+            for (int h = 0; h < 2; ++h) {
+                int n = 0;
+                for (int t = tp[rb]; t < tp[rb + 1]; ++t) n += (tinfo_half(hs.tinfo[t]) >> h) & 1;
+                if (n * (T / 64) > kSmShortChunks) hs.sm_long.push_back((g * hs.n_rb + rb) * 2 + h);
+            }
+    }
     // pair lists: merge the (kt-ascending) lists of row-blocks 2j and 2j+1
     hs.n_pair = (hs.n_rb + 1) / 2;
     hs.pp.assign((size_t)hs.n_lh * (hs.n_pair + 1), 0);
@@ -345,7 +358,7 @@ enum BlobGroup { G_BASE = 0, G_ITEMS, G_PAIR, G_FP, G_COL, G_N };
 constexpr int kMaxCta = 1024;  // bound on persistent CTAs per launch (the workspace reserves it)
 
 struct BlobLayout {  // int32-word offsets inside the blob
-    size_t tp, tinfo, kv, desc, items, cta, iri, psl, comb, pdesc, pent, pcta, fp, fpcta, cdesc, cent, ccta;
+    size_t tp, tinfo, kv, desc, items, cta, iri, psl, comb, pdesc, pent, pcta, fp, fpcta, cdesc, cent, ccta, slong;
     size_t g_off[G_N], g_len[G_N];
     size_t words;
 };
@@ -407,6 +420,7 @@ BlobLayout blob_layout(const HostSched& h, size_t n_desc, size_t n_cta_ptr, size
     L.items = o; o += h.items.size();
     L.cta = o; o += n_cta_ptr;
     L.psl = o; o += n_desc;          // SR_SPLIT_KV: partial slot of each descriptor
+    L.slong = o; o += std::max<size_t>(h.sm_long.size(), 1);  // unfused softmax: long-row halves
     pad();                           // int4 records below
     L.comb = o; o += std::max<size_t>(h.comb.size(), 4);
     L.iri = o; o += 4 * h.items.size();  // the standalone IR kernel's row-blocks (longest first), as descriptors
@@ -507,6 +521,7 @@ std::shared_ptr<DevBlob> make_blob(const HostSched& h0, int n_sm, bool split)
         o += 4;
     }
     put(L.psl, psl);
+    put(L.slong, h.sm_long);
     put(L.comb, h.comb);
     o = L.pdesc;  // pair item descriptors {g * n_pair + j, e0, e1, tp[lh][0]}
     for (int32_t it : h.pitems) {
@@ -554,6 +569,7 @@ std::shared_ptr<DevBlob> make_blob(const HostSched& h0, int n_sm, bool split)
     d.mean_rb_tiles = (int)((h.tinfo.size() + (size_t)h.n_lh * h.n_rb - 1) / ((size_t)h.n_lh * h.n_rb));
     d.n_items = (int)(desc.size() / 4);
     d.n_comb = split ? (int)(h.comb.size() / 4) : 0;
+    d.n_sm_long = (int)h.sm_long.size();
     {   // the IR kernel's team classes over iri (longest first): 8 warps for > 4 * kIrWarpTiles tiles,
         // then 4, 2, 1 (each warp merges <= kIrWarpTiles tiles in registers)
         auto lh_of_g2 = [&](int g) { return h0.lh_mode == LH_ONE ? 0 : (h0.lh_mode == LH_BATCH ? g / h0.H : g % h0.H); };
@@ -587,6 +603,7 @@ DevSched place(const DevBlob& db, void* region, bool has_kv)
     d.cta_ptr = b + L.cta;
     d.ir_desc = (const int4*)(b + L.iri);
     d.psl = b + L.psl;
+    d.sm_long = b + L.slong;
     d.comb = (const int4*)(b + L.comb);
     d.pair_desc = (const int4*)(b + L.pdesc);
     d.pent = (const int4*)(b + L.pent);

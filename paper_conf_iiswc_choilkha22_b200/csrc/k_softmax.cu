@@ -209,14 +209,22 @@ __device__ __forceinline__ __half2 ex2_h2(__half2 t)  // one MUFU op for two fp1
     return u2h(y);
 }
 
-template <int T, int NI, bool BF>
+// LONG: the launch for the halves listed in sc.sm_long (rows of more than kSmShortChunks chunks): each
+// CTA takes kLongRows of a listed half's 64 rows, one row per warp, so the few long rows of a layer
+// (global tokens) spread over many SMs instead of 8 warps walking 64 rows in turn.
+constexpr int kLongRows = 8;
+
+template <int T, int NI, bool BF, bool LONG = false>
 __global__ void __launch_bounds__(256) row_softmax_reg(const Params p, int lo, int hi)  // halves with lo < chunks <= hi
 {
     __shared__ int64_t slot_list[1024];  // stored tiles of this half, as slot ids
     __shared__ int n_tiles;
     constexpr int XB = kRowBlock * T * 2, CPT = T / 64;
     const DevSched& sc = p.sc;
-    const int item = blockIdx.x >> 1, half = blockIdx.x & 1;  // item = g * n_rb + rb
+    const int hsel = LONG ? __ldg(sc.sm_long + blockIdx.x / (kHalf / kLongRows)) : (int)blockIdx.x;
+    const int item = hsel >> 1, half = hsel & 1;  // item = g * n_rb + rb
+    const int row_lo = LONG ? (int)(blockIdx.x % (kHalf / kLongRows)) * kLongRows : 0;
+    const int row_hi = LONG ? row_lo + kLongRows : kHalf;
     const int g = item / sc.n_rb, rb = item % sc.n_rb;
     const int32_t* tp = sc.tp + (size_t)lh_of(sc, g, p.H) * (sc.n_rb + 1);
     const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
@@ -237,13 +245,13 @@ __global__ void __launch_bounds__(256) row_softmax_reg(const Params p, int lo, i
     }
     __syncthreads();
     const int nch = n_tiles * CPT;  // 64-key chunks of each row of this half
-    if (nch <= lo || nch > hi) return;  // another launch's length class (or nothing stored)
+    if (!LONG && (nch <= lo || nch > hi)) return;  // another launch's length class (or nothing stored)
     const int sub = lane >> 3;  // chunk within a group of 4
     const int ni = (nch + 3) / 4;  // 16-B words per lane actually used by this half's rows (warp-uniform)
     const __half2 l2e = __float2half2_rn(1.4426950408889634f);
     // NR rows of the warp in flight at once (short rows: more of them, so a warp keeps ~8 loads out)
     constexpr int NR = NI >= 8 ? 1 : 8 / NI;
-    for (int rr0 = warp * NR; rr0 < kHalf; rr0 += 8 * NR) {
+    for (int rr0 = row_lo + warp * NR; rr0 < row_hi; rr0 += 8 * NR) {
         uint4 x[NR][NI];
         int64_t base[NR];
 #pragma unroll
@@ -355,14 +363,17 @@ cudaError_t launch_softmax_reg(const Params& p, cudaStream_t st, int64_t* nl, in
 template <int T, bool BF>
 cudaError_t launch_softmax_classes(const Params& p, cudaStream_t st, int64_t* nl, int max_ch)
 {
-    // rows of <= 16 chunks with a short-row instantiation (several rows in flight per warp); longer
-    // ones (global rows of BigBird / Longformer) with a second launch sized for them
+    // rows of <= kSmShortChunks chunks with a short-row instantiation (several rows in flight per
+    // warp); the halves with longer rows (global rows of BigBird / Longformer) with a second launch
+    // over their list, kLongRows rows per CTA (measured, C4: the long class 55 -> see DESIGN.md)
     int ni = 2;
     while (4 * ni < max_ch) ni *= 2;
     if (ni <= 8) return launch_softmax_reg<T, BF>(p, st, nl, ni, 0, INT32_MAX);
-    cudaError_t e = launch_softmax_reg<T, BF>(p, st, nl, 4, 0, 16);
-    if (e != cudaSuccess) return e;
-    return launch_softmax_reg<T, BF>(p, st, nl, ni, 16, INT32_MAX);
+    cudaError_t e = launch_softmax_reg<T, BF>(p, st, nl, 4, 0, kSmShortChunks);
+    if (e != cudaSuccess || p.sc.n_sm_long == 0) return e;
+    const dim3 grid((unsigned)((int64_t)p.sc.n_sm_long * (kHalf / kLongRows)));
+    return ni == 16 ? launch_pdl(row_softmax_reg<T, 16, BF, true>, grid, dim3(256), 0, st, nl, p, 0, 0)
+                    : launch_pdl(row_softmax_reg<T, 8, BF, true>, grid, dim3(256), 0, st, nl, p, 0, 0);
 }
 
 cudaError_t launch_softmax(const Params& p, cudaStream_t st, int64_t* nl)

@@ -22,6 +22,7 @@ constexpr int kRowBlock = 128;  // M of every tcgen05 tile
 constexpr int kHalf = 64;       // validity granularity of tile rows
 constexpr int kIrWarpTiles = 8;  // IR kernel: tiles one warp merges in registers
 constexpr int kSplitRefSms = 148; // SR_SPLIT_KV chunk size reference: about two chunks per SM of a B200
+constexpr int kSmShortChunks = 16; // unfused softmax: rows of up to this many 64-key chunks form the short class
 
 // Where the IR sub-layer runs: its own kernel (SR_IR_KERNEL, the paper's layout), folded into
 // GEMM2 (SR_FUSE_IR), or merged by warps of GEMM1 as the row's tiles are produced (default).
@@ -74,6 +75,9 @@ struct DevSched {
     const int32_t* psl;
     const int4* comb;
     int n_comb;
+    // unfused softmax: 64-row halves whose rows exceed kSmShortChunks chunks, (item * 2 + half)
+    const int32_t* sm_long;
+    int n_sm_long;
 };
 
 // Everything a kernel needs to know about one call.
