@@ -295,7 +295,7 @@ __global__ void __launch_bounds__(384, 1)
             }
         } else if (warp == 3) {
             // ------------------------------------------------------------------ X' + m' producer
-            // X' is streamed (evict_first) unless X' and dS' together fit in half the L2 (p.x_evict_first)
+            // X' is streamed (evict_first) unless X' and dS' together fit in 0.8 of the L2 (p.x_evict_first)
             const uint64_t pol_x = p.x_evict_first ? policy_evict_first() : policy_evict_normal();
             int n = 0;  // macro tile counter, as the MMA warp and the epilogue count them
             for (ItemWalk iw(p.sc, it_begin, it_end); iw.more();) {

@@ -1,5 +1,5 @@
 #!/bin/bash
-# Round-2 evidence captures on the GPU box (then, here: python tools/make_profiles.py r2):
+# A round's evidence captures on the GPU box (then, here: python tools/make_profiles.py ROUND):
 # ncu launch lists of short bench runs per config (DRAM bytes per kernel -> profiles/ncu_traffic.json),
 # --set full of the one-launch kernel (C3, C4), and the compute-sanitizer pass.
 set -u
@@ -20,5 +20,5 @@ for c in 3 4; do
   timeout 300 ncu --set full --clock-control none --import-source on -k regex:ir_kernel -s 1 -c 1 \
     -o gpurun_out/full_c${c}_ir_kernel -f python tools/run_layer.py $c ir_kernel 3 > /dev/null 2>&1
 done
-bash tools/sanitize.sh
+[ "${SKIP_SANITIZE:-0}" = 1 ] || bash tools/sanitize.sh
 ls gpurun_out

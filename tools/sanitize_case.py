@@ -22,9 +22,12 @@ cases = [
     ("C3s", "dense", 1, 4, 1024, 128, "bf16", dict(causal=True)),
     ("C4s", "block", 1, 2, 1024, 64, "f16", dict(layout=W.bigbird_layout(2, 1024, 64))),
     ("C5s", "window", 1, 2, 1024, 64, "f16", dict(window=512, n_global=8)),
+    # one BigBird head at S = 4096: global rows of 64 chunks take the unfused softmax's long-row launch
+    ("C4l", "block", 1, 1, 4096, 64, "f16", dict(layout=W.bigbird_layout(1, 4096, 64))),
 ]
 paths = [("default", {}), ("unfused", dict(fused=False)), ("ir_kernel", dict(ir_kernel=True)),
-         ("sd", dict(sd=True)), ("two_kernels", dict(two_kernels=True))]
+         ("sd", dict(sd=True)), ("two_kernels", dict(two_kernels=True)), ("concurrent", dict(concurrent=True)),
+         ("split_kv", dict(split_kv=True))]
 worst = 0.0
 for name, kind, B, H, S, D, dt, kw in cases:
     t, q, k, v = qkv(B, H, S, D, dt, seed=5)
