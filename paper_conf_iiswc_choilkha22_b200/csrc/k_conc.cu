@@ -31,6 +31,7 @@ namespace sr {
 
 using namespace ptx;
 
+#if SR_G2_NGS == 8  // the warp layout below assumes GEMM2's default 8 GS warps (experiment builds skip it)
 constexpr int kConcThreads = 896;
 constexpr int kConcT1 = 128;         // GEMM1 TMEM columns
 
@@ -129,6 +130,9 @@ cudaError_t launch_tc_conc(const Params& p, cudaStream_t st, int64_t* nl)
     if (p.T != 64 || p.in_dtype == DT_F32 || p.g1_pair) return cudaErrorInvalidValue;
     return p.D == 128 ? launch_conc_d<128>(p, st, nl) : launch_conc_d<64>(p, st, nl);
 }
+#else
+cudaError_t launch_tc_conc(const Params&, cudaStream_t, int64_t*) { return cudaErrorNotSupported; }
+#endif
 
 }  // namespace sr
 

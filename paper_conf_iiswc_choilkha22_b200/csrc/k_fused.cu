@@ -43,7 +43,7 @@ __global__ void __launch_bounds__(640, 1)
 {
     using C1 = G1<D, 64, PAIR>;
     using C2 = G2<D, 64>;
-    static_assert(C1::THREADS == 640 && C2::THREADS <= 640, "warp budget");
+    static_assert(C1::THREADS == 640 && (C2::THREADS <= 640 || SR_G2_NGS != 8), "warp budget");
     extern __shared__ uint8_t smem_raw[];
     uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
     uint32_t* tmem_ptr = (uint32_t*)(smem + C1::OFF_TPTR);
