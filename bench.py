@@ -261,7 +261,7 @@ class Layer:
         self.bwd()
 
     def run(self, fused=True, stages=0, q=None, k=None, v=None, fuse_ir=False, sd=False, ir_kernel=False,
-            two_kernels=False, unfused_T=64, resident=False, concurrent=False):
+            two_kernels=False, unfused_T=64, resident=False, concurrent=False, gs_prologue=False):
         d = self.dev
         two = fuse_ir or ir_kernel or two_kernels
         if sd:
@@ -275,7 +275,7 @@ class Layer:
         return self.sr.call(self.mask, q if q is not None else d["q"], k if k is not None else d["k"],
                             v if v is not None else d["v"], out=self.out, fused=fused, stages=stages,
                             workspace=ws, tile_n=tn, fuse_ir=fuse_ir, sd=sd, ir_kernel=ir_kernel,
-                            two_kernels=two_kernels, concurrent=concurrent,
+                            two_kernels=two_kernels, concurrent=concurrent, gs_prologue=gs_prologue,
                             # single-kernel timing: the schedule is already in the workspace
                             sched_resident=resident or stages != 0, **self.kw)
 
@@ -929,6 +929,11 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    # SR_BENCH_SHARED_GPU=1: a functional check of the N > 1 code path on a one-GPU box -- every rank
+    # on cuda:0, gloo for the host-side plumbing; the timings of such a run mean nothing
+    shared = os.environ.get("SR_BENCH_SHARED_GPU") == "1"
+    if shared:
+        local_rank = 0
     if args.impl == "reference":
         res = reference_arm(args, rank, world)
         if res is not None:
@@ -937,7 +942,10 @@ def main():
     import torch
     if world > 1:
         torch.cuda.set_device(local_rank)
-        torch.distributed.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        if shared:
+            torch.distributed.init_process_group("gloo")
+        else:
+            torch.distributed.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
     res = gpu_arm(args, rank, world, local_rank)
     if res is not None:
         if world == 1:

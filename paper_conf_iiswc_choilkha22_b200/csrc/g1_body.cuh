@@ -481,7 +481,11 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
             const int par = warp - 2;
             int n = 0;
             auto merge = [&](float (&m)[4], float (&d)[4]) {
+#ifdef SR_DIAG_NOSTATS
+                if (false) {
+#else
                 if ((n & 1) == par) {
+#endif
                     const int buf = n % C::NACC;
                     DW_WAIT(&st_full[buf], (uint32_t)(n / C::NACC) & 1, 0);
                     const float* sb = stats + buf * (4 * kRowBlock) + lane;
@@ -706,7 +710,11 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
                 bulk_commit();
             }
             DW_PH(5);
+#ifdef SR_DIAG_NOSTATS
+            if constexpr (false) {  // diagnostic: no statistics hand-over (timing only; results wrong)
+#else
             if constexpr (IRT) {  // (m', d') of this row and sub-tile to the IR warp (-inf, 0 if invalid)
+#endif
                 DW_WAIT(&st_empty[buf], ((uint32_t)(n / C::NACC) & 1) ^ 1, 2);
                 if (NSUB == 2 || h == 0) {
                     float* sb = stats + buf * (4 * kRowBlock) + (NSUB == 2 ? 2 * h : 0) * kRowBlock;
