@@ -191,7 +191,9 @@ sr_status build_sched(const Request& r, HostSched& hs)
     hs.items.resize(it.size());
     for (size_t i = 0; i < it.size(); ++i) hs.items[i] = it[i].second;
     if (r.kv_len) hs.kv_len.assign(r.kv_len, r.kv_len + r.B);
-    for (int g = 0; g < BH; ++g) {  // long softmax halves (global rows of BigBird / Longformer, dense rows)
+    // long softmax halves (global rows of BigBird / Longformer, dense rows), listed only for layers
+    // whose longest rows take the softmax's two-launch path (> 4 x 8 chunks, k_softmax.cu)
+    for (int g = 0; hs.max_rb_tiles * (T / 64) > 32 && g < BH; ++g) {
         const int lh = hs.lh_mode == LH_ONE ? 0 : (hs.lh_mode == LH_BATCH ? g / r.H : g % r.H);
         const int32_t* tp = &hs.tp[(size_t)lh * (hs.n_rb + 1)];
         for (int rb = 0; rb < hs.n_rb; ++rb)
@@ -354,7 +356,7 @@ sr_status check_request(sr_entry e, int B, int H, int S, int D, int in_dtype,
 
 // Word groups of the blob, each a contiguous, 16-B aligned range; a call uploads only the groups
 // its kernels read.
-enum BlobGroup { G_BASE = 0, G_ITEMS, G_PAIR, G_FP, G_COL, G_N };
+enum BlobGroup { G_BASE = 0, G_ITEMS, G_PAIR, G_FP, G_COL, G_SML, G_N };
 constexpr int kMaxCta = 1024;  // bound on persistent CTAs per launch (the workspace reserves it)
 
 struct BlobLayout {  // int32-word offsets inside the blob
@@ -420,7 +422,6 @@ BlobLayout blob_layout(const HostSched& h, size_t n_desc, size_t n_cta_ptr, size
     L.items = o; o += h.items.size();
     L.cta = o; o += n_cta_ptr;
     L.psl = o; o += n_desc;          // SR_SPLIT_KV: partial slot of each descriptor
-    L.slong = o; o += std::max<size_t>(h.sm_long.size(), 1);  // unfused softmax: long-row halves
     pad();                           // int4 records below
     L.comb = o; o += std::max<size_t>(h.comb.size(), 4);
     L.iri = o; o += 4 * h.items.size();  // the standalone IR kernel's row-blocks (longest first), as descriptors
@@ -439,6 +440,9 @@ BlobLayout blob_layout(const HostSched& h, size_t n_desc, size_t n_cta_ptr, size
     L.cent = o; o += std::max<size_t>(h.cent.size(), 4);
     L.ccta = o; o += n_ccta_ptr;
     grp(G_COL, s);
+    s = o;  // G_SML: the unfused softmax's long-row halves (uploaded by the unfused path only)
+    L.slong = o; o += std::max<size_t>(h.sm_long.size(), 1);
+    grp(G_SML, s);
     L.words = o;
     return L;
 }
@@ -967,7 +971,8 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
     // the schedule groups this call's kernels read, uploaded into the workspace ahead of them
     const bool one_pair = fused == 1 && one && p.g1_pair;
     const unsigned groups = one_pair ? (1u << G_BASE | 1u << G_PAIR | 1u << G_FP)
-                                     : (1u << G_BASE | 1u << G_ITEMS | (p.g1_pair ? 1u << G_PAIR : 0u));
+                                     : (1u << G_BASE | 1u << G_ITEMS | (p.g1_pair ? 1u << G_PAIR : 0u) |
+                                        (!fused && !cs->hs.sm_long.empty() ? 1u << G_SML : 0u));
     if (!(ex->flags & SR_SCHED_RESIDENT) && (ce = upload(*db, region, groups, st, &nl)) != cudaSuccess) {
         g_launches += nl;
         return fail(SR_ERR_CUDA, "schedule upload: %s", cudaGetErrorString(ce));
