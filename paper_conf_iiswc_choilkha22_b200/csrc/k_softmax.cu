@@ -215,16 +215,19 @@ __device__ __forceinline__ __half2 ex2_h2(__half2 t)  // one MUFU op for two fp1
 constexpr int kLongRows = 8;
 
 template <int T, int NI, bool BF, bool LONG = false>
-__global__ void __launch_bounds__(256) row_softmax_reg(const Params p, int lo, int hi)  // halves with lo < chunks <= hi
+__global__ void __launch_bounds__(256) row_softmax_reg(const Params p, int lo, int hi, int rsplit)  // halves with lo < chunks <= hi
 {
     __shared__ int64_t slot_list[1024];  // stored tiles of this half, as slot ids
     __shared__ int n_tiles;
     constexpr int XB = kRowBlock * T * 2, CPT = T / 64;
     const DevSched& sc = p.sc;
-    const int hsel = LONG ? __ldg(sc.sm_long + blockIdx.x / (kHalf / kLongRows)) : (int)blockIdx.x;
+    // a half's 64 rows over rsplit CTAs (LONG: kHalf / kLongRows): more, smaller CTAs shorten the
+    // grid's last partial wave
+    const int rs = LONG ? kHalf / kLongRows : rsplit;
+    const int hsel = LONG ? __ldg(sc.sm_long + blockIdx.x / rs) : (int)(blockIdx.x / rs);
     const int item = hsel >> 1, half = hsel & 1;  // item = g * n_rb + rb
-    const int row_lo = LONG ? (int)(blockIdx.x % (kHalf / kLongRows)) * kLongRows : 0;
-    const int row_hi = LONG ? row_lo + kLongRows : kHalf;
+    const int row_lo = (int)(blockIdx.x % rs) * (kHalf / rs);
+    const int row_hi = row_lo + kHalf / rs;
     const int g = item / sc.n_rb, rb = item % sc.n_rb;
     const int32_t* tp = sc.tp + (size_t)lh_of(sc, g, p.H) * (sc.n_rb + 1);
     const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
@@ -351,12 +354,16 @@ cudaError_t launch_softmax_t(const Params& p, cudaStream_t st, int64_t* nl)
 template <int T, bool BF>
 cudaError_t launch_softmax_reg(const Params& p, cudaStream_t st, int64_t* nl, int ni, int lo, int hi)
 {
-    const dim3 grid((unsigned)((int64_t)p.B * p.H * p.sc.n_rb * 2));
+    static const int env_rs = [] { const char* e = getenv("SR_SOFTMAX_RSPLIT"); return e ? atoi(e) : 0; }();
+    // rows of 17-32 chunks (one row per warp at a time): two CTAs per half (measured, back to back:
+    // C3 107.2 -> 101.9 us); shorter rows keep one (C2, C4-C6 within noise or slower split)
+    const int rs = env_rs == 1 || env_rs == 2 || env_rs == 4 || env_rs == 8 ? env_rs : (ni == 8 ? 2 : 1);
+    const dim3 grid((unsigned)((int64_t)p.B * p.H * p.sc.n_rb * 2 * rs));
     switch (ni) {
-    case 2: return launch_pdl(row_softmax_reg<T, 2, BF>, grid, dim3(256), 0, st, nl, p, lo, hi);
-    case 4: return launch_pdl(row_softmax_reg<T, 4, BF>, grid, dim3(256), 0, st, nl, p, lo, hi);
-    case 8: return launch_pdl(row_softmax_reg<T, 8, BF>, grid, dim3(256), 0, st, nl, p, lo, hi);
-    default: return launch_pdl(row_softmax_reg<T, 16, BF>, grid, dim3(256), 0, st, nl, p, lo, hi);
+    case 2: return launch_pdl(row_softmax_reg<T, 2, BF>, grid, dim3(256), 0, st, nl, p, lo, hi, rs);
+    case 4: return launch_pdl(row_softmax_reg<T, 4, BF>, grid, dim3(256), 0, st, nl, p, lo, hi, rs);
+    case 8: return launch_pdl(row_softmax_reg<T, 8, BF>, grid, dim3(256), 0, st, nl, p, lo, hi, rs);
+    default: return launch_pdl(row_softmax_reg<T, 16, BF>, grid, dim3(256), 0, st, nl, p, lo, hi, rs);
     }
 }
 
@@ -372,8 +379,8 @@ cudaError_t launch_softmax_classes(const Params& p, cudaStream_t st, int64_t* nl
     cudaError_t e = launch_softmax_reg<T, BF>(p, st, nl, 4, 0, kSmShortChunks);
     if (e != cudaSuccess || p.sc.n_sm_long == 0) return e;
     const dim3 grid((unsigned)((int64_t)p.sc.n_sm_long * (kHalf / kLongRows)));
-    return ni == 16 ? launch_pdl(row_softmax_reg<T, 16, BF, true>, grid, dim3(256), 0, st, nl, p, 0, 0)
-                    : launch_pdl(row_softmax_reg<T, 8, BF, true>, grid, dim3(256), 0, st, nl, p, 0, 0);
+    return ni == 16 ? launch_pdl(row_softmax_reg<T, 16, BF, true>, grid, dim3(256), 0, st, nl, p, 0, 0, 0)
+                    : launch_pdl(row_softmax_reg<T, 8, BF, true>, grid, dim3(256), 0, st, nl, p, 0, 0, 0);
 }
 
 cudaError_t launch_softmax(const Params& p, cudaStream_t st, int64_t* nl)
