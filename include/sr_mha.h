@@ -43,7 +43,10 @@
  *    Calls are asynchronous: device-side faults surface at the caller's next synchronisation (as
  *    with cuBLAS).  Two calls in flight at once (other streams, other threads) need two workspaces.
  *  - A row whose every key is masked outputs 0 (reading R9).
- *  - Supported: S % 128 == 0, S >= 128; D in {64, 128}; in_dtype F16 or BF16 (tensor-core path) or
+ *  - Supported: S % 64 == 0, S >= 64 (tile_n = 128 needs S % 128 == 0; with S % 128 == 64 the default
+ *    sub-vector is 64 and the last 128-row tile is half inside the head -- its other half is never
+ *    computed into the workspace and no row beyond S of out / dq / dk / dv is written);
+ *    D in {64, 128}; in_dtype F16 or BF16 (tensor-core path) or
  *    F32 (SIMT fp32 path, every mask kind); out_dtype == in_dtype or F32; block == 64.
  *    Anything else returns SR_ERR_UNSUPPORTED before touching the device.
  *

@@ -108,7 +108,9 @@ sr_status build_sched(const Request& r, HostSched& hs)
     const int S = r.S, T = r.T;
     hs.T = T;
     hs.H = r.H;
-    hs.n_rb = S / kRowBlock;
+    // S % 128 == 64: the last row-block's upper 64-row half lies beyond the head (never valid: its
+    // tiles are neither computed into X' nor read, and every kernel skips writes of rows >= S)
+    hs.n_rb = (S + kRowBlock - 1) / kRowBlock;
     const int nkt = S / T;
     std::vector<std::vector<std::pair<int, int>>> lists;  // per (lh, rb): (kt, half bits)
     if (r.entry == SR_E_DENSE || r.entry == SR_E_WINDOW) {
@@ -123,10 +125,12 @@ sr_status build_sched(const Request& r, HostSched& hs)
                     for (int h = 0; h < 2; ++h) {
                         int r0 = rb * kRowBlock + h * kHalf, r1 = r0 + kHalf - 1;
                         bool ok;
-                        if (r.entry == SR_E_DENSE)
+                        if (r0 >= S)
+                            ok = false;
+                        else if (r.entry == SR_E_DENSE)
                             ok = c0 < kvl && (!r.causal || c0 <= r1);
                         else
-                            ok = window_half_valid(r0, r1, c0, c1, r.window / 2, r.n_global, r.causal);
+                            ok = window_half_valid(r0, r1, c0, std::min(c1, S - 1), r.window / 2, r.n_global, r.causal);
                         if (ok) bits |= 1 << h;
                     }
                     if (bits) L.push_back({kt, bits});
@@ -145,6 +149,7 @@ sr_status build_sched(const Request& r, HostSched& hs)
                 std::map<int, int> cols;
                 for (int h = 0; h < 2; ++h) {
                     int br = 2 * rb + h;
+                    if (br >= nb) continue;  // S % 128 == 64: no block-row beyond the head
                     for (int32_t t = rp[br]; t < rp[br + 1]; ++t) {
                         int c = lay->col_idx[t];
                         if (r.causal && c > br) continue;  // block entirely above the diagonal
@@ -229,7 +234,7 @@ sr_status build_sched(const Request& r, HostSched& hs)
     if (!hs.tinfo.empty()) hs.pair_saving = 1.0 - (double)(hs.pent.size() / 4) / (double)hs.tinfo.size();
     // column lists (the transpose of the row lists, for dK = dS'^T Q and dV = P^T dO): per 128-key
     // column block, the row-blocks that list one of its key tiles, ascending
-    hs.n_cb = S / kRowBlock;
+    hs.n_cb = (S + kRowBlock - 1) / kRowBlock;
     const int per = kRowBlock / T;  // key tiles per column block
     hs.cpp.assign((size_t)hs.n_lh * (hs.n_cb + 1), 0);
     for (int lh = 0; lh < hs.n_lh; ++lh) {
@@ -294,14 +299,18 @@ sr_status check_request(sr_entry e, int B, int H, int S, int D, int in_dtype,
         return fail(SR_ERR_INVALID, "B, H, S, D must be positive (got %d %d %d %d)", B, H, S, D);
     if (in_dtype != SR_F32 && in_dtype != SR_F16 && in_dtype != SR_BF16)
         return fail(SR_ERR_INVALID, "unknown in_dtype %d", in_dtype);
-    if (S % kRowBlock != 0) return fail(SR_ERR_UNSUPPORTED, "S=%d must be a multiple of 128", S);
+    if (S % kHalf != 0) return fail(SR_ERR_UNSUPPORTED, "S=%d must be a multiple of 64", S);
     if (S > 65536 * 64) return fail(SR_ERR_UNSUPPORTED, "S=%d too large", S);
     if (D != 64 && D != 128) return fail(SR_ERR_UNSUPPORTED, "D=%d must be 64 or 128", D);
-    if ((int64_t)B * H * (S / kRowBlock) > INT32_MAX / 2)
+    if ((int64_t)B * H * ((S + kRowBlock - 1) / kRowBlock) > INT32_MAX / 2)
         return fail(SR_ERR_UNSUPPORTED, "too many (head, row-block) items");
     if (tile_n != 0 && tile_n != 64 && tile_n != 128)
         return fail(SR_ERR_UNSUPPORTED, "tile_n=%d must be 0, 64 or 128", tile_n);
     int T = tile_n ? tile_n : default_T(e, in_dtype, mode);
+    if (T == 128 && S % 128 != 0) {  // 128-key sub-vectors need S % 128 == 0; the default falls back to 64
+        if (tile_n) return fail(SR_ERR_UNSUPPORTED, "tile_n=128 needs S %% 128 == 0 (S=%d)", S);
+        T = 64;
+    }
     if (in_dtype == SR_F32 && T != 64) return fail(SR_ERR_UNSUPPORTED, "fp32 path uses T=64");
     r = Request{e, B, H, S, causal ? 1 : 0, T};
     if (e == SR_E_DENSE) {
@@ -919,7 +928,7 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
 
     Params p{};
     p.q = q; p.k = k; p.v = v; p.out = out;
-    p.B = B; p.H = H; p.S = S; p.D = D; p.T = r.T;
+    p.B = B; p.H = H; p.S = S; p.Spad = (S + kRowBlock - 1) / kRowBlock * kRowBlock; p.D = D; p.T = r.T;
     p.scale = scale;
     p.scale_log2 = scale * 1.4426950408889634f;
     p.causal = r.causal;
@@ -1063,7 +1072,7 @@ sr_status run_bwd(sr_entry e, const void* q, const void* k, const void* v, const
 
     Params p{};
     p.q = q; p.k = k; p.v = v; p.out = const_cast<void*>(out);
-    p.B = B; p.H = H; p.S = S; p.D = D; p.T = r.T;
+    p.B = B; p.H = H; p.S = S; p.Spad = (S + kRowBlock - 1) / kRowBlock * kRowBlock; p.D = D; p.T = r.T;
     p.scale = scale;
     p.scale_log2 = scale * 1.4426950408889634f;
     p.causal = r.causal;

@@ -526,8 +526,8 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
                 ++n;
             };
             auto flush = [&](int g, int rb, const float (&m)[4], const float (&d)[4]) {
-                const int64_t nrow = (int64_t)p.B * p.H * p.S;
-                const int64_t row = (int64_t)g * p.S + rb * kRowBlock + lane + 2 * par * nrow;
+                const int64_t nrow = (int64_t)p.B * p.H * p.Spad;  // rowstat rows: per head, whole row-blocks
+                const int64_t row = (int64_t)g * p.Spad + rb * kRowBlock + lane + 2 * par * nrow;
 #pragma unroll
                 for (int j = 0; j < 4; ++j) {
                     p.rowstat[row + 32 * j] = m[j] * p.scale;  // -inf stays -inf

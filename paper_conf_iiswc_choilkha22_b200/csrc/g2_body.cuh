@@ -49,8 +49,10 @@ enum : int { SH_TILE = 1, SH_END = 2, SH_EMPTY = 4, SH_FIRST = 8, SH_LAST = 16, 
 // never written: zero rows for the invalid 64-row halves of a P tile read as an smem MMA operand
 static __device__ __align__(128) uint8_t g_zero_g2[kHalf * 128];
 struct G2Hdr {  // X'-stage / O-buffer header
-    int32_t flags, hv0, hv1, nsub, orow_lo, orow_hi, pad0, pad1;
-};
+    int32_t flags, hv0, hv1, nsub, orow_lo, orow_hi, nv, pad1;  // nv: rows of the block inside the head (< 128 only
+};                                                               // for the last row-block when S % 128 == 64)
+// rows of row-block rb that lie inside the head (S % 128 == 64 leaves the last one half outside)
+__device__ __forceinline__ int rows_in_head(const Params& p, int rb) { return min(kRowBlock, p.S - rb * kRowBlock); }
 
 // MW_ = 64 / BUDGET / TCOLS (concurrent kernel, k_conc.cu): 64-key macro tiles in BUDGET bytes of
 // shared memory and TCOLS TMEM columns (GEMM1 holds the rest of both)
@@ -216,7 +218,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                     if (elect_one()) {
                         const int64_t orow = (int64_t)I.g * p.S + I.rb * kRowBlock;
                         *xhdr(s) = G2Hdr{SH_EMPTY | SH_FIRST | SH_LAST, 0, 0, 0, (int32_t)(orow & 0xffffffff),
-                                         (int32_t)(orow >> 32), 0, 0};
+                                         (int32_t)(orow >> 32), rows_in_head(p, I.rb), 0};
                         mbar_arrive(&x_full[s]);
                     }
                     __syncwarp();
@@ -238,7 +240,8 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                     if (elect_one()) {
                     const int64_t orow = (int64_t)I.g * p.S + I.rb * kRowBlock;
                     *xhdr(s) = G2Hdr{SH_TILE | (t == I.t0 ? SH_FIRST : 0) | (t + NSUB >= I.t1 ? SH_LAST : 0), hv[0],
-                                     hv[1], nsub, (int32_t)(orow & 0xffffffff), (int32_t)(orow >> 32), 0, 0};
+                                     hv[1], nsub, (int32_t)(orow & 0xffffffff), (int32_t)(orow >> 32),
+                                     rows_in_head(p, I.rb), 0};
                     mbar_arrive_expect_tx(&x_full[s], bytes);
                     const uint8_t* xs = src + (I.slot0 + t) * (int64_t)C::XS;  // sub-tiles t, t+1 are adjacent
                     auto xload = [&](uint8_t* d, const uint8_t* g, uint32_t n) {
@@ -285,12 +288,12 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
             // in the ring (lane: rows l + 32 j)
             int si = 0;
             uint32_t sph = 0;
-            const int64_t nrow = (int64_t)p.B * p.H * p.S;
+            const int64_t nrow = (int64_t)p.B * p.H * p.Spad;  // rowstat rows: per head, whole row-blocks
             for (ItemWalk iw(sc, it_begin, it_end, p.p2_reverse); iw.more();) {
                 take_item(iw.it - it_begin);  // CONC: the item's row statistics are written
                 const ItemInfo I = iw.next();
                 if (I.t0 == I.t1) continue;
-                const int64_t row = (int64_t)I.g * p.S + I.rb * kRowBlock + lane;
+                const int64_t row = (int64_t)I.g * p.Spad + I.rb * kRowBlock + lane;
                 float mv[4], iv[4];
 #pragma unroll
                 for (int j = 0; j < 4; ++j) {  // GEMM1's two IR warps' partials (m_w, d_w) of the row
@@ -528,7 +531,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                 __syncwarp();
                 if (lane == 0) mbar_arrive(&x_empty[s]);
             }
-            if (h.flags & SH_LAST) {  // this warp's D/2 columns of its 32 output rows
+            if ((h.flags & SH_LAST) && r < h.nv) {  // this warp's D/2 columns of its 32 output rows
                 if (p.out_dtype == DT_F32) {
                     float4* O = reinterpret_cast<float4*>((float*)p.out + orow * D + hh * DH);
 #pragma unroll
@@ -550,10 +553,10 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
             const uint32_t idesc = idesc_f16(p.in_dtype == DT_BF16 ? 1 : 0, kRowBlock, D, 0, 1);
             int s = 0, a = 0, o = 0, xs = 0;
             uint32_t sph = 0, aph = 0, oph = 0, xph = 0;
-            auto post = [&](int flags, int64_t orow, bool second) {  // O header to the epilogue, arrival 1 of 2
+            auto post = [&](int flags, int64_t orow, int nv, bool second) {  // O header, arrival 1 of 2
                 DW_WAIT(&o_empty[o], oph ^ 1, 2);
                 if (elect_one()) {
-                    ohdr[o] = G2Hdr{flags, 0, 0, 0, (int32_t)(orow & 0xffffffff), (int32_t)(orow >> 32), 0, 0};
+                    ohdr[o] = G2Hdr{flags, 0, 0, 0, (int32_t)(orow & 0xffffffff), (int32_t)(orow >> 32), nv, 0};
                     mbar_arrive(&o_full[o]);
                     if (second) mbar_arrive(&o_full[o]);  // no MMA commit will follow
                 }
@@ -571,12 +574,13 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                 // a chunk of a split row-block (SR_SPLIT_KV) writes fp32 partial rows to its slot
                 const int ps = (!AS && p.partial) ? __ldg(sc.psl + at(it)) : -1;
                 const int64_t orow = ps >= 0 ? (int64_t)ps * kRowBlock : (int64_t)I.g * p.S + I.rb * kRowBlock;
+                const int nv = ps >= 0 ? kRowBlock : rows_in_head(p, I.rb);  // a partial slot holds all 128
                 if (I.t0 == I.t1) {  // no kept key in these rows: the epilogue writes zeros
-                    post(SH_EMPTY, orow, true);
+                    post(SH_EMPTY, orow, nv, true);
                     next_o();
                     continue;
                 }
-                post(SH_TILE | (ps >= 0 ? SH_PARTIAL : 0), orow, false);
+                post(SH_TILE | (ps >= 0 ? SH_PARTIAL : 0), orow, nv, false);
                 const uint32_t d_tmem = tmem_o + o * D;
                 for (int t = I.t0; t < I.t1; t += NSUB) {
                     const int nk = min(NSUB, I.t1 - t) * (T / 16);  // K steps of 16 keys
@@ -612,7 +616,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                 __syncwarp();
                 next_o();
             }
-            post(SH_END, 0, true);
+            post(SH_END, 0, 0, true);
         }
     } else if (GS && !AS && R1 && warp >= 4 && warp < 4 + C::NGS) {
         // ------------------------------------------------------------------ GS transform
@@ -727,7 +731,8 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
             if (h.flags & SH_END) break;
             const int64_t orow = (((int64_t)h.orow_hi << 32) | (uint32_t)h.orow_lo) + r;
             if (h.flags & SH_EMPTY) {  // no kept key anywhere in these rows: output 0 (reading R9)
-                if (p.out_dtype == DT_F32) {
+                if (r >= h.nv) {       // (a row beyond the head: not ours to write)
+                } else if (p.out_dtype == DT_F32) {
                     float4* O = reinterpret_cast<float4*>((float*)p.out + orow * D);
                     for (int c = 0; c < D / 4; ++c) O[c] = make_float4(0.f, 0.f, 0.f, 0.f);
                 } else {
@@ -742,7 +747,8 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                     uint32_t v[32];
                     tmem_ld32(taddr + c * 32, v);
                     tmem_wait_ld();
-                    if (part || p.out_dtype == DT_F32) {
+                    if (r >= h.nv) {  // a row beyond the head (S % 128 == 64): loaded with the warp, not stored
+                    } else if (part || p.out_dtype == DT_F32) {
                         float4* O = reinterpret_cast<float4*>((part ? p.partial : (float*)p.out) + orow * D + c * 32);
 #pragma unroll
                         for (int u = 0; u < 8; ++u)

@@ -60,12 +60,14 @@ __global__ void __launch_bounds__(kPrepThreads) bwd_prep(const Params p)
     // the statistics threads issue their IR-partial loads first, so the two memory round trips of a
     // block (dO / O, then rowstat) overlap instead of running back to back
     const int64_t rs = row0 + threadIdx.x;
+    // rowstat / bstat rows are laid out per head in whole row-blocks (p.Spad): the row's index there
+    const int64_t nrowp = (int64_t)p.B * p.H * p.Spad, rsp = (rs / p.S) * p.Spad + rs % p.S;
     float ma = -INFINITY, da = 0.f, mb = -INFINITY, db = 0.f;
     if (threadIdx.x < RPB && rs < nrow) {
-        ma = __ldcg(p.rowstat + rs);
-        da = __ldcg(p.rowstat + nrow + rs);
-        mb = __ldcg(p.rowstat + 2 * nrow + rs);
-        db = __ldcg(p.rowstat + 3 * nrow + rs);
+        ma = __ldcg(p.rowstat + rsp);
+        da = __ldcg(p.rowstat + nrowp + rsp);
+        mb = __ldcg(p.rowstat + 2 * nrowp + rsp);
+        db = __ldcg(p.rowstat + 3 * nrowp + rsp);
     }
     float acc = 0.f;
     if (row < nrow) {
@@ -120,9 +122,9 @@ __global__ void __launch_bounds__(kPrepThreads) bwd_prep(const Params p)
         const int64_t r = rs;
         const float m = fmaxf(ma, mb);  // m = max_w m_w, d = sum_w e^{m_w - m} d_w
         const float d = m == -INFINITY ? 0.f : da * __expf(ma - m) + db * __expf(mb - m);
-        p.bstat[r] = m;
-        p.bstat[nrow + r] = d > 0.f ? 1.f / d : 0.f;
-        p.bstat[2 * nrow + r] = s_delta[threadIdx.x];
+        p.bstat[rsp] = m;
+        p.bstat[nrowp + rsp] = d > 0.f ? 1.f / d : 0.f;
+        p.bstat[2 * nrowp + rsp] = s_delta[threadIdx.x];
         if (p.bwd_dq_fused) {  // dQ of a row-block with no listed tile is 0 (the dS' kernel never visits it)
             const int g = (int)(r / p.S), rb = (int)((r % p.S) / kRowBlock);
             const int32_t* tp = p.sc.tp + (size_t)lh_of(p.sc, g, p.H) * (p.sc.n_rb + 1);
@@ -445,7 +447,7 @@ __global__ void __launch_bounds__(384, 1)
         const uint32_t lane_off = (uint32_t)((warp % 4) * 32) << 16;
         const int wrow0 = (warp % 4) * 32;
         const bool bf = p.in_dtype == DT_BF16;
-        const int64_t nrow = (int64_t)p.B * p.H * p.S;
+        const int64_t nrow = (int64_t)p.B * p.H * p.Spad;
         const uint64_t pol_ds = p.x_evict_first ? policy_evict_first() : policy_evict_normal();
         int64_t cur = -1;
         float m_row = 0.f, invd_row = 0.f, delta_row = 0.f;
@@ -465,11 +467,12 @@ __global__ void __launch_bounds__(384, 1)
             }
             const int64_t row0 = ((int64_t)Hd.row_hi << 32) | (uint32_t)Hd.row_lo;
             const int64_t slot = ((int64_t)Hd.slot_hi << 32) | (uint32_t)Hd.slot_lo;
-            if (row0 != cur) {  // a new row-block: this row's m, 1/d, delta
-                cur = row0;
-                m_row = __ldg(p.bstat + row0 + r);
-                invd_row = __ldg(p.bstat + nrow + row0 + r);
-                delta_row = __ldg(p.bstat + 2 * nrow + row0 + r);
+            if (row0 != cur) {  // a new row-block: this row's m, 1/d, delta (bstat rows per head in whole
+                cur = row0;     // row-blocks, p.Spad)
+                const int64_t prow = (row0 / p.S) * p.Spad + row0 % p.S + r;
+                m_row = __ldg(p.bstat + prow);
+                invd_row = __ldg(p.bstat + nrow + prow);
+                delta_row = __ldg(p.bstat + 2 * nrow + prow);
             }
             uint32_t xr[kMWB];  // dP of this row, fp32
             if (any) {
@@ -543,14 +546,16 @@ __global__ void __launch_bounds__(384, 1)
                 mbar_wait(&dq_full[b], (uint32_t)(Hd.pad >> 1) & 1);
                 tc_fence_after();
                 const BHdr qh = lds_hdr(dqhdr + b);
-                const int64_t qrow = (((int64_t)qh.row_hi << 32) | (uint32_t)qh.row_lo) + r;
+                const int64_t qrow0 = ((int64_t)qh.row_hi << 32) | (uint32_t)qh.row_lo, qrow = qrow0 + r;
+                const bool inhead = qrow0 % p.S + r < p.S;  // S % 128 == 64: the last block's upper half is outside
                 const uint32_t taddr = tmem_base + lane_off + C::NACC * kMWB + b * D;
 #pragma unroll
                 for (int c = 0; c < D / 32; ++c) {
                     uint32_t v[32];
                     tmem_ld32(taddr + c * 32, v);
                     tmem_wait_ld();
-                    if (p.out_dtype == DT_F32) {
+                    if (!inhead) {
+                    } else if (p.out_dtype == DT_F32) {
                         float4* O = reinterpret_cast<float4*>((float*)p.dq + qrow * D + c * 32);
 #pragma unroll
                         for (int u = 0; u < 8; ++u)
@@ -808,9 +813,11 @@ __global__ void __launch_bounds__(384, 1)
             tc_fence_after();
             const KHdr h = lds_hdr(ohdr + o);
             if (h.flags & KV_END) break;
-            const int64_t krow = (((int64_t)h.row_hi << 32) | (uint32_t)h.row_lo) + r;
+            const int64_t krow0 = ((int64_t)h.row_hi << 32) | (uint32_t)h.row_lo, krow = krow0 + r;
+            const bool inhead = krow0 % p.S + r < p.S;  // S % 128 == 64: the last key block's upper half is outside
             if (h.flags & KV_EMPTY) {
-                if (p.out_dtype == DT_F32) {
+                if (!inhead) {
+                } else if (p.out_dtype == DT_F32) {
                     float4* O = reinterpret_cast<float4*>((float*)dst + krow * D);
                     for (int c = 0; c < D / 4; ++c) O[c] = make_float4(0.f, 0.f, 0.f, 0.f);
                 } else {
@@ -824,7 +831,8 @@ __global__ void __launch_bounds__(384, 1)
                     uint32_t v[32];
                     tmem_ld32(taddr + c * 32, v);
                     tmem_wait_ld();
-                    if (p.out_dtype == DT_F32) {
+                    if (!inhead) {
+                    } else if (p.out_dtype == DT_F32) {
                         float4* O = reinterpret_cast<float4*>((float*)dst + krow * D + c * 32);
 #pragma unroll
                         for (int u = 0; u < 8; ++u)

@@ -187,6 +187,7 @@ __global__ void __launch_bounds__(256) combine_kernel(const Params p)
     const int e = (int)(idx % PER), r = e / (D / 4), c4 = e % (D / 4);
     const int4 cb = __ldg(p.sc.comb + j);  // {row-block item, first slot, chunks, 0}
     const int g = cb.x / p.sc.n_rb, rb = cb.x % p.sc.n_rb;
+    if (rb * kRowBlock + r >= p.S) return;  // a row beyond the head (S % 128 == 64)
     float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
     for (int c = 0; c < cb.z; ++c) {
         const float4 v = __ldcg(reinterpret_cast<const float4*>(p.partial + ((int64_t)(cb.y + c) * kRowBlock + r) * D) + c4);

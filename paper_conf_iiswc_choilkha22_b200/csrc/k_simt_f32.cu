@@ -26,7 +26,7 @@ __global__ void __launch_bounds__(128) simt_gemm1_ls_f32(Params p)
     const float* K = (const float*)p.k + (size_t)g * p.S * D;
     float q[D];
 #pragma unroll
-    for (int d = 0; d < D; ++d) q[d] = Q[d];
+    for (int d = 0; d < D; ++d) q[d] = i < p.S ? Q[d] : 0.f;  // rows beyond the head (S % 128 == 64): invalid half
 
     for (int t = t0; t < t1; ++t) {
         const int w = sc.tinfo[t], kt = tinfo_kt(w);
@@ -97,6 +97,7 @@ __global__ void __launch_bounds__(128) simt_gs_gemm2_f32(Params p)
             for (int d = 0; d < D; ++d) o[d] = fmaf(y, vr[d], o[d]);
         }
     }
+    if (i >= p.S) return;  // a row beyond the head (S % 128 == 64)
     float* O = (float*)p.out + ((size_t)g * p.S + i) * D;
 #pragma unroll
     for (int d = 0; d < D; ++d) O[d] = o[d];

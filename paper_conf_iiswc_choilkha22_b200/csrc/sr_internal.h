@@ -87,6 +87,7 @@ struct Params {
     const void* v;
     void* out;
     int B, H, S, D, T;
+    int Spad;          // S rounded up to whole 128-row blocks: the per-head stride of rowstat / bstat
     float scale;       // multiplies Q K^T
     float scale_log2;  // scale * log2(e): the GEMM1 epilogue works in base 2
     int causal;

@@ -72,7 +72,7 @@ def head_costs(B: int, H: int, S: int, T: int = 64, kv_len=None, layout=None, ca
     library default T = 64) plus a fixed cost of 1.5 tiles per row-block (Q load, row statistics,
     O store), the same cost model as the library's LPT CTA schedule (abi.cu).  Heads of an unpadded
     dense or windowed layer all cost the same."""
-    n_rb = S // 128
+    n_rb = -(-S // 128)  # S % 128 == 64: the last row-block is half inside the head
     fixed = 1.5 * n_rb
     if kv_len is not None:
         def tiles(kv):
@@ -92,6 +92,8 @@ def head_costs(B: int, H: int, S: int, T: int = 64, kv_len=None, layout=None, ca
             for p in range(n_rb):
                 cols = set()
                 for br in (2 * p, 2 * p + 1):
+                    if br >= rp.shape[1] - 1:
+                        continue
                     c = ci[rp[lh, br]:rp[lh, br + 1]].tolist()
                     cols.update(x for x in c if not causal or x <= br)
                 n += len(cols)

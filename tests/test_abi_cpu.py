@@ -58,7 +58,8 @@ def _call(entry_fn, q=0x10000, k=0x20000000, v=0x40000000, out=0x60000000, B_=1,
 
 @pytest.mark.parametrize("kw,status", [
     (dict(S=100), sr.SR_ERR_UNSUPPORTED),
-    (dict(S=64), sr.SR_ERR_UNSUPPORTED),
+    (dict(S=96), sr.SR_ERR_UNSUPPORTED),                  # S % 64 != 0
+    (dict(S=192, tile_n=128), sr.SR_ERR_UNSUPPORTED),     # 128-key sub-vectors need S % 128 == 0
     (dict(D=96), sr.SR_ERR_UNSUPPORTED),
     (dict(D=256), sr.SR_ERR_UNSUPPORTED),
     (dict(B_=0), sr.SR_ERR_INVALID),
@@ -172,7 +173,7 @@ def numpy_schedule(S, T, allowed_fn, BH):
     tiles = elems = 0
     for g in range(BH):
         a = allowed_fn(g)
-        for rb in range(S // 128):
+        for rb in range(-(-S // 128)):  # S % 128 == 64: the last row-block is half inside the head
             for kt in range(S // T):
                 blk = a[rb * 128:(rb + 1) * 128, kt * T:(kt + 1) * T]
                 halves = [blk[:64].any(), blk[64:].any()]
@@ -182,11 +183,11 @@ def numpy_schedule(S, T, allowed_fn, BH):
     return tiles, elems
 
 
-@pytest.mark.parametrize("T", [64, 128])
+@pytest.mark.parametrize("T,S", [(64, 512), (128, 512), (64, 320)])
 @pytest.mark.parametrize("causal", [False, True])
-def test_schedule_dense(T, causal):
-    S, H = 512, 2
-    kv = [512, 300, 65, 1]
+def test_schedule_dense(T, S, causal):
+    H = 2
+    kv = [S, 300, 65, 1]
     got = sr.schedule_stats(sr.dense_mask(kv), len(kv), H, S, causal=causal, tile_n=T)
     want = numpy_schedule(S, T, lambda g: oracle_np.allowed_matrix(S, b=g // H, kv_len=kv, causal=causal), len(kv) * H)
     assert got == want
@@ -194,16 +195,19 @@ def test_schedule_dense(T, causal):
 
 @pytest.mark.parametrize("window,n_global,causal,T", [(0, 0, False, 64), (10, 3, False, 64), (300, 8, False, 64),
                                                       (300, 8, True, 128), (130, 64, False, 128), (512, 8, True, 64)])
-def test_schedule_window(window, n_global, causal, T):
-    S = 768
+@pytest.mark.parametrize("S", [768, 448])
+def test_schedule_window(window, n_global, causal, T, S):
+    if S % 128 and T == 128:
+        pytest.skip("128-key sub-vectors need S % 128 == 0")
     got = sr.schedule_stats(sr.window_mask(window, n_global), 1, 1, S, causal=causal, tile_n=T)
     a = oracle_np.allowed_matrix(S, kind="window", window=window, n_global=n_global, causal=causal)
     assert got == numpy_schedule(S, T, lambda g: a, 1)
 
 
+@pytest.mark.parametrize("S", [1024, 576])
 @pytest.mark.parametrize("causal", [False, True])
-def test_schedule_blocksparse(causal):
-    S, H = 1024, 3
+def test_schedule_blocksparse(causal, S):
+    H = 3
     lay = W.random_layout(H, S // 64, 64, 0.3, seed=11)
     got = sr.schedule_stats(sr.block_mask(lay), 2, H, S, causal=causal)
     want = numpy_schedule(S, 64, lambda g: oracle_np.allowed_matrix(S, h=g % H, kind="block", layout=lay,

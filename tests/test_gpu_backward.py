@@ -168,3 +168,20 @@ print("ok")
     env = dict(os.environ, SR_BWD_DQ_SEPARATE="1", PYTHONPATH=root)
     r = subprocess.run([sys.executable, "-c", script], cwd=root, env=env, capture_output=True, text=True, timeout=240)
     assert r.returncode == 0 and "ok" in r.stdout, r.stdout[-2000:] + r.stderr[-4000:]
+
+
+@pytest.mark.parametrize("kind,kw", [
+    ("dense", dict(B=2, H=2, S=192, D=64, dtype="f16", causal=True, kv_len=[192, 100])),
+    ("dense", dict(B=1, H=3, S=320, D=128, dtype="bf16")),
+    ("window", dict(B=1, H=2, S=448, D=64, dtype="f16", window=128, n_global=8)),
+    ("block", dict(B=1, H=2, S=576, D=64, dtype="f16", layout="rand")),
+], ids=lambda x: str(x)[:40] if isinstance(x, dict) else x)
+def test_s_multiple_of_64(kind, kw):
+    """S % 128 == 64: the last row-block / key column block is half inside the head; no gradient row
+    of the next head is touched (every head compared in full)."""
+    kw = dict(kw)
+    if kw.get("layout") == "rand":
+        kw["layout"] = W.random_layout(kw["H"], kw["S"] // 64, 64, 0.35, seed=12)
+    B, H, S, D, dt = (kw.pop(x) for x in ("B", "H", "S", "D", "dtype"))
+    got, ref = run_bwd(kind, B, H, S, D, dt, seed=12, **kw)
+    check(got, ref, dt, what=f"{kind} S={S}")

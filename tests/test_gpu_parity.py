@@ -35,13 +35,13 @@ def _ulp_half(dtype, ref):
 
 def run_case(kind, B, H, S, D, dtype, *, causal=False, kv_len=None, layout=None, window=0, n_global=0,
              tile_n=0, fused=True, seed=0, out_f32=True, fuse_ir=False, ir_kernel=False, one_kernel=False,
-             two_kernels=False, gs_prologue=False, split_kv=False, concurrent=False):
+             two_kernels=False, gs_prologue=False, split_kv=False, concurrent=False, sd=False):
     t, q, k, v = qkv(B, H, S, D, dtype, seed)
     scale = 1 / math.sqrt(D)
     od = torch.float32 if out_f32 else TORCH[dtype]
     kw = dict(scale=scale, causal=causal, tile_n=tile_n, fused=fused, out_dtype=od, fuse_ir=fuse_ir,
               ir_kernel=ir_kernel, one_kernel=one_kernel, two_kernels=two_kernels, gs_prologue=gs_prologue,
-              split_kv=split_kv, concurrent=concurrent)
+              split_kv=split_kv, concurrent=concurrent, sd=sd)
     if kind == "dense":
         o = sr.mha_dense(q, k, v, kv_len=kv_len, **kw)
     elif kind == "block":
@@ -402,6 +402,47 @@ def test_concurrent_edge_cases(kind, kw):
     B, H, S, D, dtype = (kw.pop(x) for x in ("B", "H", "S", "D", "dtype"))
     o, ref = run_case(kind, B, H, S, D, dtype, concurrent=True, **kw)
     assert_close(o, ref, dtype, what=f"concurrent {kind}")
+
+
+S64_CASES = [
+    ("dense", dict(B=2, H=2, S=192, D=64, dtype="f16", kv_len=[192, 70])),
+    ("dense", dict(B=1, H=3, S=320, D=128, dtype="bf16", causal=True)),
+    ("window", dict(B=1, H=2, S=448, D=64, dtype="f16", window=254, n_global=8)),
+    ("window", dict(B=2, H=1, S=320, D=128, dtype="bf16", window=126, n_global=4, causal=True)),
+    ("block", dict(B=1, H=2, S=576, D=64, dtype="f16", layout="rand")),
+    ("dense", dict(B=1, H=1, S=64, D=64, dtype="f16")),  # a single 64-row half
+]
+S64_PATHS = ["default", "unfused", "two_kernels", "ir_kernel", "fuse_ir", "sd", "gs_prologue", "split_kv",
+             "concurrent"]
+
+
+@pytest.mark.parametrize("path", S64_PATHS)
+@pytest.mark.parametrize("kind,kw", S64_CASES, ids=lambda x: str(x)[:40] if isinstance(x, dict) else x)
+def test_s_multiple_of_64(kind, kw, path):
+    """S % 128 == 64 (SURVEY 8(b): S % 64 == 0): the last row-block's upper half lies beyond the head;
+    every path computes every row of every head against the oracle."""
+    kw = dict(kw)
+    if kw.get("layout") == "rand":
+        kw["layout"] = W.random_layout(kw["H"], kw["S"] // 64, 64, 0.35, seed=13)
+    B, H, S, D, dtype = (kw.pop(x) for x in ("B", "H", "S", "D", "dtype"))
+    extra = {} if path == "default" else ({"fused": False} if path == "unfused" else {path: True})
+    o, ref = run_case(kind, B, H, S, D, dtype, **extra, **kw)
+    assert_close(o, ref, dtype, what=f"{path} {kind} S={S}")
+
+
+@pytest.mark.parametrize("dtype,D", [("f16", 64), ("bf16", 128), ("f32", 64)])
+def test_s_multiple_of_64_writes_stay_inside_out(dtype, D):
+    """One head with S % 128 == 64: nothing is written past out's last row (a sentinel after it)."""
+    S = 192
+    t, q, k, v = qkv(1, 1, S, D, dtype, seed=14)
+    od = torch.float32
+    big = torch.full((S * D + 128 * D,), float("nan"), dtype=od, device="cuda")
+    out = big[:S * D].view(1, 1, S, D)
+    sr.mha_dense(q, k, v, scale=1 / math.sqrt(D), causal=True, out=out, out_dtype=od)
+    torch.cuda.synchronize()
+    assert torch.isnan(big[S * D:]).all(), "wrote past the head's last row"
+    ref = oracle.attention(t.q64, t.k64, t.v64, 1 / math.sqrt(D), oracle_mask("dense", None, True, None, 0, 0))
+    assert_close(out.double().cpu().numpy(), ref, dtype)
 
 
 # ------------------------------------------------------------------------------------ SD variant
