@@ -357,7 +357,9 @@ cudaError_t launch_softmax_reg(const Params& p, cudaStream_t st, int64_t* nl, in
     static const int env_rs = [] { const char* e = getenv("SR_SOFTMAX_RSPLIT"); return e ? atoi(e) : 0; }();
     // rows of 17-32 chunks (one row per warp at a time): two CTAs per half (measured, back to back:
     // C3 107.2 -> 101.9 us); shorter rows keep one (C2, C4-C6 within noise or slower split)
-    const int rs = env_rs == 1 || env_rs == 2 || env_rs == 4 || env_rs == 8 ? env_rs : (ni == 8 ? 2 : 1);
+    int rs = env_rs == 1 || env_rs == 2 || env_rs == 4 || env_rs == 8 ? env_rs : (ni == 8 ? 2 : 1);
+    // a CTA's rows must be whole iterations of its 8 warps x NR rows (NR = 8 / NI rows below NI = 8)
+    rs = std::min(rs, ni >= 8 ? 8 : ni);
     const dim3 grid((unsigned)((int64_t)p.B * p.H * p.sc.n_rb * 2 * rs));
     switch (ni) {
     case 2: return launch_pdl(row_softmax_reg<T, 2, BF>, grid, dim3(256), 0, st, nl, p, lo, hi, rs);
@@ -372,7 +374,7 @@ cudaError_t launch_softmax_classes(const Params& p, cudaStream_t st, int64_t* nl
 {
     // rows of <= kSmShortChunks chunks with a short-row instantiation (several rows in flight per
     // warp); the halves with longer rows (global rows of BigBird / Longformer) with a second launch
-    // over their list, kLongRows rows per CTA (measured, C4: the long class 55 -> see DESIGN.md)
+    // over their list, kLongRows rows per CTA (C4 softmax 130 -> 99 us)
     int ni = 2;
     while (4 * ni < max_ch) ni *= 2;
     if (ni <= 8) return launch_softmax_reg<T, BF>(p, st, nl, ni, 0, INT32_MAX);
