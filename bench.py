@@ -686,7 +686,11 @@ def gpu_arm(args, rank, world, local_rank):
                      "achieved_how": "algorithmic bytes of the layer (DESIGN.md §6) / the kernel's duration",
                      "frac_of_nominal_8TBps": round(achieved / NOMINAL_HBM_GBS, 4),
                      "dram_frac": (round(dram / (ms_kern * 1e-3) / 1e9 / hbm_peak, 4) if dram else None),
-                     "tensor_frac": round(flops(cfg, L.stored) / (ms_kern * 1e-3) / 1e12 / tc_peak, 4)},
+                     "tensor_frac": round(flops(cfg, L.stored) / (ms_kern * 1e-3) / 1e12 / tc_peak, 4),
+                     "burst": {"achieved": round(layer_bytes / (ms_burst * 1e-3) / 1e9, 1),
+                               "frac": round(layer_bytes / (ms_burst * 1e-3) / 1e9 / hbm_peak, 4),
+                               "what": "the same bytes over the burst step time (boost clock, before the power "
+                                       "cap engages; the step is the kernel plus its schedule upload)"}},
         "e2e": {"value": round(1e3 / ms_e2e, 2), "unit": "layers/s", "h2d_bytes_per_step": int(h2d),
                 "d2h_bytes_per_step": int(d2h), "ms_per_step": round(ms_e2e, 5),
                 "how": "K steps through the public API, each H2D of its q/k/v from pinned host memory, the "
