@@ -13,12 +13,12 @@ namespace sr {
 // Organisation (vectorised).  A thread owns 4 consecutive rows of a row-block (lane l: rows 4l ..
 // 4l+3, all in one 64-row half), so one warp-wide 16-B load (LDG.128) brings a whole tile's 128
 // statistics -- one 512-B run of the [slot][128] layout.  Each row-block gets a TEAM of TW warps
-// (TW = 1, 2, 4 or 8, so that a warp has at most kIrWarpTiles = 8 of its tiles): warp t of the team
+// (TW = 1, 2, 4 or 8, so that a warp has at most kIrWarpTiles = 4 of its tiles): warp t of the team
 // takes tiles t, t + TW, ..., loads all of them at once (m' and d' in registers: one memory round
 // trip), merges them into a partial (m, d) per row; the team's partials meet in shared memory; each
 // warp then writes r' for its own tiles from the m' it still holds.  Row-blocks come longest first
 // (sc.ir_desc) in classes of equal TW; a CTA of 8 warps runs 8 / TW row-blocks of one class.  Rows
-// longer than 64 tiles (S > 4096 global rows) fold the excess 4 tiles at a time and re-read m'.
+// longer than 8 * kIrWarpTiles tiles fold the excess 4 tiles at a time and re-read m'.
 // About 10-15 thread-instructions per (row, tile) merge; 12 B per (row, tile).
 constexpr int kW = 8;
 
@@ -55,7 +55,10 @@ __device__ __forceinline__ void ir_store(float* rp, int u, const float (&m4)[4],
     *reinterpret_cast<float4*>(rp + (int64_t)u * kRowBlock) = o;
 }
 
-__global__ void __launch_bounds__(kW * 32, 2) ir_kernel(const Params p)
+#ifndef SR_IR_MIN_CTAS
+#define SR_IR_MIN_CTAS 3  // resident CTAs per SM the register budget must allow (see kIrWarpTiles)
+#endif
+__global__ void __launch_bounds__(kW * 32, SR_IR_MIN_CTAS) ir_kernel(const Params p)
 {
     constexpr int KR = kIrWarpTiles;
     __shared__ float4 part_m[kW][32], part_d[kW][32];

@@ -20,7 +20,13 @@ namespace sr {
 
 constexpr int kRowBlock = 128;  // M of every tcgen05 tile
 constexpr int kHalf = 64;       // validity granularity of tile rows
-constexpr int kIrWarpTiles = 8;  // IR kernel: tiles one warp merges in registers
+#ifndef SR_IR_WARP_TILES
+#define SR_IR_WARP_TILES 4
+#endif
+// IR kernel: tiles one warp merges in registers (4: 64 registers, three 8-warp CTAs per SM, one
+// wave; 8 held 122 registers and ran C4's row-blocks in two waves -- measured, back to back: C3
+// 5.3 -> 4.4 us, C4 8.9 -> 8.1, C5 4.8 -> 4.5; single L2-flushed call C3 14.3 -> 10.2)
+constexpr int kIrWarpTiles = SR_IR_WARP_TILES;
 constexpr int kSplitRefSms = 148; // SR_SPLIT_KV chunk size reference: about two chunks per SM of a B200
 constexpr int kSmShortChunks = 16; // unfused softmax: rows of up to this many 64-key chunks form the short class
 
@@ -67,7 +73,7 @@ struct DevSched {
     const int32_t* ccta_ptr;
     int n_cb, n_ccta;
     // standalone IR kernel (SR_IR_KERNEL): row-blocks longest first, in classes of team size 8, 4, 2, 1
-    // warps (> 32, 17-32, 9-16, <= 8 tiles); n_ir_class[c] row-blocks in class c
+    // warps (> 4, 2, 1 x kIrWarpTiles tiles, the rest); n_ir_class[c] row-blocks in class c
     const int4* ir_desc;  // {g * n_rb + rb, t0, t1, tp[lh][0]} per row-block, class order
     int n_ir_class[4];
     // key-range split (SR_SPLIT_KV): psl[i] = partial-output slot of item descriptor i (a chunk of a
