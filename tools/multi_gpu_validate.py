@@ -28,8 +28,16 @@ def main():
     a = ap.parse_args()
     rank, world = int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1))
     lr = int(os.environ.get("LOCAL_RANK", 0))
+    # SR_BENCH_SHARED_GPU=1: every rank on cuda:0 and the gather over gloo on host copies (a functional
+    # check of the sharded layer's assembly on a one-GPU box)
+    shared = os.environ.get("SR_BENCH_SHARED_GPU") == "1"
+    if shared:
+        lr = 0
     torch.cuda.set_device(lr)
-    dist.init_process_group("nccl", device_id=torch.device("cuda", lr))
+    if shared:
+        dist.init_process_group("gloo")
+    else:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", lr))
     cfg = W.config(a.config)
     t = W.config_tensors(cfg)
     lay = W.config_layout(cfg)
@@ -52,14 +60,20 @@ def main():
     else:
         o = sr.mha_sliding_window(q, k, v, cfg.window, cfg.n_global, **kw)
     # gather variable-size shards: pad to the largest, all_gather_into_tensor, trim on rank 0
-    n = torch.tensor([sh.n], device="cuda")
+    cdev = "cpu" if shared else "cuda"
+    n = torch.tensor([sh.n], device=cdev)
     ns = [torch.zeros_like(n) for _ in range(world)]
     dist.all_gather(ns, n)
     n_max = int(max(x.item() for x in ns))
-    buf = torch.zeros(n_max, cfg.S, cfg.D, device="cuda")
-    buf[:sh.n] = o.reshape(sh.n, cfg.S, cfg.D)
-    allb = torch.empty(world * n_max, cfg.S, cfg.D, device="cuda")
-    dist.all_gather_into_tensor(allb, buf)
+    buf = torch.zeros(n_max, cfg.S, cfg.D, device=cdev)
+    buf[:sh.n] = o.reshape(sh.n, cfg.S, cfg.D).to(cdev)
+    if shared:
+        parts = [torch.empty_like(buf) for _ in range(world)]
+        dist.all_gather(parts, buf)
+        allb = torch.cat(parts).cuda()
+    else:
+        allb = torch.empty(world * n_max, cfg.S, cfg.D, device="cuda")
+        dist.all_gather_into_tensor(allb, buf)
     if rank == 0:
         full = torch.cat([allb[r * n_max:r * n_max + int(ns[r].item())] for r in range(world)]).reshape(-1, cfg.D)
         rng = np.random.Generator(np.random.PCG64(0))
