@@ -915,14 +915,9 @@ sr_status run(sr_entry e, int fused, const void* q, const void* k, const void* v
             one = false;
         }
     }
-    // concurrent GEMM1 / GEMM2 kernel (k_conc.cu): D = 128 one-launch layers (SR_CONC=1 selects it;
-    // experiment switch while it is being measured)
-    bool conc = conc_req;
-    {
-        static const int env_conc = [] { const char* e = getenv("SR_CONC"); return e ? atoi(e) : 0; }();
-        conc = conc || (env_conc == 1 && one && !split && fused == 1 &&
-                        !(ex->flags & (variant_bits | SR_RUN_GEMM1 | SR_RUN_REDUCE | SR_RUN_GEMM2)));
-    }
+    // the concurrent GEMM1 / GEMM2 kernel (k_conc.cu) runs only when asked for (SR_CONCURRENT):
+    // measured slower than the one-launch default on every config
+    const bool conc = conc_req;
     std::shared_ptr<DevBlob> db = device_blob(*cs, n_sm, split);
     void* region = (char*)ex->workspace + wi.off_sched;
 
