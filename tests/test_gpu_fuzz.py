@@ -84,3 +84,22 @@ def test_fuzz_backward(i):
     kind, B, H, S, D, dtype, kw, _path, grads_f32 = draw(10_000 + i)
     got, ref = run_bwd(kind, B, H, S, D, dtype, seed=200 + i, grads_f32=grads_f32, **kw)
     check(got, ref, dtype, grads_f32=grads_f32, what=f"bwd case {i}: {kind} B{B} H{H} S{S} D{D} {dtype} {kw.get('causal')}")
+
+
+N_F32 = 24
+
+
+@pytest.mark.parametrize("i", range(N_F32))
+def test_fuzz_fp32(i):
+    """The fp32 mode (SIMT chain, BASELINE config 1's tolerance 1e-5) on seeded random requests."""
+    kind, B, H, S, D, _dtype, kw, _path, _ = draw(20_000 + i)
+    t, q, k, v = qkv(B, H, S, D, "f32", seed=300 + i)
+    scale = 1 / math.sqrt(D)
+    mask = {"dense": lambda: sr.dense_mask(kw.get("kv_len")), "block": lambda: sr.block_mask(kw["layout"]),
+            "window": lambda: sr.window_mask(kw["window"], kw["n_global"])}[kind]()
+    o = sr.call(mask, q, k, v, scale=scale, causal=kw["causal"])
+    torch.cuda.synchronize()
+    ref = oracle.attention(t.q64, t.k64, t.v64, scale,
+                           oracle_mask(kind, kw.get("kv_len"), kw["causal"], kw.get("layout"), kw.get("window", 0),
+                                       kw.get("n_global", 0)))
+    assert_close(o.double().cpu().numpy(), ref, "f32", what=f"fp32 case {i}: {kind} B{B} H{H} S{S} D{D}")
