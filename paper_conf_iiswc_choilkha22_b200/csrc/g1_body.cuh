@@ -203,10 +203,10 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
             // Q of row-blocks 2j and 2j+1 per item, then one K stage per union macro tile
             int qi = 0, ks = 0;
             uint32_t qph = 0, kph = 0;
-            int4 nd = it_begin < it_end ? __ldg(sc.pair_desc + p1at(it_begin)) : make_int4(0, 0, 0, 0);
+            int4 nd = it_begin < it_end ? __ldca(sc.pair_desc + p1at(it_begin)) : make_int4(0, 0, 0, 0);
             for (int it = it_begin; it < it_end; ++it) {
                 const int4 d = nd;
-                if (it + 1 < it_end) nd = __ldg(sc.pair_desc + p1at(it + 1));
+                if (it + 1 < it_end) nd = __ldca(sc.pair_desc + p1at(it + 1));
                 const int g = d.x / sc.n_pair, j = d.x % sc.n_pair, e0 = d.y, e1 = d.z;
                 if (e0 == e1) continue;
                 const int nrb = 2 * j + 1 < sc.n_rb ? 2 : 1;
@@ -230,14 +230,14 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
                 if (++qi == C::NQ) { qi = 0; qph ^= 1; }
                 int wn[NSUB];
 #pragma unroll
-                for (int s2 = 0; s2 < NSUB; ++s2) wn[s2] = e0 + s2 < e1 ? __ldg(&sc.pent[e0 + s2].x) : 0;
+                for (int s2 = 0; s2 < NSUB; ++s2) wn[s2] = e0 + s2 < e1 ? __ldca(&sc.pent[e0 + s2].x) : 0;
                 for (int e = e0; e < e1; e += NSUB) {
                     const int nsub = min(NSUB, e1 - e);
                     int w[NSUB];
 #pragma unroll
                     for (int s2 = 0; s2 < NSUB; ++s2) {
                         w[s2] = wn[s2];
-                        wn[s2] = e + NSUB + s2 < e1 ? __ldg(&sc.pent[e + NSUB + s2].x) : 0;
+                        wn[s2] = e + NSUB + s2 < e1 ? __ldca(&sc.pent[e + NSUB + s2].x) : 0;
                     }
                     DW_WAIT(&k_empty[ks], kph ^ 1, 1);
                     if (elect_one()) {
@@ -258,27 +258,27 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
             const uint32_t idesc = idesc_f16(p.in_dtype == DT_BF16 ? 1 : 0, kRowBlock, C::MW, 0, 0);
             int qi = 0, ks = 0, n = 0;
             uint32_t qph = 0, kph = 0;
-            int4 nd = it_begin < it_end ? __ldg(sc.pair_desc + p1at(it_begin)) : make_int4(0, 0, 0, 0);
+            int4 nd = it_begin < it_end ? __ldca(sc.pair_desc + p1at(it_begin)) : make_int4(0, 0, 0, 0);
             for (int it = it_begin; it < it_end; ++it) {
                 const int4 d = nd;
-                if (it + 1 < it_end) nd = __ldg(sc.pair_desc + p1at(it + 1));
+                if (it + 1 < it_end) nd = __ldca(sc.pair_desc + p1at(it + 1));
                 const int g = d.x / sc.n_pair, j = d.x % sc.n_pair, e0 = d.y, e1 = d.z;
                 if (e0 == e1) continue;
                 const int nrb = 2 * j + 1 < sc.n_rb ? 2 : 1;
-                const int kvl = sc.kv_len ? __ldg(sc.kv_len + g / p.H) : p.S;
+                const int kvl = sc.kv_len ? __ldca(sc.kv_len + g / p.H) : p.S;
                 const int64_t slot0 = (int64_t)g * sc.slots_per_head - d.w;
                 DW_WAIT(&q_full[qi], qph, 0);
                 tc_fence_after();
                 const uint32_t q_addr = smem_u32(smem + C::OFF_Q + qi * C::QS);
                 int4 wn[NSUB];
 #pragma unroll
-                for (int s2 = 0; s2 < NSUB; ++s2) wn[s2] = e0 + s2 < e1 ? __ldg(sc.pent + e0 + s2) : make_int4(0, -1, -1, 0);
+                for (int s2 = 0; s2 < NSUB; ++s2) wn[s2] = e0 + s2 < e1 ? __ldca(sc.pent + e0 + s2) : make_int4(0, -1, -1, 0);
                 for (int e = e0; e < e1; e += NSUB) {
                     int4 w[NSUB];
 #pragma unroll
                     for (int s2 = 0; s2 < NSUB; ++s2) {
                         w[s2] = wn[s2];
-                        wn[s2] = e + NSUB + s2 < e1 ? __ldg(sc.pent + e + NSUB + s2) : make_int4(0, -1, -1, 0);
+                        wn[s2] = e + NSUB + s2 < e1 ? __ldca(sc.pent + e + NSUB + s2) : make_int4(0, -1, -1, 0);
                     }
                     DW_WAIT(&k_full[ks], kph, 1);
                     tc_fence_after();
@@ -359,14 +359,14 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
                 if (++qi == C::NQ) { qi = 0; qph ^= 1; }
                 int wn[NSUB];  // schedule words of the next macro tile, prefetched one step ahead
 #pragma unroll
-                for (int s = 0; s < NSUB; ++s) wn[s] = I.t0 + s < I.t1 ? __ldg(sc.tinfo + I.t0 + s) : 0;
+                for (int s = 0; s < NSUB; ++s) wn[s] = I.t0 + s < I.t1 ? __ldca(sc.tinfo + I.t0 + s) : 0;
                 for (int t = I.t0; t < I.t1; t += NSUB) {
                     const int nsub = min(NSUB, I.t1 - t);
                     int w[NSUB];
 #pragma unroll
                     for (int s = 0; s < NSUB; ++s) {
                         w[s] = wn[s];
-                        wn[s] = t + NSUB + s < I.t1 ? __ldg(sc.tinfo + t + NSUB + s) : 0;
+                        wn[s] = t + NSUB + s < I.t1 ? __ldca(sc.tinfo + t + NSUB + s) : 0;
                     }
                     DW_WAIT(&k_empty[ks], kph ^ 1, 1);
                     if (elect_one()) {
@@ -415,15 +415,15 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
                     if constexpr (CONC) post_marks(2, kord);
                     continue;
                 }
-                const int kvl = sc.kv_len ? __ldg(sc.kv_len + I.g / p.H) : p.S;
+                const int kvl = sc.kv_len ? __ldca(sc.kv_len + I.g / p.H) : p.S;
                 DW_WAIT(&q_full[qi], qph, 0);
                 tc_fence_after();
                 const uint32_t q_addr = smem_u32(smem + C::OFF_Q + qi * C::QB);
-                int wn0 = __ldg(sc.tinfo + I.t0), wn1 = (NSUB > 1 && I.t0 + 1 < I.t1) ? __ldg(sc.tinfo + I.t0 + 1) : -1;
+                int wn0 = __ldca(sc.tinfo + I.t0), wn1 = (NSUB > 1 && I.t0 + 1 < I.t1) ? __ldca(sc.tinfo + I.t0 + 1) : -1;
                 for (int t = I.t0; t < I.t1; t += NSUB, ++n) {
                     const int w0 = wn0, w1 = NSUB > 1 ? wn1 : -1;
-                    if (t + NSUB < I.t1) wn0 = __ldg(sc.tinfo + t + NSUB);  // prefetch the next macro tile
-                    wn1 = (NSUB > 1 && t + NSUB + 1 < I.t1) ? __ldg(sc.tinfo + t + NSUB + 1) : -1;
+                    if (t + NSUB < I.t1) wn0 = __ldca(sc.tinfo + t + NSUB);  // prefetch the next macro tile
+                    wn1 = (NSUB > 1 && t + NSUB + 1 < I.t1) ? __ldca(sc.tinfo + t + NSUB + 1) : -1;
                     const int ab = n % C::NACC;
                     DW_WAIT(&acc_empty[ab], ((n / C::NACC) & 1) ^ 1, 2);
                     const int64_t slot = I.slot0 + t;
@@ -535,10 +535,10 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
                 }
             };
             if (PAIR) {
-                int4 nd = it_begin < it_end ? __ldg(sc.pair_desc + p1at(it_begin)) : make_int4(0, 0, 0, 0);
+                int4 nd = it_begin < it_end ? __ldca(sc.pair_desc + p1at(it_begin)) : make_int4(0, 0, 0, 0);
                 for (int it = it_begin; it < it_end; ++it) {
                     const int4 dd = nd;
-                    if (it + 1 < it_end) nd = __ldg(sc.pair_desc + p1at(it + 1));
+                    if (it + 1 < it_end) nd = __ldca(sc.pair_desc + p1at(it + 1));
                     const int g = dd.x / sc.n_pair, j = dd.x % sc.n_pair, e0 = dd.y, e1 = dd.z;
                     if (e0 == e1) continue;
                     const int nrb = 2 * j + 1 < sc.n_rb ? 2 : 1;
@@ -549,7 +549,7 @@ __device__ __forceinline__ void g1_roles(const CUtensorMap& tmQ, const CUtensorM
                         int hb = 0;  // union of the sub-tiles' half bits: bits 0-1 row-block 0, 2-3 row-block 1
 #pragma unroll
                         for (int s2 = 0; s2 < NSUB; ++s2)
-                            if (e + s2 < e1) hb |= (__ldg(&sc.pent[e + s2].x) >> 16) & 15;
+                            if (e + s2 < e1) hb |= (__ldca(&sc.pent[e + s2].x) >> 16) & 15;
                         if (hb & 3) merge(m0, d0);
                         if (nrb == 2 && (hb & 12)) merge(m1, d1);
                     }

@@ -226,11 +226,11 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                     continue;
                 }
                 int wn[2];  // schedule words of the next macro tile, prefetched one step ahead
-                for (int u = 0; u < NSUB; ++u) wn[u] = I.t0 + u < I.t1 ? __ldg(sc.tinfo + I.t0 + u) : 0;
+                for (int u = 0; u < NSUB; ++u) wn[u] = I.t0 + u < I.t1 ? __ldca(sc.tinfo + I.t0 + u) : 0;
                 for (int t = I.t0; t < I.t1; t += NSUB) {
                     const int nsub = min(NSUB, I.t1 - t);
                     int hv[2] = {tinfo_half(wn[0]), NSUB > 1 ? tinfo_half(wn[1]) : 0};
-                    for (int u = 0; u < NSUB; ++u) wn[u] = t + NSUB + u < I.t1 ? __ldg(sc.tinfo + t + NSUB + u) : 0;
+                    for (int u = 0; u < NSUB; ++u) wn[u] = t + NSUB + u < I.t1 ? __ldca(sc.tinfo + t + NSUB + u) : 0;
                     uint32_t bytes = GS ? nsub * kRowBlock * 4 : 0;
 #ifndef SR_DIAG2_NOX
                     for (int u = 0; u < nsub; ++u) bytes += ((GS && !AS) ? (hv[u] == 3 ? 2 : 1) : 2) * (T / 64) * (kHalf * 128);
@@ -335,14 +335,14 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                     float m8[4][8], d8[4][8];
                     int w8[8];
 #pragma unroll
-                    for (int u = 0; u < 8; ++u) w8[u] = tb + u < I.t1 ? __ldg(sc.tinfo + tb + u) : 0;
+                    for (int u = 0; u < 8; ++u) w8[u] = tb + u < I.t1 ? __ldca(sc.tinfo + tb + u) : 0;
 #pragma unroll
                     for (int u = 0; u < 8; ++u)
 #pragma unroll
                         for (int j = 0; j < 4; ++j) {
                             const bool in = tb + u < I.t1;
-                            m8[j][u] = in ? __ldg(mp + (int64_t)(tb + u) * kRowBlock + 32 * j) : -INFINITY;
-                            d8[j][u] = in ? __ldg(dp + (int64_t)(tb + u) * kRowBlock + 32 * j) : 0.f;
+                            m8[j][u] = in ? __ldca(mp + (int64_t)(tb + u) * kRowBlock + 32 * j) : -INFINITY;
+                            d8[j][u] = in ? __ldca(dp + (int64_t)(tb + u) * kRowBlock + 32 * j) : 0.f;
                         }
 #pragma unroll
                     for (int j = 0; j < 4; ++j) {
@@ -383,11 +383,11 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
             for (ItemWalk iw(sc, it_begin, it_end, p.p2_reverse); iw.more();) {
                 const ItemInfo I = iw.next();
                 int wn[2];  // schedule words of the next macro tile, prefetched one step ahead
-                for (int u = 0; u < NSUB; ++u) wn[u] = I.t0 + u < I.t1 ? __ldg(sc.tinfo + I.t0 + u) : 0;
+                for (int u = 0; u < NSUB; ++u) wn[u] = I.t0 + u < I.t1 ? __ldca(sc.tinfo + I.t0 + u) : 0;
                 for (int t = I.t0; t < I.t1; t += NSUB) {
                     const int nsub = min(NSUB, I.t1 - t);
                     int kt[2] = {tinfo_kt(wn[0]), NSUB > 1 ? tinfo_kt(wn[1]) : 0};
-                    for (int u = 0; u < NSUB; ++u) wn[u] = t + NSUB + u < I.t1 ? __ldg(sc.tinfo + t + NSUB + u) : 0;
+                    for (int u = 0; u < NSUB; ++u) wn[u] = t + NSUB + u < I.t1 ? __ldca(sc.tinfo + t + NSUB + u) : 0;
                     DW_WAIT(&v_empty[s], sph ^ 1, 0);
                     if (elect_one()) {
 #ifdef SR_DIAG2_NOV
@@ -409,7 +409,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                             const int tp = t + C::NV * NSUB;
                             for (int u = 0; u < NSUB; ++u)
                                 if (tp + u < I.t1) {
-                                    const int ktp = tinfo_kt(__ldg(sc.tinfo + tp + u));
+                                    const int ktp = tinfo_kt(__ldca(sc.tinfo + tp + u));
                                     for (int h = 0; h < D / 64; ++h) tma_prefetch_2d(&tmV, h * 64, I.g * p.S + ktp * T);
                                 }
                         }
@@ -572,7 +572,7 @@ __device__ __forceinline__ void g2_roles(const CUtensorMap& tmV, const Params& p
                 const ItemInfo I = nxt;
                 if (it + 1 < it_end) nxt = decode_item(sc, at(it + 1));  // prefetch
                 // a chunk of a split row-block (SR_SPLIT_KV) writes fp32 partial rows to its slot
-                const int ps = (!AS && p.partial) ? __ldg(sc.psl + at(it)) : -1;
+                const int ps = (!AS && p.partial) ? __ldca(sc.psl + at(it)) : -1;
                 const int64_t orow = ps >= 0 ? (int64_t)ps * kRowBlock : (int64_t)I.g * p.S + I.rb * kRowBlock;
                 const int nv = ps >= 0 ? kRowBlock : rows_in_head(p, I.rb);  // a partial slot holds all 128
                 if (I.t0 == I.t1) {  // no kept key in these rows: the epilogue writes zeros

@@ -76,18 +76,18 @@ __global__ void __launch_bounds__(kPrepThreads) bwd_prep(const Params p)
         float4 o32[EPT / 4];
 #pragma unroll
         for (int k = 0; k < EPT / 8; ++k)  // chunk c + k * TPR of the row: coalesced across the row's threads
-            g[k] = __ldg(reinterpret_cast<const uint4*>((const uint16_t*)p.dout + row * D) + c + k * TPR);
+            g[k] = __ldcg(reinterpret_cast<const uint4*>((const uint16_t*)p.dout + row * D) + c + k * TPR);
         if (p.out_dtype == DT_F32) {
 #pragma unroll
             for (int k = 0; k < EPT / 8; ++k) {
                 const float4* o4 = reinterpret_cast<const float4*>((const float*)p.out + row * D) + 2 * (c + k * TPR);
-                o32[2 * k] = __ldg(o4);
-                o32[2 * k + 1] = __ldg(o4 + 1);
+                o32[2 * k] = __ldcg(o4);
+                o32[2 * k + 1] = __ldcg(o4 + 1);
             }
         } else {
 #pragma unroll
             for (int k = 0; k < EPT / 8; ++k)
-                o16[k] = __ldg(reinterpret_cast<const uint4*>((const uint16_t*)p.out + row * D) + c + k * TPR);
+                o16[k] = __ldcg(reinterpret_cast<const uint4*>((const uint16_t*)p.out + row * D) + c + k * TPR);
         }
 #pragma unroll
         for (int k = 0; k < EPT / 8; ++k) {
@@ -128,7 +128,7 @@ __global__ void __launch_bounds__(kPrepThreads) bwd_prep(const Params p)
         if (p.bwd_dq_fused) {  // dQ of a row-block with no listed tile is 0 (the dS' kernel never visits it)
             const int g = (int)(r / p.S), rb = (int)((r % p.S) / kRowBlock);
             const int32_t* tp = p.sc.tp + (size_t)lh_of(p.sc, g, p.H) * (p.sc.n_rb + 1);
-            if (__ldg(tp + rb + 1) == __ldg(tp + rb)) {
+            if (__ldcg(tp + rb + 1) == __ldcg(tp + rb)) {
                 if (p.out_dtype == DT_F32) {
                     float4* O = reinterpret_cast<float4*>((float*)p.dq + r * D);
                     for (int c = 0; c < D / 4; ++c) O[c] = make_float4(0.f, 0.f, 0.f, 0.f);
@@ -233,7 +233,7 @@ __global__ void __launch_bounds__(384, 1)
     const uint32_t tmem_base = *tmem_ptr;
     griddep_launch_dependents();
     griddep_wait();
-    const int it_begin = __ldg(p.sc.cta_ptr + blockIdx.x), it_end = __ldg(p.sc.cta_ptr + blockIdx.x + 1);
+    const int it_begin = __ldcg(p.sc.cta_ptr + blockIdx.x), it_end = __ldcg(p.sc.cta_ptr + blockIdx.x + 1);
 
     if (warp < 4) {
         reg_dealloc<56>();  // 4 warps x 32 x (168 - 56) = 8 warps x 32 x (224 - 168)
@@ -258,7 +258,7 @@ __global__ void __launch_bounds__(384, 1)
                     const int nsub = min(NSUB, I.t1 - t);
                     int w[NSUB];
 #pragma unroll
-                    for (int s = 0; s < NSUB; ++s) w[s] = s < nsub ? __ldg(p.sc.tinfo + t + s) : 0;
+                    for (int s = 0; s < NSUB; ++s) w[s] = s < nsub ? __ldcg(p.sc.tinfo + t + s) : 0;
                     mbar_wait(&k_empty[ks], kph ^ 1);
                     if (elect_one()) {
                         mbar_arrive_expect_tx(&k_full[ks], nsub * T * D * 2);
@@ -282,7 +282,7 @@ __global__ void __launch_bounds__(384, 1)
                     const int nsub = min(NSUB, I.t1 - t);
                     int w[NSUB];
 #pragma unroll
-                    for (int s = 0; s < NSUB; ++s) w[s] = s < nsub ? __ldg(p.sc.tinfo + t + s) : 0;
+                    for (int s = 0; s < NSUB; ++s) w[s] = s < nsub ? __ldcg(p.sc.tinfo + t + s) : 0;
                     mbar_wait(&kq_empty[ks], kph ^ 1);
                     if (elect_one()) {
                         mbar_arrive_expect_tx(&kq_full[ks], nsub * T * D * 2);
@@ -308,7 +308,7 @@ __global__ void __launch_bounds__(384, 1)
                     uint32_t bytes = 0;
 #pragma unroll
                     for (int u = 0; u < NSUB; ++u) {
-                        hv[u] = u < nsub ? tinfo_half(__ldg(p.sc.tinfo + t + u)) : 0;
+                        hv[u] = u < nsub ? tinfo_half(__ldcg(p.sc.tinfo + t + u)) : 0;
                         if (u < nsub) bytes += (hv[u] == 3 ? 2 : 1) * (T / 64) * (kHalf * 128) + kRowBlock * 4;
                     }
                     const int xs = (n % 2) * C::NXW + (n / 2) % C::NXW;
@@ -383,8 +383,8 @@ __global__ void __launch_bounds__(384, 1)
                 const uint32_t q_addr = smem_u32(smem + C::OFF_Q + qi * C::QB);
                 ++nitem;
                 for (int t = I.t0; t < I.t1; t += NSUB, ++n) {
-                    const int w0 = __ldg(p.sc.tinfo + t);
-                    const int w1 = (NSUB > 1 && t + 1 < I.t1) ? __ldg(p.sc.tinfo + t + 1) : -1;
+                    const int w0 = __ldcg(p.sc.tinfo + t);
+                    const int w1 = (NSUB > 1 && t + 1 < I.t1) ? __ldcg(p.sc.tinfo + t + 1) : -1;
                     const int ab = n % C::NACC;
                     mbar_wait(&acc_empty[ab], ((n / C::NACC) & 1) ^ 1);
                     const int64_t slot = I.slot0 + t;
@@ -470,9 +470,9 @@ __global__ void __launch_bounds__(384, 1)
             if (row0 != cur) {  // a new row-block: this row's m, 1/d, delta (bstat rows per head in whole
                 cur = row0;     // row-blocks, p.Spad)
                 const int64_t prow = (row0 / p.S) * p.Spad + row0 % p.S + r;
-                m_row = __ldg(p.bstat + prow);
-                invd_row = __ldg(p.bstat + nrow + prow);
-                delta_row = __ldg(p.bstat + 2 * nrow + prow);
+                m_row = __ldcg(p.bstat + prow);
+                invd_row = __ldcg(p.bstat + nrow + prow);
+                delta_row = __ldcg(p.bstat + 2 * nrow + prow);
             }
             uint32_t xr[kMWB];  // dP of this row, fp32
             if (any) {
@@ -653,7 +653,7 @@ __global__ void __launch_bounds__(384, 1)
     const uint32_t tmem_base = *tmem_ptr;
     griddep_launch_dependents();
     griddep_wait();
-    const int it_begin = __ldg(p.sc.ccta_ptr + cta), it_end = __ldg(p.sc.ccta_ptr + cta + 1);
+    const int it_begin = __ldcg(p.sc.ccta_ptr + cta), it_end = __ldcg(p.sc.ccta_ptr + cta + 1);
     const int T = p.T;
     const uint8_t* asrc = (const uint8_t*)(PV ? p.xprime : p.dsbuf);
     const int XS = kRowBlock * T * 2;
@@ -664,11 +664,11 @@ __global__ void __launch_bounds__(384, 1)
         int s = 0;
         uint32_t sph = 0;
         for (int it = it_begin; it < it_end; ++it) {
-            const int4 d = __ldg(p.sc.col_desc + it);
+            const int4 d = __ldcg(p.sc.col_desc + it);
             const int g = d.x / p.sc.n_cb;
             const int64_t slot0 = (int64_t)g * p.sc.slots_per_head - d.w;
             for (int e = d.y; e < d.z; ++e) {
-                const int4 ce = __ldg(p.sc.cent + e);
+                const int4 ce = __ldcg(p.sc.cent + e);
                 const int rb = ce.x & 0xFFFF, ha = (ce.x >> 16) & 3, hb = (ce.x >> 18) & 3;
                 // key chunk ch (64 keys) comes from tile ti[ch], its 64-key column block cc[ch]
                 const int ti[2] = {ce.y, T == 128 ? ce.y : ce.z};
@@ -730,7 +730,7 @@ __global__ void __launch_bounds__(384, 1)
             __syncwarp();
         };
         for (int it = it_begin; it < it_end; ++it) {
-            const int4 d = __ldg(p.sc.col_desc + it);
+            const int4 d = __ldcg(p.sc.col_desc + it);
             const int g = d.x / p.sc.n_cb, c = d.x % p.sc.n_cb;
             const int64_t krow = (int64_t)g * p.S + c * kMWB;
             if (d.y == d.z) {  // no query row reaches these keys: zero gradients

@@ -78,7 +78,7 @@ __global__ void __launch_bounds__(kConcThreads, 1)
     const uint32_t tmem_base = *tmem_ptr;
     griddep_launch_dependents();
     griddep_wait();
-    const int it_begin = __ldg(sc.cta_ptr + blockIdx.x), it_end = __ldg(sc.cta_ptr + blockIdx.x + 1);
+    const int it_begin = __ldca(sc.cta_ptr + blockIdx.x), it_end = __ldca(sc.cta_ptr + blockIdx.x + 1);
     // each role group under its own register budget (setmaxnreg dominates the group's code)
     if (warp < 4) {
         reg_dealloc<48>();

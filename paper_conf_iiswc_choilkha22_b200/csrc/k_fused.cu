@@ -62,7 +62,7 @@ __global__ void __launch_bounds__(640, 1)
 
     // phase 2's row-blocks (with PAIR the host pointed cta_ptr / item_desc at the pair assignment
     // unrolled into row-blocks, so both phases cover the same rows)
-    const int it_begin = __ldg(sc.cta_ptr + blockIdx.x), it_end = __ldg(sc.cta_ptr + blockIdx.x + 1);
+    const int it_begin = __ldca(sc.cta_ptr + blockIdx.x), it_end = __ldca(sc.cta_ptr + blockIdx.x + 1);
     // phase 2 applies Global Scaling accumulator-side for fp16 (X' and V share the MMA type; see
     // g2_body.cuh AS) unless p.gs_prologue; bf16 V needs the prologue form (Y rounded to bf16)
     // (D = 64: the scaling warps hold D/2 fp32 of O each within the 96-register phase-2 budget)
@@ -70,8 +70,8 @@ __global__ void __launch_bounds__(640, 1)
     PH_MARK(1);
     // ---- phase 1: GEMM1 + LS + IR over the CTA's row-blocks (all 20 warps)
     if constexpr (PAIR)
-        g1_roles<D, 64, true, true, true>(tmQ, tmK, p, sc, smem, tmem_base, __ldg(sc.pcta_ptr + blockIdx.x),
-                                          __ldg(sc.pcta_ptr + blockIdx.x + 1));
+        g1_roles<D, 64, true, true, true>(tmQ, tmK, p, sc, smem, tmem_base, __ldca(sc.pcta_ptr + blockIdx.x),
+                                          __ldca(sc.pcta_ptr + blockIdx.x + 1));
     else
         g1_roles<D, 64, true, false, true>(tmQ, tmK, p, sc, smem, tmem_base, it_begin, it_end);
     // back to the launch split (phase 1 leaves warps 0-3 at 64 registers, the epilogue at 104)
@@ -106,7 +106,7 @@ __global__ void __launch_bounds__(640, 1)
         g_diag_phases[blockIdx.x * 8 + 4] = it_end - it_begin;
         unsigned long long nt = 0;  // the CTA's listed tiles and its SM
         for (int it = it_begin; it < it_end; ++it) {
-            const int4 d = __ldg(sc.item_desc + it);
+            const int4 d = __ldca(sc.item_desc + it);
             nt += d.z - d.y;
         }
         unsigned smid;

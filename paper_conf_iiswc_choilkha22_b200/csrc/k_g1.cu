@@ -38,7 +38,7 @@ __global__ void __launch_bounds__(T == 64 ? 640 : 384, 1)
     // this CTA's items (row-blocks, or pairs of row-blocks): a contiguous range of the host's
     // longest-processing-time assignment
     const int32_t* cptr = PAIR ? p.sc.pcta_ptr : p.sc.cta_ptr;
-    g1_roles<D, T, LS, PAIR, IRT>(tmQ, tmK, p, p.sc, smem, tmem_base, __ldg(cptr + blockIdx.x), __ldg(cptr + blockIdx.x + 1));
+    g1_roles<D, T, LS, PAIR, IRT>(tmQ, tmK, p, p.sc, smem, tmem_base, __ldca(cptr + blockIdx.x), __ldca(cptr + blockIdx.x + 1));
     tc_fence_before();
     __syncthreads();
     if (warp == 2) {

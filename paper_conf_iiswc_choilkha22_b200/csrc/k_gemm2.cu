@@ -34,8 +34,8 @@ __global__ void __launch_bounds__(G2<D, T>::THREADS, 1) tc_gemm2(const __grid_co
     // own prologue, then wait for our producer kernel's results before touching them
     griddep_launch_dependents();
     griddep_wait();
-    g2_roles<D, T, GS, FI, RS>(tmV, p, p.sc, smem, tmem_base, __ldg(p.sc.cta_ptr + blockIdx.x),
-                               __ldg(p.sc.cta_ptr + blockIdx.x + 1));
+    g2_roles<D, T, GS, FI, RS>(tmV, p, p.sc, smem, tmem_base, __ldca(p.sc.cta_ptr + blockIdx.x),
+                               __ldca(p.sc.cta_ptr + blockIdx.x + 1));
     tc_fence_before();
     __syncthreads();
     if (warp == 2) {

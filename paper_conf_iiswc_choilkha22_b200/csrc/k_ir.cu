@@ -22,7 +22,7 @@ namespace sr {
 // About 10-15 thread-instructions per (row, tile) merge; 12 B per (row, tile).
 constexpr int kW = 8;
 
-__device__ __forceinline__ float4 ldg4(const float* p) { return __ldg(reinterpret_cast<const float4*>(p)); }
+__device__ __forceinline__ float4 ldg4(const float* p) { return __ldcg(reinterpret_cast<const float4*>(p)); }
 
 // base-2 m' of tile u (pointer offset in tiles) for the thread's 4 rows (-inf on an invalid half:
 // its statistics were never written) and d' (0 there)
@@ -37,7 +37,7 @@ __device__ __forceinline__ void ir_load(const float* mp, const float* dp, const 
         mm = ldg4(mp + (int64_t)u * kRowBlock);
         if (with_d) dd = ldg4(dp + (int64_t)u * kRowBlock);
     }
-    const bool v = in && ((__ldg(ti + u) >> hbit) & 1);
+    const bool v = in && ((__ldcg(ti + u) >> hbit) & 1);
     if (!v) dd = make_float4(0.f, 0.f, 0.f, 0.f);
     m4[0] = v ? mm.x * l2e : -INFINITY; m4[1] = v ? mm.y * l2e : -INFINITY;
     m4[2] = v ? mm.z * l2e : -INFINITY; m4[3] = v ? mm.w * l2e : -INFINITY;
@@ -84,7 +84,7 @@ __global__ void __launch_bounds__(kW * 32, SR_IR_MIN_CTAS) ir_kernel(const Param
     float* rp = nullptr;
     const int32_t* ti = nullptr;
     if (live) {
-        const int4 dsc = __ldg(sc.ir_desc + idx);  // one 16-B load: row-block, its tile range, head base
+        const int4 dsc = __ldcg(sc.ir_desc + idx);  // one 16-B load: row-block, its tile range, head base
         const int g = dsc.x / sc.n_rb, t0 = dsc.y, t1 = dsc.z, base = dsc.w;
         const int64_t s0 = ((int64_t)g * sc.slots_per_head - base + t0 + tmw) * kRowBlock + 4 * lane;
         mp = p.mprime + s0; dp = p.dprime + s0; rp = p.rprime + s0; ti = sc.tinfo + t0 + tmw;
@@ -188,7 +188,7 @@ __global__ void __launch_bounds__(256) combine_kernel(const Params p)
     const int j = (int)(idx / PER);
     if (j >= p.sc.n_comb) return;
     const int e = (int)(idx % PER), r = e / (D / 4), c4 = e % (D / 4);
-    const int4 cb = __ldg(p.sc.comb + j);  // {row-block item, first slot, chunks, 0}
+    const int4 cb = __ldcg(p.sc.comb + j);  // {row-block item, first slot, chunks, 0}
     const int g = cb.x / p.sc.n_rb, rb = cb.x % p.sc.n_rb;
     if (rb * kRowBlock + r >= p.S) return;  // a row beyond the head (S % 128 == 64)
     float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);

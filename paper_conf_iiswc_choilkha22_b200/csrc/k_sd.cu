@@ -27,9 +27,9 @@ __global__ void __launch_bounds__(128) sd_tile_kernel(const Params p)
     const int32_t* tp = sc.tp + (size_t)lh_of(sc, g, p.H) * (sc.n_rb + 1);
     griddep_launch_dependents();
     griddep_wait();
-    const int t = __ldg(tp) + local;
+    const int t = __ldcg(tp) + local;
     // slots past the end of a head's list (lists of different lengths per layout head) are unused
-    const int hb = t < __ldg(tp + sc.n_rb) ? tinfo_half(__ldg(sc.tinfo + t)) : 0;
+    const int hb = t < __ldcg(tp + sc.n_rb) ? tinfo_half(__ldcg(sc.tinfo + t)) : 0;
     if (hb == 0) return;
     // LS: scores S (plain GEMM1 output, in pbuf) -> X' (xprime);  GS: X' -> Y = X' r' (pbuf)
     const uint8_t* src = (const uint8_t*)(LS ? p.pbuf : p.xprime) + slot * (int64_t)XB;
@@ -71,7 +71,7 @@ __global__ void __launch_bounds__(128) sd_tile_kernel(const Params p)
                     p.dprime[slot * kRowBlock + r] = sum;
                 }
             } else {  // GS: element-wise scaling by the row's reconstruction factor
-                const float rr_ = __ldg(p.rprime + slot * kRowBlock + r);
+                const float rr_ = __ldcg(p.rprime + slot * kRowBlock + r);
 #pragma unroll
                 for (int c = 0; c < NP; ++c)
                     sts_u32(base + c * (kRowBlock * 128),

@@ -37,14 +37,14 @@ __global__ void __launch_bounds__(256) row_softmax(const Params p, int R, int ca
     const int32_t* tp = sc.tp + (size_t)lh_of(sc, g, p.H) * (sc.n_rb + 1);
     griddep_launch_dependents();
     griddep_wait();
-    const int t0 = __ldg(tp + rb), t1 = __ldg(tp + rb + 1);
-    const int64_t slot0 = (int64_t)g * sc.slots_per_head - __ldg(tp);
+    const int t0 = __ldcg(tp + rb), t1 = __ldcg(tp + rb + 1);
+    const int64_t slot0 = (int64_t)g * sc.slots_per_head - __ldcg(tp);
     const uint32_t slice = (uint32_t)R * 128;
     // bulk copies of the slice's chunks k0 .. k1-1 (in row order) between HBM and shared memory
     auto copy_chunks = [&](int k0, int k1, bool load) {
         int k = 0;
         for (int t = t0; t < t1 && k < k1; ++t) {
-            if (!((tinfo_half(__ldg(sc.tinfo + t)) >> myhalf) & 1)) continue;
+            if (!((tinfo_half(__ldcg(sc.tinfo + t)) >> myhalf) & 1)) continue;
             const int64_t off = (slot0 + t) * (int64_t)XB + r0 * 128;
             for (int ch = 0; ch < T / 64; ++ch, ++k) {
                 if (k < k0 || k >= k1) continue;
@@ -56,7 +56,7 @@ __global__ void __launch_bounds__(256) row_softmax(const Params p, int R, int ca
     };
     if (threadIdx.x == 0) {
         int n = 0;
-        for (int t = t0; t < t1; ++t) n += ((tinfo_half(__ldg(sc.tinfo + t)) >> myhalf) & 1) ? T / 64 : 0;
+        for (int t = t0; t < t1; ++t) n += ((tinfo_half(__ldcg(sc.tinfo + t)) >> myhalf) & 1) ? T / 64 : 0;
         n_chunks = n;
         mbar_init(&bar, 1);
         fence_mbar_init();
@@ -224,7 +224,7 @@ __global__ void __launch_bounds__(256) row_softmax_reg(const Params p, int lo, i
     // a half's 64 rows over rsplit CTAs (LONG: kHalf / kLongRows): more, smaller CTAs shorten the
     // grid's last partial wave
     const int rs = LONG ? kHalf / kLongRows : rsplit;
-    const int hsel = LONG ? __ldg(sc.sm_long + blockIdx.x / rs) : (int)(blockIdx.x / rs);
+    const int hsel = LONG ? __ldcg(sc.sm_long + blockIdx.x / rs) : (int)(blockIdx.x / rs);
     const int item = hsel >> 1, half = hsel & 1;  // item = g * n_rb + rb
     const int row_lo = (int)(blockIdx.x % rs) * (kHalf / rs);
     const int row_hi = row_lo + kHalf / rs;
@@ -233,13 +233,13 @@ __global__ void __launch_bounds__(256) row_softmax_reg(const Params p, int lo, i
     const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
     griddep_launch_dependents();
     griddep_wait();
-    const int t0 = __ldg(tp + rb), t1 = __ldg(tp + rb + 1);
-    const int64_t slot0 = (int64_t)g * sc.slots_per_head - __ldg(tp);
+    const int t0 = __ldcg(tp + rb), t1 = __ldcg(tp + rb + 1);
+    const int64_t slot0 = (int64_t)g * sc.slots_per_head - __ldcg(tp);
     if (warp == 0) {  // compact the tiles whose `half` is valid (ballot + prefix, 32 at a time)
         int n = 0;
         for (int tb = t0; tb < t1; tb += 32) {
             const int t = tb + lane;
-            const bool v = t < t1 && ((tinfo_half(__ldg(sc.tinfo + t)) >> half) & 1);
+            const bool v = t < t1 && ((tinfo_half(__ldcg(sc.tinfo + t)) >> half) & 1);
             const unsigned m = __ballot_sync(0xffffffffu, v);
             if (v) slot_list[n + __popc(m & ((1u << lane) - 1))] = slot0 + t;
             n += __popc(m);
@@ -266,7 +266,7 @@ __global__ void __launch_bounds__(256) row_softmax_reg(const Params p, int lo, i
                 const int k = 4 * i + sub;
                 x[q][i] = make_uint4(0xFC00FC00u, 0xFC00FC00u, 0xFC00FC00u, 0xFC00FC00u);  // -inf (fp16)
                 if (k < nch)
-                    x[q][i] = __ldg(reinterpret_cast<const uint4*>((const uint8_t*)p.xprime + slot_list[k / CPT] * (int64_t)XB +
+                    x[q][i] = __ldcg(reinterpret_cast<const uint4*>((const uint8_t*)p.xprime + slot_list[k / CPT] * (int64_t)XB +
                                                                    (k % CPT) * (kRowBlock * 128) + base[q]));
             }
         }

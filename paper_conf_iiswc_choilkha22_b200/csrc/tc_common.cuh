@@ -10,6 +10,15 @@
 namespace sr {
 
 constexpr int kSmemMax = 232448;  // 227 KB opt-in dynamic shared memory per CTA on sm_100
+// Loads of anything a kernel of the same stream writes (the per-call schedule, kv_len, S / P / X'
+// read through registers, m' / d' / r', row statistics, out / dO in the backward) are weak loads
+// after griddepcontrol.wait -- __ldca (L1-cached; the GEMM kernels' schedule words) or __ldcg (L2) --
+// never __ldg: every kernel is launched with programmatic dependent launch, so its CTAs may start
+// before the producing kernel has written, and ld.global.nc (the read-only path, outside the memory
+// model's visibility guarantees) then served stale lines even after the wait.  Found by a graph of
+// eight unfused calls with different masks (tests/test_gpu_ownership.py::test_graph_capture_every_path;
+// __ldca keeps the GEMMs' speed, measured: all-__ldcg cost C2 +4 %, C4 +2.5 %).  Bulk / TMA copies
+// read through L2 and need no such care.
 #ifndef SR_CONC_NI
 #define SR_CONC_NI 2
 #endif
@@ -64,7 +73,7 @@ struct ItemInfo {
 
 __device__ __forceinline__ int4 item_desc(const DevSched& sc, int it)
 {
-    return it < 0 ? make_int4(0, 0, 0, 0) : __ldg(sc.item_desc + it);  // precomputed on the host
+    return it < 0 ? make_int4(0, 0, 0, 0) : __ldca(sc.item_desc + it);  // precomputed on the host
 }
 __device__ __forceinline__ ItemInfo item_info(const DevSched& sc, int4 d)
 {

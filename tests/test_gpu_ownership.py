@@ -135,3 +135,34 @@ def test_python_binding_checks_buffers():
         layer.backward(torch.ones_like(q), dq=torch.empty(1, 1, 64, 64, dtype=torch.float16, device="cuda"))
     with pytest.raises(ValueError):
         sr.call_bwd(sr.dense_mask(None), q, k[:, :, :64].contiguous(), v, o, torch.ones_like(q), workspace=layer.ws)
+
+
+PATHS = {"unfused": dict(fused=False), "two_kernels": dict(two_kernels=True), "fuse_ir": dict(fuse_ir=True),
+         "ir_kernel": dict(ir_kernel=True), "sd": dict(sd=True), "gs_prologue": dict(gs_prologue=True),
+         "split_kv": dict(split_kv=True), "concurrent": dict(concurrent=True)}
+
+
+@pytest.mark.parametrize("path", list(PATHS))
+def test_graph_capture_every_path(path):
+    """Every variant path is a self-contained sequence of kernel nodes too: 8 first-seen masks per
+    path captured in one graph (workspace sized for the path), replayed, against the oracle."""
+    kw = PATHS[path]
+    t, q, k, v = qkv(B, H, S, D, "f16", seed=6)
+    kvs = _kv_lists(8, seed=list(PATHS).index(path) + 7)
+    wmode = dict(fused=kw.get("fused", True), sd=kw.get("sd", False))
+    ws = torch.empty(max(sr.workspace_info(sr.dense_mask(kv), B, H, S, D, sr.SR_F16, **wmode)["total_bytes"]
+                         for kv in kvs), dtype=torch.uint8, device="cuda")
+    outs = [torch.empty(B, H, S, D, dtype=torch.float32, device="cuda") for _ in kvs]
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g):
+        for kv, o in zip(kvs, outs):
+            sr.call(sr.dense_mask(kv), q, k, v, out=o, out_dtype=torch.float32, workspace=ws, causal=True, **kw)
+    for o in outs:
+        o.zero_()
+    g.replay()
+    torch.cuda.synchronize()
+    scale = 1 / math.sqrt(D)
+    for kv, o in zip(kvs, outs):
+        ref = oracle.attention(t.q64, t.k64, t.v64, scale, oracle_mask("dense", kv, True))
+        assert np.abs(o.double().cpu().numpy() - ref).max() <= 1e-2, (path, kv)
