@@ -345,6 +345,28 @@ def region(torch, g, K, spin=SPIN_CYCLES, warm=None):
     return a.elapsed_time(b) / K
 
 
+def sustained_regions(torch, g, K, n, preload_s, min_replays=1):
+    """Replays of the K-step graph enqueued for `preload_s` seconds with no synchronisation, then n
+    event-timed regions of one replay each, back to back, one synchronize at the end: the regions run
+    in the power state the preceding load settled into, with no idle gap in which the clock can
+    boost.  Device ms per step of each region."""
+    t_end = time.perf_counter() + preload_s
+    done = 0
+    while done < min_replays or time.perf_counter() < t_end:
+        g.replay()
+        done += 1
+    evs = []
+    for _ in range(n):
+        a = torch.cuda.Event(enable_timing=True)
+        b = torch.cuda.Event(enable_timing=True)
+        a.record()
+        g.replay()
+        b.record()
+        evs.append((a, b))
+    torch.cuda.synchronize()
+    return [a.elapsed_time(b) / K for a, b in evs]
+
+
 def back_to_back(torch, fns, K, W_, reps=3):
     """Warm-up replays covering >= W_ steps, then `reps` timed regions of K steps; per-step ms list."""
     g = steps_graph(torch, fns, K)
@@ -450,19 +472,19 @@ def gpu_arm(args, rank, world, local_rank):
         while time.perf_counter() < t_end:
             g_tp.replay()
     torch.cuda.synchronize()
-    barrier(torch, world)
-    # THE timed region: exactly K steps, right after >= W untimed warm-up steps on the same stream
-    # (a replay of the same K-step graph), barrier + synchronize before the warm-up and after
-    ms_rank = region(torch, g_tp, K, warm=g_tp)
-    barrier(torch, world)
-    extra = []
-    for _ in range(4):
-        barrier(torch, world)
-        extra.append(region(torch, g_tp, K, warm=g_tp))
-    # the one-launch kernel alone (schedule resident: no upload launch), in the same power state,
-    # right after the headline regions: the roofline's kernel duration
+    # the one-launch kernel alone (schedule resident: no upload launch), for the roofline's kernel
+    # duration; its graph is built now, so no capture (and its idle gaps) falls between the timed regions
     g_res = steps_graph(torch, [(lambda x=x: x.run(resident=True)) for x in sets], K) if not f32 else None
-    ms_res = [region(torch, g_res, K, warm=g_res) for _ in range(3)] if g_res is not None else None
+    barrier(torch, world)
+    # THE timed region: exactly K steps, after >= W untimed warm-up steps on the same stream -- 0.3 s of
+    # replays of the same K-step graph enqueued with no synchronisation, so the region starts in the
+    # sustained (power-capped) state instead of on a clock that boosted during an idle gap -- then the
+    # region and 4 more, back to back; barrier + synchronize before the warm-up and after
+    sus = sustained_regions(torch, g_tp, K, 5, 0.3, min_replays=-(-Wm // K))
+    ms_rank, extra = sus[0], sus[1:]
+    barrier(torch, world)
+    # the kernel alone in the same state, right after (0.1 s of its own replays first)
+    ms_res = sustained_regions(torch, g_res, K, 3, 0.1) if g_res is not None else None
     clocks = clk.stop()
     ms_step = dist_max(torch, ms_rank, world)
     step_spread = spread([dist_max(torch, x, world) for x in [ms_rank] + extra])
@@ -649,8 +671,9 @@ def gpu_arm(args, rank, world, local_rank):
         "n_gpus": world, "steps": K, "warmup": Wm,
         "ms_per_step": round(ms_step, 5),
         "timing": f"one region of exactly K={K} back-to-back layer calls (C ABI, captured in one CUDA graph) between "
-                  f"two events, right after max(W={Wm}, K) untimed warm-up steps on the same stream, barrier + "
-                  "synchronize before the warm-up and after the region, max over ranks; "
+                  f"two events, right after >= W={Wm} untimed warm-up steps on the same stream (0.3 s of replays "
+                  "enqueued with no synchronisation: the sustained, power-capped state), barrier + synchronize "
+                  "before the warm-up and after the region, max over ranks; "
                   f"{n_sets} rotating input/workspace sets "
                   f"({rot_bytes / 2**20:.0f} MiB > 2x L2) so no step finds its data in L2; step_ms = spread over "
                   "that region and 4 more",
