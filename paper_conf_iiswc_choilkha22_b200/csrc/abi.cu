@@ -524,12 +524,13 @@ std::shared_ptr<DevBlob> make_blob(const HostSched& h0, int n_sm, bool split)
     put(L.items, h.items);
     put(L.cta, cta_ptr);
     size_t o;
-    o = L.iri;  // the IR kernel's row-block descriptors {item, t0, t1, tp[lh][0]}, before the LPT pass (longest first)
+    o = L.iri;  // the IR kernel's row-block descriptors {first slot, tiles, first tile, item}, before the
+                // LPT pass (longest first); the slot is g * slots_per_head + t0 - tp[lh][0] (no division on the device)
     for (int32_t it : h0.items) {
         const int g = it / h0.n_rb, rb = it % h0.n_rb;
         const int32_t* tp = &h0.tp[(size_t)(h0.lh_mode == LH_ONE ? 0 : (h0.lh_mode == LH_BATCH ? g / h0.H : g % h0.H)) *
                                    (h0.n_rb + 1)];
-        const int32_t dd[4] = {it, tp[rb], tp[rb + 1], tp[0]};
+        const int32_t dd[4] = {(int32_t)((int64_t)g * h0.slots_per_head + tp[rb] - tp[0]), tp[rb + 1] - tp[rb], tp[rb], it};
         std::copy(dd, dd + 4, w.begin() + o);
         o += 4;
     }

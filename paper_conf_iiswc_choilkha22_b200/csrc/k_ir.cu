@@ -16,11 +16,16 @@ namespace sr {
 // (TW = 1, 2, 4 or 8, so that a warp has at most kIrWarpTiles = 4 of its tiles): warp t of the team
 // takes tiles t, t + TW, ..., loads all of them at once (m' and d' in registers: one memory round
 // trip), merges them into a partial (m, d) per row; the team's partials meet in shared memory; each
-// warp then writes r' for its own tiles from the m' it still holds.  Row-blocks come longest first
-// (sc.ir_desc) in classes of equal TW; a CTA of 8 warps runs 8 / TW row-blocks of one class.  Rows
-// longer than 8 * kIrWarpTiles tiles fold the excess 4 tiles at a time and re-read m'.
-// About 10-15 thread-instructions per (row, tile) merge; 12 B per (row, tile).
+// warp then writes r' for its own tiles.  Row-blocks come longest first (sc.ir_desc) in classes of
+// equal TW; a CTA of 8 warps runs 8 / TW row-blocks of one class, and the team size is a template
+// parameter (the class is decoded with shifts; the team loops unroll).  Rows longer than
+// 8 * kIrWarpTiles tiles fold the excess 2 tiles at a time and re-read m'.
+// Exponentials: the merge computes e_k = 2^{m'_k - m_w} against the warp's own maximum m_w and keeps
+// it, so r'_k = e_k * (2^{m_w - m} / d) costs one multiply per (row, tile) instead of a second
+// exponential (the per-row factor is one ex2).  12 B per (row, tile); ncu at C4: 34
+// thread-instructions per (row, tile), down from 46 with runtime team sizes and two exponentials.
 constexpr int kW = 8;
+constexpr int kFold = 2;  // tiles per folding step beyond 8 * kIrWarpTiles (register budget)
 
 __device__ __forceinline__ float4 ldg4(const float* p) { return __ldcg(reinterpret_cast<const float4*>(p)); }
 
@@ -44,100 +49,89 @@ __device__ __forceinline__ void ir_load(const float* mp, const float* dp, const 
     d4[0] = dd.x; d4[1] = dd.y; d4[2] = dd.z; d4[3] = dd.w;
 }
 
-__device__ __forceinline__ void ir_store(float* rp, int u, const float (&m4)[4], const float (&mneg)[4],
-                                         const float (&inv_d)[4])
+// r'_k of tile u = s4 (the thread's 4 rows), 0 for invalid halves and fully masked sub-vectors
+__device__ __forceinline__ void ir_store(float* rp, int u, const float (&s4)[4])
 {
-    float4 o;  // r'_k = 2^{m'_k - m} / d  (0 for invalid halves and fully masked sub-vectors)
-    o.x = ptx::ex2(m4[0] + mneg[0]) * inv_d[0];
-    o.y = ptx::ex2(m4[1] + mneg[1]) * inv_d[1];
-    o.z = ptx::ex2(m4[2] + mneg[2]) * inv_d[2];
-    o.w = ptx::ex2(m4[3] + mneg[3]) * inv_d[3];
-    *reinterpret_cast<float4*>(rp + (int64_t)u * kRowBlock) = o;
+    *reinterpret_cast<float4*>(rp + (int64_t)u * kRowBlock) = make_float4(s4[0], s4[1], s4[2], s4[3]);
 }
 
 #ifndef SR_IR_MIN_CTAS
 #define SR_IR_MIN_CTAS 3  // resident CTAs per SM the register budget must allow (see kIrWarpTiles)
 #endif
-__global__ void __launch_bounds__(kW * 32, SR_IR_MIN_CTAS) ir_kernel(const Params p)
+
+// one team of TW warps per row-block; row-block idx of the class that starts at `first` (nc of them)
+template <int TW>
+__device__ __forceinline__ void ir_team(const Params& p, int idx, bool live, float4 (*part_m)[32], float4 (*part_d)[32])
 {
     constexpr int KR = kIrWarpTiles;
-    __shared__ float4 part_m[kW][32], part_d[kW][32];
-    ptx::griddep_launch_dependents();  // PDL: GEMM2's prologue may start now ...
-    ptx::griddep_wait();               // ... and GEMM1's m', d' must be complete before we read them
     const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+    const int team = warp / TW, tmw = warp % TW;  // team within the CTA, warp within the team
     const DevSched& sc = p.sc;
-    // this CTA's class: team size TW, and the row-block of this warp's team
-    int b = blockIdx.x, first = 0, tw = kW, nc = 0;
-    for (int c = 0; c < 4; ++c, tw >>= 1) {
-        const int per = kW / tw, ncta = (sc.n_ir_class[c] + per - 1) / per;
-        nc = sc.n_ir_class[c];
-        if (b < ncta) break;
-        b -= ncta;
-        first += nc;
-    }
-    if (tw == 0) return;  // (not reached: the grid covers the classes exactly)
-    const int team = warp / tw, tmw = warp % tw;  // team within the CTA, warp within the team
-    const int idx = first + b * (kW / tw) + team;
-    const bool live = idx < first + nc;
     int n = 0;
     const float *mp = nullptr, *dp = nullptr;
     float* rp = nullptr;
     const int32_t* ti = nullptr;
     if (live) {
-        const int4 dsc = __ldcg(sc.ir_desc + idx);  // one 16-B load: row-block, its tile range, head base
-        const int g = dsc.x / sc.n_rb, t0 = dsc.y, t1 = dsc.z, base = dsc.w;
-        const int64_t s0 = ((int64_t)g * sc.slots_per_head - base + t0 + tmw) * kRowBlock + 4 * lane;
-        mp = p.mprime + s0; dp = p.dprime + s0; rp = p.rprime + s0; ti = sc.tinfo + t0 + tmw;
-        n = t1 - t0;
+        const int4 dsc = __ldcg(sc.ir_desc + idx);  // one 16-B load: first slot, tiles, first tile index
+        const int64_t s0 = ((int64_t)dsc.x + tmw) * kRowBlock + 4 * lane;
+        mp = p.mprime + s0; dp = p.dprime + s0; rp = p.rprime + s0; ti = sc.tinfo + dsc.z + tmw;
+        n = dsc.y;
     }
     const int hbit = 16 + (lane >> 4);
-    const int nw = n > tmw ? (n - tmw + tw - 1) / tw : 0;  // tiles of this warp: tmw, tmw + tw, ...
-    float mk[KR][4], dk[KR][4];  // [tile][row]
+    const int nw = n > tmw ? (n - tmw + TW - 1) / TW : 0;  // tiles of this warp: tmw, tmw + TW, ...
+    float mk[KR][4], dk[KR][4];  // [tile][row]; mk becomes e_k = 2^{m'_k - m_w}
 #pragma unroll
-    for (int u = 0; u < KR; ++u) ir_load(mp, dp, ti, hbit, u * tw, u < nw, mk[u], dk[u], true);  // all in flight
-    float m[4], d[4];
+    for (int u = 0; u < KR; ++u) ir_load(mp, dp, ti, hbit, u * TW, u < nw, mk[u], dk[u], true);  // all in flight
+    float m[4], d[4], mw[4];  // running (m, d); mw: the maximum the kept e_k are relative to
 #pragma unroll
     for (int r = 0; r < 4; ++r) {
-        m[r] = -INFINITY;
+        float mx = -INFINITY;
 #pragma unroll
-        for (int u = 0; u < KR; ++u) m[r] = fmaxf(m[r], mk[u][r]);
-        const float ms = m[r] == -INFINITY ? 0.f : m[r];
+        for (int u = 0; u < KR; ++u) mx = fmaxf(mx, mk[u][r]);
+        const float ms = mx == -INFINITY ? 0.f : mx;
         float acc = 0.f;
 #pragma unroll
-        for (int u = 0; u < KR; ++u) acc = fmaf(dk[u][r], ptx::ex2(mk[u][r] - ms), acc);
+        for (int u = 0; u < KR; ++u) {
+            mk[u][r] = ptx::ex2(mk[u][r] - ms);  // 0 for -inf
+            acc = fmaf(dk[u][r], mk[u][r], acc);
+        }
+        m[r] = mx;
+        mw[r] = mx;
         d[r] = acc;
     }
-    for (int tb = KR; tb < nw; tb += 4) {  // rows longer than 8 * kIrWarpTiles tiles
-        float m4[4][4], d4[4][4];
+    for (int tb = KR; tb < nw; tb += kFold) {  // rows longer than 8 * kIrWarpTiles tiles
+        float m4[kFold][4], d4[kFold][4];
 #pragma unroll
-        for (int u = 0; u < 4; ++u) ir_load(mp, dp, ti, hbit, (tb + u) * tw, tb + u < nw, m4[u], d4[u], true);
+        for (int u = 0; u < kFold; ++u) ir_load(mp, dp, ti, hbit, (tb + u) * TW, tb + u < nw, m4[u], d4[u], true);
 #pragma unroll
         for (int r = 0; r < 4; ++r) {
-            const float mn = fmaxf(fmaxf(m[r], fmaxf(m4[0][r], m4[1][r])), fmaxf(m4[2][r], m4[3][r]));
+            const float mn = fmaxf(m[r], fmaxf(m4[0][r], m4[1][r]));
             if (mn == -INFINITY) continue;
             float acc = d[r] * ptx::ex2(m[r] - mn);  // ex2(-inf) = 0 while nothing was seen yet
 #pragma unroll
-            for (int u = 0; u < 4; ++u) acc = fmaf(d4[u][r], ptx::ex2(m4[u][r] - mn), acc);
+            for (int u = 0; u < kFold; ++u) acc = fmaf(d4[u][r], ptx::ex2(m4[u][r] - mn), acc);
             m[r] = mn;
             d[r] = acc;
         }
     }
-    // the team's partial (m, d) of each row: m = max_w m_w, d = sum_w 2^{m_w - m} d_w
+    // the team's (m, d) of each row: m = max_w m_w, d = sum_w 2^{m_w - m} d_w
     float mneg[4], inv_d[4];
-    if (tw > 1) {
+    if constexpr (TW > 1) {
         part_m[warp][lane] = make_float4(m[0], m[1], m[2], m[3]);
         part_d[warp][lane] = make_float4(d[0], d[1], d[2], d[3]);
         __syncthreads();  // the whole CTA is one class: uniform
         float M[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY}, D[4] = {0.f, 0.f, 0.f, 0.f};
-        const int w0 = team * tw;
-        for (int w = w0; w < w0 + tw; ++w) {
-            const float4 pm = part_m[w][lane];
+        const int w0 = team * TW;
+#pragma unroll
+        for (int w = 0; w < TW; ++w) {
+            const float4 pm = part_m[w0 + w][lane];
             M[0] = fmaxf(M[0], pm.x); M[1] = fmaxf(M[1], pm.y); M[2] = fmaxf(M[2], pm.z); M[3] = fmaxf(M[3], pm.w);
         }
 #pragma unroll
         for (int r = 0; r < 4; ++r) mneg[r] = M[r] == -INFINITY ? 0.f : -M[r];
-        for (int w = w0; w < w0 + tw; ++w) {
-            const float4 pm = part_m[w][lane], pd = part_d[w][lane];
+#pragma unroll
+        for (int w = 0; w < TW; ++w) {
+            const float4 pm = part_m[w0 + w][lane], pd = part_d[w0 + w][lane];
             D[0] = fmaf(pd.x, ptx::ex2(pm.x + mneg[0]), D[0]);
             D[1] = fmaf(pd.y, ptx::ex2(pm.y + mneg[1]), D[1]);
             D[2] = fmaf(pd.z, ptx::ex2(pm.z + mneg[2]), D[2]);
@@ -152,16 +146,56 @@ __global__ void __launch_bounds__(kW * 32, SR_IR_MIN_CTAS) ir_kernel(const Param
             inv_d[r] = d[r] > 0.f ? 1.f / d[r] : 0.f;
         }
     }
+    // r'_k = e_k * 2^{m_w - m} / d for the kept tiles (e_k = 0 wherever m'_k = -inf, and a warp that
+    // saw no valid tile has m_w = -inf: factor 0, never inf * 0)
+    float fac[4];
+#pragma unroll
+    for (int r = 0; r < 4; ++r) fac[r] = mw[r] == -INFINITY ? 0.f : ptx::ex2(mw[r] + mneg[r]) * inv_d[r];
 #pragma unroll
     for (int u = 0; u < KR; ++u)
-        if (u < nw) ir_store(rp, u * tw, mk[u], mneg, inv_d);
-    for (int tb = KR; tb < nw; tb += 4) {
-        float m4[4][4], d4[4][4];
+        if (u < nw) {
+            float s4[4];
 #pragma unroll
-        for (int u = 0; u < 4; ++u) ir_load(mp, dp, ti, hbit, (tb + u) * tw, tb + u < nw, m4[u], d4[u], false);
+            for (int r = 0; r < 4; ++r) s4[r] = mk[u][r] * fac[r];
+            ir_store(rp, u * TW, s4);
+        }
+    for (int tb = KR; tb < nw; tb += kFold) {  // the folded tiles: m' re-read, r'_k = 2^{m'_k - m} / d
+        float m4[kFold][4], d4[kFold][4];
 #pragma unroll
-        for (int u = 0; u < 4; ++u)
-            if (tb + u < nw) ir_store(rp, (tb + u) * tw, m4[u], mneg, inv_d);
+        for (int u = 0; u < kFold; ++u) ir_load(mp, dp, ti, hbit, (tb + u) * TW, tb + u < nw, m4[u], d4[u], false);
+#pragma unroll
+        for (int u = 0; u < kFold; ++u)
+            if (tb + u < nw) {
+                float s4[4];
+#pragma unroll
+                for (int r = 0; r < 4; ++r) s4[r] = ptx::ex2(m4[u][r] + mneg[r]) * inv_d[r];
+                ir_store(rp, (tb + u) * TW, s4);
+            }
+    }
+}
+
+__global__ void __launch_bounds__(kW * 32, SR_IR_MIN_CTAS) ir_kernel(const Params p)
+{
+    __shared__ float4 part_m[kW][32], part_d[kW][32];
+    ptx::griddep_launch_dependents();  // PDL: GEMM2's prologue may start now ...
+    ptx::griddep_wait();               // ... and GEMM1's m', d' must be complete before we read them
+    // this CTA's class c (team size 8 >> c, 1 << c row-blocks per CTA) and its first row-block
+    int b = blockIdx.x, first = 0, c = 0;
+    for (; c < 4; ++c) {
+        const int nc = p.sc.n_ir_class[c], ncta = (nc + (1 << c) - 1) >> c;
+        if (b < ncta) break;
+        b -= ncta;
+        first += nc;
+    }
+    if (c == 4) return;  // (not reached: the grid covers the classes exactly)
+    const int team = (threadIdx.x / 32) >> (3 - c);
+    const int idx = first + (b << c) + team;
+    const bool live = idx < first + p.sc.n_ir_class[c];
+    switch (c) {
+        case 0: ir_team<8>(p, idx, live, part_m, part_d); break;
+        case 1: ir_team<4>(p, idx, live, part_m, part_d); break;
+        case 2: ir_team<2>(p, idx, live, part_m, part_d); break;
+        default: ir_team<1>(p, idx, live, part_m, part_d); break;
     }
 }
 

@@ -23,9 +23,9 @@ constexpr int kHalf = 64;       // validity granularity of tile rows
 #ifndef SR_IR_WARP_TILES
 #define SR_IR_WARP_TILES 4
 #endif
-// IR kernel: tiles one warp merges in registers (4: 64 registers, three 8-warp CTAs per SM, one
-// wave; 8 held 122 registers and ran C4's row-blocks in two waves -- measured, back to back: C3
-// 5.3 -> 4.4 us, C4 8.9 -> 8.1, C5 4.8 -> 4.5; single L2-flushed call C3 14.3 -> 10.2)
+// IR kernel: tiles one warp merges in registers (4: 80 registers, three 8-warp CTAs per SM; 8 held
+// 122 registers and ran C4's row-blocks in two waves; a form staging the statistics in shared memory
+// by bulk copies was slower back to back -- measured, profiles/r2_experiments.txt)
 constexpr int kIrWarpTiles = SR_IR_WARP_TILES;
 constexpr int kSplitRefSms = 148; // SR_SPLIT_KV chunk size reference: about two chunks per SM of a B200
 constexpr int kSmShortChunks = 16; // unfused softmax: rows of up to this many 64-key chunks form the short class
@@ -74,7 +74,7 @@ struct DevSched {
     int n_cb, n_ccta;
     // standalone IR kernel (SR_IR_KERNEL): row-blocks longest first, in classes of team size 8, 4, 2, 1
     // warps (> 4, 2, 1 x kIrWarpTiles tiles, the rest); n_ir_class[c] row-blocks in class c
-    const int4* ir_desc;  // {g * n_rb + rb, t0, t1, tp[lh][0]} per row-block, class order
+    const int4* ir_desc;  // {g * slots_per_head + t0 - tp[lh][0], t1 - t0, t0, item} per row-block, class order
     int n_ir_class[4];
     // key-range split (SR_SPLIT_KV): psl[i] = partial-output slot of item descriptor i (a chunk of a
     // split row-block) or -1; comb[j] = {row-block item, first slot, chunks, 0} of split row-block j
