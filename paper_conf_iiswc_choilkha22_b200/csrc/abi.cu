@@ -584,15 +584,26 @@ std::shared_ptr<DevBlob> make_blob(const HostSched& h0, int n_sm, bool split)
     d.n_items = (int)(desc.size() / 4);
     d.n_comb = split ? (int)(h.comb.size() / 4) : 0;
     d.n_sm_long = (int)h.sm_long.size();
-    {   // the IR kernel's team classes over iri (longest first): 8 warps for > 4 * kIrWarpTiles tiles,
-        // then 4, 2, 1 (each warp merges <= kIrWarpTiles tiles in registers)
+    {   // the IR kernel's team classes over iri (longest first): 8 warps for > 4 * KR tiles, then 4, 2,
+        // 1 (each warp merges <= KR tiles in registers); KR = kIrWarpTiles unless its CTAs need more
+        // than one wave on n_sm SMs, then kIrWarpTilesWide
         auto lh_of_g2 = [&](int g) { return h0.lh_mode == LH_ONE ? 0 : (h0.lh_mode == LH_BATCH ? g / h0.H : g % h0.H); };
-        for (int c = 0; c < 4; ++c) d.n_ir_class[c] = 0;
-        for (int32_t it : h0.items) {
-            const int g = it / h0.n_rb, rb = it % h0.n_rb;
-            const int32_t* tp = &h0.tp[(size_t)lh_of_g2(g) * (h0.n_rb + 1)];
-            const int n = tp[rb + 1] - tp[rb];
-            d.n_ir_class[n > 4 * kIrWarpTiles ? 0 : n > 2 * kIrWarpTiles ? 1 : n > kIrWarpTiles ? 2 : 3]++;
+        auto classes = [&](int kr, int (&nc)[4]) {
+            for (int c = 0; c < 4; ++c) nc[c] = 0;
+            for (int32_t it : h0.items) {
+                const int g = it / h0.n_rb, rb = it % h0.n_rb;
+                const int32_t* tp = &h0.tp[(size_t)lh_of_g2(g) * (h0.n_rb + 1)];
+                const int n = tp[rb + 1] - tp[rb];
+                nc[n > 4 * kr ? 0 : n > 2 * kr ? 1 : n > kr ? 2 : 3]++;
+            }
+            int64_t ctas = 0;
+            for (int c = 0; c < 4; ++c) ctas += (nc[c] + (1 << c) - 1) >> c;
+            return ctas;
+        };
+        d.ir_warp_tiles = kIrWarpTiles;
+        if (classes(kIrWarpTiles, d.n_ir_class) > (int64_t)kIrCtasPerSm * n_sm) {
+            d.ir_warp_tiles = kIrWarpTilesWide;
+            classes(kIrWarpTilesWide, d.n_ir_class);
         }
     }
     d.n_cta = (int)cta_ptr.size() - 1;

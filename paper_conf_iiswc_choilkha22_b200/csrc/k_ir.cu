@@ -60,10 +60,9 @@ __device__ __forceinline__ void ir_store(float* rp, int u, const float (&s4)[4])
 #endif
 
 // one team of TW warps per row-block; row-block idx of the class that starts at `first` (nc of them)
-template <int TW>
+template <int TW, int KR>
 __device__ __forceinline__ void ir_team(const Params& p, int idx, bool live, float4 (*part_m)[32], float4 (*part_d)[32])
 {
-    constexpr int KR = kIrWarpTiles;
     const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
     const int team = warp / TW, tmw = warp % TW;  // team within the CTA, warp within the team
     const DevSched& sc = p.sc;
@@ -174,6 +173,7 @@ __device__ __forceinline__ void ir_team(const Params& p, int idx, bool live, flo
     }
 }
 
+template <int KR>
 __global__ void __launch_bounds__(kW * 32, SR_IR_MIN_CTAS) ir_kernel(const Params p)
 {
     __shared__ float4 part_m[kW][32], part_d[kW][32];
@@ -192,10 +192,10 @@ __global__ void __launch_bounds__(kW * 32, SR_IR_MIN_CTAS) ir_kernel(const Param
     const int idx = first + (b << c) + team;
     const bool live = idx < first + p.sc.n_ir_class[c];
     switch (c) {
-        case 0: ir_team<8>(p, idx, live, part_m, part_d); break;
-        case 1: ir_team<4>(p, idx, live, part_m, part_d); break;
-        case 2: ir_team<2>(p, idx, live, part_m, part_d); break;
-        default: ir_team<1>(p, idx, live, part_m, part_d); break;
+        case 0: ir_team<8, KR>(p, idx, live, part_m, part_d); break;
+        case 1: ir_team<4, KR>(p, idx, live, part_m, part_d); break;
+        case 2: ir_team<2, KR>(p, idx, live, part_m, part_d); break;
+        default: ir_team<1, KR>(p, idx, live, part_m, part_d); break;
     }
 }
 
@@ -204,7 +204,10 @@ cudaError_t launch_ir(const Params& p, cudaStream_t st, int64_t* nlaunch)
     int64_t blocks = 0;  // per class c (team size 8 >> c): ceil(rows / (8 / team size)) CTAs
     for (int c = 0; c < 4; ++c) blocks += (p.sc.n_ir_class[c] + (1 << c) - 1) >> c;
     if (blocks == 0) return cudaSuccess;
-    return launch_pdl(ir_kernel, dim3((unsigned)blocks), dim3(kW * 32), 0, st, nlaunch, p);
+    // the classes were cut for ir_warp_tiles tiles per warp on the host (make_blob)
+    if (p.sc.ir_warp_tiles == kIrWarpTilesWide)
+        return launch_pdl(ir_kernel<kIrWarpTilesWide>, dim3((unsigned)blocks), dim3(kW * 32), 0, st, nlaunch, p);
+    return launch_pdl(ir_kernel<kIrWarpTiles>, dim3((unsigned)blocks), dim3(kW * 32), 0, st, nlaunch, p);
 }
 
 // ---------------------------------------------------------------- SR_SPLIT_KV combine

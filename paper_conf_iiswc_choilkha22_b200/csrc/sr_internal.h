@@ -25,7 +25,11 @@ constexpr int kHalf = 64;       // validity granularity of tile rows
 #endif
 // IR kernel: tiles one warp merges in registers (4: 80 registers, three 8-warp CTAs per SM; 8 held
 // 122 registers and ran C4's row-blocks in two waves; a form staging the statistics in shared memory
-// by bulk copies was slower back to back -- measured, profiles/r2_experiments.txt)
+// by bulk copies was slower back to back -- measured, profiles/r2_experiments.txt).  kIrWarpTilesWide
+// (6, still three CTAs per SM) is taken when the 4-tile classes would need more than one wave of
+// CTAs: fewer, wider teams then run in one wave (C4 6.76 -> 6.14 us back to back).
+constexpr int kIrWarpTilesWide = 6;
+constexpr int kIrCtasPerSm = 3;
 constexpr int kIrWarpTiles = SR_IR_WARP_TILES;
 constexpr int kSplitRefSms = 148; // SR_SPLIT_KV chunk size reference: about two chunks per SM of a B200
 constexpr int kSmShortChunks = 16; // unfused softmax: rows of up to this many 64-key chunks form the short class
@@ -73,9 +77,10 @@ struct DevSched {
     const int32_t* ccta_ptr;
     int n_cb, n_ccta;
     // standalone IR kernel (SR_IR_KERNEL): row-blocks longest first, in classes of team size 8, 4, 2, 1
-    // warps (> 4, 2, 1 x kIrWarpTiles tiles, the rest); n_ir_class[c] row-blocks in class c
+    // warps (> 4, 2, 1 x ir_warp_tiles tiles, the rest); n_ir_class[c] row-blocks in class c
     const int4* ir_desc;  // {g * slots_per_head + t0 - tp[lh][0], t1 - t0, t0, item} per row-block, class order
     int n_ir_class[4];
+    int ir_warp_tiles;  // kIrWarpTiles or kIrWarpTilesWide: the tiles per warp the classes were cut for
     // key-range split (SR_SPLIT_KV): psl[i] = partial-output slot of item descriptor i (a chunk of a
     // split row-block) or -1; comb[j] = {row-block item, first slot, chunks, 0} of split row-block j
     const int32_t* psl;

@@ -475,6 +475,9 @@ LONG_CASES = [
     ("dense", dict(B=1, H=2, S=8192, D=128, dtype="bf16", kv_len=[8000])),
     ("window", dict(B=1, H=1, S=32768, D=64, dtype="f16", window=512, n_global=8)),
     ("dense", dict(B=1, H=2, S=32768, D=64, dtype="f16")),  # X' = 4 GiB
+    # 2048 row-blocks: more IR CTAs than one wave, so the IR kernel takes its 6-tiles-per-warp
+    # classes (rows of up to 64 tiles: staged and folded)
+    ("dense", dict(B=2, H=16, S=8192, D=64, dtype="f16", causal=True)),
 ]
 
 
