@@ -606,6 +606,11 @@ std::shared_ptr<DevBlob> make_blob(const HostSched& h0, int n_sm, bool split)
             classes(kIrWarpTilesWide, d.n_ir_class);
         }
     }
+    // fp32 SIMT kernels: the fewest threads per row that still give >= 2 CTAs per SM (each thread
+    // then owns the most columns), else 32
+    d.simt_tpr = 32;
+    for (int tpr = 4; tpr < 32; tpr *= 2)
+        if ((int64_t)d.n_items * tpr >= 2 * (int64_t)n_sm) { d.simt_tpr = tpr; break; }
     d.n_cta = (int)cta_ptr.size() - 1;
     d.n_pair = h.n_pair;
     d.n_pcta = (int)h.pcta_ptr.size() - 1;

@@ -81,6 +81,7 @@ struct DevSched {
     const int4* ir_desc;  // {g * slots_per_head + t0 - tp[lh][0], t1 - t0, t0, item} per row-block, class order
     int n_ir_class[4];
     int ir_warp_tiles;  // kIrWarpTiles or kIrWarpTilesWide: the tiles per warp the classes were cut for
+    int simt_tpr;       // fp32 SIMT kernels: threads per query row (4, 8, 16, 32; k_simt_f32.cu)
     // key-range split (SR_SPLIT_KV): psl[i] = partial-output slot of item descriptor i (a chunk of a
     // split row-block) or -1; comb[j] = {row-block item, first slot, chunks, 0} of split row-block j
     const int32_t* psl;
