@@ -13,19 +13,21 @@ namespace sr {
 // Organisation (vectorised).  A thread owns 4 consecutive rows of a row-block (lane l: rows 4l ..
 // 4l+3, all in one 64-row half), so one warp-wide 16-B load (LDG.128) brings a whole tile's 128
 // statistics -- one 512-B run of the [slot][128] layout.  Each row-block gets a TEAM of TW warps
-// (TW = 1, 2, 4 or 8, so that a warp has at most kIrWarpTiles = 4 of its tiles): warp t of the team
+// (TW = 1, 2, 4 or 8, so that a warp has at most KR of its tiles; KR = kIrWarpTiles = 4, or
+// kIrWarpTilesWide = 6 when the 4-tile classes would need more than one wave of CTAs -- chosen on the
+// host, sc.ir_warp_tiles): warp t of the team
 // takes tiles t, t + TW, ..., loads all of them at once (m' and d' in registers: one memory round
 // trip), merges them into a partial (m, d) per row; the team's partials meet in shared memory; each
 // warp then writes r' for its own tiles.  Row-blocks come longest first (sc.ir_desc) in classes of
 // equal TW; a CTA of 8 warps runs 8 / TW row-blocks of one class, and the team size is a template
-// parameter (the class is decoded with shifts; the team loops unroll).  Rows longer than
-// 8 * kIrWarpTiles tiles fold the excess 2 tiles at a time and re-read m'.
+// parameter (the class is decoded with shifts; the team loops unroll).  Rows longer than 8 * KR
+// tiles fold the excess 2 tiles at a time and re-read m'.
 // Exponentials: the merge computes e_k = 2^{m'_k - m_w} against the warp's own maximum m_w and keeps
 // it, so r'_k = e_k * (2^{m_w - m} / d) costs one multiply per (row, tile) instead of a second
 // exponential (the per-row factor is one ex2).  12 B per (row, tile); ncu at C4: 34
 // thread-instructions per (row, tile), down from 46 with runtime team sizes and two exponentials.
 constexpr int kW = 8;
-constexpr int kFold = 2;  // tiles per folding step beyond 8 * kIrWarpTiles (register budget)
+constexpr int kFold = 2;  // tiles per folding step beyond 8 * KR (register budget)
 
 __device__ __forceinline__ float4 ldg4(const float* p) { return __ldcg(reinterpret_cast<const float4*>(p)); }
 
