@@ -126,6 +126,20 @@ def test_fp32_masks(kind):
     assert_close(o, ref, "f32", what=kind)
 
 
+@pytest.mark.parametrize("B,H,D,tpr", [(2, 8, 64, 4), (1, 8, 128, 8), (1, 4, 64, 16), (1, 2, 128, 32)],
+                         ids=["tpr4", "tpr8", "tpr16", "tpr32"])
+def test_fp32_threads_per_row(B, H, D, tpr):
+    """The fp32 SIMT kernels at each threads-per-row width the host picks from the item count
+    (k_simt_f32.cu: the fewest of 4 / 8 / 16 giving >= 2 CTAs per SM on 148 SMs, else 32), with
+    S % 128 == 64, causal and a padded batch entry; every element against the oracle at 1e-5."""
+    S = 576  # 4.5 row-blocks
+    items = B * H * -(-S // 128)
+    assert (items >= 74) == (tpr == 4) and (37 <= items < 74) == (tpr == 8) and (19 <= items < 37) == (tpr == 16)
+    for kw in (dict(causal=True), dict(kv_len=[S, 333][:B])):
+        o, ref = run_case("dense", B, H, S, D, "f32", **kw)
+        assert_close(o, ref, "f32", what=f"tpr {tpr} {kw}")
+
+
 # ------------------------------------------------------------------------------------ tensor cores
 
 DENSE_CASES = [
